@@ -1,0 +1,104 @@
+"""CPU replay of CSP's three stages (Sec. 4.1) on oracle pieces.
+
+Test infrastructure: per layer, every rank groups its frontier by owner
+(contiguous id ranges), ships the ids to the owners ("shuffle"), each
+owner runs ``oracle.sample_rows`` on ITS OWN CSR shard ("sample"), the rows go
+back to the requester in request order ("reshuffle") and the requester builds
+its block with ``oracle.build_block``.  Two transports: in-process lists, or
+``torch.distributed`` all_to_all over gloo (world_size >= 2 on CPU).  Used to
+pin the oracle's partition invariance (R8, R16) and the Fig. 5
+message pattern.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+import oracle
+
+
+def owner_of(ids, bounds) -> np.ndarray:
+    return np.searchsorted(np.asarray(bounds), np.asarray(ids, np.int64), side="right") - 1
+
+
+def _shard(indptr, indices, lo, hi):
+    ip = indptr[lo: hi + 1]
+    return ip - ip[0], indices[ip[0]: ip[-1]]
+
+
+def replay_inprocess(indptr, indices, bounds, rank_seeds, fanouts, rng_seed, log=None):
+    """All P ranks in one process.  Returns blocks[r][l] (oracle dicts)."""
+    N = len(indptr) - 1
+    P = len(bounds) - 1
+    shards = [_shard(indptr, indices, int(bounds[o]), int(bounds[o + 1])) for o in range(P)]
+    frontier = [np.asarray(s, np.int32) for s in rank_seeds]
+    blocks = [[] for _ in range(P)]
+    for l, k in enumerate(fanouts):
+        # shuffle: requests[r][o] = (frontier positions, ids) that r sends to o
+        own = [owner_of(f, bounds) for f in frontier]
+        req = [[np.nonzero(own[r] == o)[0] for o in range(P)] for r in range(P)]
+        if log is not None:
+            log.append({"layer": l, "shuffle": {f"{r}->{o}": frontier[r][req[r][o]].tolist()
+                                                for r in range(P) for o in range(P)}})
+        # sample at the owner on its shard
+        res = [[None] * P for _ in range(P)]
+        for o in range(P):
+            ip, ix = shards[o]
+            for r in range(P):
+                ids = frontier[r][req[r][o]]
+                res[r][o] = oracle.sample_rows(ip, ix, ids, k, l, rng_seed, id_offset=int(bounds[o]))
+        # reshuffle back to request order, then build the block
+        for r in range(P):
+            F = len(frontier[r])
+            cnt = np.zeros(F, np.int32)
+            rows = np.full((F, k), -1, np.int32)
+            for o in range(P):
+                c, rw = res[r][o]
+                cnt[req[r][o]] = c
+                rows[req[r][o]] = rw
+            if log is not None:
+                log[-1].setdefault("reshuffle_rows", {}).update(
+                    {f"{o}->{r}": {int(frontier[r][i]): rows[i, :cnt[i]].tolist() for i in req[r][o]}
+                     for o in range(P) if o != r and len(req[r][o])})
+            b = oracle.build_block(N, frontier[r], cnt, rows)
+            blocks[r].append(b)
+            frontier[r] = b["src_ids"]
+    return blocks
+
+
+def replay_distributed(indptr_shard, indices_shard, bounds, seeds, fanouts, rng_seed, num_nodes):
+    """One rank of the replay over torch.distributed (gloo).  Each rank holds
+    ONLY its own CSR shard.  Returns this rank's blocks."""
+    import torch
+    import torch.distributed as dist
+    P = dist.get_world_size()
+    r = dist.get_rank()
+    frontier = np.asarray(seeds, np.int32)
+    blocks = []
+    for l, k in enumerate(fanouts):
+        own = owner_of(frontier, bounds)
+        order = np.argsort(own, kind="stable")
+        send_counts = np.bincount(own, minlength=P).astype(np.int64)
+        # count notification first, then the ids
+        recv_counts = torch.zeros(P, dtype=torch.int64)
+        dist.all_to_all_single(recv_counts, torch.from_numpy(send_counts))
+        recv_counts = recv_counts.numpy()
+        recv_ids = torch.zeros(int(recv_counts.sum()), dtype=torch.int32)
+        dist.all_to_all_single(recv_ids, torch.from_numpy(frontier[order].copy()),
+                               output_split_sizes=recv_counts.tolist(),
+                               input_split_sizes=send_counts.tolist())
+        cnt, rows = oracle.sample_rows(indptr_shard, indices_shard, recv_ids.numpy(), k, l, rng_seed,
+                                       id_offset=int(bounds[r]))
+        packed = np.concatenate([cnt[:, None], rows], axis=1).astype(np.int32)   # [n, 1 + k]
+        back = torch.zeros((len(frontier), 1 + k), dtype=torch.int32)
+        dist.all_to_all_single(back, torch.from_numpy(packed),
+                               output_split_sizes=send_counts.tolist(),
+                               input_split_sizes=recv_counts.tolist())
+        back = back.numpy()
+        cnt_f = np.zeros(len(frontier), np.int32)
+        rows_f = np.zeros((len(frontier), k), np.int32)
+        cnt_f[order] = back[:, 0]
+        rows_f[order] = back[:, 1:]
+        b = oracle.build_block(num_nodes, frontier, cnt_f, rows_f)
+        blocks.append(b)
+        frontier = b["src_ids"]
+    return blocks
