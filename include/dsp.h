@@ -1,0 +1,189 @@
+/*
+ * dsp.h -- C ABI of libdsp.so: DSP's collective sampling primitive (CSP) and
+ * feature gather on B200 (sm_100a).  ABI version 1.
+ *
+ * PAPER.md = "DSP: Efficient GNN Training with Multiple GPUs" (PPoPP'23);
+ * "P:L<n>" cites its line n.  DESIGN.md "Readings" R1..R23 fix every point
+ * the paper leaves open.
+ *
+ * Model.  The graph's topology (CSR of in-neighbours, global ids in the rows)
+ * and its node features are partitioned over `world_size` GPUs by contiguous
+ * ranges of renumbered global ids: rank r owns [bounds[r], bounds[r+1])
+ * (P:L112-116 data layout, P:L222 renumbering / range check).  One dsp_ctx
+ * per (process, GPU) -- or several ctxs driven by one host thread with
+ * dsp_sample_group.  A mini-batch's seeds are sampled layer by layer with CSP
+ * (shuffle -> sample -> reshuffle) into per-layer blocks, then
+ * the features of the sampled nodes are gathered (P:L126 loader).
+ *
+ * Conventions (all functions):
+ *   * Every function returns a dsp_status; none throws, aborts or prints.
+ *     dsp_last_error(ctx) gives a one-line detail of the last failure.
+ *   * Pointers documented as DEVICE must be CUDA device pointers on the ctx's
+ *     device; HOST pointers are ordinary host memory; "host or device" is
+ *     detected with cudaPointerGetAttributes.
+ *   * `stream` is a cudaStream_t passed as void* (0 = legacy default stream).
+ *   * The caller owns every buffer it passes; the library owns its copies of
+ *     the shards and its peer-visible exchange buffers.
+ *   * No allocation after dsp_reserve: dsp_sample / dsp_gather_features use
+ *     only the caller's workspace and library buffers sized at reserve time
+ *     (the paper's deadlock hazard of cudaMalloc against in-flight
+ *     communication, does not arise).
+ *   * COLLECTIVE calls must be made by every rank in the same order with the
+ *     same scalar arguments (the "fixed launch order" that CCC enforces,
+ *     P:L210-216, with a trivial leader).  Mismatched fanouts / rng_seed are
+ *     detected in the exchange header and reported as DSP_ERR_STATE.
+ */
+#ifndef DSP_H_
+#define DSP_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define DSP_ABI_VERSION 1
+#define DSP_MAX_WORLD 8      /* one NVSwitch node */
+#define DSP_MAX_LAYERS 8
+#define DSP_MAX_FANOUT 32    /* one lane per sampled slot */
+#define DSP_HANDLE_BYTES 512 /* size of an exported peer handle */
+
+typedef enum {
+  DSP_OK = 0,
+  DSP_ERR_INVALID_ARG = -1,   /* bad scalar / null pointer / bad layout      */
+  DSP_ERR_OUT_OF_RANGE = -2,  /* a node id outside [0, N)                    */
+  DSP_ERR_DUPLICATE_SEED = -3,/* a seed appears twice in one rank's batch    */
+  DSP_ERR_CAPACITY = -4,      /* a buffer or workspace is too small          */
+  DSP_ERR_STATE = -5,         /* call out of order / ranks disagree          */
+  DSP_ERR_CUDA = -6,          /* a CUDA runtime call failed                  */
+  DSP_ERR_PEER = -7,          /* peer mapping (CUDA IPC / P2P) failed        */
+  DSP_ERR_OOM = -8            /* device allocation failed                    */
+} dsp_status;
+
+typedef struct dsp_ctx dsp_ctx; /* opaque; one host thread at a time */
+
+/* ABI version (DSP_ABI_VERSION). */
+int dsp_abi_version(void);
+/* Static string for a status code. */
+const char *dsp_status_str(int status);
+/* Detail of the last failure on ctx (owned by ctx, valid until its next call);
+   "" when none.  ctx may be NULL (then: last failure of dsp_create). */
+const char *dsp_last_error(const dsp_ctx *ctx);
+
+/* ------------------------------------------------------------ lifecycle */
+
+/* Creates a ctx for `rank` of `world_size` (1..DSP_MAX_WORLD) on CUDA device
+   `cuda_device`.  Several ctxs may share a device (virtual ranks driven by
+   dsp_sample_group).  *out is set on success. */
+dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp_ctx **out);
+
+/* Frees everything the library owns (shards, exchange buffers, peer
+   mappings).  COLLECTIVE in effect: peers must have stopped using this ctx's
+   memory (barrier first).  NULL is a no-op. */
+void dsp_destroy(dsp_ctx *ctx);
+
+/* ------------------------------------------------------------ partition */
+
+/* Loads this rank's partition.  Once per ctx.
+   bounds  : HOST int64[world_size + 1]; bounds[0] = 0, non-decreasing,
+             bounds[world_size] = N with N < 2^31; identical on all ranks.
+   indptr  : host or device int64[n_r + 1], n_r = bounds[rank+1] - bounds[rank],
+             indptr[0] = 0, non-decreasing.
+   indices : host or device int32[indptr[n_r]]: GLOBAL ids of the
+             in-neighbours of local row v (global id bounds[rank] + v), each
+             row strictly ascending (R9).
+   features: host or device fp32[n_r][dim] row-major, or NULL for none.
+   dim     : 4 <= dim <= 4096 and dim % 4 == 0 (16-byte rows); ignored when
+             features is NULL.
+   The library copies everything into its own device memory (the feature
+   shard into peer-mappable memory); the caller may free its buffers on
+   return. */
+dsp_status dsp_load_partition(dsp_ctx *ctx, const int64_t *bounds, const int64_t *indptr,
+                              const int32_t *indices, const float *features, int32_t dim);
+
+/* Sizes the library's peer-visible exchange buffers for batches of up to
+   max_seeds seeds per rank and the given fan-outs (fanouts: HOST
+   int32[num_layers], 1 <= fanouts[l] <= 32, 1 <= num_layers <= 8).
+   COLLECTIVE (identical arguments on every rank).  After dsp_load_partition. */
+dsp_status dsp_reserve(dsp_ctx *ctx, int32_t max_seeds, const int32_t *fanouts, int32_t num_layers);
+
+/* Peer handles (CUDA IPC for other processes, raw pointers within one
+   process).  After dsp_reserve, every rank exports DSP_HANDLE_BYTES bytes;
+   the caller all-gathers them (e.g. torch.distributed) into `all`
+   (HOST, world_size * DSP_HANDLE_BYTES bytes, rank order) and imports them.
+   Sampling and gather need the import when world_size > 1. */
+dsp_status dsp_export_handle(const dsp_ctx *ctx, void *out);
+dsp_status dsp_import_handles(dsp_ctx *ctx, const void *all);
+
+/* ------------------------------------------------------------- sampling */
+
+typedef struct {
+  /* one sampled layer ("block"); arrays are DEVICE memory owned by the CALLER */
+  int32_t *indptr;     int64_t cap_indptr; /* out [num_dst+1]: edge offsets per dst         */
+  int32_t *indices;    int64_t cap_edges;  /* out [num_edges]: LOCAL src ids in [0,num_src) */
+  int32_t *src_ids;    int64_t cap_src;    /* out [num_src]: global ids; [0,num_dst) = dst  */
+  int32_t num_dst;     int32_t num_src;    /* out (host), filled on success                 */
+  int64_t num_edges;                       /* out (host)                                    */
+} dsp_block;
+
+/* Capacities for a call: with F_0 = num_seeds (per-rank maximum), for each
+   layer l: max_edges[l] = F_l * fanouts[l], max_src[l] = min(N, F_l +
+   max_edges[l]), F_{l+1} = max_src[l].  *workspace_bytes: the device
+   workspace dsp_sample needs.  max_src / max_edges: HOST int64[num_layers]
+   (either may be NULL).  num_seeds must not exceed the reserved max_seeds. */
+dsp_status dsp_sample_bounds(const dsp_ctx *ctx, int32_t num_seeds, const int32_t *fanouts,
+                             int32_t num_layers, int64_t *max_src, int64_t *max_edges,
+                             size_t *workspace_bytes);
+
+/* CSP node-wise uniform sampling without replacement (DESIGN.md
+   R1-R17).  COLLECTIVE: every rank calls with identical fanouts, num_layers
+   and rng_seed; seeds differ per rank (0 seeds allowed; the rank still takes
+   part in every exchange).
+   seeds    : DEVICE int32[num_seeds], unique (else DSP_ERR_DUPLICATE_SEED),
+              each in [0, N) (else DSP_ERR_OUT_OF_RANGE); any owner.
+   fanouts  : HOST int32[num_layers]; fanouts[l] applies at sampling layer l
+              (l = 0 is the seeds' hop, R1).
+   blocks   : HOST dsp_block[num_layers] in SAMPLING order; capacities must
+              cover dsp_sample_bounds (else DSP_ERR_CAPACITY before any work).
+              blocks[l].src_ids is the frontier of layer l+1; the last block's
+              src_ids are the unique nodes whose features the loader needs.
+   workspace: DEVICE, >= workspace_bytes from dsp_sample_bounds.
+   Stream-ordered on `stream`; returns after one stream synchronisation with
+   the host-side sizes filled.  The result is a pure function of (graph,
+   seeds, fanouts, rng_seed): bit-identical for any world_size / bounds and
+   across runs.  On a device-detected error the call returns it and the
+   block contents are unspecified. */
+dsp_status dsp_sample(dsp_ctx *ctx, const int32_t *seeds, int32_t num_seeds, const int32_t *fanouts,
+                      int32_t num_layers, uint64_t rng_seed, dsp_block *blocks, void *workspace,
+                      size_t workspace_bytes, void *stream);
+
+/* The same collective for n_ctx ctxs of one world driven by ONE host thread
+   (virtual ranks sharing a device, or one process owning several GPUs).
+   Array arguments are indexed by position in ctxs (any rank order, all ranks
+   of the world present).  Stages are issued rank by rank per stage, so
+   virtual ranks may share one stream. */
+dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *seeds,
+                            const int32_t *num_seeds, const int32_t *fanouts, int32_t num_layers,
+                            uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
+                            size_t workspace_bytes, void *const *streams);
+
+/* --------------------------------------------------------------- gather */
+
+/* Feature gather for the sampled nodes (P:L126 loader, hot features; P:L132:
+   one-sided access over NVLink).  ONE-SIDED (not collective): rows owned by
+   peers are read directly from their shards over NVLink, so it cannot
+   deadlock against CSP.
+   ids: DEVICE int32[n] global ids in [0, N); out: DEVICE fp32[n][dim],
+   16-byte aligned, row-major.  out[r][c] = features of ids[r], bit-exact.
+   Asynchronous on `stream`; an out-of-range id latches an error that
+   dsp_sync reports (its row is left unwritten). */
+dsp_status dsp_gather_features(dsp_ctx *ctx, const int32_t *ids, int64_t n, float *out, void *stream);
+
+/* Synchronises `stream` and reports a latched device error (then clears it). */
+dsp_status dsp_sync(dsp_ctx *ctx, void *stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DSP_H_ */

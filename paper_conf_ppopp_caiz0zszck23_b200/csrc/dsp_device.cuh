@@ -1,0 +1,161 @@
+// dsp_device.cuh -- device primitives for the CSP hot path on sm_100a:
+// counter-based Philox draws, warp-cooperative Floyd sampling, the relabel
+// hash table, peer-memory flags.  Written for B200 from PAPER.md + DESIGN.md;
+// shares nothing with oracle/.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace dsp {
+
+constexpr unsigned FULL_MASK = 0xffffffffu;
+constexpr unsigned long long EMPTY_SLOT = ~0ull;
+
+// ---------------------------------------------------------------- errors
+enum : int {
+  E_OK = 0, E_INVALID = -1, E_RANGE = -2, E_DUP = -3, E_CAP = -4, E_STATE = -5,
+};
+
+__device__ __forceinline__ void latch(int *err, int code) {
+  atomicCAS(err, 0, code);
+}
+
+// ---------------------------------------------------------------- Philox
+// Philox4x32-10 (Salmon et al., SC'11).  Counter/key layout: DESIGN.md R5.
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
+#pragma unroll
+  for (int round = 0; round < 10; ++round) {
+    if (round) {
+      k.x += 0x9E3779B9u;
+      k.y += 0xBB67AE85u;
+    }
+    const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+    const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+    c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+  }
+  return c;
+}
+
+// draw(slot, v, l) in [0, m): high 64 bits of (x1:x0) * m   (R6)
+__device__ __forceinline__ uint32_t draw_range(uint2 key, uint32_t slot, int32_t v, int32_t l,
+                                               uint32_t m) {
+  const uint4 x = philox4x32_10(make_uint4(slot, (uint32_t)v, (uint32_t)l, 0x44535031u), key);
+  const unsigned long long w = ((unsigned long long)x.y << 32) | x.x;
+  return (uint32_t)__umul64hi(w, (unsigned long long)m);
+}
+
+// ------------------------------------------------------------ hash table
+// Open addressing, linear probing, one 64-bit word per slot:
+//   word = key << 32 | val,  EMPTY = all ones (keys are < 2^31).
+// val is the minimum "order key" inserted for that key: dst index i (< F)
+// or F + i*k + slot for a sampled edge, so after all insertions val < F
+// means "is a dst" and val == F + q means "edge slot q is the first
+// occurrence".
+__device__ __forceinline__ uint32_t hash32(uint32_t x) {
+  x ^= x >> 16;
+  x *= 0x85EBCA6Bu;
+  x ^= x >> 13;
+  x *= 0xC2B2AE35u;
+  x ^= x >> 16;
+  return x;
+}
+
+// Inserts (key, val) keeping the minimum val.  Returns the slot index and the
+// previous val of the key in *old (0xffffffff if the key was new).
+__device__ __forceinline__ uint32_t table_insert_min(unsigned long long *tbl, uint32_t mask,
+                                                     uint32_t key, uint32_t val, uint32_t *old) {
+  const unsigned long long want = ((unsigned long long)key << 32) | val;
+  uint32_t idx = hash32(key) & mask;
+  while (true) {
+    unsigned long long cur = *(volatile unsigned long long *)&tbl[idx];
+    if (cur == EMPTY_SLOT) {
+      const unsigned long long prev = atomicCAS(&tbl[idx], EMPTY_SLOT, want);
+      if (prev == EMPTY_SLOT) {
+        *old = 0xffffffffu;
+        return idx;
+      }
+      cur = prev;
+    }
+    if ((uint32_t)(cur >> 32) == key) {
+      uint32_t o = (uint32_t)cur;
+      if (o > val) o = (uint32_t)atomicMin(&tbl[idx], want);
+      *old = o;
+      return idx;
+    }
+    idx = (idx + 1) & mask;
+  }
+}
+
+// ------------------------------------------------------ peer-memory flags
+__device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+
+// ------------------------------------------------------------- owner map
+struct Bounds {
+  int64_t b[9];  // DSP_MAX_WORLD + 1
+  int32_t world;
+};
+__device__ __forceinline__ int owner_of(const Bounds &bd, int64_t g) {
+  int o = 0;
+#pragma unroll
+  for (int r = 1; r < 8; ++r) o += (r < bd.world && g >= bd.b[r]) ? 1 : 0;
+  return o;
+}
+
+// ------------------------------------------------------- one node's sample
+// Lane group of G lanes (G = next pow2 >= k) samples node v.  Returns, per
+// lane t: whether slot `*slot` of the node holds sampled neighbour *u, and
+// the node's count min(deg, k).  Warp-uniform control flow (every lane of the
+// warp calls it): full rows and inactive groups run the same instructions.
+//
+// Floyd's algorithm (R7): lane t < k draws r_t in [0, d-k+t];
+// step t takes j_t = d-k+t if r_t equals an earlier choice, else r_t.  The
+// positions are then ranked (sorted ascending) by pairwise comparison, so
+// slot = rank and neighbours come out in row order.
+template <int G>
+__device__ __forceinline__ void sample_node(bool ok, int32_t v, int64_t row_start, int64_t deg,
+                                            int k, int layer, uint2 key,
+                                            const int32_t *__restrict__ indices, bool *valid,
+                                            int *slot, int32_t *u, int *count) {
+  const int lane = threadIdx.x & 31;
+  const int t = lane & (G - 1);
+  const int gbase = lane & ~(G - 1);
+  const unsigned gmask = (G == 32) ? FULL_MASK : (((1u << G) - 1u) << gbase);
+  const bool full = deg <= k;
+  uint32_t chosen = (uint32_t)t;
+  if (ok && !full && t < k) {
+    const uint32_t j = (uint32_t)(deg - k + t);
+    chosen = draw_range(key, (uint32_t)t, v, layer, j + 1u);
+  }
+  // Floyd resolution, slot by slot
+  for (int tt = 1; tt < k; ++tt) {
+    const uint32_t x = __shfl_sync(FULL_MASK, chosen, tt, G);
+    const bool hit = (t < tt) && (chosen == x);
+    const unsigned m = __ballot_sync(FULL_MASK, hit) & gmask;
+    if (t == tt && m != 0u) chosen = (uint32_t)(deg - k + tt);
+  }
+  // rank = number of chosen positions smaller than mine (they are distinct)
+  int rank = 0;
+  for (int s = 0; s < k; ++s) {
+    const uint32_t c = __shfl_sync(FULL_MASK, chosen, s, G);
+    rank += (c < chosen) ? 1 : 0;
+  }
+  const int cnt = ok ? (int)(full ? deg : k) : 0;
+  *count = cnt;
+  *valid = t < cnt;
+  *slot = full ? t : rank;
+  *u = *valid ? __ldg(indices + row_start + chosen) : -1;
+}
+
+}  // namespace dsp

@@ -1,0 +1,880 @@
+// dsp_runtime.cu -- host runtime behind the C ABI of include/dsp.h:
+// context, partition load, peer mapping (CUDA IPC / P2P), workspace
+// planning, and the CSP layer driver that issues the kernels of
+// dsp_kernels.cuh.  sm_100a only.
+#include <cuda_runtime.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/dsp.h"
+#include "dsp_kernels.cuh"
+
+using namespace dsp;
+
+namespace {
+
+constexpr uint32_t HANDLE_MAGIC = 0x44535048u;  // "DSPH"
+thread_local std::string g_create_error;
+
+struct PeerHandle {  // fits in DSP_HANDLE_BYTES
+  uint32_t magic;
+  int32_t rank, world, device;
+  int64_t pid;
+  uint64_t boot_id;  // distinguishes processes of different hosts / boots
+  uint64_t feat_ptr, xch_ptr;
+  int64_t feat_bytes, xch_bytes;
+  int32_t has_feat, has_xch;
+  cudaIpcMemHandle_t feat_ipc, xch_ipc;
+  int64_t bounds[DSP_MAX_WORLD + 1];
+  int32_t dim, max_seeds;
+};
+static_assert(sizeof(PeerHandle) <= DSP_HANDLE_BYTES, "handle too large");
+
+uint64_t boot_id() {
+  static uint64_t id = [] {
+    uint64_t h = 1469598103934665603ull;
+    FILE *f = fopen("/proc/sys/kernel/random/boot_id", "r");
+    if (f) {
+      int c;
+      while ((c = fgetc(f)) != EOF) h = (h ^ (uint64_t)c) * 1099511628211ull;
+      fclose(f);
+    }
+    char host[256] = {0};
+    gethostname(host, sizeof(host) - 1);
+    for (char *p = host; *p; ++p) h = (h ^ (uint64_t)*p) * 1099511628211ull;
+    return h;
+  }();
+  return id;
+}
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+int64_t next_pow2(int64_t x) {
+  int64_t p = 1;
+  while (p < x) p <<= 1;
+  return p;
+}
+
+int group_of(int k) {
+  int g = 1;
+  while (g < k) g <<= 1;
+  return g;
+}
+
+// Per-layer bounds (dsp_sample_bounds) and the workspace plan.
+struct Plan {
+  int L;
+  int64_t F[DSP_MAX_LAYERS + 1];   // max frontier per layer
+  int64_t E[DSP_MAX_LAYERS];       // max edges
+  int64_t S[DSP_MAX_LAYERS];       // max src
+  int64_t cap[DSP_MAX_LAYERS];     // table capacity
+  int64_t max_F, max_slots, max_cap, max_tiles;
+  size_t off_cnt, off_perm, off_hpos, off_status, off_tbl, bytes;
+};
+
+}  // namespace
+
+struct dsp_ctx {
+  int rank = 0, world = 1, device = 0;
+  std::string err;
+  bool loaded = false, reserved = false, imported = false, broken = false;
+  int64_t bounds[DSP_MAX_WORLD + 1] = {0};
+  int64_t N = 0, lo = 0, n_local = 0, nnz = 0;
+  int32_t dim = 0;
+  int64_t *d_indptr = nullptr;
+  int32_t *d_indices = nullptr;
+  float *d_feat = nullptr;
+  int64_t feat_bytes = 0;
+  int *d_err = nullptr;  // gather error latch
+  // exchange
+  int32_t max_seeds = 0, L = 0, kmax = 0;
+  int32_t fanouts[DSP_MAX_LAYERS] = {0};
+  XchLayout xl{};
+  char *d_xch = nullptr;
+  // peers
+  const float *peer_feat[DSP_MAX_WORLD] = {nullptr};
+  char *peer_xch[DSP_MAX_WORLD] = {nullptr};
+  void *ipc_opened[2 * DSP_MAX_WORLD] = {nullptr};
+  unsigned long long seq = 0;
+  // host staging
+  WsHeader *h_hdr = nullptr;  // pinned
+  int num_sms = 148;
+};
+
+namespace {
+
+dsp_status fail(dsp_ctx *c, dsp_status s, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  if (c)
+    c->err = buf;
+  else
+    g_create_error = buf;
+  return s;
+}
+
+#define CUDA_TRY(ctx, call)                                                                  \
+  do {                                                                                       \
+    cudaError_t e_ = (call);                                                                 \
+    if (e_ != cudaSuccess) {                                                                 \
+      cudaGetLastError();                                                                    \
+      return fail((ctx), e_ == cudaErrorMemoryAllocation ? DSP_ERR_OOM : DSP_ERR_CUDA,       \
+                  "%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_));         \
+    }                                                                                        \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    cudaGetDevice(&cur);
+    if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+bool is_device_ptr(const void *p) {
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
+}
+
+dsp_status check_fanouts(dsp_ctx *c, const int32_t *fanouts, int32_t L) {
+  if (L < 1 || L > DSP_MAX_LAYERS || !fanouts)
+    return fail(c, DSP_ERR_INVALID_ARG, "num_layers must be in [1, %d]", DSP_MAX_LAYERS);
+  for (int l = 0; l < L; ++l)
+    if (fanouts[l] < 1 || fanouts[l] > DSP_MAX_FANOUT)
+      return fail(c, DSP_ERR_INVALID_ARG, "fanouts[%d] = %d not in [1, %d]", l, fanouts[l], DSP_MAX_FANOUT);
+  return DSP_OK;
+}
+
+Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L) {
+  Plan p{};
+  p.L = L;
+  p.F[0] = num_seeds;
+  p.max_F = num_seeds;
+  p.max_slots = 0;
+  p.max_cap = 64;
+  for (int l = 0; l < L; ++l) {
+    p.E[l] = p.F[l] * fanouts[l];
+    p.S[l] = std::min<int64_t>(N, p.F[l] + p.E[l]);
+    p.S[l] = std::max<int64_t>(p.S[l], p.F[l]);
+    p.F[l + 1] = p.S[l];
+    p.cap[l] = next_pow2(std::max<int64_t>(64, 2 * p.S[l]));
+    p.max_F = std::max(p.max_F, p.F[l]);
+    p.max_slots = std::max(p.max_slots, p.E[l]);
+    p.max_cap = std::max(p.max_cap, p.cap[l]);
+  }
+  p.max_tiles = (p.max_slots + SCAN_TILE - 1) / SCAN_TILE + 1;
+  size_t o = align_up(sizeof(WsHeader), 256);
+  p.off_cnt = o;
+  o = align_up(o + sizeof(int32_t) * std::max<int64_t>(1, p.max_F), 256);
+  p.off_perm = o;
+  o = align_up(o + sizeof(int32_t) * std::max<int64_t>(1, p.max_F), 256);
+  p.off_hpos = o;
+  o = align_up(o + sizeof(int32_t) * std::max<int64_t>(1, p.max_slots), 256);
+  p.off_status = o;  // ticket + tile status, immediately followed by the table
+  o = o + sizeof(unsigned long long) * (1 + p.max_tiles);
+  o = align_up(o, 256);
+  p.off_tbl = o;
+  o = o + sizeof(unsigned long long) * p.max_cap;
+  p.bytes = align_up(o, 256);
+  return p;
+}
+
+XchLayout make_xch_layout(int64_t cap, int kmax) {
+  XchLayout x{};
+  x.cap = cap;
+  x.kmax = kmax;
+  size_t o = 0;
+  x.off_inbox_flag = o;
+  o += sizeof(unsigned long long) * 16;
+  x.off_ret_flag = o;
+  o += sizeof(unsigned long long) * 16;
+  x.off_inbox_hdr = o;
+  o += sizeof(uint4) * 16;
+  o = align_up(o, 256);
+  x.off_inbox = o;
+  o = align_up(o + sizeof(int32_t) * 16 * (size_t)cap, 256);
+  x.off_ret_cnt = o;
+  o = align_up(o + sizeof(int32_t) * 16 * (size_t)cap, 256);
+  x.off_ret_rows = o;
+  o = align_up(o + sizeof(int32_t) * 16 * (size_t)cap * kmax, 256);
+  x.bytes = o;
+  return x;
+}
+
+Bounds make_bounds(const dsp_ctx *c) {
+  Bounds b{};
+  for (int r = 0; r <= DSP_MAX_WORLD; ++r) b.b[r] = r <= c->world ? c->bounds[r] : c->N;
+  b.world = c->world;
+  return b;
+}
+
+int grid_for(const dsp_ctx *c, int blocks_per_sm) { return c->num_sms * blocks_per_sm; }
+
+// ---------------------------------------------------------------- driver
+// One dsp_sample call for one ctx, split into stages so that
+// dsp_sample_group can interleave several ctxs stage by stage.
+struct Call {
+  dsp_ctx *c;
+  const int32_t *seeds;
+  int32_t num_seeds;
+  const int32_t *fanouts;
+  int32_t L;
+  uint64_t rng_seed;
+  dsp_block *blocks;
+  char *ws;
+  cudaStream_t stream;
+  Plan plan;
+  WsHeader *hdr;
+  unsigned long long seq0;
+};
+
+dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_seeds,
+                        const int32_t *fanouts, int32_t L, uint64_t rng_seed, dsp_block *blocks,
+                        void *workspace, size_t ws_bytes, void *stream) {
+  k.c = c;
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (c->broken) return fail(c, DSP_ERR_STATE, "ctx unusable after an earlier exchange failure");
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition not called");
+  if (c->world > 1 && (!c->reserved || !c->imported))
+    return fail(c, DSP_ERR_STATE, "world_size > 1 needs dsp_reserve + dsp_import_handles first");
+  dsp_status st = check_fanouts(c, fanouts, L);
+  if (st != DSP_OK) return st;
+  if (num_seeds < 0 || (num_seeds > 0 && !seeds))
+    return fail(c, DSP_ERR_INVALID_ARG, "bad seeds / num_seeds");
+  if (!blocks || !workspace) return fail(c, DSP_ERR_INVALID_ARG, "blocks / workspace is NULL");
+  if (c->reserved) {
+    if (num_seeds > c->max_seeds)
+      return fail(c, DSP_ERR_CAPACITY, "num_seeds %d > reserved max_seeds %d", num_seeds, c->max_seeds);
+    if (L != c->L) return fail(c, DSP_ERR_STATE, "num_layers %d != reserved %d", L, c->L);
+    for (int l = 0; l < L; ++l)
+      if (fanouts[l] != c->fanouts[l])
+        return fail(c, DSP_ERR_STATE, "fanouts[%d] = %d != reserved %d", l, fanouts[l], c->fanouts[l]);
+  }
+  // workspace and exchange capacities are planned for the reserved maximum so
+  // that every rank derives the same sizes
+  const int64_t plan_seeds = c->reserved ? c->max_seeds : num_seeds;
+  k.plan = make_plan(c->N, plan_seeds, fanouts, L);
+  if (ws_bytes < k.plan.bytes)
+    return fail(c, DSP_ERR_CAPACITY, "workspace %zu B < required %zu B", ws_bytes, k.plan.bytes);
+  for (int l = 0; l < L; ++l) {
+    if ((uint64_t)k.plan.F[l] + (uint64_t)k.plan.E[l] >= (1ull << 31))
+      return fail(c, DSP_ERR_CAPACITY, "layer %d: frontier * (1 + fanout) exceeds 2^31", l);
+    if (!blocks[l].indptr || !blocks[l].indices || !blocks[l].src_ids)
+      return fail(c, DSP_ERR_INVALID_ARG, "blocks[%d] has a NULL array", l);
+    if (blocks[l].cap_indptr < k.plan.F[l] + 1 || blocks[l].cap_edges < k.plan.E[l] ||
+        blocks[l].cap_src < k.plan.S[l])
+      return fail(c, DSP_ERR_CAPACITY,
+                  "blocks[%d] capacities (%lld, %lld, %lld) < bounds (%lld, %lld, %lld)", l,
+                  (long long)blocks[l].cap_indptr, (long long)blocks[l].cap_edges,
+                  (long long)blocks[l].cap_src, (long long)(k.plan.F[l] + 1),
+                  (long long)k.plan.E[l], (long long)k.plan.S[l]);
+  }
+  k.seeds = seeds;
+  k.num_seeds = num_seeds;
+  k.fanouts = fanouts;
+  k.L = L;
+  k.rng_seed = rng_seed;
+  k.blocks = blocks;
+  k.ws = static_cast<char *>(workspace);
+  k.stream = static_cast<cudaStream_t>(stream);
+  k.hdr = reinterpret_cast<WsHeader *>(k.ws);
+  k.seq0 = c->seq;
+  return DSP_OK;
+}
+
+dsp_status stage_begin(Call &k) {
+  DeviceGuard g(k.c->device);
+  CUDA_TRY(k.c, cudaMemsetAsync(k.hdr, 0, sizeof(WsHeader), k.stream));
+  return DSP_OK;
+}
+
+// table + tile status reset for layer l
+dsp_status stage_clear(Call &k, int l) {
+  DeviceGuard g(k.c->device);
+  const size_t bytes = (k.plan.off_tbl - k.plan.off_status) + sizeof(unsigned long long) * k.plan.cap[l];
+  CUDA_TRY(k.c, cudaMemsetAsync(k.ws + k.plan.off_status, 0xFF, bytes, k.stream));
+  return DSP_OK;
+}
+
+const int32_t *frontier_of(const Call &k, int l) { return l == 0 ? k.seeds : k.blocks[l - 1].src_ids; }
+
+template <int G>
+void launch_local(const LocalSampleArgs &a, int grid, cudaStream_t s) {
+  k_sample_local<G><<<grid, 256, 0, s>>>(a);
+}
+template <int G>
+void launch_remote(const RemoteSampleArgs &a, int grid, cudaStream_t s) {
+  k_sample_remote<G><<<grid, 256, 0, s>>>(a);
+}
+template <int G>
+void launch_unpermute(const UnpermuteArgs &a, int grid, cudaStream_t s) {
+  k_unpermute_insert<G><<<grid, 256, 0, s>>>(a);
+}
+
+#define DISPATCH_G(G, FN, ...)                 \
+  switch (G) {                                 \
+    case 1: FN<1>(__VA_ARGS__); break;         \
+    case 2: FN<2>(__VA_ARGS__); break;         \
+    case 4: FN<4>(__VA_ARGS__); break;         \
+    case 8: FN<8>(__VA_ARGS__); break;         \
+    case 16: FN<16>(__VA_ARGS__); break;       \
+    default: FN<32>(__VA_ARGS__); break;       \
+  }
+
+uint2 key_of(uint64_t rng_seed) { return make_uint2((uint32_t)rng_seed, (uint32_t)(rng_seed >> 32)); }
+
+// world == 1: fused sample + insert
+dsp_status stage_sample_local(Call &k, int l) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  LocalSampleArgs a{};
+  a.frontier = frontier_of(k, l);
+  a.F0 = k.num_seeds;
+  a.layer = l;
+  a.k = k.fanouts[l];
+  a.key = key_of(k.rng_seed);
+  a.indptr = c->d_indptr;
+  a.indices = c->d_indices;
+  a.lo = c->lo;
+  a.n_local = c->n_local;
+  a.tbl = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_tbl);
+  a.mask = (uint32_t)(k.plan.cap[l] - 1);
+  a.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt);
+  a.hpos = reinterpret_cast<int32_t *>(k.ws + k.plan.off_hpos);
+  a.hdr = k.hdr;
+  DISPATCH_G(group_of(a.k), launch_local, a, grid_for(c, 8), k.stream);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+XchPeers peers_of(const dsp_ctx *c) {
+  XchPeers p{};
+  for (int r = 0; r < DSP_MAX_WORLD; ++r) p.base[r] = r < c->world ? c->peer_xch[r] : nullptr;
+  return p;
+}
+
+dsp_status stage_shuffle(Call &k, int l) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  BucketArgs a{};
+  a.frontier = frontier_of(k, l);
+  a.F0 = k.num_seeds;
+  a.layer = l;
+  a.k = k.fanouts[l];
+  a.seed_lo = (uint32_t)k.rng_seed;
+  a.seed_hi = (uint32_t)(k.rng_seed >> 32);
+  a.rank = c->rank;
+  a.seq = k.seq0 + 1 + l;
+  a.parity = (int)(a.seq & 1);
+  a.bd = make_bounds(c);
+  a.L = c->xl;
+  a.peers = peers_of(c);
+  a.perm = reinterpret_cast<int32_t *>(k.ws + k.plan.off_perm);
+  a.hdr = k.hdr;
+  k_bucket_scatter<<<grid_for(c, 2), 256, 0, k.stream>>>(a);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+dsp_status stage_sample_remote(Call &k, int l) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  RemoteSampleArgs a{};
+  a.layer = l;
+  a.k = k.fanouts[l];
+  a.key = key_of(k.rng_seed);
+  a.rank = c->rank;
+  a.seq = k.seq0 + 1 + l;
+  a.parity = (int)(a.seq & 1);
+  a.indptr = c->d_indptr;
+  a.indices = c->d_indices;
+  a.lo = c->lo;
+  a.n_local = c->n_local;
+  a.bd = make_bounds(c);
+  a.L = c->xl;
+  a.peers = peers_of(c);
+  a.hdr = k.hdr;
+  DISPATCH_G(group_of(a.k), launch_remote, a, grid_for(c, 8), k.stream);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+dsp_status stage_unpermute(Call &k, int l) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  UnpermuteArgs a{};
+  a.frontier = frontier_of(k, l);
+  a.layer = l;
+  a.k = k.fanouts[l];
+  a.rank = c->rank;
+  a.seq = k.seq0 + 1 + l;
+  a.parity = (int)(a.seq & 1);
+  a.bd = make_bounds(c);
+  a.L = c->xl;
+  a.self = c->d_xch;
+  a.perm = reinterpret_cast<int32_t *>(k.ws + k.plan.off_perm);
+  a.tbl = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_tbl);
+  a.mask = (uint32_t)(k.plan.cap[l] - 1);
+  a.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt);
+  a.hpos = reinterpret_cast<int32_t *>(k.ws + k.plan.off_hpos);
+  a.hdr = k.hdr;
+  DISPATCH_G(group_of(a.k), launch_unpermute, a, grid_for(c, 8), k.stream);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+dsp_status stage_scan_indices(Call &k, int l) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  ScanArgs s{};
+  s.layer = l;
+  s.k = k.fanouts[l];
+  s.frontier = frontier_of(k, l);
+  s.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt);
+  s.hpos = reinterpret_cast<int32_t *>(k.ws + k.plan.off_hpos);
+  s.tbl = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_tbl);
+  s.status = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_status);
+  s.indptr_out = k.blocks[l].indptr;
+  s.src_ids_out = k.blocks[l].src_ids;
+  s.hdr = k.hdr;
+  const int64_t tiles = std::max<int64_t>(1, (k.plan.E[l] + SCAN_TILE - 1) / SCAN_TILE);
+  const int scan_grid = (int)std::min<int64_t>(tiles, grid_for(c, 4));
+  k_scan_assign<<<scan_grid, SCAN_THREADS, 0, k.stream>>>(s);
+  CUDA_TRY(c, cudaGetLastError());
+  IndicesArgs w{};
+  w.layer = l;
+  w.k = k.fanouts[l];
+  w.cnt = s.cnt;
+  w.hpos = s.hpos;
+  w.tbl = s.tbl;
+  w.indptr = k.blocks[l].indptr;
+  w.indices_out = k.blocks[l].indices;
+  w.hdr = k.hdr;
+  const int64_t need = std::max<int64_t>(1, (k.plan.E[l] + 255) / 256);
+  k_write_indices<<<(int)std::min<int64_t>(need, grid_for(c, 8)), 256, 0, k.stream>>>(w);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+dsp_status stage_end_async(Call &k) {
+  DeviceGuard g(k.c->device);
+  CUDA_TRY(k.c, cudaMemcpyAsync(k.c->h_hdr, k.hdr, sizeof(WsHeader), cudaMemcpyDeviceToHost, k.stream));
+  return DSP_OK;
+}
+
+dsp_status stage_finish(Call &k) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  CUDA_TRY(c, cudaStreamSynchronize(k.stream));
+  c->seq = k.seq0 + k.L;
+  const WsHeader &h = *c->h_hdr;
+  if (h.err != 0) {
+    if (h.err == E_STATE && c->world > 1) c->broken = true;
+    return fail(c, (dsp_status)h.err, "device-detected error %d (%s) during dsp_sample", h.err,
+                dsp_status_str(h.err));
+  }
+  for (int l = 0; l < k.L; ++l) {
+    k.blocks[l].num_dst = h.F[l];
+    k.blocks[l].num_src = h.S[l];
+    k.blocks[l].num_edges = h.E[l];
+  }
+  return DSP_OK;
+}
+
+dsp_status run_layer_stages(std::vector<Call> &calls, int l) {
+  dsp_status st;
+  for (auto &k : calls)
+    if ((st = stage_clear(k, l)) != DSP_OK) return st;
+  if (calls[0].c->world == 1) {
+    for (auto &k : calls)
+      if ((st = stage_sample_local(k, l)) != DSP_OK) return st;
+  } else {
+    for (auto &k : calls)
+      if ((st = stage_shuffle(k, l)) != DSP_OK) return st;
+    for (auto &k : calls)
+      if ((st = stage_sample_remote(k, l)) != DSP_OK) return st;
+    for (auto &k : calls)
+      if ((st = stage_unpermute(k, l)) != DSP_OK) return st;
+  }
+  for (auto &k : calls)
+    if ((st = stage_scan_indices(k, l)) != DSP_OK) return st;
+  return DSP_OK;
+}
+
+dsp_status run_calls(std::vector<Call> &calls) {
+  dsp_status st;
+  for (auto &k : calls)
+    if ((st = stage_begin(k)) != DSP_OK) return st;
+  for (int l = 0; l < calls[0].L; ++l)
+    if ((st = run_layer_stages(calls, l)) != DSP_OK) return st;
+  for (auto &k : calls)
+    if ((st = stage_end_async(k)) != DSP_OK) return st;
+  dsp_status first = DSP_OK;
+  for (auto &k : calls) {
+    st = stage_finish(k);
+    if (st != DSP_OK && first == DSP_OK) first = st;
+  }
+  return first;
+}
+
+void release(dsp_ctx *c) {
+  DeviceGuard g(c->device);
+  for (int i = 0; i < 2 * DSP_MAX_WORLD; ++i)
+    if (c->ipc_opened[i]) {
+      cudaIpcCloseMemHandle(c->ipc_opened[i]);
+      c->ipc_opened[i] = nullptr;
+    }
+  cudaFree(c->d_indptr);
+  cudaFree(c->d_indices);
+  cudaFree(c->d_feat);
+  cudaFree(c->d_xch);
+  cudaFree(c->d_err);
+  if (c->h_hdr) cudaFreeHost(c->h_hdr);
+  cudaGetLastError();
+}
+
+}  // namespace
+
+// ======================================================================= ABI
+extern "C" {
+
+int dsp_abi_version(void) { return DSP_ABI_VERSION; }
+
+const char *dsp_status_str(int s) {
+  switch (s) {
+    case DSP_OK: return "DSP_OK";
+    case DSP_ERR_INVALID_ARG: return "DSP_ERR_INVALID_ARG";
+    case DSP_ERR_OUT_OF_RANGE: return "DSP_ERR_OUT_OF_RANGE";
+    case DSP_ERR_DUPLICATE_SEED: return "DSP_ERR_DUPLICATE_SEED";
+    case DSP_ERR_CAPACITY: return "DSP_ERR_CAPACITY";
+    case DSP_ERR_STATE: return "DSP_ERR_STATE";
+    case DSP_ERR_CUDA: return "DSP_ERR_CUDA";
+    case DSP_ERR_PEER: return "DSP_ERR_PEER";
+    case DSP_ERR_OOM: return "DSP_ERR_OOM";
+    default: return "DSP_ERR_UNKNOWN";
+  }
+}
+
+const char *dsp_last_error(const dsp_ctx *ctx) { return ctx ? ctx->err.c_str() : g_create_error.c_str(); }
+
+dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp_ctx **out) {
+  g_create_error.clear();
+  if (!out) return fail(nullptr, DSP_ERR_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (world_size < 1 || world_size > DSP_MAX_WORLD || rank < 0 || rank >= world_size)
+    return fail(nullptr, DSP_ERR_INVALID_ARG, "rank %d / world_size %d invalid (max %d)", rank,
+                world_size, DSP_MAX_WORLD);
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || cuda_device < 0 || cuda_device >= ndev) {
+    cudaGetLastError();
+    return fail(nullptr, DSP_ERR_CUDA, "CUDA device %d not available (%d devices)", cuda_device, ndev);
+  }
+  cudaDeviceProp prop;
+  if (cudaGetDeviceProperties(&prop, cuda_device) != cudaSuccess)
+    return fail(nullptr, DSP_ERR_CUDA, "cudaGetDeviceProperties failed");
+  if (prop.major != 10)
+    return fail(nullptr, DSP_ERR_CUDA, "device %d is sm_%d%d; libdsp is built for sm_100a only",
+                cuda_device, prop.major, prop.minor);
+  dsp_ctx *c = new dsp_ctx();
+  c->rank = rank;
+  c->world = world_size;
+  c->device = cuda_device;
+  c->num_sms = prop.multiProcessorCount;
+  DeviceGuard g(cuda_device);
+  if (cudaMallocHost(&c->h_hdr, sizeof(WsHeader)) != cudaSuccess ||
+      cudaMalloc(&c->d_err, sizeof(int)) != cudaSuccess || cudaMemset(c->d_err, 0, sizeof(int)) != cudaSuccess) {
+    cudaGetLastError();
+    release(c);
+    delete c;
+    return fail(nullptr, DSP_ERR_OOM, "host/device allocation failed in dsp_create");
+  }
+  *out = c;
+  return DSP_OK;
+}
+
+void dsp_destroy(dsp_ctx *ctx) {
+  if (!ctx) return;
+  release(ctx);
+  delete ctx;
+}
+
+dsp_status dsp_load_partition(dsp_ctx *c, const int64_t *bounds, const int64_t *indptr,
+                              const int32_t *indices, const float *features, int32_t dim) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (c->loaded) return fail(c, DSP_ERR_STATE, "partition already loaded");
+  if (!bounds || !indptr) return fail(c, DSP_ERR_INVALID_ARG, "bounds / indptr is NULL");
+  if (bounds[0] != 0) return fail(c, DSP_ERR_INVALID_ARG, "bounds[0] must be 0");
+  for (int r = 0; r < c->world; ++r)
+    if (bounds[r + 1] < bounds[r]) return fail(c, DSP_ERR_INVALID_ARG, "bounds must be non-decreasing");
+  if (bounds[c->world] >= (1ll << 31)) return fail(c, DSP_ERR_INVALID_ARG, "N must be < 2^31");
+  if (features && (dim < 4 || dim > 4096 || dim % 4 != 0))
+    return fail(c, DSP_ERR_INVALID_ARG, "dim %d must be a multiple of 4 in [4, 4096]", dim);
+  DeviceGuard g(c->device);
+  for (int r = 0; r <= c->world; ++r) c->bounds[r] = bounds[r];
+  c->N = bounds[c->world];
+  c->lo = bounds[c->rank];
+  c->n_local = bounds[c->rank + 1] - c->lo;
+  const size_t ip_bytes = sizeof(int64_t) * (size_t)(c->n_local + 1);
+  CUDA_TRY(c, cudaMalloc(&c->d_indptr, ip_bytes));
+  CUDA_TRY(c, cudaMemcpy(c->d_indptr, indptr, ip_bytes, cudaMemcpyDefault));
+  int64_t first = 0;
+  CUDA_TRY(c, cudaMemcpy(&first, c->d_indptr, sizeof(int64_t), cudaMemcpyDeviceToHost));
+  CUDA_TRY(c, cudaMemcpy(&c->nnz, c->d_indptr + c->n_local, sizeof(int64_t), cudaMemcpyDeviceToHost));
+  if (first != 0 || c->nnz < 0) return fail(c, DSP_ERR_INVALID_ARG, "indptr[0] must be 0");
+  if (c->nnz > 0 && !indices) return fail(c, DSP_ERR_INVALID_ARG, "indices is NULL");
+  CUDA_TRY(c, cudaMalloc(&c->d_indices, sizeof(int32_t) * (size_t)std::max<int64_t>(1, c->nnz)));
+  if (c->nnz > 0)
+    CUDA_TRY(c, cudaMemcpy(c->d_indices, indices, sizeof(int32_t) * (size_t)c->nnz, cudaMemcpyDefault));
+  if (features) {
+    c->dim = dim;
+    c->feat_bytes = (int64_t)sizeof(float) * dim * std::max<int64_t>(1, c->n_local);
+    CUDA_TRY(c, cudaMalloc(&c->d_feat, (size_t)c->feat_bytes));
+    if (c->n_local > 0)
+      CUDA_TRY(c, cudaMemcpy(c->d_feat, features, sizeof(float) * dim * (size_t)c->n_local, cudaMemcpyDefault));
+  }
+  c->peer_feat[c->rank] = c->d_feat;
+  c->loaded = true;
+  (void)is_device_ptr;
+  return DSP_OK;
+}
+
+dsp_status dsp_reserve(dsp_ctx *c, int32_t max_seeds, const int32_t *fanouts, int32_t L) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
+  if (c->reserved) return fail(c, DSP_ERR_STATE, "already reserved");
+  dsp_status st = check_fanouts(c, fanouts, L);
+  if (st != DSP_OK) return st;
+  if (max_seeds < 0) return fail(c, DSP_ERR_INVALID_ARG, "max_seeds < 0");
+  Plan p = make_plan(c->N, max_seeds, fanouts, L);
+  for (int l = 0; l < L; ++l)
+    if ((uint64_t)p.F[l] + (uint64_t)p.E[l] >= (1ull << 31))
+      return fail(c, DSP_ERR_CAPACITY, "layer %d: frontier * (1 + fanout) exceeds 2^31", l);
+  c->max_seeds = max_seeds;
+  c->L = L;
+  c->kmax = 0;
+  for (int l = 0; l < L; ++l) {
+    c->fanouts[l] = fanouts[l];
+    c->kmax = std::max(c->kmax, fanouts[l]);
+  }
+  if (c->world > 1) {
+    DeviceGuard g(c->device);
+    c->xl = make_xch_layout(std::max<int64_t>(1, p.max_F), c->kmax);
+    CUDA_TRY(c, cudaMalloc(&c->d_xch, c->xl.bytes));
+    CUDA_TRY(c, cudaMemset(c->d_xch, 0, c->xl.bytes));
+    CUDA_TRY(c, cudaDeviceSynchronize());
+  }
+  c->peer_xch[c->rank] = c->d_xch;
+  c->reserved = true;
+  return DSP_OK;
+}
+
+dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
+  dsp_ctx *c = const_cast<dsp_ctx *>(cc);
+  if (!c || !out) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded || !c->reserved) return fail(c, DSP_ERR_STATE, "load_partition + reserve first");
+  PeerHandle h;
+  memset(&h, 0, sizeof(h));
+  h.magic = HANDLE_MAGIC;
+  h.rank = c->rank;
+  h.world = c->world;
+  h.device = c->device;
+  h.pid = (int64_t)getpid();
+  h.boot_id = boot_id();
+  h.feat_ptr = (uint64_t)(uintptr_t)c->d_feat;
+  h.xch_ptr = (uint64_t)(uintptr_t)c->d_xch;
+  h.feat_bytes = c->feat_bytes;
+  h.xch_bytes = (int64_t)c->xl.bytes;
+  h.dim = c->dim;
+  h.max_seeds = c->max_seeds;
+  for (int r = 0; r <= c->world; ++r) h.bounds[r] = c->bounds[r];
+  DeviceGuard g(c->device);
+  if (c->d_feat) {
+    h.has_feat = 1;
+    CUDA_TRY(c, cudaIpcGetMemHandle(&h.feat_ipc, c->d_feat));
+  }
+  if (c->d_xch) {
+    h.has_xch = 1;
+    CUDA_TRY(c, cudaIpcGetMemHandle(&h.xch_ipc, c->d_xch));
+  }
+  memset(out, 0, DSP_HANDLE_BYTES);
+  memcpy(out, &h, sizeof(h));
+  return DSP_OK;
+}
+
+dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
+  if (!c || !all) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded || !c->reserved) return fail(c, DSP_ERR_STATE, "load_partition + reserve first");
+  if (c->imported) return fail(c, DSP_ERR_STATE, "handles already imported");
+  DeviceGuard g(c->device);
+  const int64_t my_pid = (int64_t)getpid();
+  for (int r = 0; r < c->world; ++r) {
+    PeerHandle h;
+    memcpy(&h, static_cast<const char *>(all) + (size_t)r * DSP_HANDLE_BYTES, sizeof(h));
+    if (h.magic != HANDLE_MAGIC || h.rank != r || h.world != c->world)
+      return fail(c, DSP_ERR_INVALID_ARG, "handle %d is not rank %d of this world", r, r);
+    for (int q = 0; q <= c->world; ++q)
+      if (h.bounds[q] != c->bounds[q])
+        return fail(c, DSP_ERR_STATE, "rank %d has different bounds", r);
+    if (h.dim != c->dim || h.max_seeds != c->max_seeds)
+      return fail(c, DSP_ERR_STATE, "rank %d has a different dim / max_seeds", r);
+    if (r == c->rank) continue;
+    const bool same_process = h.pid == my_pid && h.boot_id == boot_id();
+    if (same_process) {
+      if (h.device != c->device) {
+        cudaError_t e = cudaDeviceEnablePeerAccess(h.device, 0);
+        if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) {
+          cudaGetLastError();
+          return fail(c, DSP_ERR_PEER, "cudaDeviceEnablePeerAccess(%d -> %d): %s", c->device, h.device,
+                      cudaGetErrorString(e));
+        }
+        cudaGetLastError();
+      }
+      c->peer_feat[r] = reinterpret_cast<const float *>(h.feat_ptr);
+      c->peer_xch[r] = reinterpret_cast<char *>(h.xch_ptr);
+    } else {
+      if (h.has_feat) {
+        void *p = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&p, h.feat_ipc, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+          cudaGetLastError();
+          return fail(c, DSP_ERR_PEER, "cudaIpcOpenMemHandle(features of rank %d): %s", r, cudaGetErrorString(e));
+        }
+        c->ipc_opened[2 * r] = p;
+        c->peer_feat[r] = static_cast<const float *>(p);
+      }
+      if (h.has_xch) {
+        void *p = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&p, h.xch_ipc, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+          cudaGetLastError();
+          return fail(c, DSP_ERR_PEER, "cudaIpcOpenMemHandle(exchange of rank %d): %s", r, cudaGetErrorString(e));
+        }
+        c->ipc_opened[2 * r + 1] = p;
+        c->peer_xch[r] = static_cast<char *>(p);
+      }
+    }
+  }
+  c->imported = true;
+  return DSP_OK;
+}
+
+dsp_status dsp_sample_bounds(const dsp_ctx *cc, int32_t num_seeds, const int32_t *fanouts, int32_t L,
+                             int64_t *max_src, int64_t *max_edges, size_t *workspace_bytes) {
+  dsp_ctx *c = const_cast<dsp_ctx *>(cc);
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
+  dsp_status st = check_fanouts(c, fanouts, L);
+  if (st != DSP_OK) return st;
+  if (num_seeds < 0) return fail(c, DSP_ERR_INVALID_ARG, "num_seeds < 0");
+  if (c->reserved && num_seeds > c->max_seeds)
+    return fail(c, DSP_ERR_CAPACITY, "num_seeds %d > reserved max_seeds %d", num_seeds, c->max_seeds);
+  Plan p = make_plan(c->N, c->reserved ? c->max_seeds : num_seeds, fanouts, L);
+  for (int l = 0; l < L; ++l) {
+    if (max_src) max_src[l] = p.S[l];
+    if (max_edges) max_edges[l] = p.E[l];
+  }
+  if (workspace_bytes) *workspace_bytes = p.bytes;
+  return DSP_OK;
+}
+
+dsp_status dsp_sample(dsp_ctx *c, const int32_t *seeds, int32_t num_seeds, const int32_t *fanouts,
+                      int32_t L, uint64_t rng_seed, dsp_block *blocks, void *workspace,
+                      size_t workspace_bytes, void *stream) {
+  std::vector<Call> calls(1);
+  dsp_status st = prepare_call(calls[0], c, seeds, num_seeds, fanouts, L, rng_seed, blocks, workspace,
+                               workspace_bytes, stream);
+  if (st != DSP_OK) return st;
+  return run_calls(calls);
+}
+
+dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n, const int32_t *const *seeds,
+                            const int32_t *num_seeds, const int32_t *fanouts, int32_t L,
+                            uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
+                            size_t workspace_bytes, void *const *streams) {
+  if (!ctxs || n < 1 || !seeds || !num_seeds || !blocks || !workspaces || !streams)
+    return DSP_ERR_INVALID_ARG;
+  const int world = ctxs[0] ? ctxs[0]->world : 0;
+  if (n != world) return fail(ctxs[0], DSP_ERR_INVALID_ARG, "dsp_sample_group needs all %d ranks", world);
+  std::vector<int> seen(world, 0);
+  for (int i = 0; i < n; ++i) {
+    if (!ctxs[i] || ctxs[i]->world != world || seen[ctxs[i]->rank]++)
+      return fail(ctxs[0], DSP_ERR_INVALID_ARG, "ctxs must be the distinct ranks of one world");
+    for (int j = 0; j < i; ++j)
+      if (ctxs[j]->device == ctxs[i]->device && streams[j] != streams[i])
+        return fail(ctxs[0], DSP_ERR_INVALID_ARG,
+                    "virtual ranks on one device must share a stream (stage-by-stage issue)");
+  }
+  std::vector<Call> calls(n);
+  for (int i = 0; i < n; ++i) {
+    dsp_status st = prepare_call(calls[i], ctxs[i], seeds[i], num_seeds[i], fanouts, L, rng_seed,
+                                 blocks[i], workspaces[i], workspace_bytes, streams[i]);
+    if (st != DSP_OK) return st;
+  }
+  return run_calls(calls);
+}
+
+dsp_status dsp_gather_features(dsp_ctx *c, const int32_t *ids, int64_t n, float *out, void *stream) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded || !c->d_feat) return fail(c, DSP_ERR_STATE, "no feature shard loaded");
+  if (c->world > 1 && !c->imported) return fail(c, DSP_ERR_STATE, "dsp_import_handles first");
+  if (n < 0 || (n > 0 && (!ids || !out))) return fail(c, DSP_ERR_INVALID_ARG, "bad ids / out / n");
+  if (((uintptr_t)out & 15u) != 0) return fail(c, DSP_ERR_INVALID_ARG, "out must be 16-byte aligned");
+  if (n == 0) return DSP_OK;
+  DeviceGuard g(c->device);
+  GatherArgs a{};
+  a.ids = ids;
+  a.n = n;
+  a.dim4 = c->dim / 4;
+  a.out = reinterpret_cast<float4 *>(out);
+  for (int r = 0; r < DSP_MAX_WORLD; ++r)
+    a.base[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_feat[r]) : nullptr;
+  a.bd = make_bounds(c);
+  a.err = c->d_err;
+  const int64_t total = n * a.dim4;
+  const int64_t want = (total + 256 * 4 - 1) / (256 * 4);
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, grid_for(c, 8)));
+  k_gather<4><<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(a);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+dsp_status dsp_sync(dsp_ctx *c, void *stream) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  DeviceGuard g(c->device);
+  CUDA_TRY(c, cudaStreamSynchronize(static_cast<cudaStream_t>(stream)));
+  int e = 0;
+  CUDA_TRY(c, cudaMemcpy(&e, c->d_err, sizeof(int), cudaMemcpyDeviceToHost));
+  if (e != 0) {
+    CUDA_TRY(c, cudaMemset(c->d_err, 0, sizeof(int)));
+    return fail(c, (dsp_status)e, "device-detected error %d (%s) in dsp_gather_features", e, dsp_status_str(e));
+  }
+  return DSP_OK;
+}
+
+}  // extern "C"

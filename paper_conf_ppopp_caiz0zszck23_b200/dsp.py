@@ -1,0 +1,342 @@
+"""Thin Python binding of libdsp.so (include/dsp.h), same names as the C ABI.
+
+Argument marshalling only: every step of sampling and gathering runs in the
+CUDA kernels behind the C ABI.  torch is used for device memory (workspace,
+blocks, outputs), streams and -- for world_size > 1 across processes -- the
+all-gather of the peer handles (torch.distributed plumbing).  There is no CPU
+fallback: if libdsp.so is missing or no sm_100 GPU is present, calls raise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Callable, NamedTuple, Sequence
+
+import numpy as np
+
+from . import _build
+
+DSP_OK = 0
+DSP_ERR_INVALID_ARG = -1
+DSP_ERR_OUT_OF_RANGE = -2
+DSP_ERR_DUPLICATE_SEED = -3
+DSP_ERR_CAPACITY = -4
+DSP_ERR_STATE = -5
+DSP_ERR_CUDA = -6
+DSP_ERR_PEER = -7
+DSP_ERR_OOM = -8
+DSP_MAX_WORLD = 8
+DSP_MAX_LAYERS = 8
+DSP_MAX_FANOUT = 32
+DSP_HANDLE_BYTES = 512
+
+#: every symbol include/dsp.h declares
+ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_create", "dsp_destroy",
+               "dsp_load_partition", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
+               "dsp_sample_bounds", "dsp_sample", "dsp_sample_group", "dsp_gather_features",
+               "dsp_sync")
+
+
+class DSPError(RuntimeError):
+    def __init__(self, status: int, detail: str = ""):
+        self.status = status
+        super().__init__(f"{_status_name(status)}: {detail}")
+
+
+class dsp_block(ctypes.Structure):
+    _fields_ = [("indptr", ctypes.c_void_p), ("cap_indptr", ctypes.c_int64),
+                ("indices", ctypes.c_void_p), ("cap_edges", ctypes.c_int64),
+                ("src_ids", ctypes.c_void_p), ("cap_src", ctypes.c_int64),
+                ("num_dst", ctypes.c_int32), ("num_src", ctypes.c_int32),
+                ("num_edges", ctypes.c_int64)]
+
+
+_lib = None
+
+
+def lib(path: str | None = None):
+    """Loads libdsp.so from the package directory (never from a JIT cache)."""
+    global _lib
+    if _lib is None:
+        path = path or _build.LIB
+        if not os.path.exists(path):
+            raise RuntimeError(f"libdsp.so not built ({path}); run __graft_entry__.build()")
+        L = ctypes.CDLL(path)
+        P, i32, i64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+        L.dsp_abi_version.restype = ctypes.c_int
+        L.dsp_status_str.argtypes = [ctypes.c_int]
+        L.dsp_status_str.restype = ctypes.c_char_p
+        L.dsp_last_error.argtypes = [P]
+        L.dsp_last_error.restype = ctypes.c_char_p
+        L.dsp_create.argtypes = [i32, i32, i32, ctypes.POINTER(ctypes.c_void_p)]
+        L.dsp_destroy.argtypes = [P]
+        L.dsp_destroy.restype = None
+        L.dsp_load_partition.argtypes = [P, P, P, P, P, i32]
+        L.dsp_reserve.argtypes = [P, i32, P, i32]
+        L.dsp_export_handle.argtypes = [P, P]
+        L.dsp_import_handles.argtypes = [P, P]
+        L.dsp_sample_bounds.argtypes = [P, i32, P, i32, P, P, ctypes.POINTER(ctypes.c_size_t)]
+        L.dsp_sample.argtypes = [P, P, i32, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t, P]
+        L.dsp_sample_group.argtypes = [P, i32, P, P, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t, P]
+        L.dsp_gather_features.argtypes = [P, P, i64, P, P]
+        L.dsp_sync.argtypes = [P, P]
+        for name in ("dsp_create", "dsp_load_partition", "dsp_reserve", "dsp_export_handle",
+                     "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_group",
+                     "dsp_gather_features", "dsp_sync"):
+            getattr(L, name).restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _status_name(s: int) -> str:
+    try:
+        return lib().dsp_status_str(s).decode()
+    except Exception:  # library unavailable while formatting an error
+        return f"status {s}"
+
+
+def _check(status: int, ctx=None):
+    if status != DSP_OK:
+        detail = lib().dsp_last_error(ctx).decode() if True else ""
+        raise DSPError(status, detail)
+
+
+def _p(x) -> ctypes.c_void_p:
+    """Raw pointer of a torch tensor, numpy array or int."""
+    if x is None:
+        return ctypes.c_void_p(0)
+    if isinstance(x, int):
+        return ctypes.c_void_p(x)
+    if isinstance(x, np.ndarray):
+        return x.ctypes.data_as(ctypes.c_void_p)
+    return ctypes.c_void_p(x.data_ptr())
+
+
+def _i32_array(xs) -> np.ndarray:
+    return np.ascontiguousarray(np.asarray(xs, dtype=np.int32))
+
+
+# ------------------------------------------------------- C-ABI, same names
+
+def dsp_abi_version() -> int:
+    return int(lib().dsp_abi_version())
+
+
+def dsp_status_str(status: int) -> str:
+    return lib().dsp_status_str(status).decode()
+
+
+def dsp_last_error(ctx) -> str:
+    return lib().dsp_last_error(ctx).decode()
+
+
+def dsp_create(rank: int, world_size: int, cuda_device: int) -> ctypes.c_void_p:
+    out = ctypes.c_void_p()
+    _check(lib().dsp_create(rank, world_size, cuda_device, ctypes.byref(out)), None)
+    return out
+
+
+def dsp_destroy(ctx) -> None:
+    lib().dsp_destroy(ctx)
+
+
+def dsp_load_partition(ctx, bounds, indptr, indices, features, dim: int) -> None:
+    b = np.ascontiguousarray(bounds, dtype=np.int64)
+    _check(lib().dsp_load_partition(ctx, _p(b), _p(indptr), _p(indices), _p(features), dim), ctx)
+
+
+def dsp_reserve(ctx, max_seeds: int, fanouts) -> None:
+    f = _i32_array(fanouts)
+    _check(lib().dsp_reserve(ctx, max_seeds, _p(f), len(f)), ctx)
+
+
+def dsp_export_handle(ctx) -> bytes:
+    buf = ctypes.create_string_buffer(DSP_HANDLE_BYTES)
+    _check(lib().dsp_export_handle(ctx, buf), ctx)
+    return buf.raw
+
+
+def dsp_import_handles(ctx, handles: Sequence[bytes]) -> None:
+    blob = b"".join(handles)
+    buf = ctypes.create_string_buffer(blob, len(blob))
+    _check(lib().dsp_import_handles(ctx, buf), ctx)
+
+
+def dsp_sample_bounds(ctx, num_seeds: int, fanouts):
+    f = _i32_array(fanouts)
+    ms = np.zeros(len(f), np.int64)
+    me = np.zeros(len(f), np.int64)
+    ws = ctypes.c_size_t()
+    _check(lib().dsp_sample_bounds(ctx, num_seeds, _p(f), len(f), _p(ms), _p(me), ctypes.byref(ws)), ctx)
+    return ms, me, int(ws.value)
+
+
+def dsp_sample(ctx, seeds, num_seeds: int, fanouts, rng_seed: int, blocks, workspace,
+               workspace_bytes: int, stream: int) -> None:
+    f = _i32_array(fanouts)
+    _check(lib().dsp_sample(ctx, _p(seeds), num_seeds, _p(f), len(f), ctypes.c_uint64(rng_seed),
+                            blocks, _p(workspace), workspace_bytes, ctypes.c_void_p(stream)), ctx)
+
+
+def dsp_sample_group(ctxs, seeds, num_seeds, fanouts, rng_seed: int, blocks, workspaces,
+                     workspace_bytes: int, streams) -> None:
+    n = len(ctxs)
+    f = _i32_array(fanouts)
+    c_ctxs = (ctypes.c_void_p * n)(*[c.value for c in ctxs])
+    c_seeds = (ctypes.c_void_p * n)(*[_p(s).value for s in seeds])
+    c_ns = (ctypes.c_int32 * n)(*num_seeds)
+    c_blocks = (ctypes.c_void_p * n)(*[ctypes.cast(b, ctypes.c_void_p).value for b in blocks])
+    c_ws = (ctypes.c_void_p * n)(*[_p(w).value for w in workspaces])
+    c_st = (ctypes.c_void_p * n)(*streams)
+    _check(lib().dsp_sample_group(c_ctxs, n, c_seeds, c_ns, _p(f), len(f), ctypes.c_uint64(rng_seed),
+                                  c_blocks, c_ws, workspace_bytes, c_st), ctxs[0])
+
+
+def dsp_gather_features(ctx, ids, n: int, out, stream: int) -> None:
+    _check(lib().dsp_gather_features(ctx, _p(ids), n, _p(out), ctypes.c_void_p(stream)), ctx)
+
+
+def dsp_sync(ctx, stream: int) -> None:
+    _check(lib().dsp_sync(ctx, ctypes.c_void_p(stream)), ctx)
+
+
+# ------------------------------------------------------------ conveniences
+
+class Block(NamedTuple):
+    """One sampled layer; tensors are views of the Sampler's device buffers."""
+    num_dst: int
+    num_src: int
+    num_edges: int
+    indptr: "object"   # torch.int32 [num_dst + 1]
+    indices: "object"  # torch.int32 [num_edges] local src ids
+    src_ids: "object"  # torch.int32 [num_src] global ids
+
+
+class Sampler:
+    """One rank of a CSP world: ctx + partition + caller-owned buffers.
+
+    ``exchange(blob) -> list[bytes]`` all-gathers the peer handles when
+    world_size > 1 (see :func:`torch_exchange`)."""
+
+    def __init__(self, bounds, indptr, indices, features, fanouts, max_seeds: int, rank: int = 0,
+                 world_size: int = 1, device: int | None = None,
+                 exchange: Callable[[bytes], list] | None = None, connect: bool = True):
+        import torch
+        self.torch = torch
+        self.device = torch.cuda.current_device() if device is None else device
+        self.rank, self.world = rank, world_size
+        self.fanouts = [int(k) for k in fanouts]
+        self.max_seeds = int(max_seeds)
+        self.dim = 0 if features is None else int(features.shape[1])
+        self.ctx = dsp_create(rank, world_size, self.device)
+        try:
+            dsp_load_partition(self.ctx, bounds, indptr, indices, features, self.dim)
+            dsp_reserve(self.ctx, self.max_seeds, self.fanouts)
+            ms, me, ws = dsp_sample_bounds(self.ctx, self.max_seeds, self.fanouts)
+        except Exception:
+            dsp_destroy(self.ctx)
+            raise
+        dev = torch.device("cuda", self.device)
+        self.workspace_bytes = ws
+        self.workspace = torch.empty(ws, dtype=torch.uint8, device=dev)
+        F = [self.max_seeds] + [int(x) for x in ms[:-1]]
+        self._bufs = []
+        self._cblocks = (dsp_block * len(self.fanouts))()
+        for l in range(len(self.fanouts)):
+            ip = torch.empty(F[l] + 1, dtype=torch.int32, device=dev)
+            ix = torch.empty(max(1, int(me[l])), dtype=torch.int32, device=dev)
+            sr = torch.empty(max(1, int(ms[l])), dtype=torch.int32, device=dev)
+            self._bufs.append((ip, ix, sr))
+            b = self._cblocks[l]
+            b.indptr, b.cap_indptr = ip.data_ptr(), ip.numel()
+            b.indices, b.cap_edges = ix.data_ptr(), int(me[l])
+            b.src_ids, b.cap_src = sr.data_ptr(), int(ms[l])
+        self.max_src = [int(x) for x in ms]
+        self.max_edges = [int(x) for x in me]
+        self.connected = False
+        if connect and (world_size == 1 or exchange is not None):
+            handles = [dsp_export_handle(self.ctx)] if world_size == 1 else exchange(dsp_export_handle(self.ctx))
+            if world_size > 1:
+                dsp_import_handles(self.ctx, handles)
+            self.connected = True
+
+    def stream(self) -> int:
+        return self.torch.cuda.current_stream(self.device).cuda_stream
+
+    def sample(self, seeds, rng_seed: int) -> list[Block]:
+        torch = self.torch
+        assert seeds.dtype == torch.int32 and seeds.is_cuda and seeds.is_contiguous()
+        dsp_sample(self.ctx, seeds, seeds.numel(), self.fanouts, rng_seed, self._cblocks, self.workspace,
+                   self.workspace_bytes, self.stream())
+        return self.blocks()
+
+    def blocks(self) -> list[Block]:
+        out = []
+        for l, (ip, ix, sr) in enumerate(self._bufs):
+            b = self._cblocks[l]
+            out.append(Block(b.num_dst, b.num_src, b.num_edges, ip[: b.num_dst + 1], ix[: b.num_edges],
+                             sr[: b.num_src]))
+        return out
+
+    def gather(self, ids, out=None):
+        torch = self.torch
+        n = ids.numel()
+        if out is None:
+            out = torch.empty((n, self.dim), dtype=torch.float32, device=ids.device)
+        dsp_gather_features(self.ctx, ids, n, out, self.stream())
+        return out
+
+    def sync(self) -> None:
+        dsp_sync(self.ctx, self.stream())
+
+    def close(self) -> None:
+        if getattr(self, "ctx", None) is not None:
+            dsp_destroy(self.ctx)
+            self.ctx = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def torch_exchange(group=None) -> Callable[[bytes], list]:
+    """all-gather of the peer handles over torch.distributed (plumbing)."""
+    import torch.distributed as dist
+
+    def ex(blob: bytes) -> list:
+        out = [None] * dist.get_world_size(group)
+        dist.all_gather_object(out, blob, group=group)
+        return out
+    return ex
+
+
+class LocalGroup:
+    """All ranks of a world in one process, driven by one host thread through
+    dsp_sample_group.  Ranks may share a device (virtual ranks: stages are
+    issued rank by rank on the device's current stream) or sit on several
+    GPUs of this node."""
+
+    def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int]):
+        P = len(shards)
+        assert len(devices) == P and len(bounds) == P + 1
+        self.samplers = [Sampler(bounds, s[0], s[1], s[2], fanouts, max_seeds, rank=r, world_size=P,
+                                 device=devices[r], connect=False) for r, s in enumerate(shards)]
+        handles = [dsp_export_handle(s.ctx) for s in self.samplers]
+        for s in self.samplers:
+            if P > 1:
+                dsp_import_handles(s.ctx, handles)
+            s.connected = True
+        self.fanouts = list(fanouts)
+
+    def sample(self, seeds_per_rank, rng_seed: int) -> list[list[Block]]:
+        S = self.samplers
+        dsp_sample_group([s.ctx for s in S], seeds_per_rank, [x.numel() for x in seeds_per_rank],
+                         self.fanouts, rng_seed, [s._cblocks for s in S], [s.workspace for s in S],
+                         S[0].workspace_bytes, [s.stream() for s in S])
+        return [s.blocks() for s in S]
+
+    def close(self):
+        for s in self.samplers:
+            s.close()

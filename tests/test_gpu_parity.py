@@ -1,0 +1,255 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle,
+bit-exact on every block array and on the gathered feature bits.
+
+Sizes: the tiny config on every batch of an epoch (many tiles + ragged
+tails), the products-shaped graph at full size in the launch configuration
+bench.py times (whole batches: the oracle finishes one in well under a
+second), virtual multi-rank worlds (P = 2, 4, 8 ranks sharing the GPU through
+dsp_sample_group, same kernels and peer-write protocol as multi-GPU), the
+paper's worked examples, and the edge cases (empty / ragged batches, deg <= k,
+k = 1 and k = 32, duplicate and out-of-range seeds)."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+@pytest.fixture(scope="module")
+def pkg():
+    if not torch.cuda.is_available():
+        pytest.fail("GPU tests need a CUDA device (run under gpurun)")
+    import paper_conf_ppopp_caiz0zszck23_b200 as p
+    from paper_conf_ppopp_caiz0zszck23_b200 import _build
+    _build.build()
+    torch.cuda.set_device(0)
+    return p
+
+
+def assert_blocks_equal(got, ref, where=""):
+    assert len(got) == len(ref)
+    for l, (b, r) in enumerate(zip(got, ref)):
+        assert b.num_dst == r["num_dst"] and b.num_src == r["num_src"] and b.num_edges == r["num_edges"], \
+            f"{where} layer {l} sizes {(b.num_dst, b.num_src, b.num_edges)} vs " \
+            f"{(r['num_dst'], r['num_src'], r['num_edges'])}"
+        for key in ("indptr", "indices", "src_ids"):
+            got_a = getattr(b, key).cpu().numpy()
+            if not np.array_equal(got_a, r[key]):
+                bad = np.nonzero(got_a != r[key])[0][:5] if got_a.shape == r[key].shape else "shape"
+                raise AssertionError(f"{where} layer {l} {key} differs at {bad}")
+
+
+def seeds_of(cfg, P, rank, epoch=0, batch=None):
+    train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
+    return datagen.rank_seed_batches(train, datagen.bounds(cfg.num_nodes, P), rank, batch or cfg.batch, epoch)
+
+
+@pytest.fixture(scope="module")
+def tiny():
+    cfg = datagen.CONFIGS["tiny"]
+    ip, ix = datagen.make_graph(cfg)
+    feats = datagen.features(0, cfg.num_nodes, cfg.dim)
+    return cfg, ip, ix, feats
+
+
+# ------------------------------------------------------------------- P = 1
+
+def test_tiny_every_batch_of_an_epoch(pkg, tiny):
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch)
+    batches = seeds_of(cfg, 1, 0)
+    assert len(batches) > 100
+    for step, seeds in enumerate(batches):
+        rng = datagen.BASE_SEED + step
+        blocks = s.sample(torch.from_numpy(seeds).cuda(), rng)
+        ref = oracle.sample(ip, ix, seeds, cfg.fanouts, rng)
+        assert_blocks_equal(blocks, ref, f"tiny step {step}")
+        if step % 10 == 0:
+            out = s.gather(blocks[-1].src_ids)
+            s.sync()
+            exp = oracle.gather(feats, ref[-1]["src_ids"])
+            assert np.array_equal(out.cpu().numpy().view(np.uint32), exp.view(np.uint32))
+    s.close()
+
+
+@pytest.mark.parametrize("fanouts", [(1,), (32,), (3, 7, 2), (32, 1), (9, 17)])
+def test_fanout_range_and_ragged_batches(pkg, tiny, fanouts):
+    """k = 1 (random-walk step), k = 32 (full warp), odd k (ragged lane groups),
+    and batch sizes that are not a multiple of anything."""
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, fanouts, 100)
+    rng = np.random.default_rng(5)
+    for B in (1, 2, 33, 97, 100):
+        seeds = rng.choice(cfg.num_nodes, size=B, replace=False).astype(np.int32)
+        blocks = s.sample(torch.from_numpy(seeds).cuda(), 1000 + B)
+        assert_blocks_equal(blocks, oracle.sample(ip, ix, seeds, fanouts, 1000 + B), f"B={B}")
+    s.close()
+
+
+def test_empty_batch(pkg, tiny):
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8)
+    blocks = s.sample(torch.zeros(0, dtype=torch.int32, device="cuda"), 3)
+    assert all(b.num_dst == 0 and b.num_edges == 0 and b.num_src == 0 for b in blocks)
+    assert blocks[0].indptr.cpu().tolist() == [0]
+    s.close()
+
+
+def test_errors_latched_and_reported(pkg, tiny):
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 16)
+    with pytest.raises(pkg.DSPError) as e:
+        s.sample(torch.tensor([5, 9, 5], dtype=torch.int32, device="cuda"), 1)
+    assert e.value.status == pkg.dsp.DSP_ERR_DUPLICATE_SEED
+    with pytest.raises(pkg.DSPError) as e:
+        s.sample(torch.tensor([5, cfg.num_nodes], dtype=torch.int32, device="cuda"), 1)
+    assert e.value.status == pkg.dsp.DSP_ERR_OUT_OF_RANGE
+    with pytest.raises(pkg.DSPError) as e:
+        s.sample(torch.arange(17, dtype=torch.int32, device="cuda"), 1)
+    assert e.value.status == pkg.dsp.DSP_ERR_CAPACITY
+    # the ctx stays usable after a device-detected error
+    seeds = np.array([1, 2, 3], np.int32)
+    assert_blocks_equal(s.sample(torch.from_numpy(seeds).cuda(), 4), oracle.sample(ip, ix, seeds, cfg.fanouts, 4))
+    with pytest.raises(pkg.DSPError) as e:
+        s.gather(torch.tensor([-1], dtype=torch.int32, device="cuda"))
+        s.sync()
+    assert e.value.status == pkg.dsp.DSP_ERR_OUT_OF_RANGE
+    s.close()
+
+
+def _csr_from_rows(n, rows):
+    ip = np.zeros(n + 1, np.int64)
+    cols = []
+    for v in range(n):
+        r = sorted(rows.get(str(v), []))
+        cols += r
+        ip[v + 1] = ip[v] + len(r)
+    return ip, np.array(cols, np.int32)
+
+
+def test_fig3_worked_example_on_gpu(pkg):
+    g = json.load(open(os.path.join(GOLDEN, "fig3_worked_example.json")))
+    ip, ix = _csr_from_rows(g["num_nodes"], g["rows"])
+    feats = datagen.features(0, g["num_nodes"], 4)
+    s = pkg.Sampler([0, g["num_nodes"]], ip, ix, feats, g["fanouts"], 1)
+    blocks = s.sample(torch.tensor(g["seeds"], dtype=torch.int32, device="cuda"), 77)
+    for b, e in zip(blocks, g["blocks"]):
+        for key in ("indptr", "indices", "src_ids"):
+            assert getattr(b, key).cpu().tolist() == e[key]
+    s.close()
+
+
+def test_fig5_csp_example_virtual_two_gpus(pkg):
+    g = json.load(open(os.path.join(GOLDEN, "fig5_csp_example.json")))
+    ip, ix = _csr_from_rows(g["num_nodes"], g["rows"])
+    bnds = np.array(g["bounds"], np.int64)
+    feats = datagen.features(0, g["num_nodes"], 4)
+    shards = []
+    for r in range(2):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi]))
+    grp = pkg.LocalGroup(bnds, shards, g["fanouts"], 2, devices=[0, 0])
+    seeds = [torch.tensor(x, dtype=torch.int32, device="cuda") for x in g["rank_seeds"]]
+    res = grp.sample(seeds, 9)
+    for r in range(2):
+        for b, e in zip(res[r], g["blocks"][r]):
+            for key in ("indptr", "indices", "src_ids"):
+                assert getattr(b, key).cpu().tolist() == e[key], (r, key)
+        # one-sided gather across the two shards
+        out = grp.samplers[r].gather(res[r][-1].src_ids)
+        grp.samplers[r].sync()
+        assert np.array_equal(out.cpu().numpy(), feats[res[r][-1].src_ids.cpu().numpy()])
+    grp.close()
+
+
+# ------------------------------------------------------- virtual P = 2,4,8
+
+@pytest.mark.parametrize("P", [2, 4, 8])
+def test_tiny_virtual_ranks(pkg, tiny, P):
+    cfg, ip, ix, feats = tiny
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi]))
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P)
+    per_rank = [seeds_of(cfg, P, r, batch=32) for r in range(P)]
+    steps = min(len(x) for x in per_rank)
+    for step in range(min(steps, 6)):
+        seeds = [per_rank[r][step] for r in range(P)]
+        if step == 1:
+            seeds[0] = seeds[0][:0]                  # a rank with an empty batch still joins
+        if step == 2:
+            seeds[P - 1] = np.concatenate([seeds[P - 1][:5], per_rank[0][step][:3]])  # remote seeds
+        res = grp.sample([torch.from_numpy(np.ascontiguousarray(s)).cuda() for s in seeds], 0x5EED + step)
+        for r in range(P):
+            ref = oracle.sample(ip, ix, seeds[r], cfg.fanouts, 0x5EED + step)
+            assert_blocks_equal(res[r], ref, f"P={P} rank {r} step {step}")
+            out = grp.samplers[r].gather(res[r][-1].src_ids)
+            grp.samplers[r].sync()
+            exp = oracle.gather(feats, ref[-1]["src_ids"])
+            assert np.array_equal(out.cpu().numpy().view(np.uint32), exp.view(np.uint32))
+    grp.close()
+
+
+# ----------------------------------------------------- products, full size
+
+@pytest.fixture(scope="module")
+def products():
+    cfg = datagen.CONFIGS["products"]
+    ip, ix = datagen.make_graph(cfg)
+    return cfg, ip, ix
+
+
+@pytest.mark.slow
+def test_products_full_size_p1(pkg, products):
+    """BASELINE.json configs[1] in bench.py's launch configuration: whole
+    1024-seed batches compared bit-exactly; the gather checked on every row
+    against the closed-form feature recipe."""
+    cfg, ip, ix = products
+    feats = datagen.features(0, cfg.num_nodes, cfg.dim)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch)
+    batches = seeds_of(cfg, 1, 0)
+    for step in (0, 1, len(batches) - 1):
+        seeds = batches[step]
+        rng = datagen.BASE_SEED + step
+        blocks = s.sample(torch.from_numpy(seeds).cuda(), rng)
+        ref = oracle.sample(ip, ix, seeds, cfg.fanouts, rng)
+        assert_blocks_equal(blocks, ref, f"products step {step}")
+        out = s.gather(blocks[-1].src_ids)
+        s.sync()
+        exp = datagen.features_of(ref[-1]["src_ids"], cfg.dim)
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), exp.view(np.uint32))
+    s.close()
+
+
+@pytest.mark.slow
+def test_products_virtual_p4(pkg, products):
+    cfg, ip, ix = products
+    P = 4
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, datagen.features(lo, hi, cfg.dim)))
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, cfg.batch, devices=[0] * P)
+    seeds = [seeds_of(cfg, P, r)[0] for r in range(P)]
+    res = grp.sample([torch.from_numpy(s).cuda() for s in seeds], 0x5EED)
+    for r in range(P):
+        assert_blocks_equal(res[r], oracle.sample(ip, ix, seeds[r], cfg.fanouts, 0x5EED), f"rank {r}")
+    out = grp.samplers[1].gather(res[1][-1].src_ids)
+    grp.samplers[1].sync()
+    exp = datagen.features_of(res[1][-1].src_ids.cpu().numpy(), cfg.dim)
+    assert np.array_equal(out.cpu().numpy().view(np.uint32), exp.view(np.uint32))
+    grp.close()
