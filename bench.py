@@ -215,36 +215,44 @@ def cpu_baseline(cfg, ip, ix, feats, batches, seconds: float):
 
 # ----------------------------------------------------------------- product
 
+def algorithmic_bytes(sizes, L, dim):
+    """24 B per frontier node, 8 B per sampled edge, 4 B per
+    new unique node, and 2 * dim * 4 B per gathered row (read + write)."""
+    F = sum(int(sizes[3 * l]) for l in range(L))
+    E = sum(int(sizes[3 * l + 2]) for l in range(L))
+    new = sum(int(sizes[3 * l + 1]) - int(sizes[3 * l]) for l in range(L))
+    U = int(sizes[3 * (L - 1) + 1])
+    return 24 * F + 8 * E + 4 * new, 2 * U * dim * 4
+
+
 def run_dsp(args):
     import datagen
     import paper_conf_ppopp_caiz0zszck23_b200 as pkg
     rank, world, local = setup_dist(args.gpus)
     torch.cuda.set_device(local)
-    cfg_name = args.config
-    cfg, ip, ix, bnds, sip, six, feats, train = load_workload(cfg_name, rank, world)
+    cfg, ip, ix, bnds, sip, six, feats, train = load_workload(args.config, rank, world)
     ex = pkg.torch_exchange() if world > 1 else None
     s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, cfg.batch, rank=rank, world_size=world,
-                    device=local, exchange=ex)
+                    device=local, exchange=ex, n_slots=2)
+    L = len(cfg.fanouts)
     steps_epoch = datagen.steps_per_epoch(train, bnds, cfg.batch)
     batches = datagen.rank_seed_batches(train, bnds, rank, cfg.batch, 0)[:steps_epoch]
-    need = args.warmup + args.steps
     dev_batches = torch.from_numpy(np.ascontiguousarray(batches)).cuda()   # inputs resident in HBM
-    max_rows = s.max_src[-1]
-    out = torch.empty((max_rows, cfg.dim), dtype=torch.float32, device="cuda")
     stream = torch.cuda.current_stream()
+    K, W = args.steps, args.warmup
+    h_sizes = torch.zeros((W + K, 3 * L), dtype=torch.int64).pin_memory()
 
-    def step(i, timed_gather=None):
-        seeds = dev_batches[i % len(batches)]
-        blocks = s.sample(seeds, datagen.BASE_SEED + i)
-        U = blocks[-1].num_src
-        if timed_gather is not None:
-            timed_gather[0].record(stream)
-        s.gather(blocks[-1].src_ids, out[:U])
-        if timed_gather is not None:
-            timed_gather[1].record(stream)
-        return blocks
+    def step(i, ev=None):
+        # one step = the whole hot path (CSP over all layers + feature gather), enqueued
+        # asynchronously; two output sets alternate (queue capacity 2, P:L198-200)
+        if ev is not None:
+            ev[0].record(stream)
+        s.sample_gather(dev_batches[i % len(batches)], datagen.BASE_SEED + i, slot=i % 2,
+                        sizes_out=h_sizes[i], async_=True)
+        if ev is not None:
+            ev[1].record(stream)
 
-    for i in range(args.warmup):
+    for i in range(W):
         step(i)
     s.sync()
     barrier()
@@ -252,37 +260,70 @@ def run_dsp(args):
 
     # ---- timed region: K steps, inputs resident, device time via CUDA events
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    gev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    edges = rows = seeds_n = 0
+    sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
     with ClockSampler(local) as clk:
         ev0.record(stream)
-        for j in range(args.steps):
-            blocks = step(args.warmup + j, gev[j])
-            edges += sum(b.num_edges for b in blocks)
-            rows += blocks[-1].num_src
-            seeds_n += blocks[0].num_dst
+        for j in range(K):
+            step(W + j, sev[j])
         ev1.record(stream)
         s.sync()
         torch.cuda.synchronize()
     barrier()
     t_ms = ev0.elapsed_time(ev1)
-    g_ms = [a.elapsed_time(b) for a, b in gev]
+    step_ms = [a.elapsed_time(b) for a, b in sev]
+    sz = h_sizes.numpy()[W: W + K]
+    edges = float(sum(int(sz[j, 3 * l + 2]) for j in range(K) for l in range(L)))
+    rows = float(sum(int(sz[j, 3 * (L - 1) + 1]) for j in range(K)))
+    seeds_n = float(sum(int(sz[j, 0]) for j in range(K)))
+    samp_b = gath_b = 0
+    for j in range(K):
+        a, b = algorithmic_bytes(sz[j], L, cfg.dim)
+        samp_b += a
+        gath_b += b
     t_max = reduce_max_over_ranks(t_ms)
     tot_edges = reduce_sum_over_ranks(edges)
     tot_rows = reduce_sum_over_ranks(rows)
     tot_seeds = reduce_sum_over_ranks(seeds_n)
-    g_mean = float(np.mean(g_ms))
-    gather_bytes_per_launch = 2.0 * (rows / args.steps) * cfg.dim * 4      # read + write, algorithmic
-    achieved = gather_bytes_per_launch / (g_mean * 1e-3) / 1e9
     peak, peak_kind = measured_peaks()
+    step_mean = float(np.mean(step_ms))
+    achieved = (samp_b + gath_b) / K / (step_mean * 1e-3) / 1e9
+
+    # ---- breakdown (not the headline): the two calls separately
+    ids_dev = None
+    bd = {}
+    if not args.no_breakdown:
+        g_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+        s_ms = []
+        nrow = []
+        out = s.feat_buffer(0)
+        for j in range(K):
+            i = W + j
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            blocks = s.sample(dev_batches[i % len(batches)], datagen.BASE_SEED + i)
+            a1.record(stream)
+            ids_dev = blocks[-1].src_ids
+            g_ev[j][0].record(stream)
+            s.gather(ids_dev, out[: ids_dev.numel()])
+            g_ev[j][1].record(stream)
+            nrow.append(ids_dev.numel())
+            torch.cuda.synchronize()
+            s_ms.append(a0.elapsed_time(a1))
+        s.sync()
+        g_ms = [a.elapsed_time(b) for a, b in g_ev]
+        g_bytes = [2.0 * n * cfg.dim * 4 for n in nrow]
+        bd = {"sample_call_ms_mean": float(np.mean(s_ms)), "gather_call_ms_mean": float(np.mean(g_ms)),
+              "gather_GBps": float(np.mean([b / (m * 1e-3) / 1e9 for b, m in zip(g_bytes, g_ms)])),
+              "gather_frac_of_hbm": float(np.mean([b / (m * 1e-3) / 1e9 for b, m in zip(g_bytes, g_ms)])) / peak,
+              "note": "dsp_sample (synchronous, host sizes) and dsp_gather_features timed separately"}
 
     # ---- e2e: the same steps through the C ABI with HOST buffers: pinned seeds
-    # H2D, sample, gather, D2H of the blocks and the gathered features
+    # H2D, sample + gather, D2H of the blocks and the gathered features
     h_seeds = torch.from_numpy(np.ascontiguousarray(batches)).pin_memory()
-    h_feat = torch.empty((max_rows, cfg.dim), dtype=torch.float32).pin_memory()
+    h_feat = torch.empty((s.max_src[-1], cfg.dim), dtype=torch.float32).pin_memory()
     h_blk = [tuple(torch.empty(x.numel(), dtype=torch.int32).pin_memory() for x in bufs) for bufs in s._bufs]
     d_seed = torch.empty(cfg.batch, dtype=torch.int32, device="cuda")
-    e2e_steps = max(3, min(args.steps, 20))
+    e2e_steps = max(3, min(K, 20))
     h2d = d2h = 0
     barrier()
     torch.cuda.synchronize()
@@ -290,19 +331,17 @@ def run_dsp(args):
     e2e_edges = 0
     e0.record(stream)
     for j in range(e2e_steps):
-        i = args.warmup + j
+        i = W + j
         d_seed.copy_(h_seeds[i % len(batches)], non_blocking=True)
         h2d += d_seed.numel() * 4
-        blocks = s.sample(d_seed, datagen.BASE_SEED + i)
-        U = blocks[-1].num_src
-        s.gather(blocks[-1].src_ids, out[:U])
+        blocks, feat = s.sample_gather(d_seed, datagen.BASE_SEED + i, slot=0)
         for b, hb in zip(blocks, h_blk):
             hb[0][: b.num_dst + 1].copy_(b.indptr, non_blocking=True)
             hb[1][: b.num_edges].copy_(b.indices, non_blocking=True)
             hb[2][: b.num_src].copy_(b.src_ids, non_blocking=True)
             d2h += 4 * (b.num_dst + 1 + b.num_edges + b.num_src)
-        h_feat[:U].copy_(out[:U], non_blocking=True)
-        d2h += U * cfg.dim * 4
+        h_feat[: feat.shape[0]].copy_(feat, non_blocking=True)
+        d2h += feat.numel() * 4
         e2e_edges += sum(b.num_edges for b in blocks)
     e1.record(stream)
     torch.cuda.synchronize()
@@ -313,32 +352,35 @@ def run_dsp(args):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(cfg, ip, ix, feats, batches, args.cpu_seconds)
 
-    kern_per_step = (3 if world == 1 else 5) * len(cfg.fanouts) + 1
+    kern_per_step = 1 if world == 1 else 5 * L + 1
     if rank == 0:
         line = {
             "metric": METRIC, "value": tot_edges / (t_max * 1e-3), "unit": "edges/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_max / args.steps,
+            "steps": K, "warmup": W, "ms_per_step": t_max / K,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32+f32",
             "data": "synthetic",
             "config": {"workload": cfg.name if world == 1 else f"{cfg.name}-P{world}",
                        "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes,
                        "nnz": int(ip[-1]), "dim": cfg.dim, "parallelism": f"csp{world}",
-                       "l2": "inputs larger than L2 (CSR + features >> 126 MB; per-step gather moves ~0.5 GB)"},
+                       "l2": "inputs larger than L2 (CSR 0.5 GB + features 1.1 GB >> 126 MB L2)",
+                       "step": "dsp_sample_gather (async, 2 output sets)"},
             "seeds_per_s": tot_seeds / (t_max * 1e-3),
             "feature_GBps": tot_rows * cfg.dim * 4 / (t_max * 1e-3) / 1e9,
-            "gather_kernel_GBps": achieved,
-            "edges_per_step": tot_edges / args.steps / world,
-            "rows_per_step": tot_rows / args.steps / world,
-            "roofline": {"kernel": "k_gather", "bound": "hbm" if world == 1 else "nvlink",
-                         "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                         "traffic": ncu_traffic("k_gather"), "peak_kind": peak_kind,
-                         "algorithmic_bytes_per_launch": gather_bytes_per_launch,
-                         "gather_ms_mean": g_mean, "gather_share_of_step": g_mean / (t_ms / args.steps)},
+            "edges_per_step": tot_edges / K / world,
+            "rows_per_step": tot_rows / K / world,
+            "roofline": {"kernel": "k_csp_persistent" if world == 1 else "k_gather",
+                         "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                         "frac": achieved / peak, "traffic": ncu_traffic("k_csp_persistent"),
+                         "peak_kind": peak_kind,
+                         "algorithmic_bytes_per_launch": (samp_b + gath_b) / K,
+                         "sampling_bytes_per_launch": samp_b / K, "gather_bytes_per_launch": gath_b / K,
+                         "launch_ms_mean": step_mean},
+            "breakdown": bd,
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_edges / (e2e_ms * 1e-3), "unit": "edges/s",
                     "h2d_bytes_per_step": h2d // e2e_steps, "d2h_bytes_per_step": d2h // e2e_steps,
-                    "steps": e2e_steps},
-            "gpu_launches": kern_per_step * args.steps,
+                    "steps": e2e_steps, "api": "dsp_sample_gather (synchronous) + D2H of blocks and features"},
+            "gpu_launches": kern_per_step * K,
             "clocks": clk.summary(),
         }
         print(json.dumps(line), flush=True)
@@ -358,6 +400,7 @@ def main(argv=None):
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-max-seconds", type=float, default=60.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-breakdown", action="store_true")
     args = ap.parse_args(argv)
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

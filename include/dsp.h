@@ -92,7 +92,8 @@ void dsp_destroy(dsp_ctx *ctx);
              indptr[0] = 0, non-decreasing.
    indices : host or device int32[indptr[n_r]]: GLOBAL ids of the
              in-neighbours of local row v (global id bounds[rank] + v), each
-             row strictly ascending (R9).
+             row strictly ascending (R9); an id outside [0, N)
+             fails the load with DSP_ERR_OUT_OF_RANGE.
    features: host or device fp32[n_r][dim] row-major, or NULL for none.
    dim     : 4 <= dim <= 4096 and dim % 4 == 0 (16-byte rows); ignored when
              features is NULL.
@@ -148,7 +149,11 @@ dsp_status dsp_sample_bounds(const dsp_ctx *ctx, int32_t num_seeds, const int32_
               cover dsp_sample_bounds (else DSP_ERR_CAPACITY before any work).
               blocks[l].src_ids is the frontier of layer l+1; the last block's
               src_ids are the unique nodes whose features the loader needs.
-   workspace: DEVICE, >= workspace_bytes from dsp_sample_bounds.
+   workspace: DEVICE, 256-byte aligned, >= workspace_bytes from
+              dsp_sample_bounds, ZERO-FILLED before its first use; afterwards
+              it belongs to the library (it carries the relabel map's epoch
+              from call to call, so the map is never cleared): pass it back
+              unmodified, or zero it again.  One workspace per ctx at a time.
    Stream-ordered on `stream`; returns after one stream synchronisation with
    the host-side sizes filled.  The result is a pure function of (graph,
    seeds, fanouts, rng_seed): bit-identical for any world_size / bounds and
@@ -167,6 +172,33 @@ dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *
                             const int32_t *num_seeds, const int32_t *fanouts, int32_t num_layers,
                             uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
                             size_t workspace_bytes, void *const *streams);
+
+/* Flag for dsp_sample_gather. */
+#define DSP_ASYNC 1u
+
+/* One whole step of the hot path in ONE stream-ordered call: dsp_sample
+   followed by the feature gather of the last block's src_ids (the loader
+   right after the sampler), with no host round trip in between.
+   With world_size == 1 the step runs as a single persistent kernel.
+   Same arguments, rules and collectiveness as dsp_sample, plus:
+   feat_out     : DEVICE fp32 [feat_cap_rows][dim], 16-byte aligned; rows
+                  [0, blocks[L-1].num_src) receive the features of
+                  blocks[L-1].src_ids, bit-exact.
+   feat_cap_rows: >= max_src[L-1] of dsp_sample_bounds (else DSP_ERR_CAPACITY).
+   sizes_out    : NULL, or int64[3 * num_layers] (HOST pinned or DEVICE)
+                  receiving {num_dst, num_src, num_edges} per layer.
+   flags        : 0 = synchronous: returns after one stream synchronisation
+                  with blocks[l].num_* (and sizes_out) filled and device
+                  errors reported.  DSP_ASYNC = returns once the step is
+                  enqueued; blocks[l].num_* are NOT filled, sizes_out is
+                  written when the stream reaches the end of the step, and
+                  device errors latch until dsp_sync.  Consecutive async
+                  steps may reuse the same workspace and outputs in stream
+                  order (the producer/consumer pipeline of P:L198-200). */
+dsp_status dsp_sample_gather(dsp_ctx *ctx, const int32_t *seeds, int32_t num_seeds, const int32_t *fanouts,
+                             int32_t num_layers, uint64_t rng_seed, dsp_block *blocks, float *feat_out,
+                             int64_t feat_cap_rows, void *workspace, size_t workspace_bytes,
+                             int64_t *sizes_out, uint32_t flags, void *stream);
 
 /* --------------------------------------------------------------- gather */
 

@@ -28,7 +28,8 @@ def stale() -> bool:
 def build(force: bool = False, verbose: bool = False) -> str:
     if force or stale():
         tmp = LIB + f".tmp{os.getpid()}"
-        cmd = [NVCC, *NVCC_FLAGS, *(["-Xptxas", "-v"] if verbose else []), "-o", tmp, *SOURCES]
+        extra = ["-DDSP_DEBUG_STAMPS"] if os.environ.get("DSP_DEBUG_STAMPS") else []
+        cmd = [NVCC, *NVCC_FLAGS, *extra, *(["-Xptxas", "-v"] if verbose else []), "-o", tmp, *SOURCES]
         subprocess.check_call(cmd)
         os.replace(tmp, LIB)
     return LIB

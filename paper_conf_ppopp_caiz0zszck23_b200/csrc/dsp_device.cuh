@@ -60,12 +60,12 @@ __device__ __forceinline__ uint32_t hash32(uint32_t x) {
   return x;
 }
 
-// Inserts (key, val) keeping the minimum val.  Returns the slot index and the
-// previous val of the key in *old (0xffffffff if the key was new).
-__device__ __forceinline__ uint32_t table_insert_min(unsigned long long *tbl, uint32_t mask,
-                                                     uint32_t key, uint32_t val, uint32_t *old) {
+// Inserts (key, val) keeping the minimum val, probing from slot `idx`.
+// Returns the slot index and the previous val of the key in *old
+// (0xffffffff if the key was new).
+__device__ __forceinline__ uint32_t table_insert_min_from(unsigned long long *tbl, uint32_t mask, uint32_t idx,
+                                                          uint32_t key, uint32_t val, uint32_t *old) {
   const unsigned long long want = ((unsigned long long)key << 32) | val;
-  uint32_t idx = hash32(key) & mask;
   while (true) {
     unsigned long long cur = *(volatile unsigned long long *)&tbl[idx];
     if (cur == EMPTY_SLOT) {
@@ -84,6 +84,25 @@ __device__ __forceinline__ uint32_t table_insert_min(unsigned long long *tbl, ui
     }
     idx = (idx + 1) & mask;
   }
+}
+
+__device__ __forceinline__ uint32_t table_insert_min(unsigned long long *tbl, uint32_t mask, uint32_t key,
+                                                     uint32_t val, uint32_t *old) {
+  return table_insert_min_from(tbl, mask, hash32(key) & mask, key, val, old);
+}
+
+// Completion of an insertion whose first CAS at its home slot `idx` (issued
+// speculatively, expecting an empty slot) returned `prev` != EMPTY.
+__device__ __forceinline__ uint32_t table_insert_finish(unsigned long long *tbl, uint32_t mask, uint32_t idx,
+                                                        uint32_t key, uint32_t val, unsigned long long prev,
+                                                        uint32_t *old) {
+  if ((uint32_t)(prev >> 32) == key) {
+    uint32_t o = (uint32_t)prev;
+    if (o > val) o = (uint32_t)atomicMin(&tbl[idx], ((unsigned long long)key << 32) | val);
+    *old = o;
+    return idx;
+  }
+  return table_insert_min_from(tbl, mask, (idx + 1) & mask, key, val, old);
 }
 
 // ------------------------------------------------------ peer-memory flags

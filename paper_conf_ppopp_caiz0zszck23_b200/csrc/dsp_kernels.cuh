@@ -1,325 +1,678 @@
-// dsp_kernels.cuh -- the CSP layer kernels and the feature gather (sm_100a).
+// dsp_kernels.cuh -- CSP layer phases and the feature gather (sm_100a).
 //
-// Per layer l:
-//   world == 1 : k_sample_local           (sample + hash insert, fused)
-//   world  > 1 : k_bucket_scatter         (shuffle: ids -> owners' inboxes over NVLink)
-//                k_sample_remote          (sample at the owner, rows -> requesters)
-//                k_unpermute_insert       (reshuffle consumer + hash insert)
-//   then       : k_scan_assign            (single-pass scan: indptr, first occurrences,
-//                                          new local ids, src_ids)
-//                k_write_indices          (local src ids per edge)
-// and k_gather for the loader.
+// Phases of one layer l:
+//   sample  : world == 1: sample every frontier node, record the sampled
+//             neighbour of each edge slot and mark dst / src in the relabel
+//             map (fused).  world > 1: bucket scatter -> sample at the owner ->
+//             unpermute + mark (exchange through NVLink peer memory)
+//   scan    : prefix over edge slots: block indptr, first occurrences, new
+//             local ids, src_ids
+//   indices : local src id of every edge
+// and the gather of the last block's src_ids.
+//
+// Relabel map: first[p][u] for every global id u, a
+// 64-bit word (epoch << 32) | ~x where x is the smallest "order key" marked
+// for u in this layer: the dst index i (< F) or F + q for edge slot q.  One
+// fire-and-forget atomicMax per mark (no return value, no probing); a newer
+// epoch beats every stale word, so the map is never cleared.  Edge slots are
+// ordered exactly as the output edges (dst index, then row position), so
+// "x == F + q" identifies the first occurrence of a new src node.
+//
+// world == 1 runs the whole call in ONE persistent cooperative kernel
+// (k_csp_persistent, one 1024-thread block per SM) with grid barriers between
+// phases; world > 1 issues one kernel per phase so that ranks sharing a GPU
+// can be interleaved stage by stage and exchanges never wait inside a kernel
+// on work queued behind it.
+//
+// Data a phase reads after another phase of the same kernel wrote it is read
+// with ld.global.cg (L2), never through the non-coherent path.
 #pragma once
 #include "dsp_device.cuh"
 
 namespace dsp {
 
-// Device-side per-call state at the start of the caller's workspace.  The
-// host copies it back once per dsp_sample.
+constexpr int NT = 256;    // threads per block of the per-phase kernels
+constexpr int PNT = 1024;  // threads per block of the persistent kernel (1 block per SM)
+constexpr int MAX_PERSIST_BLOCKS = 1024;
+
+// Persistent part of the workspace (offset 0).  Zero-filled before first use.
+struct WsPersist {
+  uint32_t epoch;  // last relabel epoch used with this workspace
+  uint32_t pad[63];
+};
+
+// Per-call state (memset to 0 by the host before every call).
 struct WsHeader {
-  int32_t err;
-  int32_t pad0;
   int32_t F[9];          // frontier size per layer (F[0] = num_seeds)
   int32_t S[8];          // num_src per layer
   int64_t E[8];          // num_edges per layer
-  uint32_t done;         // last-block counter (bucket / remote sample)
+  int64_t sizes[24];     // {num_dst, num_src, num_edges} per layer, for async callers
+  uint32_t done;         // last-block counter
   uint32_t bucket[8];    // per-owner send counters (bucket scatter)
-  uint32_t pad1[3];
+  uint32_t bar_count;    // grid barrier arrivals
+  uint32_t pad[6];
+  unsigned long long t[24];   // %globaltimer at kernel start and when block 0 leaves each grid barrier
+  unsigned long long ta[24];  // %globaltimer when block 0 arrives at each grid barrier
+  unsigned long long dbg[32]; // debug stamps (DSP_DEBUG_STAMPS builds only)
 };
 
-// ----------------------------------------------------------- local sample
-struct LocalSampleArgs {
-  const int32_t *frontier;  // layer 0: seeds; else the previous block's src_ids
-  int32_t F0;               // layer 0 only
-  int32_t layer, k;
-  uint2 key;                // rng_seed
-  const int64_t *indptr;    // this rank's CSR
-  const int32_t *indices;
-  int64_t lo, n_local;      // rows [lo, lo + n_local) are local
-  unsigned long long *tbl;
-  uint32_t mask;
-  int32_t *cnt;             // [F]
-  int32_t *hpos;            // [F*k] table slot of each sampled edge
-  WsHeader *hdr;
+// One parity (layer % 2) of the workspace.
+struct LayerBufs {
+  int32_t *cnt;                 // [F] sampled count per frontier node
+  int32_t *rows;                // [F*k] sampled neighbour (global id) of edge slot q = i*k + slot
+  unsigned long long *status;   // [0] tile ticket, [1 + t] tile status (look-back scan)
+  unsigned long long *first;    // [N] relabel map
 };
 
-__device__ __forceinline__ int frontier_size(const WsHeader *hdr, int layer, int F0) {
-  return layer == 0 ? F0 : *(volatile const int32_t *)&hdr->F[layer];
+struct Outputs {
+  int32_t *indptr[8];
+  int32_t *indices[8];
+  int32_t *src_ids[8];
+};
+
+__device__ __forceinline__ int ldcg_i32(const int32_t *p) { return __ldcg(p); }
+__device__ __forceinline__ unsigned long long ldcg_u64(const unsigned long long *p) { return __ldcg(p); }
+__device__ __forceinline__ int ld_volatile_i32(const int32_t *p) { return *(volatile const int32_t *)p; }
+__device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long *p) {
+  return *(volatile const unsigned long long *)p;
 }
 
-// World size 1: sample every frontier node and insert dst + sampled srcs into
-// the relabel table in the same pass.
-template <int G>
-__global__ void __launch_bounds__(256) k_sample_local(LocalSampleArgs a) {
-  const int F = frontier_size(a.hdr, a.layer, a.F0);
-  if (a.layer == 0 && blockIdx.x == 0 && threadIdx.x == 0) a.hdr->F[0] = a.F0;
-  constexpr int NPW = 32 / G;  // nodes per warp-iteration
-  const int lane = threadIdx.x & 31;
-  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int nwarps = (gridDim.x * blockDim.x) >> 5;
-  const int k = a.k;
-  for (int base = warp * NPW; base < F; base += nwarps * NPW) {
-    const int i = base + lane / G;
-    const bool active = i < F;
-    int32_t v = active ? __ldg(a.frontier + i) : 0;
-    const int64_t lv = (int64_t)v - a.lo;
-    const bool ok = active && v >= 0 && lv >= 0 && lv < a.n_local;
-    if (active && !ok && (lane & (G - 1)) == 0) latch(&a.hdr->err, E_RANGE);
-    int64_t s = 0, d = 0;
-    if (ok) {
-      s = __ldg(a.indptr + lv);
-      d = __ldg(a.indptr + lv + 1) - s;
+// ------------------------------------------------------------ relabel map
+__device__ __forceinline__ unsigned long long mark_word(uint32_t epoch, uint32_t x) {
+  return ((unsigned long long)epoch << 32) | (0xffffffffu - x);
+}
+// x of a word of the current epoch
+__device__ __forceinline__ uint32_t mark_x(unsigned long long w) { return 0xffffffffu - (uint32_t)w; }
+__device__ __forceinline__ void mark(unsigned long long *first, int32_t u, uint32_t epoch, uint32_t x) {
+  atomicMax(first + u, mark_word(epoch, x));  // result unused: compiles to a reduction (RED)
+}
+
+// q / k for a fixed small divisor k: one 64-bit multiply-high with
+// m = ceil(2^64 / k), exact for q < 2^59 (m = 0 encodes k = 1).
+struct FastDiv {
+  unsigned long long m;
+  uint32_t k;
+};
+__host__ __device__ __forceinline__ FastDiv make_fastdiv(uint32_t k) {
+  FastDiv f;
+  f.k = k;
+  f.m = k <= 1 ? 0ull : (~0ull / k) + 1ull;
+  return f;
+}
+__device__ __forceinline__ uint32_t fdiv(uint64_t q, const FastDiv &f) {
+  return f.m ? (uint32_t)__umul64hi(q, f.m) : (uint32_t)q;
+}
+
+#ifdef DSP_DEBUG_STAMPS
+// stamp idx once VAL is available (thread 0 of block 0, first iteration)
+#define DSTAMP(hdr, idx, VAL, layer)                                                   \
+  do {                                                                                 \
+    if (blockIdx.x == 0 && threadIdx.x == 0 && dbg_first && (VAL) != 0x7fffffff)       \
+      (hdr)->dbg[(layer) * 8 + (idx)] = globaltimer_ns();                              \
+  } while (0)
+#else
+#define DSTAMP(hdr, idx, VAL, layer) \
+  do {                               \
+  } while (0)
+#endif
+
+// Items [0, total) of a phase: each block takes one contiguous chunk of
+// ceil(total / nblocks) (small layers spread over every SM instead of
+// filling the first blocks), threads stride inside it.
+struct Span {
+  int64_t end, first, step;
+};
+__device__ __forceinline__ Span block_span(int64_t total) {
+  const int64_t chunk = (total + gridDim.x - 1) / gridDim.x;
+  const int64_t b = min(total, (int64_t)blockIdx.x * chunk);
+  const int64_t e = min(total, b + chunk);
+  return Span{e, b + threadIdx.x, (int64_t)blockDim.x};
+}
+__device__ __forceinline__ Span grid_span(int64_t total) {
+  return Span{total, (int64_t)blockIdx.x * blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x};
+}
+
+// ------------------------------------------------------------ grid barrier
+__device__ __forceinline__ void red_add_release_gpu(uint32_t *p, uint32_t v) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_acquire_gpu_u32(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+
+// Grid barrier for the persistent kernel (all blocks co-resident through the
+// cooperative launch).  hdr->bar_count is a monotonic arrival counter zeroed
+// by the host before the launch; each block tracks the target in a register.
+// bar.sync orders the block's writes before thread 0's release reduction (no
+// return value, so no extra round trip); pollers acquire.  1.25 us at 148
+// blocks, vs 2.5 us for an atomicAdd + generation barrier over 592 blocks
+// (tools/micro/barrier_bench.cu).
+__device__ __forceinline__ void grid_barrier(WsHeader *hdr, uint32_t &target) {
+  __syncthreads();
+  target += gridDim.x;
+  if (threadIdx.x == 0) {
+    const uint32_t g = target / gridDim.x;
+    if (blockIdx.x == 0 && g < 23u) hdr->ta[g] = globaltimer_ns();
+    red_add_release_gpu(&hdr->bar_count, 1u);
+    while (ld_acquire_gpu_u32(&hdr->bar_count) < target) {
     }
-    bool valid;
-    int slot, cnt;
-    int32_t u;
-    sample_node<G>(ok, v, s, d, k, a.layer, a.key, a.indices, &valid, &slot, &u, &cnt);
-    if (ok && (lane & (G - 1)) == 0) {
-      a.cnt[i] = cnt;
-      uint32_t old;
-      table_insert_min(a.tbl, a.mask, (uint32_t)v, (uint32_t)i, &old);
-      if (a.layer == 0 && old < (uint32_t)F && old != (uint32_t)i) latch(&a.hdr->err, E_DUP);
-    } else if (active && !ok && (lane & (G - 1)) == 0) {
-      a.cnt[i] = 0;
-    }
-    if (valid) {
-      const int64_t q = (int64_t)i * k + slot;
-      uint32_t old;
-      a.hpos[q] = (int32_t)table_insert_min(a.tbl, a.mask, (uint32_t)u, (uint32_t)(F + q), &old);
-    }
+    if (blockIdx.x == 0 && g < 23u) hdr->t[g] = globaltimer_ns();
+  }
+  __syncthreads();
+}
+
+// ---------------------------------------------------------------- sampling
+// Marks of one frontier node (dst, index i) and its sampled edges.  At
+// layer 0 the dst mark returns the previous word: another dst of the same
+// epoch there means a duplicate seed.
+__device__ __forceinline__ void mark_dst(unsigned long long *first, int32_t v, int i, int F, int layer,
+                                         uint32_t epoch, int *err) {
+  if (layer == 0) {
+    const unsigned long long old = atomicMax(first + v, mark_word(epoch, (uint32_t)i));
+    if ((uint32_t)(old >> 32) == epoch && mark_x(old) < (uint32_t)F) latch(err, E_DUP);
+  } else {
+    mark(first, v, epoch, (uint32_t)i);
   }
 }
 
-// ------------------------------------------------------------ scan/assign
-// Decoupled look-back scan over edge slots q in [0, F*k) of two counts:
-// valid (edge exists) and first (first occurrence of a new src node).
-// Tile status word: [63:62] flag (3 = not ready, 1 = aggregate, 2 = inclusive)
-// [61:31] first count, [30:0] valid count.  The status array and the tile
-// ticket are reset to all ones by the per-layer table memset.
-constexpr int SCAN_THREADS = 256;
-constexpr int SCAN_ITEMS = 8;
-constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;
-constexpr unsigned long long ST_VAL_MASK = (1ull << 62) - 1;
-constexpr unsigned long long ST_AGG = 1ull << 62;
-constexpr unsigned long long ST_INC = 2ull << 62;
+// Lane-group sampling (G lanes per node, G = next pow2 >= k): the draws run
+// on separate lanes, Floyd's resolution and the ranking via shuffles
+// (sample_node).  Used for k > 16.
+template <int G>
+__device__ __forceinline__ void phase_sample_lanes(const int32_t *frontier, int F, int layer, int k, uint2 key,
+                                                   const int64_t *__restrict__ indptr,
+                                                   const int32_t *__restrict__ indices, int64_t lo,
+                                                   int64_t n_local, const LayerBufs &B, uint32_t epoch,
+                                                   int32_t *src_out, int *err, WsHeader *hdr) {
+  constexpr int NPW = 32 / G;  // nodes per warp-iteration
+  const int lane = threadIdx.x & 31;
+  const bool leader = (lane & (G - 1)) == 0;
+  const Span sp = block_span(F);
+  const int64_t b0 = sp.first - threadIdx.x;  // first node of this block's chunk
+  const int wib = threadIdx.x >> 5, wpb = blockDim.x >> 5;
+  bool dbg_first = true;
+  (void)hdr;
+  for (int64_t base = b0 + (int64_t)wib * NPW; base < sp.end; base += (int64_t)wpb * NPW) {
+    const int i = (int)(base + lane / G);
+    const bool active = i < sp.end;
+    DSTAMP(hdr, 0, 0, layer);
+    const int32_t v = active ? ldcg_i32(frontier + i) : 0;
+    DSTAMP(hdr, 1, v, layer);
+    const int64_t lv = (int64_t)v - lo;
+    const bool ok = active && v >= 0 && lv >= 0 && lv < n_local;
+    int64_t s = 0, d = 0;
+    if (ok) {
+      s = __ldg(indptr + lv);
+      d = __ldg(indptr + lv + 1) - s;
+    }
+    DSTAMP(hdr, 2, (int)d, layer);
+    bool valid;
+    int slot, cnt;
+    int32_t u;
+    sample_node<G>(ok, v, s, d, k, layer, key, indices, &valid, &slot, &u, &cnt);
+    DSTAMP(hdr, 3, u, layer);
+    if (active && leader) {
+      B.cnt[i] = cnt;
+      if (src_out) src_out[i] = v;  // dst copy (R17)
+      if (ok)
+        mark_dst(B.first, v, i, F, layer, epoch, err);
+      else
+        latch(err, E_RANGE);
+    }
+    if (valid) {
+      const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)slot;
+      B.rows[q] = u;
+      mark(B.first, u, epoch, (uint32_t)F + q);
+    }
+    DSTAMP(hdr, 5, 0, layer);
+    dbg_first = false;
+  }
+}
 
-struct ScanArgs {
-  int32_t layer, k;
-  const int32_t *frontier;
-  const int32_t *cnt;
-  const int32_t *hpos;
-  unsigned long long *tbl;
-  unsigned long long *status;  // [0] = ticket, [1 + tile] = tile status
-  int32_t *indptr_out;         // [F+1]
-  int32_t *src_ids_out;        // [F + new]
-  WsHeader *hdr;
-};
+// Thread-per-node sampling for k <= KB: the draws, Floyd's resolution and the
+// ranking run in one thread's registers; the k adjacency loads and the k + 1
+// marks are issued back to back (memory-level parallelism k per thread, every
+// frontier node in flight at once).
+template <int KB>
+__device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F, int layer, int k, uint2 key,
+                                                 const int64_t *__restrict__ indptr,
+                                                 const int32_t *__restrict__ indices, int64_t lo,
+                                                 int64_t n_local, const LayerBufs &B, uint32_t epoch,
+                                                 int32_t *src_out, int *err, WsHeader *hdr) {
+  const Span sp = block_span(F);
+  bool dbg_first = true;
+  (void)hdr;
+  for (int64_t ii = sp.first; ii < sp.end; ii += sp.step) {
+    const int i = (int)ii;
+    DSTAMP(hdr, 0, 0, layer);
+    const int32_t v = ldcg_i32(frontier + i);
+    DSTAMP(hdr, 1, v, layer);
+    if (src_out) src_out[i] = v;  // dst copy (R17)
+    const int64_t lv = (int64_t)v - lo;
+    if (v < 0 || lv < 0 || lv >= n_local) {
+      latch(err, E_RANGE);
+      B.cnt[i] = 0;
+      continue;
+    }
+    const int64_t rs = __ldg(indptr + lv);
+    const int64_t d = __ldg(indptr + lv + 1) - rs;
+    DSTAMP(hdr, 2, (int)d, layer);
+    const bool full = d <= k;
+    const int cnt = full ? (int)d : k;
+    uint32_t pos[KB];
+#pragma unroll
+    for (int t = 0; t < KB; ++t) pos[t] = (uint32_t)t;
+    if (!full) {
+#pragma unroll
+      for (int t = 0; t < KB; ++t)
+        if (t < k) pos[t] = draw_range(key, (uint32_t)t, v, layer, (uint32_t)(d - k + t + 1));
+      // Floyd: step t keeps r_t unless an earlier step chose it, then takes j_t
+#pragma unroll
+      for (int t = 1; t < KB; ++t) {
+        if (t < k) {
+          bool hit = false;
+#pragma unroll
+          for (int q = 0; q < t; ++q) hit |= (pos[q] == pos[t]);
+          if (hit) pos[t] = (uint32_t)(d - k + t);
+        }
+      }
+    }
+    int32_t u[KB];
+    unsigned long long slots = 0;  // 4 bits per position: its rank (slot in ascending row order)
+#pragma unroll
+    for (int t = 0; t < KB; ++t) {
+      uint32_t r = 0;
+#pragma unroll
+      for (int q = 0; q < KB; ++q) r += (q < cnt && pos[q] < pos[t]) ? 1u : 0u;
+      slots |= (unsigned long long)r << (4 * t);
+      u[t] = (t < cnt) ? __ldg(indices + rs + pos[t]) : 0;
+    }
+    DSTAMP(hdr, 3, u[0] + u[KB - 1], layer);
+    B.cnt[i] = cnt;
+    mark_dst(B.first, v, i, F, layer, epoch, err);
+    const uint32_t q0 = (uint32_t)i * (uint32_t)k;
+#pragma unroll
+    for (int t = 0; t < KB; ++t) {
+      if (t < cnt) {
+        const uint32_t q = q0 + (uint32_t)((slots >> (4 * t)) & 15u);
+        B.rows[q] = u[t];
+        mark(B.first, u[t], epoch, (uint32_t)F + q);
+      }
+    }
+    DSTAMP(hdr, 5, 0, layer);
+    dbg_first = false;
+  }
+}
+
+// ------------------------------------------- scan, two-phase (persistent)
+// Inside the persistent kernel every block is resident, so the scan over
+// edge slots is a static partition: pass 1 computes each item's flags, the
+// per-(stripe, warp) counts and the block aggregate (published to `agg`);
+// after a grid barrier pass 2 adds the aggregates of the preceding blocks and
+// writes the outputs.  Items are striped (item j of thread t is slot
+// tile + j*PNT + t) so every load is a coalesced warp access; the in-block
+// prefix comes from warp ballots plus a table kept in shared memory across
+// the barrier, the flags in registers.
+constexpr int SCAN2_IPT = 8;
+constexpr int SCAN2_TILE = PNT * SCAN2_IPT;
 
 __device__ __forceinline__ unsigned long long pack2(uint32_t valid, uint32_t first) {
   return ((unsigned long long)first << 31) | valid;
 }
 
-__device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long *p) {
-  return *(volatile const unsigned long long *)p;
-}
+struct Scan2Smem {
+  unsigned long long tab[SCAN2_IPT * (PNT / 32)];  // exclusive prefix of (stripe j, warp w)
+  unsigned long long red[2 * (PNT / 32) + 2];
+};
 
-__global__ void __launch_bounds__(SCAN_THREADS) k_scan_assign(ScanArgs a) {
-  __shared__ unsigned long long s_warp[SCAN_THREADS / 32];
-  __shared__ unsigned long long s_prefix;
-  __shared__ uint32_t s_tile;
-  const int F = *(volatile const int32_t *)&a.hdr->F[a.layer];
-  const int k = a.k;
-  const int64_t total = (int64_t)F * k;
-  const int64_t ntiles = total > 0 ? (total + SCAN_TILE - 1) / SCAN_TILE : 1;
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  unsigned long long *ticket = a.status;
-  unsigned long long *st = a.status + 1;
+struct Scan2Regs {
+  uint32_t vbits, fbits;
+};
 
-  while (true) {
-    if (tid == 0) s_tile = (uint32_t)(atomicAdd(ticket, 1ull) + 1ull);  // starts at ~0
-    __syncthreads();
-    const int64_t tile = s_tile;
-    __syncthreads();
-    if (tile >= ntiles) break;
-    const int64_t q0 = tile * SCAN_TILE + (int64_t)tid * SCAN_ITEMS;
-
-    // pass 1: per-item flags
-    uint32_t vbits = 0, fbits = 0;
-    uint32_t keys[SCAN_ITEMS];
+__device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, uint32_t epoch, int64_t tile0,
+                                            int64_t tile_end, Scan2Regs &R, unsigned long long *agg_slot,
+                                            Scan2Smem &sm) {
+  const uint32_t total = (uint32_t)tile_end;  // < 2^31 by the host's plan check
+  const FastDiv fd = make_fastdiv((uint32_t)k);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const uint32_t q0 = (uint32_t)tile0 + threadIdx.x;
+  // all loads first: counts + sampled ids, then the map words of the valid slots
+  int32_t c[SCAN2_IPT], u[SCAN2_IPT];
 #pragma unroll
-    for (int j = 0; j < SCAN_ITEMS; ++j) {
-      const int64_t q = q0 + j;
-      keys[j] = 0;
-      if (q < total) {
-        const int i = (int)(q / k);
-        const int t = (int)(q - (int64_t)i * k);
-        if (t < __ldg(a.cnt + i)) {
-          vbits |= 1u << j;
-          const unsigned long long w = ld_volatile_u64(a.tbl + __ldg(a.hpos + q));
-          keys[j] = (uint32_t)(w >> 32);
-          if ((uint32_t)w == (uint32_t)(F + q)) fbits |= 1u << j;
-        }
-      }
+  for (int j = 0; j < SCAN2_IPT; ++j) {
+    const uint32_t q = q0 + j * PNT;
+    c[j] = -1;
+    u[j] = 0;
+    if (q < total) {
+      const uint32_t i = fdiv(q, fd);
+      c[j] = ldcg_i32(B.cnt + i) - (int32_t)(q - i * (uint32_t)k);  // > 0 iff slot q holds an edge
+      u[j] = ldcg_i32(B.rows + q);  // garbage unless valid; dereferenced only then
     }
-    const unsigned long long mine = pack2(__popc(vbits), __popc(fbits));
-
-    // block exclusive scan of `mine`
-    unsigned long long incl = mine;
+  }
+  unsigned long long w[SCAN2_IPT];
+#pragma unroll
+  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? ldcg_u64(B.first + u[j]) : 0ull;
+  R.vbits = R.fbits = 0;
+#pragma unroll
+  for (int j = 0; j < SCAN2_IPT; ++j) {
+    const bool valid = c[j] > 0;
+    const bool first = valid && w[j] == mark_word(epoch, (uint32_t)F + q0 + j * PNT);
+    R.vbits |= (valid ? 1u : 0u) << j;
+    R.fbits |= (first ? 1u : 0u) << j;
+    const uint32_t bv = __ballot_sync(FULL_MASK, valid), bf = __ballot_sync(FULL_MASK, first);
+    if (lane == 0) sm.tab[j * (PNT / 32) + wid] = pack2(__popc(bv), __popc(bf));
+  }
+  __syncthreads();
+  if (wid == 0) {  // exclusive scan of the (stripe, warp) counts, stripe-major
+    constexpr int PER = SCAN2_IPT * (PNT / 32) / 32;
+    unsigned long long v[PER], run = 0;
+#pragma unroll
+    for (int e = 0; e < PER; ++e) {
+      v[e] = sm.tab[lane * PER + e];
+      run += v[e];
+    }
+    unsigned long long incl = run;
 #pragma unroll
     for (int off = 1; off < 32; off <<= 1) {
       const unsigned long long y = __shfl_up_sync(FULL_MASK, incl, off);
       if (lane >= off) incl += y;
     }
-    if (lane == 31) s_warp[wid] = incl;
-    __syncthreads();
-    if (wid == 0) {
-      unsigned long long w = lane < SCAN_THREADS / 32 ? s_warp[lane] : 0ull;
+    unsigned long long p = incl - run;
 #pragma unroll
-      for (int off = 1; off < SCAN_THREADS / 32; off <<= 1) {
-        const unsigned long long y = __shfl_up_sync(FULL_MASK, w, off);
-        if (lane >= off) w += y;
-      }
-      if (lane < SCAN_THREADS / 32) s_warp[lane] = w;  // inclusive warp totals
+    for (int e = 0; e < PER; ++e) {
+      sm.tab[lane * PER + e] = p;
+      p += v[e];
     }
-    __syncthreads();
-    const unsigned long long warp_excl = wid ? s_warp[wid - 1] : 0ull;
-    const unsigned long long thread_excl = warp_excl + incl - mine;
-    const unsigned long long agg = s_warp[SCAN_THREADS / 32 - 1];
+    if (lane == 31) __stcg(agg_slot, incl);
+  }
+  __syncthreads();
+}
 
-    // decoupled look-back (warp 0)
-    if (wid == 0) {
-      unsigned long long prefix = 0;
-      if (tile == 0) {
-        if (lane == 0) *(volatile unsigned long long *)&st[0] = ST_INC | agg;
-      } else {
-        if (lane == 0) *(volatile unsigned long long *)&st[tile] = ST_AGG | agg;
-        int64_t idx = tile - 1;
-        while (true) {
-          const int64_t p = idx - lane;
-          unsigned long long s = ST_INC;  // virtual inclusive zero before tile 0
-          if (p >= 0) {
-            do {
-              s = ld_volatile_u64(&st[p]);
-            } while ((s >> 62) == 3ull);
-          }
-          const unsigned incm = __ballot_sync(FULL_MASK, (s >> 62) == 2ull);
-          const int stop = incm ? (__ffs(incm) - 1) : 31;
-          unsigned long long v = (lane <= stop) ? (s & ST_VAL_MASK) : 0ull;
+// prefix of block `blk` and the round total from the published aggregates
+__device__ __forceinline__ void scan2_prefix(const unsigned long long *agg, int nblk, int blk, Scan2Smem &sm,
+                                             unsigned long long *prefix, unsigned long long *round_total) {
+  unsigned long long p = 0, t = 0;
+  for (int b = threadIdx.x; b < nblk; b += PNT) {
+    const unsigned long long x = __ldcg(agg + b);
+    t += x;
+    if (b < blk) p += x;
+  }
 #pragma unroll
-          for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(FULL_MASK, v, off);
-          prefix += v;
-          if (incm) break;
-          idx -= 32;
-        }
-        if (lane == 0) *(volatile unsigned long long *)&st[tile] = ST_INC | (prefix + agg);
-      }
-      if (lane == 0) s_prefix = prefix;
+  for (int off = 16; off > 0; off >>= 1) {
+    p += __shfl_xor_sync(FULL_MASK, p, off);
+    t += __shfl_xor_sync(FULL_MASK, t, off);
+  }
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (lane == 0) {
+    sm.red[wid] = p;
+    sm.red[PNT / 32 + wid] = t;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long pp = 0, tt = 0;
+    for (int w = 0; w < PNT / 32; ++w) {
+      pp += sm.red[w];
+      tt += sm.red[PNT / 32 + w];
     }
-    __syncthreads();
-    const unsigned long long base = s_prefix + thread_excl;
-    uint32_t pv = (uint32_t)(base & 0x7fffffffull);
-    uint32_t pf = (uint32_t)((base >> 31) & 0x7fffffffull);
+    sm.red[2 * (PNT / 32)] = pp;
+    sm.red[2 * (PNT / 32) + 1] = tt;
+  }
+  __syncthreads();
+  *prefix = sm.red[2 * (PNT / 32)];
+  *round_total = sm.red[2 * (PNT / 32) + 1];
+  __syncthreads();
+}
 
-    // pass 2: outputs
+// Block indptr at t == 0 slots; for first occurrences: new id nid = F + rank,
+// map word := (epoch, nid), src_out[nid] = u.  The dst copy is written by the
+// sample phase.
+__device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, uint32_t epoch, int64_t tile0,
+                                            int64_t tile_end, const Scan2Regs &R, unsigned long long base,
+                                            const Scan2Smem &sm, int32_t *indptr_out, int32_t *src_out) {
+  const uint32_t total = (uint32_t)tile_end;
+  const FastDiv fd = make_fastdiv((uint32_t)k);
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const uint32_t lt = (1u << lane) - 1u;
+  const uint32_t q0 = (uint32_t)tile0 + threadIdx.x;
+  int32_t u[SCAN2_IPT];
 #pragma unroll
-    for (int j = 0; j < SCAN_ITEMS; ++j) {
-      const int64_t q = q0 + j;
-      if (q < total) {
-        const int i = (int)(q / k);
-        const int t = (int)(q - (int64_t)i * k);
-        if (t == 0) {
-          a.indptr_out[i] = (int32_t)pv;
-          a.src_ids_out[i] = __ldg(a.frontier + i);
-        }
-        if (fbits & (1u << j)) {
-          const uint32_t nid = (uint32_t)F + pf;
-          a.tbl[__ldg(a.hpos + q)] = ((unsigned long long)keys[j] << 32) | nid;
-          a.src_ids_out[nid] = (int32_t)keys[j];
-        }
-        pv += (vbits >> j) & 1u;
-        pf += (fbits >> j) & 1u;
+  for (int j = 0; j < SCAN2_IPT; ++j) u[j] = ((R.fbits >> j) & 1u) ? ldcg_i32(B.rows + q0 + j * PNT) : 0;
+#pragma unroll
+  for (int j = 0; j < SCAN2_IPT; ++j) {
+    const uint32_t bv = __ballot_sync(FULL_MASK, (R.vbits >> j) & 1u);
+    const uint32_t bf = __ballot_sync(FULL_MASK, (R.fbits >> j) & 1u);
+    const uint32_t q = q0 + j * PNT;
+    if (q < total) {
+      const unsigned long long b = base + sm.tab[j * (PNT / 32) + wid];
+      const uint32_t i = fdiv(q, fd);
+      if (q == i * (uint32_t)k) indptr_out[i] = (int32_t)((uint32_t)(b & 0x7fffffffull) + __popc(bv & lt));
+      if ((R.fbits >> j) & 1u) {
+        const uint32_t nid = (uint32_t)F + (uint32_t)((b >> 31) & 0x7fffffffull) + __popc(bf & lt);
+        B.first[u[j]] = mark_word(epoch, nid);  // only this slot writes u's word in this phase
+        src_out[nid] = u[j];
       }
-    }
-    if (tile == ntiles - 1 && tid == 0) {
-      const unsigned long long tot = s_prefix + agg;
-      const int32_t E = (int32_t)(tot & 0x7fffffffull);
-      const int32_t nnew = (int32_t)((tot >> 31) & 0x7fffffffull);
-      a.indptr_out[F] = E;
-      a.hdr->E[a.layer] = E;
-      a.hdr->S[a.layer] = F + nnew;
-      a.hdr->F[a.layer + 1] = F + nnew;
     }
   }
 }
 
 // ---------------------------------------------------------- write indices
-struct IndicesArgs {
-  int32_t layer, k;
-  const int32_t *cnt;
-  const int32_t *hpos;
-  const unsigned long long *tbl;
-  const int32_t *indptr;  // block indptr
-  int32_t *indices_out;
-  WsHeader *hdr;
-};
-
-__global__ void __launch_bounds__(256) k_write_indices(IndicesArgs a) {
-  const int F = *(volatile const int32_t *)&a.hdr->F[a.layer];
-  const int k = a.k;
-  const int64_t total = (int64_t)F * k;
-  for (int64_t q = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; q < total;
-       q += (int64_t)gridDim.x * blockDim.x) {
-    const int i = (int)(q / k);
-    const int t = (int)(q - (int64_t)i * k);
-    if (t < __ldg(a.cnt + i)) {
-      const unsigned long long w = a.tbl[__ldg(a.hpos + q)];
-      a.indices_out[__ldg(a.indptr + i) + t] = (int32_t)(uint32_t)w;
+// indices[indptr[i] + t] = local id of the src of slot q = i*k + t.
+__device__ __forceinline__ void phase_indices(int F, int k, const LayerBufs &B, const int32_t *indptr,
+                                              int32_t *indices_out, const Span &sp) {
+  constexpr int U = 4;  // items per thread in flight
+  const FastDiv fd = make_fastdiv((uint32_t)k);
+  const uint32_t end = (uint32_t)sp.end, step = (uint32_t)sp.step;
+  (void)F;
+  for (uint32_t q0 = (uint32_t)sp.first; q0 < end; q0 += step * U) {
+    int32_t c[U], u[U], ip[U];
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const uint32_t q = q0 + j * step;
+      c[j] = -1;
+      u[j] = 0;
+      ip[j] = 0;
+      if (q < end) {
+        const uint32_t i = fdiv(q, fd);
+        const int32_t t = (int32_t)(q - i * (uint32_t)k);
+        c[j] = ldcg_i32(B.cnt + i) - t;  // > 0 iff slot q holds an edge
+        u[j] = ldcg_i32(B.rows + q);
+        ip[j] = ldcg_i32(indptr + i) + t;
+      }
     }
+    unsigned long long w[U];
+#pragma unroll
+    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? ldcg_u64(B.first + u[j]) : 0ull;
+#pragma unroll
+    for (int j = 0; j < U; ++j)
+      if (c[j] > 0) indices_out[ip[j]] = (int32_t)mark_x(w[j]);
   }
 }
 
 // ----------------------------------------------------------------- gather
 struct GatherArgs {
   const int32_t *ids;
-  int64_t n;
-  int32_t dim4;             // dim / 4
+  int64_t n;                // rows (ignored when n_dev is set)
+  const int32_t *n_dev;     // device row count (fused call), or nullptr
+  int32_t dim4;             // dim / 4  (output row length in float4)
+  int32_t stride4;          // shard row stride in float4 (rows padded to 64 B)
   float4 *out;
   const float4 *base[8];    // feature shard of each rank (local or peer-mapped)
   Bounds bd;
   int *err;
 };
 
-// One float4 per thread-iteration over the flat [n][dim4] output; UNROLL
-// independent 16-byte loads in flight per thread before any store.
+__device__ __forceinline__ float4 ld_stream_f4(const float4 *p) {
+  float4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+  return v;
+}
+
+// Flat [n][dim4] float4 index space; UNROLL independent 16-byte loads in
+// flight per thread before any store (Little's law over HBM / NVLink).
+// 32-bit index math (the host guarantees n * dim4 < 2^31).
 template <int UNROLL>
-__global__ void __launch_bounds__(256) k_gather(GatherArgs a) {
-  const int64_t total = a.n * a.dim4;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t start = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-  for (int64_t e0 = start; e0 < total; e0 += stride * UNROLL) {
-    float4 v[UNROLL];
-    int64_t e[UNROLL];
-    bool ok[UNROLL];
+__device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int64_t tid64, int64_t nthreads64) {
+  const uint32_t total = (uint32_t)(n * a.dim4);
+  const uint32_t tid = (uint32_t)tid64, nthreads = (uint32_t)nthreads64;
+  const uint32_t dim4 = (uint32_t)a.dim4;
+  const int32_t N = (int32_t)a.bd.b[a.bd.world];
+  for (uint32_t e0 = tid; e0 < total; e0 += nthreads * UNROLL) {
+    int32_t g[UNROLL];
+    uint32_t c[UNROLL];
 #pragma unroll
     for (int u = 0; u < UNROLL; ++u) {
-      e[u] = e0 + (int64_t)u * stride;
-      ok[u] = false;
-      if (e[u] < total) {
-        const int64_t r = e[u] / a.dim4;
-        const int64_t c = e[u] - r * a.dim4;
-        const int32_t g = __ldg(a.ids + r);
-        if (g >= 0 && g < a.bd.b[a.bd.world]) {
-          const int o = owner_of(a.bd, g);
-          v[u] = __ldg(a.base[o] + (g - a.bd.b[o]) * a.dim4 + c);
-          ok[u] = true;
-        } else {
-          latch(a.err, E_RANGE);
-        }
+      const uint32_t e = e0 + (uint32_t)u * nthreads;
+      g[u] = -1;
+      c[u] = 0;
+      if (e < total) {
+        const uint32_t r = e / dim4;
+        c[u] = e - r * dim4;
+        g[u] = ldcg_i32(a.ids + r);
+      }
+    }
+    float4 v[UNROLL];
+#pragma unroll
+    for (int u = 0; u < UNROLL; ++u) {
+      if (g[u] >= 0 && g[u] < N) {
+        const int o = owner_of(a.bd, g[u]);
+        v[u] = ld_stream_f4(a.base[o] + (size_t)(uint32_t)(g[u] - (int32_t)a.bd.b[o]) * (uint32_t)a.stride4 + c[u]);
       }
     }
 #pragma unroll
-    for (int u = 0; u < UNROLL; ++u)
-      if (ok[u]) a.out[e[u]] = v[u];
+    for (int u = 0; u < UNROLL; ++u) {
+      const uint32_t e = e0 + (uint32_t)u * nthreads;
+      if (e < total) {
+        if (g[u] >= 0 && g[u] < N)
+          __stcs(a.out + e, v[u]);
+        else
+          latch(a.err, E_RANGE);
+      }
+    }
+  }
+}
+
+constexpr int GATHER_UNROLL = 4;
+
+__global__ void __launch_bounds__(NT) k_gather(GatherArgs a) {
+  const int64_t n = a.n_dev ? (int64_t)ld_volatile_i32(a.n_dev) : a.n;
+  phase_gather<GATHER_UNROLL>(a, n, blockIdx.x * (int64_t)NT + threadIdx.x, (int64_t)gridDim.x * NT);
+}
+
+// ============================================ world == 1: persistent kernel
+struct PersistArgs {
+  const int32_t *seeds;
+  int32_t B;
+  int32_t L;
+  int32_t k[8];
+  uint2 key;
+  const int64_t *indptr;
+  const int32_t *indices;
+  int64_t lo, n_local;
+  Outputs out;
+  LayerBufs buf[2];
+  unsigned long long *agg;  // [2][MAX_PERSIST_BLOCKS] scan aggregates
+  WsPersist *persist;
+  WsHeader *hdr;
+  int *err;
+  int32_t gather;           // fuse the gather of the last block's src_ids
+  GatherArgs g;
+};
+
+__device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32_t *frontier, int F, int l,
+                                               uint32_t epoch) {
+  const int k = a.k[l];
+  const LayerBufs &B = a.buf[l & 1];
+  if (k <= 8) {
+    phase_sample_tpn<8>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch, a.out.src_ids[l],
+                        a.err, a.hdr);
+  } else if (k <= 16) {
+    phase_sample_tpn<16>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch, a.out.src_ids[l],
+                         a.err, a.hdr);
+  } else {
+    phase_sample_lanes<32>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
+                           a.out.src_ids[l], a.err, a.hdr);
+  }
+}
+
+// The whole CSP call for world == 1 (and the fused gather) in one launch:
+// per layer  sample(l) + indices(l-1) | scan pass 1 | scan pass 2, separated
+// by grid barriers; no host round trip, no table clearing (epochs).
+__global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
+  __shared__ Scan2Smem sm;
+  const int64_t tid = blockIdx.x * (int64_t)PNT + threadIdx.x;
+  const int64_t nthreads = (int64_t)gridDim.x * PNT;
+  const int blk = blockIdx.x, nblk = gridDim.x;
+  uint32_t bar = 0;  // grid barrier target
+  const uint32_t e0 = *(volatile const uint32_t *)&a.persist->epoch;
+
+  // the host cleared the header just before the launch
+  if (tid == 0) {
+    a.hdr->t[0] = globaltimer_ns();
+    a.hdr->F[0] = a.B;
+  }
+  int F = a.B;  // frontier size of layer l, tracked in every block
+  int Fprev = 0;
+  for (int l = 0; l < a.L; ++l) {
+    const uint32_t epoch = e0 + 1 + l;
+    const int32_t *frontier = l == 0 ? a.seeds : a.out.src_ids[l - 1];
+    const int k = a.k[l];
+    // S(l): sample + marks; indices of layer l-1 in the same phase
+    persist_sample(a, frontier, F, l, epoch);
+    if (l > 0)
+      phase_indices(Fprev, a.k[l - 1], a.buf[(l - 1) & 1], a.out.indptr[l - 1], a.out.indices[l - 1],
+                    block_span((int64_t)Fprev * a.k[l - 1]));
+    grid_barrier(a.hdr, bar);
+    // scan over the F*k edge slots: each block one contiguous chunk of <= SCAN2_TILE slots per round
+    const int64_t total = (int64_t)F * k;
+    const int64_t rounds = total > 0 ? (total + (int64_t)nblk * SCAN2_TILE - 1) / ((int64_t)nblk * SCAN2_TILE) : 1;
+    const int64_t per_round = (total + rounds - 1) / rounds;
+    const int64_t chunk = (per_round + nblk - 1) / nblk;
+    unsigned long long carry = 0;
+    for (int64_t r = 0; r < rounds; ++r) {
+      Scan2Regs R;
+      const int64_t r0 = r * per_round, r1 = min(total, r0 + per_round);
+      const int64_t tile0 = min(r1, r0 + (int64_t)blk * chunk), tile_end = min(r1, tile0 + chunk);
+      unsigned long long *agg = a.agg + (r & 1) * MAX_PERSIST_BLOCKS;
+      scan2_pass1(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, agg + blk, sm);
+      grid_barrier(a.hdr, bar);
+      unsigned long long prefix, round_total;
+      scan2_prefix(agg, nblk, blk, sm, &prefix, &round_total);
+      scan2_pass2(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
+                  a.out.src_ids[l]);
+      carry += round_total;
+      if (r + 1 < rounds) grid_barrier(a.hdr, bar);
+    }
+    const int32_t E = (int32_t)(carry & 0x7fffffffull);
+    const int32_t nnew = (int32_t)((carry >> 31) & 0x7fffffffull);
+    if (tid == 0) {
+      a.out.indptr[l][F] = E;
+      a.hdr->E[l] = E;
+      a.hdr->S[l] = F + nnew;
+      a.hdr->F[l + 1] = F + nnew;
+      a.hdr->sizes[3 * l + 0] = F;
+      a.hdr->sizes[3 * l + 1] = F + nnew;
+      a.hdr->sizes[3 * l + 2] = E;
+    }
+    Fprev = F;
+    F = F + nnew;
+    grid_barrier(a.hdr, bar);
+  }
+  // last layer's indices + the gather of its src_ids (F = num_src of the last block)
+  const int l = a.L - 1;
+  phase_indices(Fprev, a.k[l], a.buf[l & 1], a.out.indptr[l], a.out.indices[l], block_span((int64_t)Fprev * a.k[l]));
+  if (a.gather) phase_gather<GATHER_UNROLL>(a.g, F, tid, nthreads);
+  // the last block to finish advances the workspace epoch and stamps the end
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(&a.hdr->done, 1u) == gridDim.x - 1) {
+      a.persist->epoch = e0 + (uint32_t)a.L;
+      a.hdr->t[23] = globaltimer_ns();
+      a.hdr->done = 0u;
+    }
   }
 }
 
@@ -406,6 +759,10 @@ __device__ __forceinline__ bool last_block_done(uint32_t *done) {
   return false;
 }
 
+__device__ __forceinline__ int frontier_size(const WsHeader *hdr, int layer, int F0) {
+  return layer == 0 ? F0 : ld_volatile_i32(&hdr->F[layer]);
+}
+
 struct BucketArgs {
   const int32_t *frontier;
   int32_t F0, layer, k;
@@ -417,6 +774,7 @@ struct BucketArgs {
   XchPeers peers;
   int32_t *perm;            // [F] slot of frontier i in its owner's inbox
   WsHeader *hdr;
+  int *err;
 };
 
 // Shuffle: group the frontier by owner (range check) and
@@ -424,18 +782,19 @@ struct BucketArgs {
 // inside a bucket is irrelevant (results come back to the same slot).  The
 // last block publishes the per-owner counts + header, then the flag
 // (count notification before use).
-__global__ void __launch_bounds__(256) k_bucket_scatter(BucketArgs a) {
+__global__ void __launch_bounds__(NT) k_bucket_scatter(BucketArgs a) {
   __shared__ uint32_t s_cnt[8], s_base[8];
   const int F = frontier_size(a.hdr, a.layer, a.F0);
-  if (a.layer == 0 && blockIdx.x == 0 && threadIdx.x == 0 && F <= a.L.cap) a.hdr->F[0] = a.F0;
-  if (F > a.L.cap && blockIdx.x == 0 && threadIdx.x == 0) {
-    latch(&a.hdr->err, E_CAP);
-    a.hdr->F[a.layer] = 0;  // later kernels of this layer see an empty frontier
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if (F > a.L.cap) {
+      latch(a.err, E_CAP);
+      a.hdr->F[a.layer] = 0;  // later kernels of this layer see an empty frontier
+    } else if (a.layer == 0) {
+      a.hdr->F[0] = a.F0;
+    }
   }
   const int limit = F > a.L.cap ? 0 : F;
-  const int chunk = blockDim.x;
-  for (int b0 = blockIdx.x * chunk; b0 < ((limit + chunk - 1) / chunk) * chunk;
-       b0 += gridDim.x * chunk) {
+  for (int b0 = blockIdx.x * NT; b0 < ((limit + NT - 1) / NT) * NT; b0 += gridDim.x * NT) {
     if (threadIdx.x < 8) s_cnt[threadIdx.x] = 0;
     __syncthreads();
     const int i = b0 + threadIdx.x;
@@ -445,7 +804,7 @@ __global__ void __launch_bounds__(256) k_bucket_scatter(BucketArgs a) {
     if (i < limit) {
       v = __ldg(a.frontier + i);
       if (v < 0 || v >= a.bd.b[a.bd.world]) {
-        latch(&a.hdr->err, E_RANGE);
+        latch(a.err, E_RANGE);
       } else {
         o = owner_of(a.bd, v);
         local = atomicAdd(&s_cnt[o], 1u);
@@ -486,23 +845,24 @@ struct RemoteSampleArgs {
   XchLayout L;
   XchPeers peers;
   WsHeader *hdr;
+  int *err;
 };
 
 // Sample stage at the owner: one kernel over every task received in
 // this layer, results written straight into each requester's
 // return slots over NVLink, then the return flags.
 template <int G>
-__global__ void __launch_bounds__(256) k_sample_remote(RemoteSampleArgs a) {
+__global__ void __launch_bounds__(NT) k_sample_remote(RemoteSampleArgs a) {
   __shared__ uint32_t s_off[9];
   char *self = a.peers.base[a.rank];
   const int world = a.bd.world;
-  if (wait_flags(xch_inbox_flag(self, a.L, a.parity, 0), world, a.seq, &a.hdr->err)) {
+  if (wait_flags(xch_inbox_flag(self, a.L, a.parity, 0), world, a.seq, a.err)) {
     if (threadIdx.x == 0) {
       uint32_t acc = 0;
       for (int s = 0; s < world; ++s) {
         const uint4 h = __ldcv(xch_inbox_hdr(self, a.L, a.parity, s));
         if (h.y != ((uint32_t)a.k | ((uint32_t)a.layer << 8)) || h.z != a.key.x || h.w != a.key.y)
-          latch(&a.hdr->err, E_STATE);
+          latch(a.err, E_STATE);
         s_off[s] = acc;
         acc += (h.x <= (uint32_t)a.L.cap) ? h.x : 0u;
       }
@@ -512,8 +872,8 @@ __global__ void __launch_bounds__(256) k_sample_remote(RemoteSampleArgs a) {
     const int T = (int)s_off[world];
     constexpr int NPW = 32 / G;
     const int lane = threadIdx.x & 31;
-    const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int nwarps = (gridDim.x * blockDim.x) >> 5;
+    const int warp = (blockIdx.x * NT + threadIdx.x) >> 5;
+    const int nwarps = (gridDim.x * NT) >> 5;
     const int k = a.k;
     for (int base = warp * NPW; base < T; base += nwarps * NPW) {
       const int q = base + lane / G;
@@ -523,10 +883,10 @@ __global__ void __launch_bounds__(256) k_sample_remote(RemoteSampleArgs a) {
         while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
       }
       const int j = q - (int)s_off[s];
-      int32_t v = active ? *(volatile int32_t *)(xch_inbox(self, a.L, a.parity, s) + j) : 0;
+      const int32_t v = active ? __ldcv(xch_inbox(self, a.L, a.parity, s) + j) : 0;
       const int64_t lv = (int64_t)v - a.lo;
       const bool ok = active && lv >= 0 && lv < a.n_local;
-      if (active && !ok && (lane & (G - 1)) == 0) latch(&a.hdr->err, E_STATE);
+      if (active && !ok && (lane & (G - 1)) == 0) latch(a.err, E_STATE);
       int64_t rs = 0, d = 0;
       if (ok) {
         rs = __ldg(a.indptr + lv);
@@ -556,53 +916,208 @@ struct UnpermuteArgs {
   XchLayout L;
   char *self;
   const int32_t *perm;
-  unsigned long long *tbl;
-  uint32_t mask;
-  int32_t *cnt;
-  int32_t *hpos;
+  LayerBufs buf;
+  const WsPersist *persist;
+  int32_t *src_out;         // dst copy
   WsHeader *hdr;
+  int *err;
 };
 
 // Reshuffle consumer ("transferred back to the GPU requesting"):
-// frontier node i reads its row from the owner's return slot perm[i], and
-// the dst + sampled srcs go into the relabel table (as k_sample_local does).
+// frontier node i reads its row from the owner's return slot perm[i]; the
+// edge slots, counts, dst copy and marks are written as the local sample does.
 template <int G>
-__global__ void __launch_bounds__(256) k_unpermute_insert(UnpermuteArgs a) {
+__global__ void __launch_bounds__(NT) k_unpermute_mark(UnpermuteArgs a) {
   const int world = a.bd.world;
-  if (!wait_flags(xch_ret_flag(a.self, a.L, a.parity, 0), world, a.seq, &a.hdr->err)) return;
-  const int F = *(volatile const int32_t *)&a.hdr->F[a.layer];
+  if (!wait_flags(xch_ret_flag(a.self, a.L, a.parity, 0), world, a.seq, a.err)) return;
+  const uint32_t epoch = a.persist->epoch + 1u + (uint32_t)a.layer;
+  const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
   const int lim = F > a.L.cap ? 0 : F;
   constexpr int NPW = 32 / G;
   const int lane = threadIdx.x & 31;
   const int t = lane & (G - 1);
-  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int nwarps = (gridDim.x * blockDim.x) >> 5;
+  const int warp = (blockIdx.x * NT + threadIdx.x) >> 5;
+  const int nwarps = (gridDim.x * NT) >> 5;
   const int k = a.k;
   for (int base = warp * NPW; base < lim; base += nwarps * NPW) {
     const int i = base + lane / G;
     if (i >= lim) continue;
     const int32_t v = __ldg(a.frontier + i);
+    if (t == 0) a.src_out[i] = v;
     if (v < 0 || v >= a.bd.b[world]) {  // latched by the bucket kernel
-      if (t == 0) a.cnt[i] = 0;
+      if (t == 0) a.buf.cnt[i] = 0;
       continue;
     }
     const int o = owner_of(a.bd, v);
     const int j = __ldg(a.perm + i);
-    const int c = *(volatile int32_t *)(xch_ret_cnt(a.self, a.L, a.parity, o) + j);
+    const int c = __ldcv(xch_ret_cnt(a.self, a.L, a.parity, o) + j);
     if (t == 0) {
-      a.cnt[i] = c;
-      uint32_t old;
-      table_insert_min(a.tbl, a.mask, (uint32_t)v, (uint32_t)i, &old);
-      if (a.layer == 0 && old < (uint32_t)F && old != (uint32_t)i) latch(&a.hdr->err, E_DUP);
+      a.buf.cnt[i] = c;
+      mark_dst(a.buf.first, v, i, F, a.layer, epoch, a.err);
     }
     if (t < c) {
-      const int32_t u =
-          *(volatile int32_t *)(xch_ret_rows(a.self, a.L, a.parity, o) + (int64_t)j * a.L.kmax + t);
-      const int64_t q = (int64_t)i * k + t;
-      uint32_t old;
-      a.hpos[q] = (int32_t)table_insert_min(a.tbl, a.mask, (uint32_t)u, (uint32_t)(F + q), &old);
+      const int32_t u = __ldcv(xch_ret_rows(a.self, a.L, a.parity, o) + (int64_t)j * a.L.kmax + t);
+      const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)t;
+      a.buf.rows[q] = u;
+      mark(a.buf.first, u, epoch, (uint32_t)F + q);
     }
   }
 }
+
+// ------------------------------------------- scan as look-back (world > 1)
+// Single-pass decoupled look-back over edge slots (tile status word:
+// [63:62] flag 3 = not ready, 1 = aggregate, 2 = inclusive; [61:31] first
+// count; [30:0] valid count; status[0] = tile ticket; all ones at start).
+constexpr int SCAN_ITEMS = 8;
+constexpr int SCAN_TILE = NT * SCAN_ITEMS;
+constexpr unsigned long long ST_VAL_MASK = (1ull << 62) - 1;
+constexpr unsigned long long ST_AGG = 1ull << 62;
+constexpr unsigned long long ST_INC = 2ull << 62;
+
+struct ScanArgs {
+  int32_t layer, k;
+  LayerBufs buf;
+  const WsPersist *persist;
+  int32_t *indptr_out;
+  int32_t *src_ids_out;
+  int32_t *indices_out;
+  WsHeader *hdr;
+};
+
+__global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
+  __shared__ unsigned long long s_warp[NT / 32];
+  __shared__ unsigned long long s_prefix;
+  __shared__ uint32_t s_tile;
+  const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
+  const uint32_t epoch = a.persist->epoch + 1u + (uint32_t)a.layer;
+  const int k = a.k;
+  const FastDiv fd = make_fastdiv((uint32_t)k);
+  const LayerBufs &B = a.buf;
+  const uint32_t total = (uint32_t)((int64_t)F * k);
+  const int64_t ntiles = total > 0 ? ((int64_t)total + SCAN_TILE - 1) / SCAN_TILE : 1;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  unsigned long long *ticket = B.status;
+  unsigned long long *st = B.status + 1;
+
+  while (true) {
+    if (tid == 0) s_tile = (uint32_t)(atomicAdd(ticket, 1ull) + 1ull);  // ticket starts at ~0
+    __syncthreads();
+    const int64_t tile = s_tile;
+    __syncthreads();
+    if (tile >= ntiles) break;
+    const uint32_t q0 = (uint32_t)(tile * SCAN_TILE) + (uint32_t)tid * SCAN_ITEMS;
+
+    uint32_t vbits = 0, fbits = 0;
+    int32_t c[SCAN_ITEMS], u[SCAN_ITEMS];
+#pragma unroll
+    for (int j = 0; j < SCAN_ITEMS; ++j) {
+      const uint32_t q = q0 + j;
+      c[j] = -1;
+      u[j] = 0;
+      if (q < total) {
+        const uint32_t i = fdiv(q, fd);
+        c[j] = __ldg(B.cnt + i) - (int32_t)(q - i * (uint32_t)k);
+        u[j] = __ldg(B.rows + q);
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < SCAN_ITEMS; ++j) {
+      if (c[j] > 0) {
+        vbits |= 1u << j;
+        if (__ldg(B.first + u[j]) == mark_word(epoch, (uint32_t)F + q0 + j)) fbits |= 1u << j;
+      }
+    }
+    const unsigned long long mine = pack2(__popc(vbits), __popc(fbits));
+
+    unsigned long long incl = mine;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+      const unsigned long long y = __shfl_up_sync(FULL_MASK, incl, off);
+      if (lane >= off) incl += y;
+    }
+    if (lane == 31) s_warp[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+      unsigned long long w = lane < NT / 32 ? s_warp[lane] : 0ull;
+#pragma unroll
+      for (int off = 1; off < NT / 32; off <<= 1) {
+        const unsigned long long y = __shfl_up_sync(FULL_MASK, w, off);
+        if (lane >= off) w += y;
+      }
+      if (lane < NT / 32) s_warp[lane] = w;
+    }
+    __syncthreads();
+    const unsigned long long thread_excl = (wid ? s_warp[wid - 1] : 0ull) + incl - mine;
+    const unsigned long long agg = s_warp[NT / 32 - 1];
+
+    if (wid == 0) {  // decoupled look-back
+      unsigned long long prefix = 0;
+      if (tile == 0) {
+        if (lane == 0) *(volatile unsigned long long *)&st[0] = ST_INC | agg;
+      } else {
+        if (lane == 0) *(volatile unsigned long long *)&st[tile] = ST_AGG | agg;
+        int64_t idx = tile - 1;
+        while (true) {
+          const int64_t p = idx - lane;
+          unsigned long long s = ST_INC;  // virtual inclusive zero before tile 0
+          if (p >= 0) {
+            do {
+              s = ld_volatile_u64(&st[p]);
+            } while ((s >> 62) == 3ull);
+          }
+          const unsigned incm = __ballot_sync(FULL_MASK, (s >> 62) == 2ull);
+          const int stop = incm ? (__ffs(incm) - 1) : 31;
+          unsigned long long v = (lane <= stop) ? (s & ST_VAL_MASK) : 0ull;
+#pragma unroll
+          for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(FULL_MASK, v, off);
+          prefix += v;
+          if (incm) break;
+          idx -= 32;
+        }
+        if (lane == 0) *(volatile unsigned long long *)&st[tile] = ST_INC | (prefix + agg);
+      }
+      if (lane == 0) s_prefix = prefix;
+    }
+    __syncthreads();
+    const unsigned long long base = s_prefix + thread_excl;
+    uint32_t pv = (uint32_t)(base & 0x7fffffffull);
+    uint32_t pf = (uint32_t)((base >> 31) & 0x7fffffffull);
+#pragma unroll
+    for (int j = 0; j < SCAN_ITEMS; ++j) {
+      const uint32_t q = q0 + j;
+      if (q < total) {
+        const uint32_t i = fdiv(q, fd);
+        if (q == i * (uint32_t)k) a.indptr_out[i] = (int32_t)pv;
+        if (fbits & (1u << j)) {
+          const uint32_t nid = (uint32_t)F + pf;
+          B.first[u[j]] = mark_word(epoch, nid);
+          a.src_ids_out[nid] = u[j];
+        }
+        pv += (vbits >> j) & 1u;
+        pf += (fbits >> j) & 1u;
+      }
+    }
+    if (tile == ntiles - 1 && tid == 0) {
+      const unsigned long long tot = s_prefix + agg;
+      const int32_t E = (int32_t)(tot & 0x7fffffffull);
+      const int32_t nnew = (int32_t)((tot >> 31) & 0x7fffffffull);
+      a.indptr_out[F] = E;
+      a.hdr->E[a.layer] = E;
+      a.hdr->S[a.layer] = F + nnew;
+      a.hdr->F[a.layer + 1] = F + nnew;
+      a.hdr->sizes[3 * a.layer + 0] = F;
+      a.hdr->sizes[3 * a.layer + 1] = F + nnew;
+      a.hdr->sizes[3 * a.layer + 2] = E;
+    }
+  }
+}
+
+__global__ void __launch_bounds__(NT) k_write_indices(ScanArgs a) {
+  const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
+  phase_indices(F, a.k, a.buf, a.indptr_out, a.indices_out, grid_span((int64_t)F * a.k));
+}
+
+// end of a stage-by-stage call: advance the workspace epoch
+__global__ void k_epoch_advance(WsPersist *persist, uint32_t L) { persist->epoch += L; }
 
 }  // namespace dsp

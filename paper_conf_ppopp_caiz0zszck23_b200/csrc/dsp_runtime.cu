@@ -1,6 +1,6 @@
 // dsp_runtime.cu -- host runtime behind the C ABI of include/dsp.h:
-// context, partition load, peer mapping (CUDA IPC / P2P), workspace
-// planning, and the CSP layer driver that issues the kernels of
+// context, partition load (padded feature rows), peer mapping (CUDA IPC /
+// P2P), workspace planning, and the CSP driver that issues the kernels of
 // dsp_kernels.cuh.  sm_100a only.
 #include <cuda_runtime.h>
 #include <unistd.h>
@@ -19,7 +19,20 @@ using namespace dsp;
 
 namespace {
 
+// Every adjacency entry must be a global id in [0, N): the relabel map is
+// indexed by it.
+__global__ void k_validate_indices(const int32_t *indices, int64_t nnz, int64_t N, int *bad) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < nnz; e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t u = indices[e];
+    if (u < 0 || u >= N) {
+      atomicAdd(bad, 1);
+      return;
+    }
+  }
+}
+
 constexpr uint32_t HANDLE_MAGIC = 0x44535048u;  // "DSPH"
+constexpr int FEAT_ALIGN_FLOATS = 16;           // shard rows padded to 64 B (HBM access granule)
 thread_local std::string g_create_error;
 
 struct PeerHandle {  // fits in DSP_HANDLE_BYTES
@@ -32,7 +45,7 @@ struct PeerHandle {  // fits in DSP_HANDLE_BYTES
   int32_t has_feat, has_xch;
   cudaIpcMemHandle_t feat_ipc, xch_ipc;
   int64_t bounds[DSP_MAX_WORLD + 1];
-  int32_t dim, max_seeds;
+  int32_t dim, max_seeds, feat_stride, pad;
 };
 static_assert(sizeof(PeerHandle) <= DSP_HANDLE_BYTES, "handle too large");
 
@@ -67,15 +80,16 @@ int group_of(int k) {
   return g;
 }
 
-// Per-layer bounds (dsp_sample_bounds) and the workspace plan.
+// Per-layer bounds (dsp_sample_bounds) and the workspace plan:
+//   persist | hdr | agg[2][MAX_PERSIST_BLOCKS] | cnt[2][max_F] | perm[max_F] | rows[2][max_slots]
+//   | status[2][status_len] | first[2][N]
 struct Plan {
   int L;
   int64_t F[DSP_MAX_LAYERS + 1];   // max frontier per layer
   int64_t E[DSP_MAX_LAYERS];       // max edges
   int64_t S[DSP_MAX_LAYERS];       // max src
-  int64_t cap[DSP_MAX_LAYERS];     // table capacity
-  int64_t max_F, max_slots, max_cap, max_tiles;
-  size_t off_cnt, off_perm, off_hpos, off_status, off_tbl, bytes;
+  int64_t max_F, max_slots, status_len;
+  size_t off_hdr, off_agg, off_cnt[2], off_perm, off_rows[2], off_status[2], off_first[2], bytes;
 };
 
 }  // namespace
@@ -86,12 +100,12 @@ struct dsp_ctx {
   bool loaded = false, reserved = false, imported = false, broken = false;
   int64_t bounds[DSP_MAX_WORLD + 1] = {0};
   int64_t N = 0, lo = 0, n_local = 0, nnz = 0;
-  int32_t dim = 0;
+  int32_t dim = 0, feat_stride = 0;  // feature row length / padded stride (floats)
   int64_t *d_indptr = nullptr;
   int32_t *d_indices = nullptr;
   float *d_feat = nullptr;
   int64_t feat_bytes = 0;
-  int *d_err = nullptr;  // gather error latch
+  int *d_err = nullptr;  // latched device error of this ctx
   // exchange
   int32_t max_seeds = 0, L = 0, kmax = 0;
   int32_t fanouts[DSP_MAX_LAYERS] = {0};
@@ -102,9 +116,12 @@ struct dsp_ctx {
   char *peer_xch[DSP_MAX_WORLD] = {nullptr};
   void *ipc_opened[2 * DSP_MAX_WORLD] = {nullptr};
   unsigned long long seq = 0;
-  // host staging
-  WsHeader *h_hdr = nullptr;  // pinned
+  // host staging (pinned)
+  WsHeader *h_hdr = nullptr;
+  int *h_err = nullptr;
   int num_sms = 148;
+  int persist_blocks_per_sm = 1;
+  int gather_blocks_per_sm = 1;
 };
 
 namespace {
@@ -145,15 +162,6 @@ struct DeviceGuard {
   }
 };
 
-bool is_device_ptr(const void *p) {
-  cudaPointerAttributes at;
-  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
-    cudaGetLastError();
-    return false;
-  }
-  return at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged;
-}
-
 dsp_status check_fanouts(dsp_ctx *c, const int32_t *fanouts, int32_t L) {
   if (L < 1 || L > DSP_MAX_LAYERS || !fanouts)
     return fail(c, DSP_ERR_INVALID_ARG, "num_layers must be in [1, %d]", DSP_MAX_LAYERS);
@@ -167,33 +175,40 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L) {
   Plan p{};
   p.L = L;
   p.F[0] = num_seeds;
-  p.max_F = num_seeds;
-  p.max_slots = 0;
-  p.max_cap = 64;
+  p.max_F = std::max<int64_t>(1, num_seeds);
+  p.max_slots = 1;
   for (int l = 0; l < L; ++l) {
     p.E[l] = p.F[l] * fanouts[l];
-    p.S[l] = std::min<int64_t>(N, p.F[l] + p.E[l]);
-    p.S[l] = std::max<int64_t>(p.S[l], p.F[l]);
+    p.S[l] = std::max<int64_t>(p.F[l], std::min<int64_t>(N, p.F[l] + p.E[l]));
     p.F[l + 1] = p.S[l];
-    p.cap[l] = next_pow2(std::max<int64_t>(64, 2 * p.S[l]));
     p.max_F = std::max(p.max_F, p.F[l]);
     p.max_slots = std::max(p.max_slots, p.E[l]);
-    p.max_cap = std::max(p.max_cap, p.cap[l]);
   }
-  p.max_tiles = (p.max_slots + SCAN_TILE - 1) / SCAN_TILE + 1;
-  size_t o = align_up(sizeof(WsHeader), 256);
-  p.off_cnt = o;
-  o = align_up(o + sizeof(int32_t) * std::max<int64_t>(1, p.max_F), 256);
+  p.status_len = align_up((size_t)((p.max_slots + SCAN_TILE - 1) / SCAN_TILE + 2), 2);
+  size_t o = align_up(sizeof(WsPersist), 256);
+  p.off_hdr = o;
+  o = align_up(o + sizeof(WsHeader), 256);
+  p.off_agg = o;
+  o = align_up(o + sizeof(unsigned long long) * 2 * MAX_PERSIST_BLOCKS, 256);
+  for (int b = 0; b < 2; ++b) {
+    p.off_cnt[b] = o;
+    o = align_up(o + sizeof(int32_t) * p.max_F, 256);
+  }
   p.off_perm = o;
-  o = align_up(o + sizeof(int32_t) * std::max<int64_t>(1, p.max_F), 256);
-  p.off_hpos = o;
-  o = align_up(o + sizeof(int32_t) * std::max<int64_t>(1, p.max_slots), 256);
-  p.off_status = o;  // ticket + tile status, immediately followed by the table
-  o = o + sizeof(unsigned long long) * (1 + p.max_tiles);
-  o = align_up(o, 256);
-  p.off_tbl = o;
-  o = o + sizeof(unsigned long long) * p.max_cap;
-  p.bytes = align_up(o, 256);
+  o = align_up(o + sizeof(int32_t) * p.max_F, 256);
+  for (int b = 0; b < 2; ++b) {
+    p.off_rows[b] = o;
+    o = align_up(o + sizeof(int32_t) * p.max_slots, 256);
+  }
+  for (int b = 0; b < 2; ++b) {
+    p.off_status[b] = o;
+    o = align_up(o + sizeof(unsigned long long) * p.status_len, 256);
+  }
+  for (int b = 0; b < 2; ++b) {
+    p.off_first[b] = o;
+    o = align_up(o + sizeof(unsigned long long) * std::max<int64_t>(1, N), 256);
+  }
+  p.bytes = o;
   return p;
 }
 
@@ -228,6 +243,21 @@ Bounds make_bounds(const dsp_ctx *c) {
 
 int grid_for(const dsp_ctx *c, int blocks_per_sm) { return c->num_sms * blocks_per_sm; }
 
+GatherArgs make_gather(const dsp_ctx *c, const int32_t *ids, int64_t n, const int32_t *n_dev, float *out) {
+  GatherArgs a{};
+  a.ids = ids;
+  a.n = n;
+  a.n_dev = n_dev;
+  a.dim4 = c->dim / 4;
+  a.stride4 = c->feat_stride / 4;
+  a.out = reinterpret_cast<float4 *>(out);
+  for (int r = 0; r < DSP_MAX_WORLD; ++r)
+    a.base[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_feat[r]) : nullptr;
+  a.bd = make_bounds(c);
+  a.err = c->d_err;
+  return a;
+}
+
 // ---------------------------------------------------------------- driver
 // One dsp_sample call for one ctx, split into stages so that
 // dsp_sample_group can interleave several ctxs stage by stage.
@@ -244,11 +274,26 @@ struct Call {
   Plan plan;
   WsHeader *hdr;
   unsigned long long seq0;
+  float *feat_out;     // fused gather (or nullptr)
+  int64_t *sizes_out;  // async sizes destination (or nullptr)
+  bool async;
 };
+
+LayerBufs bufs_of(const Call &k, int parity) {
+  LayerBufs b{};
+  b.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt[parity]);
+  b.rows = reinterpret_cast<int32_t *>(k.ws + k.plan.off_rows[parity]);
+  b.status = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_status[parity]);
+  b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_first[parity]);
+  return b;
+}
+
+WsPersist *persist_of(const Call &k) { return reinterpret_cast<WsPersist *>(k.ws); }
 
 dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_seeds,
                         const int32_t *fanouts, int32_t L, uint64_t rng_seed, dsp_block *blocks,
                         void *workspace, size_t ws_bytes, void *stream) {
+  k = Call{};
   k.c = c;
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
@@ -275,6 +320,7 @@ dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_s
   k.plan = make_plan(c->N, plan_seeds, fanouts, L);
   if (ws_bytes < k.plan.bytes)
     return fail(c, DSP_ERR_CAPACITY, "workspace %zu B < required %zu B", ws_bytes, k.plan.bytes);
+  if (((uintptr_t)workspace & 255u) != 0) return fail(c, DSP_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
   for (int l = 0; l < L; ++l) {
     if ((uint64_t)k.plan.F[l] + (uint64_t)k.plan.E[l] >= (1ull << 31))
       return fail(c, DSP_ERR_CAPACITY, "layer %d: frontier * (1 + fanout) exceeds 2^31", l);
@@ -296,7 +342,7 @@ dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_s
   k.blocks = blocks;
   k.ws = static_cast<char *>(workspace);
   k.stream = static_cast<cudaStream_t>(stream);
-  k.hdr = reinterpret_cast<WsHeader *>(k.ws);
+  k.hdr = reinterpret_cast<WsHeader *>(k.ws + k.plan.off_hdr);
   k.seq0 = c->seq;
   return DSP_OK;
 }
@@ -307,27 +353,59 @@ dsp_status stage_begin(Call &k) {
   return DSP_OK;
 }
 
-// table + tile status reset for layer l
-dsp_status stage_clear(Call &k, int l) {
-  DeviceGuard g(k.c->device);
-  const size_t bytes = (k.plan.off_tbl - k.plan.off_status) + sizeof(unsigned long long) * k.plan.cap[l];
-  CUDA_TRY(k.c, cudaMemsetAsync(k.ws + k.plan.off_status, 0xFF, bytes, k.stream));
+const int32_t *frontier_of(const Call &k, int l) { return l == 0 ? k.seeds : k.blocks[l - 1].src_ids; }
+
+uint2 key_of(uint64_t rng_seed) { return make_uint2((uint32_t)rng_seed, (uint32_t)(rng_seed >> 32)); }
+
+// world == 1: the whole call (+ optional gather) in one cooperative kernel
+dsp_status stage_persistent(Call &k) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  PersistArgs a{};
+  a.seeds = k.seeds;
+  a.B = k.num_seeds;
+  a.L = k.L;
+  for (int l = 0; l < k.L; ++l) {
+    a.k[l] = k.fanouts[l];
+    a.out.indptr[l] = k.blocks[l].indptr;
+    a.out.indices[l] = k.blocks[l].indices;
+    a.out.src_ids[l] = k.blocks[l].src_ids;
+  }
+  a.agg = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_agg);
+  a.persist = persist_of(k);
+  a.key = key_of(k.rng_seed);
+  a.indptr = c->d_indptr;
+  a.indices = c->d_indices;
+  a.lo = c->lo;
+  a.n_local = c->n_local;
+  a.buf[0] = bufs_of(k, 0);
+  a.buf[1] = bufs_of(k, 1);
+  a.hdr = k.hdr;
+  a.err = c->d_err;
+  a.gather = k.feat_out != nullptr;
+  if (a.gather) a.g = make_gather(c, k.blocks[k.L - 1].src_ids, 0, nullptr, k.feat_out);
+  void *args[] = {&a};
+  CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_persistent,
+                                          dim3(c->num_sms * c->persist_blocks_per_sm), dim3(PNT), args, 0,
+                                          k.stream));
   return DSP_OK;
 }
 
-const int32_t *frontier_of(const Call &k, int l) { return l == 0 ? k.seeds : k.blocks[l - 1].src_ids; }
+// ------------------------------------------------ world > 1, stage by stage
+dsp_status stage_clear(Call &k, int l) {  // look-back scan status + ticket of layer l
+  DeviceGuard g(k.c->device);
+  CUDA_TRY(k.c, cudaMemsetAsync(k.ws + k.plan.off_status[l & 1], 0xFF,
+                                sizeof(unsigned long long) * k.plan.status_len, k.stream));
+  return DSP_OK;
+}
 
 template <int G>
-void launch_local(const LocalSampleArgs &a, int grid, cudaStream_t s) {
-  k_sample_local<G><<<grid, 256, 0, s>>>(a);
-}
-template <int G>
 void launch_remote(const RemoteSampleArgs &a, int grid, cudaStream_t s) {
-  k_sample_remote<G><<<grid, 256, 0, s>>>(a);
+  k_sample_remote<G><<<grid, NT, 0, s>>>(a);
 }
 template <int G>
 void launch_unpermute(const UnpermuteArgs &a, int grid, cudaStream_t s) {
-  k_unpermute_insert<G><<<grid, 256, 0, s>>>(a);
+  k_unpermute_mark<G><<<grid, NT, 0, s>>>(a);
 }
 
 #define DISPATCH_G(G, FN, ...)                 \
@@ -339,32 +417,6 @@ void launch_unpermute(const UnpermuteArgs &a, int grid, cudaStream_t s) {
     case 16: FN<16>(__VA_ARGS__); break;       \
     default: FN<32>(__VA_ARGS__); break;       \
   }
-
-uint2 key_of(uint64_t rng_seed) { return make_uint2((uint32_t)rng_seed, (uint32_t)(rng_seed >> 32)); }
-
-// world == 1: fused sample + insert
-dsp_status stage_sample_local(Call &k, int l) {
-  dsp_ctx *c = k.c;
-  DeviceGuard g(c->device);
-  LocalSampleArgs a{};
-  a.frontier = frontier_of(k, l);
-  a.F0 = k.num_seeds;
-  a.layer = l;
-  a.k = k.fanouts[l];
-  a.key = key_of(k.rng_seed);
-  a.indptr = c->d_indptr;
-  a.indices = c->d_indices;
-  a.lo = c->lo;
-  a.n_local = c->n_local;
-  a.tbl = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_tbl);
-  a.mask = (uint32_t)(k.plan.cap[l] - 1);
-  a.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt);
-  a.hpos = reinterpret_cast<int32_t *>(k.ws + k.plan.off_hpos);
-  a.hdr = k.hdr;
-  DISPATCH_G(group_of(a.k), launch_local, a, grid_for(c, 8), k.stream);
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
-}
 
 XchPeers peers_of(const dsp_ctx *c) {
   XchPeers p{};
@@ -390,7 +442,9 @@ dsp_status stage_shuffle(Call &k, int l) {
   a.peers = peers_of(c);
   a.perm = reinterpret_cast<int32_t *>(k.ws + k.plan.off_perm);
   a.hdr = k.hdr;
-  k_bucket_scatter<<<grid_for(c, 2), 256, 0, k.stream>>>(a);
+  a.err = c->d_err;
+  const int64_t need = std::max<int64_t>(1, (k.plan.F[l] + NT - 1) / NT);
+  k_bucket_scatter<<<(int)std::min<int64_t>(need, grid_for(c, 2)), NT, 0, k.stream>>>(a);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
 }
@@ -413,6 +467,7 @@ dsp_status stage_sample_remote(Call &k, int l) {
   a.L = c->xl;
   a.peers = peers_of(c);
   a.hdr = k.hdr;
+  a.err = c->d_err;
   DISPATCH_G(group_of(a.k), launch_remote, a, grid_for(c, 8), k.stream);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
@@ -432,11 +487,11 @@ dsp_status stage_unpermute(Call &k, int l) {
   a.L = c->xl;
   a.self = c->d_xch;
   a.perm = reinterpret_cast<int32_t *>(k.ws + k.plan.off_perm);
-  a.tbl = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_tbl);
-  a.mask = (uint32_t)(k.plan.cap[l] - 1);
-  a.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt);
-  a.hpos = reinterpret_cast<int32_t *>(k.ws + k.plan.off_hpos);
+  a.buf = bufs_of(k, l & 1);
+  a.persist = persist_of(k);
+  a.src_out = k.blocks[l].src_ids;
   a.hdr = k.hdr;
+  a.err = c->d_err;
   DISPATCH_G(group_of(a.k), launch_unpermute, a, grid_for(c, 8), k.stream);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
@@ -448,86 +503,99 @@ dsp_status stage_scan_indices(Call &k, int l) {
   ScanArgs s{};
   s.layer = l;
   s.k = k.fanouts[l];
-  s.frontier = frontier_of(k, l);
-  s.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt);
-  s.hpos = reinterpret_cast<int32_t *>(k.ws + k.plan.off_hpos);
-  s.tbl = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_tbl);
-  s.status = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_status);
+  s.buf = bufs_of(k, l & 1);
+  s.persist = persist_of(k);
   s.indptr_out = k.blocks[l].indptr;
   s.src_ids_out = k.blocks[l].src_ids;
+  s.indices_out = k.blocks[l].indices;
   s.hdr = k.hdr;
   const int64_t tiles = std::max<int64_t>(1, (k.plan.E[l] + SCAN_TILE - 1) / SCAN_TILE);
-  const int scan_grid = (int)std::min<int64_t>(tiles, grid_for(c, 4));
-  k_scan_assign<<<scan_grid, SCAN_THREADS, 0, k.stream>>>(s);
+  k_scan_assign<<<(int)std::min<int64_t>(tiles, grid_for(c, 4)), NT, 0, k.stream>>>(s);
   CUDA_TRY(c, cudaGetLastError());
-  IndicesArgs w{};
-  w.layer = l;
-  w.k = k.fanouts[l];
-  w.cnt = s.cnt;
-  w.hpos = s.hpos;
-  w.tbl = s.tbl;
-  w.indptr = k.blocks[l].indptr;
-  w.indices_out = k.blocks[l].indices;
-  w.hdr = k.hdr;
-  const int64_t need = std::max<int64_t>(1, (k.plan.E[l] + 255) / 256);
-  k_write_indices<<<(int)std::min<int64_t>(need, grid_for(c, 8)), 256, 0, k.stream>>>(w);
+  const int64_t need = std::max<int64_t>(1, (k.plan.E[l] + NT - 1) / NT);
+  k_write_indices<<<(int)std::min<int64_t>(need, grid_for(c, 8)), NT, 0, k.stream>>>(s);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
 }
 
+dsp_status stage_gather_dev(Call &k) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  const int l = k.L - 1;
+  GatherArgs a = make_gather(c, k.blocks[l].src_ids, 0, &k.hdr->S[l], k.feat_out);
+  k_gather<<<grid_for(c, c->gather_blocks_per_sm), NT, 0, k.stream>>>(a);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+// ------------------------------------------------------------- end of call
 dsp_status stage_end_async(Call &k) {
-  DeviceGuard g(k.c->device);
-  CUDA_TRY(k.c, cudaMemcpyAsync(k.c->h_hdr, k.hdr, sizeof(WsHeader), cudaMemcpyDeviceToHost, k.stream));
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  if (k.async) {
+    if (k.sizes_out)
+      CUDA_TRY(c, cudaMemcpyAsync(k.sizes_out, k.hdr->sizes, sizeof(int64_t) * 3 * k.L, cudaMemcpyDefault,
+                                  k.stream));
+  } else {
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_hdr, k.hdr, sizeof(WsHeader), cudaMemcpyDeviceToHost, k.stream));
+    CUDA_TRY(c, cudaMemcpyAsync(c->h_err, c->d_err, sizeof(int), cudaMemcpyDeviceToHost, k.stream));
+  }
   return DSP_OK;
 }
 
 dsp_status stage_finish(Call &k) {
   dsp_ctx *c = k.c;
   DeviceGuard g(c->device);
-  CUDA_TRY(c, cudaStreamSynchronize(k.stream));
   c->seq = k.seq0 + k.L;
-  const WsHeader &h = *c->h_hdr;
-  if (h.err != 0) {
-    if (h.err == E_STATE && c->world > 1) c->broken = true;
-    return fail(c, (dsp_status)h.err, "device-detected error %d (%s) during dsp_sample", h.err,
-                dsp_status_str(h.err));
+  if (k.async) return DSP_OK;
+  CUDA_TRY(c, cudaStreamSynchronize(k.stream));
+  const int e = *c->h_err;
+  if (e != 0) {
+    CUDA_TRY(c, cudaMemset(c->d_err, 0, sizeof(int)));
+    if (e == E_STATE && c->world > 1) c->broken = true;
+    return fail(c, (dsp_status)e, "device-detected error %d (%s)", e, dsp_status_str(e));
   }
+  const WsHeader &h = *c->h_hdr;
   for (int l = 0; l < k.L; ++l) {
     k.blocks[l].num_dst = h.F[l];
     k.blocks[l].num_src = h.S[l];
     k.blocks[l].num_edges = h.E[l];
   }
-  return DSP_OK;
-}
-
-dsp_status run_layer_stages(std::vector<Call> &calls, int l) {
-  dsp_status st;
-  for (auto &k : calls)
-    if ((st = stage_clear(k, l)) != DSP_OK) return st;
-  if (calls[0].c->world == 1) {
-    for (auto &k : calls)
-      if ((st = stage_sample_local(k, l)) != DSP_OK) return st;
-  } else {
-    for (auto &k : calls)
-      if ((st = stage_shuffle(k, l)) != DSP_OK) return st;
-    for (auto &k : calls)
-      if ((st = stage_sample_remote(k, l)) != DSP_OK) return st;
-    for (auto &k : calls)
-      if ((st = stage_unpermute(k, l)) != DSP_OK) return st;
-  }
-  for (auto &k : calls)
-    if ((st = stage_scan_indices(k, l)) != DSP_OK) return st;
+  if (k.sizes_out)
+    for (int l = 0; l < k.L; ++l) {
+      k.sizes_out[3 * l + 0] = h.F[l];
+      k.sizes_out[3 * l + 1] = h.S[l];
+      k.sizes_out[3 * l + 2] = h.E[l];
+    }
   return DSP_OK;
 }
 
 dsp_status run_calls(std::vector<Call> &calls) {
   dsp_status st;
-  for (auto &k : calls)
-    if ((st = stage_begin(k)) != DSP_OK) return st;
-  for (int l = 0; l < calls[0].L; ++l)
-    if ((st = run_layer_stages(calls, l)) != DSP_OK) return st;
-  for (auto &k : calls)
-    if ((st = stage_end_async(k)) != DSP_OK) return st;
+#define EACH(STAGE)                                   \
+  for (auto &k : calls)                               \
+    if ((st = (STAGE)) != DSP_OK) return st;
+  EACH(stage_begin(k));
+  if (calls[0].c->world == 1) {
+    EACH(stage_persistent(k));
+  } else {
+    for (int l = 0; l < calls[0].L; ++l) {
+      EACH(stage_clear(k, l));
+      EACH(stage_shuffle(k, l));
+      EACH(stage_sample_remote(k, l));
+      EACH(stage_unpermute(k, l));
+      EACH(stage_scan_indices(k, l));
+    }
+    for (auto &k : calls)
+      if (k.feat_out && (st = stage_gather_dev(k)) != DSP_OK) return st;
+    for (auto &k : calls) {
+      DeviceGuard g(k.c->device);
+      k_epoch_advance<<<1, 1, 0, k.stream>>>(persist_of(k), (uint32_t)k.L);
+      CUDA_TRY(k.c, cudaGetLastError());
+    }
+  }
+  EACH(stage_end_async(k));
+#undef EACH
   dsp_status first = DSP_OK;
   for (auto &k : calls) {
     st = stage_finish(k);
@@ -549,7 +617,14 @@ void release(dsp_ctx *c) {
   cudaFree(c->d_xch);
   cudaFree(c->d_err);
   if (c->h_hdr) cudaFreeHost(c->h_hdr);
+  if (c->h_err) cudaFreeHost(c->h_err);
   cudaGetLastError();
+}
+
+dsp_status check_gather_out(dsp_ctx *c, const float *out) {
+  if (!c->d_feat) return fail(c, DSP_ERR_STATE, "no feature shard loaded");
+  if (((uintptr_t)out & 15u) != 0) return fail(c, DSP_ERR_INVALID_ARG, "feature output must be 16-byte aligned");
+  return DSP_OK;
 }
 
 }  // namespace
@@ -594,13 +669,30 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   if (prop.major != 10)
     return fail(nullptr, DSP_ERR_CUDA, "device %d is sm_%d%d; libdsp is built for sm_100a only",
                 cuda_device, prop.major, prop.minor);
+  if (!prop.cooperativeLaunch)
+    return fail(nullptr, DSP_ERR_CUDA, "device %d lacks cooperative launch", cuda_device);
   dsp_ctx *c = new dsp_ctx();
   c->rank = rank;
   c->world = world_size;
   c->device = cuda_device;
   c->num_sms = prop.multiProcessorCount;
   DeviceGuard g(cuda_device);
+  int occ = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_csp_persistent, PNT, 0) != cudaSuccess || occ < 1) {
+    cudaGetLastError();
+    delete c;
+    return fail(nullptr, DSP_ERR_CUDA, "occupancy query for the persistent kernel failed");
+  }
+  c->persist_blocks_per_sm = occ;
+  if (occ * c->num_sms > MAX_PERSIST_BLOCKS) c->persist_blocks_per_sm = MAX_PERSIST_BLOCKS / c->num_sms;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_gather, NT, 0) != cudaSuccess || occ < 1) {
+    cudaGetLastError();
+    delete c;
+    return fail(nullptr, DSP_ERR_CUDA, "occupancy query for the gather kernel failed");
+  }
+  c->gather_blocks_per_sm = occ;
   if (cudaMallocHost(&c->h_hdr, sizeof(WsHeader)) != cudaSuccess ||
+      cudaMallocHost(&c->h_err, sizeof(int)) != cudaSuccess ||
       cudaMalloc(&c->d_err, sizeof(int)) != cudaSuccess || cudaMemset(c->d_err, 0, sizeof(int)) != cudaSuccess) {
     cudaGetLastError();
     release(c);
@@ -643,18 +735,26 @@ dsp_status dsp_load_partition(dsp_ctx *c, const int64_t *bounds, const int64_t *
   if (first != 0 || c->nnz < 0) return fail(c, DSP_ERR_INVALID_ARG, "indptr[0] must be 0");
   if (c->nnz > 0 && !indices) return fail(c, DSP_ERR_INVALID_ARG, "indices is NULL");
   CUDA_TRY(c, cudaMalloc(&c->d_indices, sizeof(int32_t) * (size_t)std::max<int64_t>(1, c->nnz)));
-  if (c->nnz > 0)
+  if (c->nnz > 0) {
     CUDA_TRY(c, cudaMemcpy(c->d_indices, indices, sizeof(int32_t) * (size_t)c->nnz, cudaMemcpyDefault));
+    CUDA_TRY(c, cudaMemset(c->d_err, 0, sizeof(int)));
+    k_validate_indices<<<c->num_sms * 8, 256>>>(c->d_indices, c->nnz, c->N, c->d_err);
+    int bad = 0;
+    CUDA_TRY(c, cudaMemcpy(&bad, c->d_err, sizeof(int), cudaMemcpyDeviceToHost));
+    CUDA_TRY(c, cudaMemset(c->d_err, 0, sizeof(int)));
+    if (bad) return fail(c, DSP_ERR_OUT_OF_RANGE, "indices contain ids outside [0, N)");
+  }
   if (features) {
     c->dim = dim;
-    c->feat_bytes = (int64_t)sizeof(float) * dim * std::max<int64_t>(1, c->n_local);
+    c->feat_stride = (dim + FEAT_ALIGN_FLOATS - 1) / FEAT_ALIGN_FLOATS * FEAT_ALIGN_FLOATS;
+    c->feat_bytes = (int64_t)sizeof(float) * c->feat_stride * std::max<int64_t>(1, c->n_local);
     CUDA_TRY(c, cudaMalloc(&c->d_feat, (size_t)c->feat_bytes));
     if (c->n_local > 0)
-      CUDA_TRY(c, cudaMemcpy(c->d_feat, features, sizeof(float) * dim * (size_t)c->n_local, cudaMemcpyDefault));
+      CUDA_TRY(c, cudaMemcpy2D(c->d_feat, sizeof(float) * c->feat_stride, features, sizeof(float) * dim,
+                               sizeof(float) * dim, (size_t)c->n_local, cudaMemcpyDefault));
   }
   c->peer_feat[c->rank] = c->d_feat;
   c->loaded = true;
-  (void)is_device_ptr;
   return DSP_OK;
 }
 
@@ -707,10 +807,11 @@ dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
   h.feat_bytes = c->feat_bytes;
   h.xch_bytes = (int64_t)c->xl.bytes;
   h.dim = c->dim;
+  h.feat_stride = c->feat_stride;
   h.max_seeds = c->max_seeds;
   for (int r = 0; r <= c->world; ++r) h.bounds[r] = c->bounds[r];
   DeviceGuard g(c->device);
-  if (c->d_feat) {
+  if (c->d_feat && c->world > 1) {
     h.has_feat = 1;
     CUDA_TRY(c, cudaIpcGetMemHandle(&h.feat_ipc, c->d_feat));
   }
@@ -736,9 +837,8 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
     if (h.magic != HANDLE_MAGIC || h.rank != r || h.world != c->world)
       return fail(c, DSP_ERR_INVALID_ARG, "handle %d is not rank %d of this world", r, r);
     for (int q = 0; q <= c->world; ++q)
-      if (h.bounds[q] != c->bounds[q])
-        return fail(c, DSP_ERR_STATE, "rank %d has different bounds", r);
-    if (h.dim != c->dim || h.max_seeds != c->max_seeds)
+      if (h.bounds[q] != c->bounds[q]) return fail(c, DSP_ERR_STATE, "rank %d has different bounds", r);
+    if (h.dim != c->dim || h.feat_stride != c->feat_stride || h.max_seeds != c->max_seeds)
       return fail(c, DSP_ERR_STATE, "rank %d has a different dim / max_seeds", r);
     if (r == c->rank) continue;
     const bool same_process = h.pid == my_pid && h.boot_id == boot_id();
@@ -811,6 +911,29 @@ dsp_status dsp_sample(dsp_ctx *c, const int32_t *seeds, int32_t num_seeds, const
   return run_calls(calls);
 }
 
+dsp_status dsp_sample_gather(dsp_ctx *c, const int32_t *seeds, int32_t num_seeds, const int32_t *fanouts,
+                             int32_t L, uint64_t rng_seed, dsp_block *blocks, float *feat_out,
+                             int64_t feat_cap_rows, void *workspace, size_t workspace_bytes,
+                             int64_t *sizes_out, uint32_t flags, void *stream) {
+  std::vector<Call> calls(1);
+  dsp_status st = prepare_call(calls[0], c, seeds, num_seeds, fanouts, L, rng_seed, blocks, workspace,
+                               workspace_bytes, stream);
+  if (st != DSP_OK) return st;
+  if ((flags & ~DSP_ASYNC) != 0) return fail(c, DSP_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
+  if (!feat_out) return fail(c, DSP_ERR_INVALID_ARG, "feat_out is NULL");
+  if ((st = check_gather_out(c, feat_out)) != DSP_OK) return st;
+  if (c->world > 1 && !c->imported) return fail(c, DSP_ERR_STATE, "dsp_import_handles first");
+  if (feat_cap_rows < calls[0].plan.S[L - 1])
+    return fail(c, DSP_ERR_CAPACITY, "feat_cap_rows %lld < max_src[L-1] %lld", (long long)feat_cap_rows,
+                (long long)calls[0].plan.S[L - 1]);
+  if (calls[0].plan.S[L - 1] * (c->dim / 4) >= (1ll << 31))
+    return fail(c, DSP_ERR_CAPACITY, "max_src[L-1] * dim / 4 must be < 2^31");
+  calls[0].feat_out = feat_out;
+  calls[0].sizes_out = sizes_out;
+  calls[0].async = (flags & DSP_ASYNC) != 0;
+  return run_calls(calls);
+}
+
 dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n, const int32_t *const *seeds,
                             const int32_t *num_seeds, const int32_t *fanouts, int32_t L,
                             uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
@@ -840,25 +963,18 @@ dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n, const int32_t *cons
 dsp_status dsp_gather_features(dsp_ctx *c, const int32_t *ids, int64_t n, float *out, void *stream) {
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
-  if (!c->loaded || !c->d_feat) return fail(c, DSP_ERR_STATE, "no feature shard loaded");
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "no partition loaded");
   if (c->world > 1 && !c->imported) return fail(c, DSP_ERR_STATE, "dsp_import_handles first");
   if (n < 0 || (n > 0 && (!ids || !out))) return fail(c, DSP_ERR_INVALID_ARG, "bad ids / out / n");
-  if (((uintptr_t)out & 15u) != 0) return fail(c, DSP_ERR_INVALID_ARG, "out must be 16-byte aligned");
+  dsp_status st = check_gather_out(c, out);
+  if (st != DSP_OK) return st;
   if (n == 0) return DSP_OK;
   DeviceGuard g(c->device);
-  GatherArgs a{};
-  a.ids = ids;
-  a.n = n;
-  a.dim4 = c->dim / 4;
-  a.out = reinterpret_cast<float4 *>(out);
-  for (int r = 0; r < DSP_MAX_WORLD; ++r)
-    a.base[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_feat[r]) : nullptr;
-  a.bd = make_bounds(c);
-  a.err = c->d_err;
-  const int64_t total = n * a.dim4;
-  const int64_t want = (total + 256 * 4 - 1) / (256 * 4);
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, grid_for(c, 8)));
-  k_gather<4><<<grid, 256, 0, static_cast<cudaStream_t>(stream)>>>(a);
+  GatherArgs a = make_gather(c, ids, n, nullptr, out);
+  if (n * a.dim4 >= (1ll << 31)) return fail(c, DSP_ERR_CAPACITY, "n * dim / 4 must be < 2^31 per call");
+  const int64_t want = (n * a.dim4 + (int64_t)NT * GATHER_UNROLL - 1) / ((int64_t)NT * GATHER_UNROLL);
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, grid_for(c, c->gather_blocks_per_sm)));
+  k_gather<<<grid, NT, 0, static_cast<cudaStream_t>(stream)>>>(a);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
 }
@@ -872,7 +988,8 @@ dsp_status dsp_sync(dsp_ctx *c, void *stream) {
   CUDA_TRY(c, cudaMemcpy(&e, c->d_err, sizeof(int), cudaMemcpyDeviceToHost));
   if (e != 0) {
     CUDA_TRY(c, cudaMemset(c->d_err, 0, sizeof(int)));
-    return fail(c, (dsp_status)e, "device-detected error %d (%s) in dsp_gather_features", e, dsp_status_str(e));
+    if (e == E_STATE && c->world > 1) c->broken = true;
+    return fail(c, (dsp_status)e, "device-detected error %d (%s)", e, dsp_status_str(e));
   }
   return DSP_OK;
 }

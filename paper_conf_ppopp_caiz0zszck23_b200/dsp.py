@@ -33,8 +33,9 @@ DSP_HANDLE_BYTES = 512
 #: every symbol include/dsp.h declares
 ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_create", "dsp_destroy",
                "dsp_load_partition", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
-               "dsp_sample_bounds", "dsp_sample", "dsp_sample_group", "dsp_gather_features",
-               "dsp_sync")
+               "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
+               "dsp_gather_features", "dsp_sync")
+DSP_ASYNC = 1
 
 
 class DSPError(RuntimeError):
@@ -77,11 +78,13 @@ def lib(path: str | None = None):
         L.dsp_import_handles.argtypes = [P, P]
         L.dsp_sample_bounds.argtypes = [P, i32, P, i32, P, P, ctypes.POINTER(ctypes.c_size_t)]
         L.dsp_sample.argtypes = [P, P, i32, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t, P]
+        L.dsp_sample_gather.argtypes = [P, P, i32, P, i32, ctypes.c_uint64, P, P, i64, P, ctypes.c_size_t, P,
+                                         ctypes.c_uint32, P]
         L.dsp_sample_group.argtypes = [P, i32, P, P, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t, P]
         L.dsp_gather_features.argtypes = [P, P, i64, P, P]
         L.dsp_sync.argtypes = [P, P]
         for name in ("dsp_create", "dsp_load_partition", "dsp_reserve", "dsp_export_handle",
-                     "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_group",
+                     "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                      "dsp_gather_features", "dsp_sync"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
@@ -178,6 +181,14 @@ def dsp_sample(ctx, seeds, num_seeds: int, fanouts, rng_seed: int, blocks, works
                             blocks, _p(workspace), workspace_bytes, ctypes.c_void_p(stream)), ctx)
 
 
+def dsp_sample_gather(ctx, seeds, num_seeds: int, fanouts, rng_seed: int, blocks, feat_out, feat_cap_rows: int,
+                      workspace, workspace_bytes: int, sizes_out, flags: int, stream: int) -> None:
+    f = _i32_array(fanouts)
+    _check(lib().dsp_sample_gather(ctx, _p(seeds), num_seeds, _p(f), len(f), ctypes.c_uint64(rng_seed), blocks,
+                                   _p(feat_out), feat_cap_rows, _p(workspace), workspace_bytes, _p(sizes_out),
+                                   flags, ctypes.c_void_p(stream)), ctx)
+
+
 def dsp_sample_group(ctxs, seeds, num_seeds, fanouts, rng_seed: int, blocks, workspaces,
                      workspace_bytes: int, streams) -> None:
     n = len(ctxs)
@@ -220,7 +231,7 @@ class Sampler:
 
     def __init__(self, bounds, indptr, indices, features, fanouts, max_seeds: int, rank: int = 0,
                  world_size: int = 1, device: int | None = None,
-                 exchange: Callable[[bytes], list] | None = None, connect: bool = True):
+                 exchange: Callable[[bytes], list] | None = None, connect: bool = True, n_slots: int = 1):
         import torch
         self.torch = torch
         self.device = torch.cuda.current_device() if device is None else device
@@ -238,19 +249,23 @@ class Sampler:
             raise
         dev = torch.device("cuda", self.device)
         self.workspace_bytes = ws
-        self.workspace = torch.empty(ws, dtype=torch.uint8, device=dev)
+        self.workspace = torch.zeros(ws, dtype=torch.uint8, device=dev)  # zero-filled before first use
         F = [self.max_seeds] + [int(x) for x in ms[:-1]]
-        self._bufs = []
-        self._cblocks = (dsp_block * len(self.fanouts))()
-        for l in range(len(self.fanouts)):
-            ip = torch.empty(F[l] + 1, dtype=torch.int32, device=dev)
-            ix = torch.empty(max(1, int(me[l])), dtype=torch.int32, device=dev)
-            sr = torch.empty(max(1, int(ms[l])), dtype=torch.int32, device=dev)
-            self._bufs.append((ip, ix, sr))
-            b = self._cblocks[l]
-            b.indptr, b.cap_indptr = ip.data_ptr(), ip.numel()
-            b.indices, b.cap_edges = ix.data_ptr(), int(me[l])
-            b.src_ids, b.cap_src = sr.data_ptr(), int(ms[l])
+        self._sets = []
+        for _ in range(max(1, n_slots)):   # output sets (a queue of capacity n_slots)
+            bufs = []
+            cblocks = (dsp_block * len(self.fanouts))()
+            for l in range(len(self.fanouts)):
+                ip = torch.empty(F[l] + 1, dtype=torch.int32, device=dev)
+                ix = torch.empty(max(1, int(me[l])), dtype=torch.int32, device=dev)
+                sr = torch.empty(max(1, int(ms[l])), dtype=torch.int32, device=dev)
+                bufs.append((ip, ix, sr))
+                b = cblocks[l]
+                b.indptr, b.cap_indptr = ip.data_ptr(), ip.numel()
+                b.indices, b.cap_edges = ix.data_ptr(), int(me[l])
+                b.src_ids, b.cap_src = sr.data_ptr(), int(ms[l])
+            self._sets.append([bufs, cblocks, None])
+        self._bufs, self._cblocks = self._sets[0][0], self._sets[0][1]
         self.max_src = [int(x) for x in ms]
         self.max_edges = [int(x) for x in me]
         self.connected = False
@@ -270,12 +285,39 @@ class Sampler:
                    self.workspace_bytes, self.stream())
         return self.blocks()
 
-    def blocks(self) -> list[Block]:
+    def sample_gather(self, seeds, rng_seed: int, slot: int = 0, sizes_out=None, async_: bool = False):
+        """One whole step (sample + gather) in one call into output set `slot`.
+        Synchronous: returns (blocks, features view).  async_: returns None;
+        sizes land in sizes_out (pinned host / device int64[3L]) in stream order."""
+        torch = self.torch
+        assert seeds.dtype == torch.int32 and seeds.is_cuda and seeds.is_contiguous()
+        feat_out = self.feat_buffer(slot)
+        dsp_sample_gather(self.ctx, seeds, seeds.numel(), self.fanouts, rng_seed, self._sets[slot][1], feat_out,
+                          feat_out.shape[0], self.workspace, self.workspace_bytes, sizes_out,
+                          DSP_ASYNC if async_ else 0, self.stream())
+        if async_:
+            return None
+        blocks = self.blocks(slot)
+        return blocks, feat_out[: blocks[-1].num_src]
+
+    def feat_buffer(self, slot: int = 0):
+        if self._sets[slot][2] is None:
+            self._sets[slot][2] = self.torch.empty((self.max_src[-1], self.dim), dtype=self.torch.float32,
+                                                   device=self.torch.device("cuda", self.device))
+        return self._sets[slot][2]
+
+    def blocks(self, slot: int = 0, sizes=None) -> list[Block]:
+        """Views of output set `slot`; sizes from the last synchronous call, or
+        from an int64[3L] array filled by an async call."""
+        bufs, cblocks, _ = self._sets[slot]
         out = []
-        for l, (ip, ix, sr) in enumerate(self._bufs):
-            b = self._cblocks[l]
-            out.append(Block(b.num_dst, b.num_src, b.num_edges, ip[: b.num_dst + 1], ix[: b.num_edges],
-                             sr[: b.num_src]))
+        for l, (ip, ix, sr) in enumerate(bufs):
+            if sizes is None:
+                b = cblocks[l]
+                nd, ns, ne = b.num_dst, b.num_src, b.num_edges
+            else:
+                nd, ns, ne = (int(x) for x in sizes[3 * l: 3 * l + 3])
+            out.append(Block(nd, ns, ne, ip[: nd + 1], ix[: ne], sr[: ns]))
         return out
 
     def gather(self, ids, out=None):

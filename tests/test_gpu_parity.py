@@ -253,3 +253,51 @@ def test_products_virtual_p4(pkg, products):
     exp = datagen.features_of(res[1][-1].src_ids.cpu().numpy(), cfg.dim)
     assert np.array_equal(out.cpu().numpy().view(np.uint32), exp.view(np.uint32))
     grp.close()
+
+
+# ------------------------------------------------------ fused step (one call)
+
+def test_sample_gather_sync_and_async(pkg, tiny):
+    """dsp_sample_gather: the whole step in one call (one persistent kernel at
+    world 1); synchronous and DSP_ASYNC with two alternating output sets."""
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2)
+    batches = seeds_of(cfg, 1, 0)
+    for step in range(4):
+        blocks, feat = s.sample_gather(torch.from_numpy(batches[step]).cuda(), 50 + step, slot=step % 2)
+        ref = oracle.sample(ip, ix, batches[step], cfg.fanouts, 50 + step)
+        assert_blocks_equal(blocks, ref, f"sync step {step}")
+        assert np.array_equal(feat.cpu().numpy().view(np.uint32),
+                              oracle.gather(feats, ref[-1]["src_ids"]).view(np.uint32))
+    L = len(cfg.fanouts)
+    sizes = torch.zeros((6, 3 * L), dtype=torch.int64).pin_memory()
+    dev = [torch.from_numpy(batches[10 + j]).cuda() for j in range(6)]
+    for j in range(6):
+        s.sample_gather(dev[j], 900 + j, slot=j % 2, sizes_out=sizes[j], async_=True)
+    s.sync()
+    for j in range(6):
+        ref = oracle.sample(ip, ix, batches[10 + j], cfg.fanouts, 900 + j)
+        exp = [v for r in ref for v in (r["num_dst"], r["num_src"], r["num_edges"])]
+        assert sizes[j].tolist() == exp
+        if j >= 4:   # the last two steps are still in the two output sets
+            blocks = s.blocks(j % 2, sizes=sizes[j].tolist())
+            assert_blocks_equal(blocks, ref, f"async step {j}")
+            feat = s.feat_buffer(j % 2)[: blocks[-1].num_src]
+            assert np.array_equal(feat.cpu().numpy().view(np.uint32),
+                                  oracle.gather(feats, ref[-1]["src_ids"]).view(np.uint32))
+    s.close()
+
+
+@pytest.mark.slow
+def test_products_fused_step(pkg, products):
+    cfg, ip, ix = products
+    feats = datagen.features(0, cfg.num_nodes, cfg.dim)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2)
+    batches = seeds_of(cfg, 1, 0)
+    for step in (5, 6):
+        blocks, feat = s.sample_gather(torch.from_numpy(batches[step]).cuda(), 7 + step, slot=step % 2)
+        ref = oracle.sample(ip, ix, batches[step], cfg.fanouts, 7 + step)
+        assert_blocks_equal(blocks, ref, f"products fused step {step}")
+        exp = datagen.features_of(ref[-1]["src_ids"], cfg.dim)
+        assert np.array_equal(feat.cpu().numpy().view(np.uint32), exp.view(np.uint32))
+    s.close()
