@@ -244,18 +244,23 @@ def run_dsp(args):
     K, W = args.steps, args.warmup
     h_sizes = torch.zeros((W + K, 3 * L), dtype=torch.int64).pin_memory()
 
+    pipelined = not args.no_pipeline
+
     def step(i, ev=None):
-        # one step = the whole hot path (CSP over all layers + feature gather), enqueued
-        # asynchronously; two output sets alternate (queue capacity 2)
+        # one step = the whole hot path (CSP over all layers + feature gather) for one
+        # batch.  Pipelined (default): the launch of step i samples batch i while its
+        # loader warps gather batch i-1 (the paper's pipeline); two output
+        # sets alternate (queue capacity 2); flush() gathers the last batch.
         if ev is not None:
             ev[0].record(stream)
         s.sample_gather(dev_batches[i % len(batches)], datagen.BASE_SEED + i, slot=i % 2,
-                        sizes_out=h_sizes[i], async_=True)
+                        sizes_out=h_sizes[i], async_=True, pipelined=pipelined)
         if ev is not None:
             ev[1].record(stream)
 
     for i in range(W):
         step(i)
+    s.flush()
     s.sync()
     barrier()
     torch.cuda.synchronize()
@@ -267,6 +272,7 @@ def run_dsp(args):
         ev0.record(stream)
         for j in range(K):
             step(W + j, sev[j])
+        s.flush()  # the gather of the last timed batch is inside the timed region
         ev1.record(stream)
         s.sync()
         torch.cuda.synchronize()
@@ -365,7 +371,8 @@ def run_dsp(args):
                        "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes,
                        "nnz": int(ip[-1]), "dim": cfg.dim, "parallelism": f"csp{world}",
                        "l2": "inputs larger than L2 (CSR 0.5 GB + features 1.1 GB >> 126 MB L2)",
-                       "step": "dsp_sample_gather (async, 2 output sets)"},
+                       "step": "dsp_sample_gather (DSP_PIPELINED: sampler(t) || loader(t-1), 2 output sets)"
+                       if pipelined else "dsp_sample_gather (async, 2 output sets)"},
             "seeds_per_s": tot_seeds / (t_max * 1e-3),
             "feature_GBps": tot_rows * cfg.dim * 4 / (t_max * 1e-3) / 1e9,
             "edges_per_step": tot_edges / K / world,
@@ -403,6 +410,7 @@ def main(argv=None):
     ap.add_argument("--ref-max-seconds", type=float, default=60.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-breakdown", action="store_true")
+    ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
     args = ap.parse_args(argv)
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

@@ -173,8 +173,9 @@ dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *
                             uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
                             size_t workspace_bytes, void *const *streams);
 
-/* Flag for dsp_sample_gather. */
+/* Flags for dsp_sample_gather. */
 #define DSP_ASYNC 1u
+#define DSP_PIPELINED 2u
 
 /* One whole step of the hot path in ONE stream-ordered call: dsp_sample
    followed by the feature gather of the last block's src_ids (the loader
@@ -194,11 +195,25 @@ dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *
                   written when the stream reaches the end of the step, and
                   device errors latch until dsp_sync.  Consecutive async
                   steps may reuse the same workspace and outputs in stream
-                  order (the producer/consumer pipeline of P:L198-200). */
+                  order (the producer/consumer pipeline of P:L198-200).
+                  DSP_PIPELINED (implies DSP_ASYNC) = the loader of the
+                  paper's pipeline runs one step behind the sampler
+                  (P:L198-200): this call samples its seeds into `blocks`
+                  while, in the same launch, it gathers the features owed by
+                  the PREVIOUS pipelined call of this ctx into that call's
+                  feat_out; this call's features are written by the next
+                  pipelined call or by dsp_pipeline_flush.  The caller keeps
+                  the previous call's blocks and feat_out alive until then
+                  (e.g. two output sets used alternately, a queue of capacity
+                  2).  A non-pipelined call flushes first. */
 dsp_status dsp_sample_gather(dsp_ctx *ctx, const int32_t *seeds, int32_t num_seeds, const int32_t *fanouts,
                              int32_t num_layers, uint64_t rng_seed, dsp_block *blocks, float *feat_out,
                              int64_t feat_cap_rows, void *workspace, size_t workspace_bytes,
                              int64_t *sizes_out, uint32_t flags, void *stream);
+
+/* Enqueues the gather still owed by the last DSP_PIPELINED call (no-op when
+   none is pending).  Stream-ordered on `stream`. */
+dsp_status dsp_pipeline_flush(dsp_ctx *ctx, void *stream);
 
 /* --------------------------------------------------------------- gather */
 

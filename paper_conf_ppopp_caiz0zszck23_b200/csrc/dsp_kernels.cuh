@@ -25,7 +25,8 @@
 // on work queued behind it.
 //
 // Data a phase reads after another phase of the same kernel wrote it is read
-// with ld.global.cg (L2), never through the non-coherent path.
+// with plain (weak) loads after the grid barrier's release/acquire, never
+// through the non-coherent path.
 #pragma once
 #include "dsp_device.cuh"
 
@@ -50,7 +51,9 @@ struct WsHeader {
   uint32_t done;         // last-block counter
   uint32_t bucket[8];    // per-owner send counters (bucket scatter)
   uint32_t bar_count;    // grid barrier arrivals
-  uint32_t pad[6];
+  uint32_t gcursor;      // next gather chunk (pipelined launches)
+  uint32_t chunks_loader, chunks_helper;  // gather chunks done by loader / sampling warps
+  uint32_t pad[3];
   unsigned long long t[24];   // %globaltimer at kernel start and when block 0 leaves each grid barrier
   unsigned long long ta[24];  // %globaltimer when block 0 arrives at each grid barrier
   unsigned long long dbg[32]; // debug stamps (DSP_DEBUG_STAMPS builds only)
@@ -72,6 +75,11 @@ struct Outputs {
 
 __device__ __forceinline__ int ldcg_i32(const int32_t *p) { return __ldcg(p); }
 __device__ __forceinline__ unsigned long long ldcg_u64(const unsigned long long *p) { return __ldcg(p); }
+// Weak load of data written earlier in the same kernel by other blocks and
+// published by a grid barrier (release / acquire): may be served by L1,
+// never through the non-coherent path.
+__device__ __forceinline__ int ldw_i32(const int32_t *p) { return *p; }
+__device__ __forceinline__ unsigned long long ldw_u64(const unsigned long long *p) { return *p; }
 __device__ __forceinline__ int ld_volatile_i32(const int32_t *p) { return *(volatile const int32_t *)p; }
 __device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long *p) {
   return *(volatile const unsigned long long *)p;
@@ -122,11 +130,21 @@ __device__ __forceinline__ uint32_t fdiv(uint64_t q, const FastDiv &f) {
 struct Span {
   int64_t end, first, step;
 };
+// The threads of a persistent block that run the sampling phases ("team"):
+// the whole block, or all but the loader warps of a pipelined launch.
+template <int TEAM>
+__device__ __forceinline__ void team_sync() {
+  if (TEAM == PNT)
+    __syncthreads();
+  else
+    asm volatile("bar.sync 1, %0;" ::"n"(TEAM) : "memory");
+}
+template <int TEAM = PNT>
 __device__ __forceinline__ Span block_span(int64_t total) {
   const int64_t chunk = (total + gridDim.x - 1) / gridDim.x;
   const int64_t b = min(total, (int64_t)blockIdx.x * chunk);
   const int64_t e = min(total, b + chunk);
-  return Span{e, b + threadIdx.x, (int64_t)blockDim.x};
+  return Span{e, b + threadIdx.x, (int64_t)TEAM};
 }
 __device__ __forceinline__ Span grid_span(int64_t total) {
   return Span{total, (int64_t)blockIdx.x * blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x};
@@ -149,8 +167,9 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu_u32(const uint32_t *p) {
 // return value, so no extra round trip); pollers acquire.  1.25 us at 148
 // blocks, vs 2.5 us for an atomicAdd + generation barrier over 592 blocks
 // (tools/micro/barrier_bench.cu).
+template <int TEAM = PNT>
 __device__ __forceinline__ void grid_barrier(WsHeader *hdr, uint32_t &target) {
-  __syncthreads();
+  team_sync<TEAM>();
   target += gridDim.x;
   if (threadIdx.x == 0) {
     const uint32_t g = target / gridDim.x;
@@ -160,7 +179,7 @@ __device__ __forceinline__ void grid_barrier(WsHeader *hdr, uint32_t &target) {
     }
     if (blockIdx.x == 0 && g < 23u) hdr->t[g] = globaltimer_ns();
   }
-  __syncthreads();
+  team_sync<TEAM>();
 }
 
 // ---------------------------------------------------------------- sampling
@@ -180,7 +199,7 @@ __device__ __forceinline__ void mark_dst(unsigned long long *first, int32_t v, i
 // Lane-group sampling (G lanes per node, G = next pow2 >= k): the draws run
 // on separate lanes, Floyd's resolution and the ranking via shuffles
 // (sample_node).  Used for k > 16.
-template <int G>
+template <int G, int TEAM = PNT>
 __device__ __forceinline__ void phase_sample_lanes(const int32_t *frontier, int F, int layer, int k, uint2 key,
                                                    const int64_t *__restrict__ indptr,
                                                    const int32_t *__restrict__ indices, int64_t lo,
@@ -189,16 +208,16 @@ __device__ __forceinline__ void phase_sample_lanes(const int32_t *frontier, int 
   constexpr int NPW = 32 / G;  // nodes per warp-iteration
   const int lane = threadIdx.x & 31;
   const bool leader = (lane & (G - 1)) == 0;
-  const Span sp = block_span(F);
+  const Span sp = block_span<TEAM>(F);
   const int64_t b0 = sp.first - threadIdx.x;  // first node of this block's chunk
-  const int wib = threadIdx.x >> 5, wpb = blockDim.x >> 5;
+  const int wib = threadIdx.x >> 5, wpb = TEAM >> 5;
   bool dbg_first = true;
   (void)hdr;
   for (int64_t base = b0 + (int64_t)wib * NPW; base < sp.end; base += (int64_t)wpb * NPW) {
     const int i = (int)(base + lane / G);
     const bool active = i < sp.end;
     DSTAMP(hdr, 0, 0, layer);
-    const int32_t v = active ? ldcg_i32(frontier + i) : 0;
+    const int32_t v = active ? ldw_i32(frontier + i) : 0;
     DSTAMP(hdr, 1, v, layer);
     const int64_t lv = (int64_t)v - lo;
     const bool ok = active && v >= 0 && lv >= 0 && lv < n_local;
@@ -235,19 +254,19 @@ __device__ __forceinline__ void phase_sample_lanes(const int32_t *frontier, int 
 // ranking run in one thread's registers; the k adjacency loads and the k + 1
 // marks are issued back to back (memory-level parallelism k per thread, every
 // frontier node in flight at once).
-template <int KB>
+template <int KB, int TEAM = PNT>
 __device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F, int layer, int k, uint2 key,
                                                  const int64_t *__restrict__ indptr,
                                                  const int32_t *__restrict__ indices, int64_t lo,
                                                  int64_t n_local, const LayerBufs &B, uint32_t epoch,
                                                  int32_t *src_out, int *err, WsHeader *hdr) {
-  const Span sp = block_span(F);
+  const Span sp = block_span<TEAM>(F);
   bool dbg_first = true;
   (void)hdr;
   for (int64_t ii = sp.first; ii < sp.end; ii += sp.step) {
     const int i = (int)ii;
     DSTAMP(hdr, 0, 0, layer);
-    const int32_t v = ldcg_i32(frontier + i);
+    const int32_t v = ldw_i32(frontier + i);
     DSTAMP(hdr, 1, v, layer);
     if (src_out) src_out[i] = v;  // dst copy (R17)
     const int64_t lv = (int64_t)v - lo;
@@ -312,28 +331,30 @@ __device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F,
 // per-(stripe, warp) counts and the block aggregate (published to `agg`);
 // after a grid barrier pass 2 adds the aggregates of the preceding blocks and
 // writes the outputs.  Items are striped (item j of thread t is slot
-// tile + j*PNT + t) so every load is a coalesced warp access; the in-block
+// tile + j*TEAM + t) so every load is a coalesced warp access; the in-block
 // prefix comes from warp ballots plus a table kept in shared memory across
 // the barrier, the flags in registers.
 constexpr int SCAN2_IPT = 8;
-constexpr int SCAN2_TILE = PNT * SCAN2_IPT;
+
 
 __device__ __forceinline__ unsigned long long pack2(uint32_t valid, uint32_t first) {
   return ((unsigned long long)first << 31) | valid;
 }
 
+template <int TEAM>
 struct Scan2Smem {
-  unsigned long long tab[SCAN2_IPT * (PNT / 32)];  // exclusive prefix of (stripe j, warp w)
-  unsigned long long red[2 * (PNT / 32) + 2];
+  unsigned long long tab[SCAN2_IPT * (TEAM / 32)];  // exclusive prefix of (stripe j, warp w)
+  unsigned long long red[2 * (TEAM / 32) + 2];
 };
 
 struct Scan2Regs {
   uint32_t vbits, fbits;
 };
 
+template <int TEAM>
 __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, uint32_t epoch, int64_t tile0,
                                             int64_t tile_end, Scan2Regs &R, unsigned long long *agg_slot,
-                                            Scan2Smem &sm) {
+                                            Scan2Smem<TEAM> &sm) {
   const uint32_t total = (uint32_t)tile_end;  // < 2^31 by the host's plan check
   const FastDiv fd = make_fastdiv((uint32_t)k);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -342,31 +363,31 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
   int32_t c[SCAN2_IPT], u[SCAN2_IPT];
 #pragma unroll
   for (int j = 0; j < SCAN2_IPT; ++j) {
-    const uint32_t q = q0 + j * PNT;
+    const uint32_t q = q0 + j * TEAM;
     c[j] = -1;
     u[j] = 0;
     if (q < total) {
       const uint32_t i = fdiv(q, fd);
-      c[j] = ldcg_i32(B.cnt + i) - (int32_t)(q - i * (uint32_t)k);  // > 0 iff slot q holds an edge
-      u[j] = ldcg_i32(B.rows + q);  // garbage unless valid; dereferenced only then
+      c[j] = ldw_i32(B.cnt + i) - (int32_t)(q - i * (uint32_t)k);  // > 0 iff slot q holds an edge
+      u[j] = ldw_i32(B.rows + q);  // garbage unless valid; dereferenced only then
     }
   }
   unsigned long long w[SCAN2_IPT];
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? ldcg_u64(B.first + u[j]) : 0ull;
+  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? ldw_u64(B.first + u[j]) : 0ull;
   R.vbits = R.fbits = 0;
 #pragma unroll
   for (int j = 0; j < SCAN2_IPT; ++j) {
     const bool valid = c[j] > 0;
-    const bool first = valid && w[j] == mark_word(epoch, (uint32_t)F + q0 + j * PNT);
+    const bool first = valid && w[j] == mark_word(epoch, (uint32_t)F + q0 + j * TEAM);
     R.vbits |= (valid ? 1u : 0u) << j;
     R.fbits |= (first ? 1u : 0u) << j;
     const uint32_t bv = __ballot_sync(FULL_MASK, valid), bf = __ballot_sync(FULL_MASK, first);
-    if (lane == 0) sm.tab[j * (PNT / 32) + wid] = pack2(__popc(bv), __popc(bf));
+    if (lane == 0) sm.tab[j * (TEAM / 32) + wid] = pack2(__popc(bv), __popc(bf));
   }
-  __syncthreads();
+  team_sync<TEAM>();
   if (wid == 0) {  // exclusive scan of the (stripe, warp) counts, stripe-major
-    constexpr int PER = SCAN2_IPT * (PNT / 32) / 32;
+    constexpr int PER = SCAN2_IPT * (TEAM / 32) / 32;
     unsigned long long v[PER], run = 0;
 #pragma unroll
     for (int e = 0; e < PER; ++e) {
@@ -387,14 +408,15 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
     }
     if (lane == 31) __stcg(agg_slot, incl);
   }
-  __syncthreads();
+  team_sync<TEAM>();
 }
 
 // prefix of block `blk` and the round total from the published aggregates
-__device__ __forceinline__ void scan2_prefix(const unsigned long long *agg, int nblk, int blk, Scan2Smem &sm,
+template <int TEAM>
+__device__ __forceinline__ void scan2_prefix(const unsigned long long *agg, int nblk, int blk, Scan2Smem<TEAM> &sm,
                                              unsigned long long *prefix, unsigned long long *round_total) {
   unsigned long long p = 0, t = 0;
-  for (int b = threadIdx.x; b < nblk; b += PNT) {
+  for (int b = threadIdx.x; b < nblk; b += TEAM) {
     const unsigned long long x = __ldcg(agg + b);
     t += x;
     if (b < blk) p += x;
@@ -407,30 +429,31 @@ __device__ __forceinline__ void scan2_prefix(const unsigned long long *agg, int 
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   if (lane == 0) {
     sm.red[wid] = p;
-    sm.red[PNT / 32 + wid] = t;
+    sm.red[TEAM / 32 + wid] = t;
   }
-  __syncthreads();
+  team_sync<TEAM>();
   if (threadIdx.x == 0) {
     unsigned long long pp = 0, tt = 0;
-    for (int w = 0; w < PNT / 32; ++w) {
+    for (int w = 0; w < TEAM / 32; ++w) {
       pp += sm.red[w];
-      tt += sm.red[PNT / 32 + w];
+      tt += sm.red[TEAM / 32 + w];
     }
-    sm.red[2 * (PNT / 32)] = pp;
-    sm.red[2 * (PNT / 32) + 1] = tt;
+    sm.red[2 * (TEAM / 32)] = pp;
+    sm.red[2 * (TEAM / 32) + 1] = tt;
   }
-  __syncthreads();
-  *prefix = sm.red[2 * (PNT / 32)];
-  *round_total = sm.red[2 * (PNT / 32) + 1];
-  __syncthreads();
+  team_sync<TEAM>();
+  *prefix = sm.red[2 * (TEAM / 32)];
+  *round_total = sm.red[2 * (TEAM / 32) + 1];
+  team_sync<TEAM>();
 }
 
 // Block indptr at t == 0 slots; for first occurrences: new id nid = F + rank,
 // map word := (epoch, nid), src_out[nid] = u.  The dst copy is written by the
 // sample phase.
+template <int TEAM>
 __device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, uint32_t epoch, int64_t tile0,
                                             int64_t tile_end, const Scan2Regs &R, unsigned long long base,
-                                            const Scan2Smem &sm, int32_t *indptr_out, int32_t *src_out) {
+                                            const Scan2Smem<TEAM> &sm, int32_t *indptr_out, int32_t *src_out) {
   const uint32_t total = (uint32_t)tile_end;
   const FastDiv fd = make_fastdiv((uint32_t)k);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -438,14 +461,14 @@ __device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, ui
   const uint32_t q0 = (uint32_t)tile0 + threadIdx.x;
   int32_t u[SCAN2_IPT];
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) u[j] = ((R.fbits >> j) & 1u) ? ldcg_i32(B.rows + q0 + j * PNT) : 0;
+  for (int j = 0; j < SCAN2_IPT; ++j) u[j] = ((R.fbits >> j) & 1u) ? ldw_i32(B.rows + q0 + j * TEAM) : 0;
 #pragma unroll
   for (int j = 0; j < SCAN2_IPT; ++j) {
     const uint32_t bv = __ballot_sync(FULL_MASK, (R.vbits >> j) & 1u);
     const uint32_t bf = __ballot_sync(FULL_MASK, (R.fbits >> j) & 1u);
-    const uint32_t q = q0 + j * PNT;
+    const uint32_t q = q0 + j * TEAM;
     if (q < total) {
-      const unsigned long long b = base + sm.tab[j * (PNT / 32) + wid];
+      const unsigned long long b = base + sm.tab[j * (TEAM / 32) + wid];
       const uint32_t i = fdiv(q, fd);
       if (q == i * (uint32_t)k) indptr_out[i] = (int32_t)((uint32_t)(b & 0x7fffffffull) + __popc(bv & lt));
       if ((R.fbits >> j) & 1u) {
@@ -476,14 +499,14 @@ __device__ __forceinline__ void phase_indices(int F, int k, const LayerBufs &B, 
       if (q < end) {
         const uint32_t i = fdiv(q, fd);
         const int32_t t = (int32_t)(q - i * (uint32_t)k);
-        c[j] = ldcg_i32(B.cnt + i) - t;  // > 0 iff slot q holds an edge
-        u[j] = ldcg_i32(B.rows + q);
-        ip[j] = ldcg_i32(indptr + i) + t;
+        c[j] = ldw_i32(B.cnt + i) - t;  // > 0 iff slot q holds an edge
+        u[j] = ldw_i32(B.rows + q);
+        ip[j] = ldw_i32(indptr + i) + t;
       }
     }
     unsigned long long w[U];
 #pragma unroll
-    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? ldcg_u64(B.first + u[j]) : 0ull;
+    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? ldw_u64(B.first + u[j]) : 0ull;
 #pragma unroll
     for (int j = 0; j < U; ++j)
       if (c[j] > 0) indices_out[ip[j]] = (int32_t)mark_x(w[j]);
@@ -519,6 +542,7 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
   const uint32_t tid = (uint32_t)tid64, nthreads = (uint32_t)nthreads64;
   const uint32_t dim4 = (uint32_t)a.dim4;
   const int32_t N = (int32_t)a.bd.b[a.bd.world];
+  const unsigned long long pol = l2_policy_evict_first();
   for (uint32_t e0 = tid; e0 < total; e0 += nthreads * UNROLL) {
     int32_t g[UNROLL];
     uint32_t c[UNROLL];
@@ -530,7 +554,7 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
       if (e < total) {
         const uint32_t r = e / dim4;
         c[u] = e - r * dim4;
-        g[u] = ldcg_i32(a.ids + r);
+        g[u] = ldw_i32(a.ids + r);
       }
     }
     float4 v[UNROLL];
@@ -538,7 +562,7 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
     for (int u = 0; u < UNROLL; ++u) {
       if (g[u] >= 0 && g[u] < N) {
         const int o = owner_of(a.bd, g[u]);
-        v[u] = ld_stream_f4(a.base[o] + (size_t)(uint32_t)(g[u] - (int32_t)a.bd.b[o]) * (uint32_t)a.stride4 + c[u]);
+        v[u] = ld_f4_hint(a.base[o] + (size_t)(uint32_t)(g[u] - (int32_t)a.bd.b[o]) * (uint32_t)a.stride4 + c[u], pol);
       }
     }
 #pragma unroll
@@ -546,7 +570,7 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
       const uint32_t e = e0 + (uint32_t)u * nthreads;
       if (e < total) {
         if (g[u] >= 0 && g[u] < N)
-          __stcs(a.out + e, v[u]);
+          st_f4_hint(a.out + e, v[u], pol);
         else
           latch(a.err, E_RANGE);
       }
@@ -562,6 +586,10 @@ __global__ void __launch_bounds__(NT) k_gather(GatherArgs a) {
 }
 
 // ============================================ world == 1: persistent kernel
+constexpr int LOADER_WARPS = 4;                      // TMA gather warps of a pipelined launch
+constexpr int LOADER_SLOTS = 2;                      // ring slots per loader warp
+constexpr int PIPE_TEAM = PNT - 32 * LOADER_WARPS;   // sampling threads of a pipelined launch
+
 struct PersistArgs {
   const int32_t *seeds;
   int32_t B;
@@ -577,39 +605,191 @@ struct PersistArgs {
   WsPersist *persist;
   WsHeader *hdr;
   int *err;
-  int32_t gather;           // fuse the gather of the last block's src_ids
-  GatherArgs g;
+  int32_t gather;           // fuse the gather of this call's last block (non-pipelined)
+  GatherArgs g;             // this call's gather
+  // pipelined: gather owed by the previous call, by the loader warps + idle samplers
+  int32_t prev;             // 1 if there is one
+  GatherArgs gp;            // ids / n_dev / out of the previous call
+  int32_t *pend_n;          // where this call's row count goes (read by the next call / flush)
+  int32_t rows_per_chunk;   // R
+  int32_t slot_bytes;       // ring slot size (>= R * row bytes)
 };
 
+template <int TEAM>
 __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32_t *frontier, int F, int l,
                                                uint32_t epoch) {
   const int k = a.k[l];
   const LayerBufs &B = a.buf[l & 1];
   if (k <= 8) {
-    phase_sample_tpn<8>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch, a.out.src_ids[l],
-                        a.err, a.hdr);
+    phase_sample_tpn<8, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
+                              a.out.src_ids[l], a.err, a.hdr);
   } else if (k <= 16) {
-    phase_sample_tpn<16>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch, a.out.src_ids[l],
-                         a.err, a.hdr);
+    phase_sample_tpn<16, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
+                               a.out.src_ids[l], a.err, a.hdr);
   } else {
-    phase_sample_lanes<32>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
-                           a.out.src_ids[l], a.err, a.hdr);
+    phase_sample_lanes<32, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
+                                 a.out.src_ids[l], a.err, a.hdr);
   }
 }
 
-// The whole CSP call for world == 1 (and the fused gather) in one launch:
-// per layer  sample(l) + indices(l-1) | scan pass 1 | scan pass 2, separated
-// by grid barriers; no host round trip, no table clearing (epochs).
+// Loader warp of a pipelined launch: gathers chunks of R consecutive output
+// rows of the previous call with TMA bulk copies (one cp.async.bulk per row
+// into a shared-memory ring slot, completion counted on the slot's mbarrier,
+// then one bulk store of the R contiguous output rows).  Chunks come from a
+// grid-wide cursor, so the sampling warps can join when they are done.
+// 4 warps per SM sustain ~5 TB/s on random 400-byte rows
+// (tools/micro/tma_gather_bench.cu), leaving 28 warps for the sampling.
+__device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, uint64_t *bars, int64_t n) {
+  const int lane = threadIdx.x & 31;
+  const GatherArgs &g = a.gp;
+  const int R = a.rows_per_chunk;
+  const uint32_t row_bytes = (uint32_t)g.dim4 * 16u, stride_bytes = (uint32_t)g.stride4 * 16u;
+  const int64_t nchunks = (n + R - 1) / R;
+  const char *base = reinterpret_cast<const char *>(g.base[0]);
+  char *out = reinterpret_cast<char *>(g.out);
+  const unsigned long long pol = l2_policy_evict_first();
+  int issued = 0, done = 0;
+  int chunk0 = 0, chunk1 = 0;  // chunk held by slot 0 / slot 1 (LOADER_SLOTS == 2)
+  bool exhausted = false;
+  while (true) {
+    while (!exhausted && issued - done < LOADER_SLOTS) {
+      int c = 0;
+      if (lane == 0) c = (int)atomicAdd(&a.hdr->gcursor, 1u);
+      c = __shfl_sync(FULL_MASK, c, 0);
+      if (c >= nchunks) {
+        exhausted = true;
+        break;
+      }
+      const int s = issued % LOADER_SLOTS;
+      if (issued >= LOADER_SLOTS) {  // the slot's previous store must have read its smem
+        if (lane == 0) bulk_wait_read<LOADER_SLOTS - 1>();
+        __syncwarp();
+      }
+      const int rows = (int)min((int64_t)R, n - (int64_t)c * R);
+      if (lane == 0) mbar_expect_tx(&bars[s], (uint32_t)rows * row_bytes);
+      __syncwarp();
+      if (lane < rows) {
+        const int32_t id = __ldg(g.ids + (int64_t)c * R + lane);
+        if (id >= 0 && id < (int32_t)g.bd.b[1])
+          bulk_g2s_hint(ring + (size_t)s * a.slot_bytes + (size_t)lane * row_bytes,
+                        base + (size_t)(uint32_t)id * stride_bytes, row_bytes, &bars[s], pol);
+        else  // keep the byte count consistent; the error is reported
+          latch(g.err, E_RANGE);
+      }
+      if (s == 0) chunk0 = c; else chunk1 = c;
+      ++issued;
+    }
+    if (done == issued) break;
+    if (lane == 0) atomicAdd(&a.hdr->chunks_loader, 1u);
+    const int s = done % LOADER_SLOTS;
+    const int c = s == 0 ? chunk0 : chunk1;
+    const int rows = (int)min((int64_t)R, n - (int64_t)c * R);
+    bool bad = false;
+    if (lane == 0) {
+      // an out-of-range id never delivers its bytes: do not wait forever on it
+      const unsigned long long t0 = globaltimer_ns();
+      while (!mbar_try_wait(&bars[s], (uint32_t)(done / LOADER_SLOTS) & 1u)) {
+        if (*(volatile int *)g.err != 0 && globaltimer_ns() - t0 > 1000000ull) {
+          bad = true;
+          break;
+        }
+      }
+      if (!bad) {
+        bulk_s2g_hint(out + (size_t)c * R * row_bytes, ring + (size_t)s * a.slot_bytes, (uint32_t)rows * row_bytes, pol);
+        bulk_commit();
+      }
+    }
+    bad = __shfl_sync(FULL_MASK, bad, 0);
+    __syncwarp();
+    ++done;
+    if (bad) break;
+  }
+  if (lane == 0) bulk_wait_all();
+}
+
+// A sampling warp that finished its phases takes remaining chunks of the
+// previous call's gather with 16-byte register loads.
+__device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
+  const int lane = threadIdx.x & 31;
+  const GatherArgs &g = a.gp;
+  const int R = a.rows_per_chunk;
+  const int64_t nchunks = (n + R - 1) / R;
+  const uint32_t dim4 = (uint32_t)g.dim4;
+  const unsigned long long pol = l2_policy_evict_first();
+  while (true) {
+    int c = 0;
+    if (lane == 0) c = (int)atomicAdd(&a.hdr->gcursor, 1u);
+    c = __shfl_sync(FULL_MASK, c, 0);
+    if (c >= nchunks) break;
+    if (lane == 0) atomicAdd(&a.hdr->chunks_helper, 1u);
+    const int64_t r0 = (int64_t)c * R;
+    const uint32_t total = (uint32_t)(min((int64_t)R, n - r0) * dim4);
+    for (uint32_t e0 = lane; e0 < total; e0 += 32 * 4) {
+      float4 v[4];
+      int32_t id[4];
+      uint32_t col[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t e = e0 + 32u * u;
+        id[u] = -1;
+        col[u] = 0;
+        if (e < total) {
+          const uint32_t r = e / dim4;
+          col[u] = e - r * dim4;
+          id[u] = __ldg(g.ids + r0 + r);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+        if (id[u] >= 0 && id[u] < (int32_t)g.bd.b[1])
+          v[u] = ld_f4_hint(g.base[0] + (size_t)(uint32_t)id[u] * g.stride4 + col[u], pol);
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const uint32_t e = e0 + 32u * u;
+        if (e < total) {
+          if (id[u] >= 0 && id[u] < (int32_t)g.bd.b[1])
+            st_f4_hint(g.out + r0 * dim4 + e, v[u], pol);
+          else
+            latch(g.err, E_RANGE);
+        }
+      }
+    }
+  }
+}
+
+// The whole CSP call for world == 1 in one launch: per layer sample(l) +
+// indices(l-1) | scan pass 1 | scan pass 2, separated by grid barriers; then
+// indices(L-1) and either this call's gather (all warps) or, pipelined, the
+// previous call's gather by the loader warps running alongside the sampling
+// (the paper's loader(t-1) || sampler(t)).  No host round trip,
+// no map clearing (epochs).
+template <int TEAM, bool PIPE>
 __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
-  __shared__ Scan2Smem sm;
-  const int64_t tid = blockIdx.x * (int64_t)PNT + threadIdx.x;
-  const int64_t nthreads = (int64_t)gridDim.x * PNT;
+  __shared__ Scan2Smem<TEAM> sm;
+  __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];
+  extern __shared__ __align__(128) char ring_smem[];
   const int blk = blockIdx.x, nblk = gridDim.x;
+
+  if (PIPE && threadIdx.x >= TEAM) {  // ------------------------------ loader warps
+    const int w = (threadIdx.x - TEAM) >> 5;
+    if ((threadIdx.x & 31) == 0)
+      for (int s2 = 0; s2 < LOADER_SLOTS; ++s2) mbar_init(&bars[w][s2], 1);
+    mbar_init_fence();
+    __syncwarp();
+    if (a.prev) {
+      const int64_t n = ld_volatile_i32(a.gp.n_dev);
+      loader_warp(a, ring_smem + (size_t)w * LOADER_SLOTS * a.slot_bytes, bars[w], n);
+    }
+    if (blockIdx.x == 0 && threadIdx.x == TEAM) a.hdr->t[22] = globaltimer_ns();  // loader warp 0 of block 0 done
+    return;
+  }
+
+  // ------------------------------------------------------------ sampling team
+  const int64_t tid = blockIdx.x * (int64_t)TEAM + threadIdx.x;
+  const int64_t nthreads = (int64_t)gridDim.x * TEAM;
   uint32_t bar = 0;  // grid barrier target
   const uint32_t e0 = *(volatile const uint32_t *)&a.persist->epoch;
-
-  // the host cleared the header just before the launch
-  if (tid == 0) {
+  if (tid == 0) {  // the host cleared the header just before the launch
     a.hdr->t[0] = globaltimer_ns();
     a.hdr->F[0] = a.B;
   }
@@ -619,15 +799,15 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
     const uint32_t epoch = e0 + 1 + l;
     const int32_t *frontier = l == 0 ? a.seeds : a.out.src_ids[l - 1];
     const int k = a.k[l];
-    // S(l): sample + marks; indices of layer l-1 in the same phase
-    persist_sample(a, frontier, F, l, epoch);
+    persist_sample<TEAM>(a, frontier, F, l, epoch);
     if (l > 0)
       phase_indices(Fprev, a.k[l - 1], a.buf[(l - 1) & 1], a.out.indptr[l - 1], a.out.indices[l - 1],
-                    block_span((int64_t)Fprev * a.k[l - 1]));
-    grid_barrier(a.hdr, bar);
-    // scan over the F*k edge slots: each block one contiguous chunk of <= SCAN2_TILE slots per round
+                    block_span<TEAM>((int64_t)Fprev * a.k[l - 1]));
+    grid_barrier<TEAM>(a.hdr, bar);
+    // scan over the F*k edge slots: each block one contiguous chunk of <= TEAM*IPT slots per round
+    constexpr int64_t TILE = (int64_t)TEAM * SCAN2_IPT;
     const int64_t total = (int64_t)F * k;
-    const int64_t rounds = total > 0 ? (total + (int64_t)nblk * SCAN2_TILE - 1) / ((int64_t)nblk * SCAN2_TILE) : 1;
+    const int64_t rounds = total > 0 ? (total + (int64_t)nblk * TILE - 1) / ((int64_t)nblk * TILE) : 1;
     const int64_t per_round = (total + rounds - 1) / rounds;
     const int64_t chunk = (per_round + nblk - 1) / nblk;
     unsigned long long carry = 0;
@@ -636,14 +816,14 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
       const int64_t r0 = r * per_round, r1 = min(total, r0 + per_round);
       const int64_t tile0 = min(r1, r0 + (int64_t)blk * chunk), tile_end = min(r1, tile0 + chunk);
       unsigned long long *agg = a.agg + (r & 1) * MAX_PERSIST_BLOCKS;
-      scan2_pass1(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, agg + blk, sm);
-      grid_barrier(a.hdr, bar);
+      scan2_pass1<TEAM>(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, agg + blk, sm);
+      grid_barrier<TEAM>(a.hdr, bar);
       unsigned long long prefix, round_total;
-      scan2_prefix(agg, nblk, blk, sm, &prefix, &round_total);
-      scan2_pass2(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
-                  a.out.src_ids[l]);
+      scan2_prefix<TEAM>(agg, nblk, blk, sm, &prefix, &round_total);
+      scan2_pass2<TEAM>(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
+                        a.out.src_ids[l]);
       carry += round_total;
-      if (r + 1 < rounds) grid_barrier(a.hdr, bar);
+      if (r + 1 < rounds) grid_barrier<TEAM>(a.hdr, bar);
     }
     const int32_t E = (int32_t)(carry & 0x7fffffffull);
     const int32_t nnew = (int32_t)((carry >> 31) & 0x7fffffffull);
@@ -658,14 +838,20 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
     }
     Fprev = F;
     F = F + nnew;
-    grid_barrier(a.hdr, bar);
+    grid_barrier<TEAM>(a.hdr, bar);
   }
-  // last layer's indices + the gather of its src_ids (F = num_src of the last block)
+  // last layer's indices (F = num_src of the last block)
   const int l = a.L - 1;
-  phase_indices(Fprev, a.k[l], a.buf[l & 1], a.out.indptr[l], a.out.indices[l], block_span((int64_t)Fprev * a.k[l]));
-  if (a.gather) phase_gather<GATHER_UNROLL>(a.g, F, tid, nthreads);
-  // the last block to finish advances the workspace epoch and stamps the end
-  __syncthreads();
+  phase_indices(Fprev, a.k[l], a.buf[l & 1], a.out.indptr[l], a.out.indices[l],
+                block_span<TEAM>((int64_t)Fprev * a.k[l]));
+  if (PIPE) {
+    if (tid == 0) *a.pend_n = F;  // this call's rows, gathered by the next pipelined call / flush
+    if (a.prev) helper_warp(a, ld_volatile_i32(a.gp.n_dev));
+  } else if (a.gather) {
+    phase_gather<GATHER_UNROLL>(a.g, F, tid, nthreads);
+  }
+  // the last sampling block to finish advances the workspace epoch and stamps the end
+  team_sync<TEAM>();
   if (threadIdx.x == 0) {
     __threadfence();
     if (atomicAdd(&a.hdr->done, 1u) == gridDim.x - 1) {

@@ -122,6 +122,11 @@ struct dsp_ctx {
   int num_sms = 148;
   int persist_blocks_per_sm = 1;
   int gather_blocks_per_sm = 1;
+  // pipelined steps: the gather owed by the previous DSP_PIPELINED call
+  int32_t *d_pend = nullptr;          // its row count (device, written by its kernel)
+  const int32_t *pend_ids = nullptr;  // its last block's src_ids
+  float *pend_out = nullptr;          // its feature output
+  bool pending = false;
 };
 
 namespace {
@@ -277,6 +282,7 @@ struct Call {
   float *feat_out;     // fused gather (or nullptr)
   int64_t *sizes_out;  // async sizes destination (or nullptr)
   bool async;
+  bool pipelined;      // gather this call's rows in the next pipelined call / flush
 };
 
 LayerBufs bufs_of(const Call &k, int parity) {
@@ -382,12 +388,38 @@ dsp_status stage_persistent(Call &k) {
   a.buf[1] = bufs_of(k, 1);
   a.hdr = k.hdr;
   a.err = c->d_err;
-  a.gather = k.feat_out != nullptr;
+  a.gather = k.feat_out != nullptr && !k.pipelined;
   if (a.gather) a.g = make_gather(c, k.blocks[k.L - 1].src_ids, 0, nullptr, k.feat_out);
+  const dim3 grid(c->num_sms * c->persist_blocks_per_sm), block(PNT);
   void *args[] = {&a};
-  CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_persistent,
-                                          dim3(c->num_sms * c->persist_blocks_per_sm), dim3(PNT), args, 0,
+  if (!k.pipelined) {
+    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_persistent<PNT, false>, grid, block, args, 0,
+                                            k.stream));
+    return DSP_OK;
+  }
+  a.prev = c->pending ? 1 : 0;
+  if (a.prev) a.gp = make_gather(c, c->pend_ids, 0, c->d_pend, c->pend_out);
+  a.pend_n = c->d_pend;
+  const int row_bytes = c->dim * 4;
+  a.slot_bytes = (int)align_up((size_t)std::max(12800, row_bytes), 128);
+  a.rows_per_chunk = std::max(1, std::min(32, a.slot_bytes / std::max(1, row_bytes)));
+  const size_t smem = (size_t)LOADER_WARPS * LOADER_SLOTS * a.slot_bytes;
+  CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_persistent<PIPE_TEAM, true>, grid, block, args, smem,
                                           k.stream));
+  c->pend_ids = k.blocks[k.L - 1].src_ids;
+  c->pend_out = k.feat_out;
+  c->pending = true;
+  return DSP_OK;
+}
+
+// gather owed by the last pipelined call (k_gather with the device row count)
+dsp_status stage_flush(dsp_ctx *c, cudaStream_t stream) {
+  if (!c->pending) return DSP_OK;
+  DeviceGuard g(c->device);
+  GatherArgs a = make_gather(c, c->pend_ids, 0, c->d_pend, c->pend_out);
+  k_gather<<<grid_for(c, std::min(6, c->gather_blocks_per_sm)), NT, 0, stream>>>(a);
+  CUDA_TRY(c, cudaGetLastError());
+  c->pending = false;
   return DSP_OK;
 }
 
@@ -523,7 +555,7 @@ dsp_status stage_gather_dev(Call &k) {
   DeviceGuard g(c->device);
   const int l = k.L - 1;
   GatherArgs a = make_gather(c, k.blocks[l].src_ids, 0, &k.hdr->S[l], k.feat_out);
-  k_gather<<<grid_for(c, c->gather_blocks_per_sm), NT, 0, k.stream>>>(a);
+  k_gather<<<grid_for(c, std::min(6, c->gather_blocks_per_sm)), NT, 0, k.stream>>>(a);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
 }
@@ -575,6 +607,10 @@ dsp_status run_calls(std::vector<Call> &calls) {
 #define EACH(STAGE)                                   \
   for (auto &k : calls)                               \
     if ((st = (STAGE)) != DSP_OK) return st;
+  // a non-pipelined call first settles a pending pipelined gather; so does a
+  // pipelined call of the stage-by-stage path (no loader warps there)
+  for (auto &k : calls)
+    if (k.c->pending && (!k.pipelined || k.c->world > 1) && (st = stage_flush(k.c, k.stream)) != DSP_OK) return st;
   EACH(stage_begin(k));
   if (calls[0].c->world == 1) {
     EACH(stage_persistent(k));
@@ -586,8 +622,18 @@ dsp_status run_calls(std::vector<Call> &calls) {
       EACH(stage_unpermute(k, l));
       EACH(stage_scan_indices(k, l));
     }
-    for (auto &k : calls)
-      if (k.feat_out && (st = stage_gather_dev(k)) != DSP_OK) return st;
+    for (auto &k : calls) {
+      if (k.feat_out && k.pipelined) {  // this call's rows: gathered by the next call / flush
+        DeviceGuard g(k.c->device);
+        CUDA_TRY(k.c, cudaMemcpyAsync(k.c->d_pend, &k.hdr->S[k.L - 1], sizeof(int32_t), cudaMemcpyDeviceToDevice,
+                                      k.stream));
+        k.c->pend_ids = k.blocks[k.L - 1].src_ids;
+        k.c->pend_out = k.feat_out;
+        k.c->pending = true;
+      } else if (k.feat_out && (st = stage_gather_dev(k)) != DSP_OK) {
+        return st;
+      }
+    }
     for (auto &k : calls) {
       DeviceGuard g(k.c->device);
       k_epoch_advance<<<1, 1, 0, k.stream>>>(persist_of(k), (uint32_t)k.L);
@@ -616,6 +662,7 @@ void release(dsp_ctx *c) {
   cudaFree(c->d_feat);
   cudaFree(c->d_xch);
   cudaFree(c->d_err);
+  cudaFree(c->d_pend);
   if (c->h_hdr) cudaFreeHost(c->h_hdr);
   if (c->h_err) cudaFreeHost(c->h_err);
   cudaGetLastError();
@@ -677,14 +724,20 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   c->device = cuda_device;
   c->num_sms = prop.multiProcessorCount;
   DeviceGuard g(cuda_device);
-  int occ = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_csp_persistent, PNT, 0) != cudaSuccess || occ < 1) {
+  int occ = 0, occ_pipe = 0;
+  const int pipe_smem = LOADER_WARPS * LOADER_SLOTS * 16384;  // largest ring (dim 4096)
+  if (cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_csp_persistent<PNT, false>, PNT, 0) != cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_pipe, k_csp_persistent<PIPE_TEAM, true>, PNT, pipe_smem) !=
+          cudaSuccess ||
+      occ < 1 || occ_pipe < 1) {
     cudaGetLastError();
     delete c;
     return fail(nullptr, DSP_ERR_CUDA, "occupancy query for the persistent kernel failed");
   }
-  c->persist_blocks_per_sm = occ;
-  if (occ * c->num_sms > MAX_PERSIST_BLOCKS) c->persist_blocks_per_sm = MAX_PERSIST_BLOCKS / c->num_sms;
+  c->persist_blocks_per_sm = std::min(occ, occ_pipe);
+  if (c->persist_blocks_per_sm * c->num_sms > MAX_PERSIST_BLOCKS) c->persist_blocks_per_sm = MAX_PERSIST_BLOCKS / c->num_sms;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_gather, NT, 0) != cudaSuccess || occ < 1) {
     cudaGetLastError();
     delete c;
@@ -693,7 +746,8 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   c->gather_blocks_per_sm = occ;
   if (cudaMallocHost(&c->h_hdr, sizeof(WsHeader)) != cudaSuccess ||
       cudaMallocHost(&c->h_err, sizeof(int)) != cudaSuccess ||
-      cudaMalloc(&c->d_err, sizeof(int)) != cudaSuccess || cudaMemset(c->d_err, 0, sizeof(int)) != cudaSuccess) {
+      cudaMalloc(&c->d_err, sizeof(int)) != cudaSuccess || cudaMemset(c->d_err, 0, sizeof(int)) != cudaSuccess ||
+      cudaMalloc(&c->d_pend, sizeof(int32_t)) != cudaSuccess) {
     cudaGetLastError();
     release(c);
     delete c;
@@ -919,7 +973,7 @@ dsp_status dsp_sample_gather(dsp_ctx *c, const int32_t *seeds, int32_t num_seeds
   dsp_status st = prepare_call(calls[0], c, seeds, num_seeds, fanouts, L, rng_seed, blocks, workspace,
                                workspace_bytes, stream);
   if (st != DSP_OK) return st;
-  if ((flags & ~DSP_ASYNC) != 0) return fail(c, DSP_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
+  if ((flags & ~(DSP_ASYNC | DSP_PIPELINED)) != 0) return fail(c, DSP_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
   if (!feat_out) return fail(c, DSP_ERR_INVALID_ARG, "feat_out is NULL");
   if ((st = check_gather_out(c, feat_out)) != DSP_OK) return st;
   if (c->world > 1 && !c->imported) return fail(c, DSP_ERR_STATE, "dsp_import_handles first");
@@ -930,8 +984,15 @@ dsp_status dsp_sample_gather(dsp_ctx *c, const int32_t *seeds, int32_t num_seeds
     return fail(c, DSP_ERR_CAPACITY, "max_src[L-1] * dim / 4 must be < 2^31");
   calls[0].feat_out = feat_out;
   calls[0].sizes_out = sizes_out;
-  calls[0].async = (flags & DSP_ASYNC) != 0;
+  calls[0].pipelined = (flags & DSP_PIPELINED) != 0;
+  calls[0].async = (flags & (DSP_ASYNC | DSP_PIPELINED)) != 0;
   return run_calls(calls);
+}
+
+dsp_status dsp_pipeline_flush(dsp_ctx *c, void *stream) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  return stage_flush(c, static_cast<cudaStream_t>(stream));
 }
 
 dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n, const int32_t *const *seeds,
@@ -973,7 +1034,8 @@ dsp_status dsp_gather_features(dsp_ctx *c, const int32_t *ids, int64_t n, float 
   GatherArgs a = make_gather(c, ids, n, nullptr, out);
   if (n * a.dim4 >= (1ll << 31)) return fail(c, DSP_ERR_CAPACITY, "n * dim / 4 must be < 2^31 per call");
   const int64_t want = (n * a.dim4 + (int64_t)NT * GATHER_UNROLL - 1) / ((int64_t)NT * GATHER_UNROLL);
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, grid_for(c, c->gather_blocks_per_sm)));
+  // resident blocks only (a partial extra wave costs more than it hides; tools/micro/tma_gather_bench.cu)
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, grid_for(c, std::min(6, c->gather_blocks_per_sm))));
   k_gather<<<grid, NT, 0, static_cast<cudaStream_t>(stream)>>>(a);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;

@@ -34,8 +34,9 @@ DSP_HANDLE_BYTES = 512
 ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_create", "dsp_destroy",
                "dsp_load_partition", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
                "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
-               "dsp_gather_features", "dsp_sync")
+               "dsp_pipeline_flush", "dsp_gather_features", "dsp_sync")
 DSP_ASYNC = 1
+DSP_PIPELINED = 2
 
 
 class DSPError(RuntimeError):
@@ -82,9 +83,11 @@ def lib(path: str | None = None):
                                          ctypes.c_uint32, P]
         L.dsp_sample_group.argtypes = [P, i32, P, P, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t, P]
         L.dsp_gather_features.argtypes = [P, P, i64, P, P]
+        L.dsp_pipeline_flush.argtypes = [P, P]
         L.dsp_sync.argtypes = [P, P]
         for name in ("dsp_create", "dsp_load_partition", "dsp_reserve", "dsp_export_handle",
                      "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
+                     "dsp_pipeline_flush",
                      "dsp_gather_features", "dsp_sync"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
@@ -203,6 +206,10 @@ def dsp_sample_group(ctxs, seeds, num_seeds, fanouts, rng_seed: int, blocks, wor
                                   c_blocks, c_ws, workspace_bytes, c_st), ctxs[0])
 
 
+def dsp_pipeline_flush(ctx, stream: int) -> None:
+    _check(lib().dsp_pipeline_flush(ctx, ctypes.c_void_p(stream)), ctx)
+
+
 def dsp_gather_features(ctx, ids, n: int, out, stream: int) -> None:
     _check(lib().dsp_gather_features(ctx, _p(ids), n, _p(out), ctypes.c_void_p(stream)), ctx)
 
@@ -285,17 +292,20 @@ class Sampler:
                    self.workspace_bytes, self.stream())
         return self.blocks()
 
-    def sample_gather(self, seeds, rng_seed: int, slot: int = 0, sizes_out=None, async_: bool = False):
+    def sample_gather(self, seeds, rng_seed: int, slot: int = 0, sizes_out=None, async_: bool = False,
+                      pipelined: bool = False):
         """One whole step (sample + gather) in one call into output set `slot`.
         Synchronous: returns (blocks, features view).  async_: returns None;
-        sizes land in sizes_out (pinned host / device int64[3L]) in stream order."""
+        sizes land in sizes_out (pinned host / device int64[3L]) in stream order.
+        pipelined: the features of this step are written by the next pipelined
+        step (or flush()), which gathers them while it samples."""
         torch = self.torch
         assert seeds.dtype == torch.int32 and seeds.is_cuda and seeds.is_contiguous()
         feat_out = self.feat_buffer(slot)
+        flags = DSP_PIPELINED if pipelined else (DSP_ASYNC if async_ else 0)
         dsp_sample_gather(self.ctx, seeds, seeds.numel(), self.fanouts, rng_seed, self._sets[slot][1], feat_out,
-                          feat_out.shape[0], self.workspace, self.workspace_bytes, sizes_out,
-                          DSP_ASYNC if async_ else 0, self.stream())
-        if async_:
+                          feat_out.shape[0], self.workspace, self.workspace_bytes, sizes_out, flags, self.stream())
+        if async_ or pipelined:
             return None
         blocks = self.blocks(slot)
         return blocks, feat_out[: blocks[-1].num_src]
@@ -330,6 +340,9 @@ class Sampler:
 
     def sync(self) -> None:
         dsp_sync(self.ctx, self.stream())
+
+    def flush(self) -> None:
+        dsp_pipeline_flush(self.ctx, self.stream())
 
     def close(self) -> None:
         if getattr(self, "ctx", None) is not None:

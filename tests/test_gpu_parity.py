@@ -301,3 +301,56 @@ def test_products_fused_step(pkg, products):
         exp = datagen.features_of(ref[-1]["src_ids"], cfg.dim)
         assert np.array_equal(feat.cpu().numpy().view(np.uint32), exp.view(np.uint32))
     s.close()
+
+
+def _check_step(s, slot, sizes, seeds, rng, ip, ix, feats_of):
+    ref = oracle.sample(ip, ix, seeds, s.fanouts, rng)
+    exp = [v for r in ref for v in (r["num_dst"], r["num_src"], r["num_edges"])]
+    assert [int(x) for x in sizes] == exp
+    blocks = s.blocks(slot, sizes=[int(x) for x in sizes])
+    assert_blocks_equal(blocks, ref, f"pipelined rng {rng}")
+    feat = s.feat_buffer(slot)[: blocks[-1].num_src]
+    assert np.array_equal(feat.cpu().numpy().view(np.uint32), feats_of(ref[-1]["src_ids"]).view(np.uint32))
+
+
+def test_pipelined_steps(pkg, tiny):
+    """DSP_PIPELINED: step j samples batch j while its loader warps gather the
+    features of batch j-1; flush gathers the last one."""
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2)
+    batches = seeds_of(cfg, 1, 0)
+    L = len(cfg.fanouts)
+    sizes = torch.zeros((8, 3 * L), dtype=torch.int64).pin_memory()
+    feats_of = lambda ids: oracle.gather(feats, ids)
+    for j in range(8):
+        s.sample_gather(torch.from_numpy(batches[j]).cuda(), 300 + j, slot=j % 2, sizes_out=sizes[j], pipelined=True)
+        if j >= 1:
+            s.sync()
+            _check_step(s, (j - 1) % 2, sizes[j - 1], batches[j - 1], 300 + j - 1, ip, ix, feats_of)
+    s.flush()
+    s.sync()
+    _check_step(s, 7 % 2, sizes[7], batches[7], 307, ip, ix, feats_of)
+    # a non-pipelined call after pipelined ones settles nothing twice and still matches
+    blocks, feat = s.sample_gather(torch.from_numpy(batches[9]).cuda(), 99, slot=0)
+    assert_blocks_equal(blocks, oracle.sample(ip, ix, batches[9], cfg.fanouts, 99))
+    s.close()
+
+
+@pytest.mark.slow
+def test_products_pipelined(pkg, products):
+    cfg, ip, ix = products
+    feats = datagen.features(0, cfg.num_nodes, cfg.dim)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2)
+    batches = seeds_of(cfg, 1, 0)
+    L = len(cfg.fanouts)
+    sizes = torch.zeros((3, 3 * L), dtype=torch.int64).pin_memory()
+    feats_of = lambda ids: datagen.features_of(ids, cfg.dim)
+    for j in range(3):
+        s.sample_gather(torch.from_numpy(batches[20 + j]).cuda(), 40 + j, slot=j % 2, sizes_out=sizes[j],
+                        pipelined=True)
+    s.sync()
+    _check_step(s, 1, sizes[1], batches[21], 41, ip, ix, feats_of)
+    s.flush()
+    s.sync()
+    _check_step(s, 0, sizes[2], batches[22], 42, ip, ix, feats_of)
+    s.close()

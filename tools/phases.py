@@ -16,7 +16,8 @@ train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
 batches = datagen.rank_seed_batches(train, bnds, 0, cfg.batch, 0)
 steps = int(sys.argv[1]) if len(sys.argv) > 1 else 10
 rows = []
-for mode in ("sample", "sample_gather"):
+modes = ["sample", "sample_gather", "pipelined"] if not os.environ.get("MODES") else os.environ["MODES"].split(",")
+for mode in modes:
     acc = []
     for i in range(steps):
         seeds = torch.from_numpy(batches[i]).cuda()
@@ -24,11 +25,18 @@ for mode in ("sample", "sample_gather"):
             seeds = seeds[:0]
         if mode == "sample":
             s.sample(seeds, 100 + i)
+        elif mode == "pipelined":
+            s.sample_gather(seeds, 100 + i, slot=i % 2, pipelined=True)
+            s.sync()
         else:
             s.sample_gather(seeds, 100 + i, slot=i % 2)
         t = s.workspace[:1024].view(torch.int64)[81:105].cpu().numpy()
         ta = s.workspace[:1024].view(torch.int64)[105:129].cpu().numpy()
-        nb = sum(1 for g in range(1, 23) if t[g] > t[0])
+        nb = sum(1 for g in range(1, 22) if t[g] > t[0])
+        if mode == "pipelined" and i == steps - 1:
+            hv = s.workspace[:1024].view(torch.int32)
+            print("  pipelined: loader warp0/block0 done at %.1f us; chunks loader %d helper %d" % (
+                (t[22] - t[0]) / 1e3, int(hv[158]), int(hv[159])))
         stamps = [t[0]] + [t[g] for g in range(1, nb + 1)] + [t[23]]
         work = [ta[g] - (t[g - 1]) for g in range(1, nb + 1)]
         acc.append(np.concatenate([np.diff(np.array(stamps, dtype=np.int64)) / 1e3, np.array(work) / 1e3]))
