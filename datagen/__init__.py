@@ -3,7 +3,7 @@
 This module holds none of the sampling method's arithmetic: it only makes the
 graph (R-MAT, symmetrised, renumbered by a Feistel bijection), the fp32
 feature table, the train-id set and the per-rank seed batches.  See
-``datagen.c`` for the recipe and DESIGN.md "Input recipe" for the reasoning.
+``datagen.cpp`` for the recipe and DESIGN.md "Input recipe" for the reasoning.
 """
 from __future__ import annotations
 
@@ -16,7 +16,7 @@ import subprocess
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_SRC = os.path.join(_HERE, "datagen.c")
+_SRC = os.path.join(_HERE, "datagen.cpp")
 _LIB = os.path.join(_HERE, "libdatagen.so")
 
 GRAPH_SEED = 1
@@ -54,7 +54,7 @@ CONFIGS = {
 def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
-        subprocess.check_call(["gcc", "-O3", "-march=x86-64-v3", "-std=c11", "-fPIC", "-shared",
+        subprocess.check_call(["g++", "-O3", "-march=x86-64-v3", "-std=c++17", "-fPIC", "-shared",
                                "-fopenmp", "-Wall", "-o", tmp, _SRC])
         os.replace(tmp, _LIB)
     return _LIB
