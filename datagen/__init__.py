@@ -76,6 +76,8 @@ def lib():
         L.datagen_features.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64,
                                        ctypes.c_int, P]
         L.datagen_features_of.argtypes = [P, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, P]
+        L.datagen_node_weights.argtypes = [ctypes.c_int64, ctypes.c_uint64, P]
+        L.datagen_edge_weights.argtypes = [P, ctypes.c_int64, P, P]
         L.datagen_permute.argtypes = [ctypes.c_int64, ctypes.c_uint64, ctypes.c_int64]
         L.datagen_permute.restype = ctypes.c_int64
         L.datagen_permute_many.argtypes = [ctypes.c_int64, ctypes.c_uint64, P, ctypes.c_int64, P]
@@ -117,6 +119,26 @@ def features_of(ids, dim: int, feat_seed: int = FEAT_SEED):
     ids = np.ascontiguousarray(ids, np.int32)
     out = np.empty((len(ids), dim), np.float32)
     lib().datagen_features_of(_ptr(ids), len(ids), dim, feat_seed, _ptr(out))
+    return out
+
+
+WEIGHT_SEED = 3
+
+
+def node_weights(n: int, seed: int = WEIGHT_SEED) -> np.ndarray:
+    """Biased-sampling node weights w_u: ~1/32 zeros, else k/16 in (0, 256]."""
+    out = np.empty(n, np.float32)
+    lib().datagen_node_weights(n, seed, _ptr(out))
+    return out
+
+
+def edge_weights(indices: np.ndarray, w: np.ndarray) -> np.ndarray:
+    """Weight stored with each edge e_{v,u}: w[u] ("DSP stores node weight w_u along
+    with edge e_{v,u}")."""
+    ix = np.ascontiguousarray(indices, np.int32)
+    w = np.ascontiguousarray(w, np.float32)
+    out = np.empty(len(ix), np.float32)
+    lib().datagen_edge_weights(_ptr(ix), len(ix), _ptr(w), _ptr(out))
     return out
 
 

@@ -228,6 +228,23 @@ void datagen_features(int64_t lo, int64_t hi, int32_t dim, uint64_t feat_seed, i
       out[(g - lo) * dim + col] = feat_value((uint64_t)g, (uint64_t)col, (uint64_t)dim, feat_seed);
 }
 
+// Node weights for biased sampling: about 1/32 of the nodes get
+// weight 0, the others a multiple of 1/16 in (0, 256] (exact in fp32 and in
+// the 16.16 fixed point the method uses).
+void datagen_node_weights(int64_t n, uint64_t seed, float *out) {
+#pragma omp parallel for schedule(static)
+  for (int64_t u = 0; u < n; ++u) {
+    const uint64_t h = splitmix64(seed ^ ((uint64_t)u * 0x9E3779B97F4A7C15ull));
+    out[u] = (h & 31u) == 0 ? 0.0f : (float)((h >> 40) % 4096u + 1u) / 16.0f;
+  }
+}
+
+// edge weight = weight of the edge's neighbour: out[e] = w[indices[e]]
+void datagen_edge_weights(const int32_t *indices, int64_t nnz, const float *w, float *out) {
+#pragma omp parallel for schedule(static)
+  for (int64_t e = 0; e < nnz; ++e) out[e] = w[indices[e]];
+}
+
 // features of arbitrary ids (for checking samples of huge tables)
 void datagen_features_of(const int32_t *ids, int64_t n, int32_t dim, uint64_t feat_seed, float *out) {
 #pragma omp parallel for schedule(static)

@@ -43,7 +43,7 @@ def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         tmp = _LIB + f".tmp{os.getpid()}"
         subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-Wall", "-Wextra",
-                               "-o", tmp, _SRC])
+                               "-o", tmp, _SRC, "-lm"])
         os.replace(tmp, _LIB)
     return _LIB
 
@@ -84,6 +84,18 @@ def lib():
                                     ctypes.c_uint64, ctypes.POINTER(_Block)]
         L.oracle_free_block.argtypes = [ctypes.POINTER(_Block)]
         L.oracle_gather.argtypes = [ctypes.c_int64, ctypes.c_int32, P, P, ctypes.c_int64, P]
+        L.oracle_weight_fixed.argtypes = [ctypes.c_float]
+        L.oracle_weight_fixed.restype = ctypes.c_uint32
+        L.oracle_biased_picks.argtypes = [ctypes.c_uint64, ctypes.c_int32, ctypes.c_int32, P, ctypes.c_int64,
+                                          ctypes.c_int32, P]
+        L.oracle_biased_picks.restype = ctypes.c_int32
+        L.oracle_node_positions_biased.argtypes = [ctypes.c_uint64, ctypes.c_int32, ctypes.c_int32, P,
+                                                   ctypes.c_int64, ctypes.c_int32, P]
+        L.oracle_node_positions_biased.restype = ctypes.c_int32
+        L.oracle_sample_rows_ex.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64, P, ctypes.c_int64,
+                                            ctypes.c_int32, ctypes.c_int32, ctypes.c_uint64, P, P]
+        L.oracle_sample_ex.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_int32, P, ctypes.c_int32,
+                                       ctypes.c_uint64, ctypes.POINTER(_Block)]
         _lib = L
     return _lib
 
@@ -134,15 +146,37 @@ def node_positions(rng_seed: int, v: int, l: int, d: int, k: int) -> np.ndarray:
 
 # ------------------------------------------------------------- sampling
 
-def sample_rows(indptr, indices, ids, k: int, l: int, rng_seed: int, id_offset: int = 0):
-    """Owner-side sampling stage for global ``ids`` over a CSR (shard)."""
+def weight_fixed(w: float) -> int:
+    """Fixed-point edge weight floor(w * 2^16) (0xffffffff = invalid)."""
+    return int(lib().oracle_weight_fixed(w))
+
+
+def biased_picks(rng_seed: int, v: int, l: int, a, k: int) -> np.ndarray:
+    """Successive weighted picks (draw order) over integer weights ``a``."""
+    a = _c(a, np.uint32)
+    out = np.zeros(max(32, k), np.int64)
+    c = lib().oracle_biased_picks(rng_seed, v, l, _ptr(a), len(a), k, _ptr(out))
+    return out[:c].copy()
+
+
+def node_positions_biased(rng_seed: int, v: int, l: int, a, k: int) -> np.ndarray:
+    a = _c(a, np.uint32)
+    out = np.zeros(max(32, k), np.int64)
+    c = lib().oracle_node_positions_biased(rng_seed, v, l, _ptr(a), len(a), k, _ptr(out))
+    return out[:c].copy()
+
+
+def sample_rows(indptr, indices, ids, k: int, l: int, rng_seed: int, id_offset: int = 0, weights=None):
+    """Owner-side sampling stage for global ``ids`` over a CSR (shard);
+    ``weights`` = fp32 per edge (biased sampling) or None (uniform)."""
     ip = _c(indptr, np.int64)
     ix = _c(indices, np.int32)
     ids = _c(ids, np.int32)
+    w = None if weights is None else _c(weights, np.float32)
     cnt = np.zeros(len(ids), np.int32)
     rows = np.zeros(len(ids) * k, np.int32)
-    rc = lib().oracle_sample_rows(len(ip) - 1, _ptr(ip), _ptr(ix), id_offset, _ptr(ids), len(ids), k,
-                                  l, rng_seed, _ptr(cnt), _ptr(rows))
+    rc = lib().oracle_sample_rows_ex(len(ip) - 1, _ptr(ip), _ptr(ix), None if w is None else _ptr(w), id_offset,
+                                     _ptr(ids), len(ids), k, l, rng_seed, _ptr(cnt), _ptr(rows))
     if rc != OK:
         raise OracleError(rc, "oracle_sample_rows")
     return cnt, rows.reshape(len(ids), k)
@@ -175,16 +209,18 @@ def build_block(N: int, frontier, cnt, rows) -> dict:
     return out
 
 
-def sample(indptr, indices, seeds, fanouts, rng_seed: int) -> list[dict]:
-    """Multi-layer node-wise sampling for one rank's seeds on the whole graph."""
+def sample(indptr, indices, seeds, fanouts, rng_seed: int, weights=None) -> list[dict]:
+    """Multi-layer node-wise sampling for one rank's seeds on the whole graph
+    (biased when ``weights``, fp32 per edge, is given)."""
     ip = _c(indptr, np.int64)
     ix = _c(indices, np.int32)
     sd = _c(seeds, np.int32)
     fo = _c(fanouts, np.int32)
+    w = None if weights is None else _c(weights, np.float32)
     L = len(fo)
     blocks = (_Block * max(L, 1))()
-    rc = lib().oracle_sample(len(ip) - 1, _ptr(ip), _ptr(ix), _ptr(sd), len(sd), _ptr(fo), L,
-                             rng_seed, blocks)
+    rc = lib().oracle_sample_ex(len(ip) - 1, _ptr(ip), _ptr(ix), None if w is None else _ptr(w), _ptr(sd),
+                                len(sd), _ptr(fo), L, rng_seed, blocks)
     if rc != OK:
         raise OracleError(rc, "oracle_sample")
     out = [_block_to_numpy(blocks[l]) for l in range(L)]

@@ -20,16 +20,19 @@ def owner_of(ids, bounds) -> np.ndarray:
     return np.searchsorted(np.asarray(bounds), np.asarray(ids, np.int64), side="right") - 1
 
 
-def _shard(indptr, indices, lo, hi):
+def _shard(indptr, indices, lo, hi, weights=None):
     ip = indptr[lo: hi + 1]
-    return ip - ip[0], indices[ip[0]: ip[-1]]
+    w = None if weights is None else weights[ip[0]: ip[-1]]
+    return ip - ip[0], indices[ip[0]: ip[-1]], w
 
 
-def replay_inprocess(indptr, indices, bounds, rank_seeds, fanouts, rng_seed, log=None):
-    """All P ranks in one process.  Returns blocks[r][l] (oracle dicts)."""
+def replay_inprocess(indptr, indices, bounds, rank_seeds, fanouts, rng_seed, log=None, weights=None):
+    """All P ranks in one process.  Returns blocks[r][l] (oracle dicts).
+    ``weights`` (fp32 per edge) selects biased sampling; each owner uses its
+    own shard of them."""
     N = len(indptr) - 1
     P = len(bounds) - 1
-    shards = [_shard(indptr, indices, int(bounds[o]), int(bounds[o + 1])) for o in range(P)]
+    shards = [_shard(indptr, indices, int(bounds[o]), int(bounds[o + 1]), weights) for o in range(P)]
     frontier = [np.asarray(s, np.int32) for s in rank_seeds]
     blocks = [[] for _ in range(P)]
     for l, k in enumerate(fanouts):
@@ -42,10 +45,10 @@ def replay_inprocess(indptr, indices, bounds, rank_seeds, fanouts, rng_seed, log
         # sample at the owner on its shard
         res = [[None] * P for _ in range(P)]
         for o in range(P):
-            ip, ix = shards[o]
+            ip, ix, w = shards[o]
             for r in range(P):
                 ids = frontier[r][req[r][o]]
-                res[r][o] = oracle.sample_rows(ip, ix, ids, k, l, rng_seed, id_offset=int(bounds[o]))
+                res[r][o] = oracle.sample_rows(ip, ix, ids, k, l, rng_seed, id_offset=int(bounds[o]), weights=w)
         # reshuffle back to request order, then build the block
         for r in range(P):
             F = len(frontier[r])
