@@ -163,13 +163,14 @@ def run_reference(args):
     import oracle
     cfg, ip, ix, bnds, sip, six, feats, train = load_workload(args.config, 0, 1)
     batches = datagen.rank_seed_batches(train, bnds, 0, cfg.batch, 0)
+    ew = datagen.edge_weights(ix, datagen.node_weights(cfg.num_nodes)) if args.scheme == "biased" else None
     edges = rows = 0
     steps_done = 0
     t_all = 0.0
     for step in range(args.warmup + args.steps):
         seeds = batches[step % len(batches)]
         t0 = time.perf_counter()
-        blocks = oracle.sample(ip, ix, seeds, cfg.fanouts, datagen.BASE_SEED + step)
+        blocks = oracle.sample(ip, ix, seeds, cfg.fanouts, datagen.BASE_SEED + step, weights=ew)
         out = oracle.gather(feats, blocks[-1]["src_ids"])
         dt = time.perf_counter() - t0
         if step >= args.warmup:
@@ -196,7 +197,7 @@ def run_reference(args):
     return 0
 
 
-def cpu_baseline(cfg, ip, ix, feats, batches, seconds: float):
+def cpu_baseline(cfg, ip, ix, feats, batches, seconds: float, weights=None):
     import datagen
     import oracle
     t_all = 0.0
@@ -205,7 +206,7 @@ def cpu_baseline(cfg, ip, ix, feats, batches, seconds: float):
     while t_all < seconds and n < len(batches):
         seeds = batches[n]
         t0 = time.perf_counter()
-        blocks = oracle.sample(ip, ix, seeds, cfg.fanouts, datagen.BASE_SEED + n)
+        blocks = oracle.sample(ip, ix, seeds, cfg.fanouts, datagen.BASE_SEED + n, weights=weights)
         oracle.gather(feats, blocks[-1]["src_ids"])
         t_all += time.perf_counter() - t0
         edges += sum(int(b["num_edges"]) for b in blocks)
@@ -234,8 +235,10 @@ def run_dsp(args):
     torch.cuda.set_device(local)
     cfg, ip, ix, bnds, sip, six, feats, train = load_workload(args.config, rank, world)
     ex = pkg.torch_exchange() if world > 1 else None
+    biased = args.scheme == "biased"
+    ew = datagen.edge_weights(six, datagen.node_weights(cfg.num_nodes)) if biased else None
     s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, cfg.batch, rank=rank, world_size=world,
-                    device=local, exchange=ex, n_slots=2)
+                    device=local, exchange=ex, n_slots=2, edge_weights=ew)
     L = len(cfg.fanouts)
     steps_epoch = datagen.steps_per_epoch(train, bnds, cfg.batch)
     batches = datagen.rank_seed_batches(train, bnds, rank, cfg.batch, 0)[:steps_epoch]
@@ -254,7 +257,7 @@ def run_dsp(args):
         if ev is not None:
             ev[0].record(stream)
         s.sample_gather(dev_batches[i % len(batches)], datagen.BASE_SEED + i, slot=i % 2,
-                        sizes_out=h_sizes[i], async_=True, pipelined=pipelined)
+                        sizes_out=h_sizes[i], async_=True, pipelined=pipelined, biased=biased)
         if ev is not None:
             ev[1].record(stream)
 
@@ -308,7 +311,7 @@ def run_dsp(args):
             i = W + j
             a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a0.record(stream)
-            blocks = s.sample(dev_batches[i % len(batches)], datagen.BASE_SEED + i)
+            blocks = s.sample(dev_batches[i % len(batches)], datagen.BASE_SEED + i, biased=biased)
             a1.record(stream)
             ids_dev = blocks[-1].src_ids
             g_ev[j][0].record(stream)
@@ -342,7 +345,7 @@ def run_dsp(args):
         i = W + j
         d_seed.copy_(h_seeds[i % len(batches)], non_blocking=True)
         h2d += d_seed.numel() * 4
-        blocks, feat = s.sample_gather(d_seed, datagen.BASE_SEED + i, slot=0)
+        blocks, feat = s.sample_gather(d_seed, datagen.BASE_SEED + i, slot=0, biased=biased)
         for b, hb in zip(blocks, h_blk):
             hb[0][: b.num_dst + 1].copy_(b.indptr, non_blocking=True)
             hb[1][: b.num_edges].copy_(b.indices, non_blocking=True)
@@ -358,7 +361,7 @@ def run_dsp(args):
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(cfg, ip, ix, feats, batches, args.cpu_seconds)
+        cpu = cpu_baseline(cfg, ip, ix, feats, batches, args.cpu_seconds, weights=ew)
 
     kern_per_step = 1 if world == 1 else 5 * L + 1
     if rank == 0:
@@ -367,7 +370,8 @@ def run_dsp(args):
             "steps": K, "warmup": W, "ms_per_step": t_max / K,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32+f32",
             "data": "synthetic",
-            "config": {"workload": cfg.name if world == 1 else f"{cfg.name}-P{world}",
+            "config": {"workload": (cfg.name if world == 1 else f"{cfg.name}-P{world}")
+                       + ("-biased" if biased else ""), "scheme": args.scheme,
                        "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes,
                        "nnz": int(ip[-1]), "dim": cfg.dim, "parallelism": f"csp{world}",
                        "l2": "inputs larger than L2 (CSR 0.5 GB + features 1.1 GB >> 126 MB L2)",
@@ -411,6 +415,8 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-breakdown", action="store_true")
     ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
+    ap.add_argument("--scheme", choices=["uniform", "biased"], default="uniform",
+                    help="node-wise scheme (Table 2 IsBiased); biased uses synthetic node weights")
     args = ap.parse_args(argv)
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

@@ -103,6 +103,15 @@ void dsp_destroy(dsp_ctx *ctx);
 dsp_status dsp_load_partition(dsp_ctx *ctx, const int64_t *bounds, const int64_t *indptr,
                               const int32_t *indices, const float *features, int32_t dim);
 
+/* Edge weights for biased sampling (Sec. 4.2: "each node u ... is
+   associated with a non-negative weight w_u ... DSP stores node weight w_u
+   along with edge e_{v,u}").  edge_weights: host or device fp32[nnz_r]
+   aligned with this rank's `indices` (the weight of the edge's neighbour);
+   each must lie in [0, 65536) (else DSP_ERR_INVALID_ARG) and is used as the
+   16.16 fixed-point integer floor(w * 65536) (R24).  Once per ctx,
+   after dsp_load_partition.  Copied; the caller may free its buffer. */
+dsp_status dsp_load_weights(dsp_ctx *ctx, const float *edge_weights);
+
 /* Sizes the library's peer-visible exchange buffers for batches of up to
    max_seeds seeds per rank and the given fan-outs (fanouts: HOST
    int32[num_layers], 1 <= fanouts[l] <= 32, 1 <= num_layers <= 8).
@@ -118,6 +127,15 @@ dsp_status dsp_export_handle(const dsp_ctx *ctx, void *out);
 dsp_status dsp_import_handles(dsp_ctx *ctx, const void *all);
 
 /* ------------------------------------------------------------- sampling */
+
+/* Flags.  DSP_BIASED (dsp_sample, dsp_sample_group, dsp_sample_gather):
+   biased node-wise sampling with the weights of dsp_load_weights (
+   Table 2 `IsBiased`): k successive draws without replacement, each
+   neighbour with probability weight / total weight of the not-yet-drawn ones
+   (R24-R26); ranks must agree (checked in the exchange header). */
+#define DSP_ASYNC 1u
+#define DSP_PIPELINED 2u
+#define DSP_BIASED 4u
 
 typedef struct {
   /* one sampled layer ("block"); arrays are DEVICE memory owned by the CALLER */
@@ -149,6 +167,7 @@ dsp_status dsp_sample_bounds(const dsp_ctx *ctx, int32_t num_seeds, const int32_
               cover dsp_sample_bounds (else DSP_ERR_CAPACITY before any work).
               blocks[l].src_ids is the frontier of layer l+1; the last block's
               src_ids are the unique nodes whose features the loader needs.
+   flags    : 0 or DSP_BIASED.
    workspace: DEVICE, 256-byte aligned, >= workspace_bytes from
               dsp_sample_bounds, ZERO-FILLED before its first use; afterwards
               it belongs to the library (it carries the relabel map's epoch
@@ -161,7 +180,7 @@ dsp_status dsp_sample_bounds(const dsp_ctx *ctx, int32_t num_seeds, const int32_
    block contents are unspecified. */
 dsp_status dsp_sample(dsp_ctx *ctx, const int32_t *seeds, int32_t num_seeds, const int32_t *fanouts,
                       int32_t num_layers, uint64_t rng_seed, dsp_block *blocks, void *workspace,
-                      size_t workspace_bytes, void *stream);
+                      size_t workspace_bytes, uint32_t flags, void *stream);
 
 /* The same collective for n_ctx ctxs of one world driven by ONE host thread
    (virtual ranks sharing a device, or one process owning several GPUs).
@@ -171,11 +190,8 @@ dsp_status dsp_sample(dsp_ctx *ctx, const int32_t *seeds, int32_t num_seeds, con
 dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *seeds,
                             const int32_t *num_seeds, const int32_t *fanouts, int32_t num_layers,
                             uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
-                            size_t workspace_bytes, void *const *streams);
+                            size_t workspace_bytes, uint32_t flags, void *const *streams);
 
-/* Flags for dsp_sample_gather. */
-#define DSP_ASYNC 1u
-#define DSP_PIPELINED 2u
 
 /* One whole step of the hot path in ONE stream-ordered call: dsp_sample
    followed by the feature gather of the last block's src_ids (the loader

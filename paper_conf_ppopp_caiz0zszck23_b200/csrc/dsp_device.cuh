@@ -245,4 +245,95 @@ __device__ __forceinline__ void sample_node(bool ok, int32_t v, int64_t row_star
   *u = *valid ? __ldg(indices + row_start + chosen) : -1;
 }
 
+// -------------------------------------------------- one node's biased sample
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long x) {
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) x += __shfl_xor_sync(FULL_MASK, x, off);
+  return x;
+}
+__device__ __forceinline__ unsigned long long warp_incl_scan_u64(unsigned long long x) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int off = 1; off < 32; off <<= 1) {
+    const unsigned long long y = __shfl_up_sync(FULL_MASK, x, off);
+    if (lane >= off) x += y;
+  }
+  return x;
+}
+
+// Biased sample of node v by a whole warp (R24-R26): with
+// a[p] the 16.16 fixed-point weight of row position p, successive sampling
+// without replacement: k times, r = mulhi(Philox{t, v, l, "DSPB"}, W) with W
+// the total weight of the positions not yet picked, and the pick is the first
+// position (row order) whose running weight exceeds r.  When at most k
+// positions have a positive weight they are all taken, no draw.  Lane t < cnt
+// returns the t-th position in ascending row order in *pos.  Warp-uniform.
+__device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t row_start, int64_t deg, int k,
+                                                  int layer, uint2 key, const uint32_t *__restrict__ w,
+                                                  uint32_t *pos) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t lt = (1u << lane) - 1u;
+  if (!ok) return 0;
+  const uint32_t *a = w + row_start;
+  const int d = (int)deg;
+  int npos = 0;
+  for (int c0 = 0; c0 < d; c0 += 32) npos += __popc(__ballot_sync(FULL_MASK, c0 + lane < d && a[c0 + lane] > 0u));
+  if (npos <= k) {  // every positive-weight position, in row order
+    int base = 0;
+    uint32_t mine = 0xffffffffu;
+    for (int c0 = 0; c0 < d; c0 += 32) {
+      const bool f = c0 + lane < d && a[c0 + lane] > 0u;
+      const uint32_t b = __ballot_sync(FULL_MASK, f);
+      // lane t takes the position whose rank among the positive ones is t
+      const int want = lane - base;
+      if (want >= 0 && want < __popc(b)) mine = c0 + (__fns(b, 0, want + 1));
+      base += __popc(b);
+    }
+    *pos = mine;
+    return npos;
+  }
+  uint32_t pick = 0xffffffffu;  // lane t: pick of round t
+  for (int t = 0; t < k; ++t) {
+    // total weight of the positions not picked yet
+    unsigned long long part = 0;
+    for (int c0 = 0; c0 < d; c0 += 32) {
+      const int p = c0 + lane;
+      if (p < d) {
+        bool taken = false;
+        for (int j = 0; j < t; ++j) taken |= __shfl_sync(FULL_MASK, pick, j) == (uint32_t)p;
+        if (!taken) part += a[p];
+      } else {
+        for (int j = 0; j < t; ++j) (void)__shfl_sync(FULL_MASK, pick, j);
+      }
+    }
+    const unsigned long long W = warp_sum_u64(part);
+    const uint4 x = philox4x32_10(make_uint4((uint32_t)t, (uint32_t)v, (uint32_t)layer, 0x44535042u), key);
+    const unsigned long long r = __umul64hi(((unsigned long long)x.y << 32) | x.x, W);
+    unsigned long long acc = 0;
+    uint32_t found = 0xffffffffu;
+    for (int c0 = 0; c0 < d && found == 0xffffffffu; c0 += 32) {
+      const int p = c0 + lane;
+      bool taken = p >= d;
+      for (int j = 0; j < t; ++j) taken |= __shfl_sync(FULL_MASK, pick, j) == (uint32_t)p;
+      const unsigned long long val = taken ? 0ull : (unsigned long long)a[p];
+      const unsigned long long incl = warp_incl_scan_u64(val);
+      const uint32_t cross = __ballot_sync(FULL_MASK, acc + incl > r);
+      if (cross) found = (uint32_t)(c0 + __ffs(cross) - 1);
+      acc += __shfl_sync(FULL_MASK, incl, 31);
+    }
+    if (lane == t) pick = found;
+  }
+  // ascending row order: lane t takes the pick of rank t
+  uint32_t mine = 0xffffffffu;
+  for (int s2 = 0; s2 < k; ++s2) {
+    const uint32_t c = __shfl_sync(FULL_MASK, pick, s2);
+    int rank = 0;
+    for (int j = 0; j < k; ++j) rank += __shfl_sync(FULL_MASK, pick, j) < c ? 1 : 0;
+    if (rank == lane) mine = c;
+  }
+  (void)lt;
+  *pos = mine;
+  return k;
+}
+
 }  // namespace dsp

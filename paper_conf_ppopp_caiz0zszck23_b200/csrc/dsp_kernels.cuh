@@ -325,6 +325,48 @@ __device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F,
   }
 }
 
+// Biased sampling: one warp per node, sample_node_biased; the
+// sampled neighbours come out in ascending row order (slot = lane).
+template <int TEAM = PNT>
+__device__ __forceinline__ void phase_sample_biased(const int32_t *frontier, int F, int layer, int k, uint2 key,
+                                                    const int64_t *__restrict__ indptr,
+                                                    const int32_t *__restrict__ indices,
+                                                    const uint32_t *__restrict__ weights, int64_t lo,
+                                                    int64_t n_local, const LayerBufs &B, uint32_t epoch,
+                                                    int32_t *src_out, int *err) {
+  const int lane = threadIdx.x & 31;
+  const Span sp = block_span<TEAM>(F);
+  const int64_t b0 = sp.first - threadIdx.x;
+  const int wib = threadIdx.x >> 5, wpb = TEAM >> 5;
+  for (int64_t i64 = b0 + wib; i64 < sp.end; i64 += wpb) {
+    const int i = (int)i64;
+    const int32_t v = ldw_i32(frontier + i);
+    const int64_t lv = (int64_t)v - lo;
+    const bool ok = v >= 0 && lv >= 0 && lv < n_local;
+    int64_t s = 0, d = 0;
+    if (ok) {
+      s = __ldg(indptr + lv);
+      d = __ldg(indptr + lv + 1) - s;
+    }
+    uint32_t pos;
+    const int cnt = sample_node_biased(ok, v, s, d, k, layer, key, weights, &pos);
+    if (lane == 0) {
+      B.cnt[i] = cnt;
+      if (src_out) src_out[i] = v;
+      if (ok)
+        mark_dst(B.first, v, i, F, layer, epoch, err);
+      else
+        latch(err, E_RANGE);
+    }
+    if (lane < cnt) {
+      const int32_t u = __ldg(indices + s + pos);
+      const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)lane;
+      B.rows[q] = u;
+      mark(B.first, u, epoch, (uint32_t)F + q);
+    }
+  }
+}
+
 // ------------------------------------------- scan, two-phase (persistent)
 // Inside the persistent kernel every block is resident, so the scan over
 // edge slots is a static partition: pass 1 computes each item's flags, the
@@ -598,6 +640,8 @@ struct PersistArgs {
   uint2 key;
   const int64_t *indptr;
   const int32_t *indices;
+  const uint32_t *weights;  // 16.16 edge weights (biased sampling) or nullptr
+  int32_t biased;
   int64_t lo, n_local;
   Outputs out;
   LayerBufs buf[2];
@@ -620,7 +664,10 @@ __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32
                                                uint32_t epoch) {
   const int k = a.k[l];
   const LayerBufs &B = a.buf[l & 1];
-  if (k <= 8) {
+  if (a.biased) {
+    phase_sample_biased<TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.weights, a.lo, a.n_local, B, epoch,
+                              a.out.src_ids[l], a.err);
+  } else if (k <= 8) {
     phase_sample_tpn<8, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
                               a.out.src_ids[l], a.err, a.hdr);
   } else if (k <= 16) {
@@ -951,7 +998,7 @@ __device__ __forceinline__ int frontier_size(const WsHeader *hdr, int layer, int
 
 struct BucketArgs {
   const int32_t *frontier;
-  int32_t F0, layer, k;
+  int32_t F0, layer, k, biased;
   uint32_t seed_lo, seed_hi;
   int32_t rank, parity;
   unsigned long long seq;
@@ -1011,7 +1058,7 @@ __global__ void __launch_bounds__(NT) k_bucket_scatter(BucketArgs a) {
       const uint32_t c = *(volatile uint32_t *)&a.hdr->bucket[o];
       a.hdr->bucket[o] = 0u;
       *xch_inbox_hdr(a.peers.base[o], a.L, a.parity, a.rank) =
-          make_uint4(c, (uint32_t)a.k | ((uint32_t)a.layer << 8), a.seed_lo, a.seed_hi);
+          make_uint4(c, (uint32_t)a.k | ((uint32_t)a.layer << 8) | ((uint32_t)a.biased << 16), a.seed_lo, a.seed_hi);
     }
     __threadfence_system();
     for (int o = 0; o < a.bd.world; ++o)
@@ -1021,6 +1068,8 @@ __global__ void __launch_bounds__(NT) k_bucket_scatter(BucketArgs a) {
 
 struct RemoteSampleArgs {
   int32_t layer, k;
+  int32_t biased;
+  const uint32_t *weights;
   uint2 key;
   int32_t rank, parity;
   unsigned long long seq;
@@ -1047,7 +1096,8 @@ __global__ void __launch_bounds__(NT) k_sample_remote(RemoteSampleArgs a) {
       uint32_t acc = 0;
       for (int s = 0; s < world; ++s) {
         const uint4 h = __ldcv(xch_inbox_hdr(self, a.L, a.parity, s));
-        if (h.y != ((uint32_t)a.k | ((uint32_t)a.layer << 8)) || h.z != a.key.x || h.w != a.key.y)
+        if (h.y != ((uint32_t)a.k | ((uint32_t)a.layer << 8) | ((uint32_t)a.biased << 16)) || h.z != a.key.x ||
+            h.w != a.key.y)
           latch(a.err, E_STATE);
         s_off[s] = acc;
         acc += (h.x <= (uint32_t)a.L.cap) ? h.x : 0u;
@@ -1081,7 +1131,15 @@ __global__ void __launch_bounds__(NT) k_sample_remote(RemoteSampleArgs a) {
       bool valid;
       int slot, cnt;
       int32_t u;
-      sample_node<G>(ok, v, rs, d, k, a.layer, a.key, a.indices, &valid, &slot, &u, &cnt);
+      if (G == 32 && a.biased) {
+        uint32_t pos;
+        cnt = sample_node_biased(ok, v, rs, d, k, a.layer, a.key, a.weights, &pos);
+        slot = lane;
+        valid = lane < cnt;
+        u = valid ? __ldg(a.indices + rs + pos) : -1;
+      } else {
+        sample_node<G>(ok, v, rs, d, k, a.layer, a.key, a.indices, &valid, &slot, &u, &cnt);
+      }
       char *req = a.peers.base[s];
       if (active && (lane & (G - 1)) == 0) xch_ret_cnt(req, a.L, a.parity, a.rank)[j] = cnt;
       if (valid) xch_ret_rows(req, a.L, a.parity, a.rank)[(int64_t)j * a.L.kmax + slot] = u;
@@ -1301,6 +1359,20 @@ __global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
 __global__ void __launch_bounds__(NT) k_write_indices(ScanArgs a) {
   const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
   phase_indices(F, a.k, a.buf, a.indptr_out, a.indices_out, grid_span((int64_t)F * a.k));
+}
+
+// fp32 edge weights -> 16.16 fixed point a = floor(w * 2^16), w in [0, 2^16)
+// (R24); an invalid weight is counted in *bad.
+__global__ void k_weights_fixed(const float *w, int64_t n, uint32_t *out, int *bad) {
+  for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
+    const float x = w[e];
+    if (!(x >= 0.0f) || x >= 65536.0f) {
+      atomicAdd(bad, 1);
+      out[e] = 0;
+    } else {
+      out[e] = (uint32_t)floorf(x * 65536.0f);
+    }
+  }
 }
 
 // end of a stage-by-stage call: advance the workspace epoch

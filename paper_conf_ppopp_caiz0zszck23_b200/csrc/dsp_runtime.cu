@@ -103,6 +103,7 @@ struct dsp_ctx {
   int32_t dim = 0, feat_stride = 0;  // feature row length / padded stride (floats)
   int64_t *d_indptr = nullptr;
   int32_t *d_indices = nullptr;
+  uint32_t *d_weights = nullptr;  // 16.16 edge weights (biased sampling)
   float *d_feat = nullptr;
   int64_t feat_bytes = 0;
   int *d_err = nullptr;  // latched device error of this ctx
@@ -283,6 +284,7 @@ struct Call {
   int64_t *sizes_out;  // async sizes destination (or nullptr)
   bool async;
   bool pipelined;      // gather this call's rows in the next pipelined call / flush
+  bool biased;         // DSP_BIASED
 };
 
 LayerBufs bufs_of(const Call &k, int parity) {
@@ -298,11 +300,15 @@ WsPersist *persist_of(const Call &k) { return reinterpret_cast<WsPersist *>(k.ws
 
 dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_seeds,
                         const int32_t *fanouts, int32_t L, uint64_t rng_seed, dsp_block *blocks,
-                        void *workspace, size_t ws_bytes, void *stream) {
+                        void *workspace, size_t ws_bytes, uint32_t flags, void *stream) {
   k = Call{};
   k.c = c;
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
+  if ((flags & ~(DSP_ASYNC | DSP_PIPELINED | DSP_BIASED)) != 0)
+    return fail(c, DSP_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
+  k.biased = (flags & DSP_BIASED) != 0;
+  if (k.biased && !c->d_weights) return fail(c, DSP_ERR_STATE, "DSP_BIASED needs dsp_load_weights first");
   if (c->broken) return fail(c, DSP_ERR_STATE, "ctx unusable after an earlier exchange failure");
   if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition not called");
   if (c->world > 1 && (!c->reserved || !c->imported))
@@ -382,6 +388,8 @@ dsp_status stage_persistent(Call &k) {
   a.key = key_of(k.rng_seed);
   a.indptr = c->d_indptr;
   a.indices = c->d_indices;
+  a.weights = c->d_weights;
+  a.biased = k.biased ? 1 : 0;
   a.lo = c->lo;
   a.n_local = c->n_local;
   a.buf[0] = bufs_of(k, 0);
@@ -464,6 +472,7 @@ dsp_status stage_shuffle(Call &k, int l) {
   a.F0 = k.num_seeds;
   a.layer = l;
   a.k = k.fanouts[l];
+  a.biased = k.biased ? 1 : 0;
   a.seed_lo = (uint32_t)k.rng_seed;
   a.seed_hi = (uint32_t)(k.rng_seed >> 32);
   a.rank = c->rank;
@@ -487,6 +496,8 @@ dsp_status stage_sample_remote(Call &k, int l) {
   RemoteSampleArgs a{};
   a.layer = l;
   a.k = k.fanouts[l];
+  a.biased = k.biased ? 1 : 0;
+  a.weights = c->d_weights;
   a.key = key_of(k.rng_seed);
   a.rank = c->rank;
   a.seq = k.seq0 + 1 + l;
@@ -500,7 +511,7 @@ dsp_status stage_sample_remote(Call &k, int l) {
   a.peers = peers_of(c);
   a.hdr = k.hdr;
   a.err = c->d_err;
-  DISPATCH_G(group_of(a.k), launch_remote, a, grid_for(c, 8), k.stream);
+  DISPATCH_G(k.biased ? 32 : group_of(a.k), launch_remote, a, grid_for(c, 8), k.stream);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
 }
@@ -659,6 +670,7 @@ void release(dsp_ctx *c) {
     }
   cudaFree(c->d_indptr);
   cudaFree(c->d_indices);
+  cudaFree(c->d_weights);
   cudaFree(c->d_feat);
   cudaFree(c->d_xch);
   cudaFree(c->d_err);
@@ -812,6 +824,43 @@ dsp_status dsp_load_partition(dsp_ctx *c, const int64_t *bounds, const int64_t *
   return DSP_OK;
 }
 
+dsp_status dsp_load_weights(dsp_ctx *c, const float *edge_weights) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
+  if (c->d_weights) return fail(c, DSP_ERR_STATE, "weights already loaded");
+  if (!edge_weights && c->nnz > 0) return fail(c, DSP_ERR_INVALID_ARG, "edge_weights is NULL");
+  DeviceGuard g(c->device);
+  const size_t n = (size_t)std::max<int64_t>(1, c->nnz);
+  CUDA_TRY(c, cudaMalloc(&c->d_weights, sizeof(uint32_t) * n));
+  if (c->nnz > 0) {
+    float *tmp = nullptr;
+    CUDA_TRY(c, cudaMalloc(&tmp, sizeof(float) * n));
+    cudaError_t e = cudaMemcpy(tmp, edge_weights, sizeof(float) * (size_t)c->nnz, cudaMemcpyDefault);
+    if (e == cudaSuccess) e = cudaMemset(c->d_err, 0, sizeof(int));
+    if (e == cudaSuccess) {
+      k_weights_fixed<<<c->num_sms * 8, 256>>>(tmp, c->nnz, c->d_weights, c->d_err);
+      e = cudaGetLastError();
+    }
+    int bad = 0;
+    if (e == cudaSuccess) e = cudaMemcpy(&bad, c->d_err, sizeof(int), cudaMemcpyDeviceToHost);
+    cudaFree(tmp);
+    cudaMemset(c->d_err, 0, sizeof(int));
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      cudaFree(c->d_weights);
+      c->d_weights = nullptr;
+      return fail(c, DSP_ERR_CUDA, "dsp_load_weights: %s", cudaGetErrorString(e));
+    }
+    if (bad) {
+      cudaFree(c->d_weights);
+      c->d_weights = nullptr;
+      return fail(c, DSP_ERR_INVALID_ARG, "%d edge weights outside [0, 65536)", bad);
+    }
+  }
+  return DSP_OK;
+}
+
 dsp_status dsp_reserve(dsp_ctx *c, int32_t max_seeds, const int32_t *fanouts, int32_t L) {
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
@@ -957,10 +1006,12 @@ dsp_status dsp_sample_bounds(const dsp_ctx *cc, int32_t num_seeds, const int32_t
 
 dsp_status dsp_sample(dsp_ctx *c, const int32_t *seeds, int32_t num_seeds, const int32_t *fanouts,
                       int32_t L, uint64_t rng_seed, dsp_block *blocks, void *workspace,
-                      size_t workspace_bytes, void *stream) {
+                      size_t workspace_bytes, uint32_t flags, void *stream) {
   std::vector<Call> calls(1);
+  if ((flags & (DSP_ASYNC | DSP_PIPELINED)) != 0)
+    return fail(c, DSP_ERR_INVALID_ARG, "dsp_sample takes DSP_BIASED only (async steps: dsp_sample_gather)");
   dsp_status st = prepare_call(calls[0], c, seeds, num_seeds, fanouts, L, rng_seed, blocks, workspace,
-                               workspace_bytes, stream);
+                               workspace_bytes, flags, stream);
   if (st != DSP_OK) return st;
   return run_calls(calls);
 }
@@ -971,9 +1022,8 @@ dsp_status dsp_sample_gather(dsp_ctx *c, const int32_t *seeds, int32_t num_seeds
                              int64_t *sizes_out, uint32_t flags, void *stream) {
   std::vector<Call> calls(1);
   dsp_status st = prepare_call(calls[0], c, seeds, num_seeds, fanouts, L, rng_seed, blocks, workspace,
-                               workspace_bytes, stream);
+                               workspace_bytes, flags, stream);
   if (st != DSP_OK) return st;
-  if ((flags & ~(DSP_ASYNC | DSP_PIPELINED)) != 0) return fail(c, DSP_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
   if (!feat_out) return fail(c, DSP_ERR_INVALID_ARG, "feat_out is NULL");
   if ((st = check_gather_out(c, feat_out)) != DSP_OK) return st;
   if (c->world > 1 && !c->imported) return fail(c, DSP_ERR_STATE, "dsp_import_handles first");
@@ -998,7 +1048,7 @@ dsp_status dsp_pipeline_flush(dsp_ctx *c, void *stream) {
 dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n, const int32_t *const *seeds,
                             const int32_t *num_seeds, const int32_t *fanouts, int32_t L,
                             uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
-                            size_t workspace_bytes, void *const *streams) {
+                            size_t workspace_bytes, uint32_t flags, void *const *streams) {
   if (!ctxs || n < 1 || !seeds || !num_seeds || !blocks || !workspaces || !streams)
     return DSP_ERR_INVALID_ARG;
   const int world = ctxs[0] ? ctxs[0]->world : 0;
@@ -1014,8 +1064,10 @@ dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n, const int32_t *cons
   }
   std::vector<Call> calls(n);
   for (int i = 0; i < n; ++i) {
+    if ((flags & (DSP_ASYNC | DSP_PIPELINED)) != 0)
+      return fail(ctxs[0], DSP_ERR_INVALID_ARG, "dsp_sample_group takes DSP_BIASED only");
     dsp_status st = prepare_call(calls[i], ctxs[i], seeds[i], num_seeds[i], fanouts, L, rng_seed,
-                                 blocks[i], workspaces[i], workspace_bytes, streams[i]);
+                                 blocks[i], workspaces[i], workspace_bytes, flags, streams[i]);
     if (st != DSP_OK) return st;
   }
   return run_calls(calls);

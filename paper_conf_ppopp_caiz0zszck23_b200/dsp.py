@@ -32,11 +32,12 @@ DSP_HANDLE_BYTES = 512
 
 #: every symbol include/dsp.h declares
 ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_create", "dsp_destroy",
-               "dsp_load_partition", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
+               "dsp_load_partition", "dsp_load_weights", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
                "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                "dsp_pipeline_flush", "dsp_gather_features", "dsp_sync")
 DSP_ASYNC = 1
 DSP_PIPELINED = 2
+DSP_BIASED = 4
 
 
 class DSPError(RuntimeError):
@@ -75,17 +76,19 @@ def lib(path: str | None = None):
         L.dsp_destroy.restype = None
         L.dsp_load_partition.argtypes = [P, P, P, P, P, i32]
         L.dsp_reserve.argtypes = [P, i32, P, i32]
+        L.dsp_load_weights.argtypes = [P, P]
         L.dsp_export_handle.argtypes = [P, P]
         L.dsp_import_handles.argtypes = [P, P]
         L.dsp_sample_bounds.argtypes = [P, i32, P, i32, P, P, ctypes.POINTER(ctypes.c_size_t)]
-        L.dsp_sample.argtypes = [P, P, i32, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t, P]
+        L.dsp_sample.argtypes = [P, P, i32, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t, ctypes.c_uint32, P]
         L.dsp_sample_gather.argtypes = [P, P, i32, P, i32, ctypes.c_uint64, P, P, i64, P, ctypes.c_size_t, P,
                                          ctypes.c_uint32, P]
-        L.dsp_sample_group.argtypes = [P, i32, P, P, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t, P]
+        L.dsp_sample_group.argtypes = [P, i32, P, P, P, i32, ctypes.c_uint64, P, P, ctypes.c_size_t,
+                                        ctypes.c_uint32, P]
         L.dsp_gather_features.argtypes = [P, P, i64, P, P]
         L.dsp_pipeline_flush.argtypes = [P, P]
         L.dsp_sync.argtypes = [P, P]
-        for name in ("dsp_create", "dsp_load_partition", "dsp_reserve", "dsp_export_handle",
+        for name in ("dsp_create", "dsp_load_partition", "dsp_load_weights", "dsp_reserve", "dsp_export_handle",
                      "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                      "dsp_pipeline_flush",
                      "dsp_gather_features", "dsp_sync"):
@@ -151,6 +154,10 @@ def dsp_load_partition(ctx, bounds, indptr, indices, features, dim: int) -> None
     _check(lib().dsp_load_partition(ctx, _p(b), _p(indptr), _p(indices), _p(features), dim), ctx)
 
 
+def dsp_load_weights(ctx, edge_weights) -> None:
+    _check(lib().dsp_load_weights(ctx, _p(edge_weights)), ctx)
+
+
 def dsp_reserve(ctx, max_seeds: int, fanouts) -> None:
     f = _i32_array(fanouts)
     _check(lib().dsp_reserve(ctx, max_seeds, _p(f), len(f)), ctx)
@@ -178,10 +185,10 @@ def dsp_sample_bounds(ctx, num_seeds: int, fanouts):
 
 
 def dsp_sample(ctx, seeds, num_seeds: int, fanouts, rng_seed: int, blocks, workspace,
-               workspace_bytes: int, stream: int) -> None:
+               workspace_bytes: int, flags: int, stream: int) -> None:
     f = _i32_array(fanouts)
     _check(lib().dsp_sample(ctx, _p(seeds), num_seeds, _p(f), len(f), ctypes.c_uint64(rng_seed),
-                            blocks, _p(workspace), workspace_bytes, ctypes.c_void_p(stream)), ctx)
+                            blocks, _p(workspace), workspace_bytes, flags, ctypes.c_void_p(stream)), ctx)
 
 
 def dsp_sample_gather(ctx, seeds, num_seeds: int, fanouts, rng_seed: int, blocks, feat_out, feat_cap_rows: int,
@@ -193,7 +200,7 @@ def dsp_sample_gather(ctx, seeds, num_seeds: int, fanouts, rng_seed: int, blocks
 
 
 def dsp_sample_group(ctxs, seeds, num_seeds, fanouts, rng_seed: int, blocks, workspaces,
-                     workspace_bytes: int, streams) -> None:
+                     workspace_bytes: int, flags: int, streams) -> None:
     n = len(ctxs)
     f = _i32_array(fanouts)
     c_ctxs = (ctypes.c_void_p * n)(*[c.value for c in ctxs])
@@ -203,7 +210,7 @@ def dsp_sample_group(ctxs, seeds, num_seeds, fanouts, rng_seed: int, blocks, wor
     c_ws = (ctypes.c_void_p * n)(*[_p(w).value for w in workspaces])
     c_st = (ctypes.c_void_p * n)(*streams)
     _check(lib().dsp_sample_group(c_ctxs, n, c_seeds, c_ns, _p(f), len(f), ctypes.c_uint64(rng_seed),
-                                  c_blocks, c_ws, workspace_bytes, c_st), ctxs[0])
+                                  c_blocks, c_ws, workspace_bytes, flags, c_st), ctxs[0])
 
 
 def dsp_pipeline_flush(ctx, stream: int) -> None:
@@ -238,7 +245,8 @@ class Sampler:
 
     def __init__(self, bounds, indptr, indices, features, fanouts, max_seeds: int, rank: int = 0,
                  world_size: int = 1, device: int | None = None,
-                 exchange: Callable[[bytes], list] | None = None, connect: bool = True, n_slots: int = 1):
+                 exchange: Callable[[bytes], list] | None = None, connect: bool = True, n_slots: int = 1,
+                 edge_weights=None):
         import torch
         self.torch = torch
         self.device = torch.cuda.current_device() if device is None else device
@@ -249,10 +257,14 @@ class Sampler:
         self.ctx = dsp_create(rank, world_size, self.device)
         try:
             dsp_load_partition(self.ctx, bounds, indptr, indices, features, self.dim)
+            if edge_weights is not None:
+                dsp_load_weights(self.ctx, np.ascontiguousarray(edge_weights, np.float32)
+                                 if isinstance(edge_weights, np.ndarray) else edge_weights)
             dsp_reserve(self.ctx, self.max_seeds, self.fanouts)
             ms, me, ws = dsp_sample_bounds(self.ctx, self.max_seeds, self.fanouts)
         except Exception:
             dsp_destroy(self.ctx)
+            self.ctx = None
             raise
         dev = torch.device("cuda", self.device)
         self.workspace_bytes = ws
@@ -285,15 +297,15 @@ class Sampler:
     def stream(self) -> int:
         return self.torch.cuda.current_stream(self.device).cuda_stream
 
-    def sample(self, seeds, rng_seed: int) -> list[Block]:
+    def sample(self, seeds, rng_seed: int, biased: bool = False) -> list[Block]:
         torch = self.torch
         assert seeds.dtype == torch.int32 and seeds.is_cuda and seeds.is_contiguous()
         dsp_sample(self.ctx, seeds, seeds.numel(), self.fanouts, rng_seed, self._cblocks, self.workspace,
-                   self.workspace_bytes, self.stream())
+                   self.workspace_bytes, DSP_BIASED if biased else 0, self.stream())
         return self.blocks()
 
     def sample_gather(self, seeds, rng_seed: int, slot: int = 0, sizes_out=None, async_: bool = False,
-                      pipelined: bool = False):
+                      pipelined: bool = False, biased: bool = False):
         """One whole step (sample + gather) in one call into output set `slot`.
         Synchronous: returns (blocks, features view).  async_: returns None;
         sizes land in sizes_out (pinned host / device int64[3L]) in stream order.
@@ -302,7 +314,7 @@ class Sampler:
         torch = self.torch
         assert seeds.dtype == torch.int32 and seeds.is_cuda and seeds.is_contiguous()
         feat_out = self.feat_buffer(slot)
-        flags = DSP_PIPELINED if pipelined else (DSP_ASYNC if async_ else 0)
+        flags = (DSP_PIPELINED if pipelined else (DSP_ASYNC if async_ else 0)) | (DSP_BIASED if biased else 0)
         dsp_sample_gather(self.ctx, seeds, seeds.numel(), self.fanouts, rng_seed, self._sets[slot][1], feat_out,
                           feat_out.shape[0], self.workspace, self.workspace_bytes, sizes_out, flags, self.stream())
         if async_ or pipelined:
@@ -374,10 +386,12 @@ class LocalGroup:
     GPUs of this node."""
 
     def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int]):
+        """shards[r] = (indptr, indices, features[, edge_weights]) of rank r."""
         P = len(shards)
         assert len(devices) == P and len(bounds) == P + 1
         self.samplers = [Sampler(bounds, s[0], s[1], s[2], fanouts, max_seeds, rank=r, world_size=P,
-                                 device=devices[r], connect=False) for r, s in enumerate(shards)]
+                                 device=devices[r], connect=False, edge_weights=s[3] if len(s) > 3 else None)
+                         for r, s in enumerate(shards)]
         handles = [dsp_export_handle(s.ctx) for s in self.samplers]
         for s in self.samplers:
             if P > 1:
@@ -385,11 +399,11 @@ class LocalGroup:
             s.connected = True
         self.fanouts = list(fanouts)
 
-    def sample(self, seeds_per_rank, rng_seed: int) -> list[list[Block]]:
+    def sample(self, seeds_per_rank, rng_seed: int, biased: bool = False) -> list[list[Block]]:
         S = self.samplers
         dsp_sample_group([s.ctx for s in S], seeds_per_rank, [x.numel() for x in seeds_per_rank],
                          self.fanouts, rng_seed, [s._cblocks for s in S], [s.workspace for s in S],
-                         S[0].workspace_bytes, [s.stream() for s in S])
+                         S[0].workspace_bytes, DSP_BIASED if biased else 0, [s.stream() for s in S])
         return [s.blocks() for s in S]
 
     def close(self):

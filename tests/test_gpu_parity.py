@@ -354,3 +354,59 @@ def test_products_pipelined(pkg, products):
     s.sync()
     _check_step(s, 0, sizes[2], batches[22], 42, ip, ix, feats_of)
     s.close()
+
+
+# ------------------------------------------------------------ biased
+
+@pytest.fixture(scope="module")
+def tiny_weights(tiny):
+    cfg, ip, ix, feats = tiny
+    return datagen.edge_weights(ix, datagen.node_weights(cfg.num_nodes))
+
+
+@pytest.mark.parametrize("fanouts", [(5, 5), (1, 32), (15, 10, 5)])
+def test_biased_tiny(pkg, tiny, tiny_weights, fanouts):
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, fanouts, 64, edge_weights=tiny_weights)
+    batches = seeds_of(cfg, 1, 0)
+    for step in range(6):
+        blocks = s.sample(torch.from_numpy(batches[step]).cuda(), 70 + step, biased=True)
+        ref = oracle.sample(ip, ix, batches[step], fanouts, 70 + step, weights=tiny_weights)
+        assert_blocks_equal(blocks, ref, f"biased step {step}")
+    blocks, feat = s.sample_gather(torch.from_numpy(batches[7]).cuda(), 5, biased=True)
+    ref = oracle.sample(ip, ix, batches[7], fanouts, 5, weights=tiny_weights)
+    assert_blocks_equal(blocks, ref, "biased fused")
+    assert np.array_equal(feat.cpu().numpy(), oracle.gather(feats, ref[-1]["src_ids"]))
+    s.close()
+
+
+@pytest.mark.parametrize("P", [2, 4])
+def test_biased_virtual_ranks(pkg, tiny, tiny_weights, P):
+    cfg, ip, ix, feats = tiny
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi], tiny_weights[ip[lo]:ip[hi]]))
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P)
+    seeds = [seeds_of(cfg, P, r, batch=32)[0] for r in range(P)]
+    res = grp.sample([torch.from_numpy(x).cuda() for x in seeds], 0xB1A5, biased=True)
+    for r in range(P):
+        assert_blocks_equal(res[r], oracle.sample(ip, ix, seeds[r], cfg.fanouts, 0xB1A5, weights=tiny_weights),
+                            f"biased P={P} rank {r}")
+    grp.close()
+
+
+def test_biased_errors(pkg, tiny):
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8)
+    with pytest.raises(pkg.DSPError) as e:   # no weights loaded
+        s.sample(torch.arange(4, dtype=torch.int32, device="cuda"), 1, biased=True)
+    assert e.value.status == pkg.dsp.DSP_ERR_STATE
+    s.close()
+    bad = np.ones(len(ix), np.float32)
+    bad[7] = -1.0
+    with pytest.raises(pkg.DSPError) as e:
+        pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8, edge_weights=bad)
+    assert e.value.status == pkg.dsp.DSP_ERR_INVALID_ARG
