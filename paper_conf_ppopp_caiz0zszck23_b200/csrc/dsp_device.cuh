@@ -268,23 +268,200 @@ __device__ __forceinline__ unsigned long long warp_incl_scan_u64(unsigned long l
 // position (row order) whose running weight exceeds r.  When at most k
 // positions have a positive weight they are all taken, no draw.  Lane t < cnt
 // returns the t-th position in ascending row order in *pos.  Warp-uniform.
+//
+// Rows of up to 32*BSEG positions keep their weights in registers, lane l
+// holding the contiguous segment [l*S, (l+1)*S): a round is one warp sum, one
+// warp scan of the lane totals and a scan inside the crossing lane's segment,
+// and the pick is removed by zeroing one register.  Longer rows re-read the
+// weights and test membership against the picks so far.
+constexpr int BSEG = 8;
+
+__device__ __forceinline__ uint32_t biased_sort_picks(uint32_t pick, int k) {
+  const int lane = threadIdx.x & 31;
+  uint32_t mine = 0xffffffffu;
+  for (int s2 = 0; s2 < k; ++s2) {
+    const uint32_t c = __shfl_sync(FULL_MASK, pick, s2);
+    int rank = 0;
+    for (int j = 0; j < k; ++j) rank += __shfl_sync(FULL_MASK, pick, j) < c ? 1 : 0;
+    if (rank == lane) mine = c;
+  }
+  return mine;
+}
+
+__device__ __forceinline__ unsigned long long biased_word(uint2 key, int t, int32_t v, int layer) {
+  const uint4 x = philox4x32_10(make_uint4((uint32_t)t, (uint32_t)v, (uint32_t)layer, 0x44535042u), key);
+  return ((unsigned long long)x.y << 32) | x.x;
+}
+
 __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t row_start, int64_t deg, int k,
                                                   int layer, uint2 key, const uint32_t *__restrict__ w,
                                                   uint32_t *pos) {
   const int lane = threadIdx.x & 31;
-  const uint32_t lt = (1u << lane) - 1u;
   if (!ok) return 0;
   const uint32_t *a = w + row_start;
   const int d = (int)deg;
+  if (d <= 32 * BSEG) {
+    // ------------------------------------------------ weights in registers
+    const int S = (d + 31) >> 5;
+    uint32_t reg[BSEG];
+    int mypos = 0;
+#pragma unroll
+    for (int j = 0; j < BSEG; ++j) {
+      const int p = lane * S + j;
+      reg[j] = (j < S && p < d) ? __ldg(a + p) : 0u;
+      mypos += reg[j] > 0u ? 1 : 0;
+    }
+    int npos = mypos;
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) npos += __shfl_xor_sync(FULL_MASK, npos, off);
+    if (npos <= k) {  // every positive-weight position, in row order
+      int excl = mypos;
+#pragma unroll
+      for (int off = 1; off < 32; off <<= 1) {
+        const int y = __shfl_up_sync(FULL_MASK, excl, off);
+        if (lane >= off) excl += y;
+      }
+      excl -= mypos;
+      uint32_t mine = 0xffffffffu;
+      // lane t needs the position of rank t: owner lanes hand it over one rank at a time
+      for (int t = 0; t < npos; ++t) {
+        const bool own = t >= excl && t < excl + mypos;
+        uint32_t cand = 0;
+        if (own) {
+          int r = excl;
+#pragma unroll
+          for (int j = 0; j < BSEG; ++j)
+            if (reg[j] > 0u) {
+              if (r == t) cand = (uint32_t)(lane * S + j);
+              ++r;
+            }
+        }
+        const uint32_t b = __ballot_sync(FULL_MASK, own);
+        const uint32_t got = __shfl_sync(FULL_MASK, cand, __ffs(b) - 1);
+        if (lane == t) mine = got;
+      }
+      *pos = mine;
+      return npos;
+    }
+    uint32_t pick = 0xffffffffu;
+    const unsigned long long myword = lane < k ? biased_word(key, lane, v, layer) : 0ull;  // all draws at once
+    for (int t = 0; t < k; ++t) {
+      unsigned long long tot = 0;
+#pragma unroll
+      for (int j = 0; j < BSEG; ++j) tot += reg[j];
+      const unsigned long long incl = warp_incl_scan_u64(tot);
+      const unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
+      const unsigned long long r = __umul64hi(__shfl_sync(FULL_MASK, myword, t), W);
+      const uint32_t cross = __ballot_sync(FULL_MASK, incl > r);
+      const int L = __ffs(cross) - 1;
+      uint32_t found = 0;
+      if (lane == L) {
+        unsigned long long acc = incl - tot;
+        bool done = false;
+#pragma unroll
+        for (int j = 0; j < BSEG; ++j) {
+          if (!done && acc + reg[j] > r) {
+            found = (uint32_t)(lane * S + j);
+            reg[j] = 0u;  // remove the pick
+            done = true;
+          }
+          acc += reg[j];
+        }
+      }
+      found = __shfl_sync(FULL_MASK, found, L);
+      if (lane == t) pick = found;
+    }
+    *pos = biased_sort_picks(pick, k);
+    return k;
+  }
+  // ------------------------------------------- long rows: chunk sums in registers
+  // chunk c = positions [32c, 32c+32); lane l holds the sums of chunks
+  // [l*T, (l+1)*T).  A round finds the crossing chunk from the chunk sums, then
+  // the crossing position inside it (picks already in that chunk masked out).
+  if (d <= 32 * 32 * BSEG) {
+    const int nch = (d + 31) >> 5, T = (nch + 31) >> 5;
+    unsigned long long cs[BSEG];
+    int npos = 0;
+#pragma unroll
+    for (int j = 0; j < BSEG; ++j) cs[j] = 0;
+    for (int c = 0; c < nch; ++c) {
+      const int p = c * 32 + lane;
+      const uint32_t x = p < d ? __ldg(a + p) : 0u;
+      npos += __popc(__ballot_sync(FULL_MASK, x > 0u));
+      const unsigned long long sum = warp_sum_u64(x);
+      if (lane == c / T) {
+#pragma unroll
+        for (int j = 0; j < BSEG; ++j)
+          if (j == c - lane * T) cs[j] = sum;
+      }
+    }
+    if (npos <= k) {
+      int base = 0;
+      uint32_t mine = 0xffffffffu;
+      for (int c0 = 0; c0 < d; c0 += 32) {
+        const bool f = c0 + lane < d && a[c0 + lane] > 0u;
+        const uint32_t b = __ballot_sync(FULL_MASK, f);
+        const int want = lane - base;
+        if (want >= 0 && want < __popc(b)) mine = c0 + (__fns(b, 0, want + 1));
+        base += __popc(b);
+      }
+      *pos = mine;
+      return npos;
+    }
+    uint32_t pick = 0xffffffffu;
+    const unsigned long long myword = lane < k ? biased_word(key, lane, v, layer) : 0ull;  // all draws at once
+    for (int t = 0; t < k; ++t) {
+      unsigned long long tot = 0;
+#pragma unroll
+      for (int j = 0; j < BSEG; ++j) tot += cs[j];
+      const unsigned long long incl = warp_incl_scan_u64(tot);
+      const unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
+      const unsigned long long r = __umul64hi(__shfl_sync(FULL_MASK, myword, t), W);
+      const int L = __ffs(__ballot_sync(FULL_MASK, incl > r)) - 1;
+      int cstar = 0;
+      unsigned long long before = 0;  // weight of the chunks before the crossing one
+      if (lane == L) {
+        unsigned long long acc = incl - tot;
+        bool done = false;
+#pragma unroll
+        for (int j = 0; j < BSEG; ++j) {
+          if (!done && acc + cs[j] > r) {
+            cstar = lane * T + j;
+            before = acc;
+            done = true;
+          }
+          acc += cs[j];
+        }
+      }
+      cstar = __shfl_sync(FULL_MASK, cstar, L);
+      before = __shfl_sync(FULL_MASK, before, L);
+      const int p = cstar * 32 + lane;
+      bool taken = p >= d;
+      for (int j = 0; j < t; ++j) taken |= __shfl_sync(FULL_MASK, pick, j) == (uint32_t)p;
+      const unsigned long long val = taken ? 0ull : (unsigned long long)__ldg(a + min(p, d - 1));
+      const unsigned long long pin = warp_incl_scan_u64(val);
+      const int P2 = __ffs(__ballot_sync(FULL_MASK, before + pin > r)) - 1;
+      const uint32_t found = (uint32_t)(cstar * 32 + P2);
+      const unsigned long long wfound = __shfl_sync(FULL_MASK, val, P2);
+      if (lane == L) {
+#pragma unroll
+        for (int j = 0; j < BSEG; ++j)
+          if (j == cstar - lane * T) cs[j] -= wfound;  // remove the pick
+      }
+      if (lane == t) pick = found;
+    }
+    *pos = biased_sort_picks(pick, k);
+    return k;
+  }
+  // ---------------------------------------------------------- very long rows
   int npos = 0;
   for (int c0 = 0; c0 < d; c0 += 32) npos += __popc(__ballot_sync(FULL_MASK, c0 + lane < d && a[c0 + lane] > 0u));
-  if (npos <= k) {  // every positive-weight position, in row order
+  if (npos <= k) {
     int base = 0;
     uint32_t mine = 0xffffffffu;
     for (int c0 = 0; c0 < d; c0 += 32) {
       const bool f = c0 + lane < d && a[c0 + lane] > 0u;
       const uint32_t b = __ballot_sync(FULL_MASK, f);
-      // lane t takes the position whose rank among the positive ones is t
       const int want = lane - base;
       if (want >= 0 && want < __popc(b)) mine = c0 + (__fns(b, 0, want + 1));
       base += __popc(b);
@@ -292,23 +469,17 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
     *pos = mine;
     return npos;
   }
-  uint32_t pick = 0xffffffffu;  // lane t: pick of round t
+  uint32_t pick = 0xffffffffu;
   for (int t = 0; t < k; ++t) {
-    // total weight of the positions not picked yet
     unsigned long long part = 0;
     for (int c0 = 0; c0 < d; c0 += 32) {
       const int p = c0 + lane;
-      if (p < d) {
-        bool taken = false;
-        for (int j = 0; j < t; ++j) taken |= __shfl_sync(FULL_MASK, pick, j) == (uint32_t)p;
-        if (!taken) part += a[p];
-      } else {
-        for (int j = 0; j < t; ++j) (void)__shfl_sync(FULL_MASK, pick, j);
-      }
+      bool taken = p >= d;
+      for (int j = 0; j < t; ++j) taken |= __shfl_sync(FULL_MASK, pick, j) == (uint32_t)p;
+      if (!taken) part += a[p];
     }
     const unsigned long long W = warp_sum_u64(part);
-    const uint4 x = philox4x32_10(make_uint4((uint32_t)t, (uint32_t)v, (uint32_t)layer, 0x44535042u), key);
-    const unsigned long long r = __umul64hi(((unsigned long long)x.y << 32) | x.x, W);
+    const unsigned long long r = __umul64hi(biased_word(key, t, v, layer), W);
     unsigned long long acc = 0;
     uint32_t found = 0xffffffffu;
     for (int c0 = 0; c0 < d && found == 0xffffffffu; c0 += 32) {
@@ -323,16 +494,7 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
     }
     if (lane == t) pick = found;
   }
-  // ascending row order: lane t takes the pick of rank t
-  uint32_t mine = 0xffffffffu;
-  for (int s2 = 0; s2 < k; ++s2) {
-    const uint32_t c = __shfl_sync(FULL_MASK, pick, s2);
-    int rank = 0;
-    for (int j = 0; j < k; ++j) rank += __shfl_sync(FULL_MASK, pick, j) < c ? 1 : 0;
-    if (rank == lane) mine = c;
-  }
-  (void)lt;
-  *pos = mine;
+  *pos = biased_sort_picks(pick, k);
   return k;
 }
 

@@ -11,7 +11,8 @@ cfg = datagen.CONFIGS[os.environ.get("CFG", "products")]
 ip, ix = datagen.make_graph(cfg)
 feats = datagen.features(0, cfg.num_nodes, cfg.dim)
 bnds = datagen.bounds(cfg.num_nodes, 1)
-s = pkg.Sampler(bnds, ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2)
+ew = datagen.edge_weights(ix, datagen.node_weights(cfg.num_nodes)) if "biased" in os.environ.get("MODES", "") else None
+s = pkg.Sampler(bnds, ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2, edge_weights=ew)
 train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
 batches = datagen.rank_seed_batches(train, bnds, 0, cfg.batch, 0)
 steps = int(sys.argv[1]) if len(sys.argv) > 1 else 10
@@ -25,6 +26,8 @@ for mode in modes:
             seeds = seeds[:0]
         if mode == "sample":
             s.sample(seeds, 100 + i)
+        elif mode == "biased":
+            s.sample(seeds, 100 + i, biased=True)
         elif mode == "pipelined":
             s.sample_gather(seeds, 100 + i, slot=i % 2, pipelined=True)
             s.sync()
