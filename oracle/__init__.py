@@ -96,6 +96,7 @@ def lib():
                                             ctypes.c_int32, ctypes.c_int32, ctypes.c_uint64, P, P]
         L.oracle_sample_ex.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_int32, P, ctypes.c_int32,
                                        ctypes.c_uint64, ctypes.POINTER(_Block)]
+        L.oracle_random_walk.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, P]
         _lib = L
     return _lib
 
@@ -226,6 +227,18 @@ def sample(indptr, indices, seeds, fanouts, rng_seed: int, weights=None) -> list
     out = [_block_to_numpy(blocks[l]) for l in range(L)]
     for l in range(L):
         lib().oracle_free_block(ctypes.byref(blocks[l]))
+    return out
+
+
+def random_walk(indptr, indices, starts, length: int, rng_seed: int) -> np.ndarray:
+    """Walk traces int32[n][length + 1] (-1 after a dead end)."""
+    ip = _c(indptr, np.int64)
+    ix = _c(indices, np.int32)
+    st = _c(starts, np.int32)
+    out = np.zeros((len(st), length + 1), np.int32)
+    rc = lib().oracle_random_walk(len(ip) - 1, _ptr(ip), _ptr(ix), _ptr(st), len(st), length, rng_seed, _ptr(out))
+    if rc != OK:
+        raise OracleError(rc, "oracle_random_walk")
     return out
 
 
