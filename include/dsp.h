@@ -243,6 +243,19 @@ dsp_status dsp_pipeline_flush(dsp_ctx *ctx, void *stream);
    dsp_sync reports (its row is left unwritten). */
 dsp_status dsp_gather_features(dsp_ctx *ctx, const int32_t *ids, int64_t n, float *out, void *stream);
 
+/* Random walks (Sec. 4.2: "a special case of node-wise sampling,
+   whose fan-out is 1 for all layers"; R27).  Walk i starts at
+   starts[i]; step l from node v takes the neighbour that fan-out-1 node-wise
+   sampling picks for v at layer l with this rng_seed (walks meeting at a node
+   at the same step continue together); a node without neighbours ends the
+   walk and the remaining entries are -1.
+   starts: DEVICE int32[n] in [0, N) (else an error latches for dsp_sync);
+   traces: DEVICE int32[n][length + 1], traces[i][0] = starts[i];
+   1 <= length <= 1024.  world_size 1 only in this version (DSP_ERR_STATE
+   otherwise).  Asynchronous on `stream`. */
+dsp_status dsp_random_walk(dsp_ctx *ctx, const int32_t *starts, int64_t n, int32_t length, uint64_t rng_seed,
+                           int32_t *traces, void *stream);
+
 /* Synchronises `stream` and reports a latched device error (then clears it). */
 dsp_status dsp_sync(dsp_ctx *ctx, void *stream);
 

@@ -1375,6 +1375,38 @@ __global__ void k_weights_fixed(const float *w, int64_t n, uint32_t *out, int *b
   }
 }
 
+// Random walks: step l from node v takes the fan-out-1 node-wise
+// sample of v at layer l (no draw when deg <= 1); a node without neighbours
+// ends the walk (-1 for the remaining steps).  One thread per walk; each step
+// is two dependent random loads (indptr pair, adjacency entry).
+__global__ void __launch_bounds__(NT) k_random_walk(const int32_t *starts, int64_t n, int32_t length, uint2 key,
+                                                    const int64_t *__restrict__ indptr,
+                                                    const int32_t *__restrict__ indices, int64_t N,
+                                                    int32_t *traces, int *err) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    int32_t v = __ldg(starts + i);
+    int32_t *tr = traces + i * (int64_t)(length + 1);
+    if (v < 0 || v >= N) {
+      latch(err, E_RANGE);
+      v = -1;
+    }
+    tr[0] = v;
+    for (int l = 0; l < length; ++l) {
+      if (v >= 0) {
+        const int64_t s = __ldg(indptr + v);
+        const int64_t d = __ldg(indptr + v + 1) - s;
+        if (d == 0) {
+          v = -1;
+        } else {
+          const uint32_t pos = d == 1 ? 0u : draw_range(key, 0u, v, l, (uint32_t)d);
+          v = __ldg(indices + s + pos);
+        }
+      }
+      tr[l + 1] = v;
+    }
+  }
+}
+
 // end of a stage-by-stage call: advance the workspace epoch
 __global__ void k_epoch_advance(WsPersist *persist, uint32_t L) { persist->epoch += L; }
 

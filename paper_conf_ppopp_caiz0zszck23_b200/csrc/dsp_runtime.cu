@@ -1093,6 +1093,23 @@ dsp_status dsp_gather_features(dsp_ctx *c, const int32_t *ids, int64_t n, float 
   return DSP_OK;
 }
 
+dsp_status dsp_random_walk(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length, uint64_t rng_seed,
+                           int32_t *traces, void *stream) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
+  if (c->world != 1) return fail(c, DSP_ERR_STATE, "random walks over a partitioned graph are not implemented yet");
+  if (length < 1 || length > 1024) return fail(c, DSP_ERR_INVALID_ARG, "length %d not in [1, 1024]", length);
+  if (n < 0 || (n > 0 && (!starts || !traces))) return fail(c, DSP_ERR_INVALID_ARG, "bad starts / traces / n");
+  if (n == 0) return DSP_OK;
+  DeviceGuard g(c->device);
+  const int64_t want = (n + NT - 1) / NT;
+  k_random_walk<<<(int)std::min<int64_t>(want, grid_for(c, 8)), NT, 0, static_cast<cudaStream_t>(stream)>>>(
+      starts, n, length, key_of(rng_seed), c->d_indptr, c->d_indices, c->N, traces, c->d_err);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
 dsp_status dsp_sync(dsp_ctx *c, void *stream) {
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();

@@ -34,7 +34,7 @@ DSP_HANDLE_BYTES = 512
 ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_create", "dsp_destroy",
                "dsp_load_partition", "dsp_load_weights", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
                "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
-               "dsp_pipeline_flush", "dsp_gather_features", "dsp_sync")
+               "dsp_pipeline_flush", "dsp_gather_features", "dsp_random_walk", "dsp_sync")
 DSP_ASYNC = 1
 DSP_PIPELINED = 2
 DSP_BIASED = 4
@@ -87,10 +87,11 @@ def lib(path: str | None = None):
                                         ctypes.c_uint32, P]
         L.dsp_gather_features.argtypes = [P, P, i64, P, P]
         L.dsp_pipeline_flush.argtypes = [P, P]
+        L.dsp_random_walk.argtypes = [P, P, i64, i32, ctypes.c_uint64, P, P]
         L.dsp_sync.argtypes = [P, P]
         for name in ("dsp_create", "dsp_load_partition", "dsp_load_weights", "dsp_reserve", "dsp_export_handle",
                      "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
-                     "dsp_pipeline_flush",
+                     "dsp_pipeline_flush", "dsp_random_walk",
                      "dsp_gather_features", "dsp_sync"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
@@ -221,6 +222,11 @@ def dsp_gather_features(ctx, ids, n: int, out, stream: int) -> None:
     _check(lib().dsp_gather_features(ctx, _p(ids), n, _p(out), ctypes.c_void_p(stream)), ctx)
 
 
+def dsp_random_walk(ctx, starts, n: int, length: int, rng_seed: int, traces, stream: int) -> None:
+    _check(lib().dsp_random_walk(ctx, _p(starts), n, length, ctypes.c_uint64(rng_seed), _p(traces),
+                                 ctypes.c_void_p(stream)), ctx)
+
+
 def dsp_sync(ctx, stream: int) -> None:
     _check(lib().dsp_sync(ctx, ctypes.c_void_p(stream)), ctx)
 
@@ -348,6 +354,14 @@ class Sampler:
         if out is None:
             out = torch.empty((n, self.dim), dtype=torch.float32, device=ids.device)
         dsp_gather_features(self.ctx, ids, n, out, self.stream())
+        return out
+
+    def random_walk(self, starts, length: int, rng_seed: int):
+        """Walk traces int32[n][length + 1], asynchronous on the stream."""
+        torch = self.torch
+        assert starts.dtype == torch.int32 and starts.is_cuda and starts.is_contiguous()
+        out = torch.empty((starts.numel(), length + 1), dtype=torch.int32, device=starts.device)
+        dsp_random_walk(self.ctx, starts, starts.numel(), length, rng_seed, out, self.stream())
         return out
 
     def sync(self) -> None:

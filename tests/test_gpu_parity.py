@@ -410,3 +410,32 @@ def test_biased_errors(pkg, tiny):
     with pytest.raises(pkg.DSPError) as e:
         pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8, edge_weights=bad)
     assert e.value.status == pkg.dsp.DSP_ERR_INVALID_ARG
+
+
+# ------------------------------------------------------ random walks
+
+def test_random_walks_tiny(pkg, tiny):
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8)
+    isolated = np.nonzero(np.diff(ip) == 0)[0][:3]
+    starts = np.concatenate([np.arange(0, 10_000, 7), isolated, [5, 5]]).astype(np.int32)
+    for L in (1, 5, 80):
+        tr = s.random_walk(torch.from_numpy(starts).cuda(), L, 0xA11 + L)
+        s.sync()
+        assert np.array_equal(tr.cpu().numpy(), oracle.random_walk(ip, ix, starts, L, 0xA11 + L)), L
+    with pytest.raises(pkg.DSPError):
+        s.random_walk(torch.tensor([cfg.num_nodes], dtype=torch.int32, device="cuda"), 3, 1)
+        s.sync()
+    s.close()
+
+
+@pytest.mark.slow
+def test_random_walks_products(pkg, products):
+    cfg, ip, ix = products
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, None, cfg.fanouts, 8)
+    starts = np.arange(0, cfg.num_nodes, 13, dtype=np.int32)
+    tr = s.random_walk(torch.from_numpy(starts).cuda(), 40, 77)
+    s.sync()
+    sel = np.arange(0, len(starts), 101)
+    assert np.array_equal(tr.cpu().numpy()[sel], oracle.random_walk(ip, ix, starts[sel], 40, 77))
+    s.close()
