@@ -131,10 +131,15 @@ def setup_dist(n_gpus: int):
         if world == 1 and n_gpus > 1:
             raise SystemExit(f"--gpus {n_gpus} needs torchrun with {n_gpus} processes")
         raise SystemExit(f"WORLD_SIZE={world} != --gpus {n_gpus}")
+    if os.environ.get("DSP_BENCH_SAME_GPU"):   # plumbing check only: all ranks on cuda:0, gloo
+        local = 0
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if os.environ.get("DSP_BENCH_SAME_GPU"):
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     return rank, world, local
 
 

@@ -1,0 +1,82 @@
+"""The multi-process CSP path (one process per rank, CUDA IPC peer mapping,
+handle all-gather over torch.distributed, flag-synchronised exchange kernels)
+run with two processes sharing the one GPU of this environment: the same code
+path bench.py --gpus N takes with one process per GPU.  Without MPS the two
+processes' kernels time-slice, so this checks correctness, not speed.
+Each rank's blocks must equal the oracle on its seeds; the one-sided gather
+reads the peer's feature shard through the IPC mapping."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _rank(rank, world, port, q):
+    import sys
+    here = os.path.dirname(os.path.abspath(__file__))
+    sys.path[:0] = [os.path.dirname(here), here]
+    import torch.distributed as dist
+
+    import datagen
+    import oracle
+    import paper_conf_ppopp_caiz0zszck23_b200 as pkg
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+    ok, detail = True, ""
+    try:
+        cfg = datagen.CONFIGS["tiny"]
+        ip, ix = datagen.make_graph(cfg)
+        bnds = datagen.bounds(cfg.num_nodes, world)
+        lo, hi = int(bnds[rank]), int(bnds[rank + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        feats = datagen.features(lo, hi, cfg.dim)
+        s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, 32, rank=rank, world_size=world, device=0,
+                        exchange=pkg.torch_exchange(), n_slots=2)
+        train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
+        batches = datagen.rank_seed_batches(train, bnds, rank, 32, 0)
+        for step in range(3):
+            seeds = batches[step]
+            blocks, feat = s.sample_gather(torch.from_numpy(seeds).cuda(), 0x5EED + step, slot=step % 2)
+            ref = oracle.sample(ip, ix, seeds, cfg.fanouts, 0x5EED + step)
+            for b, r in zip(blocks, ref):
+                for key in ("indptr", "indices", "src_ids"):
+                    if not np.array_equal(getattr(b, key).cpu().numpy(), r[key]):
+                        ok, detail = False, f"step {step} {key}"
+            exp = datagen.features_of(ref[-1]["src_ids"], cfg.dim)
+            if not np.array_equal(feat.cpu().numpy().view(np.uint32), exp.view(np.uint32)):
+                ok, detail = False, f"step {step} features"
+        dist.barrier()
+        s.close()
+    except Exception as e:  # reported to the parent
+        ok, detail = False, repr(e)
+    finally:
+        q.put((rank, ok, detail))
+        dist.destroy_process_group()
+
+
+def test_two_processes_one_gpu():
+    if not torch.cuda.is_available():
+        pytest.fail("needs a GPU")
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rank, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = sorted(q.get(timeout=600) for _ in procs)
+    for p in procs:
+        p.join(timeout=120)
+    assert all(ok for _, ok, _ in res), res
