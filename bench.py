@@ -89,6 +89,9 @@ class ClockSampler:
 
     def __enter__(self):
         self._t.start()
+        t0 = time.time()
+        while not self.samples and time.time() - t0 < 5.0 and self._t.is_alive():
+            time.sleep(0.005)   # the first sample is taken before the timed region starts
         return self
 
     def __exit__(self, *a):
@@ -242,57 +245,81 @@ def run_dsp(args):
     ex = pkg.torch_exchange() if world > 1 else None
     biased = args.scheme == "biased"
     ew = datagen.edge_weights(six, datagen.node_weights(cfg.num_nodes)) if biased else None
+    K = max(1, args.instances) if world == 1 else 1
     s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, cfg.batch, rank=rank, world_size=world,
-                    device=local, exchange=ex, n_slots=2, edge_weights=ew)
+                    device=local, exchange=ex, n_slots=2 * K, edge_weights=ew, n_workspaces=K)
+    if K > 1:  # K steps in flight on K streams, each persistent launch on 1/K of the SMs
+        pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(local).multi_processor_count // K)
     L = len(cfg.fanouts)
     steps_epoch = datagen.steps_per_epoch(train, bnds, cfg.batch)
     batches = datagen.rank_seed_batches(train, bnds, rank, cfg.batch, 0)[:steps_epoch]
     dev_batches = torch.from_numpy(np.ascontiguousarray(batches)).cuda()   # inputs resident in HBM
     stream = torch.cuda.current_stream()
-    K, W = args.steps, args.warmup
-    h_sizes = torch.zeros((W + K, 3 * L), dtype=torch.int64).pin_memory()
-
+    streams = [torch.cuda.Stream() for _ in range(K)]
+    KS, W = args.steps, args.warmup
+    h_sizes = torch.zeros((W + KS, 3 * L), dtype=torch.int64).pin_memory()
     pipelined = not args.no_pipeline
 
     def step(i, ev=None):
         # one step = the whole hot path (CSP over all layers + feature gather) for one
         # batch.  Pipelined (default): the launch of step i samples batch i while its
-        # loader warps gather batch i-1 (the paper's pipeline); two output
-        # sets alternate (queue capacity 2); flush() gathers the last batch.
+        # loader warps gather the previous batch of the same stream (the paper's
+        # pipeline); flush() gathers the last one.  K streams each run
+        # every K-th step on 1/K of the SMs, with 2 output sets each.
+        j = i % K
+        st = streams[j]
         if ev is not None:
-            ev[0].record(stream)
-        s.sample_gather(dev_batches[i % len(batches)], datagen.BASE_SEED + i, slot=i % 2,
-                        sizes_out=h_sizes[i], async_=True, pipelined=pipelined, biased=biased)
+            ev[0].record(st)
+        s.sample_gather(dev_batches[i % len(batches)], datagen.BASE_SEED + i, slot=(i % (2 * K)),
+                        sizes_out=h_sizes[i], async_=True, pipelined=pipelined, biased=biased, ws=j, stream=st)
         if ev is not None:
-            ev[1].record(stream)
+            ev[1].record(st)
 
+    def flush_all():
+        for st in streams:
+            with torch.cuda.stream(st):
+                s.flush()
+
+    def fork():
+        for st in streams:
+            st.wait_stream(stream)
+
+    def join():
+        for st in streams:
+            stream.wait_stream(st)
+
+    fork()
     for i in range(W):
         step(i)
-    s.flush()
+    flush_all()
+    join()
     s.sync()
     barrier()
     torch.cuda.synchronize()
 
-    # ---- timed region: K steps, inputs resident, device time via CUDA events
+    # ---- timed region: KS steps, inputs resident, device time via CUDA events
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(KS)]
     with ClockSampler(local) as clk:
         ev0.record(stream)
-        for j in range(K):
+        fork()
+        for j in range(KS):
             step(W + j, sev[j])
-        s.flush()  # the gather of the last timed batch is inside the timed region
+        flush_all()  # the gathers of the last timed batches are inside the timed region
+        join()
         ev1.record(stream)
         s.sync()
         torch.cuda.synchronize()
     barrier()
+    K_ = KS
     t_ms = ev0.elapsed_time(ev1)
     step_ms = [a.elapsed_time(b) for a, b in sev]
-    sz = h_sizes.numpy()[W: W + K]
-    edges = float(sum(int(sz[j, 3 * l + 2]) for j in range(K) for l in range(L)))
-    rows = float(sum(int(sz[j, 3 * (L - 1) + 1]) for j in range(K)))
-    seeds_n = float(sum(int(sz[j, 0]) for j in range(K)))
+    sz = h_sizes.numpy()[W: W + KS]
+    edges = float(sum(int(sz[j, 3 * l + 2]) for j in range(KS) for l in range(L)))
+    rows = float(sum(int(sz[j, 3 * (L - 1) + 1]) for j in range(KS)))
+    seeds_n = float(sum(int(sz[j, 0]) for j in range(KS)))
     samp_b = gath_b = 0
-    for j in range(K):
+    for j in range(KS):
         a, b = algorithmic_bytes(sz[j], L, cfg.dim)
         samp_b += a
         gath_b += b
@@ -302,17 +329,22 @@ def run_dsp(args):
     tot_seeds = reduce_sum_over_ranks(seeds_n)
     peak, peak_kind = measured_peaks()
     step_mean = float(np.mean(step_ms))
-    achieved = (samp_b + gath_b) / K / (step_mean * 1e-3) / 1e9
+    # K launches overlap on the device: the kernel stream's achieved HBM rate is the
+    # algorithmic bytes of all timed launches over the elapsed device time
+    achieved = (samp_b + gath_b) / (t_ms * 1e-3) / 1e9
 
     # ---- breakdown (not the headline): the two calls separately
     ids_dev = None
     bd = {}
     if not args.no_breakdown:
-        g_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+        NB = min(KS, 20)
+        if K > 1:
+            pkg.dsp_set_persistent_blocks(s.ctx, 0)   # the breakdown times single full-GPU calls
+        g_ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(NB)]
         s_ms = []
         nrow = []
         out = s.feat_buffer(0)
-        for j in range(K):
+        for j in range(NB):
             i = W + j
             a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a0.record(stream)
@@ -372,7 +404,7 @@ def run_dsp(args):
     if rank == 0:
         line = {
             "metric": METRIC, "value": tot_edges / (t_max * 1e-3), "unit": "edges/s", "n_gpus": world,
-            "steps": K, "warmup": W, "ms_per_step": t_max / K,
+            "steps": KS, "warmup": W, "ms_per_step": t_max / KS,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32+f32",
             "data": "synthetic",
             "config": {"workload": (cfg.name if world == 1 else f"{cfg.name}-P{world}")
@@ -380,25 +412,28 @@ def run_dsp(args):
                        "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes,
                        "nnz": int(ip[-1]), "dim": cfg.dim, "parallelism": f"csp{world}",
                        "l2": "inputs larger than L2 (CSR 0.5 GB + features 1.1 GB >> 126 MB L2)",
-                       "step": "dsp_sample_gather (DSP_PIPELINED: sampler(t) || loader(t-1), 2 output sets)"
-                       if pipelined else "dsp_sample_gather (async, 2 output sets)"},
+                       "step": ("dsp_sample_gather (DSP_PIPELINED: sampler(t) || loader(t-1), 2 output sets)"
+                                if pipelined else "dsp_sample_gather (async, 2 output sets)")
+                       + (f", {K} streams x {torch.cuda.get_device_properties(local).multi_processor_count // K} SMs"
+                          if K > 1 else "")},
             "seeds_per_s": tot_seeds / (t_max * 1e-3),
             "feature_GBps": tot_rows * cfg.dim * 4 / (t_max * 1e-3) / 1e9,
-            "edges_per_step": tot_edges / K / world,
-            "rows_per_step": tot_rows / K / world,
+            "edges_per_step": tot_edges / KS / world,
+            "rows_per_step": tot_rows / KS / world,
             "roofline": {"kernel": "k_csp_persistent" if world == 1 else "k_gather",
                          "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": ncu_traffic("k_csp_persistent"),
                          "peak_kind": peak_kind,
-                         "algorithmic_bytes_per_launch": (samp_b + gath_b) / K,
-                         "sampling_bytes_per_launch": samp_b / K, "gather_bytes_per_launch": gath_b / K,
-                         "launch_ms_mean": step_mean},
+                         "algorithmic_bytes_per_launch": (samp_b + gath_b) / KS,
+                         "sampling_bytes_per_launch": samp_b / KS, "gather_bytes_per_launch": gath_b / KS,
+                         "launch_ms_mean": step_mean, "concurrent_launches": K,
+                         "achieved_def": "algorithmic bytes of all timed launches / elapsed device time"},
             "breakdown": bd,
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_edges / (e2e_ms * 1e-3), "unit": "edges/s",
                     "h2d_bytes_per_step": h2d // e2e_steps, "d2h_bytes_per_step": d2h // e2e_steps,
                     "steps": e2e_steps, "api": "dsp_sample_gather (synchronous) + D2H of blocks and features"},
-            "gpu_launches": kern_per_step * K,
+            "gpu_launches": kern_per_step * KS + (K if pipelined else 0),
             "clocks": clk.summary(),
         }
         print(json.dumps(line), flush=True)
@@ -411,7 +446,7 @@ def run_dsp(args):
 def main(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["dsp", "reference"], default="dsp")
     ap.add_argument("--config", default=None)
@@ -420,6 +455,7 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-breakdown", action="store_true")
     ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
+    ap.add_argument("--instances", type=int, default=2, help="concurrent step streams (world 1)")
     ap.add_argument("--scheme", choices=["uniform", "biased"], default="uniform",
                     help="node-wise scheme (Table 2 IsBiased); biased uses synthetic node weights")
     args = ap.parse_args(argv)

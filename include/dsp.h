@@ -227,6 +227,13 @@ dsp_status dsp_sample_gather(dsp_ctx *ctx, const int32_t *seeds, int32_t num_see
                              int64_t feat_cap_rows, void *workspace, size_t workspace_bytes,
                              int64_t *sizes_out, uint32_t flags, void *stream);
 
+/* Number of 1024-thread blocks of the world-1 persistent kernel (0 = the
+   default, one per SM).  A smaller grid lets several steps run concurrently
+   on different streams, each with its own workspace and outputs (e.g. two
+   steps on half of the SMs each, so one step's latency-bound sampling phases
+   overlap the other's bandwidth-bound gather).  Not collective. */
+dsp_status dsp_set_persistent_blocks(dsp_ctx *ctx, int32_t blocks);
+
 /* Enqueues the gather still owed by the last DSP_PIPELINED call (no-op when
    none is pending).  Stream-ordered on `stream`. */
 dsp_status dsp_pipeline_flush(dsp_ctx *ctx, void *stream);

@@ -38,8 +38,9 @@ constexpr int MAX_PERSIST_BLOCKS = 1024;
 
 // Persistent part of the workspace (offset 0).  Zero-filled before first use.
 struct WsPersist {
-  uint32_t epoch;  // last relabel epoch used with this workspace
-  uint32_t pad[63];
+  uint32_t epoch;      // last relabel epoch used with this workspace
+  int32_t pend_n[2];   // row counts of pipelined calls (alternating), read by the next call / flush
+  uint32_t pad[61];
 };
 
 // Per-call state (memset to 0 by the host before every call).

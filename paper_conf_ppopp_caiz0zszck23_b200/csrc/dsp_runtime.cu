@@ -122,12 +122,29 @@ struct dsp_ctx {
   int *h_err = nullptr;
   int num_sms = 148;
   int persist_blocks_per_sm = 1;
+  int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
   int gather_blocks_per_sm = 1;
-  // pipelined steps: the gather owed by the previous DSP_PIPELINED call
-  int32_t *d_pend = nullptr;          // its row count (device, written by its kernel)
-  const int32_t *pend_ids = nullptr;  // its last block's src_ids
-  float *pend_out = nullptr;          // its feature output
-  bool pending = false;
+  // pipelined steps: per workspace, the gather owed by its previous
+  // DSP_PIPELINED call (row count in the workspace's WsPersist::pend_n[parity])
+  struct Pending {
+    const char *ws = nullptr;
+    const int32_t *ids = nullptr;  // its last block's src_ids
+    float *out = nullptr;          // its feature output
+    void *stream = nullptr;
+    uint32_t calls = 0;            // pipelined calls made with this workspace
+    bool active = false;
+  } pend[8];
+  Pending *pending_of(const char *ws) {
+    for (auto &p : pend)
+      if (p.ws == ws) return &p;
+    for (auto &p : pend)
+      if (!p.ws || !p.active) {
+        p = Pending{};
+        p.ws = ws;
+        return &p;
+      }
+    return nullptr;
+  }
 };
 
 namespace {
@@ -398,36 +415,48 @@ dsp_status stage_persistent(Call &k) {
   a.err = c->d_err;
   a.gather = k.feat_out != nullptr && !k.pipelined;
   if (a.gather) a.g = make_gather(c, k.blocks[k.L - 1].src_ids, 0, nullptr, k.feat_out);
-  const dim3 grid(c->num_sms * c->persist_blocks_per_sm), block(PNT);
+  const dim3 grid(c->persist_blocks > 0 ? c->persist_blocks : c->num_sms * c->persist_blocks_per_sm), block(PNT);
   void *args[] = {&a};
   if (!k.pipelined) {
     CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_persistent<PNT, false>, grid, block, args, 0,
                                             k.stream));
     return DSP_OK;
   }
-  a.prev = c->pending ? 1 : 0;
-  if (a.prev) a.gp = make_gather(c, c->pend_ids, 0, c->d_pend, c->pend_out);
-  a.pend_n = c->d_pend;
+  dsp_ctx::Pending *pd = c->pending_of(k.ws);
+  if (!pd) return fail(c, DSP_ERR_STATE, "more than 8 workspaces with pending pipelined gathers");
+  WsPersist *ps = persist_of(k);
+  a.prev = pd->active ? 1 : 0;
+  if (a.prev) a.gp = make_gather(c, pd->ids, 0, &ps->pend_n[(pd->calls + 1) & 1], pd->out);
+  a.pend_n = &ps->pend_n[pd->calls & 1];
   const int row_bytes = c->dim * 4;
   a.slot_bytes = (int)align_up((size_t)std::max(12800, row_bytes), 128);
   a.rows_per_chunk = std::max(1, std::min(32, a.slot_bytes / std::max(1, row_bytes)));
   const size_t smem = (size_t)LOADER_WARPS * LOADER_SLOTS * a.slot_bytes;
   CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_persistent<PIPE_TEAM, true>, grid, block, args, smem,
                                           k.stream));
-  c->pend_ids = k.blocks[k.L - 1].src_ids;
-  c->pend_out = k.feat_out;
-  c->pending = true;
+  pd->ids = k.blocks[k.L - 1].src_ids;
+  pd->out = k.feat_out;
+  pd->stream = k.stream;
+  pd->active = true;
+  pd->calls += 1;
   return DSP_OK;
 }
 
-// gather owed by the last pipelined call (k_gather with the device row count)
-dsp_status stage_flush(dsp_ctx *c, cudaStream_t stream) {
-  if (!c->pending) return DSP_OK;
+// gather owed by a workspace's last pipelined call (k_gather with the device row count)
+dsp_status flush_one(dsp_ctx *c, dsp_ctx::Pending &pd) {
+  if (!pd.active) return DSP_OK;
   DeviceGuard g(c->device);
-  GatherArgs a = make_gather(c, c->pend_ids, 0, c->d_pend, c->pend_out);
-  k_gather<<<grid_for(c, std::min(6, c->gather_blocks_per_sm)), NT, 0, stream>>>(a);
+  const WsPersist *ps = reinterpret_cast<const WsPersist *>(pd.ws);
+  GatherArgs a = make_gather(c, pd.ids, 0, &ps->pend_n[(pd.calls + 1) & 1], pd.out);
+  k_gather<<<grid_for(c, std::min(6, c->gather_blocks_per_sm)), NT, 0, static_cast<cudaStream_t>(pd.stream)>>>(a);
   CUDA_TRY(c, cudaGetLastError());
-  c->pending = false;
+  pd.active = false;
+  return DSP_OK;
+}
+
+dsp_status stage_flush(dsp_ctx *c, const char *ws) {
+  for (auto &p : c->pend)
+    if (p.active && p.ws == ws) return flush_one(c, p);
   return DSP_OK;
 }
 
@@ -621,7 +650,7 @@ dsp_status run_calls(std::vector<Call> &calls) {
   // a non-pipelined call first settles a pending pipelined gather; so does a
   // pipelined call of the stage-by-stage path (no loader warps there)
   for (auto &k : calls)
-    if (k.c->pending && (!k.pipelined || k.c->world > 1) && (st = stage_flush(k.c, k.stream)) != DSP_OK) return st;
+    if ((!k.pipelined || k.c->world > 1) && (st = stage_flush(k.c, k.ws)) != DSP_OK) return st;
   EACH(stage_begin(k));
   if (calls[0].c->world == 1) {
     EACH(stage_persistent(k));
@@ -636,11 +665,15 @@ dsp_status run_calls(std::vector<Call> &calls) {
     for (auto &k : calls) {
       if (k.feat_out && k.pipelined) {  // this call's rows: gathered by the next call / flush
         DeviceGuard g(k.c->device);
-        CUDA_TRY(k.c, cudaMemcpyAsync(k.c->d_pend, &k.hdr->S[k.L - 1], sizeof(int32_t), cudaMemcpyDeviceToDevice,
-                                      k.stream));
-        k.c->pend_ids = k.blocks[k.L - 1].src_ids;
-        k.c->pend_out = k.feat_out;
-        k.c->pending = true;
+        dsp_ctx::Pending *pd = k.c->pending_of(k.ws);
+        if (!pd) return fail(k.c, DSP_ERR_STATE, "more than 8 workspaces with pending pipelined gathers");
+        pd->calls += 1;
+        CUDA_TRY(k.c, cudaMemcpyAsync(&persist_of(k)->pend_n[(pd->calls + 1) & 1], &k.hdr->S[k.L - 1],
+                                      sizeof(int32_t), cudaMemcpyDeviceToDevice, k.stream));
+        pd->ids = k.blocks[k.L - 1].src_ids;
+        pd->out = k.feat_out;
+        pd->stream = k.stream;
+        pd->active = true;
       } else if (k.feat_out && (st = stage_gather_dev(k)) != DSP_OK) {
         return st;
       }
@@ -674,7 +707,6 @@ void release(dsp_ctx *c) {
   cudaFree(c->d_feat);
   cudaFree(c->d_xch);
   cudaFree(c->d_err);
-  cudaFree(c->d_pend);
   if (c->h_hdr) cudaFreeHost(c->h_hdr);
   if (c->h_err) cudaFreeHost(c->h_err);
   cudaGetLastError();
@@ -758,8 +790,7 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   c->gather_blocks_per_sm = occ;
   if (cudaMallocHost(&c->h_hdr, sizeof(WsHeader)) != cudaSuccess ||
       cudaMallocHost(&c->h_err, sizeof(int)) != cudaSuccess ||
-      cudaMalloc(&c->d_err, sizeof(int)) != cudaSuccess || cudaMemset(c->d_err, 0, sizeof(int)) != cudaSuccess ||
-      cudaMalloc(&c->d_pend, sizeof(int32_t)) != cudaSuccess) {
+      cudaMalloc(&c->d_err, sizeof(int)) != cudaSuccess || cudaMemset(c->d_err, 0, sizeof(int)) != cudaSuccess) {
     cudaGetLastError();
     release(c);
     delete c;
@@ -1039,10 +1070,25 @@ dsp_status dsp_sample_gather(dsp_ctx *c, const int32_t *seeds, int32_t num_seeds
   return run_calls(calls);
 }
 
+dsp_status dsp_set_persistent_blocks(dsp_ctx *c, int32_t blocks) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  const int maxb = c->num_sms * c->persist_blocks_per_sm;
+  if (blocks < 0 || blocks > maxb)
+    return fail(c, DSP_ERR_INVALID_ARG, "blocks %d not in [0, %d]", blocks, maxb);
+  c->persist_blocks = blocks;
+  return DSP_OK;
+}
+
 dsp_status dsp_pipeline_flush(dsp_ctx *c, void *stream) {
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
-  return stage_flush(c, static_cast<cudaStream_t>(stream));
+  for (auto &p : c->pend)
+    if (p.active && p.stream == stream) {
+      dsp_status st = flush_one(c, p);
+      if (st != DSP_OK) return st;
+    }
+  return DSP_OK;
 }
 
 dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n, const int32_t *const *seeds,

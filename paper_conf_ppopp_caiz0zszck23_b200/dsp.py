@@ -34,7 +34,8 @@ DSP_HANDLE_BYTES = 512
 ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_create", "dsp_destroy",
                "dsp_load_partition", "dsp_load_weights", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
                "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
-               "dsp_pipeline_flush", "dsp_gather_features", "dsp_random_walk", "dsp_sync")
+               "dsp_pipeline_flush", "dsp_set_persistent_blocks", "dsp_gather_features", "dsp_random_walk",
+               "dsp_sync")
 DSP_ASYNC = 1
 DSP_PIPELINED = 2
 DSP_BIASED = 4
@@ -87,11 +88,12 @@ def lib(path: str | None = None):
                                         ctypes.c_uint32, P]
         L.dsp_gather_features.argtypes = [P, P, i64, P, P]
         L.dsp_pipeline_flush.argtypes = [P, P]
+        L.dsp_set_persistent_blocks.argtypes = [P, i32]
         L.dsp_random_walk.argtypes = [P, P, i64, i32, ctypes.c_uint64, P, P]
         L.dsp_sync.argtypes = [P, P]
         for name in ("dsp_create", "dsp_load_partition", "dsp_load_weights", "dsp_reserve", "dsp_export_handle",
                      "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
-                     "dsp_pipeline_flush", "dsp_random_walk",
+                     "dsp_pipeline_flush", "dsp_random_walk", "dsp_set_persistent_blocks",
                      "dsp_gather_features", "dsp_sync"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
@@ -222,6 +224,10 @@ def dsp_gather_features(ctx, ids, n: int, out, stream: int) -> None:
     _check(lib().dsp_gather_features(ctx, _p(ids), n, _p(out), ctypes.c_void_p(stream)), ctx)
 
 
+def dsp_set_persistent_blocks(ctx, blocks: int) -> None:
+    _check(lib().dsp_set_persistent_blocks(ctx, blocks), ctx)
+
+
 def dsp_random_walk(ctx, starts, n: int, length: int, rng_seed: int, traces, stream: int) -> None:
     _check(lib().dsp_random_walk(ctx, _p(starts), n, length, ctypes.c_uint64(rng_seed), _p(traces),
                                  ctypes.c_void_p(stream)), ctx)
@@ -252,7 +258,7 @@ class Sampler:
     def __init__(self, bounds, indptr, indices, features, fanouts, max_seeds: int, rank: int = 0,
                  world_size: int = 1, device: int | None = None,
                  exchange: Callable[[bytes], list] | None = None, connect: bool = True, n_slots: int = 1,
-                 edge_weights=None):
+                 edge_weights=None, n_workspaces: int = 1):
         import torch
         self.torch = torch
         self.device = torch.cuda.current_device() if device is None else device
@@ -274,7 +280,9 @@ class Sampler:
             raise
         dev = torch.device("cuda", self.device)
         self.workspace_bytes = ws
-        self.workspace = torch.zeros(ws, dtype=torch.uint8, device=dev)  # zero-filled before first use
+        # zero-filled before first use; several workspaces let steps run concurrently on several streams
+        self.workspaces = [torch.zeros(ws, dtype=torch.uint8, device=dev) for _ in range(max(1, n_workspaces))]
+        self.workspace = self.workspaces[0]
         F = [self.max_seeds] + [int(x) for x in ms[:-1]]
         self._sets = []
         for _ in range(max(1, n_slots)):   # output sets (a queue of capacity n_slots)
@@ -311,7 +319,7 @@ class Sampler:
         return self.blocks()
 
     def sample_gather(self, seeds, rng_seed: int, slot: int = 0, sizes_out=None, async_: bool = False,
-                      pipelined: bool = False, biased: bool = False):
+                      pipelined: bool = False, biased: bool = False, ws: int = 0, stream=None):
         """One whole step (sample + gather) in one call into output set `slot`.
         Synchronous: returns (blocks, features view).  async_: returns None;
         sizes land in sizes_out (pinned host / device int64[3L]) in stream order.
@@ -322,7 +330,8 @@ class Sampler:
         feat_out = self.feat_buffer(slot)
         flags = (DSP_PIPELINED if pipelined else (DSP_ASYNC if async_ else 0)) | (DSP_BIASED if biased else 0)
         dsp_sample_gather(self.ctx, seeds, seeds.numel(), self.fanouts, rng_seed, self._sets[slot][1], feat_out,
-                          feat_out.shape[0], self.workspace, self.workspace_bytes, sizes_out, flags, self.stream())
+                          feat_out.shape[0], self.workspaces[ws], self.workspace_bytes, sizes_out, flags,
+                          self.stream() if stream is None else stream.cuda_stream)
         if async_ or pipelined:
             return None
         blocks = self.blocks(slot)
