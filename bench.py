@@ -371,7 +371,7 @@ def run_dsp(args):
     h_feat = torch.empty((s.max_src[-1], cfg.dim), dtype=torch.float32).pin_memory()
     h_blk = [tuple(torch.empty(x.numel(), dtype=torch.int32).pin_memory() for x in bufs) for bufs in s._bufs]
     d_seed = torch.empty(cfg.batch, dtype=torch.int32, device="cuda")
-    e2e_steps = max(3, min(K, 20))
+    e2e_steps = max(3, min(KS, 20))
     h2d = d2h = 0
     barrier()
     torch.cuda.synchronize()

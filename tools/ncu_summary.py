@@ -45,7 +45,7 @@ def main(rep, launches, tag):
     for r in rows:
         d = dict(zip(hdr, r))
         u = dict(zip(hdr, units))
-        name = d["Kernel Name"].split("(")[0]
+        name = d["Kernel Name"].split("(")[0].replace("void ", "").strip()
         rec = {}
         for m, short in METRICS.items():
             if m in d and d[m] not in ("", "n/a"):
@@ -76,7 +76,7 @@ def main(rep, launches, tag):
                      f"{avg('occupancy_pct'):.1f} | {int(avg('regs'))} | {int(avg('grid'))} x {int(avg('block'))} | "
                      + ", ".join(f"{k} {100 * v:.0f}%" for k, v in st.items()) + " |")
         big = max(recs, key=lambda r: r.get("dram_read", 0) + r.get("dram_write", 0))  # the fused launch
-        traffic[name] = {"dram_bytes_per_launch": big.get("dram_read", 0) + big.get("dram_write", 0),
+        traffic[name.split("<")[0]] = {"dram_bytes_per_launch": big.get("dram_read", 0) + big.get("dram_write", 0),
                          "dram_read_bytes": big.get("dram_read", 0), "dram_write_bytes": big.get("dram_write", 0),
                          "duration_s_ncu": big.get("duration", 0), "source": f"profiles/ncu_{tag}.md",
                          "note": "largest-traffic capture of this kernel (the fused sample+gather launch bench.py times)"}
