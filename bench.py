@@ -247,7 +247,8 @@ def run_dsp(args):
     ew = datagen.edge_weights(six, datagen.node_weights(cfg.num_nodes)) if biased else None
     K = max(1, args.instances) if world == 1 else 1
     s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, cfg.batch, rank=rank, world_size=world,
-                    device=local, exchange=ex, n_slots=2 * K, edge_weights=ew, n_workspaces=K)
+                    device=local, exchange=ex, n_slots=2 * K, edge_weights=ew, n_workspaces=K,
+                    hot_rows=None if args.hot_frac is None else int(round(args.hot_frac * (len(sip) - 1))))
     if K > 1:  # K steps in flight on K streams, each persistent launch on 1/K of the SMs
         pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(local).multi_processor_count // K)
     L = len(cfg.fanouts)
@@ -408,7 +409,11 @@ def run_dsp(args):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32+f32",
             "data": "synthetic",
             "config": {"workload": (cfg.name if world == 1 else f"{cfg.name}-P{world}")
-                       + ("-biased" if biased else ""), "scheme": args.scheme,
+                       + ("-biased" if biased else "")
+                       + ("" if args.hot_frac is None else f"-hot{args.hot_frac:g}"), "scheme": args.scheme,
+                       "features": ("all rows in HBM" if args.hot_frac is None else
+                                    f"cold tier: {args.hot_frac:g} of rows (largest in-degree) in HBM, "
+                                    "the rest in pinned host memory read over UVA"),
                        "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes,
                        "nnz": int(ip[-1]), "dim": cfg.dim, "parallelism": f"csp{world}",
                        "l2": "inputs larger than L2 (CSR 0.5 GB + features 1.1 GB >> 126 MB L2)",
@@ -458,6 +463,8 @@ def main(argv=None):
     ap.add_argument("--instances", type=int, default=2, help="concurrent step streams (world 1)")
     ap.add_argument("--scheme", choices=["uniform", "biased"], default="uniform",
                     help="node-wise scheme (Table 2 IsBiased); biased uses synthetic node weights")
+    ap.add_argument("--hot-frac", type=float, default=None,
+                    help="cold-feature tier: fraction of each shard's rows kept in HBM (P:L114)")
     args = ap.parse_args(argv)
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

@@ -103,6 +103,20 @@ void dsp_destroy(dsp_ctx *ctx);
 dsp_status dsp_load_partition(dsp_ctx *ctx, const int64_t *bounds, const int64_t *indptr,
                               const int32_t *indices, const float *features, int32_t dim);
 
+/* Feature shard with a cold tier ("we cache as many hot nodes as
+   possible in GPU memory and store the other nodes (called cold nodes) in CPU
+   memory and access them using the UVA technique.  DSP uses large indegrees to
+   select hot nodes by default"; P:L224 feature position list).  Use instead of
+   passing features to dsp_load_partition (features = NULL there).
+   features: host or device fp32[n_r][dim]; hot_rows: rows kept in HBM (the
+   hot_rows largest in-degrees of this rank, ties by id; < 0 or > n_r = all);
+   the others go to pinned host memory (POSIX shm when world_size > 1, so that
+   peers' GPUs can read them too) and are read over UVA by whichever GPU
+   gathers them.  Gather results are bit-identical for any hot_rows.  Once per
+   ctx, after dsp_load_partition and before dsp_reserve / handle export; all
+   ranks must agree on using the tier. */
+dsp_status dsp_load_features_tiered(dsp_ctx *ctx, const float *features, int32_t dim, int64_t hot_rows);
+
 /* Edge weights for biased sampling (Sec. 4.2: "each node u ... is
    associated with a non-negative weight w_u ... DSP stores node weight w_u
    along with edge e_{v,u}").  edge_weights: host or device fp32[nnz_r]

@@ -564,10 +564,27 @@ struct GatherArgs {
   int32_t dim4;             // dim / 4  (output row length in float4)
   int32_t stride4;          // shard row stride in float4 (rows padded to 64 B)
   float4 *out;
-  const float4 *base[8];    // feature shard of each rank (local or peer-mapped)
+  const float4 *base[8];    // feature shard (hot rows) of each rank (local or peer-mapped)
+  // cold-feature tier: feature position list of each rank
+  // (>= 0 hot slot, < 0 cold slot -p-1) and its cold rows in host memory (UVA)
+  int32_t tiered;
+  const int32_t *fpos[8];
+  const float4 *cold[8];
   Bounds bd;
   int *err;
 };
+
+// Address of the feature row of global id g (owner o): the shard row, or with
+// the cold tier the hot slot in HBM / the cold slot in host memory read over
+// UVA by the requesting GPU ("loaded from CPU memory by the requesting GPU").
+__device__ __forceinline__ const float4 *feature_row(const GatherArgs &a, int o, int32_t g) {
+  const uint32_t lv = (uint32_t)(g - (int32_t)a.bd.b[o]);
+  const int32_t *fp = a.fpos[o];  // null: rank o keeps all its rows in HBM (in id order)
+  if (!a.tiered || !fp) return a.base[o] + (size_t)lv * (uint32_t)a.stride4;
+  const int32_t p = __ldg(fp + lv);
+  return p >= 0 ? a.base[o] + (size_t)(uint32_t)p * (uint32_t)a.stride4
+                : a.cold[o] + (size_t)(uint32_t)(-p - 1) * (uint32_t)a.stride4;
+}
 
 __device__ __forceinline__ float4 ld_stream_f4(const float4 *p) {
   float4 v;
@@ -605,7 +622,7 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
     for (int u = 0; u < UNROLL; ++u) {
       if (g[u] >= 0 && g[u] < N) {
         const int o = owner_of(a.bd, g[u]);
-        v[u] = ld_f4_hint(a.base[o] + (size_t)(uint32_t)(g[u] - (int32_t)a.bd.b[o]) * (uint32_t)a.stride4 + c[u], pol);
+        v[u] = ld_f4_hint(feature_row(a, o, g[u]) + c[u], pol);
       }
     }
 #pragma unroll
@@ -718,9 +735,11 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
       __syncwarp();
       if (lane < rows) {
         const int32_t id = __ldg(g.ids + (int64_t)c * R + lane);
-        if (id >= 0 && id < (int32_t)g.bd.b[1])
+        if (id >= 0 && id < (int32_t)g.bd.b[1])  // cold rows: the bulk copy reads host memory over UVA
           bulk_g2s_hint(ring + (size_t)s * a.slot_bytes + (size_t)lane * row_bytes,
-                        base + (size_t)(uint32_t)id * stride_bytes, row_bytes, &bars[s], pol);
+                        g.tiered ? reinterpret_cast<const char *>(feature_row(g, 0, id))
+                                 : base + (size_t)(uint32_t)id * stride_bytes,
+                        row_bytes, &bars[s], pol);
         else  // keep the byte count consistent; the error is reported
           latch(g.err, E_RANGE);
       }
@@ -789,8 +808,7 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
       }
 #pragma unroll
       for (int u = 0; u < 4; ++u)
-        if (id[u] >= 0 && id[u] < (int32_t)g.bd.b[1])
-          v[u] = ld_f4_hint(g.base[0] + (size_t)(uint32_t)id[u] * g.stride4 + col[u], pol);
+        if (id[u] >= 0 && id[u] < (int32_t)g.bd.b[1]) v[u] = ld_f4_hint(feature_row(g, 0, id[u]) + col[u], pol);
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const uint32_t e = e0 + 32u * u;
@@ -826,7 +844,10 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
     __syncwarp();
     if (a.prev) {
       const int64_t n = ld_volatile_i32(a.gp.n_dev);
-      loader_warp(a, ring_smem + (size_t)w * LOADER_SLOTS * a.slot_bytes, bars[w], n);
+      if (a.gp.tiered == 1)  // cold tier read with register loads (DSP_COLD_REGLOADS=1)
+        helper_warp(a, n);
+      else
+        loader_warp(a, ring_smem + (size_t)w * LOADER_SLOTS * a.slot_bytes, bars[w], n);
     }
     if (blockIdx.x == 0 && threadIdx.x == TEAM) a.hdr->t[22] = globaltimer_ns();  // loader warp 0 of block 0 done
     return;

@@ -3,6 +3,9 @@
 // P2P), workspace planning, and the CSP driver that issues the kernels of
 // dsp_kernels.cuh.  sm_100a only.
 #include <cuda_runtime.h>
+#include <fcntl.h>
+#include <sys/mman.h>
+#include <sys/stat.h>
 #include <unistd.h>
 
 #include <algorithm>
@@ -45,7 +48,11 @@ struct PeerHandle {  // fits in DSP_HANDLE_BYTES
   int32_t has_feat, has_xch;
   cudaIpcMemHandle_t feat_ipc, xch_ipc;
   int64_t bounds[DSP_MAX_WORLD + 1];
-  int32_t dim, max_seeds, feat_stride, pad;
+  int32_t dim, max_seeds, feat_stride, tiered;
+  cudaIpcMemHandle_t fpos_ipc;
+  uint64_t fpos_ptr, cold_ptr;
+  int64_t cold_bytes;
+  char cold_shm[48];  // POSIX shm name of the cold rows (cross-process access)
 };
 static_assert(sizeof(PeerHandle) <= DSP_HANDLE_BYTES, "handle too large");
 
@@ -106,6 +113,17 @@ struct dsp_ctx {
   uint32_t *d_weights = nullptr;  // 16.16 edge weights (biased sampling)
   float *d_feat = nullptr;
   int64_t feat_bytes = 0;
+  // cold-feature tier
+  bool tiered = false;
+  bool cold_regloads = false;         // env DSP_COLD_REGLOADS=1 (measurement switch)
+  int32_t *d_fpos = nullptr;          // feature position list [n_local]
+  float *h_cold = nullptr;            // cold rows (pinned host, UVA-mapped)
+  int64_t cold_bytes = 0;
+  char cold_shm[48] = {0};            // non-empty: h_cold is a registered POSIX shm mapping
+  const int32_t *peer_fpos[DSP_MAX_WORLD] = {nullptr};
+  const float *peer_cold[DSP_MAX_WORLD] = {nullptr};
+  void *peer_cold_map[DSP_MAX_WORLD] = {nullptr};  // shm mappings opened in this process
+  int64_t peer_cold_bytes[DSP_MAX_WORLD] = {0};
   int *d_err = nullptr;  // latched device error of this ctx
   // exchange
   int32_t max_seeds = 0, L = 0, kmax = 0;
@@ -115,7 +133,7 @@ struct dsp_ctx {
   // peers
   const float *peer_feat[DSP_MAX_WORLD] = {nullptr};
   char *peer_xch[DSP_MAX_WORLD] = {nullptr};
-  void *ipc_opened[2 * DSP_MAX_WORLD] = {nullptr};
+  void *ipc_opened[3 * DSP_MAX_WORLD] = {nullptr};  // feat, xch, fpos per peer
   unsigned long long seq = 0;
   // host staging (pinned)
   WsHeader *h_hdr = nullptr;
@@ -274,8 +292,13 @@ GatherArgs make_gather(const dsp_ctx *c, const int32_t *ids, int64_t n, const in
   a.dim4 = c->dim / 4;
   a.stride4 = c->feat_stride / 4;
   a.out = reinterpret_cast<float4 *>(out);
-  for (int r = 0; r < DSP_MAX_WORLD; ++r)
+  for (int r = 0; r < DSP_MAX_WORLD; ++r) {
     a.base[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_feat[r]) : nullptr;
+    a.fpos[r] = r < c->world ? c->peer_fpos[r] : nullptr;
+    a.cold[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_cold[r]) : nullptr;
+  }
+  // 2: loader warps bulk-copy cold rows from host memory too; 1: register loads
+  a.tiered = c->tiered ? (c->cold_regloads ? 1 : 2) : 0;
   a.bd = make_bounds(c);
   a.err = c->d_err;
   return a;
@@ -696,7 +719,24 @@ dsp_status run_calls(std::vector<Call> &calls) {
 
 void release(dsp_ctx *c) {
   DeviceGuard g(c->device);
-  for (int i = 0; i < 2 * DSP_MAX_WORLD; ++i)
+  for (int r = 0; r < DSP_MAX_WORLD; ++r)
+    if (c->peer_cold_map[r]) {
+      cudaHostUnregister(c->peer_cold_map[r]);
+      munmap(c->peer_cold_map[r], (size_t)c->peer_cold_bytes[r]);
+      c->peer_cold_map[r] = nullptr;
+    }
+  if (c->h_cold) {
+    if (c->cold_shm[0]) {
+      cudaHostUnregister(c->h_cold);
+      munmap(c->h_cold, (size_t)c->cold_bytes);
+      shm_unlink(c->cold_shm);
+    } else {
+      cudaFreeHost(c->h_cold);
+    }
+    c->h_cold = nullptr;
+  }
+  cudaFree(c->d_fpos);
+  for (int i = 0; i < 3 * DSP_MAX_WORLD; ++i)
     if (c->ipc_opened[i]) {
       cudaIpcCloseMemHandle(c->ipc_opened[i]);
       c->ipc_opened[i] = nullptr;
@@ -855,6 +895,91 @@ dsp_status dsp_load_partition(dsp_ctx *c, const int64_t *bounds, const int64_t *
   return DSP_OK;
 }
 
+dsp_status dsp_load_features_tiered(dsp_ctx *c, const float *features, int32_t dim, int64_t hot_rows) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition (with features = NULL) first");
+  if (c->d_feat || c->tiered) return fail(c, DSP_ERR_STATE, "features already loaded");
+  if (c->reserved && c->world > 1) return fail(c, DSP_ERR_STATE, "load features before dsp_reserve");
+  if (!features && c->n_local > 0) return fail(c, DSP_ERR_INVALID_ARG, "features is NULL");
+  if (dim < 4 || dim > 4096 || dim % 4 != 0)
+    return fail(c, DSP_ERR_INVALID_ARG, "dim %d must be a multiple of 4 in [4, 4096]", dim);
+  const int64_t n = c->n_local;
+  if (hot_rows < 0 || hot_rows > n) hot_rows = n;
+  DeviceGuard g(c->device);
+  c->dim = dim;
+  c->feat_stride = (dim + FEAT_ALIGN_FLOATS - 1) / FEAT_ALIGN_FLOATS * FEAT_ALIGN_FLOATS;
+  const size_t row_bytes = sizeof(float) * (size_t)dim, stride_bytes = sizeof(float) * (size_t)c->feat_stride;
+  // hot rows: the hot_rows largest in-degrees (P:L114 default criterion), ties by id
+  std::vector<int64_t> ip((size_t)n + 1);
+  CUDA_TRY(c, cudaMemcpy(ip.data(), c->d_indptr, sizeof(int64_t) * (size_t)(n + 1), cudaMemcpyDeviceToHost));
+  std::vector<int32_t> order((size_t)n);
+  for (int64_t v = 0; v < n; ++v) order[(size_t)v] = (int32_t)v;
+  std::stable_sort(order.begin(), order.end(), [&](int32_t x, int32_t y) {
+    return ip[(size_t)x + 1] - ip[(size_t)x] > ip[(size_t)y + 1] - ip[(size_t)y];
+  });
+  std::vector<char> hot((size_t)n, 0);
+  for (int64_t j = 0; j < hot_rows; ++j) hot[(size_t)order[(size_t)j]] = 1;
+  std::vector<int32_t> fpos((size_t)n);
+  int64_t nh = 0, nc = 0;
+  for (int64_t v = 0; v < n; ++v) fpos[(size_t)v] = hot[(size_t)v] ? (int32_t)nh++ : (int32_t)(-(++nc));
+  // host staging of the rows (the input may live on the device)
+  std::vector<float> src;
+  const float *hsrc = features;
+  cudaPointerAttributes at;
+  if (n > 0 && cudaPointerGetAttributes(&at, features) == cudaSuccess &&
+      (at.type == cudaMemoryTypeDevice || at.type == cudaMemoryTypeManaged)) {
+    src.resize((size_t)n * dim);
+    CUDA_TRY(c, cudaMemcpy(src.data(), features, row_bytes * (size_t)n, cudaMemcpyDeviceToHost));
+    hsrc = src.data();
+  }
+  cudaGetLastError();
+  // hot rows -> HBM (padded stride), cold rows -> pinned host memory (UVA-mapped)
+  c->feat_bytes = (int64_t)stride_bytes * std::max<int64_t>(1, nh);
+  CUDA_TRY(c, cudaMalloc(&c->d_feat, (size_t)c->feat_bytes));
+  {
+    std::vector<float> stage((size_t)std::max<int64_t>(1, nh) * c->feat_stride, 0.0f);
+    for (int64_t v = 0; v < n; ++v)
+      if (fpos[(size_t)v] >= 0) memcpy(&stage[(size_t)fpos[(size_t)v] * c->feat_stride], hsrc + (size_t)v * dim, row_bytes);
+    CUDA_TRY(c, cudaMemcpy(c->d_feat, stage.data(), stride_bytes * (size_t)nh, cudaMemcpyHostToDevice));
+  }
+  c->cold_bytes = (int64_t)stride_bytes * std::max<int64_t>(1, nc);
+  if (c->world > 1) {  // cross-process readable: POSIX shm registered with CUDA
+    static int counter = 0;
+    snprintf(c->cold_shm, sizeof(c->cold_shm), "/dsp_cold_%d_%d_%d", (int)getpid(), c->rank, counter++);
+    int fd = shm_open(c->cold_shm, O_CREAT | O_EXCL | O_RDWR, 0600);
+    if (fd < 0) return fail(c, DSP_ERR_OOM, "shm_open(%s) failed", c->cold_shm);
+    if (ftruncate(fd, (off_t)c->cold_bytes) != 0) {
+      close(fd);
+      shm_unlink(c->cold_shm);
+      return fail(c, DSP_ERR_OOM, "ftruncate of the cold shm failed");
+    }
+    void *p = mmap(nullptr, (size_t)c->cold_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+    close(fd);
+    if (p == MAP_FAILED) {
+      shm_unlink(c->cold_shm);
+      return fail(c, DSP_ERR_OOM, "mmap of the cold shm failed");
+    }
+    c->h_cold = static_cast<float *>(p);
+    CUDA_TRY(c, cudaHostRegister(c->h_cold, (size_t)c->cold_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable));
+  } else {
+    CUDA_TRY(c, cudaHostAlloc((void **)&c->h_cold, (size_t)c->cold_bytes, cudaHostAllocMapped | cudaHostAllocPortable));
+  }
+  for (int64_t v = 0; v < n; ++v)
+    if (fpos[(size_t)v] < 0)
+      memcpy(c->h_cold + (size_t)(-fpos[(size_t)v] - 1) * c->feat_stride, hsrc + (size_t)v * dim, row_bytes);
+  CUDA_TRY(c, cudaMalloc(&c->d_fpos, sizeof(int32_t) * (size_t)std::max<int64_t>(1, n)));
+  if (n > 0) CUDA_TRY(c, cudaMemcpy(c->d_fpos, fpos.data(), sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice));
+  void *dev_cold = nullptr;
+  CUDA_TRY(c, cudaHostGetDevicePointer(&dev_cold, c->h_cold, 0));
+  c->tiered = true;
+  c->cold_regloads = getenv("DSP_COLD_REGLOADS") && atoi(getenv("DSP_COLD_REGLOADS")) != 0;
+  c->peer_feat[c->rank] = c->d_feat;
+  c->peer_fpos[c->rank] = nc > 0 ? c->d_fpos : nullptr;  // all hot: fpos is the identity
+  c->peer_cold[c->rank] = static_cast<const float *>(dev_cold);
+  return DSP_OK;
+}
+
 dsp_status dsp_load_weights(dsp_ctx *c, const float *edge_weights) {
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
@@ -953,6 +1078,14 @@ dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
     h.has_xch = 1;
     CUDA_TRY(c, cudaIpcGetMemHandle(&h.xch_ipc, c->d_xch));
   }
+  h.tiered = c->tiered ? 1 : 0;
+  if (c->tiered) {
+    h.fpos_ptr = (uint64_t)(uintptr_t)c->peer_fpos[c->rank];
+    h.cold_ptr = (uint64_t)(uintptr_t)c->peer_cold[c->rank];
+    h.cold_bytes = c->cold_bytes;
+    memcpy(h.cold_shm, c->cold_shm, sizeof(h.cold_shm));
+    if (c->world > 1 && h.fpos_ptr) CUDA_TRY(c, cudaIpcGetMemHandle(&h.fpos_ipc, c->d_fpos));
+  }
   memset(out, 0, DSP_HANDLE_BYTES);
   memcpy(out, &h, sizeof(h));
   return DSP_OK;
@@ -974,6 +1107,7 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
       if (h.bounds[q] != c->bounds[q]) return fail(c, DSP_ERR_STATE, "rank %d has different bounds", r);
     if (h.dim != c->dim || h.feat_stride != c->feat_stride || h.max_seeds != c->max_seeds)
       return fail(c, DSP_ERR_STATE, "rank %d has a different dim / max_seeds", r);
+    if ((h.tiered != 0) != c->tiered) return fail(c, DSP_ERR_STATE, "all ranks must use the cold tier or none");
     if (r == c->rank) continue;
     const bool same_process = h.pid == my_pid && h.boot_id == boot_id();
     if (same_process) {
@@ -988,7 +1122,36 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
       }
       c->peer_feat[r] = reinterpret_cast<const float *>(h.feat_ptr);
       c->peer_xch[r] = reinterpret_cast<char *>(h.xch_ptr);
+      if (h.tiered) {
+        c->peer_fpos[r] = reinterpret_cast<const int32_t *>(h.fpos_ptr);
+        c->peer_cold[r] = reinterpret_cast<const float *>(h.cold_ptr);
+      }
     } else {
+      if (h.tiered && h.fpos_ptr) {
+        void *p = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&p, h.fpos_ipc, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+          cudaGetLastError();
+          return fail(c, DSP_ERR_PEER, "cudaIpcOpenMemHandle(fpos of rank %d): %s", r, cudaGetErrorString(e));
+        }
+        c->ipc_opened[2 * DSP_MAX_WORLD + r] = p;
+        c->peer_fpos[r] = static_cast<const int32_t *>(p);
+        int fd = shm_open(h.cold_shm, O_RDWR, 0);
+        if (fd < 0) return fail(c, DSP_ERR_PEER, "shm_open(%s) of rank %d failed", h.cold_shm, r);
+        void *m = mmap(nullptr, (size_t)h.cold_bytes, PROT_READ | PROT_WRITE, MAP_SHARED, fd, 0);
+        close(fd);
+        if (m == MAP_FAILED) return fail(c, DSP_ERR_PEER, "mmap of rank %d's cold rows failed", r);
+        c->peer_cold_map[r] = m;
+        c->peer_cold_bytes[r] = h.cold_bytes;
+        e = cudaHostRegister(m, (size_t)h.cold_bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+        void *dp = nullptr;
+        if (e == cudaSuccess) e = cudaHostGetDevicePointer(&dp, m, 0);
+        if (e != cudaSuccess) {
+          cudaGetLastError();
+          return fail(c, DSP_ERR_PEER, "cudaHostRegister of rank %d's cold rows: %s", r, cudaGetErrorString(e));
+        }
+        c->peer_cold[r] = static_cast<const float *>(dp);
+      }
       if (h.has_feat) {
         void *p = nullptr;
         cudaError_t e = cudaIpcOpenMemHandle(&p, h.feat_ipc, cudaIpcMemLazyEnablePeerAccess);

@@ -32,7 +32,7 @@ DSP_HANDLE_BYTES = 512
 
 #: every symbol include/dsp.h declares
 ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_create", "dsp_destroy",
-               "dsp_load_partition", "dsp_load_weights", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
+               "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
                "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                "dsp_pipeline_flush", "dsp_set_persistent_blocks", "dsp_gather_features", "dsp_random_walk",
                "dsp_sync")
@@ -78,6 +78,7 @@ def lib(path: str | None = None):
         L.dsp_load_partition.argtypes = [P, P, P, P, P, i32]
         L.dsp_reserve.argtypes = [P, i32, P, i32]
         L.dsp_load_weights.argtypes = [P, P]
+        L.dsp_load_features_tiered.argtypes = [P, P, i32, i64]
         L.dsp_export_handle.argtypes = [P, P]
         L.dsp_import_handles.argtypes = [P, P]
         L.dsp_sample_bounds.argtypes = [P, i32, P, i32, P, P, ctypes.POINTER(ctypes.c_size_t)]
@@ -91,7 +92,7 @@ def lib(path: str | None = None):
         L.dsp_set_persistent_blocks.argtypes = [P, i32]
         L.dsp_random_walk.argtypes = [P, P, i64, i32, ctypes.c_uint64, P, P]
         L.dsp_sync.argtypes = [P, P]
-        for name in ("dsp_create", "dsp_load_partition", "dsp_load_weights", "dsp_reserve", "dsp_export_handle",
+        for name in ("dsp_create", "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve", "dsp_export_handle",
                      "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                      "dsp_pipeline_flush", "dsp_random_walk", "dsp_set_persistent_blocks",
                      "dsp_gather_features", "dsp_sync"):
@@ -155,6 +156,10 @@ def dsp_destroy(ctx) -> None:
 def dsp_load_partition(ctx, bounds, indptr, indices, features, dim: int) -> None:
     b = np.ascontiguousarray(bounds, dtype=np.int64)
     _check(lib().dsp_load_partition(ctx, _p(b), _p(indptr), _p(indices), _p(features), dim), ctx)
+
+
+def dsp_load_features_tiered(ctx, features, dim: int, hot_rows: int) -> None:
+    _check(lib().dsp_load_features_tiered(ctx, _p(features), dim, hot_rows), ctx)
 
 
 def dsp_load_weights(ctx, edge_weights) -> None:
@@ -258,7 +263,7 @@ class Sampler:
     def __init__(self, bounds, indptr, indices, features, fanouts, max_seeds: int, rank: int = 0,
                  world_size: int = 1, device: int | None = None,
                  exchange: Callable[[bytes], list] | None = None, connect: bool = True, n_slots: int = 1,
-                 edge_weights=None, n_workspaces: int = 1):
+                 edge_weights=None, n_workspaces: int = 1, hot_rows: int | None = None):
         import torch
         self.torch = torch
         self.device = torch.cuda.current_device() if device is None else device
@@ -268,7 +273,11 @@ class Sampler:
         self.dim = 0 if features is None else int(features.shape[1])
         self.ctx = dsp_create(rank, world_size, self.device)
         try:
-            dsp_load_partition(self.ctx, bounds, indptr, indices, features, self.dim)
+            if hot_rows is None:
+                dsp_load_partition(self.ctx, bounds, indptr, indices, features, self.dim)
+            else:  # cold-feature tier: hot_rows rows in HBM, the rest in host memory
+                dsp_load_partition(self.ctx, bounds, indptr, indices, None, 0)
+                dsp_load_features_tiered(self.ctx, features, self.dim, hot_rows)
             if edge_weights is not None:
                 dsp_load_weights(self.ctx, np.ascontiguousarray(edge_weights, np.float32)
                                  if isinstance(edge_weights, np.ndarray) else edge_weights)
@@ -408,12 +417,14 @@ class LocalGroup:
     issued rank by rank on the device's current stream) or sit on several
     GPUs of this node."""
 
-    def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int]):
-        """shards[r] = (indptr, indices, features[, edge_weights]) of rank r."""
+    def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int], hot_rows=None):
+        """shards[r] = (indptr, indices, features[, edge_weights]) of rank r;
+        hot_rows[r] (optional) enables the cold-feature tier."""
         P = len(shards)
         assert len(devices) == P and len(bounds) == P + 1
         self.samplers = [Sampler(bounds, s[0], s[1], s[2], fanouts, max_seeds, rank=r, world_size=P,
-                                 device=devices[r], connect=False, edge_weights=s[3] if len(s) > 3 else None)
+                                 device=devices[r], connect=False, edge_weights=s[3] if len(s) > 3 else None,
+                                 hot_rows=None if hot_rows is None else hot_rows[r])
                          for r, s in enumerate(shards)]
         handles = [dsp_export_handle(s.ctx) for s in self.samplers]
         for s in self.samplers:

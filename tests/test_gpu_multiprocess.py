@@ -23,7 +23,7 @@ def _free_port():
     return p
 
 
-def _rank(rank, world, port, q):
+def _rank(rank, world, port, q, hot=None):
     import sys
     here = os.path.dirname(os.path.abspath(__file__))
     sys.path[:0] = [os.path.dirname(here), here]
@@ -43,7 +43,8 @@ def _rank(rank, world, port, q):
         sip, six = datagen.shard(ip, ix, lo, hi)
         feats = datagen.features(lo, hi, cfg.dim)
         s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, 32, rank=rank, world_size=world, device=0,
-                        exchange=pkg.torch_exchange(), n_slots=2)
+                        exchange=pkg.torch_exchange(), n_slots=2,
+                        hot_rows=None if hot is None else (hi - lo) * hot // 4)
         train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
         batches = datagen.rank_seed_batches(train, bnds, rank, 32, 0)
         for step in range(3):
@@ -66,14 +67,17 @@ def _rank(rank, world, port, q):
         dist.destroy_process_group()
 
 
-def test_two_processes_one_gpu():
+@pytest.mark.parametrize("hot", [None, 1])
+def test_two_processes_one_gpu(hot):
+    """hot = 1: the cold-feature tier with 3/4 of each shard in host memory
+    (POSIX shm mapped into the peer process), read over UVA by both GPUs' gathers."""
     if not torch.cuda.is_available():
         pytest.fail("needs a GPU")
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_rank, args=(r, 2, port, q)) for r in range(2)]
+    procs = [ctx.Process(target=_rank, args=(r, 2, port, q, hot)) for r in range(2)]
     for p in procs:
         p.start()
     res = sorted(q.get(timeout=600) for _ in procs)
