@@ -96,6 +96,13 @@ def lib():
                                             ctypes.c_int32, ctypes.c_int32, ctypes.c_uint64, P, P]
         L.oracle_sample_ex.argtypes = [ctypes.c_int64, P, P, P, P, ctypes.c_int32, P, ctypes.c_int32,
                                        ctypes.c_uint64, ctypes.POINTER(_Block)]
+        L.oracle_draw_word_tag.argtypes = [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int32, ctypes.c_int32,
+                                           ctypes.c_uint32]
+        L.oracle_draw_word_tag.restype = ctypes.c_uint64
+        L.oracle_layer_alloc.argtypes = [ctypes.c_uint64, ctypes.c_int32, ctypes.c_int32, P, ctypes.c_int32,
+                                         ctypes.c_int32, P]
+        L.oracle_sample_layerwise.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, ctypes.c_int32,
+                                              ctypes.c_uint64, ctypes.POINTER(_Block)]
         L.oracle_random_walk.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, P]
         _lib = L
     return _lib
@@ -224,6 +231,41 @@ def sample(indptr, indices, seeds, fanouts, rng_seed: int, weights=None) -> list
                                 len(sd), _ptr(fo), L, rng_seed, blocks)
     if rc != OK:
         raise OracleError(rc, "oracle_sample")
+    out = [_block_to_numpy(blocks[l]) for l in range(L)]
+    for l in range(L):
+        lib().oracle_free_block(ctypes.byref(blocks[l]))
+    return out
+
+
+def draw_word_tag(rng_seed: int, slot: int, v: int, l: int, tag: int) -> int:
+    """x1:x0 of Philox({slot, v, l, tag}, seed)."""
+    return int(lib().oracle_draw_word_tag(rng_seed, slot, v, l, tag))
+
+
+def layer_alloc(rng_seed: int, g0: int, l: int, W, n: int) -> np.ndarray:
+    """Eq. 2 allocation: draw counts c[i] of n draws with
+    replacement over the frontier with probability W_i / sum W."""
+    w = _c(W, np.uint64)
+    c = np.zeros(max(1, len(w)), np.int32)
+    rc = lib().oracle_layer_alloc(rng_seed, g0, l, _ptr(w), len(w), n, _ptr(c))
+    if rc != OK:
+        raise OracleError(rc, "oracle_layer_alloc")
+    return c[:len(w)].copy()
+
+
+def sample_layerwise(indptr, indices, seeds, sizes, rng_seed: int) -> list[dict]:
+    """Multi-layer layer-wise sampling (Eq. 2 allocation + node-wise sampling
+    of c_u neighbours without replacement) for one rank's seeds."""
+    ip = _c(indptr, np.int64)
+    ix = _c(indices, np.int32)
+    sd = _c(seeds, np.int32)
+    sz = _c(sizes, np.int32)
+    L = len(sz)
+    blocks = (_Block * max(L, 1))()
+    rc = lib().oracle_sample_layerwise(len(ip) - 1, _ptr(ip), _ptr(ix), _ptr(sd), len(sd), _ptr(sz), L,
+                                       rng_seed, blocks)
+    if rc != OK:
+        raise OracleError(rc, "oracle_sample_layerwise")
     out = [_block_to_numpy(blocks[l]) for l in range(L)]
     for l in range(L):
         lib().oracle_free_block(ctypes.byref(blocks[l]))

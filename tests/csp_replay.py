@@ -105,3 +105,45 @@ def replay_distributed(indptr_shard, indices_shard, bounds, seeds, fanouts, rng_
         blocks.append(b)
         frontier = b["src_ids"]
     return blocks
+
+
+def replay_layerwise_inprocess(indptr, indices, bounds, rank_seeds, sizes, rng_seed):
+    """Layer-wise CSP replayed on P in-process ranks: per layer a
+    requester asks the owners for its frontier's degrees (W_u, shuffle), draws
+    the Eq. 2 allocation itself (``oracle.layer_alloc``), pushes (u, c_u) to
+    the owners, which sample c_u neighbours on their own shard
+    (``oracle.node_positions``), and builds its block from the returned rows."""
+    N = len(indptr) - 1
+    P = len(bounds) - 1
+    shards = [_shard(indptr, indices, int(bounds[o]), int(bounds[o + 1])) for o in range(P)]
+    frontier = [np.asarray(s, np.int32) for s in rank_seeds]
+    g0 = [int(s[0]) if len(s) else 0 for s in rank_seeds]
+    blocks = [[] for _ in range(P)]
+    for l, n in enumerate(sizes):
+        for r in range(P):
+            f = frontier[r]
+            own = owner_of(f, bounds)
+            # degree query at the owners
+            W = np.zeros(len(f), np.uint64)
+            for i, (v, o) in enumerate(zip(f.tolist(), own.tolist())):
+                ip, _, _ = shards[o]
+                lv = v - int(bounds[o])
+                W[i] = ip[lv + 1] - ip[lv]
+            c = oracle.layer_alloc(rng_seed, g0[r], l, W, n)
+            # sampling tasks pushed to the owners; rows come back in request order
+            width = max(1, int(c.max()) if len(c) else 1)
+            cnt = np.zeros(len(f), np.int32)
+            rows = np.full((len(f), width), -1, np.int32)
+            for i, (v, o) in enumerate(zip(f.tolist(), own.tolist())):
+                if c[i] == 0:
+                    continue
+                ip, ix, _ = shards[o]
+                lv = v - int(bounds[o])
+                s0, d = int(ip[lv]), int(ip[lv + 1] - ip[lv])
+                pos = oracle.node_positions(rng_seed, v, l, d, int(c[i]))
+                cnt[i] = len(pos)
+                rows[i, :len(pos)] = ix[s0 + pos]
+            b = oracle.build_block(N, f, cnt, rows)
+            blocks[r].append(b)
+            frontier[r] = b["src_ids"]
+    return blocks
