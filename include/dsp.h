@@ -47,7 +47,8 @@ extern "C" {
 #define DSP_MAX_WORLD 8      /* one NVSwitch node */
 #define DSP_MAX_LAYERS 8
 #define DSP_MAX_FANOUT 32    /* one lane per sampled slot */
-#define DSP_HANDLE_BYTES 512 /* size of an exported peer handle */
+#define DSP_HANDLE_BYTES 1024 /* size of an exported peer handle */
+#define DSP_MAX_LAYER_SIZE 8192 /* layer-wise: nodes sampled per layer (Table 7 uses 1000) */
 
 typedef enum {
   DSP_OK = 0,
@@ -132,6 +133,13 @@ dsp_status dsp_load_weights(dsp_ctx *ctx, const float *edge_weights);
    COLLECTIVE (identical arguments on every rank).  After dsp_load_partition. */
 dsp_status dsp_reserve(dsp_ctx *ctx, int32_t max_seeds, const int32_t *fanouts, int32_t num_layers);
 
+/* Layer-wise counterpart of dsp_reserve: sizes the peer-visible layer-wise
+   exchange region for batches of up to max_seeds seeds and layer sizes
+   sizes[num_layers] (HOST, each in [1, DSP_MAX_LAYER_SIZE]).  Needed for
+   DSP_LAYERWISE at every world size; with or without dsp_reserve; before
+   dsp_export_handle.  All ranks must pass the same values (checked at import). */
+dsp_status dsp_reserve_layerwise(dsp_ctx *ctx, int32_t max_seeds, const int32_t *sizes, int32_t num_layers);
+
 /* Peer handles (CUDA IPC for other processes, raw pointers within one
    process).  After dsp_reserve, every rank exports DSP_HANDLE_BYTES bytes;
    the caller all-gathers them (e.g. torch.distributed) into `all`
@@ -150,6 +158,17 @@ dsp_status dsp_import_handles(dsp_ctx *ctx, const void *all);
 #define DSP_ASYNC 1u
 #define DSP_PIPELINED 2u
 #define DSP_BIASED 4u
+/* DSP_LAYERWISE (dsp_sample, dsp_sample_group, dsp_sample_gather): `fanouts`
+   are LAYER SIZES n_l ("the total number of sampled nodes" per layer).
+   Per layer, the requester reads each frontier node's degree W_u from its
+   owner's indptr (peer memory), draws n_l times with replacement over its
+   frontier with probability W_u / sum W (Eq. 2; Philox counter
+   {j, seeds[0], l, "DSPL"}, R28-R30) and pushes (u, c_u) to the
+   owner, which samples min(c_u, deg u) neighbours of u without replacement
+   (the node-wise draws of layer l with fan-out c_u).  Blocks as node-wise
+   (dst first, then new nodes in first-occurrence order); E_l <= n_l.
+   Needs dsp_reserve_layerwise; not combinable with DSP_BIASED. */
+#define DSP_LAYERWISE 8u
 
 typedef struct {
   /* one sampled layer ("block"); arrays are DEVICE memory owned by the CALLER */
@@ -169,6 +188,12 @@ dsp_status dsp_sample_bounds(const dsp_ctx *ctx, int32_t num_seeds, const int32_
                              int32_t num_layers, int64_t *max_src, int64_t *max_edges,
                              size_t *workspace_bytes);
 
+/* Capacities of a DSP_LAYERWISE call: F_0 = num_seeds, max_edges[l] = n_l,
+   max_src[l] = min(N, F_l + n_l), F_{l+1} = max_src[l]; workspace as above. */
+dsp_status dsp_sample_bounds_layerwise(const dsp_ctx *ctx, int32_t num_seeds, const int32_t *sizes,
+                                       int32_t num_layers, int64_t *max_src, int64_t *max_edges,
+                                       size_t *workspace_bytes);
+
 /* CSP node-wise uniform sampling without replacement (DESIGN.md
    R1-R17).  COLLECTIVE: every rank calls with identical fanouts, num_layers
    and rng_seed; seeds differ per rank (0 seeds allowed; the rank still takes
@@ -181,7 +206,7 @@ dsp_status dsp_sample_bounds(const dsp_ctx *ctx, int32_t num_seeds, const int32_
               cover dsp_sample_bounds (else DSP_ERR_CAPACITY before any work).
               blocks[l].src_ids is the frontier of layer l+1; the last block's
               src_ids are the unique nodes whose features the loader needs.
-   flags    : 0 or DSP_BIASED.
+   flags    : 0, DSP_BIASED or DSP_LAYERWISE (then fanouts = layer sizes).
    workspace: DEVICE, 256-byte aligned, >= workspace_bytes from
               dsp_sample_bounds, ZERO-FILLED before its first use; afterwards
               it belongs to the library (it carries the relabel map's epoch

@@ -54,7 +54,8 @@ struct WsHeader {
   uint32_t bar_count;    // grid barrier arrivals
   uint32_t gcursor;      // next gather chunk (pipelined launches)
   uint32_t chunks_loader, chunks_helper;  // gather chunks done by loader / sampling warps
-  uint32_t pad[3];
+  uint32_t lw_big;       // layer-wise tasks with 32 < c < deg (owner side)
+  uint32_t pad[2];
   unsigned long long t[24];   // %globaltimer at kernel start and when block 0 leaves each grid barrier
   unsigned long long ta[24];  // %globaltimer when block 0 arrives at each grid barrier
   unsigned long long dbg[32]; // debug stamps (DSP_DEBUG_STAMPS builds only)

@@ -16,7 +16,7 @@
 #include <vector>
 
 #include "../../include/dsp.h"
-#include "dsp_kernels.cuh"
+#include "dsp_layerwise.cuh"
 
 using namespace dsp;
 
@@ -53,6 +53,10 @@ struct PeerHandle {  // fits in DSP_HANDLE_BYTES
   uint64_t fpos_ptr, cold_ptr;
   int64_t cold_bytes;
   char cold_shm[48];  // POSIX shm name of the cold rows (cross-process access)
+  // layer-wise exchange region + this rank's indptr (degree lookups)
+  cudaIpcMemHandle_t lxch_ipc, indptr_ipc;
+  uint64_t lxch_ptr, indptr_ptr;
+  int32_t has_lxch, lw_max_seeds, lw_L, lw_sizes[DSP_MAX_LAYERS];
 };
 static_assert(sizeof(PeerHandle) <= DSP_HANDLE_BYTES, "handle too large");
 
@@ -97,6 +101,9 @@ struct Plan {
   int64_t S[DSP_MAX_LAYERS];       // max src
   int64_t max_F, max_slots, status_len;
   size_t off_hdr, off_agg, off_cnt[2], off_perm, off_rows[2], off_status[2], off_first[2], bytes;
+  // layer-wise scheme (make_plan_lw)
+  int64_t ncap, big_cap;
+  size_t off_P, off_c, off_off, off_slot_node, off_excl, off_newid, off_big;
 };
 
 }  // namespace
@@ -133,8 +140,16 @@ struct dsp_ctx {
   // peers
   const float *peer_feat[DSP_MAX_WORLD] = {nullptr};
   char *peer_xch[DSP_MAX_WORLD] = {nullptr};
-  void *ipc_opened[3 * DSP_MAX_WORLD] = {nullptr};  // feat, xch, fpos per peer
+  void *ipc_opened[5 * DSP_MAX_WORLD] = {nullptr};  // feat, xch | fpos | lxch | indptr per peer
   unsigned long long seq = 0;
+  // layer-wise scheme (dsp_reserve_layerwise)
+  bool lw_reserved = false;
+  int32_t lw_max_seeds = 0, lw_L = 0;
+  int32_t lw_sizes[DSP_MAX_LAYERS] = {0};
+  LwLayout lxl{};
+  char *d_lxch = nullptr;
+  char *peer_lxch[DSP_MAX_WORLD] = {nullptr};
+  const int64_t *peer_indptr[DSP_MAX_WORLD] = {nullptr};
   // host staging (pinned)
   WsHeader *h_hdr = nullptr;
   int *h_err = nullptr;
@@ -212,6 +227,20 @@ dsp_status check_fanouts(dsp_ctx *c, const int32_t *fanouts, int32_t L) {
   return DSP_OK;
 }
 
+// persist | hdr | first[2][N] at fixed offsets for every plan, so that one
+// workspace can serve calls of any size and either scheme (the relabel map's
+// epoch words stay valid across them).
+size_t plan_common(Plan &p, int64_t N) {
+  size_t o = align_up(sizeof(WsPersist), 256);
+  p.off_hdr = o;
+  o = align_up(o + sizeof(WsHeader), 256);
+  for (int b = 0; b < 2; ++b) {
+    p.off_first[b] = o;
+    o = align_up(o + sizeof(unsigned long long) * std::max<int64_t>(1, N), 256);
+  }
+  return o;
+}
+
 Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L) {
   Plan p{};
   p.L = L;
@@ -226,9 +255,7 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L) {
     p.max_slots = std::max(p.max_slots, p.E[l]);
   }
   p.status_len = align_up((size_t)((p.max_slots + SCAN_TILE - 1) / SCAN_TILE + 2), 2);
-  size_t o = align_up(sizeof(WsPersist), 256);
-  p.off_hdr = o;
-  o = align_up(o + sizeof(WsHeader), 256);
+  size_t o = plan_common(p, N);
   p.off_agg = o;
   o = align_up(o + sizeof(unsigned long long) * 2 * MAX_PERSIST_BLOCKS, 256);
   for (int b = 0; b < 2; ++b) {
@@ -245,12 +272,58 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L) {
     p.off_status[b] = o;
     o = align_up(o + sizeof(unsigned long long) * p.status_len, 256);
   }
-  for (int b = 0; b < 2; ++b) {
-    p.off_first[b] = o;
-    o = align_up(o + sizeof(unsigned long long) * std::max<int64_t>(1, N), 256);
-  }
   p.bytes = o;
   return p;
+}
+
+// Layer-wise (R28): E_l <= n_l, max_src[l] = min(N, F_l + n_l).
+Plan make_plan_lw(int64_t N, int64_t num_seeds, const int32_t *sizes, int L) {
+  Plan p{};
+  p.L = L;
+  p.F[0] = num_seeds;
+  p.max_F = std::max<int64_t>(1, num_seeds);
+  p.ncap = 1;
+  for (int l = 0; l < L; ++l) {
+    p.E[l] = sizes[l];
+    p.S[l] = std::max<int64_t>(p.F[l], std::min<int64_t>(N, p.F[l] + p.E[l]));
+    p.F[l + 1] = p.S[l];
+    p.max_F = std::max(p.max_F, p.F[l]);
+    p.ncap = std::max<int64_t>(p.ncap, sizes[l]);
+  }
+  p.big_cap = 8 * (p.ncap / 32) + 8;
+  size_t o = plan_common(p, N);
+  auto take = [&](size_t &off, size_t bytes) {
+    off = o;
+    o = align_up(o + bytes, 256);
+  };
+  take(p.off_P, sizeof(unsigned long long) * (size_t)(p.max_F + 1));
+  take(p.off_c, sizeof(int32_t) * (size_t)p.max_F);
+  take(p.off_off, sizeof(int32_t) * (size_t)(p.max_F + 1));
+  take(p.off_slot_node, sizeof(int32_t) * (size_t)p.ncap);
+  take(p.off_excl, sizeof(int32_t) * (size_t)(p.ncap + 1));
+  take(p.off_newid, sizeof(int32_t) * (size_t)p.ncap);
+  take(p.off_big, sizeof(int2) * (size_t)p.big_cap);
+  p.bytes = o;
+  return p;
+}
+
+LwLayout make_lw_layout(int64_t cap, int32_t ncap) {
+  LwLayout x{};
+  x.cap = cap;
+  x.ncap = ncap;
+  size_t o = 0;
+  auto take = [&](size_t &off, size_t bytes) {
+    off = o;
+    o = align_up(o + bytes, 256);
+  };
+  take(x.off_inbox_flag, sizeof(unsigned long long) * 16);
+  take(x.off_ret_flag, sizeof(unsigned long long) * 16);
+  take(x.off_inbox_hdr, sizeof(uint4) * 16);
+  take(x.off_inbox, sizeof(int4) * 16 * (size_t)cap);
+  take(x.off_ret_cnt, sizeof(int32_t) * 2 * (size_t)cap);
+  take(x.off_ret_rows, sizeof(int32_t) * 2 * (size_t)ncap);
+  x.bytes = o;
+  return x;
 }
 
 XchLayout make_xch_layout(int64_t cap, int kmax) {
@@ -325,6 +398,7 @@ struct Call {
   bool async;
   bool pipelined;      // gather this call's rows in the next pipelined call / flush
   bool biased;         // DSP_BIASED
+  bool layerwise;      // DSP_LAYERWISE: fanouts are layer sizes
 };
 
 LayerBufs bufs_of(const Call &k, int parity) {
@@ -338,6 +412,66 @@ LayerBufs bufs_of(const Call &k, int parity) {
 
 WsPersist *persist_of(const Call &k) { return reinterpret_cast<WsPersist *>(k.ws); }
 
+dsp_status check_sizes(dsp_ctx *c, const int32_t *sizes, int32_t L) {
+  if (L < 1 || L > DSP_MAX_LAYERS || !sizes)
+    return fail(c, DSP_ERR_INVALID_ARG, "num_layers must be in [1, %d]", DSP_MAX_LAYERS);
+  for (int l = 0; l < L; ++l)
+    if (sizes[l] < 1 || sizes[l] > DSP_MAX_LAYER_SIZE)
+      return fail(c, DSP_ERR_INVALID_ARG, "layer size %d = %d not in [1, %d]", l, sizes[l], DSP_MAX_LAYER_SIZE);
+  return DSP_OK;
+}
+
+dsp_status check_blocks(dsp_ctx *c, const Plan &p, const dsp_block *blocks, int L) {
+  for (int l = 0; l < L; ++l) {
+    if ((uint64_t)p.F[l] + (uint64_t)p.E[l] >= (1ull << 31))
+      return fail(c, DSP_ERR_CAPACITY, "layer %d: frontier + edges exceeds 2^31", l);
+    if (!blocks[l].indptr || !blocks[l].indices || !blocks[l].src_ids)
+      return fail(c, DSP_ERR_INVALID_ARG, "blocks[%d] has a NULL array", l);
+    if (blocks[l].cap_indptr < p.F[l] + 1 || blocks[l].cap_edges < p.E[l] || blocks[l].cap_src < p.S[l])
+      return fail(c, DSP_ERR_CAPACITY, "blocks[%d] capacities (%lld, %lld, %lld) < bounds (%lld, %lld, %lld)", l,
+                  (long long)blocks[l].cap_indptr, (long long)blocks[l].cap_edges, (long long)blocks[l].cap_src,
+                  (long long)(p.F[l] + 1), (long long)p.E[l], (long long)p.S[l]);
+  }
+  return DSP_OK;
+}
+
+// DSP_LAYERWISE: needs dsp_reserve_layerwise with the same sizes.
+dsp_status prepare_call_lw(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_seeds, const int32_t *sizes,
+                           int32_t L, uint64_t rng_seed, dsp_block *blocks, void *workspace, size_t ws_bytes,
+                           void *stream) {
+  if (k.biased) return fail(c, DSP_ERR_INVALID_ARG, "DSP_LAYERWISE with DSP_BIASED is not supported");
+  if (c->broken) return fail(c, DSP_ERR_STATE, "ctx unusable after an earlier exchange failure");
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition not called");
+  if (!c->lw_reserved) return fail(c, DSP_ERR_STATE, "DSP_LAYERWISE needs dsp_reserve_layerwise first");
+  if (c->world > 1 && !c->imported) return fail(c, DSP_ERR_STATE, "world_size > 1 needs dsp_import_handles first");
+  dsp_status st = check_sizes(c, sizes, L);
+  if (st != DSP_OK) return st;
+  if (num_seeds < 0 || (num_seeds > 0 && !seeds)) return fail(c, DSP_ERR_INVALID_ARG, "bad seeds / num_seeds");
+  if (!blocks || !workspace) return fail(c, DSP_ERR_INVALID_ARG, "blocks / workspace is NULL");
+  if (num_seeds > c->lw_max_seeds)
+    return fail(c, DSP_ERR_CAPACITY, "num_seeds %d > reserved max_seeds %d", num_seeds, c->lw_max_seeds);
+  if (L != c->lw_L) return fail(c, DSP_ERR_STATE, "num_layers %d != reserved %d", L, c->lw_L);
+  for (int l = 0; l < L; ++l)
+    if (sizes[l] != c->lw_sizes[l])
+      return fail(c, DSP_ERR_STATE, "layer size %d = %d != reserved %d", l, sizes[l], c->lw_sizes[l]);
+  k.plan = make_plan_lw(c->N, c->lw_max_seeds, sizes, L);
+  if (ws_bytes < k.plan.bytes)
+    return fail(c, DSP_ERR_CAPACITY, "workspace %zu B < required %zu B", ws_bytes, k.plan.bytes);
+  if (((uintptr_t)workspace & 255u) != 0) return fail(c, DSP_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
+  if ((st = check_blocks(c, k.plan, blocks, L)) != DSP_OK) return st;
+  k.seeds = seeds;
+  k.num_seeds = num_seeds;
+  k.fanouts = sizes;
+  k.L = L;
+  k.rng_seed = rng_seed;
+  k.blocks = blocks;
+  k.ws = static_cast<char *>(workspace);
+  k.stream = static_cast<cudaStream_t>(stream);
+  k.hdr = reinterpret_cast<WsHeader *>(k.ws + k.plan.off_hdr);
+  k.seq0 = c->seq;
+  return DSP_OK;
+}
+
 dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_seeds,
                         const int32_t *fanouts, int32_t L, uint64_t rng_seed, dsp_block *blocks,
                         void *workspace, size_t ws_bytes, uint32_t flags, void *stream) {
@@ -345,9 +479,12 @@ dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_s
   k.c = c;
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
-  if ((flags & ~(DSP_ASYNC | DSP_PIPELINED | DSP_BIASED)) != 0)
+  if ((flags & ~(DSP_ASYNC | DSP_PIPELINED | DSP_BIASED | DSP_LAYERWISE)) != 0)
     return fail(c, DSP_ERR_INVALID_ARG, "unknown flags 0x%x", flags);
   k.biased = (flags & DSP_BIASED) != 0;
+  k.layerwise = (flags & DSP_LAYERWISE) != 0;
+  if (k.layerwise) return prepare_call_lw(k, c, seeds, num_seeds, fanouts, L, rng_seed, blocks, workspace,
+                                          ws_bytes, stream);
   if (k.biased && !c->d_weights) return fail(c, DSP_ERR_STATE, "DSP_BIASED needs dsp_load_weights first");
   if (c->broken) return fail(c, DSP_ERR_STATE, "ctx unusable after an earlier exchange failure");
   if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition not called");
@@ -613,6 +750,80 @@ dsp_status stage_scan_indices(Call &k, int l) {
   return DSP_OK;
 }
 
+// ------------------------------------------------ layer-wise stages
+LwArgs lw_args(Call &k, int l) {
+  dsp_ctx *c = k.c;
+  LwArgs a{};
+  a.seeds = k.seeds;
+  a.frontier = frontier_of(k, l);
+  a.F0 = k.num_seeds;
+  a.layer = l;
+  a.n = k.fanouts[l];
+  a.rank = c->rank;
+  a.seq = k.seq0 + 1 + l;
+  a.parity = (int)(a.seq & 1);
+  a.key = key_of(k.rng_seed);
+  a.bd = make_bounds(c);
+  for (int r = 0; r < DSP_MAX_WORLD; ++r) {
+    a.peer_indptr[r] = r < c->world ? c->peer_indptr[r] : nullptr;
+    a.peers.base[r] = r < c->world ? c->peer_lxch[r] : nullptr;
+  }
+  a.indptr = c->d_indptr;
+  a.indices = c->d_indices;
+  a.lo = c->lo;
+  a.n_local = c->n_local;
+  a.L = c->lxl;
+  a.w.P = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_P);
+  a.w.c = reinterpret_cast<int32_t *>(k.ws + k.plan.off_c);
+  a.w.off = reinterpret_cast<int32_t *>(k.ws + k.plan.off_off);
+  a.w.slot_node = reinterpret_cast<int32_t *>(k.ws + k.plan.off_slot_node);
+  a.w.excl = reinterpret_cast<int32_t *>(k.ws + k.plan.off_excl);
+  a.w.newid = reinterpret_cast<int32_t *>(k.ws + k.plan.off_newid);
+  a.w.big = reinterpret_cast<int2 *>(k.ws + k.plan.off_big);
+  a.w.big_cap = (int32_t)k.plan.big_cap;
+  a.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_first[l & 1]);
+  a.persist = persist_of(k);
+  a.out.indptr[0] = k.blocks[l].indptr;
+  a.out.indices[0] = k.blocks[l].indices;
+  a.out.src_ids[0] = k.blocks[l].src_ids;
+  a.hdr = k.hdr;
+  a.err = c->d_err;
+  return a;
+}
+
+dsp_status stage_lw(Call &k, int l, int step) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  const LwArgs a = lw_args(k, l);
+  const int64_t F = k.plan.F[l], n = k.fanouts[l];
+  switch (step) {
+    case 0:
+      k_lw_alloc<<<1, LWT, 0, k.stream>>>(a);
+      break;
+    case 1: {  // one warp per task; at most world * F tasks arrive
+      const int64_t need = std::max<int64_t>(1, (c->world * F + NT / 32 - 1) / (NT / 32));
+      k_lw_sample_remote<<<(int)std::min<int64_t>(need, grid_for(c, 8)), NT, 0, k.stream>>>(a);
+      break;
+    }
+    case 2: {
+      const int kp = (int)next_pow2(k.plan.ncap);
+      k_lw_sample_big<<<(int)std::min<int64_t>(k.plan.big_cap, c->num_sms), LWT,
+                        sizeof(int32_t) * 3 * (size_t)kp, k.stream>>>(a, kp);
+      break;
+    }
+    case 3: {
+      const int64_t need = std::max<int64_t>(1, (std::max(F, n) + NT - 1) / NT);
+      k_lw_collect<<<(int)std::min<int64_t>(need, grid_for(c, 8)), NT, 0, k.stream>>>(a);
+      break;
+    }
+    default:
+      k_lw_finish<<<1, LWT, 0, k.stream>>>(a);
+      break;
+  }
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
 dsp_status stage_gather_dev(Call &k) {
   dsp_ctx *c = k.c;
   DeviceGuard g(c->device);
@@ -671,14 +882,18 @@ dsp_status run_calls(std::vector<Call> &calls) {
   for (auto &k : calls)                               \
     if ((st = (STAGE)) != DSP_OK) return st;
   // a non-pipelined call first settles a pending pipelined gather; so does a
-  // pipelined call of the stage-by-stage path (no loader warps there)
+  // pipelined call of the stage-by-stage paths (no loader warps there)
   for (auto &k : calls)
-    if ((!k.pipelined || k.c->world > 1) && (st = stage_flush(k.c, k.ws)) != DSP_OK) return st;
+    if ((!k.pipelined || k.c->world > 1 || k.layerwise) && (st = stage_flush(k.c, k.ws)) != DSP_OK) return st;
   EACH(stage_begin(k));
-  if (calls[0].c->world == 1) {
+  if (calls[0].c->world == 1 && !calls[0].layerwise) {
     EACH(stage_persistent(k));
   } else {
     for (int l = 0; l < calls[0].L; ++l) {
+      if (calls[0].layerwise) {
+        for (int step = 0; step < 5; ++step) EACH(stage_lw(k, l, step));
+        continue;
+      }
       EACH(stage_clear(k, l));
       EACH(stage_shuffle(k, l));
       EACH(stage_sample_remote(k, l));
@@ -736,7 +951,7 @@ void release(dsp_ctx *c) {
     c->h_cold = nullptr;
   }
   cudaFree(c->d_fpos);
-  for (int i = 0; i < 3 * DSP_MAX_WORLD; ++i)
+  for (int i = 0; i < 5 * DSP_MAX_WORLD; ++i)
     if (c->ipc_opened[i]) {
       cudaIpcCloseMemHandle(c->ipc_opened[i]);
       c->ipc_opened[i] = nullptr;
@@ -746,6 +961,7 @@ void release(dsp_ctx *c) {
   cudaFree(c->d_weights);
   cudaFree(c->d_feat);
   cudaFree(c->d_xch);
+  cudaFree(c->d_lxch);
   cudaFree(c->d_err);
   if (c->h_hdr) cudaFreeHost(c->h_hdr);
   if (c->h_err) cudaFreeHost(c->h_err);
@@ -819,6 +1035,12 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
     cudaGetLastError();
     delete c;
     return fail(nullptr, DSP_ERR_CUDA, "occupancy query for the persistent kernel failed");
+  }
+  if (cudaFuncSetAttribute((const void *)k_lw_sample_big, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           (int)sizeof(int32_t) * 3 * LW_MAX_SIZE) != cudaSuccess) {
+    cudaGetLastError();
+    delete c;
+    return fail(nullptr, DSP_ERR_CUDA, "shared-memory attribute of the layer-wise kernel failed");
   }
   c->persist_blocks_per_sm = std::min(occ, occ_pipe);
   if (c->persist_blocks_per_sm * c->num_sms > MAX_PERSIST_BLOCKS) c->persist_blocks_per_sm = MAX_PERSIST_BLOCKS / c->num_sms;
@@ -1048,11 +1270,59 @@ dsp_status dsp_reserve(dsp_ctx *c, int32_t max_seeds, const int32_t *fanouts, in
   return DSP_OK;
 }
 
+dsp_status dsp_reserve_layerwise(dsp_ctx *c, int32_t max_seeds, const int32_t *sizes, int32_t L) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
+  if (c->lw_reserved) return fail(c, DSP_ERR_STATE, "layer-wise already reserved");
+  if (c->imported) return fail(c, DSP_ERR_STATE, "reserve before dsp_import_handles");
+  dsp_status st = check_sizes(c, sizes, L);
+  if (st != DSP_OK) return st;
+  if (max_seeds < 0) return fail(c, DSP_ERR_INVALID_ARG, "max_seeds < 0");
+  Plan p = make_plan_lw(c->N, max_seeds, sizes, L);
+  for (int l = 0; l < L; ++l)
+    if ((uint64_t)p.F[l] + (uint64_t)p.E[l] >= (1ull << 31))
+      return fail(c, DSP_ERR_CAPACITY, "layer %d: frontier + layer size exceeds 2^31", l);
+  DeviceGuard g(c->device);
+  c->lxl = make_lw_layout(std::max<int64_t>(1, p.max_F), (int32_t)p.ncap);
+  CUDA_TRY(c, cudaMalloc(&c->d_lxch, c->lxl.bytes));
+  CUDA_TRY(c, cudaMemset(c->d_lxch, 0, c->lxl.bytes));
+  CUDA_TRY(c, cudaDeviceSynchronize());
+  c->lw_max_seeds = max_seeds;
+  c->lw_L = L;
+  for (int l = 0; l < L; ++l) c->lw_sizes[l] = sizes[l];
+  c->peer_lxch[c->rank] = c->d_lxch;
+  c->peer_indptr[c->rank] = c->d_indptr;
+  c->lw_reserved = true;
+  return DSP_OK;
+}
+
+dsp_status dsp_sample_bounds_layerwise(const dsp_ctx *cc, int32_t num_seeds, const int32_t *sizes, int32_t L,
+                                       int64_t *max_src, int64_t *max_edges, size_t *workspace_bytes) {
+  dsp_ctx *c = const_cast<dsp_ctx *>(cc);
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
+  dsp_status st = check_sizes(c, sizes, L);
+  if (st != DSP_OK) return st;
+  if (num_seeds < 0) return fail(c, DSP_ERR_INVALID_ARG, "num_seeds < 0");
+  if (c->lw_reserved && num_seeds > c->lw_max_seeds)
+    return fail(c, DSP_ERR_CAPACITY, "num_seeds %d > reserved max_seeds %d", num_seeds, c->lw_max_seeds);
+  Plan p = make_plan_lw(c->N, c->lw_reserved ? c->lw_max_seeds : num_seeds, sizes, L);
+  for (int l = 0; l < L; ++l) {
+    if (max_src) max_src[l] = p.S[l];
+    if (max_edges) max_edges[l] = p.E[l];
+  }
+  if (workspace_bytes) *workspace_bytes = p.bytes;
+  return DSP_OK;
+}
+
 dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
   dsp_ctx *c = const_cast<dsp_ctx *>(cc);
   if (!c || !out) return DSP_ERR_INVALID_ARG;
   c->err.clear();
-  if (!c->loaded || !c->reserved) return fail(c, DSP_ERR_STATE, "load_partition + reserve first");
+  if (!c->loaded || !(c->reserved || c->lw_reserved))
+    return fail(c, DSP_ERR_STATE, "load_partition + reserve first");
   PeerHandle h;
   memset(&h, 0, sizeof(h));
   h.magic = HANDLE_MAGIC;
@@ -1086,6 +1356,18 @@ dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
     memcpy(h.cold_shm, c->cold_shm, sizeof(h.cold_shm));
     if (c->world > 1 && h.fpos_ptr) CUDA_TRY(c, cudaIpcGetMemHandle(&h.fpos_ipc, c->d_fpos));
   }
+  h.lw_max_seeds = c->lw_reserved ? c->lw_max_seeds : -1;
+  h.lw_L = c->lw_L;
+  for (int l = 0; l < DSP_MAX_LAYERS; ++l) h.lw_sizes[l] = c->lw_sizes[l];
+  if (c->lw_reserved) {
+    h.has_lxch = 1;
+    h.lxch_ptr = (uint64_t)(uintptr_t)c->d_lxch;
+    h.indptr_ptr = (uint64_t)(uintptr_t)c->d_indptr;
+    if (c->world > 1) {
+      CUDA_TRY(c, cudaIpcGetMemHandle(&h.lxch_ipc, c->d_lxch));
+      CUDA_TRY(c, cudaIpcGetMemHandle(&h.indptr_ipc, c->d_indptr));
+    }
+  }
   memset(out, 0, DSP_HANDLE_BYTES);
   memcpy(out, &h, sizeof(h));
   return DSP_OK;
@@ -1094,7 +1376,8 @@ dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
 dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
   if (!c || !all) return DSP_ERR_INVALID_ARG;
   c->err.clear();
-  if (!c->loaded || !c->reserved) return fail(c, DSP_ERR_STATE, "load_partition + reserve first");
+  if (!c->loaded || !(c->reserved || c->lw_reserved))
+    return fail(c, DSP_ERR_STATE, "load_partition + reserve first");
   if (c->imported) return fail(c, DSP_ERR_STATE, "handles already imported");
   DeviceGuard g(c->device);
   const int64_t my_pid = (int64_t)getpid();
@@ -1108,6 +1391,9 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
     if (h.dim != c->dim || h.feat_stride != c->feat_stride || h.max_seeds != c->max_seeds)
       return fail(c, DSP_ERR_STATE, "rank %d has a different dim / max_seeds", r);
     if ((h.tiered != 0) != c->tiered) return fail(c, DSP_ERR_STATE, "all ranks must use the cold tier or none");
+    if (h.lw_max_seeds != (c->lw_reserved ? c->lw_max_seeds : -1) || h.lw_L != c->lw_L ||
+        memcmp(h.lw_sizes, c->lw_sizes, sizeof(c->lw_sizes)) != 0)
+      return fail(c, DSP_ERR_STATE, "rank %d reserved a different layer-wise configuration", r);
     if (r == c->rank) continue;
     const bool same_process = h.pid == my_pid && h.boot_id == boot_id();
     if (same_process) {
@@ -1126,7 +1412,27 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
         c->peer_fpos[r] = reinterpret_cast<const int32_t *>(h.fpos_ptr);
         c->peer_cold[r] = reinterpret_cast<const float *>(h.cold_ptr);
       }
+      if (h.has_lxch) {
+        c->peer_lxch[r] = reinterpret_cast<char *>(h.lxch_ptr);
+        c->peer_indptr[r] = reinterpret_cast<const int64_t *>(h.indptr_ptr);
+      }
     } else {
+      if (h.has_lxch) {
+        void *p = nullptr, *q = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&p, h.lxch_ipc, cudaIpcMemLazyEnablePeerAccess);
+        if (e == cudaSuccess) {
+          c->ipc_opened[3 * DSP_MAX_WORLD + r] = p;
+          e = cudaIpcOpenMemHandle(&q, h.indptr_ipc, cudaIpcMemLazyEnablePeerAccess);
+        }
+        if (e != cudaSuccess) {
+          cudaGetLastError();
+          return fail(c, DSP_ERR_PEER, "cudaIpcOpenMemHandle(layer-wise region / indptr of rank %d): %s", r,
+                      cudaGetErrorString(e));
+        }
+        c->ipc_opened[4 * DSP_MAX_WORLD + r] = q;
+        c->peer_lxch[r] = static_cast<char *>(p);
+        c->peer_indptr[r] = static_cast<const int64_t *>(q);
+      }
       if (h.tiered && h.fpos_ptr) {
         void *p = nullptr;
         cudaError_t e = cudaIpcOpenMemHandle(&p, h.fpos_ipc, cudaIpcMemLazyEnablePeerAccess);

@@ -28,17 +28,19 @@ DSP_ERR_OOM = -8
 DSP_MAX_WORLD = 8
 DSP_MAX_LAYERS = 8
 DSP_MAX_FANOUT = 32
-DSP_HANDLE_BYTES = 512
+DSP_HANDLE_BYTES = 1024
+DSP_MAX_LAYER_SIZE = 8192
 
 #: every symbol include/dsp.h declares
 ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_create", "dsp_destroy",
-               "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve", "dsp_export_handle", "dsp_import_handles",
-               "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
+               "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve", "dsp_reserve_layerwise", "dsp_export_handle", "dsp_import_handles",
+               "dsp_sample_bounds", "dsp_sample_bounds_layerwise", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                "dsp_pipeline_flush", "dsp_set_persistent_blocks", "dsp_gather_features", "dsp_random_walk",
                "dsp_sync")
 DSP_ASYNC = 1
 DSP_PIPELINED = 2
 DSP_BIASED = 4
+DSP_LAYERWISE = 8
 
 
 class DSPError(RuntimeError):
@@ -79,6 +81,8 @@ def lib(path: str | None = None):
         L.dsp_reserve.argtypes = [P, i32, P, i32]
         L.dsp_load_weights.argtypes = [P, P]
         L.dsp_load_features_tiered.argtypes = [P, P, i32, i64]
+        L.dsp_reserve_layerwise.argtypes = [P, i32, P, i32]
+        L.dsp_sample_bounds_layerwise.argtypes = [P, i32, P, i32, P, P, ctypes.POINTER(ctypes.c_size_t)]
         L.dsp_export_handle.argtypes = [P, P]
         L.dsp_import_handles.argtypes = [P, P]
         L.dsp_sample_bounds.argtypes = [P, i32, P, i32, P, P, ctypes.POINTER(ctypes.c_size_t)]
@@ -92,7 +96,8 @@ def lib(path: str | None = None):
         L.dsp_set_persistent_blocks.argtypes = [P, i32]
         L.dsp_random_walk.argtypes = [P, P, i64, i32, ctypes.c_uint64, P, P]
         L.dsp_sync.argtypes = [P, P]
-        for name in ("dsp_create", "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve", "dsp_export_handle",
+        for name in ("dsp_create", "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve",
+                     "dsp_reserve_layerwise", "dsp_sample_bounds_layerwise", "dsp_export_handle",
                      "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                      "dsp_pipeline_flush", "dsp_random_walk", "dsp_set_persistent_blocks",
                      "dsp_gather_features", "dsp_sync"):
@@ -169,6 +174,20 @@ def dsp_load_weights(ctx, edge_weights) -> None:
 def dsp_reserve(ctx, max_seeds: int, fanouts) -> None:
     f = _i32_array(fanouts)
     _check(lib().dsp_reserve(ctx, max_seeds, _p(f), len(f)), ctx)
+
+
+def dsp_reserve_layerwise(ctx, max_seeds: int, sizes) -> None:
+    f = _i32_array(sizes)
+    _check(lib().dsp_reserve_layerwise(ctx, max_seeds, _p(f), len(f)), ctx)
+
+
+def dsp_sample_bounds_layerwise(ctx, num_seeds: int, sizes):
+    f = _i32_array(sizes)
+    ms = np.zeros(len(f), np.int64)
+    me = np.zeros(len(f), np.int64)
+    ws = ctypes.c_size_t(0)
+    _check(lib().dsp_sample_bounds_layerwise(ctx, num_seeds, _p(f), len(f), _p(ms), _p(me), ctypes.byref(ws)), ctx)
+    return ms, me, ws.value
 
 
 def dsp_export_handle(ctx) -> bytes:
@@ -263,11 +282,14 @@ class Sampler:
     def __init__(self, bounds, indptr, indices, features, fanouts, max_seeds: int, rank: int = 0,
                  world_size: int = 1, device: int | None = None,
                  exchange: Callable[[bytes], list] | None = None, connect: bool = True, n_slots: int = 1,
-                 edge_weights=None, n_workspaces: int = 1, hot_rows: int | None = None):
+                 edge_weights=None, n_workspaces: int = 1, hot_rows: int | None = None, scheme: str = "node"):
         import torch
         self.torch = torch
         self.device = torch.cuda.current_device() if device is None else device
         self.rank, self.world = rank, world_size
+        assert scheme in ("node", "layer")
+        self.scheme = scheme          # "layer": fanouts are layer sizes (DSP_LAYERWISE)
+        self._sflag = DSP_LAYERWISE if scheme == "layer" else 0
         self.fanouts = [int(k) for k in fanouts]
         self.max_seeds = int(max_seeds)
         self.dim = 0 if features is None else int(features.shape[1])
@@ -281,8 +303,12 @@ class Sampler:
             if edge_weights is not None:
                 dsp_load_weights(self.ctx, np.ascontiguousarray(edge_weights, np.float32)
                                  if isinstance(edge_weights, np.ndarray) else edge_weights)
-            dsp_reserve(self.ctx, self.max_seeds, self.fanouts)
-            ms, me, ws = dsp_sample_bounds(self.ctx, self.max_seeds, self.fanouts)
+            if scheme == "layer":
+                dsp_reserve_layerwise(self.ctx, self.max_seeds, self.fanouts)
+                ms, me, ws = dsp_sample_bounds_layerwise(self.ctx, self.max_seeds, self.fanouts)
+            else:
+                dsp_reserve(self.ctx, self.max_seeds, self.fanouts)
+                ms, me, ws = dsp_sample_bounds(self.ctx, self.max_seeds, self.fanouts)
         except Exception:
             dsp_destroy(self.ctx)
             self.ctx = None
@@ -324,7 +350,7 @@ class Sampler:
         torch = self.torch
         assert seeds.dtype == torch.int32 and seeds.is_cuda and seeds.is_contiguous()
         dsp_sample(self.ctx, seeds, seeds.numel(), self.fanouts, rng_seed, self._cblocks, self.workspace,
-                   self.workspace_bytes, DSP_BIASED if biased else 0, self.stream())
+                   self.workspace_bytes, (DSP_BIASED if biased else 0) | self._sflag, self.stream())
         return self.blocks()
 
     def sample_gather(self, seeds, rng_seed: int, slot: int = 0, sizes_out=None, async_: bool = False,
@@ -337,7 +363,8 @@ class Sampler:
         torch = self.torch
         assert seeds.dtype == torch.int32 and seeds.is_cuda and seeds.is_contiguous()
         feat_out = self.feat_buffer(slot)
-        flags = (DSP_PIPELINED if pipelined else (DSP_ASYNC if async_ else 0)) | (DSP_BIASED if biased else 0)
+        flags = ((DSP_PIPELINED if pipelined else (DSP_ASYNC if async_ else 0)) | (DSP_BIASED if biased else 0)
+                 | self._sflag)
         dsp_sample_gather(self.ctx, seeds, seeds.numel(), self.fanouts, rng_seed, self._sets[slot][1], feat_out,
                           feat_out.shape[0], self.workspaces[ws], self.workspace_bytes, sizes_out, flags,
                           self.stream() if stream is None else stream.cuda_stream)
@@ -417,14 +444,15 @@ class LocalGroup:
     issued rank by rank on the device's current stream) or sit on several
     GPUs of this node."""
 
-    def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int], hot_rows=None):
+    def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int], hot_rows=None,
+                 scheme: str = "node"):
         """shards[r] = (indptr, indices, features[, edge_weights]) of rank r;
         hot_rows[r] (optional) enables the cold-feature tier."""
         P = len(shards)
         assert len(devices) == P and len(bounds) == P + 1
         self.samplers = [Sampler(bounds, s[0], s[1], s[2], fanouts, max_seeds, rank=r, world_size=P,
                                  device=devices[r], connect=False, edge_weights=s[3] if len(s) > 3 else None,
-                                 hot_rows=None if hot_rows is None else hot_rows[r])
+                                 hot_rows=None if hot_rows is None else hot_rows[r], scheme=scheme)
                          for r, s in enumerate(shards)]
         handles = [dsp_export_handle(s.ctx) for s in self.samplers]
         for s in self.samplers:
@@ -437,7 +465,8 @@ class LocalGroup:
         S = self.samplers
         dsp_sample_group([s.ctx for s in S], seeds_per_rank, [x.numel() for x in seeds_per_rank],
                          self.fanouts, rng_seed, [s._cblocks for s in S], [s.workspace for s in S],
-                         S[0].workspace_bytes, DSP_BIASED if biased else 0, [s.stream() for s in S])
+                         S[0].workspace_bytes, (DSP_BIASED if biased else 0) | S[0]._sflag,
+                         [s.stream() for s in S])
         return [s.blocks() for s in S]
 
     def close(self):

@@ -23,7 +23,7 @@ def _free_port():
     return p
 
 
-def _rank(rank, world, port, q, hot=None):
+def _rank(rank, world, port, q, hot=None, scheme="node"):
     import sys
     here = os.path.dirname(os.path.abspath(__file__))
     sys.path[:0] = [os.path.dirname(here), here]
@@ -42,15 +42,17 @@ def _rank(rank, world, port, q, hot=None):
         lo, hi = int(bnds[rank]), int(bnds[rank + 1])
         sip, six = datagen.shard(ip, ix, lo, hi)
         feats = datagen.features(lo, hi, cfg.dim)
-        s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, 32, rank=rank, world_size=world, device=0,
+        sizes = (300, 600) if scheme == "layer" else cfg.fanouts
+        s = pkg.Sampler(bnds, sip, six, feats, sizes, 32, rank=rank, world_size=world, device=0,
                         exchange=pkg.torch_exchange(), n_slots=2,
-                        hot_rows=None if hot is None else (hi - lo) * hot // 4)
+                        hot_rows=None if hot is None else (hi - lo) * hot // 4, scheme=scheme)
         train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
         batches = datagen.rank_seed_batches(train, bnds, rank, 32, 0)
         for step in range(3):
             seeds = batches[step]
             blocks, feat = s.sample_gather(torch.from_numpy(seeds).cuda(), 0x5EED + step, slot=step % 2)
-            ref = oracle.sample(ip, ix, seeds, cfg.fanouts, 0x5EED + step)
+            ref = (oracle.sample_layerwise(ip, ix, seeds, sizes, 0x5EED + step) if scheme == "layer"
+                   else oracle.sample(ip, ix, seeds, cfg.fanouts, 0x5EED + step))
             for b, r in zip(blocks, ref):
                 for key in ("indptr", "indices", "src_ids"):
                     if not np.array_equal(getattr(b, key).cpu().numpy(), r[key]):
@@ -67,8 +69,8 @@ def _rank(rank, world, port, q, hot=None):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("hot", [None, 1])
-def test_two_processes_one_gpu(hot):
+@pytest.mark.parametrize("hot,scheme", [(None, "node"), (1, "node"), (None, "layer")])
+def test_two_processes_one_gpu(hot, scheme):
     """hot = 1: the cold-feature tier with 3/4 of each shard in host memory
     (POSIX shm mapped into the peer process), read over UVA by both GPUs' gathers."""
     if not torch.cuda.is_available():
@@ -77,7 +79,7 @@ def test_two_processes_one_gpu(hot):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_rank, args=(r, 2, port, q, hot)) for r in range(2)]
+    procs = [ctx.Process(target=_rank, args=(r, 2, port, q, hot, scheme)) for r in range(2)]
     for p in procs:
         p.start()
     res = sorted(q.get(timeout=600) for _ in procs)
