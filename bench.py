@@ -146,6 +146,21 @@ def setup_dist(n_gpus: int):
     return rank, world, local
 
 
+def fanouts_of(args, cfg):
+    """Node-wise fan-outs of the config, or the layer sizes of --scheme layer
+    (Table 7: batch 1024, 1000 nodes per layer for both layers)."""
+    if args.scheme == "layer":
+        return [int(x) for x in args.layer_sizes.split(",")]
+    return list(cfg.fanouts)
+
+
+def oracle_sample(args, ip, ix, seeds, fanouts, rng, weights=None):
+    import oracle
+    if args.scheme == "layer":
+        return oracle.sample_layerwise(ip, ix, seeds, fanouts, rng)
+    return oracle.sample(ip, ix, seeds, fanouts, rng, weights=weights)
+
+
 def load_workload(cfg_name, rank, world):
     import datagen
     cfg = datagen.CONFIGS[cfg_name]
@@ -178,7 +193,7 @@ def run_reference(args):
     for step in range(args.warmup + args.steps):
         seeds = batches[step % len(batches)]
         t0 = time.perf_counter()
-        blocks = oracle.sample(ip, ix, seeds, cfg.fanouts, datagen.BASE_SEED + step, weights=ew)
+        blocks = oracle_sample(args, ip, ix, seeds, fanouts_of(args, cfg), datagen.BASE_SEED + step, weights=ew)
         out = oracle.gather(feats, blocks[-1]["src_ids"])
         dt = time.perf_counter() - t0
         if step >= args.warmup:
@@ -193,8 +208,9 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": args.gpus,
         "steps": steps_done, "warmup": args.warmup, "ms_per_step": 1e3 * t_all / steps_done,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32+f32",
-        "data": "synthetic", "config": {"workload": cfg.name, "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch,
-                                         "num_nodes": cfg.num_nodes, "dim": cfg.dim},
+        "data": "synthetic", "config": {"workload": cfg.name + ("" if args.scheme == "uniform" else f"-{args.scheme}"),
+                                         "scheme": args.scheme, "fanouts": fanouts_of(args, cfg),
+                                         "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes, "dim": cfg.dim},
         "cpu_baseline": {"value": value, "unit": "edges/s", "cores": 1, "kind": "oracle",
                          "sample": f"{steps_done} batches of {cfg.batch} seeds (oracle.sample + oracle.gather)"},
         "e2e": {"value": value, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -205,7 +221,7 @@ def run_reference(args):
     return 0
 
 
-def cpu_baseline(cfg, ip, ix, feats, batches, seconds: float, weights=None):
+def cpu_baseline(args, cfg, ip, ix, feats, batches, seconds: float, weights=None):
     import datagen
     import oracle
     t_all = 0.0
@@ -214,7 +230,7 @@ def cpu_baseline(cfg, ip, ix, feats, batches, seconds: float, weights=None):
     while t_all < seconds and n < len(batches):
         seeds = batches[n]
         t0 = time.perf_counter()
-        blocks = oracle.sample(ip, ix, seeds, cfg.fanouts, datagen.BASE_SEED + n, weights=weights)
+        blocks = oracle_sample(args, ip, ix, seeds, fanouts_of(args, cfg), datagen.BASE_SEED + n, weights=weights)
         oracle.gather(feats, blocks[-1]["src_ids"])
         t_all += time.perf_counter() - t0
         edges += sum(int(b["num_edges"]) for b in blocks)
@@ -245,13 +261,16 @@ def run_dsp(args):
     ex = pkg.torch_exchange() if world > 1 else None
     biased = args.scheme == "biased"
     ew = datagen.edge_weights(six, datagen.node_weights(cfg.num_nodes)) if biased else None
-    K = max(1, args.instances) if world == 1 else 1
-    s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, cfg.batch, rank=rank, world_size=world,
+    layer = args.scheme == "layer"
+    fanouts = fanouts_of(args, cfg)
+    # concurrent instances share the ctx's exchange region on the staged paths: one stream there
+    K = max(1, args.instances) if world == 1 and not layer else 1
+    s = pkg.Sampler(bnds, sip, six, feats, fanouts, cfg.batch, rank=rank, world_size=world, scheme="layer" if layer else "node",
                     device=local, exchange=ex, n_slots=2 * K, edge_weights=ew, n_workspaces=K,
                     hot_rows=None if args.hot_frac is None else int(round(args.hot_frac * (len(sip) - 1))))
     if K > 1:  # K steps in flight on K streams, each persistent launch on 1/K of the SMs
         pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(local).multi_processor_count // K)
-    L = len(cfg.fanouts)
+    L = len(fanouts)
     steps_epoch = datagen.steps_per_epoch(train, bnds, cfg.batch)
     batches = datagen.rank_seed_batches(train, bnds, rank, cfg.batch, 0)[:steps_epoch]
     dev_batches = torch.from_numpy(np.ascontiguousarray(batches)).cuda()   # inputs resident in HBM
@@ -399,9 +418,10 @@ def run_dsp(args):
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(cfg, ip, ix, feats, batches, args.cpu_seconds, weights=ew)
+        cpu = cpu_baseline(args, cfg, ip, ix, feats, batches, args.cpu_seconds, weights=ew)
 
-    kern_per_step = 1 if world == 1 else 5 * L + 1
+    kern_per_step = 5 * L + 1 if layer else (1 if world == 1 else 5 * L + 1)
+    roof_kernel = "k_csp_persistent" if world == 1 and not layer else "k_gather"
     if rank == 0:
         line = {
             "metric": METRIC, "value": tot_edges / (t_max * 1e-3), "unit": "edges/s", "n_gpus": world,
@@ -409,12 +429,12 @@ def run_dsp(args):
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32+f32",
             "data": "synthetic",
             "config": {"workload": (cfg.name if world == 1 else f"{cfg.name}-P{world}")
-                       + ("-biased" if biased else "")
+                       + ("-biased" if biased else "") + ("-layerwise" if layer else "")
                        + ("" if args.hot_frac is None else f"-hot{args.hot_frac:g}"), "scheme": args.scheme,
                        "features": ("all rows in HBM" if args.hot_frac is None else
                                     f"cold tier: {args.hot_frac:g} of rows (largest in-degree) in HBM, "
                                     "the rest in pinned host memory read over UVA"),
-                       "fanouts": list(cfg.fanouts), "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes,
+                       "fanouts": fanouts, "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes,
                        "nnz": int(ip[-1]), "dim": cfg.dim, "parallelism": f"csp{world}",
                        "l2": "inputs larger than L2 (CSR 0.5 GB + features 1.1 GB >> 126 MB L2)",
                        "step": ("dsp_sample_gather (DSP_PIPELINED: sampler(t) || loader(t-1), 2 output sets)"
@@ -425,15 +445,16 @@ def run_dsp(args):
             "feature_GBps": tot_rows * cfg.dim * 4 / (t_max * 1e-3) / 1e9,
             "edges_per_step": tot_edges / KS / world,
             "rows_per_step": tot_rows / KS / world,
-            "roofline": {"kernel": "k_csp_persistent" if world == 1 else "k_gather",
+            "roofline": {"kernel": roof_kernel,
                          "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": ncu_traffic("k_csp_persistent"),
+                         "frac": achieved / peak, "traffic": ncu_traffic(roof_kernel) if roof_kernel == "k_csp_persistent" else None,
                          "peak_kind": peak_kind,
                          "algorithmic_bytes_per_launch": (samp_b + gath_b) / KS,
                          "sampling_bytes_per_launch": samp_b / KS, "gather_bytes_per_launch": gath_b / KS,
                          "launch_ms_mean": step_mean, "concurrent_launches": K,
                          "achieved_def": "algorithmic bytes of all timed launches / elapsed device time"},
             "breakdown": bd,
+            "epoch_sampling_s": (steps_epoch * bd["sample_call_ms_mean"] * 1e-3 if bd else None),
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_edges / (e2e_ms * 1e-3), "unit": "edges/s",
                     "h2d_bytes_per_step": h2d // e2e_steps, "d2h_bytes_per_step": d2h // e2e_steps,
@@ -461,7 +482,9 @@ def main(argv=None):
     ap.add_argument("--no-breakdown", action="store_true")
     ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
     ap.add_argument("--instances", type=int, default=2, help="concurrent step streams (world 1)")
-    ap.add_argument("--scheme", choices=["uniform", "biased"], default="uniform",
+    ap.add_argument("--layer-sizes", default="1000,1000",
+                    help="--scheme layer: nodes sampled per layer (Table 7: 1000,1000)")
+    ap.add_argument("--scheme", choices=["uniform", "biased", "layer"], default="uniform",
                     help="node-wise scheme (Table 2 IsBiased); biased uses synthetic node weights")
     ap.add_argument("--hot-frac", type=float, default=None,
                     help="cold-feature tier: fraction of each shard's rows kept in HBM (P:L114)")

@@ -109,6 +109,13 @@ __device__ __forceinline__ uint32_t table_insert_finish(unsigned long long *tbl,
 __device__ __forceinline__ void st_release_sys(unsigned long long *p, unsigned long long v) {
   asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
+__device__ __forceinline__ void st_release_gpu(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+// release store of a flag: system scope when a peer may sit on another device
+__device__ __forceinline__ void st_release_flag(unsigned long long *p, unsigned long long v, int sys) {
+  if (sys) st_release_sys(p, v); else st_release_gpu(p, v);
+}
 __device__ __forceinline__ unsigned long long ld_acquire_sys(const unsigned long long *p) {
   unsigned long long v;
   asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");

@@ -93,7 +93,26 @@ struct LwArgs {
   Outputs out;             // block l arrays in out.*[0]
   WsHeader *hdr;
   int *err;
+  int32_t sys;             // peers on other devices: system-scope fences (else GPU scope)
 };
+
+// Last-block-done with a fence of the given scope (see last_block_done).
+__device__ __forceinline__ bool lw_last_block_done(uint32_t *done, int sys) {
+  __shared__ int s_last;
+  if (sys) __threadfence_system(); else __threadfence();
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const uint32_t t = atomicAdd(done, 1u);
+    s_last = (t == gridDim.x - 1) ? 1 : 0;
+  }
+  __syncthreads();
+  if (s_last && threadIdx.x == 0) {
+    if (sys) __threadfence_system(); else __threadfence();
+    *(volatile uint32_t *)done = 0u;
+    return true;
+  }
+  return false;
+}
 
 __device__ __forceinline__ uint32_t lw_tag(int n, int layer) { return (uint32_t)n | ((uint32_t)layer << 16); }
 
@@ -128,7 +147,14 @@ __device__ __forceinline__ T block_excl_scan(T x, T *s_warp, T *total) {
   return r;
 }
 
+constexpr int LW_IPT = 4;                 // frontier nodes per thread per pass of k_lw_alloc
+constexpr int LW_SMEM_F = 8192;           // frontier sizes whose prefix + counts fit in shared memory
+constexpr size_t LW_ALLOC_SMEM = (size_t)LW_SMEM_F * (sizeof(unsigned long long) + sizeof(int32_t));
+
+// Dynamic shared memory: LW_ALLOC_SMEM (prefix u64 + counts i32 of up to
+// LW_SMEM_F frontier nodes); larger frontiers use the workspace copies.
 __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
+  extern __shared__ unsigned long long lw_alloc_smem[];
   __shared__ unsigned long long s_u64[33];
   __shared__ int32_t s_i32[33];
   __shared__ uint32_t s_cnt[8];
@@ -139,30 +165,45 @@ __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
     F = 0;
   }
   if (tid == 0 && a.layer == 0) a.hdr->F[0] = F;
+  const bool in_smem = F + 1 <= LW_SMEM_F;
+  unsigned long long *P = in_smem ? lw_alloc_smem : a.w.P;
+  int32_t *cnt = in_smem ? reinterpret_cast<int32_t *>(lw_alloc_smem + LW_SMEM_F) : a.w.c;
   const int32_t g0 = a.F0 > 0 ? __ldg(a.seeds) : 0;
-  // W_u from the owner's indptr (peer memory), with the running prefix
+  // W_u from the owner's indptr (peer memory): LW_IPT independent loads per
+  // thread in flight, then the block-wide exclusive scan
   unsigned long long carry = 0;
-  for (int b0 = 0; b0 < F; b0 += LWT) {
-    const int i = b0 + tid;
-    unsigned long long W = 0;
-    if (i < F) {
-      const int32_t v = __ldg(a.frontier + i);
-      if (v < 0 || v >= a.bd.b[a.bd.world]) {
-        latch(a.err, E_RANGE);
-      } else {
-        const int o = owner_of(a.bd, v);
-        const int64_t lv = (int64_t)v - a.bd.b[o];
-        const int64_t *ip = a.peer_indptr[o];
-        W = (unsigned long long)(ip[lv + 1] - ip[lv]);
+  for (int b0 = 0; b0 < F; b0 += LWT * LW_IPT) {
+    unsigned long long W[LW_IPT];
+    unsigned long long sum = 0;
+#pragma unroll
+    for (int j = 0; j < LW_IPT; ++j) {
+      const int i = b0 + tid * LW_IPT + j;
+      W[j] = 0;
+      if (i < F) {
+        const int32_t v = __ldg(a.frontier + i);
+        if (v < 0 || v >= a.bd.b[a.bd.world]) {
+          latch(a.err, E_RANGE);
+        } else {
+          const int o = owner_of(a.bd, v);
+          const int64_t lv = (int64_t)v - a.bd.b[o];
+          const int64_t *ip = a.peer_indptr[o];
+          W[j] = (unsigned long long)(ip[lv + 1] - ip[lv]);
+        }
+        cnt[i] = 0;
       }
-      a.w.c[i] = 0;
+      sum += W[j];
     }
     unsigned long long tot;
-    const unsigned long long ex = block_excl_scan<unsigned long long>(W, s_u64, &tot);
-    if (i < F) a.w.P[i] = carry + ex;
+    unsigned long long ex = carry + block_excl_scan<unsigned long long>(sum, s_u64, &tot);
+#pragma unroll
+    for (int j = 0; j < LW_IPT; ++j) {
+      const int i = b0 + tid * LW_IPT + j;
+      if (i < F) P[i] = ex;
+      ex += W[j];
+    }
     carry += tot;
   }
-  if (tid == 0) a.w.P[F] = carry;
+  if (tid == 0) P[F] = carry;
   const unsigned long long T = carry;
   __syncthreads();
   // Eq. 2: n draws with replacement, frontier node i with probability W_i / T
@@ -174,9 +215,9 @@ __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
       int lo = 0, hi = F - 1;  // largest i with P[i] <= r
       while (lo < hi) {
         const int mid = (lo + hi + 1) >> 1;
-        if (a.w.P[mid] <= r) lo = mid; else hi = mid - 1;
+        if (P[mid] <= r) lo = mid; else hi = mid - 1;
       }
-      atomicAdd(a.w.c + lo, 1);
+      atomicAdd(cnt + lo, 1);
     }
   __syncthreads();
   // slot offsets, slot -> node, and the tasks pushed to the owners
@@ -184,7 +225,9 @@ __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
   int32_t ocarry = 0;
   for (int b0 = 0; b0 < F; b0 += LWT) {
     const int i = b0 + tid;
-    const int32_t ci = i < F ? a.w.c[i] : 0;
+    const int32_t ci = i < F ? cnt[i] : 0;
+    int o_req = -1;
+    int4 req = make_int4(0, 0, 0, 0);
     int32_t tot;
     const int32_t ex = block_excl_scan<int32_t>(ci, s_i32, &tot);
     if (i < F) {
@@ -193,10 +236,19 @@ __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
       if (ci > 0) {
         for (int t = 0; t < ci; ++t) a.w.slot_node[off + t] = i;
         const int32_t v = __ldg(a.frontier + i);
-        const int o = owner_of(a.bd, v);
-        const uint32_t j = atomicAdd(&s_cnt[o], 1u);
-        lw_inbox(a.peers.base[o], a.L, a.parity, a.rank)[j] = make_int4(i, v, ci, off);
+        o_req = owner_of(a.bd, v);
+        req = make_int4(i, v, ci, off);
       }
+    }
+    {  // warp-aggregated slot in the owner's inbox
+      const unsigned peers = __match_any_sync(FULL_MASK, o_req);
+      const int leader = __ffs(peers) - 1;
+      const int lane = threadIdx.x & 31;
+      uint32_t base = 0;
+      if (o_req >= 0 && lane == leader) base = atomicAdd(&s_cnt[o_req], (uint32_t)__popc(peers));
+      base = __shfl_sync(FULL_MASK, base, leader);
+      if (o_req >= 0)
+        lw_inbox(a.peers.base[o_req], a.L, a.parity, a.rank)[base + __popc(peers & ((1u << lane) - 1u))] = req;
     }
     ocarry += tot;
   }
@@ -205,8 +257,9 @@ __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
   if (tid == 0) {
     for (int o = 0; o < a.bd.world; ++o)
       *lw_inbox_hdr(a.peers.base[o], a.L, a.parity, a.rank) = make_uint4(s_cnt[o], lw_tag(a.n, a.layer), a.key.x, a.key.y);
-    __threadfence_system();
-    for (int o = 0; o < a.bd.world; ++o) st_release_sys(lw_inbox_flag(a.peers.base[o], a.L, a.parity, a.rank), a.seq);
+    if (a.sys) __threadfence_system();
+    for (int o = 0; o < a.bd.world; ++o)
+      st_release_flag(lw_inbox_flag(a.peers.base[o], a.L, a.parity, a.rank), a.seq, a.sys);
   }
 }
 
@@ -264,7 +317,7 @@ __global__ void __launch_bounds__(NT) k_lw_sample_remote(LwArgs a) {
       }
     }
   }
-  last_block_done(&a.hdr->done);  // fences this kernel's peer stores
+  if (a.sys) __threadfence_system();  // this kernel's peer stores, before k_lw_sample_big's flags
 }
 
 // Tasks with 32 < c < deg: Floyd over c draws with a shared-memory hash set.
@@ -326,9 +379,10 @@ __global__ void __launch_bounds__(LWT) k_lw_sample_big(LwArgs a, int kp_max) {
     if (threadIdx.x == 0) lw_ret_cnt(req_base, a.L, a.parity)[req.x] = k;
     __syncthreads();
   }
-  if (last_block_done(&a.hdr->done)) {
+  if (lw_last_block_done(&a.hdr->done, a.sys)) {
     a.hdr->lw_big = 0u;
-    for (int s = 0; s < a.bd.world; ++s) st_release_sys(lw_ret_flag(a.peers.base[s], a.L, a.parity, a.rank), a.seq);
+    for (int s = 0; s < a.bd.world; ++s)
+      st_release_flag(lw_ret_flag(a.peers.base[s], a.L, a.parity, a.rank), a.seq, a.sys);
   }
 }
 

@@ -788,6 +788,7 @@ LwArgs lw_args(Call &k, int l) {
   a.out.src_ids[0] = k.blocks[l].src_ids;
   a.hdr = k.hdr;
   a.err = c->d_err;
+  a.sys = c->world > 1 ? 1 : 0;
   return a;
 }
 
@@ -798,7 +799,7 @@ dsp_status stage_lw(Call &k, int l, int step) {
   const int64_t F = k.plan.F[l], n = k.fanouts[l];
   switch (step) {
     case 0:
-      k_lw_alloc<<<1, LWT, 0, k.stream>>>(a);
+      k_lw_alloc<<<1, LWT, LW_ALLOC_SMEM, k.stream>>>(a);
       break;
     case 1: {  // one warp per task; at most world * F tasks arrive
       const int64_t need = std::max<int64_t>(1, (c->world * F + NT / 32 - 1) / (NT / 32));
@@ -807,7 +808,7 @@ dsp_status stage_lw(Call &k, int l, int step) {
     }
     case 2: {
       const int kp = (int)next_pow2(k.plan.ncap);
-      k_lw_sample_big<<<(int)std::min<int64_t>(k.plan.big_cap, c->num_sms), LWT,
+      k_lw_sample_big<<<(int)std::min<int64_t>(k.plan.big_cap, 32), LWT,
                         sizeof(int32_t) * 3 * (size_t)kp, k.stream>>>(a, kp);
       break;
     }
@@ -1037,7 +1038,9 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
     return fail(nullptr, DSP_ERR_CUDA, "occupancy query for the persistent kernel failed");
   }
   if (cudaFuncSetAttribute((const void *)k_lw_sample_big, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           (int)sizeof(int32_t) * 3 * LW_MAX_SIZE) != cudaSuccess) {
+                           (int)sizeof(int32_t) * 3 * LW_MAX_SIZE) != cudaSuccess ||
+      cudaFuncSetAttribute((const void *)k_lw_alloc, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           (int)LW_ALLOC_SMEM) != cudaSuccess) {
     cudaGetLastError();
     delete c;
     return fail(nullptr, DSP_ERR_CUDA, "shared-memory attribute of the layer-wise kernel failed");
