@@ -207,6 +207,13 @@ __device__ __forceinline__ int owner_of(const Bounds &bd, int64_t g) {
   return o;
 }
 
+// adjacency read: streamed at random, never reused within a call (L2 evict_first)
+__device__ __forceinline__ int32_t adj_ld(const int32_t *p) {
+  int32_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(l2_policy_evict_first()));
+  return v;
+}
+
 // ------------------------------------------------------- one node's sample
 // Lane group of G lanes (G = next pow2 >= k) samples node v.  Returns, per
 // lane t: whether slot `*slot` of the node holds sampled neighbour *u, and
@@ -249,7 +256,7 @@ __device__ __forceinline__ void sample_node(bool ok, int32_t v, int64_t row_star
   *count = cnt;
   *valid = t < cnt;
   *slot = full ? t : rank;
-  *u = *valid ? __ldg(indices + row_start + chosen) : -1;
+  *u = *valid ? adj_ld(indices + row_start + chosen) : -1;
 }
 
 // -------------------------------------------------- one node's biased sample

@@ -93,8 +93,32 @@ __device__ __forceinline__ unsigned long long mark_word(uint32_t epoch, uint32_t
 }
 // x of a word of the current epoch
 __device__ __forceinline__ uint32_t mark_x(unsigned long long w) { return 0xffffffffu - (uint32_t)w; }
+// Every access to the map carries an L2 evict_last policy: the map (8 B per
+// node and parity) is touched at random ~2 times per sampled edge, and
+// without the hint the adjacency reads and the gather's stream push it out of
+// L2, turning each mark into a DRAM read + write-back.
+__device__ __forceinline__ unsigned long long map_policy() { return l2_policy_evict_last(); }
+__device__ __forceinline__ void map_red_max(unsigned long long *p, unsigned long long v) {
+  asm volatile("red.relaxed.gpu.global.max.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(map_policy())
+               : "memory");
+}
+__device__ __forceinline__ unsigned long long map_atom_max(unsigned long long *p, unsigned long long v) {
+  unsigned long long old;
+  asm volatile("atom.relaxed.gpu.global.max.L2::cache_hint.u64 %0, [%1], %2, %3;"
+               : "=l"(old) : "l"(p), "l"(v), "l"(map_policy()) : "memory");
+  return old;
+}
+// weak load / store (ordered by the grid barriers or kernel boundaries)
+__device__ __forceinline__ unsigned long long map_ld(const unsigned long long *p) {
+  unsigned long long v;
+  asm volatile("ld.global.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(map_policy()));
+  return v;
+}
+__device__ __forceinline__ void map_st(unsigned long long *p, unsigned long long v) {
+  asm volatile("st.global.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(map_policy()) : "memory");
+}
 __device__ __forceinline__ void mark(unsigned long long *first, int32_t u, uint32_t epoch, uint32_t x) {
-  atomicMax(first + u, mark_word(epoch, x));  // result unused: compiles to a reduction (RED)
+  map_red_max(first + u, mark_word(epoch, x));
 }
 
 // q / k for a fixed small divisor k: one 64-bit multiply-high with
@@ -191,7 +215,7 @@ __device__ __forceinline__ void grid_barrier(WsHeader *hdr, uint32_t &target) {
 __device__ __forceinline__ void mark_dst(unsigned long long *first, int32_t v, int i, int F, int layer,
                                          uint32_t epoch, int *err) {
   if (layer == 0) {
-    const unsigned long long old = atomicMax(first + v, mark_word(epoch, (uint32_t)i));
+    const unsigned long long old = map_atom_max(first + v, mark_word(epoch, (uint32_t)i));
     if ((uint32_t)(old >> 32) == epoch && mark_x(old) < (uint32_t)F) latch(err, E_DUP);
   } else {
     mark(first, v, epoch, (uint32_t)i);
@@ -308,7 +332,7 @@ __device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F,
 #pragma unroll
       for (int q = 0; q < KB; ++q) r += (q < cnt && pos[q] < pos[t]) ? 1u : 0u;
       slots |= (unsigned long long)r << (4 * t);
-      u[t] = (t < cnt) ? __ldg(indices + rs + pos[t]) : 0;
+      u[t] = (t < cnt) ? adj_ld(indices + rs + pos[t]) : 0;
     }
     DSTAMP(hdr, 3, u[0] + u[KB - 1], layer);
     B.cnt[i] = cnt;
@@ -418,7 +442,7 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
   }
   unsigned long long w[SCAN2_IPT];
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? ldw_u64(B.first + u[j]) : 0ull;
+  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? map_ld(B.first + u[j]) : 0ull;
   R.vbits = R.fbits = 0;
 #pragma unroll
   for (int j = 0; j < SCAN2_IPT; ++j) {
@@ -517,7 +541,7 @@ __device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, ui
       if (q == i * (uint32_t)k) indptr_out[i] = (int32_t)((uint32_t)(b & 0x7fffffffull) + __popc(bv & lt));
       if ((R.fbits >> j) & 1u) {
         const uint32_t nid = (uint32_t)F + (uint32_t)((b >> 31) & 0x7fffffffull) + __popc(bf & lt);
-        B.first[u[j]] = mark_word(epoch, nid);  // only this slot writes u's word in this phase
+        map_st(B.first + u[j], mark_word(epoch, nid));  // only this slot writes u's word in this phase
         src_out[nid] = u[j];
       }
     }
@@ -550,7 +574,7 @@ __device__ __forceinline__ void phase_indices(int F, int k, const LayerBufs &B, 
     }
     unsigned long long w[U];
 #pragma unroll
-    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? ldw_u64(B.first + u[j]) : 0ull;
+    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? map_ld(B.first + u[j]) : 0ull;
 #pragma unroll
     for (int j = 0; j < U; ++j)
       if (c[j] > 0) indices_out[ip[j]] = (int32_t)mark_x(w[j]);
@@ -676,6 +700,7 @@ struct PersistArgs {
   int32_t *pend_n;          // where this call's row count goes (read by the next call / flush)
   int32_t rows_per_chunk;   // R
   int32_t slot_bytes;       // ring slot size (>= R * row bytes)
+  int32_t lane_rounds;      // lane groups per node while F * G <= lane_rounds * team threads
 };
 
 template <int TEAM>
@@ -686,6 +711,19 @@ __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32
   if (a.biased) {
     phase_sample_biased<TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.weights, a.lo, a.n_local, B, epoch,
                               a.out.src_ids[l], a.err);
+  } else if (k <= 16 && (int64_t)F * (k <= 4 ? 4 : k <= 8 ? 8 : 16) <= (int64_t)a.lane_rounds * gridDim.x * TEAM) {
+    // small frontier (the first layers): a lane group per node, so the k
+    // Philox draws run in parallel instead of back to back in one thread,
+    // whose dependent-instruction latency dominates when few warps are busy
+    if (k <= 4)
+      phase_sample_lanes<4, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
+                                  a.out.src_ids[l], a.err, a.hdr);
+    else if (k <= 8)
+      phase_sample_lanes<8, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
+                                  a.out.src_ids[l], a.err, a.hdr);
+    else
+      phase_sample_lanes<16, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
+                                   a.out.src_ids[l], a.err, a.hdr);
   } else if (k <= 8) {
     phase_sample_tpn<8, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.lo, a.n_local, B, epoch,
                               a.out.src_ids[l], a.err, a.hdr);
@@ -1291,7 +1329,7 @@ __global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
     for (int j = 0; j < SCAN_ITEMS; ++j) {
       if (c[j] > 0) {
         vbits |= 1u << j;
-        if (__ldg(B.first + u[j]) == mark_word(epoch, (uint32_t)F + q0 + j)) fbits |= 1u << j;
+        if (map_ld(B.first + u[j]) == mark_word(epoch, (uint32_t)F + q0 + j)) fbits |= 1u << j;
       }
     }
     const unsigned long long mine = pack2(__popc(vbits), __popc(fbits));
@@ -1357,7 +1395,7 @@ __global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
         if (q == i * (uint32_t)k) a.indptr_out[i] = (int32_t)pv;
         if (fbits & (1u << j)) {
           const uint32_t nid = (uint32_t)F + pf;
-          B.first[u[j]] = mark_word(epoch, nid);
+          map_st(B.first + u[j], mark_word(epoch, nid));
           a.src_ids_out[nid] = u[j];
         }
         pv += (vbits >> j) & 1u;

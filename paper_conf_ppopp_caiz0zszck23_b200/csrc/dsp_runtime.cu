@@ -155,6 +155,7 @@ struct dsp_ctx {
   int *h_err = nullptr;
   int num_sms = 148;
   int persist_blocks_per_sm = 1;
+  int lane_rounds = 4;  // DSP_LANE_ROUNDS (tuning knob, results unchanged)
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
   int gather_blocks_per_sm = 1;
   // pipelined steps: per workspace, the gather owed by its previous
@@ -573,6 +574,7 @@ dsp_status stage_persistent(Call &k) {
   a.buf[1] = bufs_of(k, 1);
   a.hdr = k.hdr;
   a.err = c->d_err;
+  a.lane_rounds = c->lane_rounds;
   a.gather = k.feat_out != nullptr && !k.pipelined;
   if (a.gather) a.g = make_gather(c, k.blocks[k.L - 1].src_ids, 0, nullptr, k.feat_out);
   const dim3 grid(c->persist_blocks > 0 ? c->persist_blocks : c->num_sms * c->persist_blocks_per_sm), block(PNT);
@@ -1046,6 +1048,7 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
     return fail(nullptr, DSP_ERR_CUDA, "shared-memory attribute of the layer-wise kernel failed");
   }
   c->persist_blocks_per_sm = std::min(occ, occ_pipe);
+  if (getenv("DSP_LANE_ROUNDS")) c->lane_rounds = atoi(getenv("DSP_LANE_ROUNDS"));
   if (c->persist_blocks_per_sm * c->num_sms > MAX_PERSIST_BLOCKS) c->persist_blocks_per_sm = MAX_PERSIST_BLOCKS / c->num_sms;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_gather, NT, 0) != cudaSuccess || occ < 1) {
     cudaGetLastError();

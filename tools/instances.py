@@ -10,6 +10,8 @@ import paper_conf_ppopp_caiz0zszck23_b200 as pkg
 cfg = datagen.CONFIGS[os.environ.get("CFG", "products")]
 ip, ix = datagen.make_graph(cfg)
 feats = datagen.features(0, cfg.num_nodes, cfg.dim)
+if os.environ.get("DIM"):  # e.g. DIM=4: (almost) no gather, sampling throughput alone
+    feats = np.ascontiguousarray(feats[:, : int(os.environ["DIM"])])
 bnds = datagen.bounds(cfg.num_nodes, 1)
 KMAX = 4
 s = pkg.Sampler(bnds, ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2 * KMAX, n_workspaces=KMAX)
@@ -19,7 +21,7 @@ L = len(cfg.fanouts)
 sizes = torch.zeros((4096, 3 * L), dtype=torch.int64).pin_memory()
 steps = 60
 main = torch.cuda.current_stream()
-for K in (1, 2, 3, 4):
+for K in [int(x) for x in os.environ.get("KS", "1,2,3,4").split(",")]:
     pkg.dsp_set_persistent_blocks(s.ctx, 0 if K == 1 else 148 // K)
     streams = [torch.cuda.Stream() for _ in range(K)]
     for pipelined in (False, True):
