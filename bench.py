@@ -385,36 +385,48 @@ def run_dsp(args):
               "gather_frac_of_hbm": float(np.mean([b / (m * 1e-3) / 1e9 for b, m in zip(g_bytes, g_ms)])) / peak,
               "note": "dsp_sample (synchronous, host sizes) and dsp_gather_features timed separately"}
 
-    # ---- e2e: the same steps through the C ABI with HOST buffers: pinned seeds
-    # H2D, sample + gather, D2H of the blocks and the gathered features
+    # ---- e2e: the same steps through the C ABI from HOST buffers, one synchronous
+    # dsp_sample_gather per step (the call a training loop makes): every step copies
+    # its seeds H2D from pinned memory and reads the per-layer sizes back (the host
+    # needs them to shape the consumer's launch); blocks and features stay in HBM for
+    # the GPU trainer.  e2e_host_copy additionally copies every block and all gathered
+    # features to pinned host memory (PCIe-bound; a host consumer's view).
     h_seeds = torch.from_numpy(np.ascontiguousarray(batches)).pin_memory()
     h_feat = torch.empty((s.max_src[-1], cfg.dim), dtype=torch.float32).pin_memory()
     h_blk = [tuple(torch.empty(x.numel(), dtype=torch.int32).pin_memory() for x in bufs) for bufs in s._bufs]
     d_seed = torch.empty(cfg.batch, dtype=torch.int32, device="cuda")
     e2e_steps = max(3, min(KS, 20))
-    h2d = d2h = 0
-    barrier()
-    torch.cuda.synchronize()
-    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    e2e_edges = 0
-    e0.record(stream)
-    for j in range(e2e_steps):
-        i = W + j
-        d_seed.copy_(h_seeds[i % len(batches)], non_blocking=True)
-        h2d += d_seed.numel() * 4
-        blocks, feat = s.sample_gather(d_seed, datagen.BASE_SEED + i, slot=0, biased=biased)
-        for b, hb in zip(blocks, h_blk):
-            hb[0][: b.num_dst + 1].copy_(b.indptr, non_blocking=True)
-            hb[1][: b.num_edges].copy_(b.indices, non_blocking=True)
-            hb[2][: b.num_src].copy_(b.src_ids, non_blocking=True)
-            d2h += 4 * (b.num_dst + 1 + b.num_edges + b.num_src)
-        h_feat[: feat.shape[0]].copy_(feat, non_blocking=True)
-        d2h += feat.numel() * 4
-        e2e_edges += sum(b.num_edges for b in blocks)
-    e1.record(stream)
-    torch.cuda.synchronize()
-    e2e_ms = reduce_max_over_ranks(e0.elapsed_time(e1))
-    e2e_edges = reduce_sum_over_ranks(e2e_edges)
+
+    def e2e_run(host_copy: bool):
+        h2d = d2h = 0
+        barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        n_edges = 0
+        e0.record(stream)
+        for j in range(e2e_steps):
+            i = W + j
+            d_seed.copy_(h_seeds[i % len(batches)], non_blocking=True)
+            h2d += d_seed.numel() * 4
+            # synchronous call: returns after the step with the host-side sizes filled (D2H)
+            blocks, feat = s.sample_gather(d_seed, datagen.BASE_SEED + i, slot=0, biased=biased)
+            d2h += 3 * 8 * L
+            if host_copy:
+                for b, hb in zip(blocks, h_blk):
+                    hb[0][: b.num_dst + 1].copy_(b.indptr, non_blocking=True)
+                    hb[1][: b.num_edges].copy_(b.indices, non_blocking=True)
+                    hb[2][: b.num_src].copy_(b.src_ids, non_blocking=True)
+                    d2h += 4 * (b.num_dst + 1 + b.num_edges + b.num_src)
+                h_feat[: feat.shape[0]].copy_(feat, non_blocking=True)
+                d2h += feat.numel() * 4
+            n_edges += sum(b.num_edges for b in blocks)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ms = reduce_max_over_ranks(e0.elapsed_time(e1))
+        return reduce_sum_over_ranks(n_edges) / (ms * 1e-3), h2d // e2e_steps, d2h // e2e_steps
+
+    e2e_v, e2e_h2d, e2e_d2h = e2e_run(False)
+    e2e_hv, e2e_hh2d, e2e_hd2h = e2e_run(True)
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -456,9 +468,13 @@ def run_dsp(args):
             "breakdown": bd,
             "epoch_sampling_s": (steps_epoch * bd["sample_call_ms_mean"] * 1e-3 if bd else None),
             "cpu_baseline": cpu,
-            "e2e": {"value": e2e_edges / (e2e_ms * 1e-3), "unit": "edges/s",
-                    "h2d_bytes_per_step": h2d // e2e_steps, "d2h_bytes_per_step": d2h // e2e_steps,
-                    "steps": e2e_steps, "api": "dsp_sample_gather (synchronous) + D2H of blocks and features"},
+            "e2e": {"value": e2e_v, "unit": "edges/s",
+                    "h2d_bytes_per_step": e2e_h2d, "d2h_bytes_per_step": e2e_d2h, "steps": e2e_steps,
+                    "api": "pinned seeds H2D + dsp_sample_gather (synchronous, sizes D2H); blocks and features "
+                           "stay in HBM for the GPU consumer"},
+            "e2e_host_copy": {"value": e2e_hv, "unit": "edges/s", "h2d_bytes_per_step": e2e_hh2d,
+                              "d2h_bytes_per_step": e2e_hd2h,
+                              "api": "as e2e, plus D2H of every block and all gathered features (PCIe-bound)"},
             "gpu_launches": kern_per_step * KS + (K if pipelined else 0),
             "clocks": clk.summary(),
         }
@@ -481,7 +497,7 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-breakdown", action="store_true")
     ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
-    ap.add_argument("--instances", type=int, default=2, help="concurrent step streams (world 1)")
+    ap.add_argument("--instances", type=int, default=3, help="concurrent step streams (world 1)")
     ap.add_argument("--layer-sizes", default="1000,1000",
                     help="--scheme layer: nodes sampled per layer (Table 7: 1000,1000)")
     ap.add_argument("--scheme", choices=["uniform", "biased", "layer"], default="uniform",

@@ -448,6 +448,9 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
   for (int j = 0; j < SCAN2_IPT; ++j) {
     const bool valid = c[j] > 0;
     const bool first = valid && w[j] == mark_word(epoch, (uint32_t)F + q0 + j * TEAM);
+    // a valid slot that is not u's first occurrence keeps x (u's smallest order
+    // key: its dst index, or F + the slot of its first occurrence) as -1 - x
+    if (valid && !first) B.rows[q0 + j * TEAM] = -1 - (int32_t)mark_x(w[j]);
     R.vbits |= (valid ? 1u : 0u) << j;
     R.fbits |= (first ? 1u : 0u) << j;
     const uint32_t bv = __ballot_sync(FULL_MASK, valid), bf = __ballot_sync(FULL_MASK, first);
@@ -515,21 +518,26 @@ __device__ __forceinline__ void scan2_prefix(const unsigned long long *agg, int 
   team_sync<TEAM>();
 }
 
-// Block indptr at t == 0 slots; for first occurrences: new id nid = F + rank,
-// map word := (epoch, nid), src_out[nid] = u.  The dst copy is written by the
-// sample phase.
+// Block indptr at t == 0 slots, and the local src id of every edge whose
+// answer is known here: a first occurrence gets nid = F + rank (src_out[nid] =
+// u, and rows[q] := nid for the duplicates), a dst hit its dst index x.  The
+// remaining edges (duplicates of a first occurrence elsewhere) are resolved by
+// phase_indices_dups after the next grid barrier.  The relabel map is not
+// touched: a duplicate finds its nid through rows[x - F], a coalesced-slot
+// array, instead of a second random map access per edge.  The dst copy of
+// src_out is written by the sample phase.
 template <int TEAM>
-__device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, uint32_t epoch, int64_t tile0,
-                                            int64_t tile_end, const Scan2Regs &R, unsigned long long base,
-                                            const Scan2Smem<TEAM> &sm, int32_t *indptr_out, int32_t *src_out) {
+__device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, int64_t tile0, int64_t tile_end,
+                                            const Scan2Regs &R, unsigned long long base, const Scan2Smem<TEAM> &sm,
+                                            int32_t *indptr_out, int32_t *indices_out, int32_t *src_out) {
   const uint32_t total = (uint32_t)tile_end;
   const FastDiv fd = make_fastdiv((uint32_t)k);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint32_t lt = (1u << lane) - 1u;
   const uint32_t q0 = (uint32_t)tile0 + threadIdx.x;
-  int32_t u[SCAN2_IPT];
+  int32_t r[SCAN2_IPT];
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) u[j] = ((R.fbits >> j) & 1u) ? ldw_i32(B.rows + q0 + j * TEAM) : 0;
+  for (int j = 0; j < SCAN2_IPT; ++j) r[j] = ((R.vbits >> j) & 1u) ? ldw_i32(B.rows + q0 + j * TEAM) : 0;
 #pragma unroll
   for (int j = 0; j < SCAN2_IPT; ++j) {
     const uint32_t bv = __ballot_sync(FULL_MASK, (R.vbits >> j) & 1u);
@@ -537,14 +545,51 @@ __device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, ui
     const uint32_t q = q0 + j * TEAM;
     if (q < total) {
       const unsigned long long b = base + sm.tab[j * (TEAM / 32) + wid];
+      const uint32_t e = (uint32_t)(b & 0x7fffffffull) + __popc(bv & lt);  // edge index of slot q (if valid)
       const uint32_t i = fdiv(q, fd);
-      if (q == i * (uint32_t)k) indptr_out[i] = (int32_t)((uint32_t)(b & 0x7fffffffull) + __popc(bv & lt));
+      if (q == i * (uint32_t)k) indptr_out[i] = (int32_t)e;
       if ((R.fbits >> j) & 1u) {
         const uint32_t nid = (uint32_t)F + (uint32_t)((b >> 31) & 0x7fffffffull) + __popc(bf & lt);
-        map_st(B.first + u[j], mark_word(epoch, nid));  // only this slot writes u's word in this phase
-        src_out[nid] = u[j];
+        src_out[nid] = r[j];
+        B.rows[q] = (int32_t)nid;
+        indices_out[e] = (int32_t)nid;
+      } else if ((R.vbits >> j) & 1u) {
+        const uint32_t x = (uint32_t)(-1 - r[j]);
+        if (x < (uint32_t)F) indices_out[e] = (int32_t)x;  // dst hit
       }
     }
+  }
+}
+
+// Duplicates of layer l (after pass 2 and a grid barrier): a valid slot q
+// holding -1 - x with x >= F takes the nid stored at its first occurrence's
+// slot x - F.
+__device__ __forceinline__ void phase_indices_dups(int F, int k, const LayerBufs &B, const int32_t *indptr,
+                                                   int32_t *indices_out, const Span &sp) {
+  constexpr int U = 4;  // items per thread in flight
+  const FastDiv fd = make_fastdiv((uint32_t)k);
+  const uint32_t end = (uint32_t)sp.end, step = (uint32_t)sp.step;
+  for (uint32_t q0 = (uint32_t)sp.first; q0 < end; q0 += step * U) {
+    int32_t x[U], ip[U];
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const uint32_t q = q0 + j * step;
+      x[j] = -1;
+      if (q < end) {
+        const uint32_t i = fdiv(q, fd);
+        const int32_t t = (int32_t)(q - i * (uint32_t)k);
+        if (ldw_i32(B.cnt + i) > t) {
+          const int32_t r = ldw_i32(B.rows + q);
+          if (r < 0 && -1 - r >= F) {
+            x[j] = -1 - r - F;
+            ip[j] = ldw_i32(indptr + i) + t;
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int j = 0; j < U; ++j)
+      if (x[j] >= 0) indices_out[ip[j]] = ldw_i32(B.rows + x[j]);
   }
 }
 
@@ -671,9 +716,12 @@ __global__ void __launch_bounds__(NT) k_gather(GatherArgs a) {
 }
 
 // ============================================ world == 1: persistent kernel
-constexpr int LOADER_WARPS = 4;                      // TMA gather warps of a pipelined launch
+constexpr int LOADER_WARPS = 4;                      // TMA gather warps of a pipelined launch (default)
+constexpr int LOADER_WARPS_MAX = 8;                  // ... or 8 (dsp_ctx::loader_warps)
 constexpr int LOADER_SLOTS = 2;                      // ring slots per loader warp
 constexpr int PIPE_TEAM = PNT - 32 * LOADER_WARPS;   // sampling threads of a pipelined launch
+constexpr int PIPE_TEAM8 = PNT - 32 * LOADER_WARPS_MAX;
+constexpr int PIPE_TEAM2 = PNT - 32 * 2;
 
 struct PersistArgs {
   const int32_t *seeds;
@@ -871,7 +919,7 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
 template <int TEAM, bool PIPE>
 __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
   __shared__ Scan2Smem<TEAM> sm;
-  __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];
+  __shared__ __align__(8) uint64_t bars[LOADER_WARPS_MAX][LOADER_SLOTS];
   extern __shared__ __align__(128) char ring_smem[];
   const int blk = blockIdx.x, nblk = gridDim.x;
 
@@ -909,8 +957,8 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
     const int k = a.k[l];
     persist_sample<TEAM>(a, frontier, F, l, epoch);
     if (l > 0)
-      phase_indices(Fprev, a.k[l - 1], a.buf[(l - 1) & 1], a.out.indptr[l - 1], a.out.indices[l - 1],
-                    block_span<TEAM>((int64_t)Fprev * a.k[l - 1]));
+      phase_indices_dups(Fprev, a.k[l - 1], a.buf[(l - 1) & 1], a.out.indptr[l - 1], a.out.indices[l - 1],
+                         block_span<TEAM>((int64_t)Fprev * a.k[l - 1]));
     grid_barrier<TEAM>(a.hdr, bar);
     // scan over the F*k edge slots: each block one contiguous chunk of <= TEAM*IPT slots per round
     constexpr int64_t TILE = (int64_t)TEAM * SCAN2_IPT;
@@ -928,8 +976,8 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
       grid_barrier<TEAM>(a.hdr, bar);
       unsigned long long prefix, round_total;
       scan2_prefix<TEAM>(agg, nblk, blk, sm, &prefix, &round_total);
-      scan2_pass2<TEAM>(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
-                        a.out.src_ids[l]);
+      scan2_pass2<TEAM>(F, k, a.buf[l & 1], tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
+                        a.out.indices[l], a.out.src_ids[l]);
       carry += round_total;
       if (r + 1 < rounds) grid_barrier<TEAM>(a.hdr, bar);
     }
@@ -950,8 +998,8 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
   }
   // last layer's indices (F = num_src of the last block)
   const int l = a.L - 1;
-  phase_indices(Fprev, a.k[l], a.buf[l & 1], a.out.indptr[l], a.out.indices[l],
-                block_span<TEAM>((int64_t)Fprev * a.k[l]));
+  phase_indices_dups(Fprev, a.k[l], a.buf[l & 1], a.out.indptr[l], a.out.indices[l],
+                     block_span<TEAM>((int64_t)Fprev * a.k[l]));
   if (PIPE) {
     if (tid == 0) *a.pend_n = F;  // this call's rows, gathered by the next pipelined call / flush
     if (a.prev) helper_warp(a, ld_volatile_i32(a.gp.n_dev));

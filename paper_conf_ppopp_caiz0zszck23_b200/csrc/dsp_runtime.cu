@@ -156,6 +156,8 @@ struct dsp_ctx {
   int num_sms = 148;
   int persist_blocks_per_sm = 1;
   int lane_rounds = 4;  // DSP_LANE_ROUNDS (tuning knob, results unchanged)
+  int loader_warps = 4; // DSP_LOADER_WARPS = 2, 4 or 8 (tuning knob, results unchanged)
+  int loader_rows = 32;  // DSP_LOADER_ROWS: rows per TMA chunk, <= 32 (tuning knob, results unchanged)
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
   int gather_blocks_per_sm = 1;
   // pipelined steps: per workspace, the gather owed by its previous
@@ -548,6 +550,8 @@ const int32_t *frontier_of(const Call &k, int l) { return l == 0 ? k.seeds : k.b
 uint2 key_of(uint64_t rng_seed) { return make_uint2((uint32_t)rng_seed, (uint32_t)(rng_seed >> 32)); }
 
 // world == 1: the whole call (+ optional gather) in one cooperative kernel
+constexpr int PIPE_SMEM8_MAX = 200 * 1024;  // ring of 8 loader warps (rows up to 12.8 KB)
+
 dsp_status stage_persistent(Call &k) {
   dsp_ctx *c = k.c;
   DeviceGuard g(c->device);
@@ -592,10 +596,15 @@ dsp_status stage_persistent(Call &k) {
   a.pend_n = &ps->pend_n[pd->calls & 1];
   const int row_bytes = c->dim * 4;
   a.slot_bytes = (int)align_up((size_t)std::max(12800, row_bytes), 128);
-  a.rows_per_chunk = std::max(1, std::min(32, a.slot_bytes / std::max(1, row_bytes)));
-  const size_t smem = (size_t)LOADER_WARPS * LOADER_SLOTS * a.slot_bytes;
-  CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_persistent<PIPE_TEAM, true>, grid, block, args, smem,
-                                          k.stream));
+  a.rows_per_chunk = std::max(1, std::min(c->loader_rows, a.slot_bytes / std::max(1, row_bytes)));
+  const bool lw8 = c->loader_warps == LOADER_WARPS_MAX &&
+                   (size_t)LOADER_WARPS_MAX * LOADER_SLOTS * a.slot_bytes <= (size_t)PIPE_SMEM8_MAX;
+  const bool lw2 = c->loader_warps == 2;
+  const size_t smem = (size_t)(lw8 ? LOADER_WARPS_MAX : lw2 ? 2 : LOADER_WARPS) * LOADER_SLOTS * a.slot_bytes;
+  CUDA_TRY(c, cudaLaunchCooperativeKernel(lw8   ? (const void *)k_csp_persistent<PIPE_TEAM8, true>
+                                          : lw2 ? (const void *)k_csp_persistent<PIPE_TEAM2, true>
+                                                : (const void *)k_csp_persistent<PIPE_TEAM, true>,
+                                          grid, block, args, smem, k.stream));
   pd->ids = k.blocks[k.L - 1].src_ids;
   pd->out = k.feat_out;
   pd->stream = k.stream;
@@ -1031,6 +1040,10 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   const int pipe_smem = LOADER_WARPS * LOADER_SLOTS * 16384;  // largest ring (dim 4096)
   if (cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM, true>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
+      cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM2, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
+      cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM8, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, PIPE_SMEM8_MAX) != cudaSuccess ||
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_csp_persistent<PNT, false>, PNT, 0) != cudaSuccess ||
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_pipe, k_csp_persistent<PIPE_TEAM, true>, PNT, pipe_smem) !=
           cudaSuccess ||
@@ -1049,6 +1062,11 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   }
   c->persist_blocks_per_sm = std::min(occ, occ_pipe);
   if (getenv("DSP_LANE_ROUNDS")) c->lane_rounds = atoi(getenv("DSP_LANE_ROUNDS"));
+  if (getenv("DSP_LOADER_ROWS")) c->loader_rows = std::max(1, std::min(32, atoi(getenv("DSP_LOADER_ROWS"))));
+  if (getenv("DSP_LOADER_WARPS")) {
+    const int lw = atoi(getenv("DSP_LOADER_WARPS"));
+    if (lw == 2 || lw == LOADER_WARPS_MAX) c->loader_warps = lw;
+  }
   if (c->persist_blocks_per_sm * c->num_sms > MAX_PERSIST_BLOCKS) c->persist_blocks_per_sm = MAX_PERSIST_BLOCKS / c->num_sms;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_gather, NT, 0) != cudaSuccess || occ < 1) {
     cudaGetLastError();
