@@ -35,5 +35,14 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+def build_variant(name: str, defines) -> str:
+    """Experiment build: libdsp_<name>.so with extra -D flags (selected at run time
+    with DSP_LIB=<path>); never loaded by default."""
+    out = os.path.join(HERE, f"libdsp_{name}.so")
+    cmd = [NVCC, *NVCC_FLAGS, *[f"-D{d}" for d in defines], "-o", out, *SOURCES]
+    subprocess.check_call(cmd)
+    return out
+
+
 if __name__ == "__main__":
     print(build(force=True, verbose=True))

@@ -214,6 +214,20 @@ __device__ __forceinline__ int32_t adj_ld(const int32_t *p) {
   return v;
 }
 
+// Row extent [s, s + d) of local row lv: one 16-byte load when the pair is
+// 16-byte aligned (lv even), else two 8-byte loads.
+__device__ __forceinline__ void row_extent(const int64_t *__restrict__ indptr, int64_t lv, int64_t *s, int64_t *d) {
+  if ((lv & 1) == 0) {
+    const longlong2 p = __ldg(reinterpret_cast<const longlong2 *>(indptr + lv));
+    *s = p.x;
+    *d = p.y - p.x;
+  } else {
+    const int64_t a = __ldg(indptr + lv);
+    *s = a;
+    *d = __ldg(indptr + lv + 1) - a;
+  }
+}
+
 // ------------------------------------------------------- one node's sample
 // Lane group of G lanes (G = next pow2 >= k) samples node v.  Returns, per
 // lane t: whether slot `*slot` of the node holds sampled neighbour *u, and

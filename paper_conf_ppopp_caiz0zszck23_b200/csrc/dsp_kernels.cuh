@@ -249,8 +249,7 @@ __device__ __forceinline__ void phase_sample_lanes(const int32_t *frontier, int 
     const bool ok = active && v >= 0 && lv >= 0 && lv < n_local;
     int64_t s = 0, d = 0;
     if (ok) {
-      s = __ldg(indptr + lv);
-      d = __ldg(indptr + lv + 1) - s;
+      row_extent(indptr, lv, &s, &d);
     }
     DSTAMP(hdr, 2, (int)d, layer);
     bool valid;
@@ -301,8 +300,8 @@ __device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F,
       B.cnt[i] = 0;
       continue;
     }
-    const int64_t rs = __ldg(indptr + lv);
-    const int64_t d = __ldg(indptr + lv + 1) - rs;
+    int64_t rs, d;
+    row_extent(indptr, lv, &rs, &d);
     DSTAMP(hdr, 2, (int)d, layer);
     const bool full = d <= k;
     const int cnt = full ? (int)d : k;
@@ -371,8 +370,7 @@ __device__ __forceinline__ void phase_sample_biased(const int32_t *frontier, int
     const bool ok = v >= 0 && lv >= 0 && lv < n_local;
     int64_t s = 0, d = 0;
     if (ok) {
-      s = __ldg(indptr + lv);
-      d = __ldg(indptr + lv + 1) - s;
+      row_extent(indptr, lv, &s, &d);
     }
     uint32_t pos;
     const int cnt = sample_node_biased(ok, v, s, d, k, layer, key, weights, &pos);
@@ -1234,8 +1232,7 @@ __global__ void __launch_bounds__(NT) k_sample_remote(RemoteSampleArgs a) {
       if (active && !ok && (lane & (G - 1)) == 0) latch(a.err, E_STATE);
       int64_t rs = 0, d = 0;
       if (ok) {
-        rs = __ldg(a.indptr + lv);
-        d = __ldg(a.indptr + lv + 1) - rs;
+        row_extent(a.indptr, lv, &rs, &d);
       }
       bool valid;
       int slot, cnt;

@@ -64,7 +64,8 @@ def lib(path: str | None = None):
     """Loads libdsp.so from the package directory (never from a JIT cache)."""
     global _lib
     if _lib is None:
-        path = path or _build.LIB
+        # DSP_LIB: an alternative build of the same sources (tools/variants.py experiments)
+        path = path or os.environ.get("DSP_LIB") or _build.LIB
         if not os.path.exists(path):
             raise RuntimeError(f"libdsp.so not built ({path}); run __graft_entry__.build()")
         L = ctypes.CDLL(path)
