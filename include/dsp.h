@@ -295,12 +295,33 @@ dsp_status dsp_gather_features(dsp_ctx *ctx, const int32_t *ids, int64_t n, floa
    sampling picks for v at layer l with this rng_seed (walks meeting at a node
    at the same step continue together); a node without neighbours ends the
    walk and the remaining entries are -1.
-   starts: DEVICE int32[n] in [0, N) (else an error latches for dsp_sync);
-   traces: DEVICE int32[n][length + 1], traces[i][0] = starts[i];
-   1 <= length <= 1024.  world_size 1 only in this version (DSP_ERR_STATE
-   otherwise).  Asynchronous on `stream`. */
+   starts: DEVICE int32[n] in [0, N) (any owner; else an error latches for
+   dsp_sync and the walk is all -1); traces: DEVICE int32[n][length + 1],
+   traces[i][0] = starts[i]; 1 <= length <= 1024.  Asynchronous on `stream`.
+   world_size > 1: COLLECTIVE (every rank calls with the same length and
+   rng_seed; n may differ, 0 allowed) and needs dsp_reserve_walks.  The walk
+   follows CSP with the reshuffle removed: each step the walkers move
+   to the owner of their node through its peer-mapped inbox (one exchange
+   round: counts + header + flag), the owner takes the step and
+   stores the new node straight into the trace row at the walk's origin rank
+   over NVLink.  Traces are bit-identical for any world_size / bounds. */
 dsp_status dsp_random_walk(dsp_ctx *ctx, const int32_t *starts, int64_t n, int32_t length, uint64_t rng_seed,
                            int32_t *traces, void *stream);
+
+/* Sizes the peer-visible walk region for up to max_walks walks per rank
+   (<= 2^27) of up to max_length steps (<= 1024): inboxes of
+   world_size * max_walks walkers per (parity, sender) and the trace rows of
+   this rank's walks.  All ranks pass the same values (checked at import);
+   after dsp_load_partition, before dsp_export_handle.  Needed for
+   dsp_random_walk with world_size > 1. */
+dsp_status dsp_reserve_walks(dsp_ctx *ctx, int64_t max_walks, int32_t max_length);
+
+/* dsp_random_walk for the n_ctx ranks of one world driven by ONE host thread
+   (virtual ranks sharing a device must share a stream): stages are issued
+   rank by rank.  Arrays are indexed by position in ctxs. */
+dsp_status dsp_random_walk_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *starts,
+                                 const int64_t *n, int32_t length, uint64_t rng_seed, int32_t *const *traces,
+                                 void *const *streams);
 
 /* Synchronises `stream` and reports a latched device error (then clears it). */
 dsp_status dsp_sync(dsp_ctx *ctx, void *stream);

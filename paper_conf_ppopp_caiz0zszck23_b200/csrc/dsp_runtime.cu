@@ -17,6 +17,7 @@
 
 #include "../../include/dsp.h"
 #include "dsp_layerwise.cuh"
+#include "dsp_walk.cuh"
 
 using namespace dsp;
 
@@ -57,6 +58,11 @@ struct PeerHandle {  // fits in DSP_HANDLE_BYTES
   cudaIpcMemHandle_t lxch_ipc, indptr_ipc;
   uint64_t lxch_ptr, indptr_ptr;
   int32_t has_lxch, lw_max_seeds, lw_L, lw_sizes[DSP_MAX_LAYERS];
+  // random-walk region (dsp_reserve_walks)
+  cudaIpcMemHandle_t wxch_ipc;
+  uint64_t wxch_ptr;
+  int64_t walk_max;
+  int32_t has_wxch, walk_len;
 };
 static_assert(sizeof(PeerHandle) <= DSP_HANDLE_BYTES, "handle too large");
 
@@ -140,7 +146,7 @@ struct dsp_ctx {
   // peers
   const float *peer_feat[DSP_MAX_WORLD] = {nullptr};
   char *peer_xch[DSP_MAX_WORLD] = {nullptr};
-  void *ipc_opened[5 * DSP_MAX_WORLD] = {nullptr};  // feat, xch | fpos | lxch | indptr per peer
+  void *ipc_opened[6 * DSP_MAX_WORLD] = {nullptr};  // feat, xch | fpos | lxch | indptr | walk region per peer
   unsigned long long seq = 0;
   // layer-wise scheme (dsp_reserve_layerwise)
   bool lw_reserved = false;
@@ -150,6 +156,14 @@ struct dsp_ctx {
   char *d_lxch = nullptr;
   char *peer_lxch[DSP_MAX_WORLD] = {nullptr};
   const int64_t *peer_indptr[DSP_MAX_WORLD] = {nullptr};
+  // random walks over a partitioned graph (dsp_reserve_walks)
+  bool walk_reserved = false;
+  int64_t walk_max = 0;
+  int32_t walk_len = 0;
+  WalkLayout wl{};
+  char *d_wxch = nullptr;
+  char *peer_wxch[DSP_MAX_WORLD] = {nullptr};
+  unsigned long long wseq = 0;
   // host staging (pinned)
   WsHeader *h_hdr = nullptr;
   int *h_err = nullptr;
@@ -325,6 +339,27 @@ LwLayout make_lw_layout(int64_t cap, int32_t ncap) {
   take(x.off_inbox, sizeof(int4) * 16 * (size_t)cap);
   take(x.off_ret_cnt, sizeof(int32_t) * 2 * (size_t)cap);
   take(x.off_ret_rows, sizeof(int32_t) * 2 * (size_t)ncap);
+  x.bytes = o;
+  return x;
+}
+
+WalkLayout make_walk_layout(int world, int64_t max_walks, int32_t max_len) {
+  WalkLayout x{};
+  x.max_walks = max_walks;
+  x.max_len = max_len;
+  x.cap = std::max<int64_t>(1, (int64_t)world * max_walks);
+  size_t o = 0;
+  auto take = [&](size_t &off, size_t bytes) {
+    off = o;
+    o = align_up(o + bytes, 256);
+  };
+  take(x.off_flag, sizeof(unsigned long long) * 16);
+  take(x.off_done, sizeof(unsigned long long) * 8);
+  take(x.off_hdr, sizeof(uint4) * 16);
+  take(x.off_inbox, sizeof(int2) * 16 * (size_t)x.cap);
+  take(x.off_trace, sizeof(int32_t) * (size_t)std::max<int64_t>(1, max_walks) * (size_t)(max_len + 1));
+  take(x.off_list, sizeof(int2) * 2 * (size_t)x.cap);
+  take(x.off_ctr, sizeof(uint32_t) * 16);
   x.bytes = o;
   return x;
 }
@@ -963,7 +998,7 @@ void release(dsp_ctx *c) {
     c->h_cold = nullptr;
   }
   cudaFree(c->d_fpos);
-  for (int i = 0; i < 5 * DSP_MAX_WORLD; ++i)
+  for (int i = 0; i < 6 * DSP_MAX_WORLD; ++i)
     if (c->ipc_opened[i]) {
       cudaIpcCloseMemHandle(c->ipc_opened[i]);
       c->ipc_opened[i] = nullptr;
@@ -974,10 +1009,101 @@ void release(dsp_ctx *c) {
   cudaFree(c->d_feat);
   cudaFree(c->d_xch);
   cudaFree(c->d_lxch);
+  cudaFree(c->d_wxch);
   cudaFree(c->d_err);
   if (c->h_hdr) cudaFreeHost(c->h_hdr);
   if (c->h_err) cudaFreeHost(c->h_err);
   cudaGetLastError();
+}
+
+// Random walks over a partitioned graph: one stage of one rank.
+// stage 0 = init, 1 = shuffle of step l, 2 = step l at the owner, 3 = done, 4 = finish.
+WalkArgs walk_args(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length, uint64_t rng_seed,
+                   int32_t *traces) {
+  WalkArgs a{};
+  a.starts = starts;
+  a.n = n;
+  a.length = length;
+  a.rank = c->rank;
+  a.key = key_of(rng_seed);
+  a.indptr = c->d_indptr;
+  a.indices = c->d_indices;
+  a.lo = c->lo;
+  a.n_local = c->n_local;
+  a.bd = make_bounds(c);
+  a.L = c->wl;
+  for (int r = 0; r < DSP_MAX_WORLD; ++r) a.peers.base[r] = r < c->world ? c->peer_wxch[r] : nullptr;
+  a.traces = traces;
+  a.err = c->d_err;
+  return a;
+}
+
+dsp_status walk_stage(dsp_ctx *c, WalkArgs a, int stage, int l, unsigned long long seq0, cudaStream_t st) {
+  DeviceGuard g(c->device);
+  a.step = l;
+  const int grid = grid_for(c, 4);
+  switch (stage) {
+    case 0:
+      k_walk_init<<<(int)std::max<int64_t>(1, std::min<int64_t>((a.n * (a.length + 1) + NT - 1) / NT, grid)), NT, 0,
+                    st>>>(a);
+      break;
+    case 1:
+      a.seq = seq0 + 1 + l;
+      a.parity = (int)(a.seq & 1);
+      k_walk_scatter<<<grid, NT, 0, st>>>(a);
+      break;
+    case 2:
+      a.seq = seq0 + 1 + l;
+      a.parity = (int)(a.seq & 1);
+      k_walk_step<<<grid, NT, 0, st>>>(a);
+      break;
+    case 3:
+      a.seq = seq0 + 1 + a.length;
+      k_walk_done<<<1, 32, 0, st>>>(a);
+      break;
+    default:
+      a.seq = seq0 + 1 + a.length;
+      k_walk_finish<<<(int)std::max<int64_t>(1, std::min<int64_t>((a.n * (a.length + 1) + NT - 1) / NT, grid)), NT,
+                      0, st>>>(a);
+      break;
+  }
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+dsp_status check_walk_call(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length, int32_t *traces) {
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
+  if (length < 1 || length > 1024) return fail(c, DSP_ERR_INVALID_ARG, "length %d not in [1, 1024]", length);
+  if (n < 0 || (n > 0 && (!starts || !traces))) return fail(c, DSP_ERR_INVALID_ARG, "bad starts / traces / n");
+  if (c->world > 1) {
+    if (c->broken) return fail(c, DSP_ERR_STATE, "ctx unusable after an exchange failure");
+    if (!c->walk_reserved) return fail(c, DSP_ERR_STATE, "random walks with world_size > 1 need dsp_reserve_walks");
+    if (!c->imported) return fail(c, DSP_ERR_STATE, "dsp_import_handles first");
+    if (n > c->walk_max) return fail(c, DSP_ERR_CAPACITY, "%lld walks > reserved %lld", (long long)n, (long long)c->walk_max);
+    if (length > c->walk_len) return fail(c, DSP_ERR_CAPACITY, "length %d > reserved %d", length, c->walk_len);
+  }
+  return DSP_OK;
+}
+
+// all stages of a multi-rank walk call, stage by stage over the given ranks
+dsp_status run_walks(std::vector<dsp_ctx *> &cs, std::vector<WalkArgs> &as, std::vector<cudaStream_t> &ss,
+                     int32_t length) {
+  const unsigned long long seq0 = cs[0]->wseq;
+  for (auto *c : cs)
+    if (c->wseq != seq0) return fail(cs[0], DSP_ERR_STATE, "ranks disagree on the number of walk calls");
+  dsp_status st;
+  const size_t n = cs.size();
+  for (size_t i = 0; i < n; ++i)
+    if ((st = walk_stage(cs[i], as[i], 0, 0, seq0, ss[i])) != DSP_OK) return st;
+  for (int l = 0; l < length; ++l)
+    for (int stage = 1; stage <= 2; ++stage)
+      for (size_t i = 0; i < n; ++i)
+        if ((st = walk_stage(cs[i], as[i], stage, l, seq0, ss[i])) != DSP_OK) return st;
+  for (int stage = 3; stage <= 4; ++stage)
+    for (size_t i = 0; i < n; ++i)
+      if ((st = walk_stage(cs[i], as[i], stage, 0, seq0, ss[i])) != DSP_OK) return st;
+  for (auto *c : cs) c->wseq = seq0 + 1 + (unsigned long long)length;
+  return DSP_OK;
 }
 
 dsp_status check_gather_out(dsp_ctx *c, const float *out) {
@@ -1345,7 +1471,7 @@ dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
   dsp_ctx *c = const_cast<dsp_ctx *>(cc);
   if (!c || !out) return DSP_ERR_INVALID_ARG;
   c->err.clear();
-  if (!c->loaded || !(c->reserved || c->lw_reserved))
+  if (!c->loaded || !(c->reserved || c->lw_reserved || c->walk_reserved))
     return fail(c, DSP_ERR_STATE, "load_partition + reserve first");
   PeerHandle h;
   memset(&h, 0, sizeof(h));
@@ -1392,6 +1518,13 @@ dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
       CUDA_TRY(c, cudaIpcGetMemHandle(&h.indptr_ipc, c->d_indptr));
     }
   }
+  h.walk_max = c->walk_reserved ? c->walk_max : -1;
+  h.walk_len = c->walk_len;
+  if (c->walk_reserved) {
+    h.has_wxch = 1;
+    h.wxch_ptr = (uint64_t)(uintptr_t)c->d_wxch;
+    if (c->world > 1) CUDA_TRY(c, cudaIpcGetMemHandle(&h.wxch_ipc, c->d_wxch));
+  }
   memset(out, 0, DSP_HANDLE_BYTES);
   memcpy(out, &h, sizeof(h));
   return DSP_OK;
@@ -1400,7 +1533,7 @@ dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
 dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
   if (!c || !all) return DSP_ERR_INVALID_ARG;
   c->err.clear();
-  if (!c->loaded || !(c->reserved || c->lw_reserved))
+  if (!c->loaded || !(c->reserved || c->lw_reserved || c->walk_reserved))
     return fail(c, DSP_ERR_STATE, "load_partition + reserve first");
   if (c->imported) return fail(c, DSP_ERR_STATE, "handles already imported");
   DeviceGuard g(c->device);
@@ -1418,6 +1551,8 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
     if (h.lw_max_seeds != (c->lw_reserved ? c->lw_max_seeds : -1) || h.lw_L != c->lw_L ||
         memcmp(h.lw_sizes, c->lw_sizes, sizeof(c->lw_sizes)) != 0)
       return fail(c, DSP_ERR_STATE, "rank %d reserved a different layer-wise configuration", r);
+    if (h.walk_max != (c->walk_reserved ? c->walk_max : -1) || h.walk_len != c->walk_len)
+      return fail(c, DSP_ERR_STATE, "rank %d reserved a different random-walk configuration", r);
     if (r == c->rank) continue;
     const bool same_process = h.pid == my_pid && h.boot_id == boot_id();
     if (same_process) {
@@ -1440,7 +1575,18 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
         c->peer_lxch[r] = reinterpret_cast<char *>(h.lxch_ptr);
         c->peer_indptr[r] = reinterpret_cast<const int64_t *>(h.indptr_ptr);
       }
+      if (h.has_wxch) c->peer_wxch[r] = reinterpret_cast<char *>(h.wxch_ptr);
     } else {
+      if (h.has_wxch) {
+        void *p = nullptr;
+        cudaError_t e = cudaIpcOpenMemHandle(&p, h.wxch_ipc, cudaIpcMemLazyEnablePeerAccess);
+        if (e != cudaSuccess) {
+          cudaGetLastError();
+          return fail(c, DSP_ERR_PEER, "cudaIpcOpenMemHandle(walk region of rank %d): %s", r, cudaGetErrorString(e));
+        }
+        c->ipc_opened[5 * DSP_MAX_WORLD + r] = p;
+        c->peer_wxch[r] = static_cast<char *>(p);
+      }
       if (h.has_lxch) {
         void *p = nullptr, *q = nullptr;
         cudaError_t e = cudaIpcOpenMemHandle(&p, h.lxch_ipc, cudaIpcMemLazyEnablePeerAccess);
@@ -1637,15 +1783,68 @@ dsp_status dsp_random_walk(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
   if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
-  if (c->world != 1) return fail(c, DSP_ERR_STATE, "random walks over a partitioned graph are not implemented yet");
-  if (length < 1 || length > 1024) return fail(c, DSP_ERR_INVALID_ARG, "length %d not in [1, 1024]", length);
-  if (n < 0 || (n > 0 && (!starts || !traces))) return fail(c, DSP_ERR_INVALID_ARG, "bad starts / traces / n");
+  dsp_status st = check_walk_call(c, starts, n, length, traces);
+  if (st != DSP_OK) return st;
+  if (c->world > 1) {  // COLLECTIVE: CSP push without reshuffle
+    std::vector<dsp_ctx *> cs{c};
+    std::vector<WalkArgs> as{walk_args(c, starts, n, length, rng_seed, traces)};
+    std::vector<cudaStream_t> ss{static_cast<cudaStream_t>(stream)};
+    return run_walks(cs, as, ss, length);
+  }
   if (n == 0) return DSP_OK;
   DeviceGuard g(c->device);
   const int64_t want = (n + NT - 1) / NT;
   k_random_walk<<<(int)std::min<int64_t>(want, grid_for(c, 8)), NT, 0, static_cast<cudaStream_t>(stream)>>>(
       starts, n, length, key_of(rng_seed), c->d_indptr, c->d_indices, c->N, traces, c->d_err);
   CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+dsp_status dsp_random_walk_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *starts,
+                                 const int64_t *n, int32_t length, uint64_t rng_seed, int32_t *const *traces,
+                                 void *const *streams) {
+  if (!ctxs || n_ctx < 1 || !starts || !n || !traces || !streams) return DSP_ERR_INVALID_ARG;
+  const int world = ctxs[0] ? ctxs[0]->world : 0;
+  if (n_ctx != world) return fail(ctxs[0], DSP_ERR_INVALID_ARG, "dsp_random_walk_group needs all %d ranks", world);
+  std::vector<int> seen(world, 0);
+  std::vector<dsp_ctx *> cs(n_ctx);
+  std::vector<WalkArgs> as(n_ctx);
+  std::vector<cudaStream_t> ss(n_ctx);
+  for (int i = 0; i < n_ctx; ++i) {
+    if (!ctxs[i] || ctxs[i]->world != world || seen[ctxs[i]->rank]++)
+      return fail(ctxs[0], DSP_ERR_INVALID_ARG, "ctxs must be the distinct ranks of one world");
+    for (int j = 0; j < i; ++j)
+      if (ctxs[j]->device == ctxs[i]->device && streams[j] != streams[i])
+        return fail(ctxs[0], DSP_ERR_INVALID_ARG,
+                    "virtual ranks on one device must share a stream (stage-by-stage issue)");
+    ctxs[i]->err.clear();
+    dsp_status st = check_walk_call(ctxs[i], starts[i], n[i], length, traces[i]);
+    if (st != DSP_OK) return st;
+    cs[i] = ctxs[i];
+    as[i] = walk_args(ctxs[i], starts[i], n[i], length, rng_seed, traces[i]);
+    ss[i] = static_cast<cudaStream_t>(streams[i]);
+  }
+  if (world == 1) return dsp_random_walk(ctxs[0], starts[0], n[0], length, rng_seed, traces[0], streams[0]);
+  return run_walks(cs, as, ss, length);
+}
+
+dsp_status dsp_reserve_walks(dsp_ctx *c, int64_t max_walks, int32_t max_length) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
+  if (c->walk_reserved) return fail(c, DSP_ERR_STATE, "walks already reserved");
+  if (c->imported) return fail(c, DSP_ERR_STATE, "reserve before dsp_import_handles");
+  if (max_walks < 0 || max_walks > WALK_MAX) return fail(c, DSP_ERR_INVALID_ARG, "max_walks must be in [0, 2^27]");
+  if (max_length < 1 || max_length > 1024) return fail(c, DSP_ERR_INVALID_ARG, "max_length must be in [1, 1024]");
+  DeviceGuard g(c->device);
+  c->wl = make_walk_layout(c->world, max_walks, max_length);
+  CUDA_TRY(c, cudaMalloc(&c->d_wxch, c->wl.bytes));
+  CUDA_TRY(c, cudaMemset(c->d_wxch, 0, c->wl.bytes));
+  CUDA_TRY(c, cudaDeviceSynchronize());
+  c->walk_max = max_walks;
+  c->walk_len = max_length;
+  c->peer_wxch[c->rank] = c->d_wxch;
+  c->walk_reserved = true;
   return DSP_OK;
 }
 

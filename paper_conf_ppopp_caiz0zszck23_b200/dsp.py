@@ -36,6 +36,7 @@ ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_creat
                "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve", "dsp_reserve_layerwise", "dsp_export_handle", "dsp_import_handles",
                "dsp_sample_bounds", "dsp_sample_bounds_layerwise", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                "dsp_pipeline_flush", "dsp_set_persistent_blocks", "dsp_gather_features", "dsp_random_walk",
+               "dsp_reserve_walks", "dsp_random_walk_group",
                "dsp_sync")
 DSP_ASYNC = 1
 DSP_PIPELINED = 2
@@ -96,11 +97,14 @@ def lib(path: str | None = None):
         L.dsp_pipeline_flush.argtypes = [P, P]
         L.dsp_set_persistent_blocks.argtypes = [P, i32]
         L.dsp_random_walk.argtypes = [P, P, i64, i32, ctypes.c_uint64, P, P]
+        L.dsp_reserve_walks.argtypes = [P, i64, i32]
+        L.dsp_random_walk_group.argtypes = [P, i32, P, P, i32, ctypes.c_uint64, P, P]
         L.dsp_sync.argtypes = [P, P]
         for name in ("dsp_create", "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve",
                      "dsp_reserve_layerwise", "dsp_sample_bounds_layerwise", "dsp_export_handle",
                      "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                      "dsp_pipeline_flush", "dsp_random_walk", "dsp_set_persistent_blocks",
+                     "dsp_reserve_walks", "dsp_random_walk_group",
                      "dsp_gather_features", "dsp_sync"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
@@ -258,6 +262,21 @@ def dsp_random_walk(ctx, starts, n: int, length: int, rng_seed: int, traces, str
                                  ctypes.c_void_p(stream)), ctx)
 
 
+def dsp_reserve_walks(ctx, max_walks: int, max_length: int) -> None:
+    _check(lib().dsp_reserve_walks(ctx, max_walks, max_length), ctx)
+
+
+def dsp_random_walk_group(ctxs, starts, n, length: int, rng_seed: int, traces, streams) -> None:
+    k = len(ctxs)
+    c_ctxs = (ctypes.c_void_p * k)(*[c.value if isinstance(c, ctypes.c_void_p) else c for c in ctxs])
+    c_starts = (ctypes.c_void_p * k)(*[x.data_ptr() for x in starts])
+    c_n = (ctypes.c_int64 * k)(*[int(x) for x in n])
+    c_tr = (ctypes.c_void_p * k)(*[x.data_ptr() for x in traces])
+    c_st = (ctypes.c_void_p * k)(*streams)
+    _check(lib().dsp_random_walk_group(c_ctxs, k, c_starts, c_n, length, ctypes.c_uint64(rng_seed), c_tr, c_st),
+           ctxs[0])
+
+
 def dsp_sync(ctx, stream: int) -> None:
     _check(lib().dsp_sync(ctx, ctypes.c_void_p(stream)), ctx)
 
@@ -283,7 +302,10 @@ class Sampler:
     def __init__(self, bounds, indptr, indices, features, fanouts, max_seeds: int, rank: int = 0,
                  world_size: int = 1, device: int | None = None,
                  exchange: Callable[[bytes], list] | None = None, connect: bool = True, n_slots: int = 1,
-                 edge_weights=None, n_workspaces: int = 1, hot_rows: int | None = None, scheme: str = "node"):
+                 edge_weights=None, n_workspaces: int = 1, hot_rows: int | None = None, scheme: str = "node",
+                 max_walks: int | None = None, max_walk_length: int = 1024):
+        """max_walks: reserve the random-walk region (needed for random_walk when
+        world_size > 1) for up to max_walks walks per rank of max_walk_length steps."""
         import torch
         self.torch = torch
         self.device = torch.cuda.current_device() if device is None else device
@@ -310,6 +332,8 @@ class Sampler:
             else:
                 dsp_reserve(self.ctx, self.max_seeds, self.fanouts)
                 ms, me, ws = dsp_sample_bounds(self.ctx, self.max_seeds, self.fanouts)
+            if max_walks is not None:
+                dsp_reserve_walks(self.ctx, int(max_walks), int(max_walk_length))
         except Exception:
             dsp_destroy(self.ctx)
             self.ctx = None
@@ -446,14 +470,15 @@ class LocalGroup:
     GPUs of this node."""
 
     def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int], hot_rows=None,
-                 scheme: str = "node"):
+                 scheme: str = "node", max_walks: int | None = None, max_walk_length: int = 1024):
         """shards[r] = (indptr, indices, features[, edge_weights]) of rank r;
         hot_rows[r] (optional) enables the cold-feature tier."""
         P = len(shards)
         assert len(devices) == P and len(bounds) == P + 1
         self.samplers = [Sampler(bounds, s[0], s[1], s[2], fanouts, max_seeds, rank=r, world_size=P,
                                  device=devices[r], connect=False, edge_weights=s[3] if len(s) > 3 else None,
-                                 hot_rows=None if hot_rows is None else hot_rows[r], scheme=scheme)
+                                 hot_rows=None if hot_rows is None else hot_rows[r], scheme=scheme,
+                                 max_walks=max_walks, max_walk_length=max_walk_length)
                          for r, s in enumerate(shards)]
         handles = [dsp_export_handle(s.ctx) for s in self.samplers]
         for s in self.samplers:
@@ -469,6 +494,15 @@ class LocalGroup:
                          S[0].workspace_bytes, (DSP_BIASED if biased else 0) | S[0]._sflag,
                          [s.stream() for s in S])
         return [s.blocks() for s in S]
+
+    def random_walk(self, starts_per_rank, length: int, rng_seed: int):
+        """Walk traces of every rank, CSP push without reshuffle."""
+        torch = self.samplers[0].torch
+        S = self.samplers
+        outs = [torch.empty((x.numel(), length + 1), dtype=torch.int32, device=x.device) for x in starts_per_rank]
+        dsp_random_walk_group([s.ctx for s in S], starts_per_rank, [x.numel() for x in starts_per_rank], length,
+                              rng_seed, outs, [s.stream() for s in S])
+        return outs
 
     def close(self):
         for s in self.samplers:

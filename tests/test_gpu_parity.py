@@ -429,6 +429,51 @@ def test_random_walks_tiny(pkg, tiny):
     s.close()
 
 
+@pytest.mark.parametrize("P", [2, 4, 8])
+def test_random_walks_virtual_ranks(pkg, tiny, P):
+    """Walks over a partitioned graph (CSP push, reshuffle removed):
+    every rank's traces equal the single-device oracle's, whatever P; walks
+    start on any owner, meet, terminate at isolated nodes; a rank with no
+    walks still takes part; repeated calls reuse the exchange region."""
+    cfg, ip, ix, feats = tiny
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi]))
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 8, devices=[0] * P, max_walks=3000, max_walk_length=64)
+    isolated = np.nonzero(np.diff(ip) == 0)[0][:2].astype(np.int32)
+    rng = np.random.default_rng(P)
+    for call, L in enumerate((1, 7, 64)):
+        starts = [rng.integers(0, cfg.num_nodes, size=int(rng.integers(1, 3000)), dtype=np.int64).astype(np.int32)
+                  for _ in range(P)]
+        starts[0] = np.concatenate([starts[0], isolated, starts[0][:3]])   # dead ends + shared walkers
+        if call == 1:
+            starts[P - 1] = starts[P - 1][:0]                              # a rank without walks
+        tr = grp.random_walk([torch.from_numpy(x).cuda() for x in starts], L, 0xBEEF + L)
+        for r in range(P):
+            grp.samplers[r].sync()
+            exp = oracle.random_walk(ip, ix, starts[r], L, 0xBEEF + L)
+            assert np.array_equal(tr[r].cpu().numpy(), exp), (P, r, L)
+    with pytest.raises(pkg.DSPError) as e:   # beyond the reserved length
+        grp.random_walk([torch.zeros(1, dtype=torch.int32, device="cuda") for _ in range(P)], 65, 1)
+    assert e.value.status == pkg.dsp.DSP_ERR_CAPACITY
+    grp.close()
+
+
+def test_random_walks_need_reservation(pkg, tiny):
+    cfg, ip, ix, feats = tiny
+    bnds = datagen.bounds(cfg.num_nodes, 2)
+    shards = [datagen.shard(ip, ix, int(bnds[r]), int(bnds[r + 1])) + (feats[int(bnds[r]):int(bnds[r + 1])],)
+              for r in range(2)]
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 8, devices=[0, 0])
+    with pytest.raises(pkg.DSPError) as e:
+        grp.random_walk([torch.zeros(1, dtype=torch.int32, device="cuda") for _ in range(2)], 3, 1)
+    assert e.value.status == pkg.dsp.DSP_ERR_STATE
+    grp.close()
+
+
 @pytest.mark.slow
 def test_random_walks_products(pkg, products):
     cfg, ip, ix = products
