@@ -4,7 +4,9 @@ run with two processes sharing the one GPU of this environment: the same code
 path bench.py --gpus N takes with one process per GPU.  Without MPS the two
 processes' kernels time-slice, so this checks correctness, not speed.
 Each rank's blocks must equal the oracle on its seeds; the one-sided gather
-reads the peer's feature shard through the IPC mapping."""
+reads the peer's feature shard through the IPC mapping; random walks move
+walkers between the processes and store trace entries into the peer's
+walk region."""
 import os
 import socket
 
@@ -45,7 +47,8 @@ def _rank(rank, world, port, q, hot=None, scheme="node"):
         sizes = (300, 600) if scheme == "layer" else cfg.fanouts
         s = pkg.Sampler(bnds, sip, six, feats, sizes, 32, rank=rank, world_size=world, device=0,
                         exchange=pkg.torch_exchange(), n_slots=2,
-                        hot_rows=None if hot is None else (hi - lo) * hot // 4, scheme=scheme)
+                        hot_rows=None if hot is None else (hi - lo) * hot // 4, scheme=scheme,
+                        max_walks=500, max_walk_length=16)
         train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
         batches = datagen.rank_seed_batches(train, bnds, rank, 32, 0)
         for step in range(3):
@@ -60,6 +63,12 @@ def _rank(rank, world, port, q, hot=None, scheme="node"):
             exp = datagen.features_of(ref[-1]["src_ids"], cfg.dim)
             if not np.array_equal(feat.cpu().numpy().view(np.uint32), exp.view(np.uint32)):
                 ok, detail = False, f"step {step} features"
+        # random walks over the partitioned graph: walkers cross processes
+        starts = np.random.default_rng(rank).integers(0, cfg.num_nodes, size=400 + 50 * rank).astype(np.int32)
+        tr = s.random_walk(torch.from_numpy(starts).cuda(), 16, 0xC0DE)
+        s.sync()
+        if not np.array_equal(tr.cpu().numpy(), oracle.random_walk(ip, ix, starts, 16, 0xC0DE)):
+            ok, detail = False, "random walk traces"
         dist.barrier()
         s.close()
     except Exception as e:  # reported to the parent
