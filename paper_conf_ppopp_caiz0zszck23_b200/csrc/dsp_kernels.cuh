@@ -40,8 +40,29 @@ constexpr int MAX_PERSIST_BLOCKS = 1024;
 struct WsPersist {
   uint32_t epoch;      // last relabel epoch used with this workspace
   int32_t pend_n[2];   // row counts of pipelined calls (alternating), read by the next call / flush
-  uint32_t pad[61];
+  uint32_t hclear;     // epoch at the last zeroing of the relabel hash table (tags unique within 255)
+  uint32_t hmask, hoff; // its layout then (slots - 1, offset in 256-B units)
+  uint32_t pad[58];
 };
+
+// A call using epochs (e0, e0 + L] must first zero the hash table when a tag
+// could repeat (every word alive was written after the last zeroing) or when
+// the table sits elsewhere than at the last zeroing (a plan of another size).
+__device__ __forceinline__ uint32_t hash_off(const WsPersist *ps, const unsigned long long *first) {
+  return (uint32_t)((reinterpret_cast<const char *>(first) - reinterpret_cast<const char *>(ps)) >> 8);
+}
+__device__ __forceinline__ bool hash_clear_due(const WsPersist *ps, uint32_t e0, uint32_t L, uint32_t mask,
+                                               const unsigned long long *first) {
+  if (!mask) return false;
+  const volatile WsPersist *v = ps;
+  return e0 + L >= v->hclear + 255u || v->hmask != mask || v->hoff != hash_off(ps, first);
+}
+__device__ __forceinline__ void hash_cleared(WsPersist *ps, uint32_t e0, uint32_t mask,
+                                             const unsigned long long *first) {
+  ps->hclear = e0;
+  ps->hmask = mask;
+  ps->hoff = hash_off(ps, first);
+}
 
 // Per-call state (memset to 0 by the host before every call).
 struct WsHeader {
@@ -66,7 +87,8 @@ struct LayerBufs {
   int32_t *cnt;                 // [F] sampled count per frontier node
   int32_t *rows;                // [F*k] sampled neighbour (global id) of edge slot q = i*k + slot
   unsigned long long *status;   // [0] tile ticket, [1 + t] tile status (look-back scan)
-  unsigned long long *first;    // [N] relabel map
+  unsigned long long *first;    // relabel map: [N] direct words, or [mask + 1] hash slots
+  uint32_t mask;                // 0: direct map indexed by global id; else hash table of mask + 1 slots
 };
 
 struct Outputs {
@@ -119,6 +141,72 @@ __device__ __forceinline__ void map_st(unsigned long long *p, unsigned long long
 }
 __device__ __forceinline__ void mark(unsigned long long *first, int32_t u, uint32_t epoch, uint32_t x) {
   map_red_max(first + u, mark_word(epoch, x));
+}
+
+// ------------------------------------------ relabel hash table (large N)
+// For graphs whose direct map (8 B per node and parity) cannot stay in L2,
+// the map is an open-addressing table sized to the batch (the north star's
+// "GPU hash table"): slot word = tag(8) | key(31) | ~x(25),
+// tag = epoch % 255 + 1 (0 = never used).  A key is claimed with a CAS on a
+// slot whose tag is not the current one, then lowered with the same
+// fire-and-forget max as the direct map (equal high bits: the max keeps the
+// smallest x).  Linear probing from hash32(key); the table is zeroed when the
+// epoch crosses a multiple of 255, so a tag is never reused while a word
+// carrying it is alive.  x < 2^25 (checked by the host plan).
+__device__ __forceinline__ uint32_t htag(uint32_t epoch) { return epoch % 255u + 1u; }
+__device__ __forceinline__ unsigned long long hword(uint32_t epoch, int32_t u, uint32_t x) {
+  return ((unsigned long long)htag(epoch) << 56) | ((unsigned long long)(uint32_t)u << 25) |
+         (unsigned long long)(0x1ffffffu - x);
+}
+// word of (epoch, key, x) in the layout of B
+__device__ __forceinline__ unsigned long long mword(const LayerBufs &B, uint32_t epoch, int32_t u, uint32_t x) {
+  return B.mask ? hword(epoch, u, x) : mark_word(epoch, x);
+}
+// x of a word of the current epoch
+__device__ __forceinline__ uint32_t mword_x(const LayerBufs &B, unsigned long long w) {
+  return B.mask ? 0x1ffffffu - (uint32_t)(w & 0x1ffffffull) : mark_x(w);
+}
+// claims (or finds) the slot of key u; returns its word pointer and the word seen there
+__device__ __forceinline__ unsigned long long *hash_claim(const LayerBufs &B, int32_t u, uint32_t epoch, uint32_t x,
+                                                        unsigned long long *seen) {
+  const unsigned long long want = hword(epoch, u, x), hi = want >> 25;
+  const unsigned long long tag = (unsigned long long)htag(epoch);
+  uint32_t h = hash32((uint32_t)u) & B.mask;
+  while (true) {
+    unsigned long long *p = B.first + h;
+    unsigned long long w = map_ld(p);
+    if ((w >> 56) != tag) {  // free in this epoch: claim it
+      const unsigned long long old = atomicCAS(p, w, want);
+      if (old == w) {
+        *seen = 0ull;
+        return p;
+      }
+      w = old;
+      if ((w >> 56) != tag) continue;  // still another epoch's word: retry this slot
+    }
+    if ((w >> 25) == hi) {
+      *seen = w;
+      return p;
+    }
+    h = (h + 1u) & B.mask;
+  }
+}
+// slot of key u (inserted earlier in this epoch)
+__device__ __forceinline__ unsigned long long *map_find(const LayerBufs &B, int32_t u, uint32_t epoch) {
+  if (!B.mask) return B.first + u;
+  const unsigned long long hi = ((unsigned long long)htag(epoch) << 31) | (uint32_t)u;
+  uint32_t h = hash32((uint32_t)u) & B.mask;
+  while ((map_ld(B.first + h) >> 25) != hi) h = (h + 1u) & B.mask;
+  return B.first + h;
+}
+__device__ __forceinline__ void mark(const LayerBufs &B, int32_t u, uint32_t epoch, uint32_t x) {
+  if (!B.mask) {
+    map_red_max(B.first + u, mark_word(epoch, x));
+    return;
+  }
+  unsigned long long seen;
+  unsigned long long *p = hash_claim(B, u, epoch, x, &seen);
+  if (seen) map_red_max(p, hword(epoch, u, x));
 }
 
 // q / k for a fixed small divisor k: one 64-bit multiply-high with
@@ -221,6 +309,22 @@ __device__ __forceinline__ void mark_dst(unsigned long long *first, int32_t v, i
     mark(first, v, epoch, (uint32_t)i);
   }
 }
+__device__ __forceinline__ void mark_dst(const LayerBufs &B, int32_t v, int i, int F, int layer, uint32_t epoch,
+                                         int *err) {
+  if (!B.mask) {
+    mark_dst(B.first, v, i, F, layer, epoch, err);
+    return;
+  }
+  unsigned long long seen;
+  unsigned long long *p = hash_claim(B, v, epoch, (uint32_t)i, &seen);
+  if (!seen) return;
+  if (layer == 0) {  // atomic: of two equal seeds the later sees the earlier's dst index
+    const unsigned long long old = map_atom_max(p, hword(epoch, v, (uint32_t)i));
+    if (mword_x(B, old) < (uint32_t)F) latch(err, E_DUP);
+  } else {
+    map_red_max(p, hword(epoch, v, (uint32_t)i));
+  }
+}
 
 // Lane-group sampling (G lanes per node, G = next pow2 >= k): the draws run
 // on separate lanes, Floyd's resolution and the ranking via shuffles
@@ -261,14 +365,14 @@ __device__ __forceinline__ void phase_sample_lanes(const int32_t *frontier, int 
       B.cnt[i] = cnt;
       if (src_out) src_out[i] = v;  // dst copy (R17)
       if (ok)
-        mark_dst(B.first, v, i, F, layer, epoch, err);
+        mark_dst(B, v, i, F, layer, epoch, err);
       else
         latch(err, E_RANGE);
     }
     if (valid) {
       const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)slot;
       B.rows[q] = u;
-      mark(B.first, u, epoch, (uint32_t)F + q);
+      mark(B, u, epoch, (uint32_t)F + q);
     }
     DSTAMP(hdr, 5, 0, layer);
     dbg_first = false;
@@ -335,14 +439,14 @@ __device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F,
     }
     DSTAMP(hdr, 3, u[0] + u[KB - 1], layer);
     B.cnt[i] = cnt;
-    mark_dst(B.first, v, i, F, layer, epoch, err);
+    mark_dst(B, v, i, F, layer, epoch, err);
     const uint32_t q0 = (uint32_t)i * (uint32_t)k;
 #pragma unroll
     for (int t = 0; t < KB; ++t) {
       if (t < cnt) {
         const uint32_t q = q0 + (uint32_t)((slots >> (4 * t)) & 15u);
         B.rows[q] = u[t];
-        mark(B.first, u[t], epoch, (uint32_t)F + q);
+        mark(B, u[t], epoch, (uint32_t)F + q);
       }
     }
     DSTAMP(hdr, 5, 0, layer);
@@ -378,7 +482,7 @@ __device__ __forceinline__ void phase_sample_biased(const int32_t *frontier, int
       B.cnt[i] = cnt;
       if (src_out) src_out[i] = v;
       if (ok)
-        mark_dst(B.first, v, i, F, layer, epoch, err);
+        mark_dst(B, v, i, F, layer, epoch, err);
       else
         latch(err, E_RANGE);
     }
@@ -386,7 +490,7 @@ __device__ __forceinline__ void phase_sample_biased(const int32_t *frontier, int
       const int32_t u = __ldg(indices + s + pos);
       const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)lane;
       B.rows[q] = u;
-      mark(B.first, u, epoch, (uint32_t)F + q);
+      mark(B, u, epoch, (uint32_t)F + q);
     }
   }
 }
@@ -440,15 +544,15 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
   }
   unsigned long long w[SCAN2_IPT];
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? map_ld(B.first + u[j]) : 0ull;
+  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? map_ld(map_find(B, u[j], epoch)) : 0ull;
   R.vbits = R.fbits = 0;
 #pragma unroll
   for (int j = 0; j < SCAN2_IPT; ++j) {
     const bool valid = c[j] > 0;
-    const bool first = valid && w[j] == mark_word(epoch, (uint32_t)F + q0 + j * TEAM);
+    const bool first = valid && w[j] == mword(B, epoch, u[j], (uint32_t)F + q0 + j * TEAM);
     // a valid slot that is not u's first occurrence keeps x (u's smallest order
     // key: its dst index, or F + the slot of its first occurrence) as -1 - x
-    if (valid && !first) B.rows[q0 + j * TEAM] = -1 - (int32_t)mark_x(w[j]);
+    if (valid && !first) B.rows[q0 + j * TEAM] = -1 - (int32_t)mword_x(B, w[j]);
     R.vbits |= (valid ? 1u : 0u) << j;
     R.fbits |= (first ? 1u : 0u) << j;
     const uint32_t bv = __ballot_sync(FULL_MASK, valid), bf = __ballot_sync(FULL_MASK, first);
@@ -593,8 +697,8 @@ __device__ __forceinline__ void phase_indices_dups(int F, int k, const LayerBufs
 
 // ---------------------------------------------------------- write indices
 // indices[indptr[i] + t] = local id of the src of slot q = i*k + t.
-__device__ __forceinline__ void phase_indices(int F, int k, const LayerBufs &B, const int32_t *indptr,
-                                              int32_t *indices_out, const Span &sp) {
+__device__ __forceinline__ void phase_indices(int F, int k, const LayerBufs &B, uint32_t epoch,
+                                              const int32_t *indptr, int32_t *indices_out, const Span &sp) {
   constexpr int U = 4;  // items per thread in flight
   const FastDiv fd = make_fastdiv((uint32_t)k);
   const uint32_t end = (uint32_t)sp.end, step = (uint32_t)sp.step;
@@ -617,10 +721,10 @@ __device__ __forceinline__ void phase_indices(int F, int k, const LayerBufs &B, 
     }
     unsigned long long w[U];
 #pragma unroll
-    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? map_ld(B.first + u[j]) : 0ull;
+    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? map_ld(map_find(B, u[j], epoch)) : 0ull;
 #pragma unroll
     for (int j = 0; j < U; ++j)
-      if (c[j] > 0) indices_out[ip[j]] = (int32_t)mark_x(w[j]);
+      if (c[j] > 0) indices_out[ip[j]] = (int32_t)mword_x(B, w[j]);
   }
 }
 
@@ -943,6 +1047,14 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
   const int64_t nthreads = (int64_t)gridDim.x * TEAM;
   uint32_t bar = 0;  // grid barrier target
   const uint32_t e0 = *(volatile const uint32_t *)&a.persist->epoch;
+  const bool hclear = hash_clear_due(a.persist, e0, (uint32_t)a.L, a.buf[0].mask, a.buf[0].first);
+  if (hclear) {  // zero both parities of the relabel hash table (once per ~255 / L calls)
+    for (int64_t i = tid; i <= (int64_t)a.buf[0].mask; i += nthreads) {
+      a.buf[0].first[i] = 0ull;
+      a.buf[1].first[i] = 0ull;
+    }
+    grid_barrier<TEAM>(a.hdr, bar);
+  }
   if (tid == 0) {  // the host cleared the header just before the launch
     a.hdr->t[0] = globaltimer_ns();
     a.hdr->F[0] = a.B;
@@ -1010,6 +1122,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
     __threadfence();
     if (atomicAdd(&a.hdr->done, 1u) == gridDim.x - 1) {
       a.persist->epoch = e0 + (uint32_t)a.L;
+      if (hclear) hash_cleared(a.persist, e0, a.buf[0].mask, a.buf[0].first);
       a.hdr->t[23] = globaltimer_ns();
       a.hdr->done = 0u;
     }
@@ -1303,13 +1416,13 @@ __global__ void __launch_bounds__(NT) k_unpermute_mark(UnpermuteArgs a) {
     const int c = __ldcv(xch_ret_cnt(a.self, a.L, a.parity, o) + j);
     if (t == 0) {
       a.buf.cnt[i] = c;
-      mark_dst(a.buf.first, v, i, F, a.layer, epoch, a.err);
+      mark_dst(a.buf, v, i, F, a.layer, epoch, a.err);
     }
     if (t < c) {
       const int32_t u = __ldcv(xch_ret_rows(a.self, a.L, a.parity, o) + (int64_t)j * a.L.kmax + t);
       const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)t;
       a.buf.rows[q] = u;
-      mark(a.buf.first, u, epoch, (uint32_t)F + q);
+      mark(a.buf, u, epoch, (uint32_t)F + q);
     }
   }
 }
@@ -1374,7 +1487,7 @@ __global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
     for (int j = 0; j < SCAN_ITEMS; ++j) {
       if (c[j] > 0) {
         vbits |= 1u << j;
-        if (map_ld(B.first + u[j]) == mark_word(epoch, (uint32_t)F + q0 + j)) fbits |= 1u << j;
+        if (map_ld(map_find(B, u[j], epoch)) == mword(B, epoch, u[j], (uint32_t)F + q0 + j)) fbits |= 1u << j;
       }
     }
     const unsigned long long mine = pack2(__popc(vbits), __popc(fbits));
@@ -1440,7 +1553,7 @@ __global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
         if (q == i * (uint32_t)k) a.indptr_out[i] = (int32_t)pv;
         if (fbits & (1u << j)) {
           const uint32_t nid = (uint32_t)F + pf;
-          map_st(B.first + u[j], mark_word(epoch, nid));
+          map_st(map_find(B, u[j], epoch), mword(B, epoch, u[j], nid));
           a.src_ids_out[nid] = u[j];
         }
         pv += (vbits >> j) & 1u;
@@ -1464,7 +1577,8 @@ __global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
 
 __global__ void __launch_bounds__(NT) k_write_indices(ScanArgs a) {
   const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
-  phase_indices(F, a.k, a.buf, a.indptr_out, a.indices_out, grid_span((int64_t)F * a.k));
+  const uint32_t epoch = a.persist->epoch + 1u + (uint32_t)a.layer;
+  phase_indices(F, a.k, a.buf, epoch, a.indptr_out, a.indices_out, grid_span((int64_t)F * a.k));
 }
 
 // fp32 edge weights -> 16.16 fixed point a = floor(w * 2^16), w in [0, 2^16)
@@ -1514,6 +1628,20 @@ __global__ void __launch_bounds__(NT) k_random_walk(const int32_t *starts, int64
 }
 
 // end of a stage-by-stage call: advance the workspace epoch
-__global__ void k_epoch_advance(WsPersist *persist, uint32_t L) { persist->epoch += L; }
+__global__ void k_epoch_advance(WsPersist *persist, uint32_t L, LayerBufs b0) {
+  if (hash_clear_due(persist, persist->epoch, L, b0.mask, b0.first)) hash_cleared(persist, persist->epoch, b0.mask, b0.first);
+  persist->epoch += L;
+}
+
+// start of a stage-by-stage call on a hashed relabel map: zero the table
+// when a tag could repeat (the same test k_epoch_advance applies at the end)
+__global__ void k_hash_clear(WsPersist *persist, uint32_t L, LayerBufs b0, LayerBufs b1) {
+  if (!hash_clear_due(persist, persist->epoch, L, b0.mask, b0.first)) return;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= (int64_t)b0.mask;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    b0.first[i] = 0ull;
+    b1.first[i] = 0ull;
+  }
+}
 
 }  // namespace dsp

@@ -107,6 +107,8 @@ struct Plan {
   int64_t S[DSP_MAX_LAYERS];       // max src
   int64_t max_F, max_slots, status_len;
   size_t off_hdr, off_agg, off_cnt[2], off_perm, off_rows[2], off_status[2], off_first[2], bytes;
+  int64_t hash_cap;                 // > 0: relabel hash table of hash_cap slots per parity (else direct map)
+  size_t off_hash[2];
   // layer-wise scheme (make_plan_lw)
   int64_t ncap, big_cap;
   size_t off_P, off_c, off_off, off_slot_node, off_excl, off_newid, off_big;
@@ -170,6 +172,7 @@ struct dsp_ctx {
   int num_sms = 148;
   int persist_blocks_per_sm = 1;
   int lane_rounds = 4;  // DSP_LANE_ROUNDS (tuning knob, results unchanged)
+  int relabel_mode = 0; // DSP_RELABEL = direct | hash (default: by N; results unchanged)
   int loader_warps = 4; // DSP_LOADER_WARPS = 2, 4 or 8 (tuning knob, results unchanged)
   int loader_rows = 32;  // DSP_LOADER_ROWS: rows per TMA chunk, <= 32 (tuning knob, results unchanged)
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
@@ -258,7 +261,14 @@ size_t plan_common(Plan &p, int64_t N) {
   return o;
 }
 
-Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L) {
+// The node-wise relabel map is a hash table sized to the batch (north star:
+// "dedup and relabel through a GPU hash table") when the direct map over all
+// N ids (8 B per node and parity) is too large to stay in L2; x = F + slot
+// must fit the 25-bit field of a hash word.
+constexpr int64_t DIRECT_MAP_MAX_N = 3 * 1000 * 1000;
+constexpr int64_t HASH_MAX_X = 1ll << 25;
+
+Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L, int relabel_mode = 0) {
   Plan p{};
   p.L = L;
   p.F[0] = num_seeds;
@@ -273,6 +283,19 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L) {
   }
   p.status_len = align_up((size_t)((p.max_slots + SCAN_TILE - 1) / SCAN_TILE + 2), 2);
   size_t o = plan_common(p, N);
+  // relabel_mode: 0 = by N, 1 = direct, 2 = hashed (DSP_RELABEL)
+  int64_t max_keys = 0;
+  for (int l = 0; l < L; ++l) max_keys = std::max(max_keys, p.F[l] + p.E[l]);
+  const bool hashed = max_keys < HASH_MAX_X && (relabel_mode == 2 || (relabel_mode == 0 && N > DIRECT_MAP_MAX_N));
+  p.hash_cap = 0;
+  if (hashed) {
+    p.hash_cap = 1024;
+    while (p.hash_cap < max_keys + max_keys / 2) p.hash_cap <<= 1;  // load factor <= 2/3
+    for (int b = 0; b < 2; ++b) {
+      p.off_hash[b] = o;
+      o = align_up(o + sizeof(unsigned long long) * (size_t)p.hash_cap, 256);
+    }
+  }
   p.off_agg = o;
   o = align_up(o + sizeof(unsigned long long) * 2 * MAX_PERSIST_BLOCKS, 256);
   for (int b = 0; b < 2; ++b) {
@@ -445,6 +468,11 @@ LayerBufs bufs_of(const Call &k, int parity) {
   b.rows = reinterpret_cast<int32_t *>(k.ws + k.plan.off_rows[parity]);
   b.status = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_status[parity]);
   b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_first[parity]);
+  b.mask = 0;
+  if (k.plan.hash_cap > 0) {
+    b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_hash[parity]);
+    b.mask = (uint32_t)(k.plan.hash_cap - 1);
+  }
   return b;
 }
 
@@ -544,7 +572,7 @@ dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_s
   // workspace and exchange capacities are planned for the reserved maximum so
   // that every rank derives the same sizes
   const int64_t plan_seeds = c->reserved ? c->max_seeds : num_seeds;
-  k.plan = make_plan(c->N, plan_seeds, fanouts, L);
+  k.plan = make_plan(c->N, plan_seeds, fanouts, L, c->relabel_mode);
   if (ws_bytes < k.plan.bytes)
     return fail(c, DSP_ERR_CAPACITY, "workspace %zu B < required %zu B", ws_bytes, k.plan.bytes);
   if (((uintptr_t)workspace & 255u) != 0) return fail(c, DSP_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
@@ -941,6 +969,14 @@ dsp_status run_calls(std::vector<Call> &calls) {
         for (int step = 0; step < 5; ++step) EACH(stage_lw(k, l, step));
         continue;
       }
+      if (l == 0)
+        for (auto &k : calls)
+          if (k.plan.hash_cap > 0) {
+            DeviceGuard g(k.c->device);
+            k_hash_clear<<<grid_for(k.c, 4), NT, 0, k.stream>>>(persist_of(k), (uint32_t)k.L, bufs_of(k, 0),
+                                                                 bufs_of(k, 1));
+            CUDA_TRY(k.c, cudaGetLastError());
+          }
       EACH(stage_clear(k, l));
       EACH(stage_shuffle(k, l));
       EACH(stage_sample_remote(k, l));
@@ -965,7 +1001,7 @@ dsp_status run_calls(std::vector<Call> &calls) {
     }
     for (auto &k : calls) {
       DeviceGuard g(k.c->device);
-      k_epoch_advance<<<1, 1, 0, k.stream>>>(persist_of(k), (uint32_t)k.L);
+      k_epoch_advance<<<1, 1, 0, k.stream>>>(persist_of(k), (uint32_t)k.L, bufs_of(k, 0));
       CUDA_TRY(k.c, cudaGetLastError());
     }
   }
@@ -1188,6 +1224,7 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   }
   c->persist_blocks_per_sm = std::min(occ, occ_pipe);
   if (getenv("DSP_LANE_ROUNDS")) c->lane_rounds = atoi(getenv("DSP_LANE_ROUNDS"));
+  if (const char *rm = getenv("DSP_RELABEL")) c->relabel_mode = !strcmp(rm, "hash") ? 2 : !strcmp(rm, "direct") ? 1 : 0;
   if (getenv("DSP_LOADER_ROWS")) c->loader_rows = std::max(1, std::min(32, atoi(getenv("DSP_LOADER_ROWS"))));
   if (getenv("DSP_LOADER_WARPS")) {
     const int lw = atoi(getenv("DSP_LOADER_WARPS"));
@@ -1397,7 +1434,7 @@ dsp_status dsp_reserve(dsp_ctx *c, int32_t max_seeds, const int32_t *fanouts, in
   dsp_status st = check_fanouts(c, fanouts, L);
   if (st != DSP_OK) return st;
   if (max_seeds < 0) return fail(c, DSP_ERR_INVALID_ARG, "max_seeds < 0");
-  Plan p = make_plan(c->N, max_seeds, fanouts, L);
+  Plan p = make_plan(c->N, max_seeds, fanouts, L, c->relabel_mode);
   for (int l = 0; l < L; ++l)
     if ((uint64_t)p.F[l] + (uint64_t)p.E[l] >= (1ull << 31))
       return fail(c, DSP_ERR_CAPACITY, "layer %d: frontier * (1 + fanout) exceeds 2^31", l);
@@ -1665,7 +1702,7 @@ dsp_status dsp_sample_bounds(const dsp_ctx *cc, int32_t num_seeds, const int32_t
   if (num_seeds < 0) return fail(c, DSP_ERR_INVALID_ARG, "num_seeds < 0");
   if (c->reserved && num_seeds > c->max_seeds)
     return fail(c, DSP_ERR_CAPACITY, "num_seeds %d > reserved max_seeds %d", num_seeds, c->max_seeds);
-  Plan p = make_plan(c->N, c->reserved ? c->max_seeds : num_seeds, fanouts, L);
+  Plan p = make_plan(c->N, c->reserved ? c->max_seeds : num_seeds, fanouts, L, c->relabel_mode);
   for (int l = 0; l < L; ++l) {
     if (max_src) max_src[l] = p.S[l];
     if (max_edges) max_edges[l] = p.E[l];
