@@ -526,102 +526,4 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
   return k;
 }
 
-// Biased sample of node v by a GROUP of G lanes (G = 8 or 16; rows of at most
-// G * BSEG positions, k <= G), so 32 / G short rows are sampled per warp
-// instead of one.  Same successive-sampling draws as sample_node_biased (the
-// running weight sums in row order do not depend on how the row is split
-// over lanes), hence identical picks.  Warp-uniform control flow: every lane
-// of the warp calls it; a group with !ok or a long row returns 0 and leaves
-// *pos alone.  Lane t < count of the group gets the t-th pick in row order.
-template <int G>
-__device__ __forceinline__ int sample_node_biased_g(bool ok, int32_t v, int64_t row_start, int64_t deg, int k,
-                                                    int layer, uint2 key, const uint32_t *__restrict__ w,
-                                                    uint32_t *pos) {
-  const int lane = threadIdx.x & 31, t = lane & (G - 1), gbase = lane & ~(G - 1);
-  const unsigned gmask = ((1u << G) - 1u) << gbase;
-  const bool act = ok && deg <= G * BSEG;
-  const int d = act ? (int)deg : 0;
-  const int S = (d + G - 1) / G;
-  const uint32_t *a = w + row_start;
-  uint32_t reg[BSEG];
-  int mypos = 0;
-#pragma unroll
-  for (int j = 0; j < BSEG; ++j) {
-    const int p = t * S + j;
-    reg[j] = (j < S && p < d) ? __ldg(a + p) : 0u;
-    mypos += reg[j] > 0u ? 1 : 0;
-  }
-  int npos = mypos, excl = mypos;
-#pragma unroll
-  for (int off = 1; off < G; off <<= 1) {
-    npos += __shfl_xor_sync(FULL_MASK, npos, off, G);
-    const int y = __shfl_up_sync(FULL_MASK, excl, off, G);
-    if (t >= off) excl += y;
-  }
-  excl -= mypos;
-  const bool take_all = npos <= k;
-  // k rounds of weighted picks (groups taking their whole row run them too and ignore the result)
-  uint32_t pick = 0xffffffffu;
-  const unsigned long long myword = t < k ? biased_word(key, t, v, layer) : 0ull;
-  for (int r0 = 0; r0 < k; ++r0) {
-    unsigned long long tot = 0;
-#pragma unroll
-    for (int j = 0; j < BSEG; ++j) tot += reg[j];
-    unsigned long long incl = tot;
-#pragma unroll
-    for (int off = 1; off < G; off <<= 1) {
-      const unsigned long long y = __shfl_up_sync(FULL_MASK, incl, off, G);
-      if (t >= off) incl += y;
-    }
-    const unsigned long long W = __shfl_sync(FULL_MASK, incl, G - 1, G);
-    const unsigned long long r = __umul64hi(__shfl_sync(FULL_MASK, myword, r0, G), W);
-    const uint32_t cross = (__ballot_sync(FULL_MASK, incl > r) & gmask) >> gbase;
-    const int L = cross ? __ffs(cross) - 1 : 0;
-    uint32_t found = 0;
-    if (cross && t == L && !take_all) {
-      unsigned long long acc = incl - tot;
-      bool done = false;
-#pragma unroll
-      for (int j = 0; j < BSEG; ++j) {
-        if (!done && acc + reg[j] > r) {
-          found = (uint32_t)(t * S + j);
-          reg[j] = 0u;  // remove the pick
-          done = true;
-        }
-        acc += reg[j];
-      }
-    }
-    found = __shfl_sync(FULL_MASK, found, L, G);
-    if (t == r0) pick = found;
-  }
-  // picks -> ascending row order: lane t takes the pick of rank t
-  uint32_t mine = 0xffffffffu;
-  for (int s2 = 0; s2 < k; ++s2) {
-    const uint32_t c = __shfl_sync(FULL_MASK, pick, s2, G);
-    int rank = 0;
-    for (int j = 0; j < k; ++j) rank += __shfl_sync(FULL_MASK, pick, j, G) < c ? 1 : 0;
-    if (rank == t) mine = c;
-  }
-  // take_all: lane t takes the t-th positive position (owner lanes hand it over)
-  for (int r0 = 0; r0 < k; ++r0) {
-    const bool own = r0 >= excl && r0 < excl + mypos;
-    uint32_t cand = 0;
-    if (own) {
-      int rr = excl;
-#pragma unroll
-      for (int j = 0; j < BSEG; ++j)
-        if (reg[j] > 0u) {
-          if (rr == r0) cand = (uint32_t)(t * S + j);
-          ++rr;
-        }
-    }
-    const uint32_t b = (__ballot_sync(FULL_MASK, own) & gmask) >> gbase;
-    const uint32_t got = __shfl_sync(FULL_MASK, cand, b ? __ffs(b) - 1 : 0, G);
-    if (take_all && t == r0) mine = got;
-  }
-  if (!act) return 0;
-  *pos = mine;
-  return take_all ? npos : k;
-}
-
 }  // namespace dsp

@@ -495,72 +495,6 @@ __device__ __forceinline__ void phase_sample_biased(const int32_t *frontier, int
   }
 }
 
-// Biased sampling with a lane group of G lanes per node (k <= G): 32 / G
-// short rows (<= G * BSEG positions) per warp iteration; the long rows of the
-// iteration are then sampled one at a time by the whole warp.
-template <int G, int TEAM = PNT>
-__device__ __forceinline__ void phase_sample_biased_g(const int32_t *frontier, int F, int layer, int k, uint2 key,
-                                                      const int64_t *__restrict__ indptr,
-                                                      const int32_t *__restrict__ indices,
-                                                      const uint32_t *__restrict__ weights, int64_t lo,
-                                                      int64_t n_local, const LayerBufs &B, uint32_t epoch,
-                                                      int32_t *src_out, int *err) {
-  constexpr int NPW = 32 / G;
-  const int lane = threadIdx.x & 31, t = lane & (G - 1);
-  const Span sp = block_span<TEAM>(F);
-  const int64_t b0 = sp.first - threadIdx.x;
-  const int wib = threadIdx.x >> 5, wpb = TEAM >> 5;
-  for (int64_t base = b0 + (int64_t)wib * NPW; base < sp.end; base += (int64_t)wpb * NPW) {
-    const int i = (int)(base + lane / G);
-    const bool active = i < sp.end;
-    const int32_t v = active ? ldw_i32(frontier + i) : 0;
-    const int64_t lv = (int64_t)v - lo;
-    const bool ok = active && v >= 0 && lv >= 0 && lv < n_local;
-    int64_t s = 0, d = 0;
-    if (ok) row_extent(indptr, lv, &s, &d);
-    uint32_t pos = 0;
-    const int cnt = sample_node_biased_g<G>(ok, v, s, d, k, layer, key, weights, &pos);
-    const bool is_long = ok && d > G * BSEG;
-    if (active && !is_long) {
-      if (t == 0) {
-        B.cnt[i] = cnt;
-        if (src_out) src_out[i] = v;
-        if (ok)
-          mark_dst(B, v, i, F, layer, epoch, err);
-        else
-          latch(err, E_RANGE);
-      }
-      if (t < cnt) {
-        const int32_t u = __ldg(indices + s + pos);
-        const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)t;
-        B.rows[q] = u;
-        mark(B, u, epoch, (uint32_t)F + q);
-      }
-    }
-    unsigned lm = __ballot_sync(FULL_MASK, is_long && t == 0);
-    while (lm) {  // long rows: the whole warp, one node at a time
-      const int src = __ffs(lm) - 1;
-      lm &= lm - 1;
-      const int32_t vv = __shfl_sync(FULL_MASK, v, src);
-      const int ii = __shfl_sync(FULL_MASK, i, src);
-      const int64_t ss = __shfl_sync(FULL_MASK, s, src), dd = __shfl_sync(FULL_MASK, d, src);
-      uint32_t pp = 0;
-      const int c2 = sample_node_biased(true, vv, ss, dd, k, layer, key, weights, &pp);
-      if (lane == 0) {
-        B.cnt[ii] = c2;
-        if (src_out) src_out[ii] = vv;
-        mark_dst(B, vv, ii, F, layer, epoch, err);
-      }
-      if (lane < c2) {
-        const int32_t u = __ldg(indices + ss + pp);
-        const uint32_t q = (uint32_t)ii * (uint32_t)k + (uint32_t)lane;
-        B.rows[q] = u;
-        mark(B, u, epoch, (uint32_t)F + q);
-      }
-    }
-  }
-}
-
 // ------------------------------------------- scan, two-phase (persistent)
 // Inside the persistent kernel every block is resident, so the scan over
 // edge slots is a static partition: pass 1 computes each item's flags, the
@@ -925,15 +859,8 @@ __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32
   const int k = a.k[l];
   const LayerBufs &B = a.buf[l & 1];
   if (a.biased) {
-    if (k <= 8)
-      phase_sample_biased_g<8, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.weights, a.lo, a.n_local, B,
-                                     epoch, a.out.src_ids[l], a.err);
-    else if (k <= 16)
-      phase_sample_biased_g<16, TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.weights, a.lo, a.n_local, B,
-                                      epoch, a.out.src_ids[l], a.err);
-    else
-      phase_sample_biased<TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.weights, a.lo, a.n_local, B, epoch,
-                                a.out.src_ids[l], a.err);
+    phase_sample_biased<TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.weights, a.lo, a.n_local, B, epoch,
+                              a.out.src_ids[l], a.err);
   } else if (k <= 16 && (int64_t)F * (k <= 4 ? 4 : k <= 8 ? 8 : 16) <= (int64_t)a.lane_rounds * gridDim.x * TEAM) {
     // small frontier (the first layers): a lane group per node, so the k
     // Philox draws run in parallel instead of back to back in one thread,
