@@ -270,6 +270,8 @@ def run_dsp(args):
                     hot_rows=None if args.hot_frac is None else int(round(args.hot_frac * (len(sip) - 1))))
     if K > 1:  # K steps in flight on K streams, each persistent launch on 1/K of the SMs
         pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(local).multi_processor_count // K)
+    for slot in range(2 * K):
+        s.feat_buffer(slot)   # allocate every output set now, not at its first use inside the timed region
     L = len(fanouts)
     steps_epoch = datagen.steps_per_epoch(train, bnds, cfg.batch)
     batches = datagen.rank_seed_batches(train, bnds, rank, cfg.batch, 0)[:steps_epoch]
@@ -320,14 +322,19 @@ def run_dsp(args):
     # ---- timed region: KS steps, inputs resident, device time via CUDA events
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     sev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(KS)]
+    for e in (ev0, ev1, *[x for pair in sev for x in pair]):
+        e.record(stream)   # torch creates the CUDA event at its first record: not inside the timed region
+    torch.cuda.synchronize()
     with ClockSampler(local) as clk:
         ev0.record(stream)
+        h0 = time.perf_counter()
         fork()
         for j in range(KS):
             step(W + j, sev[j])
         flush_all()  # the gathers of the last timed batches are inside the timed region
         join()
         ev1.record(stream)
+        host_issue_ms = (time.perf_counter() - h0) * 1e3
         s.sync()
         torch.cuda.synchronize()
     barrier()
@@ -448,12 +455,15 @@ def run_dsp(args):
                                     "the rest in pinned host memory read over UVA"),
                        "fanouts": fanouts, "batch_per_gpu": cfg.batch, "num_nodes": cfg.num_nodes,
                        "nnz": int(ip[-1]), "dim": cfg.dim, "parallelism": f"csp{world}",
-                       "l2": "inputs larger than L2 (CSR 0.5 GB + features 1.1 GB >> 126 MB L2)",
+                       "l2": (f"inputs larger than L2 (CSR {(ip.nbytes + ix.nbytes) / 1e9:.1f} GB + features "
+                              f"{cfg.num_nodes * cfg.dim * 4 / 1e9:.1f} GB >> "
+                              f"{getattr(torch.cuda.get_device_properties(local), 'L2_cache_size', 0) / 2**20:.0f} MB L2)"),
                        "step": ("dsp_sample_gather (DSP_PIPELINED: sampler(t) || loader(t-1), 2 output sets)"
                                 if pipelined else "dsp_sample_gather (async, 2 output sets)")
                        + (f", {K} streams x {torch.cuda.get_device_properties(local).multi_processor_count // K} SMs"
                           if K > 1 else "")},
             "seeds_per_s": tot_seeds / (t_max * 1e-3),
+            "host_issue_ms_per_step": host_issue_ms / KS,
             "feature_GBps": tot_rows * cfg.dim * 4 / (t_max * 1e-3) / 1e9,
             "edges_per_step": tot_edges / KS / world,
             "rows_per_step": tot_rows / KS / world,

@@ -217,6 +217,20 @@ __device__ __forceinline__ int32_t adj_ld(const int32_t *p) {
 // Row extent [s, s + d) of local row lv: one 16-byte load when the pair is
 // 16-byte aligned (lv even), else two 8-byte loads.
 __device__ __forceinline__ void row_extent(const int64_t *__restrict__ indptr, int64_t lv, int64_t *s, int64_t *d) {
+#ifdef DSP_INDPTR_EVICT_LAST
+  // experiment: keep the (degree-biased) indptr working set L2-resident
+  const unsigned long long pol = l2_policy_evict_last();
+  long long a, b;
+  if ((lv & 1) == 0) {
+    asm volatile("ld.global.nc.L2::cache_hint.v2.s64 {%0,%1}, [%2], %3;" : "=l"(a), "=l"(b) : "l"(indptr + lv), "l"(pol));
+  } else {
+    asm volatile("ld.global.nc.L2::cache_hint.s64 %0, [%1], %2;" : "=l"(a) : "l"(indptr + lv), "l"(pol));
+    asm volatile("ld.global.nc.L2::cache_hint.s64 %0, [%1], %2;" : "=l"(b) : "l"(indptr + lv + 1), "l"(pol));
+  }
+  *s = a;
+  *d = b - a;
+  return;
+#endif
   if ((lv & 1) == 0) {
     const longlong2 p = __ldg(reinterpret_cast<const longlong2 *>(indptr + lv));
     *s = p.x;
