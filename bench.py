@@ -507,7 +507,7 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-breakdown", action="store_true")
     ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
-    ap.add_argument("--instances", type=int, default=3, help="concurrent step streams (world 1)")
+    ap.add_argument("--instances", type=int, default=4, help="concurrent step streams (world 1)")
     ap.add_argument("--layer-sizes", default="1000,1000",
                     help="--scheme layer: nodes sampled per layer (Table 7: 1000,1000)")
     ap.add_argument("--scheme", choices=["uniform", "biased", "layer"], default="uniform",

@@ -1197,7 +1197,11 @@ __device__ __forceinline__ bool wait_flags(unsigned long long *flags0, int world
 // returns true in exactly one thread of the last block to finish.
 __device__ __forceinline__ bool last_block_done(uint32_t *done) {
   __shared__ int s_last;
+#ifdef DSP_EXPERIMENT_GPU_FENCE  // cost measurement on virtual ranks only (not valid across GPUs)
+  __threadfence();
+#else
   __threadfence_system();
+#endif
   __syncthreads();
   if (threadIdx.x == 0) {
     const uint32_t t = atomicAdd(done, 1u);

@@ -172,6 +172,7 @@ struct dsp_ctx {
   int num_sms = 148;
   int persist_blocks_per_sm = 1;
   int lane_rounds = 4;  // DSP_LANE_ROUNDS (tuning knob, results unchanged)
+  int stage_bps = 8;    // DSP_STAGE_BPS: blocks per SM of the owner-sample / unpermute kernels (tuning knob)
   int relabel_mode = 0; // DSP_RELABEL = direct | hash (default: by N; results unchanged)
   int loader_warps = 4; // DSP_LOADER_WARPS = 2, 4 or 8 (tuning knob, results unchanged)
   int loader_rows = 32;  // DSP_LOADER_ROWS: rows per TMA chunk, <= 32 (tuning knob, results unchanged)
@@ -774,7 +775,7 @@ dsp_status stage_sample_remote(Call &k, int l) {
   a.peers = peers_of(c);
   a.hdr = k.hdr;
   a.err = c->d_err;
-  DISPATCH_G(k.biased ? 32 : group_of(a.k), launch_remote, a, grid_for(c, 8), k.stream);
+  DISPATCH_G(k.biased ? 32 : group_of(a.k), launch_remote, a, grid_for(c, c->stage_bps), k.stream);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
 }
@@ -798,7 +799,7 @@ dsp_status stage_unpermute(Call &k, int l) {
   a.src_out = k.blocks[l].src_ids;
   a.hdr = k.hdr;
   a.err = c->d_err;
-  DISPATCH_G(group_of(a.k), launch_unpermute, a, grid_for(c, 8), k.stream);
+  DISPATCH_G(group_of(a.k), launch_unpermute, a, grid_for(c, c->stage_bps), k.stream);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
 }
@@ -1224,6 +1225,7 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   }
   c->persist_blocks_per_sm = std::min(occ, occ_pipe);
   if (getenv("DSP_LANE_ROUNDS")) c->lane_rounds = atoi(getenv("DSP_LANE_ROUNDS"));
+  if (getenv("DSP_STAGE_BPS")) c->stage_bps = std::max(1, std::min(8, atoi(getenv("DSP_STAGE_BPS"))));
   if (const char *rm = getenv("DSP_RELABEL")) c->relabel_mode = !strcmp(rm, "hash") ? 2 : !strcmp(rm, "direct") ? 1 : 0;
   if (getenv("DSP_LOADER_ROWS")) c->loader_rows = std::max(1, std::min(32, atoi(getenv("DSP_LOADER_ROWS"))));
   if (getenv("DSP_LOADER_WARPS")) {

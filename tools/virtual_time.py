@@ -28,7 +28,7 @@ for it in range(25):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         edges = 0
-    res = grp.sample([dev[r][it] for r in range(P)], 0x5EED + it)
+    res = grp.sample([dev[r][it % len(dev[r])] for r in range(P)], 0x5EED + it)
     if it >= 5:
         edges += sum(b.num_edges for rr in res for b in rr)
 e1.record()
