@@ -76,7 +76,8 @@ struct WsHeader {
   uint32_t gcursor;      // next gather chunk (pipelined launches)
   uint32_t chunks_loader, chunks_helper;  // gather chunks done by loader / sampling warps
   uint32_t lw_big;       // layer-wise tasks with 32 < c < deg (owner side)
-  uint32_t pad[2];
+  int32_t abort_wait;    // world > 1 persistent call: a wait timed out, later waits end at once
+  uint32_t pad[1];
   unsigned long long t[24];   // %globaltimer at kernel start and when block 0 leaves each grid barrier
   unsigned long long ta[24];  // %globaltimer when block 0 arrives at each grid barrier
   unsigned long long dbg[32]; // debug stamps (DSP_DEBUG_STAMPS builds only)
@@ -964,7 +965,9 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
 }
 
 // A sampling warp that finished its phases takes remaining chunks of the
-// previous call's gather with 16-byte register loads.
+// previous call's gather with 16-byte register loads.  MULTI (world > 1):
+// rows of every rank, read from the owner's shard (local or peer-mapped).
+template <bool MULTI = false>
 __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
   const int lane = threadIdx.x & 31;
   const GatherArgs &g = a.gp;
@@ -995,14 +998,16 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
           id[u] = __ldg(g.ids + r0 + r);
         }
       }
+      const int32_t N = (int32_t)g.bd.b[MULTI ? g.bd.world : 1];
 #pragma unroll
       for (int u = 0; u < 4; ++u)
-        if (id[u] >= 0 && id[u] < (int32_t)g.bd.b[1]) v[u] = ld_f4_hint(feature_row(g, 0, id[u]) + col[u], pol);
+        if (id[u] >= 0 && id[u] < N)
+          v[u] = ld_f4_hint(feature_row(g, MULTI ? owner_of(g.bd, id[u]) : 0, id[u]) + col[u], pol);
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const uint32_t e = e0 + 32u * u;
         if (e < total) {
-          if (id[u] >= 0 && id[u] < (int32_t)g.bd.b[1])
+          if (id[u] >= 0 && id[u] < N)
             st_f4_hint(g.out + r0 * dim4 + e, v[u], pol);
           else
             latch(g.err, E_RANGE);

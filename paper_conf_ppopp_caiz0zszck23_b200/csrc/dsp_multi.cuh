@@ -1,0 +1,412 @@
+// dsp_multi.cuh -- world > 1: the whole CSP call of one rank in ONE persistent
+// cooperative kernel (sm_100a), the exchanges done inside it over NVLink peer
+// memory.
+//
+// Per layer l (Fig. 5), with grid barriers (GB) between phases:
+//   A  shuffle   : group the frontier by owner (contiguous id ranges),
+//                  write each id straight into the owner's inbox (peer store),
+//                  perm[i] = its inbox slot;  [indices of layer l-1 meanwhile]
+//                  -- fence.sys, GB, block 0 publishes counts + header and the
+//                  inbox flag of every owner (count notification)
+//   B  sample    : wait for every rank's inbox flag; sample every received
+//                  task (one phase over all tasks) and write the row
+//                  straight into the requester's return slot (reshuffle)
+//                  -- fence.sys, GB, block 0 releases the return flags
+//   C  unpermute : wait for every owner's return flag; frontier node i takes
+//                  its row from slot perm[i] of its owner, writes the edge
+//                  slots and marks the relabel map (as the local sampler does)
+//                  -- GB
+//   D  scan      : the two-pass relabel scan of the world-1 kernel -- GB
+// then the last layer's indices and the gather (fused, or pipelined: loader
+// warps read the PREVIOUS call's rows from the owners' shards while this
+// call samples -- the paper's loader(t-1) || sampler(t)).
+//
+// Compared with the stage-by-stage path (k_bucket_scatter .. k_write_indices,
+// 5 launches per layer) this removes the per-kernel launch / drain / refill
+// and the system fence of every block of every stage kernel: one launch per
+// call, 148 fences per exchange.  Waiting inside a kernel on a peer's kernel
+// is safe because every rank's kernel is fully resident (cooperative launch on
+// its own GPU; virtual ranks sharing a GPU each get 1/P of the SMs on their
+// own stream), and every wait is bounded (20 s, then E_STATE and an abort
+// word that ends every later wait of the call at once: never a hung GPU).
+//
+// The results are the same as the staged path's (same draws, same slots,
+// same relabel), checked against the oracle in tests/test_gpu_parity.py.
+#pragma once
+#include "dsp_kernels.cuh"
+
+namespace dsp {
+
+struct MultiArgs {
+  PersistArgs p;            // the world-1 persistent kernel's arguments
+  int32_t rank;
+  unsigned long long seq0;  // exchange sequence number before this call (layer l uses seq0 + 1 + l)
+  Bounds bd;
+  XchLayout X;
+  XchPeers peers;
+  int32_t *perm;            // [F] inbox slot of frontier node i at its owner
+  int32_t *abort_word;      // set when a wait timed out: later waits of this call end at once
+};
+
+// Thread 0 of each block waits until flags[s] >= seq for every rank s; the
+// block then proceeds (bar.sync after the acquire).  Bounded: E_STATE + abort.
+template <int TEAM>
+__device__ __forceinline__ void multi_wait(unsigned long long *flags0, int world, unsigned long long seq, int *err,
+                                           int32_t *abort_word) {
+  if (threadIdx.x == 0) {
+    const unsigned long long t0 = globaltimer_ns();
+    for (int s = 0; s < world; ++s) {
+      while (ld_acquire_sys(flags0 + s) < seq) {
+        if (*(volatile int32_t *)abort_word) return;
+        if (globaltimer_ns() - t0 > WAIT_TIMEOUT_NS) {
+          latch(err, E_STATE);
+          *(volatile int32_t *)abort_word = 1;
+          break;
+        }
+        __nanosleep(32);
+      }
+    }
+  }
+}
+
+// A: shuffle.  Each block scatters its contiguous chunk of the frontier,
+// TEAM ids per round (shared-memory owner histogram, one global counter add
+// per owner and round, then the peer stores).
+template <int TEAM>
+__device__ __forceinline__ void multi_scatter(const MultiArgs &m, const int32_t *frontier, int F, int par,
+                                              uint32_t *s_cnt, uint32_t *s_base) {
+  const PersistArgs &a = m.p;
+  const Span sp = block_span<TEAM>(F);
+  const int64_t b0 = sp.first - threadIdx.x;
+  const int world = m.bd.world;
+  const int32_t N = (int32_t)m.bd.b[world];
+  for (int64_t r0 = b0; r0 < sp.end; r0 += TEAM) {
+    if (threadIdx.x < 8) s_cnt[threadIdx.x] = 0;
+    team_sync<TEAM>();
+    const int64_t i = r0 + threadIdx.x;
+    int o = -1;
+    uint32_t local = 0;
+    int32_t v = 0;
+    if (i < sp.end) {
+      v = ldw_i32(frontier + i);
+      if (v < 0 || v >= N) {
+        latch(a.err, E_RANGE);
+      } else {
+        o = owner_of(m.bd, v);
+        local = atomicAdd(&s_cnt[o], 1u);
+      }
+    }
+    team_sync<TEAM>();
+    if (threadIdx.x < world && s_cnt[threadIdx.x])
+      s_base[threadIdx.x] = atomicAdd(&a.hdr->bucket[threadIdx.x], s_cnt[threadIdx.x]);
+    team_sync<TEAM>();
+    if (o >= 0) {
+      const uint32_t j = s_base[o] + local;
+      xch_inbox(m.peers.base[o], m.X, par, m.rank)[j] = v;
+      m.perm[i] = (int32_t)j;
+    }
+  }
+}
+
+// B: the owner's sample of every received task.  Tasks are numbered over the
+// senders (s_off = prefix of the per-sender counts); thread per task for
+// k <= KB (draws, Floyd and ranking in registers, as phase_sample_tpn), the
+// row written to the requester's return slot j (count, then row in slot order).
+template <int KB, int TEAM>
+__device__ __forceinline__ void multi_sample_tpn(const MultiArgs &m, int T, const uint32_t *s_off, int layer, int k,
+                                                 int par) {
+  const PersistArgs &a = m.p;
+  const int world = m.bd.world;
+  char *self = m.peers.base[m.rank];
+  const int64_t kmax = m.X.kmax;
+  const Span sp = block_span<TEAM>(T);
+  for (int64_t qq = sp.first; qq < sp.end; qq += sp.step) {
+    const int q = (int)qq;
+    int s = 0;
+    while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
+    const int j = q - (int)s_off[s];
+    const int32_t v = __ldcv(xch_inbox(self, m.X, par, s) + j);
+    const int64_t lv = (int64_t)v - a.lo;
+    char *req = m.peers.base[s];
+    if (lv < 0 || lv >= a.n_local) {  // routed to the wrong owner: protocol error
+      latch(a.err, E_STATE);
+      xch_ret_cnt(req, m.X, par, m.rank)[j] = 0;
+      continue;
+    }
+    int64_t rs, d;
+    row_extent(a.indptr, lv, &rs, &d);
+    const bool full = d <= k;
+    const int cnt = full ? (int)d : k;
+    uint32_t pos[KB];
+#pragma unroll
+    for (int t = 0; t < KB; ++t) pos[t] = (uint32_t)t;
+    if (!full) {
+#pragma unroll
+      for (int t = 0; t < KB; ++t)
+        if (t < k) pos[t] = draw_range(a.key, (uint32_t)t, v, layer, (uint32_t)(d - k + t + 1));
+#pragma unroll
+      for (int t = 1; t < KB; ++t) {
+        if (t < k) {
+          bool hit = false;
+#pragma unroll
+          for (int qx = 0; qx < t; ++qx) hit |= (pos[qx] == pos[t]);
+          if (hit) pos[t] = (uint32_t)(d - k + t);
+        }
+      }
+    }
+    int32_t u[KB];
+    unsigned long long slots = 0;
+#pragma unroll
+    for (int t = 0; t < KB; ++t) {
+      uint32_t r = 0;
+#pragma unroll
+      for (int qx = 0; qx < KB; ++qx) r += (qx < cnt && pos[qx] < pos[t]) ? 1u : 0u;
+      slots |= (unsigned long long)r << (4 * t);
+      u[t] = (t < cnt) ? adj_ld(a.indices + rs + pos[t]) : 0;
+    }
+    xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
+    int32_t *row = xch_ret_rows(req, m.X, par, m.rank) + (int64_t)j * kmax;
+#pragma unroll
+    for (int t = 0; t < KB; ++t)
+      if (t < cnt) row[(slots >> (4 * t)) & 15u] = u[t];
+  }
+}
+
+// B for k > 16 (lane groups of 32) and biased sampling (warp per task).
+template <int TEAM>
+__device__ __forceinline__ void multi_sample_warp(const MultiArgs &m, int T, const uint32_t *s_off, int layer, int k,
+                                                  int par) {
+  const PersistArgs &a = m.p;
+  const int world = m.bd.world;
+  char *self = m.peers.base[m.rank];
+  const int lane = threadIdx.x & 31;
+  const Span sp = block_span<TEAM>(T);
+  const int64_t b0 = sp.first - threadIdx.x;
+  const int wib = threadIdx.x >> 5, wpb = TEAM >> 5;
+  for (int64_t q64 = b0 + wib; q64 < sp.end; q64 += wpb) {
+    const int q = (int)q64;
+    int s = 0;
+    while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
+    const int j = q - (int)s_off[s];
+    const int32_t v = __ldcv(xch_inbox(self, m.X, par, s) + j);
+    const int64_t lv = (int64_t)v - a.lo;
+    const bool ok = lv >= 0 && lv < a.n_local;
+    if (!ok && lane == 0) latch(a.err, E_STATE);
+    int64_t rs = 0, d = 0;
+    if (ok) row_extent(a.indptr, lv, &rs, &d);
+    bool valid;
+    int slot, cnt;
+    int32_t u;
+    if (a.biased) {
+      uint32_t pos;
+      cnt = sample_node_biased(ok, v, rs, d, k, layer, a.key, a.weights, &pos);
+      slot = lane;
+      valid = lane < cnt;
+      u = valid ? __ldg(a.indices + rs + pos) : -1;
+    } else {
+      sample_node<32>(ok, v, rs, d, k, layer, a.key, a.indices, &valid, &slot, &u, &cnt);
+    }
+    char *req = m.peers.base[s];
+    if (lane == 0) xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
+    if (valid) xch_ret_rows(req, m.X, par, m.rank)[(int64_t)j * m.X.kmax + slot] = u;
+  }
+}
+
+// C: frontier node i (thread per node) reads its row from its owner's return
+// slot perm[i]: counts, edge slots, dst copy and relabel marks.
+template <int TEAM>
+__device__ __forceinline__ void multi_unpermute(const MultiArgs &m, const int32_t *frontier, int F, int layer, int k,
+                                                int par, uint32_t epoch) {
+  const PersistArgs &a = m.p;
+  const LayerBufs &B = a.buf[layer & 1];
+  int32_t *src_out = a.out.src_ids[layer];
+  const int32_t N = (int32_t)m.bd.b[m.bd.world];
+  const Span sp = block_span<TEAM>(F);
+  for (int64_t ii = sp.first; ii < sp.end; ii += sp.step) {
+    const int i = (int)ii;
+    const int32_t v = ldw_i32(frontier + i);
+    src_out[i] = v;  // dst copy (R17)
+    if (v < 0 || v >= N) {  // latched by the shuffle
+      B.cnt[i] = 0;
+      continue;
+    }
+    const int o = owner_of(m.bd, v);
+    const int j = ldw_i32(m.perm + i);
+    const int c = __ldcv(xch_ret_cnt(m.peers.base[m.rank], m.X, par, o) + j);
+    const int32_t *row = xch_ret_rows(m.peers.base[m.rank], m.X, par, o) + (int64_t)j * m.X.kmax;
+    B.cnt[i] = c;
+    mark_dst(B, v, i, F, layer, epoch, a.err);
+    const uint32_t q0 = (uint32_t)i * (uint32_t)k;
+    if (k <= 16) {
+      int32_t u[16];
+#pragma unroll
+      for (int t = 0; t < 16; ++t) u[t] = t < c ? __ldcv(row + t) : 0;
+#pragma unroll
+      for (int t = 0; t < 16; ++t)
+        if (t < c) {
+          B.rows[q0 + t] = u[t];
+          mark(B, u[t], epoch, (uint32_t)F + q0 + (uint32_t)t);
+        }
+    } else {
+      for (int t = 0; t < c; ++t) {
+        const int32_t u = __ldcv(row + t);
+        B.rows[q0 + t] = u;
+        mark(B, u, epoch, (uint32_t)F + q0 + (uint32_t)t);
+      }
+    }
+  }
+}
+
+template <int TEAM, bool PIPE>
+__global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
+  __shared__ Scan2Smem<TEAM> sm;
+  __shared__ uint32_t s_cnt[8], s_base[8], s_off[9];
+  const PersistArgs &a = m.p;
+  const int blk = blockIdx.x, nblk = gridDim.x;
+  const int world = m.bd.world;
+
+  if (PIPE && threadIdx.x >= TEAM) {  // ------ loader warps: previous call's rows, any owner
+    if (a.prev) helper_warp<true>(a, ld_volatile_i32(a.gp.n_dev));
+    return;
+  }
+
+  const int64_t tid = blockIdx.x * (int64_t)TEAM + threadIdx.x;
+  const int64_t nthreads = (int64_t)gridDim.x * TEAM;
+  uint32_t bar = 0;
+  const uint32_t e0 = *(volatile const uint32_t *)&a.persist->epoch;
+  const bool hclear = hash_clear_due(a.persist, e0, (uint32_t)a.L, a.buf[0].mask, a.buf[0].first);
+  if (hclear) {  // zero both parities of the relabel hash table (once per ~255 / L calls)
+    for (int64_t i = tid; i <= (int64_t)a.buf[0].mask; i += nthreads) {
+      a.buf[0].first[i] = 0ull;
+      a.buf[1].first[i] = 0ull;
+    }
+    grid_barrier<TEAM>(a.hdr, bar);
+  }
+  if (tid == 0) {
+    a.hdr->t[0] = globaltimer_ns();
+    a.hdr->F[0] = a.B;
+  }
+  char *self = m.peers.base[m.rank];
+  int F = a.B;
+  int Fprev = 0;
+  for (int l = 0; l < a.L; ++l) {
+    const uint32_t epoch = e0 + 1 + l;
+    const unsigned long long seq = m.seq0 + 1 + (unsigned long long)l;
+    const int par = (int)(seq & 1ull);
+    const int32_t *frontier = l == 0 ? a.seeds : a.out.src_ids[l - 1];
+    const int k = a.k[l];
+    const int Fs = F > m.X.cap ? 0 : F;  // capacity overflow: send nothing (latched below)
+    if (F > m.X.cap && tid == 0) latch(a.err, E_CAP);
+
+    // ---- A: shuffle (+ the previous layer's duplicate indices)
+    multi_scatter<TEAM>(m, frontier, Fs, par, s_cnt, s_base);
+    if (l > 0)
+      phase_indices_dups(Fprev, a.k[l - 1], a.buf[(l - 1) & 1], a.out.indptr[l - 1], a.out.indices[l - 1],
+                         block_span<TEAM>((int64_t)Fprev * a.k[l - 1]));
+    __threadfence_system();  // this block's peer stores, before the barrier that precedes the flag
+    grid_barrier<TEAM>(a.hdr, bar);
+    if (blk == 0 && threadIdx.x == 0) {
+      for (int o = 0; o < world; ++o) {
+        const uint32_t c = *(volatile uint32_t *)&a.hdr->bucket[o];
+        a.hdr->bucket[o] = 0u;
+        *xch_inbox_hdr(m.peers.base[o], m.X, par, m.rank) =
+            make_uint4(c, (uint32_t)k | ((uint32_t)l << 8) | ((uint32_t)a.biased << 16), a.key.x, a.key.y);
+      }
+      __threadfence_system();
+      for (int o = 0; o < world; ++o) st_release_sys(xch_inbox_flag(m.peers.base[o], m.X, par, m.rank), seq);
+    }
+
+    // ---- B: sample every task received from any rank
+    multi_wait<TEAM>(xch_inbox_flag(self, m.X, par, 0), world, seq, a.err, m.abort_word);
+    if (threadIdx.x == 0) {
+      uint32_t acc = 0;
+      for (int s = 0; s < world; ++s) {
+        const uint4 h = __ldcv(xch_inbox_hdr(self, m.X, par, s));
+        if (h.y != ((uint32_t)k | ((uint32_t)l << 8) | ((uint32_t)a.biased << 16)) || h.z != a.key.x ||
+            h.w != a.key.y)
+          latch(a.err, E_STATE);  // ranks disagree on (layer, fan-out, seed, scheme)
+        s_off[s] = acc;
+        acc += (h.x <= (uint32_t)m.X.cap) ? h.x : 0u;
+      }
+      s_off[world] = *(volatile int32_t *)m.abort_word ? 0u : acc;
+    }
+    team_sync<TEAM>();
+    const int T = (int)s_off[world];
+    if (a.biased || k > 16)
+      multi_sample_warp<TEAM>(m, T, s_off, l, k, par);
+    else if (k <= 8)
+      multi_sample_tpn<8, TEAM>(m, T, s_off, l, k, par);
+    else
+      multi_sample_tpn<16, TEAM>(m, T, s_off, l, k, par);
+    __threadfence_system();
+    grid_barrier<TEAM>(a.hdr, bar);
+    if (blk == 0 && threadIdx.x == 0) {
+      __threadfence_system();
+      for (int s = 0; s < world; ++s) st_release_sys(xch_ret_flag(m.peers.base[s], m.X, par, m.rank), seq);
+    }
+
+    // ---- C: rows back in frontier order, relabel marks
+    multi_wait<TEAM>(xch_ret_flag(self, m.X, par, 0), world, seq, a.err, m.abort_word);
+    team_sync<TEAM>();
+    multi_unpermute<TEAM>(m, frontier, Fs, l, k, par, epoch);
+    grid_barrier<TEAM>(a.hdr, bar);
+
+    // ---- D: relabel scan (as k_csp_persistent)
+    constexpr int64_t TILE = (int64_t)TEAM * SCAN2_IPT;
+    const int64_t total = (int64_t)Fs * k;
+    const int64_t rounds = total > 0 ? (total + (int64_t)nblk * TILE - 1) / ((int64_t)nblk * TILE) : 1;
+    const int64_t per_round = (total + rounds - 1) / rounds;
+    const int64_t chunk = (per_round + nblk - 1) / nblk;
+    unsigned long long carry = 0;
+    for (int64_t r = 0; r < rounds; ++r) {
+      Scan2Regs R;
+      const int64_t r0 = r * per_round, r1 = min(total, r0 + per_round);
+      const int64_t tile0 = min(r1, r0 + (int64_t)blk * chunk), tile_end = min(r1, tile0 + chunk);
+      unsigned long long *agg = a.agg + (r & 1) * MAX_PERSIST_BLOCKS;
+      scan2_pass1<TEAM>(Fs, k, a.buf[l & 1], epoch, tile0, tile_end, R, agg + blk, sm);
+      grid_barrier<TEAM>(a.hdr, bar);
+      unsigned long long prefix, round_total;
+      scan2_prefix<TEAM>(agg, nblk, blk, sm, &prefix, &round_total);
+      scan2_pass2<TEAM>(Fs, k, a.buf[l & 1], tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
+                        a.out.indices[l], a.out.src_ids[l]);
+      carry += round_total;
+      if (r + 1 < rounds) grid_barrier<TEAM>(a.hdr, bar);
+    }
+    const int32_t E = (int32_t)(carry & 0x7fffffffull);
+    const int32_t nnew = (int32_t)((carry >> 31) & 0x7fffffffull);
+    if (tid == 0) {
+      a.out.indptr[l][Fs] = E;
+      a.hdr->E[l] = E;
+      a.hdr->S[l] = Fs + nnew;
+      a.hdr->F[l] = Fs;
+      a.hdr->F[l + 1] = Fs + nnew;
+      a.hdr->sizes[3 * l + 0] = Fs;
+      a.hdr->sizes[3 * l + 1] = Fs + nnew;
+      a.hdr->sizes[3 * l + 2] = E;
+    }
+    Fprev = Fs;
+    F = Fs + nnew;
+    grid_barrier<TEAM>(a.hdr, bar);
+  }
+  const int l = a.L - 1;
+  phase_indices_dups(Fprev, a.k[l], a.buf[l & 1], a.out.indptr[l], a.out.indices[l],
+                     block_span<TEAM>((int64_t)Fprev * a.k[l]));
+  if (PIPE) {
+    if (tid == 0) *a.pend_n = F;
+    if (a.prev) helper_warp<true>(a, ld_volatile_i32(a.gp.n_dev));
+  } else if (a.gather) {
+    phase_gather<GATHER_UNROLL>(a.g, F, tid, nthreads);
+  }
+  team_sync<TEAM>();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(&a.hdr->done, 1u) == gridDim.x - 1) {
+      a.persist->epoch = e0 + (uint32_t)a.L;
+      if (hclear) hash_cleared(a.persist, e0, a.buf[0].mask, a.buf[0].first);
+      a.hdr->t[23] = globaltimer_ns();
+      a.hdr->done = 0u;
+    }
+  }
+}
+
+}  // namespace dsp

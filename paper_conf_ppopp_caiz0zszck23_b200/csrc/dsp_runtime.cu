@@ -17,6 +17,7 @@
 
 #include "../../include/dsp.h"
 #include "dsp_layerwise.cuh"
+#include "dsp_multi.cuh"
 #include "dsp_walk.cuh"
 
 using namespace dsp;
@@ -177,6 +178,9 @@ struct dsp_ctx {
   int loader_warps = 4; // DSP_LOADER_WARPS = 2, 4 or 8 (tuning knob, results unchanged)
   int loader_rows = 32;  // DSP_LOADER_ROWS: rows per TMA chunk, <= 32 (tuning knob, results unchanged)
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
+  bool multi_staged = false;  // DSP_MULTI_STAGED=1: world > 1 node-wise calls stage by stage (A/B switch)
+  cudaStream_t aux = nullptr;  // virtual ranks sharing a GPU: each rank's persistent launch on its own stream
+  cudaEvent_t aux_ev[2] = {nullptr, nullptr};
   int gather_blocks_per_sm = 1;
   // pipelined steps: per workspace, the gather owed by its previous
   // DSP_PIPELINED call (row count in the workspace's WsPersist::pend_n[parity])
@@ -677,6 +681,95 @@ dsp_status stage_persistent(Call &k) {
   return DSP_OK;
 }
 
+XchPeers peers_of(const dsp_ctx *c);
+
+// world > 1, node-wise: the whole call in one cooperative kernel per rank
+// (dsp_multi.cuh).  `share` = ranks of this call group on the same GPU
+// (virtual ranks): each launch gets 1/share of the SMs, on the ctx's own
+// stream forked from / joined to the caller's, so all of them are resident.
+dsp_status stage_persistent_multi(Call &k, int share) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  MultiArgs m{};
+  PersistArgs &a = m.p;
+  a.seeds = k.seeds;
+  a.B = k.num_seeds;
+  a.L = k.L;
+  for (int l = 0; l < k.L; ++l) {
+    a.k[l] = k.fanouts[l];
+    a.out.indptr[l] = k.blocks[l].indptr;
+    a.out.indices[l] = k.blocks[l].indices;
+    a.out.src_ids[l] = k.blocks[l].src_ids;
+  }
+  a.agg = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_agg);
+  a.persist = persist_of(k);
+  a.key = key_of(k.rng_seed);
+  a.indptr = c->d_indptr;
+  a.indices = c->d_indices;
+  a.weights = c->d_weights;
+  a.biased = k.biased ? 1 : 0;
+  a.lo = c->lo;
+  a.n_local = c->n_local;
+  a.buf[0] = bufs_of(k, 0);
+  a.buf[1] = bufs_of(k, 1);
+  a.hdr = k.hdr;
+  a.err = c->d_err;
+  a.lane_rounds = c->lane_rounds;
+  a.gather = k.feat_out != nullptr && !k.pipelined;
+  if (a.gather) a.g = make_gather(c, k.blocks[k.L - 1].src_ids, 0, nullptr, k.feat_out);
+  m.rank = c->rank;
+  m.seq0 = k.seq0;
+  m.bd = make_bounds(c);
+  m.X = c->xl;
+  m.peers = peers_of(c);
+  m.perm = reinterpret_cast<int32_t *>(k.ws + k.plan.off_perm);
+  m.abort_word = &k.hdr->abort_wait;
+  int blocks = c->persist_blocks > 0 ? c->persist_blocks : c->num_sms * c->persist_blocks_per_sm;
+  if (share > 1) blocks = std::max(1, std::min(blocks, c->num_sms * c->persist_blocks_per_sm / share));
+  const dim3 grid(blocks), block(PNT);
+  cudaStream_t st = k.stream;
+  if (share > 1) {  // fork onto the ctx's own stream
+    if (!c->aux) {
+      CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking));
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[0], cudaEventDisableTiming));
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[1], cudaEventDisableTiming));
+    }
+    CUDA_TRY(c, cudaEventRecord(c->aux_ev[0], k.stream));
+    CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->aux_ev[0], 0));
+    st = c->aux;
+  }
+  void *args[] = {&m};
+  if (!k.pipelined) {
+    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_multi<PNT, false>, grid, block, args, 0, st));
+  } else {
+    dsp_ctx::Pending *pd = c->pending_of(k.ws);
+    if (!pd) return fail(c, DSP_ERR_STATE, "more than 8 workspaces with pending pipelined gathers");
+    WsPersist *ps = persist_of(k);
+    a.prev = pd->active ? 1 : 0;
+    if (a.prev) a.gp = make_gather(c, pd->ids, 0, &ps->pend_n[(pd->calls + 1) & 1], pd->out);
+    a.pend_n = &ps->pend_n[pd->calls & 1];
+    a.rows_per_chunk = 32;
+    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_multi<PIPE_TEAM, true>, grid, block, args, 0, st));
+    pd->ids = k.blocks[k.L - 1].src_ids;
+    pd->out = k.feat_out;
+    pd->stream = k.stream;
+    pd->active = true;
+    pd->calls += 1;
+  }
+  return DSP_OK;
+}
+
+// the caller's stream waits for the rank's own stream (after ALL ranks of the
+// group were launched: joining earlier would serialise the virtual ranks)
+dsp_status join_persistent_multi(Call &k, int share) {
+  dsp_ctx *c = k.c;
+  if (share <= 1) return DSP_OK;
+  DeviceGuard g(c->device);
+  CUDA_TRY(c, cudaEventRecord(c->aux_ev[1], c->aux));
+  CUDA_TRY(c, cudaStreamWaitEvent(k.stream, c->aux_ev[1], 0));
+  return DSP_OK;
+}
+
 // gather owed by a workspace's last pipelined call (k_gather with the device row count)
 dsp_status flush_one(dsp_ctx *c, dsp_ctx::Pending &pd) {
   if (!pd.active) return DSP_OK;
@@ -959,11 +1052,21 @@ dsp_status run_calls(std::vector<Call> &calls) {
     if ((st = (STAGE)) != DSP_OK) return st;
   // a non-pipelined call first settles a pending pipelined gather; so does a
   // pipelined call of the stage-by-stage paths (no loader warps there)
+  const bool multi = calls[0].c->world > 1 && !calls[0].layerwise && !calls[0].c->multi_staged;
   for (auto &k : calls)
-    if ((!k.pipelined || k.c->world > 1 || k.layerwise) && (st = stage_flush(k.c, k.ws)) != DSP_OK) return st;
+    if ((!k.pipelined || (k.c->world > 1 && !multi) || k.layerwise) && (st = stage_flush(k.c, k.ws)) != DSP_OK)
+      return st;
   EACH(stage_begin(k));
   if (calls[0].c->world == 1 && !calls[0].layerwise) {
     EACH(stage_persistent(k));
+  } else if (multi) {
+    std::vector<int> share(calls.size(), 0);
+    for (size_t i = 0; i < calls.size(); ++i)
+      for (auto &o : calls) share[i] += o.c->device == calls[i].c->device ? 1 : 0;
+    for (size_t i = 0; i < calls.size(); ++i)
+      if ((st = stage_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
+    for (size_t i = 0; i < calls.size(); ++i)
+      if ((st = join_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
   } else {
     for (int l = 0; l < calls[0].L; ++l) {
       if (calls[0].layerwise) {
@@ -1045,6 +1148,13 @@ void release(dsp_ctx *c) {
   cudaFree(c->d_weights);
   cudaFree(c->d_feat);
   cudaFree(c->d_xch);
+  if (c->aux) {
+    cudaStreamSynchronize(c->aux);
+    cudaStreamDestroy(c->aux);
+    cudaEventDestroy(c->aux_ev[0]);
+    cudaEventDestroy(c->aux_ev[1]);
+    c->aux = nullptr;
+  }
   cudaFree(c->d_lxch);
   cudaFree(c->d_wxch);
   cudaFree(c->d_err);
@@ -1226,6 +1336,7 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   c->persist_blocks_per_sm = std::min(occ, occ_pipe);
   if (getenv("DSP_LANE_ROUNDS")) c->lane_rounds = atoi(getenv("DSP_LANE_ROUNDS"));
   if (getenv("DSP_STAGE_BPS")) c->stage_bps = std::max(1, std::min(8, atoi(getenv("DSP_STAGE_BPS"))));
+  c->multi_staged = getenv("DSP_MULTI_STAGED") && atoi(getenv("DSP_MULTI_STAGED")) != 0;
   if (const char *rm = getenv("DSP_RELABEL")) c->relabel_mode = !strcmp(rm, "hash") ? 2 : !strcmp(rm, "direct") ? 1 : 0;
   if (getenv("DSP_LOADER_ROWS")) c->loader_rows = std::max(1, std::min(32, atoi(getenv("DSP_LOADER_ROWS"))));
   if (getenv("DSP_LOADER_WARPS")) {

@@ -25,6 +25,21 @@ def _free_port():
     return p
 
 
+def _check_pipelined(s, ip, ix, cfg, seeds, rng, slot, sizes):
+    import datagen
+    import oracle
+    ref = oracle.sample(ip, ix, seeds, cfg.fanouts, rng)
+    blocks = s.blocks(slot, sizes.numpy())
+    for b, r in zip(blocks, ref):
+        for key in ("indptr", "indices", "src_ids"):
+            if not np.array_equal(getattr(b, key).cpu().numpy(), r[key]):
+                raise AssertionError(f"pipelined step rng {rng:#x}: {key}")
+    feat = s.feat_buffer(slot)[: blocks[-1].num_src]
+    exp = datagen.features_of(ref[-1]["src_ids"], cfg.dim)
+    if not np.array_equal(feat.cpu().numpy().view(np.uint32), exp.view(np.uint32)):
+        raise AssertionError(f"pipelined step rng {rng:#x}: features")
+
+
 def _rank(rank, world, port, q, hot=None, scheme="node"):
     import sys
     here = os.path.dirname(os.path.abspath(__file__))
@@ -63,6 +78,20 @@ def _rank(rank, world, port, q, hot=None, scheme="node"):
             exp = datagen.features_of(ref[-1]["src_ids"], cfg.dim)
             if not np.array_equal(feat.cpu().numpy().view(np.uint32), exp.view(np.uint32)):
                 ok, detail = False, f"step {step} features"
+        if scheme == "node":
+            # pipelined steps: the launch of step t samples batch t while its
+            # loader warps gather batch t-1 from both processes' shards; flush() the last
+            sz = torch.zeros((4, 3 * len(cfg.fanouts)), dtype=torch.int64).pin_memory()
+            for step in range(4):
+                s.sample_gather(torch.from_numpy(batches[step]).cuda(), 0xABC + step, slot=step % 2,
+                                sizes_out=sz[step], pipelined=True)
+                if step >= 1:  # step-1's features were written by this launch
+                    torch.cuda.synchronize()
+                    _check_pipelined(s, ip, ix, cfg, batches[step - 1], 0xABC + step - 1, (step - 1) % 2,
+                                     sz[step - 1])
+            s.flush()
+            torch.cuda.synchronize()
+            _check_pipelined(s, ip, ix, cfg, batches[3], 0xABC + 3, 1, sz[3])
         # random walks over the partitioned graph: walkers cross processes
         starts = np.random.default_rng(rank).integers(0, cfg.num_nodes, size=400 + 50 * rank).astype(np.int32)
         tr = s.random_walk(torch.from_numpy(starts).cuda(), 16, 0xC0DE)

@@ -173,8 +173,13 @@ def test_fig5_csp_example_virtual_two_gpus(pkg):
 
 # ------------------------------------------------------- virtual P = 2,4,8
 
+@pytest.mark.parametrize("mode", ["persistent", "staged"])
 @pytest.mark.parametrize("P", [2, 4, 8])
-def test_tiny_virtual_ranks(pkg, tiny, P):
+def test_tiny_virtual_ranks(pkg, tiny, P, mode, monkeypatch):
+    """world > 1: one persistent kernel per rank (default; virtual ranks each on
+    1/P of the SMs, own stream) or the stage-by-stage kernels (DSP_MULTI_STAGED)."""
+    if mode == "staged":
+        monkeypatch.setenv("DSP_MULTI_STAGED", "1")
     cfg, ip, ix, feats = tiny
     bnds = datagen.bounds(cfg.num_nodes, P)
     shards = []
