@@ -20,9 +20,11 @@
 //
 // world == 1 runs the whole call in ONE persistent cooperative kernel
 // (k_csp_persistent, one 1024-thread block per SM) with grid barriers between
-// phases; world > 1 issues one kernel per phase so that ranks sharing a GPU
-// can be interleaved stage by stage and exchanges never wait inside a kernel
-// on work queued behind it.
+// phases; world > 1 runs it in one persistent kernel per rank as well
+// (k_csp_multi, dsp_multi.cuh), the exchanges done inside it through peer
+// memory.  The stage-by-stage kernels below (k_bucket_scatter ..
+// k_write_indices, one launch per phase) remain as the DSP_MULTI_STAGED=1
+// A/B switch (tested against the oracle like the default path).
 //
 // Data a phase reads after another phase of the same kernel wrote it is read
 // with plain (weak) loads after the grid barrier's release/acquire, never

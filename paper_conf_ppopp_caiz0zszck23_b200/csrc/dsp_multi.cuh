@@ -37,6 +37,12 @@
 
 namespace dsp {
 
+#ifdef DSP_EXPERIMENT_GPU_FENCE  // cost measurement on virtual ranks only (not valid across GPUs)
+#define MULTI_BLOCK_FENCE() __threadfence()
+#else
+#define MULTI_BLOCK_FENCE() __threadfence_system()
+#endif
+
 struct MultiArgs {
   PersistArgs p;            // the world-1 persistent kernel's arguments
   int32_t rank;
@@ -172,42 +178,48 @@ __device__ __forceinline__ void multi_sample_tpn(const MultiArgs &m, int T, cons
   }
 }
 
-// B for k > 16 (lane groups of 32) and biased sampling (warp per task).
-template <int TEAM>
-__device__ __forceinline__ void multi_sample_warp(const MultiArgs &m, int T, const uint32_t *s_off, int layer, int k,
-                                                  int par) {
+// B with a lane group of G lanes per task (G = next pow2 >= k): k > 16, and
+// small task counts (the first layers), where a thread per task would run its
+// k Philox draws back to back with few warps busy.  Biased: warp per task.
+template <int G, int TEAM>
+__device__ __forceinline__ void multi_sample_lanes(const MultiArgs &m, int T, const uint32_t *s_off, int layer, int k,
+                                                   int par) {
   const PersistArgs &a = m.p;
   const int world = m.bd.world;
   char *self = m.peers.base[m.rank];
+  constexpr int NPW = 32 / G;
   const int lane = threadIdx.x & 31;
+  const bool leader = (lane & (G - 1)) == 0;
   const Span sp = block_span<TEAM>(T);
   const int64_t b0 = sp.first - threadIdx.x;
   const int wib = threadIdx.x >> 5, wpb = TEAM >> 5;
-  for (int64_t q64 = b0 + wib; q64 < sp.end; q64 += wpb) {
-    const int q = (int)q64;
+  for (int64_t base = b0 + (int64_t)wib * NPW; base < sp.end; base += (int64_t)wpb * NPW) {
+    const int q = (int)(base + lane / G);
+    const bool active = q < sp.end;
     int s = 0;
-    while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
+    if (active)
+      while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
     const int j = q - (int)s_off[s];
-    const int32_t v = __ldcv(xch_inbox(self, m.X, par, s) + j);
+    const int32_t v = active ? __ldcv(xch_inbox(self, m.X, par, s) + j) : 0;
     const int64_t lv = (int64_t)v - a.lo;
-    const bool ok = lv >= 0 && lv < a.n_local;
-    if (!ok && lane == 0) latch(a.err, E_STATE);
+    const bool ok = active && lv >= 0 && lv < a.n_local;
+    if (active && !ok && leader) latch(a.err, E_STATE);
     int64_t rs = 0, d = 0;
     if (ok) row_extent(a.indptr, lv, &rs, &d);
     bool valid;
     int slot, cnt;
     int32_t u;
-    if (a.biased) {
+    if (G == 32 && a.biased) {
       uint32_t pos;
       cnt = sample_node_biased(ok, v, rs, d, k, layer, a.key, a.weights, &pos);
       slot = lane;
       valid = lane < cnt;
       u = valid ? __ldg(a.indices + rs + pos) : -1;
     } else {
-      sample_node<32>(ok, v, rs, d, k, layer, a.key, a.indices, &valid, &slot, &u, &cnt);
+      sample_node<G>(ok, v, rs, d, k, layer, a.key, a.indices, &valid, &slot, &u, &cnt);
     }
     char *req = m.peers.base[s];
-    if (lane == 0) xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
+    if (active && leader) xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
     if (valid) xch_ret_rows(req, m.X, par, m.rank)[(int64_t)j * m.X.kmax + slot] = u;
   }
 }
@@ -303,7 +315,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
     if (l > 0)
       phase_indices_dups(Fprev, a.k[l - 1], a.buf[(l - 1) & 1], a.out.indptr[l - 1], a.out.indices[l - 1],
                          block_span<TEAM>((int64_t)Fprev * a.k[l - 1]));
-    __threadfence_system();  // this block's peer stores, before the barrier that precedes the flag
+    MULTI_BLOCK_FENCE();  // this block's peer stores, before the barrier that precedes the flag
     grid_barrier<TEAM>(a.hdr, bar);
     if (blk == 0 && threadIdx.x == 0) {
       for (int o = 0; o < world; ++o) {
@@ -332,13 +344,17 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
     }
     team_sync<TEAM>();
     const int T = (int)s_off[world];
+    const int G = k <= 4 ? 4 : k <= 8 ? 8 : 16;
     if (a.biased || k > 16)
-      multi_sample_warp<TEAM>(m, T, s_off, l, k, par);
+      multi_sample_lanes<32, TEAM>(m, T, s_off, l, k, par);
+    else if ((int64_t)T * G <= (int64_t)a.lane_rounds * nblk * TEAM)  // few tasks: lane groups
+      (G == 4 ? multi_sample_lanes<4, TEAM> : G == 8 ? multi_sample_lanes<8, TEAM> : multi_sample_lanes<16, TEAM>)(
+          m, T, s_off, l, k, par);
     else if (k <= 8)
       multi_sample_tpn<8, TEAM>(m, T, s_off, l, k, par);
     else
       multi_sample_tpn<16, TEAM>(m, T, s_off, l, k, par);
-    __threadfence_system();
+    MULTI_BLOCK_FENCE();
     grid_barrier<TEAM>(a.hdr, bar);
     if (blk == 0 && threadIdx.x == 0) {
       __threadfence_system();
