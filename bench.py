@@ -115,6 +115,21 @@ def measured_peaks():
     return 6650.0, "fallback"
 
 
+def measure_h2d_gbps(nbytes: int = 256 << 20) -> float:
+    """Host-link bandwidth: pinned host -> device copy (best of 5)."""
+    h = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    d = torch.empty(nbytes, dtype=torch.uint8, device="cuda")
+    best = 1e30
+    for _ in range(5):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record()
+        d.copy_(h, non_blocking=True)
+        b.record()
+        torch.cuda.synchronize()
+        best = min(best, a.elapsed_time(b))
+    return nbytes / (best * 1e-3) / 1e9
+
+
 def ncu_traffic(kernel: str):
     """DRAM bytes per launch of `kernel` from the committed ncu --set full summary."""
     p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -360,6 +375,34 @@ def run_dsp(args):
     # algorithmic bytes of all timed launches over the elapsed device time
     achieved = (samp_b + gath_b) / (t_ms * 1e-3) / 1e9
 
+    # ---- bytes the scheme adds to the uniform path's algorithmic bytes, from a few
+    # untimed synchronous calls on the same batches (host-side counting only)
+    weight_b = cold_b = None
+    if biased or args.hot_frac is not None:
+        deg = np.diff(ip)   # global in-degrees (every rank holds the whole synthetic graph here)
+        if args.hot_frac is not None:   # each owner's hot set: largest in-degree, ties by smaller id (R31)
+            hot = np.zeros(len(deg), dtype=bool)
+            for r in range(world):
+                lo_r, hi_r = int(bnds[r]), int(bnds[r + 1])
+                nh = int(round(args.hot_frac * (hi_r - lo_r)))
+                dr = deg[lo_r:hi_r]
+                hot[lo_r + np.lexsort((np.arange(len(dr)), -dr))[:nh]] = True
+        wb, cb = [], []
+        for j in range(min(KS, 5)):
+            blocks = s.sample(dev_batches[(W + j) % len(batches)], datagen.BASE_SEED + W + j, biased=biased)
+            if biased:  # every weight of a row with deg > k is read (successive sampling, R25/R26)
+                tot = 0
+                for l, b in enumerate(blocks):
+                    d = deg[b.src_ids[: b.num_dst].cpu().numpy().astype(np.int64)]
+                    tot += int(d[d > fanouts[l]].sum())
+                wb.append(4.0 * tot)
+            if args.hot_frac is not None:
+                ids = blocks[-1].src_ids.cpu().numpy().astype(np.int64)
+                cb.append(float((~hot[ids]).sum()) * cfg.dim * 4)
+        s.sync()
+        weight_b = float(np.mean(wb)) if wb else None
+        cold_b = float(np.mean(cb)) if cb else None
+
     # ---- breakdown (not the headline): the two calls separately
     ids_dev = None
     bd = {}
@@ -471,6 +514,29 @@ def run_dsp(args):
 
     kern_per_step = 5 * L + 1 if layer else 1
     roof_kernel = "k_gather" if layer else ("k_csp_persistent" if world == 1 else "k_csp_multi")
+    roofline = {"kernel": roof_kernel,
+                "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak,
+                "traffic": (ncu_traffic(roof_kernel) if roof_kernel == "k_csp_persistent" and args.scheme == "uniform"
+                            and args.hot_frac is None and args.config == "products" else None),
+                "peak_kind": peak_kind,
+                "algorithmic_bytes_per_launch": (samp_b + gath_b) / KS,
+                "sampling_bytes_per_launch": samp_b / KS, "gather_bytes_per_launch": gath_b / KS,
+                "launch_ms_mean": step_mean, "concurrent_launches": K,
+                "achieved_def": "algorithmic bytes of all timed launches / elapsed device time"}
+    if weight_b is not None:   # biased: the edge weights of every row sampled with draws are read too
+        a_w = (samp_b + gath_b + weight_b * KS) / (t_ms * 1e-3) / 1e9
+        roofline.update({"achieved": a_w, "frac": a_w / peak, "weight_bytes_per_launch": weight_b,
+                         "algorithmic_bytes_per_launch": (samp_b + gath_b) / KS + weight_b})
+    if cold_b is not None:     # cold tier: the dominant stream is the cold rows over the host link
+        link = measure_h2d_gbps()
+        a_c = cold_b * KS / (t_ms * 1e-3) / 1e9
+        roofline = {"kernel": roof_kernel, "bound": "host-link", "achieved": a_c, "peak": link, "unit": "GB/s",
+                    "frac": a_c / link, "traffic": None,
+                    "peak_kind": "measured here: pinned host -> device cudaMemcpy of 256 MB",
+                    "cold_bytes_per_launch": cold_b, "hbm_algorithmic_bytes_per_launch": (samp_b + gath_b) / KS,
+                    "hbm_frac": achieved / peak, "launch_ms_mean": step_mean, "concurrent_launches": K,
+                    "achieved_def": "cold feature bytes read over the host link per launch x launches / elapsed time"}
     if rank == 0:
         line = {
             "metric": METRIC, "value": tot_edges / (t_max * 1e-3), "unit": "edges/s", "n_gpus": world,
@@ -497,14 +563,7 @@ def run_dsp(args):
             "feature_GBps": tot_rows * cfg.dim * 4 / (t_max * 1e-3) / 1e9,
             "edges_per_step": tot_edges / KS / world,
             "rows_per_step": tot_rows / KS / world,
-            "roofline": {"kernel": roof_kernel,
-                         "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": ncu_traffic(roof_kernel) if roof_kernel == "k_csp_persistent" else None,
-                         "peak_kind": peak_kind,
-                         "algorithmic_bytes_per_launch": (samp_b + gath_b) / KS,
-                         "sampling_bytes_per_launch": samp_b / KS, "gather_bytes_per_launch": gath_b / KS,
-                         "launch_ms_mean": step_mean, "concurrent_launches": K,
-                         "achieved_def": "algorithmic bytes of all timed launches / elapsed device time"},
+            "roofline": roofline,
             "breakdown": bd,
             "epoch_sampling_s": (steps_epoch * bd["sample_call_ms_mean"] * 1e-3 if bd else None),
             "cpu_baseline": cpu,
