@@ -207,6 +207,40 @@ def test_tiny_virtual_ranks(pkg, tiny, P, mode, monkeypatch):
     grp.close()
 
 
+@pytest.mark.parametrize("mode", ["persistent", "staged"])
+def test_virtual_ranks_errors(pkg, tiny, mode, monkeypatch):
+    """Device-detected errors at world > 1 (duplicate seed, out-of-range seed)
+    are reported by the group call after the exchange protocol completed, and
+    the ranks stay usable; a batch above the reserved size fails before any
+    launch on every rank."""
+    if mode == "staged":
+        monkeypatch.setenv("DSP_MULTI_STAGED", "1")
+    cfg, ip, ix, feats = tiny
+    P = 2
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi]))
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 16, devices=[0] * P)
+    t = lambda x: torch.tensor(x, dtype=torch.int32, device="cuda")
+    with pytest.raises(pkg.DSPError) as e:
+        grp.sample([t([5, 9, 5]), t([7000])], 1)
+    assert e.value.status == pkg.dsp.DSP_ERR_DUPLICATE_SEED
+    with pytest.raises(pkg.DSPError) as e:
+        grp.sample([t([5]), t([7000, cfg.num_nodes])], 1)
+    assert e.value.status == pkg.dsp.DSP_ERR_OUT_OF_RANGE
+    with pytest.raises(pkg.DSPError) as e:
+        grp.sample([t(list(range(17))), t([7000])], 1)
+    assert e.value.status == pkg.dsp.DSP_ERR_CAPACITY
+    seeds = [np.array([1, 9000, 3], np.int32), np.array([7000, 2], np.int32)]
+    res = grp.sample([torch.from_numpy(x).cuda() for x in seeds], 4)
+    for r in range(P):
+        assert_blocks_equal(res[r], oracle.sample(ip, ix, seeds[r], cfg.fanouts, 4), f"{mode} rank {r} after errors")
+    grp.close()
+
+
 # ----------------------------------------------------- products, full size
 
 @pytest.fixture(scope="module")
