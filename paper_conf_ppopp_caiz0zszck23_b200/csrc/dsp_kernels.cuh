@@ -44,8 +44,27 @@ struct WsPersist {
   int32_t pend_n[2];   // row counts of pipelined calls (alternating), read by the next call / flush
   uint32_t hclear;     // epoch at the last zeroing of the relabel hash table (tags unique within 255)
   uint32_t hmask, hoff; // its layout then (slots - 1, offset in 256-B units)
-  uint32_t pad[58];
+  uint32_t dwin;       // compact direct map: 1 + the epoch window it was last zeroed for (0 = never)
+  uint32_t pad[57];
 };
+
+// Compact direct map (4 B per node and parity, the node-wise default when the
+// graph is small enough for a direct map): word = tag(8) | ~x(24), tag = the
+// epoch's position in its window of 255 epochs, so tags grow monotonically
+// within a window and the fire-and-forget max keeps working.  A call never
+// straddles two windows (its first epoch is moved to the next window's start
+// instead) and zeroes the map when it enters a window other than the one of
+// the last zeroing (every ~255 / L calls).  x < 2^24 (checked by the host plan).
+constexpr uint32_t DWIN = 255u;
+// first epoch - 1 of a call of L layers starting after epoch e0 (same window for all L epochs)
+__host__ __device__ __forceinline__ uint32_t dwin_start(uint32_t e0, uint32_t L) {
+  return (e0 % DWIN) + L > DWIN ? (e0 / DWIN + 1u) * DWIN : e0;
+}
+__device__ __forceinline__ uint32_t dtag(uint32_t epoch) { return epoch - DWIN * ((epoch - 1u) / DWIN); }
+__device__ __forceinline__ uint32_t dword(uint32_t epoch, uint32_t x) { return (dtag(epoch) << 24) | (0xffffffu - x); }
+__device__ __forceinline__ bool dclear_due(const WsPersist *ps, uint32_t e0s) {
+  return *(volatile const uint32_t *)&ps->dwin != e0s / DWIN + 1u;
+}
 
 // A call using epochs (e0, e0 + L] must first zero the hash table when a tag
 // could repeat (every word alive was written after the last zeroing) or when
@@ -92,6 +111,8 @@ struct LayerBufs {
   unsigned long long *status;   // [0] tile ticket, [1 + t] tile status (look-back scan)
   unsigned long long *first;    // relabel map: [N] direct words, or [mask + 1] hash slots
   uint32_t mask;                // 0: direct map indexed by global id; else hash table of mask + 1 slots
+  uint32_t *first32;            // compact direct map [N] (tag | ~x words), or nullptr
+  uint32_t n32;                 // its length (N)
 };
 
 struct Outputs {
@@ -145,6 +166,24 @@ __device__ __forceinline__ void map_st(unsigned long long *p, unsigned long long
 __device__ __forceinline__ void mark(unsigned long long *first, int32_t u, uint32_t epoch, uint32_t x) {
   map_red_max(first + u, mark_word(epoch, x));
 }
+__device__ __forceinline__ void map32_red_max(uint32_t *p, uint32_t v) {
+  asm volatile("red.relaxed.gpu.global.max.L2::cache_hint.u32 [%0], %1, %2;" ::"l"(p), "r"(v), "l"(map_policy())
+               : "memory");
+}
+__device__ __forceinline__ uint32_t map32_atom_max(uint32_t *p, uint32_t v) {
+  uint32_t old;
+  asm volatile("atom.relaxed.gpu.global.max.L2::cache_hint.u32 %0, [%1], %2, %3;"
+               : "=r"(old) : "l"(p), "r"(v), "l"(map_policy()) : "memory");
+  return old;
+}
+__device__ __forceinline__ uint32_t map32_ld(const uint32_t *p) {
+  uint32_t v;
+  asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(map_policy()));
+  return v;
+}
+__device__ __forceinline__ void map32_st(uint32_t *p, uint32_t v) {
+  asm volatile("st.global.L2::cache_hint.u32 [%0], %1, %2;" ::"l"(p), "r"(v), "l"(map_policy()) : "memory");
+}
 
 // ------------------------------------------ relabel hash table (large N)
 // For graphs whose direct map (8 B per node and parity) cannot stay in L2,
@@ -163,11 +202,13 @@ __device__ __forceinline__ unsigned long long hword(uint32_t epoch, int32_t u, u
 }
 // word of (epoch, key, x) in the layout of B
 __device__ __forceinline__ unsigned long long mword(const LayerBufs &B, uint32_t epoch, int32_t u, uint32_t x) {
-  return B.mask ? hword(epoch, u, x) : mark_word(epoch, x);
+  return B.first32 ? (unsigned long long)dword(epoch, x) : B.mask ? hword(epoch, u, x) : mark_word(epoch, x);
 }
 // x of a word of the current epoch
 __device__ __forceinline__ uint32_t mword_x(const LayerBufs &B, unsigned long long w) {
-  return B.mask ? 0x1ffffffu - (uint32_t)(w & 0x1ffffffull) : mark_x(w);
+  return B.first32 ? 0xffffffu - (uint32_t)(w & 0xffffffull)
+         : B.mask  ? 0x1ffffffu - (uint32_t)(w & 0x1ffffffull)
+                   : mark_x(w);
 }
 // claims (or finds) the slot of key u; returns its word pointer and the word seen there
 __device__ __forceinline__ unsigned long long *hash_claim(const LayerBufs &B, int32_t u, uint32_t epoch, uint32_t x,
@@ -194,7 +235,7 @@ __device__ __forceinline__ unsigned long long *hash_claim(const LayerBufs &B, in
     h = (h + 1u) & B.mask;
   }
 }
-// slot of key u (inserted earlier in this epoch)
+// slot of key u (inserted earlier in this epoch); 64-bit layouts only
 __device__ __forceinline__ unsigned long long *map_find(const LayerBufs &B, int32_t u, uint32_t epoch) {
   if (!B.mask) return B.first + u;
   const unsigned long long hi = ((unsigned long long)htag(epoch) << 31) | (uint32_t)u;
@@ -202,7 +243,38 @@ __device__ __forceinline__ unsigned long long *map_find(const LayerBufs &B, int3
   while ((map_ld(B.first + h) >> 25) != hi) h = (h + 1u) & B.mask;
   return B.first + h;
 }
+// the word of key u (marked earlier in this epoch), compared with mword()
+__device__ __forceinline__ unsigned long long map_get(const LayerBufs &B, int32_t u, uint32_t epoch) {
+  if (B.first32) return (unsigned long long)map32_ld(B.first32 + u);
+  return map_ld(map_find(B, u, epoch));
+}
+// overwrite the word of key u (marked earlier in this epoch) with x
+__device__ __forceinline__ void map_put(const LayerBufs &B, int32_t u, uint32_t epoch, uint32_t x) {
+  if (B.first32) {
+    map32_st(B.first32 + u, dword(epoch, x));
+    return;
+  }
+  map_st(map_find(B, u, epoch), mword(B, epoch, u, x));
+}
+// zero both parities of the relabel map in use (hash table or compact direct map)
+__device__ __forceinline__ void map_zero(const LayerBufs &B0, const LayerBufs &B1, int64_t tid, int64_t nthreads) {
+  if (B0.first32) {
+    for (int64_t i = tid; i < (int64_t)B0.n32; i += nthreads) {
+      B0.first32[i] = 0u;
+      B1.first32[i] = 0u;
+    }
+  } else if (B0.mask) {
+    for (int64_t i = tid; i <= (int64_t)B0.mask; i += nthreads) {
+      B0.first[i] = 0ull;
+      B1.first[i] = 0ull;
+    }
+  }
+}
 __device__ __forceinline__ void mark(const LayerBufs &B, int32_t u, uint32_t epoch, uint32_t x) {
+  if (B.first32) {
+    map32_red_max(B.first32 + u, dword(epoch, x));
+    return;
+  }
   if (!B.mask) {
     map_red_max(B.first + u, mark_word(epoch, x));
     return;
@@ -314,6 +386,16 @@ __device__ __forceinline__ void mark_dst(unsigned long long *first, int32_t v, i
 }
 __device__ __forceinline__ void mark_dst(const LayerBufs &B, int32_t v, int i, int F, int layer, uint32_t epoch,
                                          int *err) {
+  if (B.first32) {
+    const uint32_t w = dword(epoch, (uint32_t)i);
+    if (layer == 0) {
+      const uint32_t old = map32_atom_max(B.first32 + v, w);
+      if ((old >> 24) == (w >> 24) && 0xffffffu - (old & 0xffffffu) < (uint32_t)F) latch(err, E_DUP);
+    } else {
+      map32_red_max(B.first32 + v, w);
+    }
+    return;
+  }
   if (!B.mask) {
     mark_dst(B.first, v, i, F, layer, epoch, err);
     return;
@@ -547,7 +629,7 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
   }
   unsigned long long w[SCAN2_IPT];
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? map_ld(map_find(B, u[j], epoch)) : 0ull;
+  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? map_get(B, u[j], epoch) : 0ull;
   R.vbits = R.fbits = 0;
 #pragma unroll
   for (int j = 0; j < SCAN2_IPT; ++j) {
@@ -724,7 +806,7 @@ __device__ __forceinline__ void phase_indices(int F, int k, const LayerBufs &B, 
     }
     unsigned long long w[U];
 #pragma unroll
-    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? map_ld(map_find(B, u[j], epoch)) : 0ull;
+    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? map_get(B, u[j], epoch) : 0ull;
 #pragma unroll
     for (int j = 0; j < U; ++j)
       if (c[j] > 0) indices_out[ip[j]] = (int32_t)mword_x(B, w[j]);
@@ -1053,13 +1135,12 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
   const int64_t tid = blockIdx.x * (int64_t)TEAM + threadIdx.x;
   const int64_t nthreads = (int64_t)gridDim.x * TEAM;
   uint32_t bar = 0;  // grid barrier target
-  const uint32_t e0 = *(volatile const uint32_t *)&a.persist->epoch;
+  uint32_t e0 = *(volatile const uint32_t *)&a.persist->epoch;
+  if (a.buf[0].first32) e0 = dwin_start(e0, (uint32_t)a.L);
   const bool hclear = hash_clear_due(a.persist, e0, (uint32_t)a.L, a.buf[0].mask, a.buf[0].first);
-  if (hclear) {  // zero both parities of the relabel hash table (once per ~255 / L calls)
-    for (int64_t i = tid; i <= (int64_t)a.buf[0].mask; i += nthreads) {
-      a.buf[0].first[i] = 0ull;
-      a.buf[1].first[i] = 0ull;
-    }
+  const bool dclear = a.buf[0].first32 && dclear_due(a.persist, e0);
+  if (hclear || dclear) {  // zero both parities of the relabel map (once per ~255 / L calls)
+    map_zero(a.buf[0], a.buf[1], tid, nthreads);
     grid_barrier<TEAM>(a.hdr, bar);
   }
   if (tid == 0) {  // the host cleared the header just before the launch
@@ -1130,6 +1211,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
     if (atomicAdd(&a.hdr->done, 1u) == gridDim.x - 1) {
       a.persist->epoch = e0 + (uint32_t)a.L;
       if (hclear) hash_cleared(a.persist, e0, a.buf[0].mask, a.buf[0].first);
+      if (dclear) a.persist->dwin = e0 / DWIN + 1u;
       a.hdr->t[23] = globaltimer_ns();
       a.hdr->done = 0u;
     }
@@ -1498,7 +1580,7 @@ __global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
     for (int j = 0; j < SCAN_ITEMS; ++j) {
       if (c[j] > 0) {
         vbits |= 1u << j;
-        if (map_ld(map_find(B, u[j], epoch)) == mword(B, epoch, u[j], (uint32_t)F + q0 + j)) fbits |= 1u << j;
+        if (map_get(B, u[j], epoch) == mword(B, epoch, u[j], (uint32_t)F + q0 + j)) fbits |= 1u << j;
       }
     }
     const unsigned long long mine = pack2(__popc(vbits), __popc(fbits));
@@ -1564,7 +1646,7 @@ __global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
         if (q == i * (uint32_t)k) a.indptr_out[i] = (int32_t)pv;
         if (fbits & (1u << j)) {
           const uint32_t nid = (uint32_t)F + pf;
-          map_st(map_find(B, u[j], epoch), mword(B, epoch, u[j], nid));
+          map_put(B, u[j], epoch, nid);
           a.src_ids_out[nid] = u[j];
         }
         pv += (vbits >> j) & 1u;
@@ -1642,6 +1724,19 @@ __global__ void __launch_bounds__(NT) k_random_walk(const int32_t *starts, int64
 __global__ void k_epoch_advance(WsPersist *persist, uint32_t L, LayerBufs b0) {
   if (hash_clear_due(persist, persist->epoch, L, b0.mask, b0.first)) hash_cleared(persist, persist->epoch, b0.mask, b0.first);
   persist->epoch += L;
+}
+
+// start of a stage-by-stage call on the compact direct map: zero it when the
+// call enters a new epoch window (k_map_begin then moves the epoch there)
+__global__ void k_map_clear(WsPersist *persist, uint32_t L, LayerBufs b0, LayerBufs b1) {
+  const uint32_t e0s = dwin_start(*(volatile const uint32_t *)&persist->epoch, L);
+  if (!dclear_due(persist, e0s)) return;
+  map_zero(b0, b1, blockIdx.x * (int64_t)blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x);
+}
+__global__ void k_map_begin(WsPersist *persist, uint32_t L) {
+  const uint32_t e0s = dwin_start(persist->epoch, L);
+  persist->dwin = e0s / DWIN + 1u;
+  persist->epoch = e0s;
 }
 
 // start of a stage-by-stage call on a hashed relabel map: zero the table

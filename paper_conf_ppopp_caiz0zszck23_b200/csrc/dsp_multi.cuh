@@ -285,13 +285,12 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
   const int64_t tid = blockIdx.x * (int64_t)TEAM + threadIdx.x;
   const int64_t nthreads = (int64_t)gridDim.x * TEAM;
   uint32_t bar = 0;
-  const uint32_t e0 = *(volatile const uint32_t *)&a.persist->epoch;
+  uint32_t e0 = *(volatile const uint32_t *)&a.persist->epoch;
+  if (a.buf[0].first32) e0 = dwin_start(e0, (uint32_t)a.L);
   const bool hclear = hash_clear_due(a.persist, e0, (uint32_t)a.L, a.buf[0].mask, a.buf[0].first);
-  if (hclear) {  // zero both parities of the relabel hash table (once per ~255 / L calls)
-    for (int64_t i = tid; i <= (int64_t)a.buf[0].mask; i += nthreads) {
-      a.buf[0].first[i] = 0ull;
-      a.buf[1].first[i] = 0ull;
-    }
+  const bool dclear = a.buf[0].first32 && dclear_due(a.persist, e0);
+  if (hclear || dclear) {  // zero both parities of the relabel map (once per ~255 / L calls)
+    map_zero(a.buf[0], a.buf[1], tid, nthreads);
     grid_barrier<TEAM>(a.hdr, bar);
   }
   if (tid == 0) {
@@ -419,6 +418,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
     if (atomicAdd(&a.hdr->done, 1u) == gridDim.x - 1) {
       a.persist->epoch = e0 + (uint32_t)a.L;
       if (hclear) hash_cleared(a.persist, e0, a.buf[0].mask, a.buf[0].first);
+      if (dclear) a.persist->dwin = e0 / DWIN + 1u;
       a.hdr->t[23] = globaltimer_ns();
       a.hdr->done = 0u;
     }

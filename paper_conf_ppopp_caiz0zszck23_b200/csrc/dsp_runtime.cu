@@ -108,6 +108,8 @@ struct Plan {
   int64_t S[DSP_MAX_LAYERS];       // max src
   int64_t max_F, max_slots, status_len;
   size_t off_hdr, off_agg, off_cnt[2], off_perm, off_rows[2], off_status[2], off_first[2], bytes;
+  size_t off_first32[2];            // compact direct map [2][N] (N <= DIRECT_MAP_MAX_N), else 0
+  bool direct32;                    // node-wise relabel through the compact direct map
   int64_t hash_cap;                 // > 0: relabel hash table of hash_cap slots per parity (else direct map)
   size_t off_hash[2];
   // layer-wise scheme (make_plan_lw)
@@ -174,7 +176,7 @@ struct dsp_ctx {
   int persist_blocks_per_sm = 1;
   int lane_rounds = 4;  // DSP_LANE_ROUNDS (tuning knob, results unchanged)
   int stage_bps = 8;    // DSP_STAGE_BPS: blocks per SM of the owner-sample / unpermute kernels (tuning knob)
-  int relabel_mode = 0; // DSP_RELABEL = direct | hash (default: by N; results unchanged)
+  int relabel_mode = 0; // DSP_RELABEL = direct | direct64 | hash (default: by N; results unchanged)
   int loader_warps = 4; // DSP_LOADER_WARPS = 2, 4 or 8 (tuning knob, results unchanged)
   int loader_rows = 32;  // DSP_LOADER_ROWS: rows per TMA chunk, <= 32 (tuning knob, results unchanged)
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
@@ -252,9 +254,19 @@ dsp_status check_fanouts(dsp_ctx *c, const int32_t *fanouts, int32_t L) {
   return DSP_OK;
 }
 
-// persist | hdr | first[2][N] at fixed offsets for every plan, so that one
-// workspace can serve calls of any size and either scheme (the relabel map's
-// epoch words stay valid across them).
+// The node-wise relabel map is a hash table sized to the batch (north star:
+// "dedup and relabel through a GPU hash table") when a direct map over all N
+// ids is too large to stay in L2; x = F + slot must fit the 25-bit field of a
+// hash word.  Otherwise it is the compact direct map (4 B per node and parity,
+// x < 2^24), or the 8-byte epoch-word direct map beyond that (and for the
+// layer-wise scheme).
+constexpr int64_t DIRECT_MAP_MAX_N = 3 * 1000 * 1000;
+constexpr int64_t HASH_MAX_X = 1ll << 25;
+constexpr int64_t DIRECT32_MAX_X = 1ll << 24;
+
+// persist | hdr | first[2][N] (| first32[2][N] for direct-map sizes) at fixed
+// offsets for every plan, so that one workspace can serve calls of any size
+// and either scheme (the relabel maps' epoch words stay valid across them).
 size_t plan_common(Plan &p, int64_t N) {
   size_t o = align_up(sizeof(WsPersist), 256);
   p.off_hdr = o;
@@ -263,15 +275,14 @@ size_t plan_common(Plan &p, int64_t N) {
     p.off_first[b] = o;
     o = align_up(o + sizeof(unsigned long long) * std::max<int64_t>(1, N), 256);
   }
+  p.off_first32[0] = p.off_first32[1] = 0;
+  if (N <= DIRECT_MAP_MAX_N)
+    for (int b = 0; b < 2; ++b) {
+      p.off_first32[b] = o;
+      o = align_up(o + sizeof(uint32_t) * std::max<int64_t>(1, N), 256);
+    }
   return o;
 }
-
-// The node-wise relabel map is a hash table sized to the batch (north star:
-// "dedup and relabel through a GPU hash table") when the direct map over all
-// N ids (8 B per node and parity) is too large to stay in L2; x = F + slot
-// must fit the 25-bit field of a hash word.
-constexpr int64_t DIRECT_MAP_MAX_N = 3 * 1000 * 1000;
-constexpr int64_t HASH_MAX_X = 1ll << 25;
 
 Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L, int relabel_mode = 0) {
   Plan p{};
@@ -292,6 +303,7 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L, int 
   int64_t max_keys = 0;
   for (int l = 0; l < L; ++l) max_keys = std::max(max_keys, p.F[l] + p.E[l]);
   const bool hashed = max_keys < HASH_MAX_X && (relabel_mode == 2 || (relabel_mode == 0 && N > DIRECT_MAP_MAX_N));
+  p.direct32 = !hashed && relabel_mode != 3 && p.off_first32[0] != 0 && max_keys < DIRECT32_MAX_X;
   p.hash_cap = 0;
   if (hashed) {
     p.hash_cap = 1024;
@@ -474,6 +486,12 @@ LayerBufs bufs_of(const Call &k, int parity) {
   b.status = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_status[parity]);
   b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_first[parity]);
   b.mask = 0;
+  b.first32 = nullptr;
+  b.n32 = 0;
+  if (k.plan.direct32) {
+    b.first32 = reinterpret_cast<uint32_t *>(k.ws + k.plan.off_first32[parity]);
+    b.n32 = (uint32_t)k.c->N;
+  }
   if (k.plan.hash_cap > 0) {
     b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_hash[parity]);
     b.mask = (uint32_t)(k.plan.hash_cap - 1);
@@ -1075,7 +1093,13 @@ dsp_status run_calls(std::vector<Call> &calls) {
       }
       if (l == 0)
         for (auto &k : calls)
-          if (k.plan.hash_cap > 0) {
+          if (k.plan.direct32) {
+            DeviceGuard g(k.c->device);
+            k_map_clear<<<grid_for(k.c, 4), NT, 0, k.stream>>>(persist_of(k), (uint32_t)k.L, bufs_of(k, 0),
+                                                                bufs_of(k, 1));
+            k_map_begin<<<1, 1, 0, k.stream>>>(persist_of(k), (uint32_t)k.L);
+            CUDA_TRY(k.c, cudaGetLastError());
+          } else if (k.plan.hash_cap > 0) {
             DeviceGuard g(k.c->device);
             k_hash_clear<<<grid_for(k.c, 4), NT, 0, k.stream>>>(persist_of(k), (uint32_t)k.L, bufs_of(k, 0),
                                                                  bufs_of(k, 1));
@@ -1337,7 +1361,8 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   if (getenv("DSP_LANE_ROUNDS")) c->lane_rounds = atoi(getenv("DSP_LANE_ROUNDS"));
   if (getenv("DSP_STAGE_BPS")) c->stage_bps = std::max(1, std::min(8, atoi(getenv("DSP_STAGE_BPS"))));
   c->multi_staged = getenv("DSP_MULTI_STAGED") && atoi(getenv("DSP_MULTI_STAGED")) != 0;
-  if (const char *rm = getenv("DSP_RELABEL")) c->relabel_mode = !strcmp(rm, "hash") ? 2 : !strcmp(rm, "direct") ? 1 : 0;
+  if (const char *rm = getenv("DSP_RELABEL"))
+    c->relabel_mode = !strcmp(rm, "hash") ? 2 : !strcmp(rm, "direct") ? 1 : !strcmp(rm, "direct64") ? 3 : 0;
   if (getenv("DSP_LOADER_ROWS")) c->loader_rows = std::max(1, std::min(32, atoi(getenv("DSP_LOADER_ROWS"))));
   if (getenv("DSP_LOADER_WARPS")) {
     const int lw = atoi(getenv("DSP_LOADER_WARPS"));

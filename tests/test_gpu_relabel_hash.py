@@ -1,11 +1,13 @@
-"""GPU parity with the relabel map as a batch-sized hash table (the default
-for graphs of more than 3M nodes -- papers / Friendster -- where a direct map
-over all N ids cannot stay in L2; forced here with DSP_RELABEL=hash on graphs
-the oracle checks quickly).  The hash table only changes where the relabel
-words live, so every block must stay bit-identical to the oracle: P = 1
-(persistent kernel, plain / fused / pipelined), virtual ranks (stage kernels),
-biased sampling, duplicate-seed detection, and enough calls on one workspace
-to cross the 255-epoch tag wrap that zeroes the table."""
+"""GPU parity under each layout of the relabel map, forced with DSP_RELABEL on
+graphs the oracle checks quickly: the batch-sized hash table (the default for
+graphs of more than 3M nodes -- papers / Friendster -- where a direct map over
+all N ids cannot stay in L2), the compact 4-byte direct map (the default
+below that) and the 8-byte epoch-word direct map.  The layout only changes
+where the relabel words live, so every block must stay bit-identical to the
+oracle: P = 1 (persistent kernel, plain / fused / pipelined), virtual ranks
+(persistent and stage-by-stage kernels), biased sampling, duplicate-seed
+detection, and enough calls on one workspace to cross the 255-epoch windows
+that zero the hash table and the compact map."""
 import os
 
 import numpy as np
@@ -29,9 +31,9 @@ def pkg():
     return p
 
 
-@pytest.fixture
-def hashed(monkeypatch):
-    monkeypatch.setenv("DSP_RELABEL", "hash")   # read by dsp_create
+@pytest.fixture(params=["hash", "direct", "direct64"])
+def hashed(request, monkeypatch):
+    monkeypatch.setenv("DSP_RELABEL", request.param)   # read by dsp_create
 
 
 @pytest.fixture(scope="module")
@@ -103,8 +105,11 @@ def test_hash_duplicate_seed(pkg, tiny, hashed):
     s.close()
 
 
+@pytest.mark.parametrize("mode", ["persistent", "staged"])
 @pytest.mark.parametrize("P", [2, 4])
-def test_hash_virtual_ranks(pkg, tiny, hashed, P):
+def test_hash_virtual_ranks(pkg, tiny, hashed, P, mode, monkeypatch):
+    if mode == "staged":
+        monkeypatch.setenv("DSP_MULTI_STAGED", "1")
     cfg, ip, ix, feats = tiny
     bnds = datagen.bounds(cfg.num_nodes, P)
     shards = []
