@@ -205,6 +205,29 @@ def run_reference(args):
     edges = rows = 0
     steps_done = 0
     t_all = 0.0
+    if args.scheme == "walk":   # a bounded sample of each step's walks (4096 of --walkers)
+        rng = np.random.default_rng(1234)
+        for step in range(args.warmup + args.steps):
+            st = rng.integers(0, cfg.num_nodes, size=min(args.walkers, 4096)).astype(np.int32)
+            t0 = time.perf_counter()
+            tr = oracle.random_walk(ip, ix, st, args.walk_length, datagen.BASE_SEED + step)
+            dt = time.perf_counter() - t0
+            if step >= args.warmup:
+                t_all += dt
+                edges += int((tr[:, 1:] >= 0).sum())
+                steps_done += 1
+                if t_all > args.ref_max_seconds:
+                    break
+        line = {"impl": "reference", "metric": METRIC, "value": edges / t_all, "unit": "edges/s",
+                "n_gpus": args.gpus, "steps": steps_done, "warmup": args.warmup,
+                "ms_per_step": 1e3 * t_all / steps_done, "higher_is_better": True, "scaling": "weak",
+                "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+                "config": {"workload": f"{cfg.name}-walk", "scheme": "walk", "walk_length": args.walk_length},
+                "cpu_baseline": {"value": edges / t_all, "unit": "edges/s", "cores": 1, "kind": "oracle",
+                                 "sample": f"{steps_done} x {min(args.walkers, 4096)} walks (oracle.random_walk)"},
+                "e2e": {"value": edges / t_all, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return 0
     for step in range(args.warmup + args.steps):
         seeds = batches[step % len(batches)]
         t0 = time.perf_counter()
@@ -265,6 +288,108 @@ def algorithmic_bytes(sizes, L, dim):
     new = sum(int(sizes[3 * l + 1]) - int(sizes[3 * l]) for l in range(L))
     U = int(sizes[3 * (L - 1) + 1])
     return 24 * F + 8 * E + 4 * new, 2 * U * dim * 4
+
+
+def run_walk(args):
+    """--scheme walk: random walks (fan-out 1 at every step, a node
+    without neighbours ends its walk) of --walk-length steps from --walkers
+    start nodes per GPU; one bench step = one dsp_random_walk call.  Metric:
+    walk steps (sampled edges) per second."""
+    import datagen
+    import paper_conf_ppopp_caiz0zszck23_b200 as pkg
+    rank, world, local = setup_dist(args.gpus)
+    torch.cuda.set_device(local)
+    cfg, ip, ix, bnds, sip, six, feats, train = load_workload(args.config, rank, world)
+    ex = pkg.torch_exchange() if world > 1 else None
+    nw, length = args.walkers, args.walk_length
+    s = pkg.Sampler(bnds, sip, six, feats, cfg.fanouts, cfg.batch, rank=rank, world_size=world, device=local,
+                    exchange=ex, max_walks=nw if world > 1 else None, max_walk_length=length)
+    lo, hi = int(bnds[rank]), int(bnds[rank + 1])
+    rng = np.random.default_rng(1234 + rank)
+    KS, W = args.steps, args.warmup
+    starts = [torch.from_numpy(rng.integers(lo, hi, size=nw).astype(np.int32)).cuda() for _ in range(4)]
+    stream = torch.cuda.current_stream()
+    for i in range(W):
+        s.random_walk(starts[i % 4], length, datagen.BASE_SEED + i)
+    s.sync()
+    barrier()
+    torch.cuda.synchronize()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    outs = []
+    with ClockSampler(local) as clk:
+        ev0.record(stream)
+        for j in range(KS):
+            outs.append(s.random_walk(starts[j % 4], length, datagen.BASE_SEED + W + j))
+        ev1.record(stream)
+        s.sync()
+        torch.cuda.synchronize()
+    barrier()
+    t_ms = ev0.elapsed_time(ev1)
+    # steps actually taken (a walk ends at a node without neighbours: -1 afterwards)
+    steps_taken = float(sum(int((o[:, 1:] >= 0).sum().item()) for o in outs))
+    t_max = reduce_max_over_ranks(t_ms)
+    tot = reduce_sum_over_ranks(steps_taken)
+    peak, peak_kind = measured_peaks()
+    # algorithmic bytes per walk step: indptr pair (16 B) + the adjacency id (4 B) + the trace entry (4 B)
+    achieved = 24.0 * steps_taken / (t_ms * 1e-3) / 1e9
+    # e2e: starts H2D from pinned host memory and the traces D2H into pinned host memory every call
+    h_starts = [x.cpu().pin_memory() for x in starts]
+    h_out = torch.empty((nw, length + 1), dtype=torch.int32).pin_memory()
+    d_st = torch.empty(nw, dtype=torch.int32, device="cuda")
+    n_e2e = max(3, min(KS, 20))
+    barrier()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    e_steps = 0
+    for j in range(n_e2e):
+        d_st.copy_(h_starts[j % 4], non_blocking=True)
+        o = s.random_walk(d_st, length, datagen.BASE_SEED + j)
+        h_out.copy_(o, non_blocking=True)
+        e_steps += nw * length
+    e1.record(stream)
+    torch.cuda.synchronize()
+    e2e_ms = reduce_max_over_ranks(e0.elapsed_time(e1))
+    e2e_frac = steps_taken / (KS * nw * length) if KS else 1.0
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": tot / (t_max * 1e-3), "unit": "edges/s", "n_gpus": world,
+            "steps": KS, "warmup": W, "ms_per_step": t_max / KS, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+            "config": {"workload": f"{cfg.name}-walk" + (f"-P{world}" if world > 1 else ""), "scheme": "walk",
+                       "walkers_per_gpu": nw, "walk_length": length, "num_nodes": cfg.num_nodes,
+                       "nnz": int(ip[-1]), "parallelism": f"csp{world}",
+                       "starts": "uniform over each rank's own node range, 4 fixed sets",
+                       "step": "dsp_random_walk (thread per walk at world 1; CSP push without reshuffle at world > 1)"},
+            "roofline": {"kernel": "k_random_walk" if world == 1 else "k_walk_step", "bound": "hbm",
+                         "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                         "traffic": None, "peak_kind": peak_kind,
+                         "algorithmic_bytes_per_launch": 24.0 * steps_taken / KS,
+                         "achieved_def": "24 B per walk step (indptr pair, adjacency id, trace entry) / elapsed time; "
+                                         "the walk is bound by dependent random DRAM requests, not bytes"},
+            "e2e": {"value": reduce_sum_over_ranks(e_steps * e2e_frac) / (e2e_ms * 1e-3), "unit": "edges/s",
+                    "h2d_bytes_per_step": nw * 4, "d2h_bytes_per_step": nw * (length + 1) * 4, "steps": n_e2e,
+                    "api": "starts H2D from pinned host memory, dsp_random_walk, traces D2H into pinned host memory"},
+            "cpu_baseline": None,
+            "gpu_launches": KS if world == 1 else KS * (2 * length + 3),
+            "clocks": clk.summary(),
+        }
+        if world == 1 and not args.no_cpu_baseline:
+            import oracle
+            n_cpu, t_cpu, st_cpu = 0, 0.0, 0
+            while t_cpu < min(args.cpu_seconds, 10.0) and n_cpu < 50:
+                st = starts[n_cpu % 4][:4096].cpu().numpy()
+                t0 = time.perf_counter()
+                tr = oracle.random_walk(ip, ix, st, length, datagen.BASE_SEED + n_cpu)
+                t_cpu += time.perf_counter() - t0
+                st_cpu += int((tr[:, 1:] >= 0).sum())
+                n_cpu += 1
+            line["cpu_baseline"] = {"value": st_cpu / t_cpu, "unit": "edges/s", "cores": 1, "kind": "oracle",
+                                    "sample": f"{n_cpu} x 4096 walks of length {length}, single host thread "
+                                              f"(oracle.random_walk), {t_cpu:.1f} s"}
+        print(json.dumps(line), flush=True)
+    s.close()
+    return 0
 
 
 def run_dsp(args):
@@ -608,7 +733,9 @@ def main(argv=None):
     ap.add_argument("--instances", type=int, default=4, help="concurrent step streams (world 1)")
     ap.add_argument("--layer-sizes", default="1000,1000",
                     help="--scheme layer: nodes sampled per layer (Table 7: 1000,1000)")
-    ap.add_argument("--scheme", choices=["uniform", "biased", "layer"], default="uniform",
+    ap.add_argument("--walkers", type=int, default=65536, help="--scheme walk: walks per GPU per step")
+    ap.add_argument("--walk-length", type=int, default=80, help="--scheme walk: steps per walk (DeepWalk's 80)")
+    ap.add_argument("--scheme", choices=["uniform", "biased", "layer", "walk"], default="uniform",
                     help="node-wise scheme (Table 2 IsBiased); biased uses synthetic node weights")
     ap.add_argument("--hot-frac", type=float, default=None,
                     help="cold-feature tier: fraction of each shard's rows kept in HBM (P:L114)")
@@ -619,6 +746,8 @@ def main(argv=None):
         args.config = "products"
     if args.impl == "reference":
         return run_reference(args)
+    if args.scheme == "walk":
+        return run_walk(args)
     return run_dsp(args)
 
 
