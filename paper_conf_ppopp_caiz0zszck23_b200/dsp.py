@@ -426,11 +426,14 @@ class Sampler:
         dsp_gather_features(self.ctx, ids, n, out, self.stream())
         return out
 
-    def random_walk(self, starts, length: int, rng_seed: int):
-        """Walk traces int32[n][length + 1], asynchronous on the stream."""
+    def random_walk(self, starts, length: int, rng_seed: int, out=None):
+        """Walk traces int32[n][length + 1], asynchronous on the stream
+        (into `out` when given: a caller-owned int32[n][length + 1] buffer)."""
         torch = self.torch
         assert starts.dtype == torch.int32 and starts.is_cuda and starts.is_contiguous()
-        out = torch.empty((starts.numel(), length + 1), dtype=torch.int32, device=starts.device)
+        if out is None:
+            out = torch.empty((starts.numel(), length + 1), dtype=torch.int32, device=starts.device)
+        assert out.dtype == torch.int32 and out.is_cuda and out.is_contiguous() and out.shape == (starts.numel(), length + 1)
         dsp_random_walk(self.ctx, starts, starts.numel(), length, rng_seed, out, self.stream())
         return out
 
