@@ -395,6 +395,44 @@ def test_products_pipelined(pkg, products):
     s.close()
 
 
+@pytest.mark.slow
+def test_products_bench_launch_configuration(pkg, products):
+    """configs[1] at full size in exactly the launch configuration bench.py
+    times: 4 concurrent step streams, each pipelined persistent launch on 37
+    SMs with its own workspace, 8 output sets, sizes returned asynchronously;
+    every step whose output set survives is checked against the oracle
+    (blocks bit-exact, every gathered row against the closed-form features)."""
+    cfg, ip, ix = products
+    feats = datagen.features(0, cfg.num_nodes, cfg.dim)
+    K = 4
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2 * K,
+                    n_workspaces=K)
+    pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(0).multi_processor_count // K)
+    batches = seeds_of(cfg, 1, 0)
+    L = len(cfg.fanouts)
+    n = 12
+    sizes = torch.zeros((n, 3 * L), dtype=torch.int64).pin_memory()
+    dev = [torch.from_numpy(batches[i]).cuda() for i in range(n)]   # resident, as in bench.py
+    main = torch.cuda.current_stream()
+    streams = [torch.cuda.Stream() for _ in range(K)]
+    for st in streams:
+        st.wait_stream(main)
+    for i in range(n):
+        s.sample_gather(dev[i], 0x5EED + i, slot=i % (2 * K), sizes_out=sizes[i],
+                        async_=True, pipelined=True, ws=i % K, stream=streams[i % K])
+    for st in streams:
+        with torch.cuda.stream(st):
+            s.flush()
+    for st in streams:
+        main.wait_stream(st)
+    s.sync()
+    torch.cuda.synchronize()
+    feats_of = lambda ids: datagen.features_of(ids, cfg.dim)
+    for i in range(n - 2 * K, n):
+        _check_step(s, i % (2 * K), sizes[i], batches[i], 0x5EED + i, ip, ix, feats_of)
+    s.close()
+
+
 # ------------------------------------------------------------ biased (P:L170)
 
 @pytest.fixture(scope="module")
