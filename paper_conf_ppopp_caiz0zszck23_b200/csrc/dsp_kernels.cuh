@@ -356,11 +356,16 @@ __device__ __forceinline__ uint32_t ld_acquire_gpu_u32(const uint32_t *p) {
 // return value, so no extra round trip); pollers acquire.  1.25 us at 148
 // blocks, vs 2.5 us for an atomicAdd + generation barrier over 592 blocks
 // (tools/micro/barrier_bench.cu).
-template <int TEAM = PNT>
+// SYS: thread 0 also issues a system-scope fence after the block barrier, so
+// every store of the block (peer memory included) is ordered before its
+// arrival (cumulativity through bar.sync), and a flag released at system scope
+// after the barrier publishes them to other GPUs.
+template <int TEAM = PNT, bool SYS = false>
 __device__ __forceinline__ void grid_barrier(WsHeader *hdr, uint32_t &target) {
   team_sync<TEAM>();
   target += gridDim.x;
   if (threadIdx.x == 0) {
+    if (SYS) __threadfence_system();
     const uint32_t g = target / gridDim.x;
     if (blockIdx.x == 0 && g < 23u) hdr->ta[g] = globaltimer_ns();
     red_add_release_gpu(&hdr->bar_count, 1u);

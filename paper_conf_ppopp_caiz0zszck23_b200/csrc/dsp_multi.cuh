@@ -6,12 +6,12 @@
 //   A  shuffle   : group the frontier by owner (contiguous id ranges),
 //                  write each id straight into the owner's inbox (peer store),
 //                  perm[i] = its inbox slot;  [indices of layer l-1 meanwhile]
-//                  -- fence.sys, GB, block 0 publishes counts + header and the
+//                  -- GB with fence.sys, block 0 publishes counts + header and the
 //                  inbox flag of every owner (count notification)
 //   B  sample    : wait for every rank's inbox flag; sample every received
 //                  task (one phase over all tasks) and write the row
 //                  straight into the requester's return slot (reshuffle)
-//                  -- fence.sys, GB, block 0 releases the return flags
+//                  -- GB with fence.sys, block 0 releases the return flags
 //   C  unpermute : wait for every owner's return flag; frontier node i takes
 //                  its row from slot perm[i] of its owner, writes the edge
 //                  slots and marks the relabel map (as the local sampler does)
@@ -36,12 +36,6 @@
 #include "dsp_kernels.cuh"
 
 namespace dsp {
-
-#ifdef DSP_EXPERIMENT_GPU_FENCE  // cost measurement on virtual ranks only (not valid across GPUs)
-#define MULTI_BLOCK_FENCE() __threadfence()
-#else
-#define MULTI_BLOCK_FENCE() __threadfence_system()
-#endif
 
 struct MultiArgs {
   PersistArgs p;            // the world-1 persistent kernel's arguments
@@ -314,8 +308,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
     if (l > 0)
       phase_indices_dups(Fprev, a.k[l - 1], a.buf[(l - 1) & 1], a.out.indptr[l - 1], a.out.indices[l - 1],
                          block_span<TEAM>((int64_t)Fprev * a.k[l - 1]));
-    MULTI_BLOCK_FENCE();  // this block's peer stores, before the barrier that precedes the flag
-    grid_barrier<TEAM>(a.hdr, bar);
+    grid_barrier<TEAM, true>(a.hdr, bar);  // + fence.sys: the block's peer stores precede the flag
     if (blk == 0 && threadIdx.x == 0) {
       for (int o = 0; o < world; ++o) {
         const uint32_t c = *(volatile uint32_t *)&a.hdr->bucket[o];
@@ -353,8 +346,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
       multi_sample_tpn<8, TEAM>(m, T, s_off, l, k, par);
     else
       multi_sample_tpn<16, TEAM>(m, T, s_off, l, k, par);
-    MULTI_BLOCK_FENCE();
-    grid_barrier<TEAM>(a.hdr, bar);
+    grid_barrier<TEAM, true>(a.hdr, bar);
     if (blk == 0 && threadIdx.x == 0) {
       __threadfence_system();
       for (int s = 0; s < world; ++s) st_release_sys(xch_ret_flag(m.peers.base[s], m.X, par, m.rank), seq);
