@@ -609,34 +609,57 @@ def run_dsp(args):
 
     def e2e_async_run():
         # the bench step with the seeds in pinned HOST memory: every step copies its seeds
-        # H2D and its per-layer sizes D2H in stream order on its step stream (the paper's
-        # pipelined loader: copies, sampling and the previous gather overlap)
+        # H2D and reads its per-layer sizes back D2H into pinned host memory.  The copies run
+        # on their own streams, ordered by events against the step streams (the paper's
+        # pipelined loader: copies, sampling and the previous gather overlap):
+        # seeds of step j land in buffer j % nbuf once step j - nbuf has consumed it; the
+        # sizes leave once step j is done.
         nbuf = 2 * K
         d_seeds = [torch.empty(cfg.batch, dtype=torch.int32, device="cuda") for _ in range(nbuf)]
         n_steps = max(3, min(KS, 200))
         h_sz = torch.zeros((n_steps, 3 * L), dtype=torch.int64).pin_memory()
+        d_sz = torch.zeros((n_steps, 3 * L), dtype=torch.int64, device="cuda")
+        cs_in, cs_out = torch.cuda.Stream(), torch.cuda.Stream()
+        ready = [torch.cuda.Event() for _ in range(nbuf)]
+        used = [torch.cuda.Event() for _ in range(nbuf)]
         barrier()
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record(stream)
         fork()
+        cs_in.wait_stream(stream)
+        cs_out.wait_stream(stream)
         for j in range(n_steps):
             i = W + j
             st = streams[j % K]
-            buf = d_seeds[j % nbuf]
-            with torch.cuda.stream(st):
-                buf.copy_(h_seeds[i % len(batches)], non_blocking=True)
-            s.sample_gather(buf, datagen.BASE_SEED + i, slot=(j % (2 * K)), sizes_out=h_sz[j], async_=True,
+            b = j % nbuf
+            with torch.cuda.stream(cs_in):
+                if j >= nbuf:
+                    cs_in.wait_event(used[b])
+                d_seeds[b].copy_(h_seeds[i % len(batches)], non_blocking=True)
+                ready[b].record(cs_in)
+            st.wait_event(ready[b])
+            s.sample_gather(d_seeds[b], datagen.BASE_SEED + i, slot=(j % (2 * K)), sizes_out=d_sz[j], async_=True,
                             pipelined=pipelined, biased=biased, ws=j % K, stream=st)
+            used[b].record(st)
+            with torch.cuda.stream(cs_out):
+                cs_out.wait_event(used[b])
+                h_sz[j].copy_(d_sz[j], non_blocking=True)
         flush_all()
         join()
+        stream.wait_stream(cs_in)
+        stream.wait_stream(cs_out)
         e1.record(stream)
         torch.cuda.synchronize()
         ms = reduce_max_over_ranks(e0.elapsed_time(e1))
         n_edges = float(h_sz.numpy()[:, 2::3].sum())
         return reduce_sum_over_ranks(n_edges) / (ms * 1e-3), cfg.batch * 4, 3 * 8 * L, n_steps
 
+    if K > 1:   # the asynchronous e2e runs the timed step's configuration: K streams x 1/K of the SMs
+        pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(local).multi_processor_count // K)
     e2e_av, e2e_ah2d, e2e_ad2h, e2e_an = e2e_async_run() if not layer else (None, 0, 0, 0)
+    if K > 1:   # one synchronous call at a time: the whole GPU
+        pkg.dsp_set_persistent_blocks(s.ctx, 0)
     e2e_v, e2e_h2d, e2e_d2h = e2e_run(False)
     e2e_hv, e2e_hh2d, e2e_hd2h = e2e_run(True)
 
@@ -701,9 +724,10 @@ def run_dsp(args):
             "cpu_baseline": cpu,
             "e2e": ({"value": e2e_av, "unit": "edges/s", "h2d_bytes_per_step": e2e_ah2d,
                      "d2h_bytes_per_step": e2e_ad2h, "steps": e2e_an,
-                     "api": "per step: seeds H2D from pinned host memory, dsp_sample_gather (pipelined, async) "
-                            "and its per-layer sizes D2H into pinned host memory, in stream order on the step's "
-                            "stream (as the timed step); blocks and features stay in HBM for the GPU consumer"}
+                     "api": "per step: seeds H2D from pinned host memory (copy stream), dsp_sample_gather "
+                            "(pipelined, async, as the timed step) and its per-layer sizes D2H into pinned host "
+                            "memory (second copy stream), ordered by events; blocks and features stay in HBM "
+                            "for the GPU consumer"}
                     if e2e_av is not None else
                     {"value": e2e_v, "unit": "edges/s", "h2d_bytes_per_step": e2e_h2d,
                      "d2h_bytes_per_step": e2e_d2h, "steps": e2e_steps,
