@@ -174,7 +174,7 @@ struct dsp_ctx {
   int *h_err = nullptr;
   int num_sms = 148;
   int persist_blocks_per_sm = 1;
-  int lane_rounds = 4;  // DSP_LANE_ROUNDS (tuning knob, results unchanged)
+  int lane_rounds = 8;  // DSP_LANE_ROUNDS (tuning knob, results unchanged; 8 measured best with 4 streams)
   int stage_bps = 8;    // DSP_STAGE_BPS: blocks per SM of the owner-sample / unpermute kernels (tuning knob)
   int relabel_mode = 0; // DSP_RELABEL = direct | direct64 | hash (default: by N; results unchanged)
   int loader_warps = 4; // DSP_LOADER_WARPS = 2, 4 or 8 (tuning knob, results unchanged)
