@@ -224,8 +224,12 @@ dsp_status dsp_sample(dsp_ctx *ctx, const int32_t *seeds, int32_t num_seeds, con
 /* The same collective for n_ctx ctxs of one world driven by ONE host thread
    (virtual ranks sharing a device, or one process owning several GPUs).
    Array arguments are indexed by position in ctxs (any rank order, all ranks
-   of the world present).  Stages are issued rank by rank per stage, so
-   virtual ranks may share one stream. */
+   of the world present).  Node-wise calls run one persistent kernel per rank
+   (the exchanges through peer memory inside it); ranks sharing a device each
+   get 1/n of its SMs on the ctx's own stream, forked from and joined to the
+   given stream after all ranks were launched.  Virtual ranks sharing a device
+   must pass the same stream.  The layer-wise scheme (and DSP_MULTI_STAGED=1)
+   issues its stage kernels rank by rank per stage on that stream. */
 dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *seeds,
                             const int32_t *num_seeds, const int32_t *fanouts, int32_t num_layers,
                             uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
@@ -235,7 +239,8 @@ dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *
 /* One whole step of the hot path in ONE stream-ordered call: dsp_sample
    followed by the feature gather of the last block's src_ids (the loader
    right after the sampler), with no host round trip in between.
-   With world_size == 1 the step runs as a single persistent kernel.
+   The step runs as a single persistent kernel per rank (world_size == 1, or
+   > 1 with the shuffle / reshuffle through NVLink peer memory inside it).
    Same arguments, rules and collectiveness as dsp_sample, plus:
    feat_out     : DEVICE fp32 [feat_cap_rows][dim], 16-byte aligned; rows
                   [0, blocks[L-1].num_src) receive the features of
@@ -255,7 +260,7 @@ dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *
                   paper's pipeline runs one step behind the sampler
                   (P:L198-200): this call samples its seeds into `blocks`
                   while, in the same launch, it gathers the features owed by
-                  the PREVIOUS pipelined call of this ctx into that call's
+                  the PREVIOUS pipelined call of this ctx on the same workspace into that call's
                   feat_out; this call's features are written by the next
                   pipelined call or by dsp_pipeline_flush.  The caller keeps
                   the previous call's blocks and feat_out alive until then
