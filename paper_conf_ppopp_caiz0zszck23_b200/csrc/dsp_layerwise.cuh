@@ -153,8 +153,10 @@ constexpr size_t LW_ALLOC_SMEM = (size_t)LW_SMEM_F * (sizeof(unsigned long long)
 
 // Dynamic shared memory: LW_ALLOC_SMEM (prefix u64 + counts i32 of up to
 // LW_SMEM_F frontier nodes); larger frontiers use the workspace copies.
-__global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
-  extern __shared__ unsigned long long lw_alloc_smem[];
+// PERS: inside the world-1 persistent kernel (k_lw_persistent): no flags, the
+// phases are ordered by its grid barriers.
+template <bool PERS>
+__device__ __forceinline__ void lw_alloc_body(const LwArgs &a, unsigned long long *lw_alloc_smem) {
   __shared__ unsigned long long s_u64[33];
   __shared__ int32_t s_i32[33];
   __shared__ uint32_t s_cnt[8];
@@ -180,7 +182,7 @@ __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
       const int i = b0 + tid * LW_IPT + j;
       W[j] = 0;
       if (i < F) {
-        const int32_t v = __ldg(a.frontier + i);
+        const int32_t v = ldw_i32(a.frontier + i);  // may be written earlier in the same kernel (PERS)
         if (v < 0 || v >= a.bd.b[a.bd.world]) {
           latch(a.err, E_RANGE);
         } else {
@@ -235,7 +237,7 @@ __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
       a.w.off[i] = off;
       if (ci > 0) {
         for (int t = 0; t < ci; ++t) a.w.slot_node[off + t] = i;
-        const int32_t v = __ldg(a.frontier + i);
+        const int32_t v = ldw_i32(a.frontier + i);  // may be written earlier in the same kernel (PERS)
         o_req = owner_of(a.bd, v);
         req = make_int4(i, v, ci, off);
       }
@@ -257,18 +259,25 @@ __global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
   if (tid == 0) {
     for (int o = 0; o < a.bd.world; ++o)
       *lw_inbox_hdr(a.peers.base[o], a.L, a.parity, a.rank) = make_uint4(s_cnt[o], lw_tag(a.n, a.layer), a.key.x, a.key.y);
-    if (a.sys) __threadfence_system();
-    for (int o = 0; o < a.bd.world; ++o)
-      st_release_flag(lw_inbox_flag(a.peers.base[o], a.L, a.parity, a.rank), a.seq, a.sys);
+    if (!PERS) {
+      if (a.sys) __threadfence_system();
+      for (int o = 0; o < a.bd.world; ++o)
+        st_release_flag(lw_inbox_flag(a.peers.base[o], a.L, a.parity, a.rank), a.seq, a.sys);
+    }
   }
+}
+__global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
+  extern __shared__ unsigned long long lw_alloc_smem[];
+  lw_alloc_body<false>(a, lw_alloc_smem);
 }
 
 // Owner side: every task received in this layer, one warp each.
-__global__ void __launch_bounds__(NT) k_lw_sample_remote(LwArgs a) {
+template <bool PERS>
+__device__ __forceinline__ void lw_sample_remote_body(const LwArgs &a) {
   __shared__ uint32_t s_off[9];
   char *self = a.peers.base[a.rank];
   const int world = a.bd.world;
-  if (wait_flags(lw_inbox_flag(self, a.L, a.parity, 0), world, a.seq, a.err)) {
+  if (PERS || wait_flags(lw_inbox_flag(self, a.L, a.parity, 0), world, a.seq, a.err)) {
     if (threadIdx.x == 0) {
       uint32_t acc = 0;
       for (int s = 0; s < world; ++s) {
@@ -282,8 +291,8 @@ __global__ void __launch_bounds__(NT) k_lw_sample_remote(LwArgs a) {
     __syncthreads();
     const int T = (int)s_off[world];
     const int lane = threadIdx.x & 31;
-    const int warp = (blockIdx.x * NT + threadIdx.x) >> 5;
-    const int nwarps = (gridDim.x * NT) >> 5;
+    const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int nwarps = (gridDim.x * blockDim.x) >> 5;
     for (int q = warp; q < T; q += nwarps) {
       int s = 0;
       while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
@@ -317,13 +326,14 @@ __global__ void __launch_bounds__(NT) k_lw_sample_remote(LwArgs a) {
       }
     }
   }
-  if (a.sys) __threadfence_system();  // this kernel's peer stores, before k_lw_sample_big's flags
+  if (!PERS && a.sys) __threadfence_system();  // this kernel's peer stores, before k_lw_sample_big's flags
 }
+__global__ void __launch_bounds__(NT) k_lw_sample_remote(LwArgs a) { lw_sample_remote_body<false>(a); }
 
 // Tasks with 32 < c < deg: Floyd over c draws with a shared-memory hash set.
 // Dynamic shared memory: kp (pow2 >= c) positions + 2 kp hash slots.
-__global__ void __launch_bounds__(LWT) k_lw_sample_big(LwArgs a, int kp_max) {
-  extern __shared__ int32_t lw_smem[];
+template <bool PERS>
+__device__ __forceinline__ void lw_sample_big_body(const LwArgs &a, int kp_max, int32_t *lw_smem) {
   int32_t *sel = lw_smem;                 // [kp_max]
   int32_t *hkeys = lw_smem + kp_max;      // [2 * kp_max]
   char *self = a.peers.base[a.rank];
@@ -379,25 +389,30 @@ __global__ void __launch_bounds__(LWT) k_lw_sample_big(LwArgs a, int kp_max) {
     if (threadIdx.x == 0) lw_ret_cnt(req_base, a.L, a.parity)[req.x] = k;
     __syncthreads();
   }
-  if (lw_last_block_done(&a.hdr->done, a.sys)) {
+  if (!PERS && lw_last_block_done(&a.hdr->done, a.sys)) {
     a.hdr->lw_big = 0u;
     for (int s = 0; s < a.bd.world; ++s)
       st_release_flag(lw_ret_flag(a.peers.base[s], a.L, a.parity, a.rank), a.seq, a.sys);
   }
 }
+__global__ void __launch_bounds__(LWT) k_lw_sample_big(LwArgs a, int kp_max) {
+  extern __shared__ int32_t lw_smem[];
+  lw_sample_big_body<false>(a, kp_max, lw_smem);
+}
 
 // Requester: dst copy + marks, first-occurrence marks of the returned rows.
-__global__ void __launch_bounds__(NT) k_lw_collect(LwArgs a) {
+template <bool PERS>
+__device__ __forceinline__ void lw_collect_body(const LwArgs &a) {
   char *self = a.peers.base[a.rank];
-  if (!wait_flags(lw_ret_flag(self, a.L, a.parity, 0), a.bd.world, a.seq, a.err)) return;
+  if (!PERS && !wait_flags(lw_ret_flag(self, a.L, a.parity, 0), a.bd.world, a.seq, a.err)) return;
   const uint32_t epoch = a.persist->epoch + 1u + (uint32_t)a.layer;
   const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
   const int Q = a.w.off[F];
   const int32_t *ret_cnt = lw_ret_cnt(self, a.L, a.parity);
   const int32_t *ret_rows = lw_ret_rows(self, a.L, a.parity);
-  const int tid = blockIdx.x * NT + threadIdx.x, nth = gridDim.x * NT;
+  const int tid = blockIdx.x * blockDim.x + threadIdx.x, nth = gridDim.x * blockDim.x;
   for (int i = tid; i < F; i += nth) {
-    const int32_t v = __ldg(a.frontier + i);
+    const int32_t v = ldw_i32(a.frontier + i);  // written by the previous layer (same kernel when PERS)
     a.out.src_ids[0][i] = v;
     if (v >= 0 && v < a.bd.b[a.bd.world]) mark_dst(a.first, v, i, F, a.layer, epoch, a.err);
   }
@@ -406,9 +421,10 @@ __global__ void __launch_bounds__(NT) k_lw_collect(LwArgs a) {
     if (q - a.w.off[i] < __ldcv(ret_cnt + i)) mark(a.first, __ldcv(ret_rows + q), epoch, (uint32_t)F + (uint32_t)q);
   }
 }
+__global__ void __launch_bounds__(NT) k_lw_collect(LwArgs a) { lw_collect_body<false>(a); }
 
 // Requester: block l from the marks (one block; Q <= n <= 8192 slots).
-__global__ void __launch_bounds__(LWT) k_lw_finish(LwArgs a) {
+__device__ __forceinline__ void lw_finish_body(const LwArgs &a) {
   __shared__ unsigned long long s_u64[33];
   char *self = a.peers.base[a.rank];
   const uint32_t epoch = a.persist->epoch + 1u + (uint32_t)a.layer;
@@ -456,6 +472,38 @@ __global__ void __launch_bounds__(LWT) k_lw_finish(LwArgs a) {
     a.hdr->sizes[3 * a.layer + 0] = F;
     a.hdr->sizes[3 * a.layer + 1] = F + nnew;
     a.hdr->sizes[3 * a.layer + 2] = E;
+  }
+}
+__global__ void __launch_bounds__(LWT) k_lw_finish(LwArgs a) { lw_finish_body(a); }
+
+// World 1: every layer of the call in ONE cooperative launch (the per-layer
+// kernels above are launch- and drain-bound at Table 7's sizes: ~1000 nodes
+// per layer).  Phases per layer, separated by grid barriers: allocation
+// (block 0), owner-side sampling (one warp per task), tasks with c > 32,
+// marks, block construction (block 0).
+struct LwPersistArgs {
+  LwArgs l[DSP_MAX_LAYERS];
+  int32_t L;
+  int32_t kp_max;
+  WsHeader *hdr;
+};
+
+__global__ void __launch_bounds__(LWT, 1) k_lw_persistent(LwPersistArgs p) {
+  extern __shared__ unsigned long long lw_dyn[];
+  uint32_t bar = 0;
+  for (int l = 0; l < p.L; ++l) {
+    const LwArgs &a = p.l[l];
+    if (blockIdx.x == 0) lw_alloc_body<true>(a, lw_dyn);
+    grid_barrier<LWT>(p.hdr, bar);
+    lw_sample_remote_body<true>(a);
+    grid_barrier<LWT>(p.hdr, bar);
+    lw_sample_big_body<true>(a, p.kp_max, reinterpret_cast<int32_t *>(lw_dyn));
+    grid_barrier<LWT>(p.hdr, bar);
+    if (blockIdx.x == 0 && threadIdx.x == 0) p.hdr->lw_big = 0u;
+    lw_collect_body<true>(a);
+    grid_barrier<LWT>(p.hdr, bar);
+    if (blockIdx.x == 0) lw_finish_body(a);
+    grid_barrier<LWT>(p.hdr, bar);
   }
 }
 

@@ -181,6 +181,7 @@ struct dsp_ctx {
   int loader_rows = 32;  // DSP_LOADER_ROWS: rows per TMA chunk, <= 32 (tuning knob, results unchanged)
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
   bool multi_staged = false;  // DSP_MULTI_STAGED=1: world > 1 node-wise calls stage by stage (A/B switch)
+  bool lw_staged = false;     // DSP_LW_STAGED=1: world-1 layer-wise calls stage by stage (A/B switch)
   cudaStream_t aux = nullptr;  // virtual ranks sharing a GPU: each rank's persistent launch on its own stream
   cudaEvent_t aux_ev[2] = {nullptr, nullptr};
   int gather_blocks_per_sm = 1;
@@ -978,6 +979,22 @@ LwArgs lw_args(Call &k, int l) {
   return a;
 }
 
+// world 1, layer-wise: every layer in one cooperative launch (k_lw_persistent)
+dsp_status stage_lw_persistent(Call &k) {
+  dsp_ctx *c = k.c;
+  DeviceGuard g(c->device);
+  LwPersistArgs p{};
+  for (int l = 0; l < k.L; ++l) p.l[l] = lw_args(k, l);
+  p.L = k.L;
+  p.kp_max = (int)next_pow2(k.plan.ncap);
+  p.hdr = k.hdr;
+  const size_t smem = std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)p.kp_max);
+  const dim3 grid(std::min(c->num_sms, 64)), block(LWT);
+  void *args[] = {&p};
+  CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_lw_persistent, grid, block, args, smem, k.stream));
+  return DSP_OK;
+}
+
 dsp_status stage_lw(Call &k, int l, int step) {
   dsp_ctx *c = k.c;
   DeviceGuard g(c->device);
@@ -1086,7 +1103,9 @@ dsp_status run_calls(std::vector<Call> &calls) {
     for (size_t i = 0; i < calls.size(); ++i)
       if ((st = join_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
   } else {
-    for (int l = 0; l < calls[0].L; ++l) {
+    const bool lw_pers = calls[0].layerwise && calls[0].c->world == 1 && !calls[0].c->lw_staged;
+    if (lw_pers) EACH(stage_lw_persistent(k));
+    for (int l = 0; l < (lw_pers ? 0 : calls[0].L); ++l) {
       if (calls[0].layerwise) {
         for (int step = 0; step < 5; ++step) EACH(stage_lw(k, l, step));
         continue;
@@ -1351,6 +1370,8 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   }
   if (cudaFuncSetAttribute((const void *)k_lw_sample_big, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            (int)sizeof(int32_t) * 3 * LW_MAX_SIZE) != cudaSuccess ||
+      cudaFuncSetAttribute((const void *)k_lw_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           (int)std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)LW_MAX_SIZE)) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_lw_alloc, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            (int)LW_ALLOC_SMEM) != cudaSuccess) {
     cudaGetLastError();
@@ -1361,6 +1382,7 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   if (getenv("DSP_LANE_ROUNDS")) c->lane_rounds = atoi(getenv("DSP_LANE_ROUNDS"));
   if (getenv("DSP_STAGE_BPS")) c->stage_bps = std::max(1, std::min(8, atoi(getenv("DSP_STAGE_BPS"))));
   c->multi_staged = getenv("DSP_MULTI_STAGED") && atoi(getenv("DSP_MULTI_STAGED")) != 0;
+  c->lw_staged = getenv("DSP_LW_STAGED") && atoi(getenv("DSP_LW_STAGED")) != 0;
   if (const char *rm = getenv("DSP_RELABEL"))
     c->relabel_mode = !strcmp(rm, "hash") ? 2 : !strcmp(rm, "direct") ? 1 : !strcmp(rm, "direct64") ? 3 : 0;
   if (getenv("DSP_LOADER_ROWS")) c->loader_rows = std::max(1, std::min(32, atoi(getenv("DSP_LOADER_ROWS"))));

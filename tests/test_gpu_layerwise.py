@@ -53,8 +53,17 @@ def _big_tasks(ip, seeds, n):
     return int(((c > 40) & (c < d * 0.9)).sum())
 
 
+@pytest.fixture(params=["persistent", "staged"])
+def lw_mode(request, monkeypatch):
+    """world 1: all layers in one cooperative launch (default) or one launch per
+    stage (DSP_LW_STAGED=1, read by dsp_create)."""
+    if request.param == "staged":
+        monkeypatch.setenv("DSP_LW_STAGED", "1")
+    return request.param
+
+
 @pytest.mark.parametrize("sizes", [(200, 300), (1000, 1000), (1,), (8192,), (50, 50, 50), (3, 4000)])
-def test_layerwise_tiny_p1(pkg, tiny, sizes):
+def test_layerwise_tiny_p1(pkg, tiny, sizes, lw_mode):
     cfg, ip, ix, feats = tiny
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, sizes, 64, scheme="layer")
     rng = np.random.default_rng(len(sizes) * 7 + sizes[0])
@@ -65,7 +74,7 @@ def test_layerwise_tiny_p1(pkg, tiny, sizes):
     s.close()
 
 
-def test_layerwise_big_tasks_exercised(pkg, tiny):
+def test_layerwise_big_tasks_exercised(pkg, tiny, lw_mode):
     """n = 1000 over 64 seeds: hub seeds get 32 < c < deg draws."""
     cfg, ip, ix, feats = tiny
     deg = np.diff(ip)
@@ -109,7 +118,7 @@ def test_layerwise_virtual_ranks(pkg, tiny, P):
     grp.close()
 
 
-def test_layerwise_fused_and_pipelined(pkg, tiny):
+def test_layerwise_fused_and_pipelined(pkg, tiny, lw_mode):
     cfg, ip, ix, feats = tiny
     sizes = (400, 800)
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, sizes, 64, n_slots=2, scheme="layer")
@@ -136,7 +145,7 @@ def test_layerwise_fused_and_pipelined(pkg, tiny):
     s.close()
 
 
-def test_layerwise_errors(pkg, tiny):
+def test_layerwise_errors(pkg, tiny, lw_mode):
     cfg, ip, ix, feats = tiny
     bn = datagen.bounds(cfg.num_nodes, 1)
     with pytest.raises(pkg.DSPError) as e:
