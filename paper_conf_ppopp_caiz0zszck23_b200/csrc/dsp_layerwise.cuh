@@ -486,14 +486,25 @@ struct LwPersistArgs {
   int32_t L;
   int32_t kp_max;
   WsHeader *hdr;
+  WsPersist *persist;       // epoch advanced by the last block
+  int32_t gather;           // gather this call's last block (fused call)
+  GatherArgs g;
+  int32_t prev;             // pipelined: gather the previous call's rows (blocks >= 1, during allocation 0)
+  GatherArgs gp;
+  int32_t *pend_n;          // pipelined: where this call's row count goes
 };
 
 __global__ void __launch_bounds__(LWT, 1) k_lw_persistent(LwPersistArgs p) {
   extern __shared__ unsigned long long lw_dyn[];
   uint32_t bar = 0;
+  if (blockIdx.x == 0 && threadIdx.x == 0) p.hdr->t[0] = globaltimer_ns();
   for (int l = 0; l < p.L; ++l) {
     const LwArgs &a = p.l[l];
-    if (blockIdx.x == 0) lw_alloc_body<true>(a, lw_dyn);
+    if (blockIdx.x == 0)
+      lw_alloc_body<true>(a, lw_dyn);
+    else if (l == 0 && p.prev)  // the other blocks gather the previous pipelined call's rows meanwhile
+      phase_gather<GATHER_UNROLL>(p.gp, ld_volatile_i32(p.gp.n_dev), (blockIdx.x - 1) * (int64_t)LWT + threadIdx.x,
+                                  (gridDim.x - 1) * (int64_t)LWT);
     grid_barrier<LWT>(p.hdr, bar);
     lw_sample_remote_body<true>(a);
     grid_barrier<LWT>(p.hdr, bar);
@@ -504,6 +515,19 @@ __global__ void __launch_bounds__(LWT, 1) k_lw_persistent(LwPersistArgs p) {
     grid_barrier<LWT>(p.hdr, bar);
     if (blockIdx.x == 0) lw_finish_body(a);
     grid_barrier<LWT>(p.hdr, bar);
+  }
+  const int32_t S = ld_volatile_i32(&p.hdr->S[p.L - 1]);
+  if (p.prev && gridDim.x == 1)  // no spare block during allocation 0
+    phase_gather<GATHER_UNROLL>(p.gp, ld_volatile_i32(p.gp.n_dev), threadIdx.x, LWT);
+  if (p.gather) phase_gather<GATHER_UNROLL>(p.g, S, blockIdx.x * (int64_t)LWT + threadIdx.x, gridDim.x * (int64_t)LWT);
+  if (p.pend_n && blockIdx.x == 0 && threadIdx.x == 0) *p.pend_n = S;
+  __syncthreads();
+  if (threadIdx.x == 0) {  // the last block advances the workspace epoch (k_epoch_advance of the staged path)
+    __threadfence();
+    if (atomicAdd(&p.hdr->done, 1u) == gridDim.x - 1) {
+      p.persist->epoch += (uint32_t)p.L;
+      p.hdr->done = 0u;
+    }
   }
 }
 

@@ -988,10 +988,29 @@ dsp_status stage_lw_persistent(Call &k) {
   p.L = k.L;
   p.kp_max = (int)next_pow2(k.plan.ncap);
   p.hdr = k.hdr;
+  p.persist = persist_of(k);
+  p.gather = k.feat_out != nullptr && !k.pipelined;
+  if (p.gather) p.g = make_gather(c, k.blocks[k.L - 1].src_ids, 0, nullptr, k.feat_out);
+  dsp_ctx::Pending *pd = nullptr;
+  if (k.feat_out && k.pipelined) {  // the previous call's rows are gathered during this call's first allocation
+    pd = c->pending_of(k.ws);
+    if (!pd) return fail(c, DSP_ERR_STATE, "more than 8 workspaces with pending pipelined gathers");
+    WsPersist *ps = persist_of(k);
+    p.prev = pd->active ? 1 : 0;
+    if (p.prev) p.gp = make_gather(c, pd->ids, 0, &ps->pend_n[(pd->calls + 1) & 1], pd->out);
+    p.pend_n = &ps->pend_n[pd->calls & 1];
+  }
   const size_t smem = std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)p.kp_max);
   const dim3 grid(std::min(c->num_sms, 64)), block(LWT);
   void *args[] = {&p};
   CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_lw_persistent, grid, block, args, smem, k.stream));
+  if (pd) {
+    pd->ids = k.blocks[k.L - 1].src_ids;
+    pd->out = k.feat_out;
+    pd->stream = k.stream;
+    pd->active = true;
+    pd->calls += 1;
+  }
   return DSP_OK;
 }
 
@@ -1088,8 +1107,10 @@ dsp_status run_calls(std::vector<Call> &calls) {
   // a non-pipelined call first settles a pending pipelined gather; so does a
   // pipelined call of the stage-by-stage paths (no loader warps there)
   const bool multi = calls[0].c->world > 1 && !calls[0].layerwise && !calls[0].c->multi_staged;
+  const bool lw_pers = calls[0].layerwise && calls[0].c->world == 1 && !calls[0].c->lw_staged;
   for (auto &k : calls)
-    if ((!k.pipelined || (k.c->world > 1 && !multi) || k.layerwise) && (st = stage_flush(k.c, k.ws)) != DSP_OK)
+    if ((!k.pipelined || (k.c->world > 1 && !multi) || (k.layerwise && !lw_pers)) &&
+        (st = stage_flush(k.c, k.ws)) != DSP_OK)
       return st;
   EACH(stage_begin(k));
   if (calls[0].c->world == 1 && !calls[0].layerwise) {
@@ -1102,10 +1123,10 @@ dsp_status run_calls(std::vector<Call> &calls) {
       if ((st = stage_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
     for (size_t i = 0; i < calls.size(); ++i)
       if ((st = join_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
+  } else if (lw_pers) {  // gather (fused, or the previous call's when pipelined) and epoch inside
+    EACH(stage_lw_persistent(k));
   } else {
-    const bool lw_pers = calls[0].layerwise && calls[0].c->world == 1 && !calls[0].c->lw_staged;
-    if (lw_pers) EACH(stage_lw_persistent(k));
-    for (int l = 0; l < (lw_pers ? 0 : calls[0].L); ++l) {
+    for (int l = 0; l < calls[0].L; ++l) {
       if (calls[0].layerwise) {
         for (int step = 0; step < 5; ++step) EACH(stage_lw(k, l, step));
         continue;
