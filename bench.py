@@ -667,8 +667,9 @@ def run_dsp(args):
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(args, cfg, ip, ix, feats, batches, args.cpu_seconds, weights=ew)
 
-    kern_per_step = 5 * L + 1 if layer else 1
-    roof_kernel = "k_gather" if layer else ("k_csp_persistent" if world == 1 else "k_csp_multi")
+    kern_per_step = (1 if world == 1 else 5 * L + 1) if layer else 1
+    roof_kernel = (("k_lw_persistent" if world == 1 else "k_gather") if layer
+                   else ("k_csp_persistent" if world == 1 else "k_csp_multi"))
     roofline = {"kernel": roof_kernel,
                 "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak,
