@@ -94,6 +94,24 @@ def test_fanout_range_and_ragged_batches(pkg, tiny, fanouts):
     s.close()
 
 
+@pytest.mark.parametrize("relabel", ["direct", "direct64", "hash"])
+def test_maximum_layers_and_fanout(pkg, tiny, relabel, monkeypatch):
+    """The ABI's limits: 8 layers of fan-out 32 (the frontier saturates at all
+    N nodes, every row of degree <= 32 is taken whole), on each relabel layout;
+    fused gather of the last block (every node) and a pipelined call."""
+    monkeypatch.setenv("DSP_RELABEL", relabel)
+    cfg, ip, ix, feats = tiny
+    fan = (32,) * 8
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, fan, 64, n_slots=2)
+    seeds = np.random.default_rng(8).choice(cfg.num_nodes, size=64, replace=False).astype(np.int32)
+    blocks, feat = s.sample_gather(torch.from_numpy(seeds).cuda(), 77, slot=0)
+    ref = oracle.sample(ip, ix, seeds, fan, 77)
+    assert_blocks_equal(blocks, ref, f"max {relabel}")
+    assert blocks[-1].num_src == len(np.unique(ref[-1]["src_ids"]))
+    assert np.array_equal(feat.cpu().numpy().view(np.uint32), oracle.gather(feats, ref[-1]["src_ids"]).view(np.uint32))
+    s.close()
+
+
 def test_empty_batch(pkg, tiny):
     cfg, ip, ix, feats = tiny
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8)
