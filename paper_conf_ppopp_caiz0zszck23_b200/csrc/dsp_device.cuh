@@ -387,16 +387,18 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
     }
     uint32_t pick = 0xffffffffu;
     const unsigned long long myword = lane < k ? biased_word(key, lane, v, layer) : 0ull;  // all draws at once
-    for (int t = 0; t < k; ++t) {
-      unsigned long long tot = 0;
+    // lane totals, their inclusive scan and the remaining weight W, scanned once and
+    // then updated in place: removing weight w at lane L lowers incl of lanes >= L by w
+    unsigned long long tot = 0;
 #pragma unroll
-      for (int j = 0; j < BSEG; ++j) tot += reg[j];
-      const unsigned long long incl = warp_incl_scan_u64(tot);
-      const unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
+    for (int j = 0; j < BSEG; ++j) tot += reg[j];
+    unsigned long long incl = warp_incl_scan_u64(tot);
+    unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
+    for (int t = 0; t < k; ++t) {
       const unsigned long long r = __umul64hi(__shfl_sync(FULL_MASK, myword, t), W);
       const uint32_t cross = __ballot_sync(FULL_MASK, incl > r);
       const int L = __ffs(cross) - 1;
-      uint32_t found = 0;
+      uint32_t found = 0, wrem = 0;
       if (lane == L) {
         unsigned long long acc = incl - tot;
         bool done = false;
@@ -404,13 +406,18 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
         for (int j = 0; j < BSEG; ++j) {
           if (!done && acc + reg[j] > r) {
             found = (uint32_t)(lane * S + j);
+            wrem = reg[j];
             reg[j] = 0u;  // remove the pick
             done = true;
           }
           acc += reg[j];
         }
+        tot -= wrem;
       }
       found = __shfl_sync(FULL_MASK, found, L);
+      wrem = __shfl_sync(FULL_MASK, wrem, L);
+      if (lane >= L) incl -= wrem;
+      W -= wrem;
       if (lane == t) pick = found;
     }
     *pos = biased_sort_picks(pick, k);
@@ -452,12 +459,12 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
     }
     uint32_t pick = 0xffffffffu;
     const unsigned long long myword = lane < k ? biased_word(key, lane, v, layer) : 0ull;  // all draws at once
-    for (int t = 0; t < k; ++t) {
-      unsigned long long tot = 0;
+    unsigned long long tot = 0;  // scanned once, then updated in place (as above)
 #pragma unroll
-      for (int j = 0; j < BSEG; ++j) tot += cs[j];
-      const unsigned long long incl = warp_incl_scan_u64(tot);
-      const unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
+    for (int j = 0; j < BSEG; ++j) tot += cs[j];
+    unsigned long long incl = warp_incl_scan_u64(tot);
+    unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
+    for (int t = 0; t < k; ++t) {
       const unsigned long long r = __umul64hi(__shfl_sync(FULL_MASK, myword, t), W);
       const int L = __ffs(__ballot_sync(FULL_MASK, incl > r)) - 1;
       int cstar = 0;
@@ -489,7 +496,10 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
 #pragma unroll
         for (int j = 0; j < BSEG; ++j)
           if (j == cstar - lane * T) cs[j] -= wfound;  // remove the pick
+        tot -= wfound;
       }
+      if (lane >= L) incl -= wfound;
+      W -= wfound;
       if (lane == t) pick = found;
     }
     *pos = biased_sort_picks(pick, k);

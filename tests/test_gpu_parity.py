@@ -493,6 +493,58 @@ def test_biased_virtual_ranks(pkg, tiny, tiny_weights, P):
     grp.close()
 
 
+def _long_row_graph():
+    """30k nodes, rows of degree <= 40 plus hubs of degree 300 / 1000 / 5000
+    (chunk-sum path, 256 < d <= 8192), 9000 / 20000 (very long rows), and a hub
+    whose 5000 weights are all zero but 3 (every positive one taken, no draw)."""
+    rng = np.random.default_rng(31)
+    N = 30000
+    degs = rng.integers(0, 41, size=N)
+    hubs = {0: 300, 1: 1000, 2: 5000, 3: 9000, 4: 20000, 5: 5000}
+    for h, d in hubs.items():
+        degs[h] = d
+    rows = []
+    for v in range(N):
+        nb = rng.choice(N - 1, size=int(degs[v]), replace=False)
+        nb[nb >= v] += 1   # no self loop
+        rows.append(np.sort(nb))
+    ip = np.zeros(N + 1, np.int64)
+    ip[1:] = np.cumsum([len(r) for r in rows])
+    ix = np.concatenate(rows).astype(np.int32)
+    w = (rng.integers(0, 5000, size=len(ix)) / 7.0).astype(np.float32)
+    w[rng.random(len(ix)) < 0.1] = 0.0
+    w[ip[5]:ip[6]] = 0.0
+    w[ip[5] + np.array([7, 2000, 4999])] = 3.5
+    return N, ip, ix, w
+
+
+def test_biased_long_rows(pkg):
+    """Biased sampling on every row-length path of the warp sampler (registers,
+    chunk sums, very long rows, <= k positive weights) at P = 1 and at virtual
+    P = 2 (the owner-side sampler of the multi-rank kernel)."""
+    N, ip, ix, w = _long_row_graph()
+    feats = datagen.features(0, N, 4)
+    fan = (15, 10)
+    seeds = np.array([0, 1, 2, 3, 4, 5, 11, 29999, 15000], np.int32)
+    s = pkg.Sampler(datagen.bounds(N, 1), ip, ix, feats, fan, 16, edge_weights=w)
+    for rng in (1, 2, 3):
+        blocks = s.sample(torch.from_numpy(seeds).cuda(), rng, biased=True)
+        assert_blocks_equal(blocks, oracle.sample(ip, ix, seeds, fan, rng, weights=w), f"long rows rng {rng}")
+    s.close()
+    bnds = datagen.bounds(N, 2)
+    shards = []
+    for r in range(2):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi], w[ip[lo]:ip[hi]]))
+    grp = pkg.LocalGroup(bnds, shards, fan, 16, devices=[0, 0])
+    rs = [seeds[:6], seeds[6:]]
+    res = grp.sample([torch.from_numpy(np.ascontiguousarray(x)).cuda() for x in rs], 9, biased=True)
+    for r in range(2):
+        assert_blocks_equal(res[r], oracle.sample(ip, ix, rs[r], fan, 9, weights=w), f"long rows P=2 rank {r}")
+    grp.close()
+
+
 def test_biased_errors(pkg, tiny):
     cfg, ip, ix, feats = tiny
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8)
