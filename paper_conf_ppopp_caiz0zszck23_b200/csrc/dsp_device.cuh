@@ -318,14 +318,18 @@ __device__ __forceinline__ unsigned long long warp_incl_scan_u64(unsigned long l
 // weights and test membership against the picks so far.
 constexpr int BSEG = 8;
 
+// Lanes t < k hold distinct picks; lane r returns the pick of rank r (ascending):
+// each lane ranks its own pick with k shuffles, then one ballot + shuffle per
+// rank moves it to its lane (3k warp ops instead of k^2).
 __device__ __forceinline__ uint32_t biased_sort_picks(uint32_t pick, int k) {
   const int lane = threadIdx.x & 31;
+  int rank = 0;
+  for (int j = 0; j < k; ++j) rank += __shfl_sync(FULL_MASK, pick, j) < pick ? 1 : 0;
   uint32_t mine = 0xffffffffu;
-  for (int s2 = 0; s2 < k; ++s2) {
-    const uint32_t c = __shfl_sync(FULL_MASK, pick, s2);
-    int rank = 0;
-    for (int j = 0; j < k; ++j) rank += __shfl_sync(FULL_MASK, pick, j) < c ? 1 : 0;
-    if (rank == lane) mine = c;
+  for (int r = 0; r < k; ++r) {
+    const uint32_t b = __ballot_sync(FULL_MASK, lane < k && rank == r);
+    const uint32_t v = __shfl_sync(FULL_MASK, pick, __ffs(b) - 1);
+    if (lane == r) mine = v;
   }
   return mine;
 }
