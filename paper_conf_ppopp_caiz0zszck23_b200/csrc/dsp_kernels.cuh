@@ -557,30 +557,39 @@ __device__ __forceinline__ void phase_sample_biased(const int32_t *frontier, int
   const Span sp = block_span<TEAM>(F);
   const int64_t b0 = sp.first - threadIdx.x;
   const int wib = threadIdx.x >> 5, wpb = TEAM >> 5;
-  for (int64_t i64 = b0 + wib; i64 < sp.end; i64 += wpb) {
-    const int i = (int)i64;
-    const int32_t v = ldw_i32(frontier + i);
-    const int64_t lv = (int64_t)v - lo;
-    const bool ok = v >= 0 && lv >= 0 && lv < n_local;
-    int64_t s = 0, d = 0;
-    if (ok) {
-      row_extent(indptr, lv, &s, &d);
-    }
-    uint32_t pos;
-    const int cnt = sample_node_biased(ok, v, s, d, k, layer, key, weights, &pos);
-    if (lane == 0) {
-      B.cnt[i] = cnt;
-      if (src_out) src_out[i] = v;
-      if (ok)
-        mark_dst(B, v, i, F, layer, epoch, err);
-      else
-        latch(err, E_RANGE);
-    }
-    if (lane < cnt) {
-      const int32_t u = __ldg(indices + s + pos);
-      const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)lane;
-      B.rows[q] = u;
-      mark(B, u, epoch, (uint32_t)F + q);
+  // The warp's next 32 nodes (its strided share) have their ids and row extents
+  // loaded at once, one per lane, then are sampled one after the other: one
+  // dependent DRAM round trip per 32 nodes instead of one per node.
+  for (int64_t g0 = b0 + wib; g0 < sp.end; g0 += (int64_t)wpb * 32) {
+    const int64_t il = g0 + (int64_t)lane * wpb;
+    const int32_t vl = il < sp.end ? ldw_i32(frontier + il) : -1;
+    const int64_t lvl = (int64_t)vl - lo;
+    const bool okl = il < sp.end && vl >= 0 && lvl >= 0 && lvl < n_local;
+    int64_t sl = 0, dl = 0;
+    if (okl) row_extent(indptr, lvl, &sl, &dl);
+    const int nn = (int)min((int64_t)32, (sp.end - g0 + wpb - 1) / wpb);
+    for (int j = 0; j < nn; ++j) {
+      const int i = (int)(g0 + (int64_t)j * wpb);
+      const int32_t v = __shfl_sync(FULL_MASK, vl, j);
+      const bool ok = __shfl_sync(FULL_MASK, okl, j);
+      const int64_t s = __shfl_sync(FULL_MASK, sl, j);
+      const int64_t d = __shfl_sync(FULL_MASK, dl, j);
+      uint32_t pos;
+      const int cnt = sample_node_biased(ok, v, s, d, k, layer, key, weights, &pos);
+      if (lane == 0) {
+        B.cnt[i] = cnt;
+        if (src_out) src_out[i] = v;
+        if (ok)
+          mark_dst(B, v, i, F, layer, epoch, err);
+        else
+          latch(err, E_RANGE);
+      }
+      if (lane < cnt) {
+        const int32_t u = __ldg(indices + s + pos);
+        const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)lane;
+        B.rows[q] = u;
+        mark(B, u, epoch, (uint32_t)F + q);
+      }
     }
   }
 }
