@@ -410,8 +410,8 @@ def run_dsp(args):
     ew = datagen.edge_weights(six, datagen.node_weights(cfg.num_nodes)) if biased else None
     layer = args.scheme == "layer"
     fanouts = fanouts_of(args, cfg)
-    # concurrent instances share the ctx's exchange region on the staged paths: one stream there
-    K = max(1, args.instances) if world == 1 and not layer else 1
+    # K concurrent step streams at world 1 (world > 1: one stream, the ranks' exchange slots are per ctx)
+    K = max(1, args.instances) if world == 1 else 1
     s = pkg.Sampler(bnds, sip, six, feats, fanouts, cfg.batch, rank=rank, world_size=world, scheme="layer" if layer else "node",
                     device=local, exchange=ex, n_slots=2 * K, edge_weights=ew, n_workspaces=K,
                     hot_rows=None if args.hot_frac is None else int(round(args.hot_frac * (len(sip) - 1))))
@@ -657,7 +657,7 @@ def run_dsp(args):
 
     if K > 1:   # the asynchronous e2e runs the timed step's configuration: K streams x 1/K of the SMs
         pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(local).multi_processor_count // K)
-    e2e_av, e2e_ah2d, e2e_ad2h, e2e_an = e2e_async_run() if not layer else (None, 0, 0, 0)
+    e2e_av, e2e_ah2d, e2e_ad2h, e2e_an = e2e_async_run()
     if K > 1:   # one synchronous call at a time: the whole GPU
         pkg.dsp_set_persistent_blocks(s.ctx, 0)
     e2e_v, e2e_h2d, e2e_d2h = e2e_run(False)

@@ -115,6 +115,7 @@ struct Plan {
   // layer-wise scheme (make_plan_lw)
   int64_t ncap, big_cap;
   size_t off_P, off_c, off_off, off_slot_node, off_excl, off_newid, off_big;
+  size_t off_lxch;                  // world 1: the layer-wise inbox / return slots in the workspace (else 0)
 };
 
 }  // namespace
@@ -335,7 +336,11 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L, int 
 }
 
 // Layer-wise (R28): E_l <= n_l, max_src[l] = min(N, F_l + n_l).
-Plan make_plan_lw(int64_t N, int64_t num_seeds, const int32_t *sizes, int L) {
+LwLayout make_lw_layout(int64_t cap, int32_t ncap);
+
+// own_xch (world 1): the inbox / return slots live in the workspace, so calls
+// on different workspaces can run concurrently (no flags: k_lw_persistent)
+Plan make_plan_lw(int64_t N, int64_t num_seeds, const int32_t *sizes, int L, bool own_xch) {
   Plan p{};
   p.L = L;
   p.F[0] = num_seeds;
@@ -361,6 +366,8 @@ Plan make_plan_lw(int64_t N, int64_t num_seeds, const int32_t *sizes, int L) {
   take(p.off_excl, sizeof(int32_t) * (size_t)(p.ncap + 1));
   take(p.off_newid, sizeof(int32_t) * (size_t)p.ncap);
   take(p.off_big, sizeof(int2) * (size_t)p.big_cap);
+  p.off_lxch = 0;
+  if (own_xch) take(p.off_lxch, make_lw_layout(std::max<int64_t>(1, p.max_F), (int32_t)p.ncap).bytes);
   p.bytes = o;
   return p;
 }
@@ -544,7 +551,7 @@ dsp_status prepare_call_lw(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t nu
   for (int l = 0; l < L; ++l)
     if (sizes[l] != c->lw_sizes[l])
       return fail(c, DSP_ERR_STATE, "layer size %d = %d != reserved %d", l, sizes[l], c->lw_sizes[l]);
-  k.plan = make_plan_lw(c->N, c->lw_max_seeds, sizes, L);
+  k.plan = make_plan_lw(c->N, c->lw_max_seeds, sizes, L, c->world == 1);
   if (ws_bytes < k.plan.bytes)
     return fail(c, DSP_ERR_CAPACITY, "workspace %zu B < required %zu B", ws_bytes, k.plan.bytes);
   if (((uintptr_t)workspace & 255u) != 0) return fail(c, DSP_ERR_INVALID_ARG, "workspace must be 256-byte aligned");
@@ -976,6 +983,8 @@ LwArgs lw_args(Call &k, int l) {
   a.hdr = k.hdr;
   a.err = c->d_err;
   a.sys = c->world > 1 ? 1 : 0;
+  if (c->world == 1 && !c->lw_staged && k.plan.off_lxch)  // persistent world-1 call: its own exchange slots
+    a.peers.base[0] = k.ws + k.plan.off_lxch;
   return a;
 }
 
@@ -1001,7 +1010,7 @@ dsp_status stage_lw_persistent(Call &k) {
     p.pend_n = &ps->pend_n[pd->calls & 1];
   }
   const size_t smem = std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)p.kp_max);
-  const dim3 grid(std::min(c->num_sms, 64)), block(LWT);
+  const dim3 grid(std::min(c->persist_blocks > 0 ? c->persist_blocks : c->num_sms, 64)), block(LWT);
   void *args[] = {&p};
   CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_lw_persistent, grid, block, args, smem, k.stream));
   if (pd) {
@@ -1647,7 +1656,7 @@ dsp_status dsp_reserve_layerwise(dsp_ctx *c, int32_t max_seeds, const int32_t *s
   dsp_status st = check_sizes(c, sizes, L);
   if (st != DSP_OK) return st;
   if (max_seeds < 0) return fail(c, DSP_ERR_INVALID_ARG, "max_seeds < 0");
-  Plan p = make_plan_lw(c->N, max_seeds, sizes, L);
+  Plan p = make_plan_lw(c->N, max_seeds, sizes, L, c->world == 1);
   for (int l = 0; l < L; ++l)
     if ((uint64_t)p.F[l] + (uint64_t)p.E[l] >= (1ull << 31))
       return fail(c, DSP_ERR_CAPACITY, "layer %d: frontier + layer size exceeds 2^31", l);
@@ -1676,7 +1685,7 @@ dsp_status dsp_sample_bounds_layerwise(const dsp_ctx *cc, int32_t num_seeds, con
   if (num_seeds < 0) return fail(c, DSP_ERR_INVALID_ARG, "num_seeds < 0");
   if (c->lw_reserved && num_seeds > c->lw_max_seeds)
     return fail(c, DSP_ERR_CAPACITY, "num_seeds %d > reserved max_seeds %d", num_seeds, c->lw_max_seeds);
-  Plan p = make_plan_lw(c->N, c->lw_reserved ? c->lw_max_seeds : num_seeds, sizes, L);
+  Plan p = make_plan_lw(c->N, c->lw_reserved ? c->lw_max_seeds : num_seeds, sizes, L, c->world == 1);
   for (int l = 0; l < L; ++l) {
     if (max_src) max_src[l] = p.S[l];
     if (max_edges) max_edges[l] = p.E[l];

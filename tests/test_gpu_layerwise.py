@@ -145,6 +145,43 @@ def test_layerwise_fused_and_pipelined(pkg, tiny, lw_mode):
     s.close()
 
 
+def test_layerwise_concurrent_streams(pkg, tiny):
+    """world 1: pipelined layer-wise calls on 3 workspaces / streams at once
+    (each persistent call keeps its exchange slots in its own workspace)."""
+    cfg, ip, ix, feats = tiny
+    sizes = (300, 500)
+    K = 3
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, sizes, 64, scheme="layer", n_slots=2 * K,
+                    n_workspaces=K)
+    pkg.dsp_set_persistent_blocks(s.ctx, 16)
+    rng = np.random.default_rng(3)
+    n = 9
+    seeds = [rng.choice(cfg.num_nodes, size=64, replace=False).astype(np.int32) for _ in range(n)]
+    dev = [torch.from_numpy(x).cuda() for x in seeds]
+    L = len(sizes)
+    hs = torch.zeros((n, 3 * L), dtype=torch.int64).pin_memory()
+    main = torch.cuda.current_stream()
+    streams = [torch.cuda.Stream() for _ in range(K)]
+    for st in streams:
+        st.wait_stream(main)
+    for i in range(n):
+        s.sample_gather(dev[i], 40 + i, slot=i % (2 * K), sizes_out=hs[i], async_=True, pipelined=True, ws=i % K,
+                        stream=streams[i % K])
+    for st in streams:
+        with torch.cuda.stream(st):
+            s.flush()
+    for st in streams:
+        main.wait_stream(st)
+    torch.cuda.synchronize()
+    for i in range(n - 2 * K, n):
+        ref = oracle.sample_layerwise(ip, ix, seeds[i], sizes, 40 + i)
+        blocks = s.blocks(i % (2 * K), sizes=[int(x) for x in hs[i]])
+        assert_blocks_equal(blocks, ref, f"concurrent {i}")
+        feat = s.feat_buffer(i % (2 * K))[: blocks[-1].num_src]
+        assert np.array_equal(feat.cpu().numpy().view(np.uint32), oracle.gather(feats, ref[-1]["src_ids"]).view(np.uint32))
+    s.close()
+
+
 def test_layerwise_errors(pkg, tiny, lw_mode):
     cfg, ip, ix, feats = tiny
     bn = datagen.bounds(cfg.num_nodes, 1)
