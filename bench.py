@@ -317,12 +317,22 @@ def run_walk(args):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     for e in (ev0, ev1):
         e.record(stream)
-    outs = [torch.empty((nw, length + 1), dtype=torch.int32, device="cuda") for _ in range(2)]  # allocated up front
+    # world 1: K walk calls in flight on K streams (each walk is a chain of dependent random
+    # reads, so more independent walks in flight = more throughput); world > 1: one stream
+    # (the walkers move through the ctx's exchange region)
+    K = max(1, args.instances) if world == 1 else 1
+    streams = [torch.cuda.Stream() for _ in range(K)] if K > 1 else [stream]
+    outs = [torch.empty((nw, length + 1), dtype=torch.int32, device="cuda") for _ in range(max(2, K))]  # up front
     torch.cuda.synchronize()
     with ClockSampler(local) as clk:
         ev0.record(stream)
+        for st in streams:
+            st.wait_stream(stream)
         for j in range(KS):
-            s.random_walk(starts[j % 4], length, datagen.BASE_SEED + W + j, out=outs[j % 2])
+            with torch.cuda.stream(streams[j % K]):
+                s.random_walk(starts[j % 4], length, datagen.BASE_SEED + W + j, out=outs[j % max(2, K)])
+        for st in streams:
+            stream.wait_stream(st)
         ev1.record(stream)
         s.sync()
         torch.cuda.synchronize()
@@ -367,7 +377,8 @@ def run_walk(args):
                        "walkers_per_gpu": nw, "walk_length": length, "num_nodes": cfg.num_nodes,
                        "nnz": int(ip[-1]), "parallelism": f"csp{world}",
                        "starts": "uniform over each rank's own node range, 4 fixed sets",
-                       "step": "dsp_random_walk (thread per walk at world 1; CSP push without reshuffle at world > 1)"},
+                       "step": "dsp_random_walk (thread per walk at world 1; CSP push without reshuffle at world > 1)"
+                               + (f", {K} streams" if K > 1 else "")},
             "roofline": {"kernel": "k_random_walk" if world == 1 else "k_walk_step", "bound": "hbm",
                          "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                          "traffic": None, "peak_kind": peak_kind,
