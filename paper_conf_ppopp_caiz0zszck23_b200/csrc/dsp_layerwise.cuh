@@ -531,4 +531,43 @@ __global__ void __launch_bounds__(LWT, 1) k_lw_persistent(LwPersistArgs p) {
   }
 }
 
+// World > 1: every layer of the call in ONE cooperative launch per rank; the
+// phases keep the flag protocol of the per-stage kernels (the requests and the
+// sampled rows cross GPUs through the peer-mapped exchange region), with grid
+// barriers where a stage used to end at a kernel boundary.  Every rank's kernel
+// is resident on its own GPU (virtual ranks: 1/P of the SMs each), so waiting
+// on a peer's flag inside the kernel is safe; waits are bounded (wait_flags).
+__global__ void __launch_bounds__(LWT, 1) k_lw_multi(LwPersistArgs p) {
+  extern __shared__ unsigned long long lw_dyn[];
+  uint32_t bar = 0;
+  if (blockIdx.x == 0 && threadIdx.x == 0) p.hdr->t[0] = globaltimer_ns();
+  for (int l = 0; l < p.L; ++l) {
+    const LwArgs &a = p.l[l];
+    if (blockIdx.x == 0)  // Eq. 2 allocation, tasks pushed to the owners + inbox flags
+      lw_alloc_body<false>(a, lw_dyn);
+    else if (l == 0 && p.prev)  // meanwhile the other blocks gather the previous pipelined call's rows
+      phase_gather<GATHER_UNROLL>(p.gp, ld_volatile_i32(p.gp.n_dev), (blockIdx.x - 1) * (int64_t)LWT + threadIdx.x,
+                                  (gridDim.x - 1) * (int64_t)LWT);
+    lw_sample_remote_body<false>(a);  // waits for every rank's tasks
+    grid_barrier<LWT>(p.hdr, bar);    // every task with c > 32 queued
+    lw_sample_big_body<false>(a, p.kp_max, reinterpret_cast<int32_t *>(lw_dyn));  // then the return flags
+    lw_collect_body<false>(a);        // waits for every owner's rows
+    grid_barrier<LWT>(p.hdr, bar);
+    if (blockIdx.x == 0) lw_finish_body(a);
+    grid_barrier<LWT>(p.hdr, bar);
+  }
+  const int32_t S = ld_volatile_i32(&p.hdr->S[p.L - 1]);
+  if (p.prev && gridDim.x == 1) phase_gather<GATHER_UNROLL>(p.gp, ld_volatile_i32(p.gp.n_dev), threadIdx.x, LWT);
+  if (p.gather) phase_gather<GATHER_UNROLL>(p.g, S, blockIdx.x * (int64_t)LWT + threadIdx.x, gridDim.x * (int64_t)LWT);
+  if (p.pend_n && blockIdx.x == 0 && threadIdx.x == 0) *p.pend_n = S;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(&p.hdr->done, 1u) == gridDim.x - 1) {
+      p.persist->epoch += (uint32_t)p.L;
+      p.hdr->done = 0u;
+    }
+  }
+}
+
 }  // namespace dsp

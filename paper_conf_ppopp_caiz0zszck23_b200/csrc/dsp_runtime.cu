@@ -988,8 +988,10 @@ LwArgs lw_args(Call &k, int l) {
   return a;
 }
 
-// world 1, layer-wise: every layer in one cooperative launch (k_lw_persistent)
-dsp_status stage_lw_persistent(Call &k) {
+// layer-wise: every layer in one cooperative launch per rank (k_lw_persistent
+// at world 1, k_lw_multi at world > 1; `share` = ranks of the call group on
+// this GPU, each launched on its own stream with 1/share of the SMs)
+dsp_status stage_lw_persistent(Call &k, int share = 1) {
   dsp_ctx *c = k.c;
   DeviceGuard g(c->device);
   LwPersistArgs p{};
@@ -1010,9 +1012,23 @@ dsp_status stage_lw_persistent(Call &k) {
     p.pend_n = &ps->pend_n[pd->calls & 1];
   }
   const size_t smem = std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)p.kp_max);
-  const dim3 grid(std::min(c->persist_blocks > 0 ? c->persist_blocks : c->num_sms, 64)), block(LWT);
+  int blocks = std::min(c->persist_blocks > 0 ? c->persist_blocks : c->num_sms, 64);
+  if (share > 1) blocks = std::max(1, std::min(blocks, c->num_sms / share));
+  const dim3 grid(blocks), block(LWT);
+  cudaStream_t st = k.stream;
+  if (share > 1) {  // fork onto the ctx's own stream (joined by join_persistent_multi)
+    if (!c->aux) {
+      CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking));
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[0], cudaEventDisableTiming));
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[1], cudaEventDisableTiming));
+    }
+    CUDA_TRY(c, cudaEventRecord(c->aux_ev[0], k.stream));
+    CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->aux_ev[0], 0));
+    st = c->aux;
+  }
   void *args[] = {&p};
-  CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_lw_persistent, grid, block, args, smem, k.stream));
+  CUDA_TRY(c, cudaLaunchCooperativeKernel(c->world > 1 ? (const void *)k_lw_multi : (const void *)k_lw_persistent,
+                                          grid, block, args, smem, st));
   if (pd) {
     pd->ids = k.blocks[k.L - 1].src_ids;
     pd->out = k.feat_out;
@@ -1116,7 +1132,7 @@ dsp_status run_calls(std::vector<Call> &calls) {
   // a non-pipelined call first settles a pending pipelined gather; so does a
   // pipelined call of the stage-by-stage paths (no loader warps there)
   const bool multi = calls[0].c->world > 1 && !calls[0].layerwise && !calls[0].c->multi_staged;
-  const bool lw_pers = calls[0].layerwise && calls[0].c->world == 1 && !calls[0].c->lw_staged;
+  const bool lw_pers = calls[0].layerwise && !calls[0].c->lw_staged;
   for (auto &k : calls)
     if ((!k.pipelined || (k.c->world > 1 && !multi) || (k.layerwise && !lw_pers)) &&
         (st = stage_flush(k.c, k.ws)) != DSP_OK)
@@ -1133,7 +1149,13 @@ dsp_status run_calls(std::vector<Call> &calls) {
     for (size_t i = 0; i < calls.size(); ++i)
       if ((st = join_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
   } else if (lw_pers) {  // gather (fused, or the previous call's when pipelined) and epoch inside
-    EACH(stage_lw_persistent(k));
+    std::vector<int> share(calls.size(), 0);
+    for (size_t i = 0; i < calls.size(); ++i)
+      for (auto &o : calls) share[i] += o.c->device == calls[i].c->device ? 1 : 0;
+    for (size_t i = 0; i < calls.size(); ++i)
+      if ((st = stage_lw_persistent(calls[i], share[i])) != DSP_OK) return st;
+    for (size_t i = 0; i < calls.size(); ++i)
+      if ((st = join_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
   } else {
     for (int l = 0; l < calls[0].L; ++l) {
       if (calls[0].layerwise) {
@@ -1401,6 +1423,8 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   if (cudaFuncSetAttribute((const void *)k_lw_sample_big, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            (int)sizeof(int32_t) * 3 * LW_MAX_SIZE) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_lw_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           (int)std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)LW_MAX_SIZE)) != cudaSuccess ||
+      cudaFuncSetAttribute((const void *)k_lw_multi, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            (int)std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)LW_MAX_SIZE)) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_lw_alloc, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            (int)LW_ALLOC_SMEM) != cudaSuccess) {

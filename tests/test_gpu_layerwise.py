@@ -89,7 +89,7 @@ def test_layerwise_big_tasks_exercised(pkg, tiny, lw_mode):
 
 
 @pytest.mark.parametrize("P", [2, 4])
-def test_layerwise_virtual_ranks(pkg, tiny, P):
+def test_layerwise_virtual_ranks(pkg, tiny, P, lw_mode):
     cfg, ip, ix, feats = tiny
     bnds = datagen.bounds(cfg.num_nodes, P)
     shards = []
