@@ -182,7 +182,10 @@ struct dsp_ctx {
   int loader_rows = 32;  // DSP_LOADER_ROWS: rows per TMA chunk, <= 32 (tuning knob, results unchanged)
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
   bool multi_staged = false;  // DSP_MULTI_STAGED=1: world > 1 node-wise calls stage by stage (A/B switch)
-  bool lw_staged = false;     // DSP_LW_STAGED=1: world-1 layer-wise calls stage by stage (A/B switch)
+  bool lw_staged = false;     // DSP_LW_STAGED=1: layer-wise calls stage by stage (A/B switch)
+  bool walk_staged = false;   // DSP_WALK_STAGED=1: world > 1 random walks stage by stage (A/B switch)
+  WsHeader *d_walk_hdr = nullptr;  // grid-barrier counter of k_walk_multi
+  int walk_blocks_per_sm = 2;
   cudaStream_t aux = nullptr;  // virtual ranks sharing a GPU: each rank's persistent launch on its own stream
   cudaEvent_t aux_ev[2] = {nullptr, nullptr};
   int gather_blocks_per_sm = 1;
@@ -1243,6 +1246,7 @@ void release(dsp_ctx *c) {
   cudaFree(c->d_weights);
   cudaFree(c->d_feat);
   cudaFree(c->d_xch);
+  cudaFree(c->d_walk_hdr);
   if (c->aux) {
     cudaStreamSynchronize(c->aux);
     cudaStreamDestroy(c->aux);
@@ -1335,6 +1339,43 @@ dsp_status run_walks(std::vector<dsp_ctx *> &cs, std::vector<WalkArgs> &as, std:
     if (c->wseq != seq0) return fail(cs[0], DSP_ERR_STATE, "ranks disagree on the number of walk calls");
   dsp_status st;
   const size_t n = cs.size();
+  if (!cs[0]->walk_staged) {  // one cooperative launch per rank (k_walk_multi)
+    std::vector<int> share(n, 0);
+    for (size_t i = 0; i < n; ++i)
+      for (auto *o : cs) share[i] += o->device == cs[i]->device ? 1 : 0;
+    for (size_t i = 0; i < n; ++i) {
+      dsp_ctx *c = cs[i];
+      DeviceGuard g(c->device);
+      CUDA_TRY(c, cudaMemsetAsync(c->d_walk_hdr, 0, sizeof(WsHeader), ss[i]));
+      cudaStream_t st_i = ss[i];
+      if (share[i] > 1) {  // virtual ranks: each on its own stream with 1/share of the SMs
+        if (!c->aux) {
+          CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking));
+          CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[0], cudaEventDisableTiming));
+          CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[1], cudaEventDisableTiming));
+        }
+        CUDA_TRY(c, cudaEventRecord(c->aux_ev[0], ss[i]));
+        CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->aux_ev[0], 0));
+        st_i = c->aux;
+      }
+      WalkPersistArgs p{};
+      p.a = as[i];
+      p.seq0 = seq0;
+      p.hdr = c->d_walk_hdr;
+      const dim3 grid(std::max(1, c->num_sms * c->walk_blocks_per_sm / share[i])), block(NT);
+      void *args[] = {&p};
+      CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_walk_multi, grid, block, args, 0, st_i));
+    }
+    for (size_t i = 0; i < n; ++i)
+      if (share[i] > 1) {
+        dsp_ctx *c = cs[i];
+        DeviceGuard g(c->device);
+        CUDA_TRY(c, cudaEventRecord(c->aux_ev[1], c->aux));
+        CUDA_TRY(c, cudaStreamWaitEvent(ss[i], c->aux_ev[1], 0));
+      }
+    for (auto *c : cs) c->wseq = seq0 + 1 + (unsigned long long)length;
+    return DSP_OK;
+  }
   for (size_t i = 0; i < n; ++i)
     if ((st = walk_stage(cs[i], as[i], 0, 0, seq0, ss[i])) != DSP_OK) return st;
   for (int l = 0; l < length; ++l)
@@ -1437,6 +1478,13 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   if (getenv("DSP_STAGE_BPS")) c->stage_bps = std::max(1, std::min(8, atoi(getenv("DSP_STAGE_BPS"))));
   c->multi_staged = getenv("DSP_MULTI_STAGED") && atoi(getenv("DSP_MULTI_STAGED")) != 0;
   c->lw_staged = getenv("DSP_LW_STAGED") && atoi(getenv("DSP_LW_STAGED")) != 0;
+  c->walk_staged = getenv("DSP_WALK_STAGED") && atoi(getenv("DSP_WALK_STAGED")) != 0;
+  {
+    int ow = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ow, k_walk_multi, NT, 0) == cudaSuccess && ow >= 1)
+      c->walk_blocks_per_sm = std::min(ow, 2);
+    cudaGetLastError();
+  }
   if (const char *rm = getenv("DSP_RELABEL"))
     c->relabel_mode = !strcmp(rm, "hash") ? 2 : !strcmp(rm, "direct") ? 1 : !strcmp(rm, "direct64") ? 3 : 0;
   if (getenv("DSP_LOADER_ROWS")) c->loader_rows = std::max(1, std::min(32, atoi(getenv("DSP_LOADER_ROWS"))));
@@ -2089,6 +2137,7 @@ dsp_status dsp_reserve_walks(dsp_ctx *c, int64_t max_walks, int32_t max_length) 
   if (max_length < 1 || max_length > 1024) return fail(c, DSP_ERR_INVALID_ARG, "max_length must be in [1, 1024]");
   DeviceGuard g(c->device);
   c->wl = make_walk_layout(c->world, max_walks, max_length);
+  CUDA_TRY(c, cudaMalloc(&c->d_walk_hdr, sizeof(WsHeader)));
   CUDA_TRY(c, cudaMalloc(&c->d_wxch, c->wl.bytes));
   CUDA_TRY(c, cudaMemset(c->d_wxch, 0, c->wl.bytes));
   CUDA_TRY(c, cudaDeviceSynchronize());

@@ -82,7 +82,7 @@ struct WalkArgs {
 
 // Origin: trace rows := -1, column 0 := start, walkers of step 0 := the
 // valid starts (list parity 0).
-__global__ void __launch_bounds__(NT) k_walk_init(WalkArgs a) {
+__device__ __forceinline__ void walk_init_body(const WalkArgs &a) {
   char *self = a.peers.base[a.rank];
   int32_t *tr = walk_trace(self, a.L);
   uint32_t *ctr = walk_ctr(self, a.L);
@@ -108,7 +108,7 @@ __global__ void __launch_bounds__(NT) k_walk_init(WalkArgs a) {
 // Shuffle of step l: every walker kept here goes to the owner of its node
 // (inbox slot order irrelevant); the last block publishes counts + header,
 // then the flags.  The list is consumed (its count reset for step l + 1).
-__global__ void __launch_bounds__(NT) k_walk_scatter(WalkArgs a) {
+__device__ __forceinline__ void walk_scatter_body(const WalkArgs &a) {
   __shared__ uint32_t s_cnt[8], s_base[8];
   char *self = a.peers.base[a.rank];
   uint32_t *ctr = walk_ctr(self, a.L);
@@ -149,7 +149,7 @@ __global__ void __launch_bounds__(NT) k_walk_scatter(WalkArgs a) {
 // Step l at the owner: every received walker takes its fan-out-1 step; the
 // new node goes to trace[l + 1] of the walk at its origin (peer store); a
 // walker that can continue stays here (list parity l + 1).
-__global__ void __launch_bounds__(NT) k_walk_step(WalkArgs a) {
+__device__ __forceinline__ void walk_step_body(const WalkArgs &a) {
   __shared__ uint32_t s_off[9];
   char *self = a.peers.base[a.rank];
   const int world = a.bd.world;
@@ -206,7 +206,7 @@ __global__ void __launch_bounds__(NT) k_walk_step(WalkArgs a) {
 }
 
 // After the last step: tell every rank that this rank's trace stores are done.
-__global__ void k_walk_done(WalkArgs a) {
+__device__ __forceinline__ void walk_done_body(const WalkArgs &a) {
   if (threadIdx.x == 0) {
     uint32_t *ctr = walk_ctr(a.peers.base[a.rank], a.L);
     ctr[0] = ctr[1] = 0u;  // walkers left after the last step are dropped
@@ -216,7 +216,7 @@ __global__ void k_walk_done(WalkArgs a) {
 }
 
 // Origin: once every rank is done, copy the trace rows to the caller.
-__global__ void __launch_bounds__(NT) k_walk_finish(WalkArgs a) {
+__device__ __forceinline__ void walk_finish_body(const WalkArgs &a) {
   char *self = a.peers.base[a.rank];
   if (!wait_flags(walk_done(self, a.L, 0), a.bd.world, a.seq, a.err)) return;
   const int32_t *tr = walk_trace(self, a.L);
@@ -225,6 +225,41 @@ __global__ void __launch_bounds__(NT) k_walk_finish(WalkArgs a) {
     const int64_t i = e / w, c = e - i * w;
     a.traces[e] = __ldcv(tr + i * W + c);
   }
+}
+
+__global__ void __launch_bounds__(NT) k_walk_init(WalkArgs a) { walk_init_body(a); }
+__global__ void __launch_bounds__(NT) k_walk_scatter(WalkArgs a) { walk_scatter_body(a); }
+__global__ void __launch_bounds__(NT) k_walk_step(WalkArgs a) { walk_step_body(a); }
+__global__ void k_walk_done(WalkArgs a) { walk_done_body(a); }
+__global__ void __launch_bounds__(NT) k_walk_finish(WalkArgs a) { walk_finish_body(a); }
+
+// The whole multi-rank walk call in ONE cooperative launch per rank: init,
+// then per step the shuffle (its last block publishes the inbox flags) and the
+// step at the owners (waiting on every rank's flag inside the kernel: all
+// ranks' kernels are resident), a grid barrier before the next step's shuffle
+// reads the list the step appended to, then done flags and the trace copy.
+struct WalkPersistArgs {
+  WalkArgs a;
+  unsigned long long seq0;
+  WsHeader *hdr;            // grid-barrier counter (zeroed by the host before the launch)
+};
+
+__global__ void __launch_bounds__(NT) k_walk_multi(WalkPersistArgs p) {
+  WalkArgs a = p.a;
+  uint32_t bar = 0;
+  walk_init_body(a);
+  grid_barrier<NT>(p.hdr, bar);
+  for (int l = 0; l < a.length; ++l) {
+    a.step = l;
+    a.seq = p.seq0 + 1 + (unsigned long long)l;
+    a.parity = (int)(a.seq & 1ull);
+    walk_scatter_body(a);
+    walk_step_body(a);
+    grid_barrier<NT>(p.hdr, bar);
+  }
+  a.seq = p.seq0 + 1 + (unsigned long long)a.length;
+  if (blockIdx.x == 0) walk_done_body(a);
+  walk_finish_body(a);
 }
 
 }  // namespace dsp

@@ -576,8 +576,11 @@ def test_random_walks_tiny(pkg, tiny):
     s.close()
 
 
+@pytest.mark.parametrize("mode", ["persistent", "staged"])
 @pytest.mark.parametrize("P", [2, 4, 8])
-def test_random_walks_virtual_ranks(pkg, tiny, P):
+def test_random_walks_virtual_ranks(pkg, tiny, P, mode, monkeypatch):
+    if mode == "staged":
+        monkeypatch.setenv("DSP_WALK_STAGED", "1")
     """Walks over a partitioned graph (P:L184: CSP push, reshuffle removed):
     every rank's traces equal the single-device oracle's, whatever P; walks
     start on any owner, meet, terminate at isolated nodes; a rank with no
