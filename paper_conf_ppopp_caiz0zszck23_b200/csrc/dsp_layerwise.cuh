@@ -155,6 +155,12 @@ constexpr size_t LW_ALLOC_SMEM = (size_t)LW_SMEM_F * (sizeof(unsigned long long)
 // LW_SMEM_F frontier nodes); larger frontiers use the workspace copies.
 // PERS: inside the world-1 persistent kernel (k_lw_persistent): no flags, the
 // phases are ordered by its grid barriers.
+#ifdef DSP_DEBUG_STAMPS
+#define LWSTAMP(a, idx) \
+  do { if (threadIdx.x == 0) (a).hdr->dbg[16 + 4 * ((a).layer & 3) + (idx)] = globaltimer_ns(); } while (0)
+#else
+#define LWSTAMP(a, idx) do { } while (0)
+#endif
 template <bool PERS>
 __device__ __forceinline__ void lw_alloc_body(const LwArgs &a, unsigned long long *lw_alloc_smem) {
   __shared__ unsigned long long s_u64[33];
@@ -171,6 +177,7 @@ __device__ __forceinline__ void lw_alloc_body(const LwArgs &a, unsigned long lon
   unsigned long long *P = in_smem ? lw_alloc_smem : a.w.P;
   int32_t *cnt = in_smem ? reinterpret_cast<int32_t *>(lw_alloc_smem + LW_SMEM_F) : a.w.c;
   const int32_t g0 = a.F0 > 0 ? __ldg(a.seeds) : 0;
+  LWSTAMP(a, 0);
   // W_u from the owner's indptr (peer memory): LW_IPT independent loads per
   // thread in flight, then the block-wide exclusive scan
   unsigned long long carry = 0;
@@ -208,6 +215,7 @@ __device__ __forceinline__ void lw_alloc_body(const LwArgs &a, unsigned long lon
   if (tid == 0) P[F] = carry;
   const unsigned long long T = carry;
   __syncthreads();
+  LWSTAMP(a, 1);
   // Eq. 2: n draws with replacement, frontier node i with probability W_i / T
   if (T > 0)
     for (int j = tid; j < a.n; j += LWT) {
@@ -222,6 +230,7 @@ __device__ __forceinline__ void lw_alloc_body(const LwArgs &a, unsigned long lon
       atomicAdd(cnt + lo, 1);
     }
   __syncthreads();
+  LWSTAMP(a, 2);
   // slot offsets, slot -> node, and the tasks pushed to the owners
   if (tid < 8) s_cnt[tid] = 0;
   int32_t ocarry = 0;
@@ -256,6 +265,7 @@ __device__ __forceinline__ void lw_alloc_body(const LwArgs &a, unsigned long lon
   }
   if (tid == 0) a.w.off[F] = ocarry;
   __syncthreads();
+  LWSTAMP(a, 3);
   if (tid == 0) {
     for (int o = 0; o < a.bd.world; ++o)
       *lw_inbox_hdr(a.peers.base[o], a.L, a.parity, a.rank) = make_uint4(s_cnt[o], lw_tag(a.n, a.layer), a.key.x, a.key.y);

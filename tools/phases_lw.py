@@ -30,3 +30,8 @@ if acc:
     print("total %.1f us" % a.sum())
     for n, v in zip(names, a):
         print(f"   {n:10s} {v:7.1f} us")
+dbg = s.workspace[:2048].view(torch.int64)[129 + 16: 129 + 24].cpu().numpy()
+if dbg.any():
+    for l in range(2):
+        d = dbg[4 * l: 4 * l + 4]
+        print(f"alloc{l} sub-steps (us): W+scan {(d[1]-d[0])/1e3:.1f}  draws {(d[2]-d[1])/1e3:.1f}  offsets+tasks {(d[3]-d[2])/1e3:.1f}")
