@@ -992,6 +992,9 @@ __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32
 // grid-wide cursor, so the sampling warps can join when they are done.
 // 4 warps per SM sustain ~5 TB/s on random 400-byte rows
 // (tools/micro/tma_gather_bench.cu), leaving 28 warps for the sampling.
+// MULTI (world > 1): rows of every rank, the bulk copy reading the owner's
+// shard (local, or a peer's over NVLink through its mapping).
+template <bool MULTI = false>
 __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, uint64_t *bars, int64_t n) {
   const int lane = threadIdx.x & 31;
   const GatherArgs &g = a.gp;
@@ -1023,10 +1026,11 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
       __syncwarp();
       if (lane < rows) {
         const int32_t id = __ldg(g.ids + (int64_t)c * R + lane);
-        if (id >= 0 && id < (int32_t)g.bd.b[1])  // cold rows: the bulk copy reads host memory over UVA
+        if (id >= 0 && id < (int32_t)g.bd.b[MULTI ? g.bd.world : 1])  // cold rows: host memory over UVA
           bulk_g2s_hint(ring + (size_t)s * a.slot_bytes + (size_t)lane * row_bytes,
-                        g.tiered ? reinterpret_cast<const char *>(feature_row(g, 0, id))
-                                 : base + (size_t)(uint32_t)id * stride_bytes,
+                        MULTI || g.tiered ? reinterpret_cast<const char *>(
+                                                feature_row(g, MULTI ? owner_of(g.bd, id) : 0, id))
+                                          : base + (size_t)(uint32_t)id * stride_bytes,
                         row_bytes, &bars[s], pol);
         else  // keep the byte count consistent; the error is reported
           latch(g.err, E_RANGE);

@@ -267,12 +267,20 @@ template <int TEAM, bool PIPE>
 __global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
   __shared__ Scan2Smem<TEAM> sm;
   __shared__ uint32_t s_cnt[8], s_base[8], s_off[9];
+  __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];
+  extern __shared__ __align__(128) char ring_smem[];
   const PersistArgs &a = m.p;
   const int blk = blockIdx.x, nblk = gridDim.x;
   const int world = m.bd.world;
 
-  if (PIPE && threadIdx.x >= TEAM) {  // ------ loader warps: previous call's rows, any owner
-    if (a.prev) helper_warp<true>(a, ld_volatile_i32(a.gp.n_dev));
+  if (PIPE && threadIdx.x >= TEAM) {  // ------ loader warps: previous call's rows from every owner (TMA)
+    const int w = (threadIdx.x - TEAM) >> 5;
+    if ((threadIdx.x & 31) == 0)
+      for (int s2 = 0; s2 < LOADER_SLOTS; ++s2) mbar_init(&bars[w][s2], 1);
+    mbar_init_fence();
+    __syncwarp();
+    if (a.prev) loader_warp<true>(a, ring_smem + (size_t)w * LOADER_SLOTS * a.slot_bytes, bars[w],
+                                  ld_volatile_i32(a.gp.n_dev));
     return;
   }
 

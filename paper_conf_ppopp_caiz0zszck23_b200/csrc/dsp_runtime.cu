@@ -777,8 +777,11 @@ dsp_status stage_persistent_multi(Call &k, int share) {
     a.prev = pd->active ? 1 : 0;
     if (a.prev) a.gp = make_gather(c, pd->ids, 0, &ps->pend_n[(pd->calls + 1) & 1], pd->out);
     a.pend_n = &ps->pend_n[pd->calls & 1];
-    a.rows_per_chunk = 32;
-    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_multi<PIPE_TEAM, true>, grid, block, args, 0, st));
+    const int row_bytes = c->dim * 4;
+    a.slot_bytes = (int)align_up((size_t)std::max(12800, row_bytes), 128);
+    a.rows_per_chunk = std::max(1, std::min(c->loader_rows, a.slot_bytes / std::max(1, row_bytes)));
+    const size_t smem = (size_t)LOADER_WARPS * LOADER_SLOTS * a.slot_bytes;
+    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_multi<PIPE_TEAM, true>, grid, block, args, smem, st));
     pd->ids = k.blocks[k.L - 1].src_ids;
     pd->out = k.feat_out;
     pd->stream = k.stream;
@@ -1453,6 +1456,8 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM8, true>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, PIPE_SMEM8_MAX) != cudaSuccess ||
+      cudaFuncSetAttribute((const void *)k_csp_multi<PIPE_TEAM, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_csp_persistent<PNT, false>, PNT, 0) != cudaSuccess ||
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_pipe, k_csp_persistent<PIPE_TEAM, true>, PNT, pipe_smem) !=
           cudaSuccess ||
