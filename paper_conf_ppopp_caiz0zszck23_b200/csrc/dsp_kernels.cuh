@@ -911,7 +911,7 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
 
 constexpr int GATHER_UNROLL = 4;
 
-__global__ void __launch_bounds__(NT) k_gather(GatherArgs a) {
+__global__ void __launch_bounds__(NT) k_gather(const __grid_constant__ GatherArgs a) {
   const int64_t n = a.n_dev ? (int64_t)ld_volatile_i32(a.n_dev) : a.n;
   phase_gather<GATHER_UNROLL>(a, n, blockIdx.x * (int64_t)NT + threadIdx.x, (int64_t)gridDim.x * NT);
 }
@@ -1126,7 +1126,7 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
 // (the paper's loader(t-1) || sampler(t)).  No host round trip,
 // no map clearing (epochs).
 template <int TEAM, bool PIPE>
-__global__ void __launch_bounds__(PNT, 1) k_csp_persistent(PersistArgs a) {
+__global__ void __launch_bounds__(PNT, 1) k_csp_persistent(const __grid_constant__ PersistArgs a) {
   __shared__ Scan2Smem<TEAM> sm;
   __shared__ __align__(8) uint64_t bars[LOADER_WARPS_MAX][LOADER_SLOTS];
   extern __shared__ __align__(128) char ring_smem[];

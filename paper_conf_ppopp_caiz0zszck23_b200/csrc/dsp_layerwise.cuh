@@ -504,7 +504,7 @@ struct LwPersistArgs {
   int32_t *pend_n;          // pipelined: where this call's row count goes
 };
 
-__global__ void __launch_bounds__(LWT, 1) k_lw_persistent(LwPersistArgs p) {
+__global__ void __launch_bounds__(LWT, 1) k_lw_persistent(const __grid_constant__ LwPersistArgs p) {
   extern __shared__ unsigned long long lw_dyn[];
   uint32_t bar = 0;
   if (blockIdx.x == 0 && threadIdx.x == 0) p.hdr->t[0] = globaltimer_ns();
@@ -547,7 +547,7 @@ __global__ void __launch_bounds__(LWT, 1) k_lw_persistent(LwPersistArgs p) {
 // barriers where a stage used to end at a kernel boundary.  Every rank's kernel
 // is resident on its own GPU (virtual ranks: 1/P of the SMs each), so waiting
 // on a peer's flag inside the kernel is safe; waits are bounded (wait_flags).
-__global__ void __launch_bounds__(LWT, 1) k_lw_multi(LwPersistArgs p) {
+__global__ void __launch_bounds__(LWT, 1) k_lw_multi(const __grid_constant__ LwPersistArgs p) {
   extern __shared__ unsigned long long lw_dyn[];
   uint32_t bar = 0;
   if (blockIdx.x == 0 && threadIdx.x == 0) p.hdr->t[0] = globaltimer_ns();

@@ -70,11 +70,16 @@ __device__ __forceinline__ void multi_wait(unsigned long long *flags0, int world
 }
 
 // A: shuffle.  Each block scatters its contiguous chunk of the frontier,
-// TEAM ids per round (shared-memory owner histogram, one global counter add
-// per owner and round, then the peer stores).
+// TEAM ids per round: a shared-memory owner histogram and one global counter
+// add per owner and round give every id its inbox slot; the round's ids are
+// then staged in shared memory grouped by owner, so the peer stores go out as
+// contiguous runs (coalesced NVLink writes) instead of one scattered 4-byte
+// store per id.
 template <int TEAM>
 __device__ __forceinline__ void multi_scatter(const MultiArgs &m, const int32_t *frontier, int F, int par,
                                               uint32_t *s_cnt, uint32_t *s_base) {
+  __shared__ int32_t s_stage[TEAM];
+  __shared__ uint32_t s_pre[9];
   const PersistArgs &a = m.p;
   const Span sp = block_span<TEAM>(F);
   const int64_t b0 = sp.first - threadIdx.x;
@@ -99,11 +104,25 @@ __device__ __forceinline__ void multi_scatter(const MultiArgs &m, const int32_t 
     team_sync<TEAM>();
     if (threadIdx.x < world && s_cnt[threadIdx.x])
       s_base[threadIdx.x] = atomicAdd(&a.hdr->bucket[threadIdx.x], s_cnt[threadIdx.x]);
+    if (threadIdx.x == 32) {  // staging offsets of the owners' runs
+      uint32_t acc = 0;
+      for (int q = 0; q < world; ++q) {
+        s_pre[q] = acc;
+        acc += s_cnt[q];
+      }
+      s_pre[world] = acc;
+    }
     team_sync<TEAM>();
     if (o >= 0) {
-      const uint32_t j = s_base[o] + local;
-      xch_inbox(m.peers.base[o], m.X, par, m.rank)[j] = v;
-      m.perm[i] = (int32_t)j;
+      s_stage[s_pre[o] + local] = v;
+      m.perm[i] = (int32_t)(s_base[o] + local);
+    }
+    team_sync<TEAM>();
+    const uint32_t t = threadIdx.x;
+    if (t < s_pre[world]) {  // staged position t -> owner q, slot s_base[q] + (t - s_pre[q])
+      int q = 0;
+      while (q + 1 < world && t >= s_pre[q + 1]) ++q;
+      xch_inbox(m.peers.base[q], m.X, par, m.rank)[s_base[q] + (t - s_pre[q])] = s_stage[t];
     }
   }
 }
@@ -264,7 +283,7 @@ __device__ __forceinline__ void multi_unpermute(const MultiArgs &m, const int32_
 }
 
 template <int TEAM, bool PIPE>
-__global__ void __launch_bounds__(PNT, 1) k_csp_multi(MultiArgs m) {
+__global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ MultiArgs m) {
   __shared__ Scan2Smem<TEAM> sm;
   __shared__ uint32_t s_cnt[8], s_base[8], s_off[9];
   __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];
