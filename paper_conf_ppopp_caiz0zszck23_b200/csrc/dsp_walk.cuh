@@ -108,11 +108,18 @@ __device__ __forceinline__ void walk_init_body(const WalkArgs &a) {
 // Shuffle of step l: every walker kept here goes to the owner of its node
 // (inbox slot order irrelevant); the last block publishes counts + header,
 // then the flags.  The list is consumed (its count reset for step l + 1).
-__device__ __forceinline__ void walk_scatter_body(const WalkArgs &a) {
+// round of a call: step, flag value, parity (per-launch in the stage kernels, per
+// iteration in k_walk_multi, whose WalkArgs stay in the grid-constant parameter space)
+struct WalkRound {
+  int32_t step, parity;
+  unsigned long long seq;
+};
+
+__device__ __forceinline__ void walk_scatter_body(const WalkArgs &a, const WalkRound rd) {
   __shared__ uint32_t s_cnt[8], s_base[8];
   char *self = a.peers.base[a.rank];
   uint32_t *ctr = walk_ctr(self, a.L);
-  const int lp = a.step & 1;
+  const int lp = rd.step & 1;
   const uint32_t n = *(volatile uint32_t *)&ctr[lp];
   const int2 *list = walk_list(self, a.L, lp);
   for (uint32_t b0 = blockIdx.x * NT; b0 < ((n + NT - 1) / NT) * NT; b0 += gridDim.x * NT) {
@@ -130,7 +137,7 @@ __device__ __forceinline__ void walk_scatter_body(const WalkArgs &a) {
     __syncthreads();
     if (threadIdx.x < a.bd.world) s_base[threadIdx.x] = atomicAdd(&ctr[2 + threadIdx.x], s_cnt[threadIdx.x]);
     __syncthreads();
-    if (o >= 0) walk_inbox(a.peers.base[o], a.L, a.parity, a.rank)[s_base[o] + local] = w;
+    if (o >= 0) walk_inbox(a.peers.base[o], a.L, rd.parity, a.rank)[s_base[o] + local] = w;
     __syncthreads();
   }
   if (last_block_done(&ctr[10])) {
@@ -138,28 +145,28 @@ __device__ __forceinline__ void walk_scatter_body(const WalkArgs &a) {
     for (int o = 0; o < a.bd.world; ++o) {
       const uint32_t c = *(volatile uint32_t *)&ctr[2 + o];
       ctr[2 + o] = 0u;
-      *walk_hdr(a.peers.base[o], a.L, a.parity, a.rank) =
-          make_uint4(c, (uint32_t)a.length | ((uint32_t)a.step << 16), a.key.x, a.key.y);
+      *walk_hdr(a.peers.base[o], a.L, rd.parity, a.rank) =
+          make_uint4(c, (uint32_t)a.length | ((uint32_t)rd.step << 16), a.key.x, a.key.y);
     }
     __threadfence_system();
-    for (int o = 0; o < a.bd.world; ++o) st_release_sys(walk_flag(a.peers.base[o], a.L, a.parity, a.rank), a.seq);
+    for (int o = 0; o < a.bd.world; ++o) st_release_sys(walk_flag(a.peers.base[o], a.L, rd.parity, a.rank), rd.seq);
   }
 }
 
 // Step l at the owner: every received walker takes its fan-out-1 step; the
 // new node goes to trace[l + 1] of the walk at its origin (peer store); a
 // walker that can continue stays here (list parity l + 1).
-__device__ __forceinline__ void walk_step_body(const WalkArgs &a) {
+__device__ __forceinline__ void walk_step_body(const WalkArgs &a, const WalkRound rd) {
   __shared__ uint32_t s_off[9];
   char *self = a.peers.base[a.rank];
   const int world = a.bd.world;
   uint32_t *ctr = walk_ctr(self, a.L);
-  if (wait_flags(walk_flag(self, a.L, a.parity, 0), world, a.seq, a.err)) {
+  if (wait_flags(walk_flag(self, a.L, rd.parity, 0), world, rd.seq, a.err)) {
     if (threadIdx.x == 0) {
       uint32_t acc = 0;
       for (int s = 0; s < world; ++s) {
-        const uint4 h = __ldcv(walk_hdr(self, a.L, a.parity, s));
-        if (h.y != ((uint32_t)a.length | ((uint32_t)a.step << 16)) || h.z != a.key.x || h.w != a.key.y)
+        const uint4 h = __ldcv(walk_hdr(self, a.L, rd.parity, s));
+        if (h.y != ((uint32_t)a.length | ((uint32_t)rd.step << 16)) || h.z != a.key.x || h.w != a.key.y)
           latch(a.err, E_STATE);
         s_off[s] = acc;
         acc += h.x <= (uint32_t)a.L.cap ? h.x : 0u;
@@ -170,7 +177,7 @@ __device__ __forceinline__ void walk_step_body(const WalkArgs &a) {
     const uint32_t total = s_off[world];
     const int64_t W = a.L.max_len + 1;
     const int lane = threadIdx.x & 31;
-    int2 *next = walk_list(self, a.L, (a.step + 1) & 1);
+    int2 *next = walk_list(self, a.L, (rd.step + 1) & 1);
     for (uint32_t b0 = blockIdx.x * NT; b0 < ((total + NT - 1) / NT) * NT; b0 += gridDim.x * NT) {
       const uint32_t q = b0 + threadIdx.x;
       bool keep = false;
@@ -178,7 +185,7 @@ __device__ __forceinline__ void walk_step_body(const WalkArgs &a) {
       if (q < total) {
         int s = 0;
         while (s + 1 < world && q >= s_off[s + 1]) ++s;
-        w = __ldcv(walk_inbox(self, a.L, a.parity, s) + (q - s_off[s]));
+        w = __ldcv(walk_inbox(self, a.L, rd.parity, s) + (q - s_off[s]));
         const int64_t lv = (int64_t)w.y - a.lo;
         int32_t u = -1;
         if (lv < 0 || lv >= a.n_local) {
@@ -186,18 +193,18 @@ __device__ __forceinline__ void walk_step_body(const WalkArgs &a) {
         } else {
           int64_t rs, d;
           row_extent(a.indptr, lv, &rs, &d);
-          if (d > 0) u = __ldg(a.indices + rs + (d == 1 ? 0u : draw_range(a.key, 0u, w.y, a.step, (uint32_t)d)));
+          if (d > 0) u = __ldg(a.indices + rs + (d == 1 ? 0u : draw_range(a.key, 0u, w.y, rd.step, (uint32_t)d)));
         }
         const int origin = (int)((uint32_t)w.x >> WALK_RANK_SHIFT);
         const int64_t i = (int64_t)((uint32_t)w.x & (uint32_t)(WALK_MAX - 1));
-        walk_trace(a.peers.base[origin], a.L)[i * W + a.step + 1] = u;
+        walk_trace(a.peers.base[origin], a.L)[i * W + rd.step + 1] = u;
         keep = u >= 0;
         w.y = u;
       }
       // warp-aggregated append of the walkers that continue
       const unsigned m = __ballot_sync(FULL_MASK, keep);
       uint32_t base = 0;
-      if (lane == 0 && m) base = atomicAdd(&ctr[(a.step + 1) & 1], (uint32_t)__popc(m));
+      if (lane == 0 && m) base = atomicAdd(&ctr[(rd.step + 1) & 1], (uint32_t)__popc(m));
       base = __shfl_sync(FULL_MASK, base, 0);
       if (keep) next[base + __popc(m & ((1u << lane) - 1u))] = w;
     }
@@ -206,19 +213,19 @@ __device__ __forceinline__ void walk_step_body(const WalkArgs &a) {
 }
 
 // After the last step: tell every rank that this rank's trace stores are done.
-__device__ __forceinline__ void walk_done_body(const WalkArgs &a) {
+__device__ __forceinline__ void walk_done_body(const WalkArgs &a, const WalkRound rd) {
   if (threadIdx.x == 0) {
     uint32_t *ctr = walk_ctr(a.peers.base[a.rank], a.L);
     ctr[0] = ctr[1] = 0u;  // walkers left after the last step are dropped
     __threadfence_system();
-    for (int o = 0; o < a.bd.world; ++o) st_release_sys(walk_done(a.peers.base[o], a.L, a.rank), a.seq);
+    for (int o = 0; o < a.bd.world; ++o) st_release_sys(walk_done(a.peers.base[o], a.L, a.rank), rd.seq);
   }
 }
 
 // Origin: once every rank is done, copy the trace rows to the caller.
-__device__ __forceinline__ void walk_finish_body(const WalkArgs &a) {
+__device__ __forceinline__ void walk_finish_body(const WalkArgs &a, const WalkRound rd) {
   char *self = a.peers.base[a.rank];
-  if (!wait_flags(walk_done(self, a.L, 0), a.bd.world, a.seq, a.err)) return;
+  if (!wait_flags(walk_done(self, a.L, 0), a.bd.world, rd.seq, a.err)) return;
   const int32_t *tr = walk_trace(self, a.L);
   const int64_t W = a.L.max_len + 1, w = a.length + 1;
   for (int64_t e = blockIdx.x * (int64_t)NT + threadIdx.x; e < a.n * w; e += (int64_t)gridDim.x * NT) {
@@ -228,10 +235,14 @@ __device__ __forceinline__ void walk_finish_body(const WalkArgs &a) {
 }
 
 __global__ void __launch_bounds__(NT) k_walk_init(WalkArgs a) { walk_init_body(a); }
-__global__ void __launch_bounds__(NT) k_walk_scatter(WalkArgs a) { walk_scatter_body(a); }
-__global__ void __launch_bounds__(NT) k_walk_step(WalkArgs a) { walk_step_body(a); }
-__global__ void k_walk_done(WalkArgs a) { walk_done_body(a); }
-__global__ void __launch_bounds__(NT) k_walk_finish(WalkArgs a) { walk_finish_body(a); }
+__global__ void __launch_bounds__(NT) k_walk_scatter(WalkArgs a) {
+  walk_scatter_body(a, WalkRound{a.step, a.parity, a.seq});
+}
+__global__ void __launch_bounds__(NT) k_walk_step(WalkArgs a) { walk_step_body(a, WalkRound{a.step, a.parity, a.seq}); }
+__global__ void k_walk_done(WalkArgs a) { walk_done_body(a, WalkRound{a.step, a.parity, a.seq}); }
+__global__ void __launch_bounds__(NT) k_walk_finish(WalkArgs a) {
+  walk_finish_body(a, WalkRound{a.step, a.parity, a.seq});
+}
 
 // The whole multi-rank walk call in ONE cooperative launch per rank: init,
 // then per step the shuffle (its last block publishes the inbox flags) and the
@@ -244,22 +255,21 @@ struct WalkPersistArgs {
   WsHeader *hdr;            // grid-barrier counter (zeroed by the host before the launch)
 };
 
-__global__ void __launch_bounds__(NT) k_walk_multi(WalkPersistArgs p) {
-  WalkArgs a = p.a;
+__global__ void __launch_bounds__(NT) k_walk_multi(const __grid_constant__ WalkPersistArgs p) {
+  const WalkArgs &a = p.a;
   uint32_t bar = 0;
   walk_init_body(a);
   grid_barrier<NT>(p.hdr, bar);
   for (int l = 0; l < a.length; ++l) {
-    a.step = l;
-    a.seq = p.seq0 + 1 + (unsigned long long)l;
-    a.parity = (int)(a.seq & 1ull);
-    walk_scatter_body(a);
-    walk_step_body(a);
+    const unsigned long long seq = p.seq0 + 1 + (unsigned long long)l;
+    const WalkRound rd{l, (int32_t)(seq & 1ull), seq};
+    walk_scatter_body(a, rd);
+    walk_step_body(a, rd);
     grid_barrier<NT>(p.hdr, bar);
   }
-  a.seq = p.seq0 + 1 + (unsigned long long)a.length;
-  if (blockIdx.x == 0) walk_done_body(a);
-  walk_finish_body(a);
+  const WalkRound fin{a.length, 0, p.seq0 + 1 + (unsigned long long)a.length};
+  if (blockIdx.x == 0) walk_done_body(a, fin);
+  walk_finish_body(a, fin);
 }
 
 }  // namespace dsp
