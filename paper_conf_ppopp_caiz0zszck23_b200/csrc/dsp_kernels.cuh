@@ -574,6 +574,12 @@ __device__ __forceinline__ void phase_sample_biased(const int32_t *frontier, int
       const bool ok = __shfl_sync(FULL_MASK, okl, j);
       const int64_t s = __shfl_sync(FULL_MASK, sl, j);
       const int64_t d = __shfl_sync(FULL_MASK, dl, j);
+      {  // the next node's weights (rows of up to 32 x 128 B) into L2 while this one is sampled
+        const int jn = min(j + 1, 31);
+        const int64_t sn = __shfl_sync(FULL_MASK, sl, jn), dn = __shfl_sync(FULL_MASK, dl, jn);
+        if (j + 1 < nn && (int64_t)lane * 32 < dn)
+          asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(weights + sn + (int64_t)lane * 32));
+      }
       uint32_t pos;
       const int cnt = sample_node_biased(ok, v, s, d, k, layer, key, weights, &pos);
       if (lane == 0) {
