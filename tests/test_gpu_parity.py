@@ -259,6 +259,33 @@ def test_virtual_ranks_errors(pkg, tiny, mode, monkeypatch):
     grp.close()
 
 
+@pytest.mark.parametrize("mode", ["persistent", "staged"])
+def test_virtual_ranks_all_empty(pkg, tiny, mode, monkeypatch):
+    """Every rank with an empty batch: the exchange still runs (empty inboxes),
+    every block comes back empty, and the next call is unaffected."""
+    if mode == "staged":
+        monkeypatch.setenv("DSP_MULTI_STAGED", "1")
+    cfg, ip, ix, feats = tiny
+    P = 2
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi]))
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 16, devices=[0] * P)
+    empty = torch.zeros(0, dtype=torch.int32, device="cuda")
+    res = grp.sample([empty, empty], 3)
+    for r in range(P):
+        assert all(b.num_dst == 0 and b.num_src == 0 and b.num_edges == 0 for b in res[r])
+        assert res[r][0].indptr.cpu().tolist() == [0]
+    seeds = [np.array([3, 9000], np.int32), np.array([7, 5001], np.int32)]
+    res = grp.sample([torch.from_numpy(x).cuda() for x in seeds], 4)
+    for r in range(P):
+        assert_blocks_equal(res[r], oracle.sample(ip, ix, seeds[r], cfg.fanouts, 4), f"{mode} rank {r}")
+    grp.close()
+
+
 # ----------------------------------------------------- products, full size
 
 @pytest.fixture(scope="module")
