@@ -237,6 +237,55 @@ __device__ __forceinline__ void multi_sample_lanes(const MultiArgs &m, int T, co
   }
 }
 
+// B for biased sampling: warp per task, as phase_sample_biased --
+// the ids and row extents of the warp's next 32 tasks loaded at once, the next
+// task's weight row prefetched into L2 while the current one is sampled.
+template <int TEAM>
+__device__ __forceinline__ void multi_sample_biased(const MultiArgs &m, int T, const uint32_t *s_off, int layer,
+                                                    int k, int par) {
+  const PersistArgs &a = m.p;
+  const int world = m.bd.world;
+  char *self = m.peers.base[m.rank];
+  const int lane = threadIdx.x & 31;
+  const Span sp = block_span<TEAM>(T);
+  const int64_t b0 = sp.first - threadIdx.x;
+  const int wib = threadIdx.x >> 5, wpb = TEAM >> 5;
+  for (int64_t g0 = b0 + wib; g0 < sp.end; g0 += (int64_t)wpb * 32) {
+    const int64_t ql = g0 + (int64_t)lane * wpb;
+    int sl = 0, jl = 0;
+    int32_t vl = 0;
+    bool okl = false;
+    int64_t rsl = 0, dl = 0;
+    if (ql < sp.end) {
+      while (sl + 1 < world && (uint32_t)ql >= s_off[sl + 1]) ++sl;
+      jl = (int)ql - (int)s_off[sl];
+      vl = __ldcv(xch_inbox(self, m.X, par, sl) + jl);
+      const int64_t lv = (int64_t)vl - a.lo;
+      okl = lv >= 0 && lv < a.n_local;
+      if (!okl) latch(a.err, E_STATE);  // routed to the wrong owner
+      else row_extent(a.indptr, lv, &rsl, &dl);
+    }
+    const int nn = (int)min((int64_t)32, (sp.end - g0 + wpb - 1) / wpb);
+    for (int t = 0; t < nn; ++t) {
+      const int s = __shfl_sync(FULL_MASK, sl, t), j = __shfl_sync(FULL_MASK, jl, t);
+      const int32_t v = __shfl_sync(FULL_MASK, vl, t);
+      const bool ok = __shfl_sync(FULL_MASK, okl, t);
+      const int64_t rs = __shfl_sync(FULL_MASK, rsl, t), d = __shfl_sync(FULL_MASK, dl, t);
+      {
+        const int tn = min(t + 1, 31);
+        const int64_t sn = __shfl_sync(FULL_MASK, rsl, tn), dn = __shfl_sync(FULL_MASK, dl, tn);
+        if (t + 1 < nn && (int64_t)lane * 32 < dn)
+          asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(a.weights + sn + (int64_t)lane * 32));
+      }
+      uint32_t pos;
+      const int cnt = sample_node_biased(ok, v, rs, d, k, layer, a.key, a.weights, &pos);
+      char *req = m.peers.base[s];
+      if (lane == 0) xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
+      if (lane < cnt) xch_ret_rows(req, m.X, par, m.rank)[(int64_t)j * m.X.kmax + lane] = __ldg(a.indices + rs + pos);
+    }
+  }
+}
+
 // C: frontier node i (thread per node) reads its row from its owner's return
 // slot perm[i]: counts, edge slots, dst copy and relabel marks.
 template <int TEAM>
@@ -364,7 +413,9 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ Mu
     team_sync<TEAM>();
     const int T = (int)s_off[world];
     const int G = k <= 4 ? 4 : k <= 8 ? 8 : 16;
-    if (a.biased || k > 16)
+    if (a.biased)
+      multi_sample_biased<TEAM>(m, T, s_off, l, k, par);
+    else if (k > 16)
       multi_sample_lanes<32, TEAM>(m, T, s_off, l, k, par);
     else if ((int64_t)T * G <= (int64_t)a.lane_rounds * nblk * TEAM)  // few tasks: lane groups
       (G == 4 ? multi_sample_lanes<4, TEAM> : G == 8 ? multi_sample_lanes<8, TEAM> : multi_sample_lanes<16, TEAM>)(
