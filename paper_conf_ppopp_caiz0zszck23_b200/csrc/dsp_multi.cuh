@@ -306,7 +306,8 @@ __device__ __forceinline__ void multi_unpermute(const MultiArgs &m, const int32_
     }
     const int o = owner_of(m.bd, v);
     const int j = ldw_i32(m.perm + i);
-    const int c = __ldcv(xch_ret_cnt(m.peers.base[m.rank], m.X, par, o) + j);
+    int c = __ldcv(xch_ret_cnt(m.peers.base[m.rank], m.X, par, o) + j);
+    c = c < 0 ? 0 : (c > k ? k : c);  // a failed exchange (E_STATE) leaves stale slots: never write past k
     const int32_t *row = xch_ret_rows(m.peers.base[m.rank], m.X, par, o) + (int64_t)j * m.X.kmax;
     B.cnt[i] = c;
     mark_dst(B, v, i, F, layer, epoch, a.err);
