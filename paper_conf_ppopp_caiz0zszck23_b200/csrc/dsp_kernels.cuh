@@ -1000,8 +1000,11 @@ __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32
 // (tools/micro/tma_gather_bench.cu), leaving 28 warps for the sampling.
 // MULTI (world > 1): rows of every rank, the bulk copy reading the owner's
 // shard (local, or a peer's over NVLink through its mapping).
-template <bool MULTI = false>
-__device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, uint64_t *bars, int64_t n) {
+// STATIC: chunks gw, gw + nw, ... instead of the grid-wide cursor (the
+// standalone k_gather_tma, whose warps all gather).
+template <bool MULTI = false, bool STATIC = false>
+__device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, uint64_t *bars, int64_t n,
+                                            int64_t gw = 0, int64_t nw = 1) {
   const int lane = threadIdx.x & 31;
   const GatherArgs &g = a.gp;
   const int R = a.rows_per_chunk;
@@ -1016,8 +1019,12 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
   while (true) {
     while (!exhausted && issued - done < LOADER_SLOTS) {
       int c = 0;
-      if (lane == 0) c = (int)atomicAdd(&a.hdr->gcursor, 1u);
-      c = __shfl_sync(FULL_MASK, c, 0);
+      if (STATIC) {
+        c = (int)min((int64_t)INT32_MAX, gw + (int64_t)issued * nw);
+      } else {
+        if (lane == 0) c = (int)atomicAdd(&a.hdr->gcursor, 1u);
+        c = __shfl_sync(FULL_MASK, c, 0);
+      }
       if (c >= nchunks) {
         exhausted = true;
         break;
@@ -1045,7 +1052,7 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
       ++issued;
     }
     if (done == issued) break;
-    if (lane == 0) atomicAdd(&a.hdr->chunks_loader, 1u);
+    if (!STATIC && lane == 0) atomicAdd(&a.hdr->chunks_loader, 1u);
     const int s = done % LOADER_SLOTS;
     const int c = s == 0 ? chunk0 : chunk1;
     const int rows = (int)min((int64_t)R, n - (int64_t)c * R);
@@ -1123,6 +1130,25 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
       }
     }
   }
+}
+
+// Standalone gather (dsp_gather_features, pending pipelined gathers): every
+// warp a TMA loader (loader_warp) over a static share of the 32-row chunks:
+// one cp.async.bulk per row into a shared-memory ring slot, one bulk store
+// of the chunk's contiguous output rows.  GTMA_WARPS x 2 slots of <= 16 KB.
+constexpr int GTMA_WARPS = 6;
+template <bool MULTI>
+__global__ void __launch_bounds__(32 * GTMA_WARPS) k_gather_tma(const __grid_constant__ PersistArgs a, int64_t n_host) {
+  __shared__ __align__(8) uint64_t bars[GTMA_WARPS][LOADER_SLOTS];
+  extern __shared__ __align__(128) char ring_smem[];
+  const int w = threadIdx.x >> 5;
+  if ((threadIdx.x & 31) == 0)
+    for (int s2 = 0; s2 < LOADER_SLOTS; ++s2) mbar_init(&bars[w][s2], 1);
+  mbar_init_fence();
+  __syncwarp();
+  const int64_t n = a.gp.n_dev ? (int64_t)ld_volatile_i32(a.gp.n_dev) : n_host;
+  loader_warp<MULTI, true>(a, ring_smem + (size_t)w * LOADER_SLOTS * a.slot_bytes, bars[w], n,
+                           (int64_t)blockIdx.x * GTMA_WARPS + w, (int64_t)gridDim.x * GTMA_WARPS);
 }
 
 // The whole CSP call for world == 1 in one launch: per layer sample(l) +

@@ -184,6 +184,7 @@ struct dsp_ctx {
   bool multi_staged = false;  // DSP_MULTI_STAGED=1: world > 1 node-wise calls stage by stage (A/B switch)
   bool lw_staged = false;     // DSP_LW_STAGED=1: layer-wise calls stage by stage (A/B switch)
   bool walk_staged = false;   // DSP_WALK_STAGED=1: world > 1 random walks stage by stage (A/B switch)
+  bool gather_reg = false;    // DSP_GATHER_REG=1: standalone gathers with register loads (A/B switch)
   WsHeader *d_walk_hdr = nullptr;  // grid-barrier counter of k_walk_multi
   int walk_blocks_per_sm = 2;
   cudaStream_t aux = nullptr;  // virtual ranks sharing a GPU: each rank's persistent launch on its own stream
@@ -802,14 +803,47 @@ dsp_status join_persistent_multi(Call &k, int share) {
   return DSP_OK;
 }
 
-// gather owed by a workspace's last pipelined call (k_gather with the device row count)
+// A standalone gather: TMA loader warps (k_gather_tma) by default, 16-byte
+// register loads (k_gather) with DSP_GATHER_REG=1 or for register-loaded cold rows.
+// n_host: the row count, or ignored when g.n_dev gives it on the device.
+dsp_status launch_gather(dsp_ctx *c, const GatherArgs &g, int64_t n_host, cudaStream_t st) {
+  if (c->gather_reg || (c->tiered && c->cold_regloads)) {
+    int grid = grid_for(c, std::min(6, c->gather_blocks_per_sm));
+    if (!g.n_dev) {  // resident blocks only (a partial extra wave costs more than it hides)
+      const int64_t want = (n_host * g.dim4 + (int64_t)NT * GATHER_UNROLL - 1) / ((int64_t)NT * GATHER_UNROLL);
+      grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, grid));
+    }
+    k_gather<<<grid, NT, 0, st>>>(g);
+    CUDA_TRY(c, cudaGetLastError());
+    return DSP_OK;
+  }
+  PersistArgs a{};
+  a.gp = g;
+  const int row_bytes = c->dim * 4;
+  a.slot_bytes = (int)align_up((size_t)std::max(12800, row_bytes), 128);
+  a.rows_per_chunk = std::max(1, std::min(c->loader_rows, a.slot_bytes / std::max(1, row_bytes)));
+  int blocks = c->num_sms;
+  if (!g.n_dev) {
+    const int64_t chunks = (n_host + a.rows_per_chunk - 1) / a.rows_per_chunk;
+    blocks = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (chunks + 2 * GTMA_WARPS - 1) / (2 * GTMA_WARPS)));
+  }
+  const size_t smem = (size_t)GTMA_WARPS * LOADER_SLOTS * a.slot_bytes;
+  if (c->world > 1)
+    k_gather_tma<true><<<blocks, 32 * GTMA_WARPS, smem, st>>>(a, n_host);
+  else
+    k_gather_tma<false><<<blocks, 32 * GTMA_WARPS, smem, st>>>(a, n_host);
+  CUDA_TRY(c, cudaGetLastError());
+  return DSP_OK;
+}
+
+// gather owed by a workspace's last pipelined call (the device row count)
 dsp_status flush_one(dsp_ctx *c, dsp_ctx::Pending &pd) {
   if (!pd.active) return DSP_OK;
   DeviceGuard g(c->device);
   const WsPersist *ps = reinterpret_cast<const WsPersist *>(pd.ws);
   GatherArgs a = make_gather(c, pd.ids, 0, &ps->pend_n[(pd.calls + 1) & 1], pd.out);
-  k_gather<<<grid_for(c, std::min(6, c->gather_blocks_per_sm)), NT, 0, static_cast<cudaStream_t>(pd.stream)>>>(a);
-  CUDA_TRY(c, cudaGetLastError());
+  dsp_status st = launch_gather(c, a, 0, static_cast<cudaStream_t>(pd.stream));
+  if (st != DSP_OK) return st;
   pd.active = false;
   return DSP_OK;
 }
@@ -1083,9 +1117,7 @@ dsp_status stage_gather_dev(Call &k) {
   DeviceGuard g(c->device);
   const int l = k.L - 1;
   GatherArgs a = make_gather(c, k.blocks[l].src_ids, 0, &k.hdr->S[l], k.feat_out);
-  k_gather<<<grid_for(c, std::min(6, c->gather_blocks_per_sm)), NT, 0, k.stream>>>(a);
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
+  return launch_gather(c, a, 0, k.stream);
 }
 
 // ------------------------------------------------------------- end of call
@@ -1484,6 +1516,14 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   c->multi_staged = getenv("DSP_MULTI_STAGED") && atoi(getenv("DSP_MULTI_STAGED")) != 0;
   c->lw_staged = getenv("DSP_LW_STAGED") && atoi(getenv("DSP_LW_STAGED")) != 0;
   c->walk_staged = getenv("DSP_WALK_STAGED") && atoi(getenv("DSP_WALK_STAGED")) != 0;
+  c->gather_reg = getenv("DSP_GATHER_REG") && atoi(getenv("DSP_GATHER_REG")) != 0;
+  if (cudaFuncSetAttribute((const void *)k_gather_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           GTMA_WARPS * LOADER_SLOTS * 16384) != cudaSuccess ||
+      cudaFuncSetAttribute((const void *)k_gather_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           GTMA_WARPS * LOADER_SLOTS * 16384) != cudaSuccess) {
+    cudaGetLastError();
+    c->gather_reg = true;  // no TMA gather: register loads
+  }
   {
     int ow = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ow, k_walk_multi, NT, 0) == cudaSuccess && ow >= 1)
@@ -2074,12 +2114,7 @@ dsp_status dsp_gather_features(dsp_ctx *c, const int32_t *ids, int64_t n, float 
   DeviceGuard g(c->device);
   GatherArgs a = make_gather(c, ids, n, nullptr, out);
   if (n * a.dim4 >= (1ll << 31)) return fail(c, DSP_ERR_CAPACITY, "n * dim / 4 must be < 2^31 per call");
-  const int64_t want = (n * a.dim4 + (int64_t)NT * GATHER_UNROLL - 1) / ((int64_t)NT * GATHER_UNROLL);
-  // resident blocks only (a partial extra wave costs more than it hides; tools/micro/tma_gather_bench.cu)
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, grid_for(c, std::min(6, c->gather_blocks_per_sm))));
-  k_gather<<<grid, NT, 0, static_cast<cudaStream_t>(stream)>>>(a);
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
+  return launch_gather(c, a, n, static_cast<cudaStream_t>(stream));
 }
 
 dsp_status dsp_random_walk(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length, uint64_t rng_seed,
