@@ -1136,7 +1136,10 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
 // warp a TMA loader (loader_warp) over a static share of the 32-row chunks:
 // one cp.async.bulk per row into a shared-memory ring slot, one bulk store
 // of the chunk's contiguous output rows.  GTMA_WARPS x 2 slots of <= 16 KB.
-constexpr int GTMA_WARPS = 6;
+#ifndef DSP_GTMA_WARPS
+#define DSP_GTMA_WARPS 6
+#endif
+constexpr int GTMA_WARPS = DSP_GTMA_WARPS;
 template <bool MULTI>
 __global__ void __launch_bounds__(32 * GTMA_WARPS) k_gather_tma(const __grid_constant__ PersistArgs a, int64_t n_host) {
   __shared__ __align__(8) uint64_t bars[GTMA_WARPS][LOADER_SLOTS];

@@ -822,7 +822,7 @@ dsp_status launch_gather(dsp_ctx *c, const GatherArgs &g, int64_t n_host, cudaSt
   const int row_bytes = c->dim * 4;
   a.slot_bytes = (int)align_up((size_t)std::max(12800, row_bytes), 128);
   a.rows_per_chunk = std::max(1, std::min(c->loader_rows, a.slot_bytes / std::max(1, row_bytes)));
-  int blocks = c->num_sms;
+  int blocks = c->num_sms * (GTMA_WARPS <= 4 ? 2 : 1);
   if (!g.n_dev) {
     const int64_t chunks = (n_host + a.rows_per_chunk - 1) / a.rows_per_chunk;
     blocks = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (chunks + 2 * GTMA_WARPS - 1) / (2 * GTMA_WARPS)));
