@@ -1,11 +1,15 @@
 """bench.py -- DSP CSP sampling + feature gather throughput on B200.
 
-One step = one pass of the whole hot path over one mini-batch per GPU:
-dsp_sample (CSP over all layers: shuffle / sample / reshuffle / relabel,
-SURVEY.md 8(a) a1-a7) followed by dsp_gather_features for the sampled nodes
-(a8).  Workload at N=1: BASELINE.json configs[1] (ogbn-products-shaped
-synthetic R-MAT, fan-out [15,10,5], 1024 seeds/GPU, dim 100); N>1:
-configs[2] (the same graph partitioned over N GPUs, weak scaling).
+One step = one pass of the whole hot path over one mini-batch per GPU: one
+dsp_sample_gather call -- CSP over all layers (shuffle / sample / reshuffle /
+relabel) and the feature gather of the sampled nodes
+(a8) -- pipelined as in the paper: the launch of step t samples
+batch t while its loader warps gather batch t-1; at N=1 four step streams run
+concurrently on 37 SMs each.  Workload at N=1: BASELINE.json configs[1]
+(ogbn-products-shaped synthetic R-MAT, fan-out [15,10,5], 1024 seeds/GPU,
+dim 100); N>1: configs[2] (the same graph partitioned over N GPUs, weak
+scaling).  --config papers | friendster, --scheme biased | layer | walk and
+--hot-frac select the other workloads.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl dsp|reference]
 
