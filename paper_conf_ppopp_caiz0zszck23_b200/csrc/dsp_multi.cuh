@@ -129,65 +129,85 @@ __device__ __forceinline__ void multi_scatter(const MultiArgs &m, const int32_t 
 
 // B: the owner's sample of every received task.  Tasks are numbered over the
 // senders (s_off = prefix of the per-sender counts); thread per task for
-// k <= KB (draws, Floyd and ranking in registers, as phase_sample_tpn), the
-// row written to the requester's return slot j (count, then row in slot order).
+// k <= KB (draws, Floyd and ranking in registers, as phase_sample_tpn).  The
+// count goes straight to the requester's return slot j; the row (slot order,
+// row j of the requester's return rows at stride k) is staged in shared
+// memory for the block's round of TEAM tasks and then copied out as one
+// contiguous run per requester (coalesced NVLink stores).
 template <int KB, int TEAM>
 __device__ __forceinline__ void multi_sample_tpn(const MultiArgs &m, int T, const uint32_t *s_off, int layer, int k,
                                                  int par) {
+  constexpr bool STAGE = KB <= 8;  // k <= 8 (the largest layer): staged; k <= 16: direct stores
+  __shared__ int32_t s_rows[STAGE ? TEAM * KB : 1];
   const PersistArgs &a = m.p;
   const int world = m.bd.world;
   char *self = m.peers.base[m.rank];
-  const int64_t kmax = m.X.kmax;
   const Span sp = block_span<TEAM>(T);
-  for (int64_t qq = sp.first; qq < sp.end; qq += sp.step) {
-    const int q = (int)qq;
-    int s = 0;
-    while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
-    const int j = q - (int)s_off[s];
-    const int32_t v = __ldcv(xch_inbox(self, m.X, par, s) + j);
-    const int64_t lv = (int64_t)v - a.lo;
-    char *req = m.peers.base[s];
-    if (lv < 0 || lv >= a.n_local) {  // routed to the wrong owner: protocol error
-      latch(a.err, E_STATE);
-      xch_ret_cnt(req, m.X, par, m.rank)[j] = 0;
-      continue;
-    }
-    int64_t rs, d;
-    row_extent(a.indptr, lv, &rs, &d);
-    const bool full = d <= k;
-    const int cnt = full ? (int)d : k;
-    uint32_t pos[KB];
+  const int64_t b0 = sp.first - threadIdx.x;
+  for (int64_t r0 = b0; r0 < sp.end; r0 += TEAM) {  // block-uniform rounds
+    const int q = (int)(r0 + threadIdx.x);
+    if (q < sp.end) {
+      int s = 0;
+      while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
+      const int j = q - (int)s_off[s];
+      const int32_t v = __ldcv(xch_inbox(self, m.X, par, s) + j);
+      const int64_t lv = (int64_t)v - a.lo;
+      char *req = m.peers.base[s];
+      if (lv < 0 || lv >= a.n_local) {  // routed to the wrong owner: protocol error
+        latch(a.err, E_STATE);
+        xch_ret_cnt(req, m.X, par, m.rank)[j] = 0;
+      } else {
+        int64_t rs, d;
+        row_extent(a.indptr, lv, &rs, &d);
+        const bool full = d <= k;
+        const int cnt = full ? (int)d : k;
+        uint32_t pos[KB];
 #pragma unroll
-    for (int t = 0; t < KB; ++t) pos[t] = (uint32_t)t;
-    if (!full) {
+        for (int t = 0; t < KB; ++t) pos[t] = (uint32_t)t;
+        if (!full) {
 #pragma unroll
-      for (int t = 0; t < KB; ++t)
-        if (t < k) pos[t] = draw_range(a.key, (uint32_t)t, v, layer, (uint32_t)(d - k + t + 1));
+          for (int t = 0; t < KB; ++t)
+            if (t < k) pos[t] = draw_range(a.key, (uint32_t)t, v, layer, (uint32_t)(d - k + t + 1));
 #pragma unroll
-      for (int t = 1; t < KB; ++t) {
-        if (t < k) {
-          bool hit = false;
+          for (int t = 1; t < KB; ++t) {
+            if (t < k) {
+              bool hit = false;
 #pragma unroll
-          for (int qx = 0; qx < t; ++qx) hit |= (pos[qx] == pos[t]);
-          if (hit) pos[t] = (uint32_t)(d - k + t);
+              for (int qx = 0; qx < t; ++qx) hit |= (pos[qx] == pos[t]);
+              if (hit) pos[t] = (uint32_t)(d - k + t);
+            }
+          }
         }
+        int32_t u[KB];
+        unsigned long long slots = 0;
+#pragma unroll
+        for (int t = 0; t < KB; ++t) {
+          uint32_t r = 0;
+#pragma unroll
+          for (int qx = 0; qx < KB; ++qx) r += (qx < cnt && pos[qx] < pos[t]) ? 1u : 0u;
+          slots |= (unsigned long long)r << (4 * t);
+          u[t] = (t < cnt) ? adj_ld(a.indices + rs + pos[t]) : 0;
+        }
+        xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
+        int32_t *row = STAGE ? s_rows + (int64_t)threadIdx.x * k : xch_ret_rows(req, m.X, par, m.rank) + (int64_t)j * k;
+#pragma unroll
+        for (int t = 0; t < KB; ++t)
+          if (t < cnt) row[(slots >> (4 * t)) & 15u] = u[t];
       }
     }
-    int32_t u[KB];
-    unsigned long long slots = 0;
-#pragma unroll
-    for (int t = 0; t < KB; ++t) {
-      uint32_t r = 0;
-#pragma unroll
-      for (int qx = 0; qx < KB; ++qx) r += (qx < cnt && pos[qx] < pos[t]) ? 1u : 0u;
-      slots |= (unsigned long long)r << (4 * t);
-      u[t] = (t < cnt) ? adj_ld(a.indices + rs + pos[t]) : 0;
+    if (!STAGE) continue;
+    team_sync<TEAM>();
+    // copy-out: the round's tasks [r0, r1) split into one contiguous run per requester
+    const int64_t r1 = min(sp.end, r0 + TEAM);
+    for (int s = 0; s < world; ++s) {
+      const int64_t q0 = max(r0, (int64_t)s_off[s]), q1 = min(r1, (int64_t)s_off[s + 1]);
+      if (q0 >= q1) continue;
+      int32_t *dst = xch_ret_rows(m.peers.base[s], m.X, par, m.rank) + (q0 - (int64_t)s_off[s]) * k;
+      const int32_t *src = s_rows + (q0 - r0) * k;
+      const int64_t len = (q1 - q0) * k;
+      for (int64_t e = threadIdx.x; e < len; e += TEAM) dst[e] = src[e];
     }
-    xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
-    int32_t *row = xch_ret_rows(req, m.X, par, m.rank) + (int64_t)j * kmax;
-#pragma unroll
-    for (int t = 0; t < KB; ++t)
-      if (t < cnt) row[(slots >> (4 * t)) & 15u] = u[t];
+    team_sync<TEAM>();
   }
 }
 
@@ -233,7 +253,7 @@ __device__ __forceinline__ void multi_sample_lanes(const MultiArgs &m, int T, co
     }
     char *req = m.peers.base[s];
     if (active && leader) xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
-    if (valid) xch_ret_rows(req, m.X, par, m.rank)[(int64_t)j * m.X.kmax + slot] = u;
+    if (valid) xch_ret_rows(req, m.X, par, m.rank)[(int64_t)j * k + slot] = u;
   }
 }
 
@@ -281,7 +301,7 @@ __device__ __forceinline__ void multi_sample_biased(const MultiArgs &m, int T, c
       const int cnt = sample_node_biased(ok, v, rs, d, k, layer, a.key, a.weights, &pos);
       char *req = m.peers.base[s];
       if (lane == 0) xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
-      if (lane < cnt) xch_ret_rows(req, m.X, par, m.rank)[(int64_t)j * m.X.kmax + lane] = __ldg(a.indices + rs + pos);
+      if (lane < cnt) xch_ret_rows(req, m.X, par, m.rank)[(int64_t)j * k + lane] = __ldg(a.indices + rs + pos);
     }
   }
 }
@@ -308,7 +328,7 @@ __device__ __forceinline__ void multi_unpermute(const MultiArgs &m, const int32_
     const int j = ldw_i32(m.perm + i);
     int c = __ldcv(xch_ret_cnt(m.peers.base[m.rank], m.X, par, o) + j);
     c = c < 0 ? 0 : (c > k ? k : c);  // a failed exchange (E_STATE) leaves stale slots: never write past k
-    const int32_t *row = xch_ret_rows(m.peers.base[m.rank], m.X, par, o) + (int64_t)j * m.X.kmax;
+    const int32_t *row = xch_ret_rows(m.peers.base[m.rank], m.X, par, o) + (int64_t)j * k;  // rows at stride k
     B.cnt[i] = c;
     mark_dst(B, v, i, F, layer, epoch, a.err);
     const uint32_t q0 = (uint32_t)i * (uint32_t)k;
