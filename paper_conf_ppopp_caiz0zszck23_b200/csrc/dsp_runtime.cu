@@ -693,8 +693,10 @@ dsp_status stage_persistent(Call &k) {
   if (a.prev) a.gp = make_gather(c, pd->ids, 0, &ps->pend_n[(pd->calls + 1) & 1], pd->out);
   a.pend_n = &ps->pend_n[pd->calls & 1];
   const int row_bytes = c->dim * 4;
-  a.slot_bytes = (int)align_up((size_t)std::max(12800, row_bytes), 128);
-  a.rows_per_chunk = std::max(1, std::min(c->loader_rows, a.slot_bytes / std::max(1, row_bytes)));
+  // ring slots sized to the chunk (rows_per_chunk rows of <= 12.8 KB in all): the ring's
+  // shared memory is taken from the L1 the sampling phases use
+  a.rows_per_chunk = std::max(1, std::min(c->loader_rows, 12800 / std::max(1, row_bytes)));
+  a.slot_bytes = (int)align_up((size_t)a.rows_per_chunk * row_bytes, 128);
   const bool lw8 = c->loader_warps == LOADER_WARPS_MAX &&
                    (size_t)LOADER_WARPS_MAX * LOADER_SLOTS * a.slot_bytes <= (size_t)PIPE_SMEM8_MAX;
   const bool lw2 = c->loader_warps == 2;
