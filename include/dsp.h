@@ -227,9 +227,8 @@ dsp_status dsp_sample(dsp_ctx *ctx, const int32_t *seeds, int32_t num_seeds, con
    of the world present).  Node-wise calls run one persistent kernel per rank
    (the exchanges through peer memory inside it); ranks sharing a device each
    get 1/n of its SMs on the ctx's own stream, forked from and joined to the
-   given stream after all ranks were launched.  Virtual ranks sharing a device
-   must pass the same stream.  The layer-wise scheme (and DSP_MULTI_STAGED=1)
-   issues its stage kernels rank by rank per stage on that stream. */
+   given stream after all ranks were launched (layer-wise calls likewise).
+   Virtual ranks sharing a device must pass the same stream. */
 dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *seeds,
                             const int32_t *num_seeds, const int32_t *fanouts, int32_t num_layers,
                             uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,
@@ -278,8 +277,38 @@ dsp_status dsp_sample_gather(dsp_ctx *ctx, const int32_t *seeds, int32_t num_see
    overlap the other's bandwidth-bound gather).  Not collective. */
 dsp_status dsp_set_persistent_blocks(dsp_ctx *ctx, int32_t blocks);
 
-/* Enqueues the gather still owed by the last DSP_PIPELINED call (no-op when
-   none is pending).  Stream-ordered on `stream`. */
+/* Performance options of a ctx (not collective).  None of them changes a
+   result: blocks and gathered rows are bit-identical for every value (the
+   GPU tests run the oracle parity under each).  Returns DSP_ERR_INVALID_ARG
+   for an unknown option or a value outside its range.
+   DSP_OPT_RELABEL_MAP     layout of the relabel map:
+                           0 = by N (default: compact 4-byte direct map for
+                           N <= 3M, else a batch-sized hash table), 1 = compact
+                           direct map, 2 = hash table, 3 = 8-byte direct map.
+                           Only before dsp_reserve / dsp_reserve_layerwise
+                           (the workspace plan depends on it; DSP_ERR_STATE
+                           afterwards); ranks may differ.
+   DSP_OPT_LANE_ROUNDS     node-wise sampling with lane groups (G lanes per
+                           node) while frontier * G <= value * sampling threads,
+                           else a thread per node; 1..1024, default 8.
+   DSP_OPT_LOADER_WARPS    TMA loader warps per SM of a DSP_PIPELINED launch:
+                           2, 4 (default) or 8.
+   DSP_OPT_LOADER_ROWS     rows per TMA gather chunk, 1..32 (default 32).
+   DSP_OPT_GATHER_REGLOADS 0 (default) = standalone gathers and cold-tier rows
+                           moved by TMA bulk copies; 1 = 16-byte register
+                           loads. */
+#define DSP_OPT_RELABEL_MAP 1
+#define DSP_OPT_LANE_ROUNDS 2
+#define DSP_OPT_LOADER_WARPS 3
+#define DSP_OPT_LOADER_ROWS 4
+#define DSP_OPT_GATHER_REGLOADS 5
+dsp_status dsp_set_option(dsp_ctx *ctx, int32_t option, int64_t value);
+
+/* Enqueues every gather still owed by this ctx's DSP_PIPELINED calls (one
+   per workspace; no-op when none is pending) on `stream`.  A call made on
+   another stream is waited for first (an event recorded on its stream), so
+   work issued on `stream` afterwards sees every feat_out written, whichever
+   stream the pipelined calls ran on. */
 dsp_status dsp_pipeline_flush(dsp_ctx *ctx, void *stream);
 
 /* --------------------------------------------------------------- gather */

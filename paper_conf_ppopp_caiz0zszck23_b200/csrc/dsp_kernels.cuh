@@ -22,9 +22,7 @@
 // (k_csp_persistent, one 1024-thread block per SM) with grid barriers between
 // phases; world > 1 runs it in one persistent kernel per rank as well
 // (k_csp_multi, dsp_multi.cuh), the exchanges done inside it through peer
-// memory.  The stage-by-stage kernels below (k_bucket_scatter ..
-// k_write_indices, one launch per phase) remain as the DSP_MULTI_STAGED=1
-// A/B switch (tested against the oracle like the default path).
+// memory.
 //
 // Data a phase reads after another phase of the same kernel wrote it is read
 // with plain (weak) loads after the grid barrier's release/acquire, never
@@ -108,7 +106,6 @@ struct WsHeader {
 struct LayerBufs {
   int32_t *cnt;                 // [F] sampled count per frontier node
   int32_t *rows;                // [F*k] sampled neighbour (global id) of edge slot q = i*k + slot
-  unsigned long long *status;   // [0] tile ticket, [1 + t] tile status (look-back scan)
   unsigned long long *first;    // relabel map: [N] direct words, or [mask + 1] hash slots
   uint32_t mask;                // 0: direct map indexed by global id; else hash table of mask + 1 slots
   uint32_t *first32;            // compact direct map [N] (tag | ~x words), or nullptr
@@ -800,39 +797,6 @@ __device__ __forceinline__ void phase_indices_dups(int F, int k, const LayerBufs
   }
 }
 
-// ---------------------------------------------------------- write indices
-// indices[indptr[i] + t] = local id of the src of slot q = i*k + t.
-__device__ __forceinline__ void phase_indices(int F, int k, const LayerBufs &B, uint32_t epoch,
-                                              const int32_t *indptr, int32_t *indices_out, const Span &sp) {
-  constexpr int U = 4;  // items per thread in flight
-  const FastDiv fd = make_fastdiv((uint32_t)k);
-  const uint32_t end = (uint32_t)sp.end, step = (uint32_t)sp.step;
-  (void)F;
-  for (uint32_t q0 = (uint32_t)sp.first; q0 < end; q0 += step * U) {
-    int32_t c[U], u[U], ip[U];
-#pragma unroll
-    for (int j = 0; j < U; ++j) {
-      const uint32_t q = q0 + j * step;
-      c[j] = -1;
-      u[j] = 0;
-      ip[j] = 0;
-      if (q < end) {
-        const uint32_t i = fdiv(q, fd);
-        const int32_t t = (int32_t)(q - i * (uint32_t)k);
-        c[j] = ldw_i32(B.cnt + i) - t;  // > 0 iff slot q holds an edge
-        u[j] = ldw_i32(B.rows + q);
-        ip[j] = ldw_i32(indptr + i) + t;
-      }
-    }
-    unsigned long long w[U];
-#pragma unroll
-    for (int j = 0; j < U; ++j) w[j] = c[j] > 0 ? map_get(B, u[j], epoch) : 0ull;
-#pragma unroll
-    for (int j = 0; j < U; ++j)
-      if (c[j] > 0) indices_out[ip[j]] = (int32_t)mword_x(B, w[j]);
-  }
-}
-
 // ----------------------------------------------------------------- gather
 struct GatherArgs {
   const int32_t *ids;
@@ -1358,375 +1322,6 @@ __device__ __forceinline__ bool last_block_done(uint32_t *done) {
   return false;
 }
 
-__device__ __forceinline__ int frontier_size(const WsHeader *hdr, int layer, int F0) {
-  return layer == 0 ? F0 : ld_volatile_i32(&hdr->F[layer]);
-}
-
-struct BucketArgs {
-  const int32_t *frontier;
-  int32_t F0, layer, k, biased;
-  uint32_t seed_lo, seed_hi;
-  int32_t rank, parity;
-  unsigned long long seq;
-  Bounds bd;
-  XchLayout L;
-  XchPeers peers;
-  int32_t *perm;            // [F] slot of frontier i in its owner's inbox
-  WsHeader *hdr;
-  int *err;
-};
-
-// Shuffle: group the frontier by owner (range check) and
-// write each id straight into the owner's inbox over NVLink; the slot order
-// inside a bucket is irrelevant (results come back to the same slot).  The
-// last block publishes the per-owner counts + header, then the flag
-// (count notification before use).
-__global__ void __launch_bounds__(NT) k_bucket_scatter(BucketArgs a) {
-  __shared__ uint32_t s_cnt[8], s_base[8];
-  const int F = frontier_size(a.hdr, a.layer, a.F0);
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    if (F > a.L.cap) {
-      latch(a.err, E_CAP);
-      a.hdr->F[a.layer] = 0;  // later kernels of this layer see an empty frontier
-    } else if (a.layer == 0) {
-      a.hdr->F[0] = a.F0;
-    }
-  }
-  const int limit = F > a.L.cap ? 0 : F;
-  for (int b0 = blockIdx.x * NT; b0 < ((limit + NT - 1) / NT) * NT; b0 += gridDim.x * NT) {
-    if (threadIdx.x < 8) s_cnt[threadIdx.x] = 0;
-    __syncthreads();
-    const int i = b0 + threadIdx.x;
-    int o = -1;
-    uint32_t local = 0;
-    int32_t v = 0;
-    if (i < limit) {
-      v = __ldg(a.frontier + i);
-      if (v < 0 || v >= a.bd.b[a.bd.world]) {
-        latch(a.err, E_RANGE);
-      } else {
-        o = owner_of(a.bd, v);
-        local = atomicAdd(&s_cnt[o], 1u);
-      }
-    }
-    __syncthreads();
-    if (threadIdx.x < a.bd.world) s_base[threadIdx.x] = atomicAdd(&a.hdr->bucket[threadIdx.x], s_cnt[threadIdx.x]);
-    __syncthreads();
-    if (o >= 0) {
-      const uint32_t j = s_base[o] + local;
-      xch_inbox(a.peers.base[o], a.L, a.parity, a.rank)[j] = v;
-      a.perm[i] = (int32_t)j;
-    }
-    __syncthreads();
-  }
-  if (last_block_done(&a.hdr->done)) {
-    for (int o = 0; o < a.bd.world; ++o) {
-      const uint32_t c = *(volatile uint32_t *)&a.hdr->bucket[o];
-      a.hdr->bucket[o] = 0u;
-      *xch_inbox_hdr(a.peers.base[o], a.L, a.parity, a.rank) =
-          make_uint4(c, (uint32_t)a.k | ((uint32_t)a.layer << 8) | ((uint32_t)a.biased << 16), a.seed_lo, a.seed_hi);
-    }
-    __threadfence_system();
-    for (int o = 0; o < a.bd.world; ++o)
-      st_release_sys(xch_inbox_flag(a.peers.base[o], a.L, a.parity, a.rank), a.seq);
-  }
-}
-
-struct RemoteSampleArgs {
-  int32_t layer, k;
-  int32_t biased;
-  const uint32_t *weights;
-  uint2 key;
-  int32_t rank, parity;
-  unsigned long long seq;
-  const int64_t *indptr;
-  const int32_t *indices;
-  int64_t lo, n_local;
-  Bounds bd;
-  XchLayout L;
-  XchPeers peers;
-  WsHeader *hdr;
-  int *err;
-};
-
-// Sample stage at the owner: one kernel over every task received in
-// this layer, results written straight into each requester's
-// return slots over NVLink, then the return flags.
-template <int G>
-__global__ void __launch_bounds__(NT) k_sample_remote(RemoteSampleArgs a) {
-  __shared__ uint32_t s_off[9];
-  char *self = a.peers.base[a.rank];
-  const int world = a.bd.world;
-  if (wait_flags(xch_inbox_flag(self, a.L, a.parity, 0), world, a.seq, a.err)) {
-    if (threadIdx.x == 0) {
-      uint32_t acc = 0;
-      for (int s = 0; s < world; ++s) {
-        const uint4 h = __ldcv(xch_inbox_hdr(self, a.L, a.parity, s));
-        if (h.y != ((uint32_t)a.k | ((uint32_t)a.layer << 8) | ((uint32_t)a.biased << 16)) || h.z != a.key.x ||
-            h.w != a.key.y)
-          latch(a.err, E_STATE);
-        s_off[s] = acc;
-        acc += (h.x <= (uint32_t)a.L.cap) ? h.x : 0u;
-      }
-      s_off[world] = acc;
-    }
-    __syncthreads();
-    const int T = (int)s_off[world];
-    constexpr int NPW = 32 / G;
-    const int lane = threadIdx.x & 31;
-    const int warp = (blockIdx.x * NT + threadIdx.x) >> 5;
-    const int nwarps = (gridDim.x * NT) >> 5;
-    const int k = a.k;
-    for (int base = warp * NPW; base < T; base += nwarps * NPW) {
-      const int q = base + lane / G;
-      const bool active = q < T;
-      int s = 0;
-      if (active) {
-        while (s + 1 < world && (uint32_t)q >= s_off[s + 1]) ++s;
-      }
-      const int j = q - (int)s_off[s];
-      const int32_t v = active ? __ldcv(xch_inbox(self, a.L, a.parity, s) + j) : 0;
-      const int64_t lv = (int64_t)v - a.lo;
-      const bool ok = active && lv >= 0 && lv < a.n_local;
-      if (active && !ok && (lane & (G - 1)) == 0) latch(a.err, E_STATE);
-      int64_t rs = 0, d = 0;
-      if (ok) {
-        row_extent(a.indptr, lv, &rs, &d);
-      }
-      bool valid;
-      int slot, cnt;
-      int32_t u;
-      if (G == 32 && a.biased) {
-        uint32_t pos;
-        cnt = sample_node_biased(ok, v, rs, d, k, a.layer, a.key, a.weights, &pos);
-        slot = lane;
-        valid = lane < cnt;
-        u = valid ? __ldg(a.indices + rs + pos) : -1;
-      } else {
-        sample_node<G>(ok, v, rs, d, k, a.layer, a.key, a.indices, &valid, &slot, &u, &cnt);
-      }
-      char *req = a.peers.base[s];
-      if (active && (lane & (G - 1)) == 0) xch_ret_cnt(req, a.L, a.parity, a.rank)[j] = cnt;
-      if (valid) xch_ret_rows(req, a.L, a.parity, a.rank)[(int64_t)j * a.L.kmax + slot] = u;
-    }
-  }
-  if (last_block_done(&a.hdr->done)) {
-    for (int s = 0; s < world; ++s)
-      st_release_sys(xch_ret_flag(a.peers.base[s], a.L, a.parity, a.rank), a.seq);
-  }
-}
-
-struct UnpermuteArgs {
-  const int32_t *frontier;
-  int32_t layer, k;
-  int32_t rank, parity;
-  unsigned long long seq;
-  Bounds bd;
-  XchLayout L;
-  char *self;
-  const int32_t *perm;
-  LayerBufs buf;
-  const WsPersist *persist;
-  int32_t *src_out;         // dst copy
-  WsHeader *hdr;
-  int *err;
-};
-
-// Reshuffle consumer ("transferred back to the GPU requesting"):
-// frontier node i reads its row from the owner's return slot perm[i]; the
-// edge slots, counts, dst copy and marks are written as the local sample does.
-template <int G>
-__global__ void __launch_bounds__(NT) k_unpermute_mark(UnpermuteArgs a) {
-  const int world = a.bd.world;
-  if (!wait_flags(xch_ret_flag(a.self, a.L, a.parity, 0), world, a.seq, a.err)) return;
-  const uint32_t epoch = a.persist->epoch + 1u + (uint32_t)a.layer;
-  const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
-  const int lim = F > a.L.cap ? 0 : F;
-  constexpr int NPW = 32 / G;
-  const int lane = threadIdx.x & 31;
-  const int t = lane & (G - 1);
-  const int warp = (blockIdx.x * NT + threadIdx.x) >> 5;
-  const int nwarps = (gridDim.x * NT) >> 5;
-  const int k = a.k;
-  for (int base = warp * NPW; base < lim; base += nwarps * NPW) {
-    const int i = base + lane / G;
-    if (i >= lim) continue;
-    const int32_t v = __ldg(a.frontier + i);
-    if (t == 0) a.src_out[i] = v;
-    if (v < 0 || v >= a.bd.b[world]) {  // latched by the bucket kernel
-      if (t == 0) a.buf.cnt[i] = 0;
-      continue;
-    }
-    const int o = owner_of(a.bd, v);
-    const int j = __ldg(a.perm + i);
-    const int c = __ldcv(xch_ret_cnt(a.self, a.L, a.parity, o) + j);
-    if (t == 0) {
-      a.buf.cnt[i] = c;
-      mark_dst(a.buf, v, i, F, a.layer, epoch, a.err);
-    }
-    if (t < c) {
-      const int32_t u = __ldcv(xch_ret_rows(a.self, a.L, a.parity, o) + (int64_t)j * a.L.kmax + t);
-      const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)t;
-      a.buf.rows[q] = u;
-      mark(a.buf, u, epoch, (uint32_t)F + q);
-    }
-  }
-}
-
-// ------------------------------------------- scan as look-back (world > 1)
-// Single-pass decoupled look-back over edge slots (tile status word:
-// [63:62] flag 3 = not ready, 1 = aggregate, 2 = inclusive; [61:31] first
-// count; [30:0] valid count; status[0] = tile ticket; all ones at start).
-constexpr int SCAN_ITEMS = 8;
-constexpr int SCAN_TILE = NT * SCAN_ITEMS;
-constexpr unsigned long long ST_VAL_MASK = (1ull << 62) - 1;
-constexpr unsigned long long ST_AGG = 1ull << 62;
-constexpr unsigned long long ST_INC = 2ull << 62;
-
-struct ScanArgs {
-  int32_t layer, k;
-  LayerBufs buf;
-  const WsPersist *persist;
-  int32_t *indptr_out;
-  int32_t *src_ids_out;
-  int32_t *indices_out;
-  WsHeader *hdr;
-};
-
-__global__ void __launch_bounds__(NT) k_scan_assign(ScanArgs a) {
-  __shared__ unsigned long long s_warp[NT / 32];
-  __shared__ unsigned long long s_prefix;
-  __shared__ uint32_t s_tile;
-  const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
-  const uint32_t epoch = a.persist->epoch + 1u + (uint32_t)a.layer;
-  const int k = a.k;
-  const FastDiv fd = make_fastdiv((uint32_t)k);
-  const LayerBufs &B = a.buf;
-  const uint32_t total = (uint32_t)((int64_t)F * k);
-  const int64_t ntiles = total > 0 ? ((int64_t)total + SCAN_TILE - 1) / SCAN_TILE : 1;
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  unsigned long long *ticket = B.status;
-  unsigned long long *st = B.status + 1;
-
-  while (true) {
-    if (tid == 0) s_tile = (uint32_t)(atomicAdd(ticket, 1ull) + 1ull);  // ticket starts at ~0
-    __syncthreads();
-    const int64_t tile = s_tile;
-    __syncthreads();
-    if (tile >= ntiles) break;
-    const uint32_t q0 = (uint32_t)(tile * SCAN_TILE) + (uint32_t)tid * SCAN_ITEMS;
-
-    uint32_t vbits = 0, fbits = 0;
-    int32_t c[SCAN_ITEMS], u[SCAN_ITEMS];
-#pragma unroll
-    for (int j = 0; j < SCAN_ITEMS; ++j) {
-      const uint32_t q = q0 + j;
-      c[j] = -1;
-      u[j] = 0;
-      if (q < total) {
-        const uint32_t i = fdiv(q, fd);
-        c[j] = __ldg(B.cnt + i) - (int32_t)(q - i * (uint32_t)k);
-        u[j] = __ldg(B.rows + q);
-      }
-    }
-#pragma unroll
-    for (int j = 0; j < SCAN_ITEMS; ++j) {
-      if (c[j] > 0) {
-        vbits |= 1u << j;
-        if (map_get(B, u[j], epoch) == mword(B, epoch, u[j], (uint32_t)F + q0 + j)) fbits |= 1u << j;
-      }
-    }
-    const unsigned long long mine = pack2(__popc(vbits), __popc(fbits));
-
-    unsigned long long incl = mine;
-#pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-      const unsigned long long y = __shfl_up_sync(FULL_MASK, incl, off);
-      if (lane >= off) incl += y;
-    }
-    if (lane == 31) s_warp[wid] = incl;
-    __syncthreads();
-    if (wid == 0) {
-      unsigned long long w = lane < NT / 32 ? s_warp[lane] : 0ull;
-#pragma unroll
-      for (int off = 1; off < NT / 32; off <<= 1) {
-        const unsigned long long y = __shfl_up_sync(FULL_MASK, w, off);
-        if (lane >= off) w += y;
-      }
-      if (lane < NT / 32) s_warp[lane] = w;
-    }
-    __syncthreads();
-    const unsigned long long thread_excl = (wid ? s_warp[wid - 1] : 0ull) + incl - mine;
-    const unsigned long long agg = s_warp[NT / 32 - 1];
-
-    if (wid == 0) {  // decoupled look-back
-      unsigned long long prefix = 0;
-      if (tile == 0) {
-        if (lane == 0) *(volatile unsigned long long *)&st[0] = ST_INC | agg;
-      } else {
-        if (lane == 0) *(volatile unsigned long long *)&st[tile] = ST_AGG | agg;
-        int64_t idx = tile - 1;
-        while (true) {
-          const int64_t p = idx - lane;
-          unsigned long long s = ST_INC;  // virtual inclusive zero before tile 0
-          if (p >= 0) {
-            do {
-              s = ld_volatile_u64(&st[p]);
-            } while ((s >> 62) == 3ull);
-          }
-          const unsigned incm = __ballot_sync(FULL_MASK, (s >> 62) == 2ull);
-          const int stop = incm ? (__ffs(incm) - 1) : 31;
-          unsigned long long v = (lane <= stop) ? (s & ST_VAL_MASK) : 0ull;
-#pragma unroll
-          for (int off = 16; off > 0; off >>= 1) v += __shfl_xor_sync(FULL_MASK, v, off);
-          prefix += v;
-          if (incm) break;
-          idx -= 32;
-        }
-        if (lane == 0) *(volatile unsigned long long *)&st[tile] = ST_INC | (prefix + agg);
-      }
-      if (lane == 0) s_prefix = prefix;
-    }
-    __syncthreads();
-    const unsigned long long base = s_prefix + thread_excl;
-    uint32_t pv = (uint32_t)(base & 0x7fffffffull);
-    uint32_t pf = (uint32_t)((base >> 31) & 0x7fffffffull);
-#pragma unroll
-    for (int j = 0; j < SCAN_ITEMS; ++j) {
-      const uint32_t q = q0 + j;
-      if (q < total) {
-        const uint32_t i = fdiv(q, fd);
-        if (q == i * (uint32_t)k) a.indptr_out[i] = (int32_t)pv;
-        if (fbits & (1u << j)) {
-          const uint32_t nid = (uint32_t)F + pf;
-          map_put(B, u[j], epoch, nid);
-          a.src_ids_out[nid] = u[j];
-        }
-        pv += (vbits >> j) & 1u;
-        pf += (fbits >> j) & 1u;
-      }
-    }
-    if (tile == ntiles - 1 && tid == 0) {
-      const unsigned long long tot = s_prefix + agg;
-      const int32_t E = (int32_t)(tot & 0x7fffffffull);
-      const int32_t nnew = (int32_t)((tot >> 31) & 0x7fffffffull);
-      a.indptr_out[F] = E;
-      a.hdr->E[a.layer] = E;
-      a.hdr->S[a.layer] = F + nnew;
-      a.hdr->F[a.layer + 1] = F + nnew;
-      a.hdr->sizes[3 * a.layer + 0] = F;
-      a.hdr->sizes[3 * a.layer + 1] = F + nnew;
-      a.hdr->sizes[3 * a.layer + 2] = E;
-    }
-  }
-}
-
-__global__ void __launch_bounds__(NT) k_write_indices(ScanArgs a) {
-  const int F = ld_volatile_i32(&a.hdr->F[a.layer]);
-  const uint32_t epoch = a.persist->epoch + 1u + (uint32_t)a.layer;
-  phase_indices(F, a.k, a.buf, epoch, a.indptr_out, a.indices_out, grid_span((int64_t)F * a.k));
-}
-
 // fp32 edge weights -> 16.16 fixed point a = floor(w * 2^16), w in [0, 2^16)
 // (R24); an invalid weight is counted in *bad.
 __global__ void k_weights_fixed(const float *w, int64_t n, uint32_t *out, int *bad) {
@@ -1770,36 +1365,6 @@ __global__ void __launch_bounds__(NT) k_random_walk(const int32_t *starts, int64
       }
       tr[l + 1] = v;
     }
-  }
-}
-
-// end of a stage-by-stage call: advance the workspace epoch
-__global__ void k_epoch_advance(WsPersist *persist, uint32_t L, LayerBufs b0) {
-  if (hash_clear_due(persist, persist->epoch, L, b0.mask, b0.first)) hash_cleared(persist, persist->epoch, b0.mask, b0.first);
-  persist->epoch += L;
-}
-
-// start of a stage-by-stage call on the compact direct map: zero it when the
-// call enters a new epoch window (k_map_begin then moves the epoch there)
-__global__ void k_map_clear(WsPersist *persist, uint32_t L, LayerBufs b0, LayerBufs b1) {
-  const uint32_t e0s = dwin_start(*(volatile const uint32_t *)&persist->epoch, L);
-  if (!dclear_due(persist, e0s)) return;
-  map_zero(b0, b1, blockIdx.x * (int64_t)blockDim.x + threadIdx.x, (int64_t)gridDim.x * blockDim.x);
-}
-__global__ void k_map_begin(WsPersist *persist, uint32_t L) {
-  const uint32_t e0s = dwin_start(persist->epoch, L);
-  persist->dwin = e0s / DWIN + 1u;
-  persist->epoch = e0s;
-}
-
-// start of a stage-by-stage call on a hashed relabel map: zero the table
-// when a tag could repeat (the same test k_epoch_advance applies at the end)
-__global__ void k_hash_clear(WsPersist *persist, uint32_t L, LayerBufs b0, LayerBufs b1) {
-  if (!hash_clear_due(persist, persist->epoch, L, b0.mask, b0.first)) return;
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i <= (int64_t)b0.mask;
-       i += (int64_t)gridDim.x * blockDim.x) {
-    b0.first[i] = 0ull;
-    b1.first[i] = 0ull;
   }
 }
 

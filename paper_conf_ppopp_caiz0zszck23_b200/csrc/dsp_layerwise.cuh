@@ -1,28 +1,31 @@
 // dsp_layerwise.cuh -- layer-wise CSP (Sec. 4.2, Eq. 2;
 // Table 7 "layer-wise sampling without replacement"; R28-R30).
 //
-// Per layer l with layer size n:
-//   k_lw_alloc        (1 block)  W_u = deg u read from the OWNER's indptr over
-//                                peer memory (8 B per frontier node instead of
-//                                its adjacency list), exclusive scan
-//                                P, n Philox draws r = mulhi64(word, T) mapped
-//                                to the frontier interval containing r (Eq. 2,
-//                                with replacement), counts c_u, slot offsets,
-//                                then the sampling tasks (u, c_u) pushed to
-//                                the owners' inboxes (shuffle).
-//   k_lw_sample_remote (grid)    owner side: one warp per task, c_u <= 32 by
-//                                the warp Floyd of the node-wise path, whole
-//                                rows when deg <= c_u; rows written straight
-//                                into the requester's return slots.
-//   k_lw_sample_big   (grid)     tasks with 32 < c_u < deg: one block per task,
-//                                draws in parallel, Floyd's resolution by one
-//                                thread against a shared-memory hash set,
-//                                bitonic sort; then the return flags.
-//   k_lw_collect      (grid)     requester: dst marks + first-occurrence marks
-//                                of the returned rows (epoch-tagged map).
-//   k_lw_finish       (1 block)  scan over the <= n edge slots, relabel,
-//                                indptr / indices / src_ids, sizes.
-// At world 1 the "peer" is the ctx itself; the same kernels run.
+// Per layer l with layer size n, phases of ONE cooperative launch per rank
+// and call (k_lw_persistent at world 1, k_lw_multi at world > 1), separated by
+// grid barriers:
+//   alloc   (block 0)  W_u = deg u read from the OWNER's indptr over peer
+//                      memory (8 B per frontier node instead of its adjacency
+//                      list), exclusive scan P, n Philox draws
+//                      r = mulhi64(word, T) mapped to the frontier interval
+//                      containing r (Eq. 2, with replacement), counts c_u,
+//                      slot offsets, then the sampling tasks (u, c_u) pushed to
+//                      the owners' inboxes (shuffle).
+//   sample  (grid)     owner side: one warp per task, c_u <= 32 by the warp
+//                      Floyd of the node-wise path, whole rows when
+//                      deg <= c_u; rows written straight into the requester's
+//                      return slots.
+//   big     (grid)     tasks with 32 < c_u < deg: one block per task, draws in
+//                      parallel, Floyd's resolution by one thread against a
+//                      shared-memory hash set, bitonic sort; then the return
+//                      flags.
+//   collect (grid)     requester: dst marks + first-occurrence marks of the
+//                      returned rows (epoch-tagged map).
+//   finish  (block 0)  scan over the <= n edge slots, relabel, indptr /
+//                      indices / src_ids, sizes.
+// At world 1 the "peer" is the ctx itself (its exchange slots sit in the
+// workspace).  The phase bodies take PERS = true (inside the persistent
+// kernel: the flag waits of a phase that follows a grid barrier are skipped).
 #pragma once
 #include "dsp_kernels.cuh"
 
@@ -276,10 +279,6 @@ __device__ __forceinline__ void lw_alloc_body(const LwArgs &a, unsigned long lon
     }
   }
 }
-__global__ void __launch_bounds__(LWT) k_lw_alloc(LwArgs a) {
-  extern __shared__ unsigned long long lw_alloc_smem[];
-  lw_alloc_body<false>(a, lw_alloc_smem);
-}
 
 // Owner side: every task received in this layer, one warp each.
 template <bool PERS>
@@ -338,7 +337,6 @@ __device__ __forceinline__ void lw_sample_remote_body(const LwArgs &a) {
   }
   if (!PERS && a.sys) __threadfence_system();  // this kernel's peer stores, before k_lw_sample_big's flags
 }
-__global__ void __launch_bounds__(NT) k_lw_sample_remote(LwArgs a) { lw_sample_remote_body<false>(a); }
 
 // Tasks with 32 < c < deg: Floyd over c draws with a shared-memory hash set.
 // Dynamic shared memory: kp (pow2 >= c) positions + 2 kp hash slots.
@@ -405,10 +403,6 @@ __device__ __forceinline__ void lw_sample_big_body(const LwArgs &a, int kp_max, 
       st_release_flag(lw_ret_flag(a.peers.base[s], a.L, a.parity, a.rank), a.seq, a.sys);
   }
 }
-__global__ void __launch_bounds__(LWT) k_lw_sample_big(LwArgs a, int kp_max) {
-  extern __shared__ int32_t lw_smem[];
-  lw_sample_big_body<false>(a, kp_max, lw_smem);
-}
 
 // Requester: dst copy + marks, first-occurrence marks of the returned rows.
 template <bool PERS>
@@ -431,7 +425,6 @@ __device__ __forceinline__ void lw_collect_body(const LwArgs &a) {
     if (q - a.w.off[i] < __ldcv(ret_cnt + i)) mark(a.first, __ldcv(ret_rows + q), epoch, (uint32_t)F + (uint32_t)q);
   }
 }
-__global__ void __launch_bounds__(NT) k_lw_collect(LwArgs a) { lw_collect_body<false>(a); }
 
 // Requester: block l from the marks (one block; Q <= n <= 8192 slots).
 __device__ __forceinline__ void lw_finish_body(const LwArgs &a) {
@@ -484,7 +477,6 @@ __device__ __forceinline__ void lw_finish_body(const LwArgs &a) {
     a.hdr->sizes[3 * a.layer + 2] = E;
   }
 }
-__global__ void __launch_bounds__(LWT) k_lw_finish(LwArgs a) { lw_finish_body(a); }
 
 // World 1: every layer of the call in ONE cooperative launch (the per-layer
 // kernels above are launch- and drain-bound at Table 7's sizes: ~1000 nodes

@@ -92,22 +92,16 @@ int64_t next_pow2(int64_t x) {
   return p;
 }
 
-int group_of(int k) {
-  int g = 1;
-  while (g < k) g <<= 1;
-  return g;
-}
-
 // Per-layer bounds (dsp_sample_bounds) and the workspace plan:
-//   persist | hdr | agg[2][MAX_PERSIST_BLOCKS] | cnt[2][max_F] | perm[max_F] | rows[2][max_slots]
-//   | status[2][status_len] | first[2][N]
+//   persist | hdr | first[2][N] (| first32[2][N] | hash[2][cap]) | agg[2][MAX_PERSIST_BLOCKS]
+//   | cnt[2][max_F] | perm[max_F] | rows[2][max_slots]
 struct Plan {
   int L;
   int64_t F[DSP_MAX_LAYERS + 1];   // max frontier per layer
   int64_t E[DSP_MAX_LAYERS];       // max edges
   int64_t S[DSP_MAX_LAYERS];       // max src
-  int64_t max_F, max_slots, status_len;
-  size_t off_hdr, off_agg, off_cnt[2], off_perm, off_rows[2], off_status[2], off_first[2], bytes;
+  int64_t max_F, max_slots;
+  size_t off_hdr, off_agg, off_cnt[2], off_perm, off_rows[2], off_first[2], bytes;
   size_t off_first32[2];            // compact direct map [2][N] (N <= DIRECT_MAP_MAX_N), else 0
   bool direct32;                    // node-wise relabel through the compact direct map
   int64_t hash_cap;                 // > 0: relabel hash table of hash_cap slots per parity (else direct map)
@@ -134,7 +128,7 @@ struct dsp_ctx {
   int64_t feat_bytes = 0;
   // cold-feature tier
   bool tiered = false;
-  bool cold_regloads = false;         // env DSP_COLD_REGLOADS=1 (measurement switch)
+  bool cold_regloads = false;         // DSP_OPT_GATHER_REGLOADS: cold rows by register loads
   int32_t *d_fpos = nullptr;          // feature position list [n_local]
   float *h_cold = nullptr;            // cold rows (pinned host, UVA-mapped)
   int64_t cold_bytes = 0;
@@ -175,20 +169,19 @@ struct dsp_ctx {
   int *h_err = nullptr;
   int num_sms = 148;
   int persist_blocks_per_sm = 1;
-  int lane_rounds = 8;  // DSP_LANE_ROUNDS (tuning knob, results unchanged; 8 measured best with 4 streams)
-  int stage_bps = 8;    // DSP_STAGE_BPS: blocks per SM of the owner-sample / unpermute kernels (tuning knob)
-  int relabel_mode = 0; // DSP_RELABEL = direct | direct64 | hash (default: by N; results unchanged)
-  int loader_warps = 4; // DSP_LOADER_WARPS = 2, 4 or 8 (tuning knob, results unchanged)
-  int loader_rows = 32;  // DSP_LOADER_ROWS: rows per TMA chunk, <= 32 (tuning knob, results unchanged)
+  // dsp_set_option (performance only; results are identical for every value)
+  int lane_rounds = 8;  // DSP_OPT_LANE_ROUNDS (8 measured best with 4 streams)
+  int relabel_mode = 0; // DSP_OPT_RELABEL_MAP: 0 by N, 1 compact direct, 2 hash, 3 8-byte direct
+  int loader_warps = 4; // DSP_OPT_LOADER_WARPS: 2, 4 or 8
+  int loader_rows = 32;  // DSP_OPT_LOADER_ROWS: rows per TMA chunk, <= 32
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
-  bool multi_staged = false;  // DSP_MULTI_STAGED=1: world > 1 node-wise calls stage by stage (A/B switch)
-  bool lw_staged = false;     // DSP_LW_STAGED=1: layer-wise calls stage by stage (A/B switch)
-  bool walk_staged = false;   // DSP_WALK_STAGED=1: world > 1 random walks stage by stage (A/B switch)
-  bool gather_reg = false;    // DSP_GATHER_REG=1: standalone gathers with register loads (A/B switch)
+  bool gather_reg = false;    // DSP_OPT_GATHER_REGLOADS: standalone gathers with register loads
+  bool tma_unavailable = false;  // the TMA gather's shared memory could not be configured
   WsHeader *d_walk_hdr = nullptr;  // grid-barrier counter of k_walk_multi
   int walk_blocks_per_sm = 2;
   cudaStream_t aux = nullptr;  // virtual ranks sharing a GPU: each rank's persistent launch on its own stream
   cudaEvent_t aux_ev[2] = {nullptr, nullptr};
+  cudaEvent_t flush_ev = nullptr;  // dsp_pipeline_flush: orders a pending gather after its call's stream
   int gather_blocks_per_sm = 1;
   // pipelined steps: per workspace, the gather owed by its previous
   // DSP_PIPELINED call (row count in the workspace's WsPersist::pend_n[parity])
@@ -303,7 +296,6 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L, int 
     p.max_F = std::max(p.max_F, p.F[l]);
     p.max_slots = std::max(p.max_slots, p.E[l]);
   }
-  p.status_len = align_up((size_t)((p.max_slots + SCAN_TILE - 1) / SCAN_TILE + 2), 2);
   size_t o = plan_common(p, N);
   // relabel_mode: 0 = by N, 1 = direct, 2 = hashed (DSP_RELABEL)
   int64_t max_keys = 0;
@@ -330,10 +322,6 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L, int 
   for (int b = 0; b < 2; ++b) {
     p.off_rows[b] = o;
     o = align_up(o + sizeof(int32_t) * p.max_slots, 256);
-  }
-  for (int b = 0; b < 2; ++b) {
-    p.off_status[b] = o;
-    o = align_up(o + sizeof(unsigned long long) * p.status_len, 256);
   }
   p.bytes = o;
   return p;
@@ -495,7 +483,6 @@ LayerBufs bufs_of(const Call &k, int parity) {
   LayerBufs b{};
   b.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt[parity]);
   b.rows = reinterpret_cast<int32_t *>(k.ws + k.plan.off_rows[parity]);
-  b.status = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_status[parity]);
   b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_first[parity]);
   b.mask = 0;
   b.first32 = nullptr;
@@ -838,152 +825,36 @@ dsp_status launch_gather(dsp_ctx *c, const GatherArgs &g, int64_t n_host, cudaSt
   return DSP_OK;
 }
 
-// gather owed by a workspace's last pipelined call (the device row count)
-dsp_status flush_one(dsp_ctx *c, dsp_ctx::Pending &pd) {
+// Gather owed by a workspace's last pipelined call (the device row count),
+// enqueued on `st`.  When the pipelined call ran on another stream, `st`
+// first waits for everything issued there so far (event), so the gather reads
+// that call's finished src_ids and row count on any stream.
+dsp_status flush_one(dsp_ctx *c, dsp_ctx::Pending &pd, cudaStream_t st) {
   if (!pd.active) return DSP_OK;
   DeviceGuard g(c->device);
+  if (static_cast<cudaStream_t>(pd.stream) != st) {
+    if (!c->flush_ev) CUDA_TRY(c, cudaEventCreateWithFlags(&c->flush_ev, cudaEventDisableTiming));
+    CUDA_TRY(c, cudaEventRecord(c->flush_ev, static_cast<cudaStream_t>(pd.stream)));
+    CUDA_TRY(c, cudaStreamWaitEvent(st, c->flush_ev, 0));
+  }
   const WsPersist *ps = reinterpret_cast<const WsPersist *>(pd.ws);
   GatherArgs a = make_gather(c, pd.ids, 0, &ps->pend_n[(pd.calls + 1) & 1], pd.out);
-  dsp_status st = launch_gather(c, a, 0, static_cast<cudaStream_t>(pd.stream));
-  if (st != DSP_OK) return st;
+  dsp_status s = launch_gather(c, a, 0, st);
+  if (s != DSP_OK) return s;
   pd.active = false;
   return DSP_OK;
 }
 
-dsp_status stage_flush(dsp_ctx *c, const char *ws) {
+dsp_status stage_flush(dsp_ctx *c, const char *ws, cudaStream_t st) {
   for (auto &p : c->pend)
-    if (p.active && p.ws == ws) return flush_one(c, p);
+    if (p.active && p.ws == ws) return flush_one(c, p, st);
   return DSP_OK;
 }
-
-// ------------------------------------------------ world > 1, stage by stage
-dsp_status stage_clear(Call &k, int l) {  // look-back scan status + ticket of layer l
-  DeviceGuard g(k.c->device);
-  CUDA_TRY(k.c, cudaMemsetAsync(k.ws + k.plan.off_status[l & 1], 0xFF,
-                                sizeof(unsigned long long) * k.plan.status_len, k.stream));
-  return DSP_OK;
-}
-
-template <int G>
-void launch_remote(const RemoteSampleArgs &a, int grid, cudaStream_t s) {
-  k_sample_remote<G><<<grid, NT, 0, s>>>(a);
-}
-template <int G>
-void launch_unpermute(const UnpermuteArgs &a, int grid, cudaStream_t s) {
-  k_unpermute_mark<G><<<grid, NT, 0, s>>>(a);
-}
-
-#define DISPATCH_G(G, FN, ...)                 \
-  switch (G) {                                 \
-    case 1: FN<1>(__VA_ARGS__); break;         \
-    case 2: FN<2>(__VA_ARGS__); break;         \
-    case 4: FN<4>(__VA_ARGS__); break;         \
-    case 8: FN<8>(__VA_ARGS__); break;         \
-    case 16: FN<16>(__VA_ARGS__); break;       \
-    default: FN<32>(__VA_ARGS__); break;       \
-  }
 
 XchPeers peers_of(const dsp_ctx *c) {
   XchPeers p{};
   for (int r = 0; r < DSP_MAX_WORLD; ++r) p.base[r] = r < c->world ? c->peer_xch[r] : nullptr;
   return p;
-}
-
-dsp_status stage_shuffle(Call &k, int l) {
-  dsp_ctx *c = k.c;
-  DeviceGuard g(c->device);
-  BucketArgs a{};
-  a.frontier = frontier_of(k, l);
-  a.F0 = k.num_seeds;
-  a.layer = l;
-  a.k = k.fanouts[l];
-  a.biased = k.biased ? 1 : 0;
-  a.seed_lo = (uint32_t)k.rng_seed;
-  a.seed_hi = (uint32_t)(k.rng_seed >> 32);
-  a.rank = c->rank;
-  a.seq = k.seq0 + 1 + l;
-  a.parity = (int)(a.seq & 1);
-  a.bd = make_bounds(c);
-  a.L = c->xl;
-  a.peers = peers_of(c);
-  a.perm = reinterpret_cast<int32_t *>(k.ws + k.plan.off_perm);
-  a.hdr = k.hdr;
-  a.err = c->d_err;
-  const int64_t need = std::max<int64_t>(1, (k.plan.F[l] + NT - 1) / NT);
-  k_bucket_scatter<<<(int)std::min<int64_t>(need, grid_for(c, 2)), NT, 0, k.stream>>>(a);
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
-}
-
-dsp_status stage_sample_remote(Call &k, int l) {
-  dsp_ctx *c = k.c;
-  DeviceGuard g(c->device);
-  RemoteSampleArgs a{};
-  a.layer = l;
-  a.k = k.fanouts[l];
-  a.biased = k.biased ? 1 : 0;
-  a.weights = c->d_weights;
-  a.key = key_of(k.rng_seed);
-  a.rank = c->rank;
-  a.seq = k.seq0 + 1 + l;
-  a.parity = (int)(a.seq & 1);
-  a.indptr = c->d_indptr;
-  a.indices = c->d_indices;
-  a.lo = c->lo;
-  a.n_local = c->n_local;
-  a.bd = make_bounds(c);
-  a.L = c->xl;
-  a.peers = peers_of(c);
-  a.hdr = k.hdr;
-  a.err = c->d_err;
-  DISPATCH_G(k.biased ? 32 : group_of(a.k), launch_remote, a, grid_for(c, c->stage_bps), k.stream);
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
-}
-
-dsp_status stage_unpermute(Call &k, int l) {
-  dsp_ctx *c = k.c;
-  DeviceGuard g(c->device);
-  UnpermuteArgs a{};
-  a.frontier = frontier_of(k, l);
-  a.layer = l;
-  a.k = k.fanouts[l];
-  a.rank = c->rank;
-  a.seq = k.seq0 + 1 + l;
-  a.parity = (int)(a.seq & 1);
-  a.bd = make_bounds(c);
-  a.L = c->xl;
-  a.self = c->d_xch;
-  a.perm = reinterpret_cast<int32_t *>(k.ws + k.plan.off_perm);
-  a.buf = bufs_of(k, l & 1);
-  a.persist = persist_of(k);
-  a.src_out = k.blocks[l].src_ids;
-  a.hdr = k.hdr;
-  a.err = c->d_err;
-  DISPATCH_G(group_of(a.k), launch_unpermute, a, grid_for(c, c->stage_bps), k.stream);
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
-}
-
-dsp_status stage_scan_indices(Call &k, int l) {
-  dsp_ctx *c = k.c;
-  DeviceGuard g(c->device);
-  ScanArgs s{};
-  s.layer = l;
-  s.k = k.fanouts[l];
-  s.buf = bufs_of(k, l & 1);
-  s.persist = persist_of(k);
-  s.indptr_out = k.blocks[l].indptr;
-  s.src_ids_out = k.blocks[l].src_ids;
-  s.indices_out = k.blocks[l].indices;
-  s.hdr = k.hdr;
-  const int64_t tiles = std::max<int64_t>(1, (k.plan.E[l] + SCAN_TILE - 1) / SCAN_TILE);
-  k_scan_assign<<<(int)std::min<int64_t>(tiles, grid_for(c, 4)), NT, 0, k.stream>>>(s);
-  CUDA_TRY(c, cudaGetLastError());
-  const int64_t need = std::max<int64_t>(1, (k.plan.E[l] + NT - 1) / NT);
-  k_write_indices<<<(int)std::min<int64_t>(need, grid_for(c, 8)), NT, 0, k.stream>>>(s);
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
 }
 
 // ------------------------------------------------ layer-wise stages
@@ -1025,7 +896,7 @@ LwArgs lw_args(Call &k, int l) {
   a.hdr = k.hdr;
   a.err = c->d_err;
   a.sys = c->world > 1 ? 1 : 0;
-  if (c->world == 1 && !c->lw_staged && k.plan.off_lxch)  // persistent world-1 call: its own exchange slots
+  if (c->world == 1 && k.plan.off_lxch)  // world-1 call: its own exchange slots
     a.peers.base[0] = k.ws + k.plan.off_lxch;
   return a;
 }
@@ -1081,47 +952,6 @@ dsp_status stage_lw_persistent(Call &k, int share = 1) {
   return DSP_OK;
 }
 
-dsp_status stage_lw(Call &k, int l, int step) {
-  dsp_ctx *c = k.c;
-  DeviceGuard g(c->device);
-  const LwArgs a = lw_args(k, l);
-  const int64_t F = k.plan.F[l], n = k.fanouts[l];
-  switch (step) {
-    case 0:
-      k_lw_alloc<<<1, LWT, LW_ALLOC_SMEM, k.stream>>>(a);
-      break;
-    case 1: {  // one warp per task; at most world * F tasks arrive
-      const int64_t need = std::max<int64_t>(1, (c->world * F + NT / 32 - 1) / (NT / 32));
-      k_lw_sample_remote<<<(int)std::min<int64_t>(need, grid_for(c, 8)), NT, 0, k.stream>>>(a);
-      break;
-    }
-    case 2: {
-      const int kp = (int)next_pow2(k.plan.ncap);
-      k_lw_sample_big<<<(int)std::min<int64_t>(k.plan.big_cap, 32), LWT,
-                        sizeof(int32_t) * 3 * (size_t)kp, k.stream>>>(a, kp);
-      break;
-    }
-    case 3: {
-      const int64_t need = std::max<int64_t>(1, (std::max(F, n) + NT - 1) / NT);
-      k_lw_collect<<<(int)std::min<int64_t>(need, grid_for(c, 8)), NT, 0, k.stream>>>(a);
-      break;
-    }
-    default:
-      k_lw_finish<<<1, LWT, 0, k.stream>>>(a);
-      break;
-  }
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
-}
-
-dsp_status stage_gather_dev(Call &k) {
-  dsp_ctx *c = k.c;
-  DeviceGuard g(c->device);
-  const int l = k.L - 1;
-  GatherArgs a = make_gather(c, k.blocks[l].src_ids, 0, &k.hdr->S[l], k.feat_out);
-  return launch_gather(c, a, 0, k.stream);
-}
-
 // ------------------------------------------------------------- end of call
 dsp_status stage_end_async(Call &k) {
   dsp_ctx *c = k.c;
@@ -1169,80 +999,25 @@ dsp_status run_calls(std::vector<Call> &calls) {
 #define EACH(STAGE)                                   \
   for (auto &k : calls)                               \
     if ((st = (STAGE)) != DSP_OK) return st;
-  // a non-pipelined call first settles a pending pipelined gather; so does a
-  // pipelined call of the stage-by-stage paths (no loader warps there)
-  const bool multi = calls[0].c->world > 1 && !calls[0].layerwise && !calls[0].c->multi_staged;
-  const bool lw_pers = calls[0].layerwise && !calls[0].c->lw_staged;
+  // a non-pipelined call first settles a pending pipelined gather of its workspace
   for (auto &k : calls)
-    if ((!k.pipelined || (k.c->world > 1 && !multi) || (k.layerwise && !lw_pers)) &&
-        (st = stage_flush(k.c, k.ws)) != DSP_OK)
-      return st;
+    if (!k.pipelined && (st = stage_flush(k.c, k.ws, k.stream)) != DSP_OK) return st;
   EACH(stage_begin(k));
   if (calls[0].c->world == 1 && !calls[0].layerwise) {
     EACH(stage_persistent(k));
-  } else if (multi) {
-    std::vector<int> share(calls.size(), 0);
-    for (size_t i = 0; i < calls.size(); ++i)
-      for (auto &o : calls) share[i] += o.c->device == calls[i].c->device ? 1 : 0;
-    for (size_t i = 0; i < calls.size(); ++i)
-      if ((st = stage_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
-    for (size_t i = 0; i < calls.size(); ++i)
-      if ((st = join_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
-  } else if (lw_pers) {  // gather (fused, or the previous call's when pipelined) and epoch inside
-    std::vector<int> share(calls.size(), 0);
-    for (size_t i = 0; i < calls.size(); ++i)
-      for (auto &o : calls) share[i] += o.c->device == calls[i].c->device ? 1 : 0;
-    for (size_t i = 0; i < calls.size(); ++i)
-      if ((st = stage_lw_persistent(calls[i], share[i])) != DSP_OK) return st;
-    for (size_t i = 0; i < calls.size(); ++i)
-      if ((st = join_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
   } else {
-    for (int l = 0; l < calls[0].L; ++l) {
-      if (calls[0].layerwise) {
-        for (int step = 0; step < 5; ++step) EACH(stage_lw(k, l, step));
-        continue;
-      }
-      if (l == 0)
-        for (auto &k : calls)
-          if (k.plan.direct32) {
-            DeviceGuard g(k.c->device);
-            k_map_clear<<<grid_for(k.c, 4), NT, 0, k.stream>>>(persist_of(k), (uint32_t)k.L, bufs_of(k, 0),
-                                                                bufs_of(k, 1));
-            k_map_begin<<<1, 1, 0, k.stream>>>(persist_of(k), (uint32_t)k.L);
-            CUDA_TRY(k.c, cudaGetLastError());
-          } else if (k.plan.hash_cap > 0) {
-            DeviceGuard g(k.c->device);
-            k_hash_clear<<<grid_for(k.c, 4), NT, 0, k.stream>>>(persist_of(k), (uint32_t)k.L, bufs_of(k, 0),
-                                                                 bufs_of(k, 1));
-            CUDA_TRY(k.c, cudaGetLastError());
-          }
-      EACH(stage_clear(k, l));
-      EACH(stage_shuffle(k, l));
-      EACH(stage_sample_remote(k, l));
-      EACH(stage_unpermute(k, l));
-      EACH(stage_scan_indices(k, l));
-    }
-    for (auto &k : calls) {
-      if (k.feat_out && k.pipelined) {  // this call's rows: gathered by the next call / flush
-        DeviceGuard g(k.c->device);
-        dsp_ctx::Pending *pd = k.c->pending_of(k.ws);
-        if (!pd) return fail(k.c, DSP_ERR_STATE, "more than 8 workspaces with pending pipelined gathers");
-        pd->calls += 1;
-        CUDA_TRY(k.c, cudaMemcpyAsync(&persist_of(k)->pend_n[(pd->calls + 1) & 1], &k.hdr->S[k.L - 1],
-                                      sizeof(int32_t), cudaMemcpyDeviceToDevice, k.stream));
-        pd->ids = k.blocks[k.L - 1].src_ids;
-        pd->out = k.feat_out;
-        pd->stream = k.stream;
-        pd->active = true;
-      } else if (k.feat_out && (st = stage_gather_dev(k)) != DSP_OK) {
+    // one cooperative launch per rank: k_csp_multi (node-wise, world > 1) or
+    // k_lw_persistent / k_lw_multi (layer-wise); ranks sharing a device each
+    // run on their own stream with 1/share of its SMs
+    std::vector<int> share(calls.size(), 0);
+    for (size_t i = 0; i < calls.size(); ++i)
+      for (auto &o : calls) share[i] += o.c->device == calls[i].c->device ? 1 : 0;
+    for (size_t i = 0; i < calls.size(); ++i)
+      if ((st = calls[i].layerwise ? stage_lw_persistent(calls[i], share[i])
+                                   : stage_persistent_multi(calls[i], share[i])) != DSP_OK)
         return st;
-      }
-    }
-    for (auto &k : calls) {
-      DeviceGuard g(k.c->device);
-      k_epoch_advance<<<1, 1, 0, k.stream>>>(persist_of(k), (uint32_t)k.L, bufs_of(k, 0));
-      CUDA_TRY(k.c, cudaGetLastError());
-    }
+    for (size_t i = 0; i < calls.size(); ++i)
+      if ((st = join_persistent_multi(calls[i], share[i])) != DSP_OK) return st;
   }
   EACH(stage_end_async(k));
 #undef EACH
@@ -1291,6 +1066,10 @@ void release(dsp_ctx *c) {
     cudaEventDestroy(c->aux_ev[1]);
     c->aux = nullptr;
   }
+  if (c->flush_ev) {
+    cudaEventDestroy(c->flush_ev);
+    c->flush_ev = nullptr;
+  }
   cudaFree(c->d_lxch);
   cudaFree(c->d_wxch);
   cudaFree(c->d_err);
@@ -1321,39 +1100,6 @@ WalkArgs walk_args(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length,
   return a;
 }
 
-dsp_status walk_stage(dsp_ctx *c, WalkArgs a, int stage, int l, unsigned long long seq0, cudaStream_t st) {
-  DeviceGuard g(c->device);
-  a.step = l;
-  const int grid = grid_for(c, 4);
-  switch (stage) {
-    case 0:
-      k_walk_init<<<(int)std::max<int64_t>(1, std::min<int64_t>((a.n * (a.length + 1) + NT - 1) / NT, grid)), NT, 0,
-                    st>>>(a);
-      break;
-    case 1:
-      a.seq = seq0 + 1 + l;
-      a.parity = (int)(a.seq & 1);
-      k_walk_scatter<<<grid, NT, 0, st>>>(a);
-      break;
-    case 2:
-      a.seq = seq0 + 1 + l;
-      a.parity = (int)(a.seq & 1);
-      k_walk_step<<<grid, NT, 0, st>>>(a);
-      break;
-    case 3:
-      a.seq = seq0 + 1 + a.length;
-      k_walk_done<<<1, 32, 0, st>>>(a);
-      break;
-    default:
-      a.seq = seq0 + 1 + a.length;
-      k_walk_finish<<<(int)std::max<int64_t>(1, std::min<int64_t>((a.n * (a.length + 1) + NT - 1) / NT, grid)), NT,
-                      0, st>>>(a);
-      break;
-  }
-  CUDA_TRY(c, cudaGetLastError());
-  return DSP_OK;
-}
-
 dsp_status check_walk_call(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length, int32_t *traces) {
   if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
   if (length < 1 || length > 1024) return fail(c, DSP_ERR_INVALID_ARG, "length %d not in [1, 1024]", length);
@@ -1374,54 +1120,41 @@ dsp_status run_walks(std::vector<dsp_ctx *> &cs, std::vector<WalkArgs> &as, std:
   const unsigned long long seq0 = cs[0]->wseq;
   for (auto *c : cs)
     if (c->wseq != seq0) return fail(cs[0], DSP_ERR_STATE, "ranks disagree on the number of walk calls");
-  dsp_status st;
   const size_t n = cs.size();
-  if (!cs[0]->walk_staged) {  // one cooperative launch per rank (k_walk_multi)
-    std::vector<int> share(n, 0);
-    for (size_t i = 0; i < n; ++i)
-      for (auto *o : cs) share[i] += o->device == cs[i]->device ? 1 : 0;
-    for (size_t i = 0; i < n; ++i) {
-      dsp_ctx *c = cs[i];
-      DeviceGuard g(c->device);
-      CUDA_TRY(c, cudaMemsetAsync(c->d_walk_hdr, 0, sizeof(WsHeader), ss[i]));
-      cudaStream_t st_i = ss[i];
-      if (share[i] > 1) {  // virtual ranks: each on its own stream with 1/share of the SMs
-        if (!c->aux) {
-          CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking));
-          CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[0], cudaEventDisableTiming));
-          CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[1], cudaEventDisableTiming));
-        }
-        CUDA_TRY(c, cudaEventRecord(c->aux_ev[0], ss[i]));
-        CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->aux_ev[0], 0));
-        st_i = c->aux;
+  // one cooperative launch per rank (k_walk_multi)
+  std::vector<int> share(n, 0);
+  for (size_t i = 0; i < n; ++i)
+    for (auto *o : cs) share[i] += o->device == cs[i]->device ? 1 : 0;
+  for (size_t i = 0; i < n; ++i) {
+    dsp_ctx *c = cs[i];
+    DeviceGuard g(c->device);
+    CUDA_TRY(c, cudaMemsetAsync(c->d_walk_hdr, 0, sizeof(WsHeader), ss[i]));
+    cudaStream_t st_i = ss[i];
+    if (share[i] > 1) {  // virtual ranks: each on its own stream with 1/share of the SMs
+      if (!c->aux) {
+        CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking));
+        CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[0], cudaEventDisableTiming));
+        CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[1], cudaEventDisableTiming));
       }
-      WalkPersistArgs p{};
-      p.a = as[i];
-      p.seq0 = seq0;
-      p.hdr = c->d_walk_hdr;
-      const dim3 grid(std::max(1, c->num_sms * c->walk_blocks_per_sm / share[i])), block(NT);
-      void *args[] = {&p};
-      CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_walk_multi, grid, block, args, 0, st_i));
+      CUDA_TRY(c, cudaEventRecord(c->aux_ev[0], ss[i]));
+      CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->aux_ev[0], 0));
+      st_i = c->aux;
     }
-    for (size_t i = 0; i < n; ++i)
-      if (share[i] > 1) {
-        dsp_ctx *c = cs[i];
-        DeviceGuard g(c->device);
-        CUDA_TRY(c, cudaEventRecord(c->aux_ev[1], c->aux));
-        CUDA_TRY(c, cudaStreamWaitEvent(ss[i], c->aux_ev[1], 0));
-      }
-    for (auto *c : cs) c->wseq = seq0 + 1 + (unsigned long long)length;
-    return DSP_OK;
+    WalkPersistArgs p{};
+    p.a = as[i];
+    p.seq0 = seq0;
+    p.hdr = c->d_walk_hdr;
+    const dim3 grid(std::max(1, c->num_sms * c->walk_blocks_per_sm / share[i])), block(NT);
+    void *args[] = {&p};
+    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_walk_multi, grid, block, args, 0, st_i));
   }
   for (size_t i = 0; i < n; ++i)
-    if ((st = walk_stage(cs[i], as[i], 0, 0, seq0, ss[i])) != DSP_OK) return st;
-  for (int l = 0; l < length; ++l)
-    for (int stage = 1; stage <= 2; ++stage)
-      for (size_t i = 0; i < n; ++i)
-        if ((st = walk_stage(cs[i], as[i], stage, l, seq0, ss[i])) != DSP_OK) return st;
-  for (int stage = 3; stage <= 4; ++stage)
-    for (size_t i = 0; i < n; ++i)
-      if ((st = walk_stage(cs[i], as[i], stage, 0, seq0, ss[i])) != DSP_OK) return st;
+    if (share[i] > 1) {
+      dsp_ctx *c = cs[i];
+      DeviceGuard g(c->device);
+      CUDA_TRY(c, cudaEventRecord(c->aux_ev[1], c->aux));
+      CUDA_TRY(c, cudaStreamWaitEvent(ss[i], c->aux_ev[1], 0));
+    }
   for (auto *c : cs) c->wseq = seq0 + 1 + (unsigned long long)length;
   return DSP_OK;
 }
@@ -1500,44 +1233,28 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
     delete c;
     return fail(nullptr, DSP_ERR_CUDA, "occupancy query for the persistent kernel failed");
   }
-  if (cudaFuncSetAttribute((const void *)k_lw_sample_big, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           (int)sizeof(int32_t) * 3 * LW_MAX_SIZE) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_lw_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  if (cudaFuncSetAttribute((const void *)k_lw_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            (int)std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)LW_MAX_SIZE)) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_lw_multi, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           (int)std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)LW_MAX_SIZE)) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_lw_alloc, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           (int)LW_ALLOC_SMEM) != cudaSuccess) {
+                           (int)std::max(LW_ALLOC_SMEM, sizeof(int32_t) * 3 * (size_t)LW_MAX_SIZE)) != cudaSuccess) {
     cudaGetLastError();
     delete c;
     return fail(nullptr, DSP_ERR_CUDA, "shared-memory attribute of the layer-wise kernel failed");
   }
   c->persist_blocks_per_sm = std::min(occ, occ_pipe);
-  if (getenv("DSP_LANE_ROUNDS")) c->lane_rounds = atoi(getenv("DSP_LANE_ROUNDS"));
-  if (getenv("DSP_STAGE_BPS")) c->stage_bps = std::max(1, std::min(8, atoi(getenv("DSP_STAGE_BPS"))));
-  c->multi_staged = getenv("DSP_MULTI_STAGED") && atoi(getenv("DSP_MULTI_STAGED")) != 0;
-  c->lw_staged = getenv("DSP_LW_STAGED") && atoi(getenv("DSP_LW_STAGED")) != 0;
-  c->walk_staged = getenv("DSP_WALK_STAGED") && atoi(getenv("DSP_WALK_STAGED")) != 0;
-  c->gather_reg = getenv("DSP_GATHER_REG") && atoi(getenv("DSP_GATHER_REG")) != 0;
   if (cudaFuncSetAttribute((const void *)k_gather_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            GTMA_WARPS * LOADER_SLOTS * 16384) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_gather_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                            GTMA_WARPS * LOADER_SLOTS * 16384) != cudaSuccess) {
     cudaGetLastError();
     c->gather_reg = true;  // no TMA gather: register loads
+    c->tma_unavailable = true;
   }
   {
     int ow = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ow, k_walk_multi, NT, 0) == cudaSuccess && ow >= 1)
       c->walk_blocks_per_sm = std::min(ow, 2);
     cudaGetLastError();
-  }
-  if (const char *rm = getenv("DSP_RELABEL"))
-    c->relabel_mode = !strcmp(rm, "hash") ? 2 : !strcmp(rm, "direct") ? 1 : !strcmp(rm, "direct64") ? 3 : 0;
-  if (getenv("DSP_LOADER_ROWS")) c->loader_rows = std::max(1, std::min(32, atoi(getenv("DSP_LOADER_ROWS"))));
-  if (getenv("DSP_LOADER_WARPS")) {
-    const int lw = atoi(getenv("DSP_LOADER_WARPS"));
-    if (lw == 2 || lw == LOADER_WARPS_MAX) c->loader_warps = lw;
   }
   if (c->persist_blocks_per_sm * c->num_sms > MAX_PERSIST_BLOCKS) c->persist_blocks_per_sm = MAX_PERSIST_BLOCKS / c->num_sms;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_gather, NT, 0) != cudaSuccess || occ < 1) {
@@ -1691,7 +1408,7 @@ dsp_status dsp_load_features_tiered(dsp_ctx *c, const float *features, int32_t d
   void *dev_cold = nullptr;
   CUDA_TRY(c, cudaHostGetDevicePointer(&dev_cold, c->h_cold, 0));
   c->tiered = true;
-  c->cold_regloads = getenv("DSP_COLD_REGLOADS") && atoi(getenv("DSP_COLD_REGLOADS")) != 0;
+  c->cold_regloads = c->gather_reg;
   c->peer_feat[c->rank] = c->d_feat;
   c->peer_fpos[c->rank] = nc > 0 ? c->d_fpos : nullptr;  // all hot: fpos is the identity
   c->peer_cold[c->rank] = static_cast<const float *>(dev_cold);
@@ -2065,12 +1782,45 @@ dsp_status dsp_set_persistent_blocks(dsp_ctx *c, int32_t blocks) {
   return DSP_OK;
 }
 
+dsp_status dsp_set_option(dsp_ctx *c, int32_t option, int64_t value) {
+  if (!c) return DSP_ERR_INVALID_ARG;
+  c->err.clear();
+  switch (option) {
+    case DSP_OPT_RELABEL_MAP:
+      if (value < 0 || value > 3) return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_RELABEL_MAP %lld not in [0, 3]", (long long)value);
+      if (c->reserved || c->lw_reserved)
+        return fail(c, DSP_ERR_STATE, "DSP_OPT_RELABEL_MAP must be set before dsp_reserve (the workspace plan depends on it)");
+      c->relabel_mode = (int)value;
+      return DSP_OK;
+    case DSP_OPT_LANE_ROUNDS:
+      if (value < 1 || value > 1024) return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_LANE_ROUNDS %lld not in [1, 1024]", (long long)value);
+      c->lane_rounds = (int)value;
+      return DSP_OK;
+    case DSP_OPT_LOADER_WARPS:
+      if (value != 2 && value != LOADER_WARPS && value != LOADER_WARPS_MAX)
+        return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_LOADER_WARPS must be 2, 4 or 8");
+      c->loader_warps = (int)value;
+      return DSP_OK;
+    case DSP_OPT_LOADER_ROWS:
+      if (value < 1 || value > 32) return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_LOADER_ROWS %lld not in [1, 32]", (long long)value);
+      c->loader_rows = (int)value;
+      return DSP_OK;
+    case DSP_OPT_GATHER_REGLOADS:
+      if (value != 0 && value != 1) return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_GATHER_REGLOADS must be 0 or 1");
+      c->gather_reg = value != 0 || c->tma_unavailable;
+      c->cold_regloads = c->gather_reg;
+      return DSP_OK;
+    default:
+      return fail(c, DSP_ERR_INVALID_ARG, "unknown option %d", option);
+  }
+}
+
 dsp_status dsp_pipeline_flush(dsp_ctx *c, void *stream) {
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
   for (auto &p : c->pend)
-    if (p.active && p.stream == stream) {
-      dsp_status st = flush_one(c, p);
+    if (p.active) {
+      dsp_status st = flush_one(c, p, static_cast<cudaStream_t>(stream));
       if (st != DSP_OK) return st;
     }
   return DSP_OK;

@@ -234,15 +234,6 @@ __device__ __forceinline__ void walk_finish_body(const WalkArgs &a, const WalkRo
   }
 }
 
-__global__ void __launch_bounds__(NT) k_walk_init(WalkArgs a) { walk_init_body(a); }
-__global__ void __launch_bounds__(NT) k_walk_scatter(WalkArgs a) {
-  walk_scatter_body(a, WalkRound{a.step, a.parity, a.seq});
-}
-__global__ void __launch_bounds__(NT) k_walk_step(WalkArgs a) { walk_step_body(a, WalkRound{a.step, a.parity, a.seq}); }
-__global__ void k_walk_done(WalkArgs a) { walk_done_body(a, WalkRound{a.step, a.parity, a.seq}); }
-__global__ void __launch_bounds__(NT) k_walk_finish(WalkArgs a) {
-  walk_finish_body(a, WalkRound{a.step, a.parity, a.seq});
-}
 
 // The whole multi-rank walk call in ONE cooperative launch per rank: init,
 // then per step the shuffle (its last block publishes the inbox flags) and the

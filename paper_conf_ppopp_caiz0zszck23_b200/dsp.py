@@ -36,12 +36,19 @@ ABI_SYMBOLS = ("dsp_abi_version", "dsp_status_str", "dsp_last_error", "dsp_creat
                "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve", "dsp_reserve_layerwise", "dsp_export_handle", "dsp_import_handles",
                "dsp_sample_bounds", "dsp_sample_bounds_layerwise", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                "dsp_pipeline_flush", "dsp_set_persistent_blocks", "dsp_gather_features", "dsp_random_walk",
-               "dsp_reserve_walks", "dsp_random_walk_group",
+               "dsp_reserve_walks", "dsp_random_walk_group", "dsp_set_option",
                "dsp_sync")
 DSP_ASYNC = 1
 DSP_PIPELINED = 2
 DSP_BIASED = 4
 DSP_LAYERWISE = 8
+DSP_OPT_RELABEL_MAP = 1
+DSP_OPT_LANE_ROUNDS = 2
+DSP_OPT_LOADER_WARPS = 3
+DSP_OPT_LOADER_ROWS = 4
+DSP_OPT_GATHER_REGLOADS = 5
+#: DSP_OPT_RELABEL_MAP values
+RELABEL_MAPS = {"auto": 0, "direct": 1, "hash": 2, "direct64": 3}
 
 
 class DSPError(RuntimeError):
@@ -100,12 +107,13 @@ def lib(path: str | None = None):
         L.dsp_reserve_walks.argtypes = [P, i64, i32]
         L.dsp_random_walk_group.argtypes = [P, i32, P, P, i32, ctypes.c_uint64, P, P]
         L.dsp_sync.argtypes = [P, P]
+        L.dsp_set_option.argtypes = [P, i32, i64]
         for name in ("dsp_create", "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve",
                      "dsp_reserve_layerwise", "dsp_sample_bounds_layerwise", "dsp_export_handle",
                      "dsp_import_handles", "dsp_sample_bounds", "dsp_sample", "dsp_sample_gather", "dsp_sample_group",
                      "dsp_pipeline_flush", "dsp_random_walk", "dsp_set_persistent_blocks",
                      "dsp_reserve_walks", "dsp_random_walk_group",
-                     "dsp_gather_features", "dsp_sync"):
+                     "dsp_gather_features", "dsp_sync", "dsp_set_option"):
             getattr(L, name).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -253,6 +261,10 @@ def dsp_gather_features(ctx, ids, n: int, out, stream: int) -> None:
     _check(lib().dsp_gather_features(ctx, _p(ids), n, _p(out), ctypes.c_void_p(stream)), ctx)
 
 
+def dsp_set_option(ctx, option: int, value: int) -> None:
+    _check(lib().dsp_set_option(ctx, option, value), ctx)
+
+
 def dsp_set_persistent_blocks(ctx, blocks: int) -> None:
     _check(lib().dsp_set_persistent_blocks(ctx, blocks), ctx)
 
@@ -303,9 +315,11 @@ class Sampler:
                  world_size: int = 1, device: int | None = None,
                  exchange: Callable[[bytes], list] | None = None, connect: bool = True, n_slots: int = 1,
                  edge_weights=None, n_workspaces: int = 1, hot_rows: int | None = None, scheme: str = "node",
-                 max_walks: int | None = None, max_walk_length: int = 1024):
+                 max_walks: int | None = None, max_walk_length: int = 1024, options: dict | None = None):
         """max_walks: reserve the random-walk region (needed for random_walk when
-        world_size > 1) for up to max_walks walks per rank of max_walk_length steps."""
+        world_size > 1) for up to max_walks walks per rank of max_walk_length steps.
+        options: {DSP_OPT_*: value} applied with dsp_set_option right after
+        dsp_create (performance only; results are identical)."""
         import torch
         self.torch = torch
         self.device = torch.cuda.current_device() if device is None else device
@@ -318,6 +332,8 @@ class Sampler:
         self.dim = 0 if features is None else int(features.shape[1])
         self.ctx = dsp_create(rank, world_size, self.device)
         try:
+            for opt, val in (options or {}).items():
+                dsp_set_option(self.ctx, int(opt), int(val))
             if hot_rows is None:
                 dsp_load_partition(self.ctx, bounds, indptr, indices, features, self.dim)
             else:  # cold-feature tier: hot_rows rows in HBM, the rest in host memory
@@ -473,15 +489,16 @@ class LocalGroup:
     GPUs of this node."""
 
     def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int], hot_rows=None,
-                 scheme: str = "node", max_walks: int | None = None, max_walk_length: int = 1024):
+                 scheme: str = "node", max_walks: int | None = None, max_walk_length: int = 1024,
+                 options: dict | None = None):
         """shards[r] = (indptr, indices, features[, edge_weights]) of rank r;
-        hot_rows[r] (optional) enables the cold-feature tier."""
+        hot_rows[r] (optional) enables the cold-feature tier; options as Sampler."""
         P = len(shards)
         assert len(devices) == P and len(bounds) == P + 1
         self.samplers = [Sampler(bounds, s[0], s[1], s[2], fanouts, max_seeds, rank=r, world_size=P,
                                  device=devices[r], connect=False, edge_weights=s[3] if len(s) > 3 else None,
                                  hot_rows=None if hot_rows is None else hot_rows[r], scheme=scheme,
-                                 max_walks=max_walks, max_walk_length=max_walk_length)
+                                 max_walks=max_walks, max_walk_length=max_walk_length, options=options)
                          for r, s in enumerate(shards)]
         handles = [dsp_export_handle(s.ctx) for s in self.samplers]
         for s in self.samplers:

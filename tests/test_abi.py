@@ -74,3 +74,12 @@ def test_product_never_imports_oracle():
                 txt = open(os.path.join(dirpath, f)).read()
                 assert not re.search(r"^\s*(import|from)\s+oracle", txt, re.M), f
                 assert "oracle.c" not in txt and "liboracle" not in txt, f
+
+
+def test_no_environment_switches_in_the_library():
+    """Every behaviour switch of libdsp.so is an ABI argument or a documented
+    dsp_set_option (include/dsp.h); the library reads no environment."""
+    csrc = os.path.join(ROOT, "paper_conf_ppopp_caiz0zszck23_b200", "csrc")
+    for f in os.listdir(csrc):
+        txt = open(os.path.join(csrc, f)).read()
+        assert "getenv" not in txt and "environ" not in txt, f

@@ -53,17 +53,8 @@ def _big_tasks(ip, seeds, n):
     return int(((c > 40) & (c < d * 0.9)).sum())
 
 
-@pytest.fixture(params=["persistent", "staged"])
-def lw_mode(request, monkeypatch):
-    """world 1: all layers in one cooperative launch (default) or one launch per
-    stage (DSP_LW_STAGED=1, read by dsp_create)."""
-    if request.param == "staged":
-        monkeypatch.setenv("DSP_LW_STAGED", "1")
-    return request.param
-
-
 @pytest.mark.parametrize("sizes", [(200, 300), (1000, 1000), (1,), (8192,), (50, 50, 50), (3, 4000)])
-def test_layerwise_tiny_p1(pkg, tiny, sizes, lw_mode):
+def test_layerwise_tiny_p1(pkg, tiny, sizes):
     cfg, ip, ix, feats = tiny
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, sizes, 64, scheme="layer")
     rng = np.random.default_rng(len(sizes) * 7 + sizes[0])
@@ -74,7 +65,7 @@ def test_layerwise_tiny_p1(pkg, tiny, sizes, lw_mode):
     s.close()
 
 
-def test_layerwise_big_tasks_exercised(pkg, tiny, lw_mode):
+def test_layerwise_big_tasks_exercised(pkg, tiny):
     """n = 1000 over 64 seeds: hub seeds get 32 < c < deg draws."""
     cfg, ip, ix, feats = tiny
     deg = np.diff(ip)
@@ -89,7 +80,7 @@ def test_layerwise_big_tasks_exercised(pkg, tiny, lw_mode):
 
 
 @pytest.mark.parametrize("P", [2, 4])
-def test_layerwise_virtual_ranks(pkg, tiny, P, lw_mode):
+def test_layerwise_virtual_ranks(pkg, tiny, P):
     cfg, ip, ix, feats = tiny
     bnds = datagen.bounds(cfg.num_nodes, P)
     shards = []
@@ -118,7 +109,7 @@ def test_layerwise_virtual_ranks(pkg, tiny, P, lw_mode):
     grp.close()
 
 
-def test_layerwise_fused_and_pipelined(pkg, tiny, lw_mode):
+def test_layerwise_fused_and_pipelined(pkg, tiny):
     cfg, ip, ix, feats = tiny
     sizes = (400, 800)
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, sizes, 64, n_slots=2, scheme="layer")
@@ -182,7 +173,7 @@ def test_layerwise_concurrent_streams(pkg, tiny):
     s.close()
 
 
-def test_layerwise_errors(pkg, tiny, lw_mode):
+def test_layerwise_errors(pkg, tiny):
     cfg, ip, ix, feats = tiny
     bn = datagen.bounds(cfg.num_nodes, 1)
     with pytest.raises(pkg.DSPError) as e:

@@ -95,14 +95,15 @@ def test_fanout_range_and_ragged_batches(pkg, tiny, fanouts):
 
 
 @pytest.mark.parametrize("relabel", ["direct", "direct64", "hash"])
-def test_maximum_layers_and_fanout(pkg, tiny, relabel, monkeypatch):
+def test_maximum_layers_and_fanout(pkg, tiny, relabel):
     """The ABI's limits: 8 layers of fan-out 32 (the frontier saturates at all
-    N nodes, every row of degree <= 32 is taken whole), on each relabel layout;
-    fused gather of the last block (every node) and a pipelined call."""
-    monkeypatch.setenv("DSP_RELABEL", relabel)
+    N nodes, every row of degree <= 32 is taken whole), on each relabel layout
+    (DSP_OPT_RELABEL_MAP); fused gather of the last block (every node) and a
+    pipelined call."""
     cfg, ip, ix, feats = tiny
     fan = (32,) * 8
-    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, fan, 64, n_slots=2)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, fan, 64, n_slots=2,
+                    options={pkg.dsp.DSP_OPT_RELABEL_MAP: pkg.dsp.RELABEL_MAPS[relabel]})
     seeds = np.random.default_rng(8).choice(cfg.num_nodes, size=64, replace=False).astype(np.int32)
     blocks, feat = s.sample_gather(torch.from_numpy(seeds).cuda(), 77, slot=0)
     ref = oracle.sample(ip, ix, seeds, fan, 77)
@@ -191,13 +192,11 @@ def test_fig5_csp_example_virtual_two_gpus(pkg):
 
 # ------------------------------------------------------- virtual P = 2,4,8
 
-@pytest.mark.parametrize("mode", ["persistent", "staged"])
+@pytest.mark.parametrize("mode", ["direct", "hash"])
 @pytest.mark.parametrize("P", [2, 4, 8])
-def test_tiny_virtual_ranks(pkg, tiny, P, mode, monkeypatch):
-    """world > 1: one persistent kernel per rank (default; virtual ranks each on
-    1/P of the SMs, own stream) or the stage-by-stage kernels (DSP_MULTI_STAGED)."""
-    if mode == "staged":
-        monkeypatch.setenv("DSP_MULTI_STAGED", "1")
+def test_tiny_virtual_ranks(pkg, tiny, P, mode):
+    """world > 1: one persistent kernel per rank (virtual ranks each on 1/P of
+    the SMs, own stream), with the compact direct or the hashed relabel map."""
     cfg, ip, ix, feats = tiny
     bnds = datagen.bounds(cfg.num_nodes, P)
     shards = []
@@ -205,7 +204,8 @@ def test_tiny_virtual_ranks(pkg, tiny, P, mode, monkeypatch):
         lo, hi = int(bnds[r]), int(bnds[r + 1])
         sip, six = datagen.shard(ip, ix, lo, hi)
         shards.append((sip, six, feats[lo:hi]))
-    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P)
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P,
+                         options={pkg.dsp.DSP_OPT_RELABEL_MAP: pkg.dsp.RELABEL_MAPS[mode]})
     per_rank = [seeds_of(cfg, P, r, batch=32) for r in range(P)]
     steps = min(len(x) for x in per_rank)
     for step in range(min(steps, 6)):
@@ -225,14 +225,12 @@ def test_tiny_virtual_ranks(pkg, tiny, P, mode, monkeypatch):
     grp.close()
 
 
-@pytest.mark.parametrize("mode", ["persistent", "staged"])
-def test_virtual_ranks_errors(pkg, tiny, mode, monkeypatch):
+@pytest.mark.parametrize("mode", ["direct", "hash"])
+def test_virtual_ranks_errors(pkg, tiny, mode):
     """Device-detected errors at world > 1 (duplicate seed, out-of-range seed)
     are reported by the group call after the exchange protocol completed, and
     the ranks stay usable; a batch above the reserved size fails before any
     launch on every rank."""
-    if mode == "staged":
-        monkeypatch.setenv("DSP_MULTI_STAGED", "1")
     cfg, ip, ix, feats = tiny
     P = 2
     bnds = datagen.bounds(cfg.num_nodes, P)
@@ -241,7 +239,8 @@ def test_virtual_ranks_errors(pkg, tiny, mode, monkeypatch):
         lo, hi = int(bnds[r]), int(bnds[r + 1])
         sip, six = datagen.shard(ip, ix, lo, hi)
         shards.append((sip, six, feats[lo:hi]))
-    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 16, devices=[0] * P)
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 16, devices=[0] * P,
+                         options={pkg.dsp.DSP_OPT_RELABEL_MAP: pkg.dsp.RELABEL_MAPS[mode]})
     t = lambda x: torch.tensor(x, dtype=torch.int32, device="cuda")
     with pytest.raises(pkg.DSPError) as e:
         grp.sample([t([5, 9, 5]), t([7000])], 1)
@@ -259,12 +258,10 @@ def test_virtual_ranks_errors(pkg, tiny, mode, monkeypatch):
     grp.close()
 
 
-@pytest.mark.parametrize("mode", ["persistent", "staged"])
-def test_virtual_ranks_all_empty(pkg, tiny, mode, monkeypatch):
+@pytest.mark.parametrize("mode", ["direct", "hash"])
+def test_virtual_ranks_all_empty(pkg, tiny, mode):
     """Every rank with an empty batch: the exchange still runs (empty inboxes),
     every block comes back empty, and the next call is unaffected."""
-    if mode == "staged":
-        monkeypatch.setenv("DSP_MULTI_STAGED", "1")
     cfg, ip, ix, feats = tiny
     P = 2
     bnds = datagen.bounds(cfg.num_nodes, P)
@@ -273,7 +270,8 @@ def test_virtual_ranks_all_empty(pkg, tiny, mode, monkeypatch):
         lo, hi = int(bnds[r]), int(bnds[r + 1])
         sip, six = datagen.shard(ip, ix, lo, hi)
         shards.append((sip, six, feats[lo:hi]))
-    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 16, devices=[0] * P)
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 16, devices=[0] * P,
+                         options={pkg.dsp.DSP_OPT_RELABEL_MAP: pkg.dsp.RELABEL_MAPS[mode]})
     empty = torch.zeros(0, dtype=torch.int32, device="cuda")
     res = grp.sample([empty, empty], 3)
     for r in range(P):
@@ -603,11 +601,8 @@ def test_random_walks_tiny(pkg, tiny):
     s.close()
 
 
-@pytest.mark.parametrize("mode", ["persistent", "staged"])
 @pytest.mark.parametrize("P", [2, 4, 8])
-def test_random_walks_virtual_ranks(pkg, tiny, P, mode, monkeypatch):
-    if mode == "staged":
-        monkeypatch.setenv("DSP_WALK_STAGED", "1")
+def test_random_walks_virtual_ranks(pkg, tiny, P):
     """Walks over a partitioned graph (P:L184: CSP push, reshuffle removed):
     every rank's traces equal the single-device oracle's, whatever P; walks
     start on any owner, meet, terminate at isolated nodes; a rank with no

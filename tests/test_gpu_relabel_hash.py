@@ -1,15 +1,14 @@
-"""GPU parity under each layout of the relabel map, forced with DSP_RELABEL on
+"""GPU parity under each layout of the relabel map, forced with
+dsp_set_option(DSP_OPT_RELABEL_MAP) on
 graphs the oracle checks quickly: the batch-sized hash table (the default for
 graphs of more than 3M nodes -- papers / Friendster -- where a direct map over
 all N ids cannot stay in L2), the compact 4-byte direct map (the default
 below that) and the 8-byte epoch-word direct map.  The layout only changes
 where the relabel words live, so every block must stay bit-identical to the
 oracle: P = 1 (persistent kernel, plain / fused / pipelined), virtual ranks
-(persistent and stage-by-stage kernels), biased sampling, duplicate-seed
+(one persistent kernel per rank), biased sampling, duplicate-seed
 detection, and enough calls on one workspace to cross the 255-epoch windows
 that zero the hash table and the compact map."""
-import os
-
 import numpy as np
 import pytest
 
@@ -32,8 +31,9 @@ def pkg():
 
 
 @pytest.fixture(params=["hash", "direct", "direct64"])
-def hashed(request, monkeypatch):
-    monkeypatch.setenv("DSP_RELABEL", request.param)   # read by dsp_create
+def hashed(request, pkg):
+    """Sampler / LocalGroup options selecting the relabel-map layout."""
+    return {pkg.dsp.DSP_OPT_RELABEL_MAP: pkg.dsp.RELABEL_MAPS[request.param]}
 
 
 @pytest.fixture(scope="module")
@@ -60,7 +60,7 @@ def test_hash_tiny_every_batch_and_tag_wrap(pkg, tiny, hashed):
     once, so the table is zeroed mid-run and tags are reused afterwards."""
     cfg, ip, ix, feats = tiny
     fan = (15, 10, 5)
-    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, fan, cfg.batch)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, fan, cfg.batch, options=hashed)
     batches = batches_of(cfg, 1, 0)
     assert 3 * len(batches) > 255
     for step, seeds in enumerate(batches):
@@ -71,7 +71,7 @@ def test_hash_tiny_every_batch_and_tag_wrap(pkg, tiny, hashed):
 
 def test_hash_fused_and_pipelined(pkg, tiny, hashed):
     cfg, ip, ix, feats = tiny
-    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2, options=hashed)
     batches = batches_of(cfg, 1, 0)
     blocks, feat = s.sample_gather(torch.from_numpy(batches[0]).cuda(), 5, slot=0)
     ref = oracle.sample(ip, ix, batches[0], cfg.fanouts, 5)
@@ -95,7 +95,7 @@ def test_hash_fused_and_pipelined(pkg, tiny, hashed):
 
 def test_hash_duplicate_seed(pkg, tiny, hashed):
     cfg, ip, ix, feats = tiny
-    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 64)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 64, options=hashed)
     for dup in ([5, 9, 5], list(range(40)) + [17]):
         with pytest.raises(pkg.DSPError) as e:
             s.sample(torch.tensor(dup, dtype=torch.int32, device="cuda"), 1)
@@ -105,11 +105,8 @@ def test_hash_duplicate_seed(pkg, tiny, hashed):
     s.close()
 
 
-@pytest.mark.parametrize("mode", ["persistent", "staged"])
 @pytest.mark.parametrize("P", [2, 4])
-def test_hash_virtual_ranks(pkg, tiny, hashed, P, mode, monkeypatch):
-    if mode == "staged":
-        monkeypatch.setenv("DSP_MULTI_STAGED", "1")
+def test_hash_virtual_ranks(pkg, tiny, hashed, P):
     cfg, ip, ix, feats = tiny
     bnds = datagen.bounds(cfg.num_nodes, P)
     shards = []
@@ -117,12 +114,12 @@ def test_hash_virtual_ranks(pkg, tiny, hashed, P, mode, monkeypatch):
         lo, hi = int(bnds[r]), int(bnds[r + 1])
         sip, six = datagen.shard(ip, ix, lo, hi)
         shards.append((sip, six, feats[lo:hi]))
-    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P)
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P, options=hashed)
     train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
     per_rank = [np.concatenate([datagen.rank_seed_batches(train, bnds, r, 32, e) for e in (0, 1)])
                 for r in range(P)]
     assert min(len(x) for x in per_rank) >= 90
-    for step in range(90):   # crosses the tag wrap on the stage-by-stage path too
+    for step in range(90):   # crosses the tag wrap
         seeds = [per_rank[r][step] for r in range(P)]
         res = grp.sample([torch.from_numpy(np.ascontiguousarray(x)).cuda() for x in seeds], 0x77 + step)
         if step % 15 == 0 or step > 80:
@@ -134,7 +131,7 @@ def test_hash_virtual_ranks(pkg, tiny, hashed, P, mode, monkeypatch):
 def test_hash_biased(pkg, tiny, hashed):
     cfg, ip, ix, feats = tiny
     w = datagen.edge_weights(ix, datagen.node_weights(cfg.num_nodes))
-    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, edge_weights=w)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, edge_weights=w, options=hashed)
     batches = batches_of(cfg, 1, 0)
     for step in range(4):
         blocks = s.sample(torch.from_numpy(batches[step]).cuda(), 60 + step, biased=True)
@@ -146,7 +143,7 @@ def test_hash_biased(pkg, tiny, hashed):
 def test_hash_products(pkg, hashed):
     cfg = datagen.CONFIGS["products"]
     ip, ix = datagen.make_graph(cfg)
-    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, None, cfg.fanouts, cfg.batch)
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, None, cfg.fanouts, cfg.batch, options=hashed)
     batches = batches_of(cfg, 1, 0)
     for step in (0, 1):
         blocks = s.sample(torch.from_numpy(batches[step]).cuda(), 5 + step)

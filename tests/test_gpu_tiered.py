@@ -45,13 +45,12 @@ def _seeds(cfg, P, r, batch):
 
 
 @pytest.mark.parametrize("hot,regloads", [(0, 0), (1, 0), (3000, 0), (10_000, 0), (-1, 0), (0, 1), (3000, 1)])
-def test_tiered_gather_p1(pkg, tiny, hot, regloads, monkeypatch):
-    """regloads = 0: the pipelined loader warps bulk-copy (TMA) cold rows
-    straight from host memory; 1: register loads (DSP_COLD_REGLOADS=1)."""
+def test_tiered_gather_p1(pkg, tiny, hot, regloads):
+    """regloads = 0: the gathers bulk-copy (TMA) cold rows straight from host
+    memory; 1: register loads (DSP_OPT_GATHER_REGLOADS = 1)."""
     cfg, ip, ix, feats = tiny
-    monkeypatch.setenv("DSP_COLD_REGLOADS", str(regloads))
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2,
-                    hot_rows=hot)
+                    hot_rows=hot, options={pkg.dsp.DSP_OPT_GATHER_REGLOADS: regloads})
     # standalone gather over ids covering every row, in a scrambled order with repeats
     rng = np.random.default_rng(hot & 0xFFFF)
     ids = np.concatenate([rng.permutation(cfg.num_nodes), rng.integers(0, cfg.num_nodes, 777)]).astype(np.int32)

@@ -137,17 +137,70 @@ def test_layerwise_dense_rows_take_exactly_n():
         assert b["num_edges"] == 60
 
 
-def test_fig3_layerwise_fanout_two():
-    """with layer-wise fan-out [2, 2] 'the total number of sampled
-    nodes should be 2' in both layers (Fig. 3 graph)."""
+def _fig3_csr():
+    """The Fig. 3 graph of tests/golden/fig3_worked_example.json (P:L81,
+    P:L146): node v's in-neighbour row is rows[str(v)], empty when absent."""
     g = json.load(open(os.path.join(GOLDEN, "fig3_worked_example.json")))
-    rows = g["rows"]
-    ip = np.concatenate([[0], np.cumsum([len(r) for r in rows])]).astype(np.int64)
-    ix = np.concatenate([np.asarray(sorted(r), np.int32) for r in rows]).astype(np.int32)
-    for s in range(50):
-        blocks = oracle.sample_layerwise(ip, ix, g["seeds"], [2, 2], s)
-        for b in blocks:
-            assert 1 <= b["num_edges"] <= 2
+    n = g["num_nodes"]
+    ip = np.zeros(n + 1, np.int64)
+    cols = []
+    for v in range(n):
+        r = sorted(g["rows"].get(str(v), []))
+        cols.extend(r)
+        ip[v + 1] = ip[v] + len(r)
+    return g, ip, np.array(cols, np.int32)
+
+
+def test_fig3_layerwise_fanout_two():
+    """P:L102 (layer-wise: 'the total number of sampled nodes' per layer is
+    the fan-out) on the Fig. 3 graph A:[C,E], C:[B,K], E:[G,H] (P:L81,
+    P:L146) with layer sizes [2, 2] (R28).
+
+    Layer 0: the frontier is {A} alone, so both Eq. 2 draws pick A (c_A = 2 =
+    deg A) and A's whole row is taken: block 0 equals the node-wise Fig. 3
+    block (indptr [0,2], src_ids [A,C,E]) for every rng_seed.
+    Layer 1: frontier [A,C,E] with W = deg = [2,2,2]; (c_A,c_C,c_E) ~
+    Multinomial(2, 1/3 each) and u takes min(c_u, 2) of its 2 neighbours
+    without replacement, so there are exactly 2 edges, each drawn from the row
+    of its dst, and the edge set has the closed-form law: {both neighbours of
+    u} with probability 1/9 for each u, {one neighbour of u, one of w} with
+    probability (2/9)(1/2)(1/2) = 1/18 for each pair u < w and each of the 4
+    neighbour choices (3 * 1/9 + 12 * 1/18 = 1)."""
+    g, ip, ix = _fig3_csr()
+    assert ip.tolist() == [0, 2, 2, 4, 6, 6, 6, 6] and ix.tolist() == [2, 3, 1, 6, 4, 5]
+    A, B, C, E, G, H, K = range(7)
+    row = {A: (C, E), C: (B, K), E: (G, H)}
+    law = {}
+    for u in (A, C, E):
+        law[frozenset({(u, row[u][0]), (u, row[u][1])})] = 1 / 9
+    for u, w in ((A, C), (A, E), (C, E)):
+        for x in row[u]:
+            for y in row[w]:
+                law[frozenset({(u, x), (w, y)})] = 1 / 18
+    assert abs(sum(law.values()) - 1) < 1e-12 and len(law) == 15
+    trials = 6000
+    seen = Counter()
+    for s in range(trials):
+        b0, b1 = oracle.sample_layerwise(ip, ix, g["seeds"], [2, 2], s)
+        exp0 = g["blocks"][0]
+        for key in ("indptr", "indices", "src_ids"):
+            assert b0[key].tolist() == exp0[key], (s, key)
+        assert (b1["num_dst"], b1["num_edges"]) == (3, 2), s
+        assert b1["src_ids"][:3].tolist() == [A, C, E]
+        assert b1["indptr"][0] == 0 and b1["indptr"][3] == 2 and np.all(np.diff(b1["indptr"]) >= 0)
+        pairs = set()
+        for i, u in enumerate((A, C, E)):
+            for e in range(b1["indptr"][i], b1["indptr"][i + 1]):
+                w = int(b1["src_ids"][b1["indices"][e]])
+                assert w in row[u], (s, u, w)
+                pairs.add((u, w))
+        assert len(pairs) == 2
+        seen[frozenset(pairs)] += 1
+    assert set(seen) <= set(law)
+    keys = sorted(law, key=lambda k: sorted(k))
+    obs = np.array([seen[k] for k in keys], float)
+    exp = np.array([law[k] * trials for k in keys])
+    assert chisquare(obs, exp).pvalue > 1e-4
 
 
 @pytest.mark.parametrize("P", [2, 3, 4])

@@ -19,9 +19,9 @@ batches = torch.from_numpy(datagen.rank_seed_batches(train, bnds, 0, cfg.batch, 
 L = len(cfg.fanouts)
 steps = 40
 for mode in os.environ.get("MODES", "hash,direct").split(","):
-    os.environ["DSP_RELABEL"] = mode
     for K in (1, 2):
-        s = pkg.Sampler(bnds, ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2 * K, n_workspaces=K)
+        s = pkg.Sampler(bnds, ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2 * K, n_workspaces=K,
+                        options={pkg.dsp.DSP_OPT_RELABEL_MAP: pkg.dsp.RELABEL_MAPS[mode]})
         if K > 1:
             pkg.dsp_set_persistent_blocks(s.ctx, 148 // K)
         sizes = torch.zeros((256, 3 * L), dtype=torch.int64).pin_memory()

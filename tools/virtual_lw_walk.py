@@ -1,6 +1,6 @@
 """Multi-rank layer-wise sampling and random walks as P virtual ranks on one GPU
 (products graph): time per synchronous group call, one cooperative launch per
-rank (default) or the stage-by-stage kernels (DSP_LW_STAGED=1 / DSP_WALK_STAGED=1).
+rank.
 python tools/virtual_lw_walk.py"""
 import os, sys, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -12,7 +12,7 @@ import paper_conf_ppopp_caiz0zszck23_b200 as pkg
 cfg = datagen.CONFIGS["products"]
 ip, ix = datagen.make_graph(cfg)
 train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
-mode = "staged" if os.environ.get("DSP_LW_STAGED") or os.environ.get("DSP_WALK_STAGED") else "persistent"
+mode = "persistent"
 for P in (2, 4):
     bnds = datagen.bounds(cfg.num_nodes, P)
     shards = []
