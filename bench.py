@@ -145,6 +145,19 @@ def ncu_traffic(kernel: str):
     return None
 
 
+def relaunch_under_torchrun(n_gpus: int, argv) -> int:
+    """`python bench.py --gpus N` without torchrun: start the N ranks the
+    driver's launcher would (one process per GPU, torch.distributed.run on
+    127.0.0.1, a free port); rank 0 prints the line."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n_gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *argv]
+    return subprocess.call(cmd)
+
+
 def setup_dist(n_gpus: int):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -263,23 +276,61 @@ def run_reference(args):
     return 0
 
 
+def host_cpu() -> dict:
+    """The host the oracle runs on: CPU model (lscpu / /proc/cpuinfo), logical
+    cores, and the cores this process may use."""
+    model = None
+    try:
+        out = subprocess.check_output(["lscpu"], text=True, stderr=subprocess.DEVNULL)
+        for line in out.splitlines():
+            if line.startswith("Model name:"):
+                model = line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    if model is None:
+        try:
+            for line in open("/proc/cpuinfo"):
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+        except Exception:
+            pass
+    return {"model": model, "logical_cores": os.cpu_count(), "cores_available": len(os.sched_getaffinity(0))}
+
+
 def cpu_baseline(args, cfg, ip, ix, feats, batches, seconds: float, weights=None):
+    """the oracle (single host thread) pinned to one core
+    (sched_setaffinity of the calling thread, the `taskset -c` of one core), on
+    the same seed batches and rng_seed schedule as the GPU run: the whole epoch
+    of this rank's batches, or as many as fit in `seconds`.  Runs after the GPU
+    timing, outside every timed region."""
     import datagen
     import oracle
-    t_all = 0.0
-    edges = 0
-    n = 0
-    while t_all < seconds and n < len(batches):
-        seeds = batches[n]
-        t0 = time.perf_counter()
-        blocks = oracle_sample(args, ip, ix, seeds, fanouts_of(args, cfg), datagen.BASE_SEED + n, weights=weights)
-        oracle.gather(feats, blocks[-1]["src_ids"])
-        t_all += time.perf_counter() - t0
-        edges += sum(int(b["num_edges"]) for b in blocks)
-        n += 1
+    host = host_cpu()
+    old = os.sched_getaffinity(0)
+    core = min(old)
+    os.sched_setaffinity(0, {core})
+    try:
+        t_all = 0.0
+        edges = 0
+        n = 0
+        while t_all < seconds and n < len(batches):
+            seeds = batches[n]
+            t0 = time.perf_counter()
+            blocks = oracle_sample(args, ip, ix, seeds, fanouts_of(args, cfg), datagen.BASE_SEED + n, weights=weights)
+            oracle.gather(feats, blocks[-1]["src_ids"])
+            t_all += time.perf_counter() - t0
+            edges += sum(int(b["num_edges"]) for b in blocks)
+            n += 1
+    finally:
+        os.sched_setaffinity(0, old)
+    full = n == len(batches)
     return {"value": edges / t_all, "unit": "edges/s", "cores": 1, "kind": "oracle",
-            "sample": f"{n} {cfg.name} batches of {cfg.batch} seeds, single host thread "
-                      f"(oracle.sample + oracle.gather), {t_all:.1f} s"}
+            "sample": (f"{'the full epoch' if full else 'a bounded sample'}: {n} of {len(batches)} {cfg.name} "
+                       f"batches of {cfg.batch} seeds (oracle.sample + oracle.gather), {t_all:.1f} s on 1 core "
+                       f"pinned (core {core}) of {host['cores_available']} available"),
+            "epoch_batches": len(batches), "batches_timed": n, "seeds_per_s": n * cfg.batch / t_all,
+            "host": host}
 
 
 # ----------------------------------------------------------------- product
@@ -292,6 +343,80 @@ def algorithmic_bytes(sizes, L, dim):
     new = sum(int(sizes[3 * l + 1]) - int(sizes[3 * l]) for l in range(L))
     U = int(sizes[3 * (L - 1) + 1])
     return 24 * F + 8 * E + 4 * new, 2 * U * dim * 4
+
+
+def peer_read_peak(s, bnds, rank: int, world: int, dim: int, reps: int = 5):
+    """NVLink denominator measured in this run: every rank at once gathers
+    contiguous runs of rows owned by each of the other ranks through
+    dsp_gather_features (TMA bulk copies reading the peers' shards over their
+    peer mappings: all GPU pairs busy), ~256 MB per rank.  Returns the
+    per-GPU receive rate (bytes read from peers / max-over-ranks time)."""
+    rows_per_peer = max(1, (256 << 20) // (dim * 4) // max(1, world - 1))
+    ids = []
+    for r in range(world):
+        if r == rank:
+            continue
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        n = min(rows_per_peer, hi - lo)
+        ids.append(np.arange(lo, lo + n, dtype=np.int32))
+    ids = torch.from_numpy(np.concatenate(ids)).cuda()
+    out = torch.empty((ids.numel(), dim), dtype=torch.float32, device="cuda")
+    for _ in range(2):
+        s.gather(ids, out)
+    s.sync()
+    best = 1e30
+    stream = torch.cuda.current_stream()
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        barrier()
+        torch.cuda.synchronize()
+        a.record(stream)
+        s.gather(ids, out)
+        b.record(stream)
+        torch.cuda.synchronize()
+        best = min(best, reduce_max_over_ranks(a.elapsed_time(b)))
+    nbytes = reduce_sum_over_ranks(float(ids.numel() * dim * 4)) / world
+    del out
+    return nbytes / (best * 1e-3) / 1e9, int(ids.numel())
+
+
+def remote_bytes(blocks, bnds, rank: int, dim: int):
+    """NVLink bytes one step of this rank causes (per
+    requester; summed over the ranks they count every byte that crosses a link
+    once): per layer 4 B per remote frontier id sent to its owner, 4 B count +
+    4 B per sampled edge returned for it; the gather reads dim * 4 B per row of
+    the last block owned by another rank."""
+    lo, hi = int(bnds[rank]), int(bnds[rank + 1])
+    csp = 0
+    for b in blocks:
+        f = b.src_ids[: b.num_dst].cpu().numpy()
+        ip = b.indptr[: b.num_dst + 1].cpu().numpy().astype(np.int64)
+        rem = (f < lo) | (f >= hi)
+        csp += 8 * int(rem.sum()) + 4 * int(np.diff(ip)[rem].sum())
+    u = blocks[-1].src_ids.cpu().numpy()
+    rows = int(((u < lo) | (u >= hi)).sum())
+    return csp, rows * dim * 4, rows
+
+
+def multi_phase_us(s, L: int):
+    """Phase durations of this rank's last synchronous k_csp_multi call from
+    the globaltimer stamps block 0 leaves in the workspace header at every
+    grid barrier: per layer A shuffle (frontier ids into the owners' inboxes),
+    B owner sample (waits for every rank's inbox flag, then samples and writes
+    the rows back), C return (waits for the return flags, unpermute + marks),
+    D relabel scan (2 barrier intervals)."""
+    ws = s.workspace[:1024].view(torch.int64)
+    t = ws[81:105].cpu().numpy()
+    nb = sum(1 for g in range(1, 23) if t[g] > t[0])
+    st = [int(t[0])] + [int(t[g]) for g in range(1, nb + 1)]
+    d = np.diff(np.array(st, dtype=np.int64)) / 1e3
+    if len(d) == 5 * L + 1:   # a call that zeroed the relabel map first
+        d = d[1:]
+    if len(d) != 5 * L:
+        return None
+    return [{"shuffle_us": float(d[5 * l]), "owner_sample_us": float(d[5 * l + 1]),
+             "return_unpermute_us": float(d[5 * l + 2]), "relabel_us": float(d[5 * l + 3] + d[5 * l + 4]),
+             "exchange_us": float(d[5 * l] + d[5 * l + 1] + d[5 * l + 2])} for l in range(L)]
 
 
 def run_walk(args):
@@ -678,12 +803,50 @@ def run_dsp(args):
     e2e_v, e2e_h2d, e2e_d2h = e2e_run(False)
     e2e_hv, e2e_hh2d, e2e_hd2h = e2e_run(True)
 
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(args, cfg, ip, ix, feats, batches, args.cpu_seconds, weights=ew)
+    # ---- world > 1: NVLink bytes of a step (from untimed synchronous calls on the
+    # timed batches: the blocks are a pure function of seeds and rng_seed), the
+    # peer-read peak measured here, and per-layer exchange time from the stamps
+    nvl = None
+    if world > 1:
+        csp_l, gat_l, rows_l, phases = [], [], [], []
+        for j in range(min(KS, 5)):
+            blocks = s.sample(dev_batches[(W + j) % len(batches)], datagen.BASE_SEED + W + j, biased=biased)
+            ph = None if layer else multi_phase_us(s, L)
+            if ph is not None:
+                phases.append(ph)
+            c_, g_, r_ = remote_bytes(blocks, bnds, rank, cfg.dim)
+            csp_l.append(c_)
+            gat_l.append(g_)
+            rows_l.append(r_)
+        s.sync()
+        csp_step = reduce_sum_over_ranks(float(np.mean(csp_l))) / world     # per GPU (mean over ranks)
+        gat_step = reduce_sum_over_ranks(float(np.mean(gat_l))) / world
+        peer_peak, peer_rows = peer_read_peak(s, bnds, rank, world, cfg.dim)
+        nvl_achieved = (csp_step + gat_step) * KS / (t_max * 1e-3) / 1e9
+        layer_us = None
+        if phases:
+            layer_us = [{k: float(np.median([p[l][k] for p in phases])) for k in phases[0][l]} for l in range(L)]
+        nvl = {"achieved": nvl_achieved, "peak": peer_peak, "frac": nvl_achieved / peer_peak,
+               "bytes_per_step_per_gpu": csp_step + gat_step, "csp_exchange_bytes_per_step_per_gpu": csp_step,
+               "gather_remote_bytes_per_step_per_gpu": gat_step,
+               "remote_row_share": float(np.mean(rows_l)) / max(1.0, rows / KS),
+               "peak_kind": (f"measured in this run: dsp_gather_features of {peer_rows} contiguous rows owned by "
+                             "the other ranks, every rank at once (TMA reads of the peers' shards over their "
+                             "peer mappings), bytes read / max-over-ranks time"
+                             + ("; DSP_BENCH_SAME_GPU: every rank on one GPU, so 'peer' reads are local HBM"
+                                if os.environ.get("DSP_BENCH_SAME_GPU") else "")),
+               "layer_phase_us_rank0": layer_us}
 
-    kern_per_step = (1 if world == 1 else 5 * L + 1) if layer else 1
-    roof_kernel = (("k_lw_persistent" if world == 1 else "k_gather") if layer
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
+        # the oracle gathers from the whole feature table (rank 0's shard alone at N > 1)
+        full = feats if world == 1 else datagen.features(0, cfg.num_nodes, cfg.dim)
+        ew_full = ew if world == 1 or ew is None else datagen.edge_weights(ix, datagen.node_weights(cfg.num_nodes))
+        cpu = cpu_baseline(args, cfg, ip, ix, full, batches, args.cpu_seconds, weights=ew_full)
+        del full
+
+    kern_per_step = 1
+    roof_kernel = (("k_lw_persistent" if world == 1 else "k_lw_multi") if layer
                    else ("k_csp_persistent" if world == 1 else "k_csp_multi"))
     roofline = {"kernel": roof_kernel,
                 "bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
@@ -699,6 +862,18 @@ def run_dsp(args):
         a_w = (samp_b + gath_b + weight_b * KS) / (t_ms * 1e-3) / 1e9
         roofline.update({"achieved": a_w, "frac": a_w / peak, "weight_bytes_per_launch": weight_b,
                          "algorithmic_bytes_per_launch": (samp_b + gath_b) / KS + weight_b})
+    if nvl is not None:        # world > 1: the gather's remote rows and the CSP exchanges cross NVLink
+        roofline = {"kernel": roof_kernel, "bound": "nvlink", "achieved": nvl["achieved"], "peak": nvl["peak"],
+                    "unit": "GB/s", "frac": nvl["frac"], "traffic": None, "peak_kind": nvl["peak_kind"],
+                    "nvlink_bytes_per_step_per_gpu": nvl["bytes_per_step_per_gpu"],
+                    "csp_exchange_bytes_per_step_per_gpu": nvl["csp_exchange_bytes_per_step_per_gpu"],
+                    "gather_remote_bytes_per_step_per_gpu": nvl["gather_remote_bytes_per_step_per_gpu"],
+                    "remote_row_share": nvl["remote_row_share"],
+                    "hbm": {"achieved": achieved, "peak": peak, "frac": achieved / peak, "peak_kind": peak_kind,
+                            "algorithmic_bytes_per_launch": (samp_b + gath_b) / KS},
+                    "launch_ms_mean": step_mean, "concurrent_launches": K,
+                    "achieved_def": "NVLink bytes per step per GPU (remote frontier ids + returned rows + remote "
+                                    "feature rows, per requester, mean over ranks) x steps / max-over-ranks time"}
     if cold_b is not None:     # cold tier: the dominant stream is the cold rows over the host link
         link = measure_h2d_gbps()
         a_c = cold_b * KS / (t_ms * 1e-3) / 1e9
@@ -755,6 +930,7 @@ def run_dsp(args):
             "e2e_host_copy": {"value": e2e_hv, "unit": "edges/s", "h2d_bytes_per_step": e2e_hh2d,
                               "d2h_bytes_per_step": e2e_hd2h,
                               "api": "as e2e_sync, plus D2H of every block and all gathered features (PCIe-bound)"},
+            "layer_phase_us_rank0": (nvl or {}).get("layer_phase_us_rank0"),
             "gpu_launches": kern_per_step * KS + (K if pipelined else 0),  # timed region: one launch per step + flushes
             "clocks": clk.summary(),
         }
@@ -772,7 +948,8 @@ def main(argv=None):
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["dsp", "reference"], default="dsp")
     ap.add_argument("--config", default=None)
-    ap.add_argument("--cpu-seconds", type=float, default=15.0)
+    ap.add_argument("--cpu-seconds", type=float, default=60.0,
+                    help="bound on the oracle's timed CPU work (products: the full 192-batch epoch takes ~40 s)")
     ap.add_argument("--ref-max-seconds", type=float, default=60.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-breakdown", action="store_true")
@@ -787,6 +964,8 @@ def main(argv=None):
     ap.add_argument("--hot-frac", type=float, default=None,
                     help="cold-feature tier: fraction of each shard's rows kept in HBM (P:L114)")
     args = ap.parse_args(argv)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ and args.impl == "dsp":
+        return relaunch_under_torchrun(args.gpus, sys.argv[1:] if argv is None else list(argv))
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
     if args.config is None:

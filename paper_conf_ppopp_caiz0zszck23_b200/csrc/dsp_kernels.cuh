@@ -253,18 +253,13 @@ __device__ __forceinline__ void map_put(const LayerBufs &B, int32_t u, uint32_t 
   }
   map_st(map_find(B, u, epoch), mword(B, epoch, u, x));
 }
-// zero both parities of the relabel map in use (hash table or compact direct map)
-__device__ __forceinline__ void map_zero(const LayerBufs &B0, const LayerBufs &B1, int64_t tid, int64_t nthreads) {
-  if (B0.first32) {
-    for (int64_t i = tid; i < (int64_t)B0.n32; i += nthreads) {
-      B0.first32[i] = 0u;
-      B1.first32[i] = 0u;
-    }
-  } else if (B0.mask) {
-    for (int64_t i = tid; i <= (int64_t)B0.mask; i += nthreads) {
-      B0.first[i] = 0ull;
-      B1.first[i] = 0ull;
-    }
+// zero the relabel map in use (hash table or compact direct map; one map
+// serves every layer of a node-wise call)
+__device__ __forceinline__ void map_zero(const LayerBufs &B, int64_t tid, int64_t nthreads) {
+  if (B.first32) {
+    for (int64_t i = tid; i < (int64_t)B.n32; i += nthreads) B.first32[i] = 0u;
+  } else if (B.mask) {
+    for (int64_t i = tid; i <= (int64_t)B.mask; i += nthreads) B.first[i] = 0ull;
   }
 }
 __device__ __forceinline__ void mark(const LayerBufs &B, int32_t u, uint32_t epoch, uint32_t x) {
@@ -1156,8 +1151,8 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(const __grid_constant
   if (a.buf[0].first32) e0 = dwin_start(e0, (uint32_t)a.L);
   const bool hclear = hash_clear_due(a.persist, e0, (uint32_t)a.L, a.buf[0].mask, a.buf[0].first);
   const bool dclear = a.buf[0].first32 && dclear_due(a.persist, e0);
-  if (hclear || dclear) {  // zero both parities of the relabel map (once per ~255 / L calls)
-    map_zero(a.buf[0], a.buf[1], tid, nthreads);
+  if (hclear || dclear) {  // zero the relabel map (once per ~255 / L calls)
+    map_zero(a.buf[0], tid, nthreads);
     grid_barrier<TEAM>(a.hdr, bar);
   }
   if (tid == 0) {  // the host cleared the header just before the launch

@@ -380,8 +380,8 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ Mu
   if (a.buf[0].first32) e0 = dwin_start(e0, (uint32_t)a.L);
   const bool hclear = hash_clear_due(a.persist, e0, (uint32_t)a.L, a.buf[0].mask, a.buf[0].first);
   const bool dclear = a.buf[0].first32 && dclear_due(a.persist, e0);
-  if (hclear || dclear) {  // zero both parities of the relabel map (once per ~255 / L calls)
-    map_zero(a.buf[0], a.buf[1], tid, nthreads);
+  if (hclear || dclear) {  // zero the relabel map (once per ~255 / L calls)
+    map_zero(a.buf[0], tid, nthreads);
     grid_barrier<TEAM>(a.hdr, bar);
   }
   if (tid == 0) {

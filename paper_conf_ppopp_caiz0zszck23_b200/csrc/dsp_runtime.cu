@@ -102,10 +102,10 @@ struct Plan {
   int64_t S[DSP_MAX_LAYERS];       // max src
   int64_t max_F, max_slots;
   size_t off_hdr, off_agg, off_cnt[2], off_perm, off_rows[2], off_first[2], bytes;
-  size_t off_first32[2];            // compact direct map [2][N] (N <= DIRECT_MAP_MAX_N), else 0
+  size_t off_first32;               // compact direct map [N] (N <= DIRECT_MAP_MAX_N), else 0
   bool direct32;                    // node-wise relabel through the compact direct map
   int64_t hash_cap;                 // > 0: relabel hash table of hash_cap slots per parity (else direct map)
-  size_t off_hash[2];
+  size_t off_hash;                  // relabel hash table [hash_cap]
   // layer-wise scheme (make_plan_lw)
   int64_t ncap, big_cap;
   size_t off_P, off_c, off_off, off_slot_node, off_excl, off_newid, off_big;
@@ -263,9 +263,14 @@ constexpr int64_t DIRECT_MAP_MAX_N = 3 * 1000 * 1000;
 constexpr int64_t HASH_MAX_X = 1ll << 25;
 constexpr int64_t DIRECT32_MAX_X = 1ll << 24;
 
-// persist | hdr | first[2][N] (| first32[2][N] for direct-map sizes) at fixed
+// persist | hdr | first[2][N] (| first32[N] for direct-map sizes) at fixed
 // offsets for every plan, so that one workspace can serve calls of any size
 // and either scheme (the relabel maps' epoch words stay valid across them).
+// Node-wise calls use ONE relabel map for all layers: layer l + 1 marks with
+// a newer epoch tag, which beats every word of layer l, and no phase reads
+// layer l's map once layer l + 1 starts marking (the duplicates of layer l are
+// resolved through its edge slots, not the map), so half the L2 footprint of a
+// map per layer parity.
 size_t plan_common(Plan &p, int64_t N) {
   size_t o = align_up(sizeof(WsPersist), 256);
   p.off_hdr = o;
@@ -274,12 +279,11 @@ size_t plan_common(Plan &p, int64_t N) {
     p.off_first[b] = o;
     o = align_up(o + sizeof(unsigned long long) * std::max<int64_t>(1, N), 256);
   }
-  p.off_first32[0] = p.off_first32[1] = 0;
-  if (N <= DIRECT_MAP_MAX_N)
-    for (int b = 0; b < 2; ++b) {
-      p.off_first32[b] = o;
-      o = align_up(o + sizeof(uint32_t) * std::max<int64_t>(1, N), 256);
-    }
+  p.off_first32 = 0;
+  if (N <= DIRECT_MAP_MAX_N) {
+    p.off_first32 = o;
+    o = align_up(o + sizeof(uint32_t) * std::max<int64_t>(1, N), 256);
+  }
   return o;
 }
 
@@ -301,15 +305,13 @@ Plan make_plan(int64_t N, int64_t num_seeds, const int32_t *fanouts, int L, int 
   int64_t max_keys = 0;
   for (int l = 0; l < L; ++l) max_keys = std::max(max_keys, p.F[l] + p.E[l]);
   const bool hashed = max_keys < HASH_MAX_X && (relabel_mode == 2 || (relabel_mode == 0 && N > DIRECT_MAP_MAX_N));
-  p.direct32 = !hashed && relabel_mode != 3 && p.off_first32[0] != 0 && max_keys < DIRECT32_MAX_X;
+  p.direct32 = !hashed && relabel_mode != 3 && p.off_first32 != 0 && max_keys < DIRECT32_MAX_X;
   p.hash_cap = 0;
   if (hashed) {
     p.hash_cap = 1024;
     while (p.hash_cap < max_keys + max_keys / 2) p.hash_cap <<= 1;  // load factor <= 2/3
-    for (int b = 0; b < 2; ++b) {
-      p.off_hash[b] = o;
-      o = align_up(o + sizeof(unsigned long long) * (size_t)p.hash_cap, 256);
-    }
+    p.off_hash = o;
+    o = align_up(o + sizeof(unsigned long long) * (size_t)p.hash_cap, 256);
   }
   p.off_agg = o;
   o = align_up(o + sizeof(unsigned long long) * 2 * MAX_PERSIST_BLOCKS, 256);
@@ -483,16 +485,16 @@ LayerBufs bufs_of(const Call &k, int parity) {
   LayerBufs b{};
   b.cnt = reinterpret_cast<int32_t *>(k.ws + k.plan.off_cnt[parity]);
   b.rows = reinterpret_cast<int32_t *>(k.ws + k.plan.off_rows[parity]);
-  b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_first[parity]);
+  b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_first[0]);  // one map for all layers
   b.mask = 0;
   b.first32 = nullptr;
   b.n32 = 0;
   if (k.plan.direct32) {
-    b.first32 = reinterpret_cast<uint32_t *>(k.ws + k.plan.off_first32[parity]);
+    b.first32 = reinterpret_cast<uint32_t *>(k.ws + k.plan.off_first32);
     b.n32 = (uint32_t)k.c->N;
   }
   if (k.plan.hash_cap > 0) {
-    b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_hash[parity]);
+    b.first = reinterpret_cast<unsigned long long *>(k.ws + k.plan.off_hash);
     b.mask = (uint32_t)(k.plan.hash_cap - 1);
   }
   return b;

@@ -25,6 +25,15 @@ METRICS = {
     "launch__grid_size": "grid",
     "launch__block_size": "block",
     "sm__throughput.avg.pct_of_peak_sustained_elapsed": "sm_pct",
+    # sector efficiency: 32-B sectors per global-load request (1 = one sector per
+    # request; 4 B useful of a 32-B sector is what a random 4-byte id costs)
+    "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum": "ld_sectors",
+    "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum": "ld_requests",
+    "lts__t_sectors_srcunit_tex_op_read.sum": "l2_read_sectors",
+    "lts__t_sector_op_read_hit_rate.pct": "l2_read_hit_pct",
+    # NVLink (world > 1 captures)
+    "nvlrx__bytes.sum": "nvl_rx",
+    "nvltx__bytes.sum": "nvl_tx",
 }
 UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1e-9, "us": 1e-6, "ms": 1e-3, "nsecond": 1e-9, "usecond": 1e-6,
               "msecond": 1e-3, "second": 1}
@@ -64,8 +73,8 @@ def main(rep, launches, tag):
     lines = [f"# ncu summary `{tag}`", "",
              f"Source: `ncu --set full --clock-control none --import-source on` (`{os.path.basename(rep)}`);"
              " cold-cache, serialised replays: absolute times are not bench values.", "",
-             "| kernel | launches | duration us | DRAM read MB | DRAM write MB | DRAM % peak | L2 hit % | warps active % | regs | grid x block | top stalls |",
-             "|---|---|---|---|---|---|---|---|---|---|---|"]
+             "| kernel | launches | duration us | DRAM read MB | DRAM write MB | DRAM % peak | L2 hit % | sectors / ld request | NVLink rx / tx MB | warps active % | regs | grid x block | top stalls |",
+             "|---|---|---|---|---|---|---|---|---|---|---|---|---|"]
     traffic = {}
     for name, recs in kern.items():
         n = len(recs)
@@ -73,6 +82,9 @@ def main(rep, launches, tag):
         st = recs[-1]["stalls"]
         lines.append(f"| `{name}` | {n} | {avg('duration') * 1e6:.1f} | {avg('dram_read') / 1e6:.1f} | "
                      f"{avg('dram_write') / 1e6:.1f} | {avg('dram_pct'):.1f} | {avg('l2_hit_pct'):.1f} | "
+                     f"{avg('ld_sectors') / max(1.0, avg('ld_requests')):.2f} | "
+                     + (f"{avg('nvl_rx') / 1e6:.1f} / {avg('nvl_tx') / 1e6:.1f}" if any('nvl_rx' in r for r in recs) else "n/a")
+                     + " | "
                      f"{avg('occupancy_pct'):.1f} | {int(avg('regs'))} | {int(avg('grid'))} x {int(avg('block'))} | "
                      + ", ".join(f"{k} {100 * v:.0f}%" for k, v in st.items()) + " |")
         big = max(recs, key=lambda r: r.get("dram_read", 0) + r.get("dram_write", 0))  # the fused launch
