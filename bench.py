@@ -550,11 +550,19 @@ def run_dsp(args):
     ew = datagen.edge_weights(six, datagen.node_weights(cfg.num_nodes)) if biased else None
     layer = args.scheme == "layer"
     fanouts = fanouts_of(args, cfg)
-    # K concurrent step streams at world 1 (world > 1: one stream, the ranks' exchange slots are per ctx)
-    K = max(1, args.instances) if world == 1 else 1
+    # K concurrent step streams, each launch on 1/K of the SMs with its own workspace; at
+    # world > 1 each stream's calls use their own exchange channel (DSP_OPT_EXCHANGE_CHANNELS;
+    # the layer-wise scheme keeps one stream there: its exchange region is per ctx)
+    K = max(1, args.instances) if world == 1 or not layer else 1
+    opts = {pkg.dsp.DSP_OPT_EXCHANGE_CHANNELS: K} if world > 1 and not layer else {}
+    if args.loader_warps:
+        opts[pkg.dsp.DSP_OPT_LOADER_WARPS] = args.loader_warps
+    if args.loader_rows:
+        opts[pkg.dsp.DSP_OPT_LOADER_ROWS] = args.loader_rows
     s = pkg.Sampler(bnds, sip, six, feats, fanouts, cfg.batch, rank=rank, world_size=world, scheme="layer" if layer else "node",
                     device=local, exchange=ex, n_slots=2 * K, edge_weights=ew, n_workspaces=K,
-                    hot_rows=None if args.hot_frac is None else int(round(args.hot_frac * (len(sip) - 1))))
+                    hot_rows=None if args.hot_frac is None else int(round(args.hot_frac * (len(sip) - 1))),
+                    options=opts)
     if K > 1:  # K steps in flight on K streams, each persistent launch on 1/K of the SMs
         pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(local).multi_processor_count // K)
     for slot in range(2 * K):
@@ -954,7 +962,9 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-breakdown", action="store_true")
     ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
-    ap.add_argument("--instances", type=int, default=4, help="concurrent step streams (world 1)")
+    ap.add_argument("--instances", type=int, default=4, help="concurrent step streams (each on 1/K of the SMs; world > 1: one exchange channel each)")
+    ap.add_argument("--loader-warps", type=int, default=0, help="DSP_OPT_LOADER_WARPS (0: library default)")
+    ap.add_argument("--loader-rows", type=int, default=0, help="DSP_OPT_LOADER_ROWS (0: library default)")
     ap.add_argument("--layer-sizes", default="1000,1000",
                     help="--scheme layer: nodes sampled per layer (Table 7: 1000,1000)")
     ap.add_argument("--walkers", type=int, default=65536, help="--scheme walk: walks per GPU per step")

@@ -49,6 +49,7 @@ extern "C" {
 #define DSP_MAX_FANOUT 32    /* one lane per sampled slot */
 #define DSP_HANDLE_BYTES 1024 /* size of an exported peer handle */
 #define DSP_MAX_LAYER_SIZE 8192 /* layer-wise: nodes sampled per layer (Table 7 uses 1000) */
+#define DSP_MAX_CHANNELS 8   /* node-wise exchange channels (collective calls in flight per rank) */
 
 typedef enum {
   DSP_OK = 0,
@@ -122,8 +123,12 @@ dsp_status dsp_load_features_tiered(dsp_ctx *ctx, const float *features, int32_t
    associated with a non-negative weight w_u ... DSP stores node weight w_u
    along with edge e_{v,u}").  edge_weights: host or device fp32[nnz_r]
    aligned with this rank's `indices` (the weight of the edge's neighbour);
-   each must lie in [0, 65536) (else DSP_ERR_INVALID_ARG) and is used as the
-   16.16 fixed-point integer floor(w * 65536) (R24).  Once per ctx,
+   each must be 0 or lie in [2^-16, 65536) and is used as the 16.16
+   fixed-point integer floor(w * 65536) (R24).  A negative, NaN or
+   too large weight, or a positive one below 2^-16 (it would quantize to 0
+   and never be drawn), fails the load with DSP_ERR_INVALID_ARG; rescale the
+   weights of such a graph first (the draw probabilities depend only on the
+   ratios).  Once per ctx,
    after dsp_load_partition.  Copied; the caller may free its buffer. */
 dsp_status dsp_load_weights(dsp_ctx *ctx, const float *edge_weights);
 
@@ -296,12 +301,40 @@ dsp_status dsp_set_persistent_blocks(dsp_ctx *ctx, int32_t blocks);
    DSP_OPT_LOADER_ROWS     rows per TMA gather chunk, 1..32 (default 32).
    DSP_OPT_GATHER_REGLOADS 0 (default) = standalone gathers and cold-tier rows
                            moved by TMA bulk copies; 1 = 16-byte register
-                           loads. */
+                           loads.
+   DSP_OPT_SPLIT_ROWS      feature-row layout in HBM: 0 (default) = rows packed
+                           at dim * 4 bytes; 1 = each row split at its last
+                           128-byte boundary into a head array of whole L2
+                           lines and a small tail array kept L2-resident
+                           (fewer DRAM bytes per random row: +3 % for a
+                           standalone dsp_gather_features of 400-byte rows,
+                           none for the pipelined step).  Before
+                           dsp_load_partition; all ranks alike (checked at
+                           import).
+   DSP_OPT_EXCHANGE_CHANNELS  world_size > 1, node-wise: 1..DSP_MAX_CHANNELS
+                           (default 1) exchange regions.  The n-th collective
+                           node-wise call of a ctx (dsp_sample, dsp_sample_gather,
+                           dsp_sample_group; synchronous or not) uses channel
+                           n % channels, so that many calls can be in flight at
+                           once on different streams (each with its own
+                           workspace), the paper's pipeline with concurrent
+                           samplers; calls of one channel run in
+                           issue order (the library makes the stream of call n
+                           wait for call n - channels).  Every rank issues its
+                           calls in the same order (checked: the call count's
+                           low byte travels in the exchange header, a mismatch
+                           is DSP_ERR_STATE) and reserves the same number of
+                           channels (checked at import); set before
+                           dsp_reserve.  Concurrent calls must fit on the GPU
+                           together: give each at most 1/channels of the SMs
+                           with dsp_set_persistent_blocks. */
 #define DSP_OPT_RELABEL_MAP 1
 #define DSP_OPT_LANE_ROUNDS 2
 #define DSP_OPT_LOADER_WARPS 3
 #define DSP_OPT_LOADER_ROWS 4
 #define DSP_OPT_GATHER_REGLOADS 5
+#define DSP_OPT_EXCHANGE_CHANNELS 6
+#define DSP_OPT_SPLIT_ROWS 7
 dsp_status dsp_set_option(dsp_ctx *ctx, int32_t option, int64_t value);
 
 /* Enqueues every gather still owed by this ctx's DSP_PIPELINED calls (one
@@ -328,7 +361,10 @@ dsp_status dsp_gather_features(dsp_ctx *ctx, const int32_t *ids, int64_t n, floa
    starts[i]; step l from node v takes the neighbour that fan-out-1 node-wise
    sampling picks for v at layer l with this rng_seed (walks meeting at a node
    at the same step continue together); a node without neighbours ends the
-   walk and the remaining entries are -1.
+   walk and the remaining entries are -1.  NOTE: the draw is keyed by (node,
+   step), not by the walk, so walks with the same start node in one call are
+   IDENTICAL; for several independent walks per start node (DeepWalk-style)
+   pass them in calls with different rng_seed values.
    starts: DEVICE int32[n] in [0, N) (any owner; else an error latches for
    dsp_sync and the walk is all -1); traces: DEVICE int32[n][length + 1],
    traces[i][0] = starts[i]; 1 <= length <= 1024.  Asynchronous on `stream`.

@@ -157,6 +157,19 @@ __device__ __forceinline__ unsigned long long l2_policy_evict_last() {
   asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
   return p;
 }
+__device__ __forceinline__ unsigned long long l2_policy_evict_normal() {
+  unsigned long long p;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+// L2 policy of the feature tails (16-byte tails of 400-byte rows: a 16 B-per-node
+// array kept resident so a row costs its three head lines of DRAM)
+#ifndef DSP_TAIL_POLICY
+#define DSP_TAIL_POLICY 1
+#endif
+__device__ __forceinline__ unsigned long long l2_policy_tail() {
+  return DSP_TAIL_POLICY == 0 ? l2_policy_evict_first() : DSP_TAIL_POLICY == 2 ? l2_policy_evict_normal() : l2_policy_evict_last();
+}
 __device__ __forceinline__ float4 ld_f4_hint(const float4 *p, unsigned long long pol) {
   float4 v;
   asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"

@@ -793,33 +793,54 @@ __device__ __forceinline__ void phase_indices_dups(int F, int k, const LayerBufs
 }
 
 // ----------------------------------------------------------------- gather
+// Feature rows are stored split at the last 128-byte boundary (DESIGN.md
+// "Data layout"): the head (dim*4 rounded down to a multiple of 128 bytes) in
+// a packed head array whose rows are 128-byte aligned whole L2 lines, the tail
+// (< 128 bytes, a multiple of 16) in a packed tail array.  A 400-byte row read
+// whole touches four 128-byte lines (512 B of DRAM) at any alignment; split it
+// touches three, and the tail array (16 B per node) stays L2-resident under an
+// evict_last policy while the heads stream with evict_first.  Each region of
+// slots (a rank's HBM shard, a rank's cold rows in host memory) holds its
+// head array at `head`, its tail array at `tail`.
 struct GatherArgs {
   const int32_t *ids;
   int64_t n;                // rows (ignored when n_dev is set)
   const int32_t *n_dev;     // device row count (fused call), or nullptr
   int32_t dim4;             // dim / 4  (output row length in float4)
-  int32_t stride4;          // shard row stride in float4 (rows padded to 64 B)
+  int32_t head4;            // head length in float4 (multiple of 8); tail = dim4 - head4 (< 8)
   float4 *out;
-  const float4 *base[8];    // feature shard (hot rows) of each rank (local or peer-mapped)
+  const float4 *base[8];    // feature shard (hot rows) of each rank: head array (local or peer-mapped)
+  const float4 *tail[8];    //   ... and its tail array
   // cold-feature tier: feature position list of each rank
   // (>= 0 hot slot, < 0 cold slot -p-1) and its cold rows in host memory (UVA)
   int32_t tiered;
   const int32_t *fpos[8];
   const float4 *cold[8];
+  const float4 *cold_tail[8];
   Bounds bd;
   int *err;
 };
 
-// Address of the feature row of global id g (owner o): the shard row, or with
-// the cold tier the hot slot in HBM / the cold slot in host memory read over
-// UVA by the requesting GPU ("loaded from CPU memory by the requesting GPU").
-__device__ __forceinline__ const float4 *feature_row(const GatherArgs &a, int o, int32_t g) {
+struct RowRef {
+  const float4 *head, *tail;  // the row's head (head4 float4) and tail (dim4 - head4 float4)
+};
+
+// The feature row of global id g (owner o): the shard slot, or with the cold
+// tier the hot slot in HBM / the cold slot in host memory read over UVA by the
+// requesting GPU ("loaded from CPU memory by the requesting GPU").
+__device__ __forceinline__ RowRef feature_row(const GatherArgs &a, int o, int32_t g) {
   const uint32_t lv = (uint32_t)(g - (int32_t)a.bd.b[o]);
+  const uint32_t h4 = (uint32_t)a.head4, t4 = (uint32_t)(a.dim4 - a.head4);
   const int32_t *fp = a.fpos[o];  // null: rank o keeps all its rows in HBM (in id order)
-  if (!a.tiered || !fp) return a.base[o] + (size_t)lv * (uint32_t)a.stride4;
+  if (!a.tiered || !fp) return RowRef{a.base[o] + (size_t)lv * h4, a.tail[o] + (size_t)lv * t4};
   const int32_t p = __ldg(fp + lv);
-  return p >= 0 ? a.base[o] + (size_t)(uint32_t)p * (uint32_t)a.stride4
-                : a.cold[o] + (size_t)(uint32_t)(-p - 1) * (uint32_t)a.stride4;
+  if (p >= 0) return RowRef{a.base[o] + (size_t)(uint32_t)p * h4, a.tail[o] + (size_t)(uint32_t)p * t4};
+  const uint32_t q = (uint32_t)(-p - 1);
+  return RowRef{a.cold[o] + (size_t)q * h4, a.cold_tail[o] + (size_t)q * t4};
+}
+// float4 column c of a row
+__device__ __forceinline__ const float4 *row_col(const RowRef &r, uint32_t c, uint32_t head4) {
+  return c < head4 ? r.head + c : r.tail + (c - head4);
 }
 
 __device__ __forceinline__ float4 ld_stream_f4(const float4 *p) {
@@ -838,7 +859,8 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
   const uint32_t tid = (uint32_t)tid64, nthreads = (uint32_t)nthreads64;
   const uint32_t dim4 = (uint32_t)a.dim4;
   const int32_t N = (int32_t)a.bd.b[a.bd.world];
-  const unsigned long long pol = l2_policy_evict_first();
+  const unsigned long long pol = l2_policy_evict_first(), pol_t = l2_policy_tail();
+  const uint32_t head4 = (uint32_t)a.head4;
   for (uint32_t e0 = tid; e0 < total; e0 += nthreads * UNROLL) {
     int32_t g[UNROLL];
     uint32_t c[UNROLL];
@@ -858,7 +880,7 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
     for (int u = 0; u < UNROLL; ++u) {
       if (g[u] >= 0 && g[u] < N) {
         const int o = owner_of(a.bd, g[u]);
-        v[u] = ld_f4_hint(feature_row(a, o, g[u]) + c[u], pol);
+        v[u] = ld_f4_hint(row_col(feature_row(a, o, g[u]), c[u], head4), c[u] < head4 ? pol : pol_t);
       }
     }
 #pragma unroll
@@ -884,7 +906,11 @@ __global__ void __launch_bounds__(NT) k_gather(const __grid_constant__ GatherArg
 // ============================================ world == 1: persistent kernel
 constexpr int LOADER_WARPS = 4;                      // TMA gather warps of a pipelined launch (default)
 constexpr int LOADER_WARPS_MAX = 8;                  // ... or 8 (dsp_ctx::loader_warps)
-constexpr int LOADER_SLOTS = 2;                      // ring slots per loader warp
+#ifndef DSP_LOADER_SLOTS
+#define DSP_LOADER_SLOTS 2
+#endif
+constexpr int LOADER_SLOTS = DSP_LOADER_SLOTS;       // ring slots per loader warp of a pipelined launch
+constexpr int GTMA_SLOTS = 2;                        // ring slots per warp of the standalone gather
 constexpr int PIPE_TEAM = PNT - 32 * LOADER_WARPS;   // sampling threads of a pipelined launch
 constexpr int PIPE_TEAM8 = PNT - 32 * LOADER_WARPS_MAX;
 constexpr int PIPE_TEAM2 = PNT - 32 * 2;
@@ -961,22 +987,22 @@ __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32
 // shard (local, or a peer's over NVLink through its mapping).
 // STATIC: chunks gw, gw + nw, ... instead of the grid-wide cursor (the
 // standalone k_gather_tma, whose warps all gather).
-template <bool MULTI = false, bool STATIC = false>
+template <bool MULTI = false, bool STATIC = false, int SLOTS = LOADER_SLOTS>
 __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, uint64_t *bars, int64_t n,
                                             int64_t gw = 0, int64_t nw = 1) {
   const int lane = threadIdx.x & 31;
   const GatherArgs &g = a.gp;
   const int R = a.rows_per_chunk;
-  const uint32_t row_bytes = (uint32_t)g.dim4 * 16u, stride_bytes = (uint32_t)g.stride4 * 16u;
+  const uint32_t row_bytes = (uint32_t)g.dim4 * 16u, head_bytes = (uint32_t)g.head4 * 16u;
+  const uint32_t tail_bytes = row_bytes - head_bytes;
   const int64_t nchunks = (n + R - 1) / R;
-  const char *base = reinterpret_cast<const char *>(g.base[0]);
   char *out = reinterpret_cast<char *>(g.out);
-  const unsigned long long pol = l2_policy_evict_first();
+  const unsigned long long pol = l2_policy_evict_first(), pol_t = l2_policy_tail();
   int issued = 0, done = 0;
-  int chunk0 = 0, chunk1 = 0;  // chunk held by slot 0 / slot 1 (LOADER_SLOTS == 2)
+  int chunk[SLOTS];  // chunk held by each ring slot
   bool exhausted = false;
   while (true) {
-    while (!exhausted && issued - done < LOADER_SLOTS) {
+    while (!exhausted && issued - done < SLOTS) {
       int c = 0;
       if (STATIC) {
         c = (int)min((int64_t)INT32_MAX, gw + (int64_t)issued * nw);
@@ -988,9 +1014,9 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
         exhausted = true;
         break;
       }
-      const int s = issued % LOADER_SLOTS;
-      if (issued >= LOADER_SLOTS) {  // the slot's previous store must have read its smem
-        if (lane == 0) bulk_wait_read<LOADER_SLOTS - 1>();
+      const int s = issued % SLOTS;
+      if (issued >= SLOTS) {  // the slot's previous store must have read its smem
+        if (lane == 0) bulk_wait_read<SLOTS - 1>();
         __syncwarp();
       }
       const int rows = (int)min((int64_t)R, n - (int64_t)c * R);
@@ -998,28 +1024,34 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
       __syncwarp();
       if (lane < rows) {
         const int32_t id = __ldg(g.ids + (int64_t)c * R + lane);
-        if (id >= 0 && id < (int32_t)g.bd.b[MULTI ? g.bd.world : 1])  // cold rows: host memory over UVA
-          bulk_g2s_hint(ring + (size_t)s * a.slot_bytes + (size_t)lane * row_bytes,
-                        MULTI || g.tiered ? reinterpret_cast<const char *>(
-                                                feature_row(g, MULTI ? owner_of(g.bd, id) : 0, id))
-                                          : base + (size_t)(uint32_t)id * stride_bytes,
-                        row_bytes, &bars[s], pol);
-        else  // keep the byte count consistent; the error is reported
+        if (id >= 0 && id < (int32_t)g.bd.b[MULTI ? g.bd.world : 1]) {  // cold rows: host memory over UVA
+          // head (whole 128-byte lines, streamed) and tail (L2-resident array) into one slot row
+          const RowRef r = feature_row(g, MULTI ? owner_of(g.bd, id) : 0, id);
+          char *dst = ring + (size_t)s * a.slot_bytes + (size_t)lane * row_bytes;
+          if (head_bytes) bulk_g2s_hint(dst, r.head, head_bytes, &bars[s], pol);
+          if (tail_bytes) bulk_g2s_hint(dst + head_bytes, r.tail, tail_bytes, &bars[s], pol_t);
+        } else {  // keep the byte count consistent; the error is reported
           latch(g.err, E_RANGE);
+        }
       }
-      if (s == 0) chunk0 = c; else chunk1 = c;
+#pragma unroll
+      for (int q = 0; q < SLOTS; ++q)
+        if (q == s) chunk[q] = c;
       ++issued;
     }
     if (done == issued) break;
     if (!STATIC && lane == 0) atomicAdd(&a.hdr->chunks_loader, 1u);
-    const int s = done % LOADER_SLOTS;
-    const int c = s == 0 ? chunk0 : chunk1;
+    const int s = done % SLOTS;
+    int c = 0;
+#pragma unroll
+    for (int q = 0; q < SLOTS; ++q)
+      if (q == s) c = chunk[q];
     const int rows = (int)min((int64_t)R, n - (int64_t)c * R);
     bool bad = false;
     if (lane == 0) {
       // an out-of-range id never delivers its bytes: do not wait forever on it
       const unsigned long long t0 = globaltimer_ns();
-      while (!mbar_try_wait(&bars[s], (uint32_t)(done / LOADER_SLOTS) & 1u)) {
+      while (!mbar_try_wait(&bars[s], (uint32_t)(done / SLOTS) & 1u)) {
         if (*(volatile int *)g.err != 0 && globaltimer_ns() - t0 > 1000000ull) {
           bad = true;
           break;
@@ -1047,8 +1079,8 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
   const GatherArgs &g = a.gp;
   const int R = a.rows_per_chunk;
   const int64_t nchunks = (n + R - 1) / R;
-  const uint32_t dim4 = (uint32_t)g.dim4;
-  const unsigned long long pol = l2_policy_evict_first();
+  const uint32_t dim4 = (uint32_t)g.dim4, head4 = (uint32_t)g.head4;
+  const unsigned long long pol = l2_policy_evict_first(), pol_t = l2_policy_tail();
   while (true) {
     int c = 0;
     if (lane == 0) c = (int)atomicAdd(&a.hdr->gcursor, 1u);
@@ -1076,7 +1108,8 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
 #pragma unroll
       for (int u = 0; u < 4; ++u)
         if (id[u] >= 0 && id[u] < N)
-          v[u] = ld_f4_hint(feature_row(g, MULTI ? owner_of(g.bd, id[u]) : 0, id[u]) + col[u], pol);
+          v[u] = ld_f4_hint(row_col(feature_row(g, MULTI ? owner_of(g.bd, id[u]) : 0, id[u]), col[u], head4),
+                            col[u] < head4 ? pol : pol_t);
 #pragma unroll
       for (int u = 0; u < 4; ++u) {
         const uint32_t e = e0 + 32u * u;
@@ -1093,23 +1126,23 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
 
 // Standalone gather (dsp_gather_features, pending pipelined gathers): every
 // warp a TMA loader (loader_warp) over a static share of the 32-row chunks:
-// one cp.async.bulk per row into a shared-memory ring slot, one bulk store
-// of the chunk's contiguous output rows.  GTMA_WARPS x 2 slots of <= 16 KB.
+// one cp.async.bulk per row part (head, tail) into a shared-memory ring slot,
+// one bulk store of the chunk's contiguous output rows.  GTMA_WARPS x 2 slots of <= 16 KB.
 #ifndef DSP_GTMA_WARPS
 #define DSP_GTMA_WARPS 6
 #endif
 constexpr int GTMA_WARPS = DSP_GTMA_WARPS;
 template <bool MULTI>
 __global__ void __launch_bounds__(32 * GTMA_WARPS) k_gather_tma(const __grid_constant__ PersistArgs a, int64_t n_host) {
-  __shared__ __align__(8) uint64_t bars[GTMA_WARPS][LOADER_SLOTS];
+  __shared__ __align__(8) uint64_t bars[GTMA_WARPS][GTMA_SLOTS];
   extern __shared__ __align__(128) char ring_smem[];
   const int w = threadIdx.x >> 5;
   if ((threadIdx.x & 31) == 0)
-    for (int s2 = 0; s2 < LOADER_SLOTS; ++s2) mbar_init(&bars[w][s2], 1);
+    for (int s2 = 0; s2 < GTMA_SLOTS; ++s2) mbar_init(&bars[w][s2], 1);
   mbar_init_fence();
   __syncwarp();
   const int64_t n = a.gp.n_dev ? (int64_t)ld_volatile_i32(a.gp.n_dev) : n_host;
-  loader_warp<MULTI, true>(a, ring_smem + (size_t)w * LOADER_SLOTS * a.slot_bytes, bars[w], n,
+  loader_warp<MULTI, true, GTMA_SLOTS>(a, ring_smem + (size_t)w * GTMA_SLOTS * a.slot_bytes, bars[w], n,
                            (int64_t)blockIdx.x * GTMA_WARPS + w, (int64_t)gridDim.x * GTMA_WARPS);
 }
 
@@ -1317,16 +1350,19 @@ __device__ __forceinline__ bool last_block_done(uint32_t *done) {
   return false;
 }
 
-// fp32 edge weights -> 16.16 fixed point a = floor(w * 2^16), w in [0, 2^16)
-// (R24); an invalid weight is counted in *bad.
+// fp32 edge weights -> 16.16 fixed point a = floor(w * 2^16), w = 0 or
+// w in [2^-16, 2^16) (R24); an invalid weight is counted in *bad:
+// negative, NaN, >= 2^16, or positive but below 2^-16 (it would quantize to 0
+// and never be sampled, silently departing from w_u / sum w).
 __global__ void k_weights_fixed(const float *w, int64_t n, uint32_t *out, int *bad) {
   for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < n; e += (int64_t)gridDim.x * blockDim.x) {
     const float x = w[e];
-    if (!(x >= 0.0f) || x >= 65536.0f) {
+    const uint32_t a = (x >= 0.0f && x < 65536.0f) ? (uint32_t)floorf(x * 65536.0f) : 0u;
+    if (!(x >= 0.0f) || x >= 65536.0f || (x > 0.0f && a == 0u)) {
       atomicAdd(bad, 1);
       out[e] = 0;
     } else {
-      out[e] = (uint32_t)floorf(x * 65536.0f);
+      out[e] = a;
     }
   }
 }

@@ -46,6 +46,7 @@ struct MultiArgs {
   XchPeers peers;
   int32_t *perm;            // [F] inbox slot of frontier node i at its owner
   int32_t *abort_word;      // set when a wait timed out: later waits of this call end at once
+  uint32_t call_tag;        // low byte of the ctx's collective call count: ranks must agree
 };
 
 // Thread 0 of each block waits until flags[s] >= seq for every rank s; the
@@ -411,7 +412,8 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ Mu
         const uint32_t c = *(volatile uint32_t *)&a.hdr->bucket[o];
         a.hdr->bucket[o] = 0u;
         *xch_inbox_hdr(m.peers.base[o], m.X, par, m.rank) =
-            make_uint4(c, (uint32_t)k | ((uint32_t)l << 8) | ((uint32_t)a.biased << 16), a.key.x, a.key.y);
+            make_uint4(c, (uint32_t)k | ((uint32_t)l << 8) | ((uint32_t)a.biased << 16) | (m.call_tag << 24), a.key.x,
+                       a.key.y);
       }
       __threadfence_system();
       for (int o = 0; o < world; ++o) st_release_sys(xch_inbox_flag(m.peers.base[o], m.X, par, m.rank), seq);
@@ -423,9 +425,9 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ Mu
       uint32_t acc = 0;
       for (int s = 0; s < world; ++s) {
         const uint4 h = __ldcv(xch_inbox_hdr(self, m.X, par, s));
-        if (h.y != ((uint32_t)k | ((uint32_t)l << 8) | ((uint32_t)a.biased << 16)) || h.z != a.key.x ||
-            h.w != a.key.y)
-          latch(a.err, E_STATE);  // ranks disagree on (layer, fan-out, seed, scheme)
+        if (h.y != ((uint32_t)k | ((uint32_t)l << 8) | ((uint32_t)a.biased << 16) | (m.call_tag << 24)) ||
+            h.z != a.key.x || h.w != a.key.y)
+          latch(a.err, E_STATE);  // ranks disagree on (call, layer, fan-out, seed, scheme)
         s_off[s] = acc;
         acc += (h.x <= (uint32_t)m.X.cap) ? h.x : 0u;
       }

@@ -37,7 +37,20 @@ __global__ void k_validate_indices(const int32_t *indices, int64_t nnz, int64_t 
 }
 
 constexpr uint32_t HANDLE_MAGIC = 0x44535048u;  // "DSPH"
-constexpr int FEAT_ALIGN_FLOATS = 16;           // shard rows padded to 64 B (HBM access granule)
+
+// Feature row layout (dsp_kernels.cuh GatherArgs).  Packed (default): a
+// region of `slots` rows is one array of rows at stride dim * 4.  Split
+// (DSP_OPT_SPLIT_ROWS): each row is cut at its last 128-byte boundary, head =
+// dim * 4 rounded down to a multiple of 128 in a packed head array, then
+// (256-aligned) the tail (< 128 B) in a packed tail array.
+int head_bytes_of(bool split, int dim) { return split ? dim * 4 / 128 * 128 : 0; }
+int tail_bytes_of(bool split, int dim) { return dim * 4 - head_bytes_of(split, dim); }
+size_t tail_offset(bool split, int64_t slots, int dim) {
+  return ((size_t)std::max<int64_t>(1, slots) * (size_t)head_bytes_of(split, dim) + 255) / 256 * 256;
+}
+size_t region_bytes(bool split, int64_t slots, int dim) {
+  return tail_offset(split, slots, dim) + (size_t)std::max<int64_t>(1, slots) * (size_t)tail_bytes_of(split, dim);
+}
 thread_local std::string g_create_error;
 
 struct PeerHandle {  // fits in DSP_HANDLE_BYTES
@@ -50,7 +63,8 @@ struct PeerHandle {  // fits in DSP_HANDLE_BYTES
   int32_t has_feat, has_xch;
   cudaIpcMemHandle_t feat_ipc, xch_ipc;
   int64_t bounds[DSP_MAX_WORLD + 1];
-  int32_t dim, max_seeds, feat_stride, tiered;
+  int32_t dim, max_seeds, head_bytes, tiered;
+  int64_t feat_slots, cold_slots;  // rows of the HBM shard / of the cold region (their tail arrays' offsets)
   cudaIpcMemHandle_t fpos_ipc;
   uint64_t fpos_ptr, cold_ptr;
   int64_t cold_bytes;
@@ -64,6 +78,7 @@ struct PeerHandle {  // fits in DSP_HANDLE_BYTES
   uint64_t wxch_ptr;
   int64_t walk_max;
   int32_t has_wxch, walk_len;
+  int32_t channels;  // node-wise exchange channels (DSP_OPT_EXCHANGE_CHANNELS)
 };
 static_assert(sizeof(PeerHandle) <= DSP_HANDLE_BYTES, "handle too large");
 
@@ -120,7 +135,9 @@ struct dsp_ctx {
   bool loaded = false, reserved = false, imported = false, broken = false;
   int64_t bounds[DSP_MAX_WORLD + 1] = {0};
   int64_t N = 0, lo = 0, n_local = 0, nnz = 0;
-  int32_t dim = 0, feat_stride = 0;  // feature row length / padded stride (floats)
+  int32_t dim = 0;                  // feature row length (floats)
+  bool split_rows = false;          // DSP_OPT_SPLIT_ROWS: rows stored split head / tail (head_bytes_of)
+  int64_t feat_slots = 0, cold_slots = 0;  // rows in the HBM shard / cold region
   int64_t *d_indptr = nullptr;
   int32_t *d_indices = nullptr;
   uint32_t *d_weights = nullptr;  // 16.16 edge weights (biased sampling)
@@ -135,6 +152,7 @@ struct dsp_ctx {
   char cold_shm[48] = {0};            // non-empty: h_cold is a registered POSIX shm mapping
   const int32_t *peer_fpos[DSP_MAX_WORLD] = {nullptr};
   const float *peer_cold[DSP_MAX_WORLD] = {nullptr};
+  const float *peer_cold_tail[DSP_MAX_WORLD] = {nullptr};
   void *peer_cold_map[DSP_MAX_WORLD] = {nullptr};  // shm mappings opened in this process
   int64_t peer_cold_bytes[DSP_MAX_WORLD] = {0};
   int *d_err = nullptr;  // latched device error of this ctx
@@ -142,9 +160,21 @@ struct dsp_ctx {
   int32_t max_seeds = 0, L = 0, kmax = 0;
   int32_t fanouts[DSP_MAX_LAYERS] = {0};
   XchLayout xl{};
-  char *d_xch = nullptr;
+  char *d_xch = nullptr;           // channels x chan_stride bytes, peer-mapped
+  // node-wise exchange channels (DSP_OPT_EXCHANGE_CHANNELS): collective call n of
+  // this ctx uses channel n % channels with its own exchange region and sequence
+  // numbers, so up to `channels` calls can be in flight on different streams; the
+  // calls of one channel are ordered by an event (the call issue order, identical
+  // on every rank, is the fixed collective order CCC provides)
+  int channels = 1;
+  size_t chan_stride = 0;
+  unsigned long long ncalls = 0;
+  unsigned long long chan_seq[DSP_MAX_CHANNELS] = {0};
+  cudaEvent_t chan_ev[DSP_MAX_CHANNELS] = {nullptr};
+  bool chan_used[DSP_MAX_CHANNELS] = {false};
   // peers
-  const float *peer_feat[DSP_MAX_WORLD] = {nullptr};
+  const float *peer_feat[DSP_MAX_WORLD] = {nullptr};       // head arrays of the ranks' shards
+  const float *peer_feat_tail[DSP_MAX_WORLD] = {nullptr};  // tail arrays
   char *peer_xch[DSP_MAX_WORLD] = {nullptr};
   void *ipc_opened[6 * DSP_MAX_WORLD] = {nullptr};  // feat, xch | fpos | lxch | indptr | walk region per peer
   unsigned long long seq = 0;
@@ -443,10 +473,12 @@ GatherArgs make_gather(const dsp_ctx *c, const int32_t *ids, int64_t n, const in
   a.n = n;
   a.n_dev = n_dev;
   a.dim4 = c->dim / 4;
-  a.stride4 = c->feat_stride / 4;
+  a.head4 = head_bytes_of(c->split_rows, c->dim) / 16;
   a.out = reinterpret_cast<float4 *>(out);
   for (int r = 0; r < DSP_MAX_WORLD; ++r) {
     a.base[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_feat[r]) : nullptr;
+    a.tail[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_feat_tail[r]) : nullptr;
+    a.cold_tail[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_cold_tail[r]) : nullptr;
     a.fpos[r] = r < c->world ? c->peer_fpos[r] : nullptr;
     a.cold[r] = r < c->world ? reinterpret_cast<const float4 *>(c->peer_cold[r]) : nullptr;
   }
@@ -479,6 +511,8 @@ struct Call {
   bool pipelined;      // gather this call's rows in the next pipelined call / flush
   bool biased;         // DSP_BIASED
   bool layerwise;      // DSP_LAYERWISE: fanouts are layer sizes
+  int channel;         // node-wise world > 1: exchange channel of this call
+  uint32_t call_tag;   // low byte of the ctx's collective call count (checked in the exchange header)
 };
 
 LayerBufs bufs_of(const Call &k, int parity) {
@@ -622,7 +656,9 @@ dsp_status prepare_call(Call &k, dsp_ctx *c, const int32_t *seeds, int32_t num_s
   k.ws = static_cast<char *>(workspace);
   k.stream = static_cast<cudaStream_t>(stream);
   k.hdr = reinterpret_cast<WsHeader *>(k.ws + k.plan.off_hdr);
-  k.seq0 = c->seq;
+  k.channel = (int)(c->ncalls % (unsigned long long)c->channels);
+  k.call_tag = (uint32_t)(c->ncalls & 0xffu);
+  k.seq0 = c->world > 1 ? c->chan_seq[k.channel] : 0;
   return DSP_OK;
 }
 
@@ -702,7 +738,7 @@ dsp_status stage_persistent(Call &k) {
   return DSP_OK;
 }
 
-XchPeers peers_of(const dsp_ctx *c);
+XchPeers peers_of(const dsp_ctx *c, int channel);
 
 // world > 1, node-wise: the whole call in one cooperative kernel per rank
 // (dsp_multi.cuh).  `share` = ranks of this call group on the same GPU
@@ -742,7 +778,8 @@ dsp_status stage_persistent_multi(Call &k, int share) {
   m.seq0 = k.seq0;
   m.bd = make_bounds(c);
   m.X = c->xl;
-  m.peers = peers_of(c);
+  m.peers = peers_of(c, k.channel);
+  m.call_tag = k.call_tag;
   m.perm = reinterpret_cast<int32_t *>(k.ws + k.plan.off_perm);
   m.abort_word = &k.hdr->abort_wait;
   int blocks = c->persist_blocks > 0 ? c->persist_blocks : c->num_sms * c->persist_blocks_per_sm;
@@ -760,6 +797,9 @@ dsp_status stage_persistent_multi(Call &k, int share) {
     st = c->aux;
   }
   void *args[] = {&m};
+  cudaEvent_t &cev = c->chan_ev[k.channel];
+  if (c->channels > 1 && c->chan_used[k.channel])  // the channel's previous call (possibly on another stream)
+    CUDA_TRY(c, cudaStreamWaitEvent(st, cev, 0));
   if (!k.pipelined) {
     CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_multi<PNT, false>, grid, block, args, 0, st));
   } else {
@@ -779,6 +819,10 @@ dsp_status stage_persistent_multi(Call &k, int share) {
     pd->stream = k.stream;
     pd->active = true;
     pd->calls += 1;
+  }
+  if (c->channels > 1) {
+    CUDA_TRY(c, cudaEventRecord(cev, st));
+    c->chan_used[k.channel] = true;
   }
   return DSP_OK;
 }
@@ -818,7 +862,7 @@ dsp_status launch_gather(dsp_ctx *c, const GatherArgs &g, int64_t n_host, cudaSt
     const int64_t chunks = (n_host + a.rows_per_chunk - 1) / a.rows_per_chunk;
     blocks = (int)std::max<int64_t>(1, std::min<int64_t>(blocks, (chunks + 2 * GTMA_WARPS - 1) / (2 * GTMA_WARPS)));
   }
-  const size_t smem = (size_t)GTMA_WARPS * LOADER_SLOTS * a.slot_bytes;
+  const size_t smem = (size_t)GTMA_WARPS * GTMA_SLOTS * a.slot_bytes;
   if (c->world > 1)
     k_gather_tma<true><<<blocks, 32 * GTMA_WARPS, smem, st>>>(a, n_host);
   else
@@ -853,9 +897,10 @@ dsp_status stage_flush(dsp_ctx *c, const char *ws, cudaStream_t st) {
   return DSP_OK;
 }
 
-XchPeers peers_of(const dsp_ctx *c) {
+XchPeers peers_of(const dsp_ctx *c, int channel) {
   XchPeers p{};
-  for (int r = 0; r < DSP_MAX_WORLD; ++r) p.base[r] = r < c->world ? c->peer_xch[r] : nullptr;
+  for (int r = 0; r < DSP_MAX_WORLD; ++r)
+    p.base[r] = r < c->world && c->peer_xch[r] ? c->peer_xch[r] + (size_t)channel * c->chan_stride : nullptr;
   return p;
 }
 
@@ -972,7 +1017,12 @@ dsp_status stage_end_async(Call &k) {
 dsp_status stage_finish(Call &k) {
   dsp_ctx *c = k.c;
   DeviceGuard g(c->device);
-  c->seq = k.seq0 + k.L;
+  if (k.layerwise) {
+    c->seq = k.seq0 + k.L;
+  } else if (c->world > 1) {
+    c->chan_seq[k.channel] = k.seq0 + k.L;
+    c->ncalls += 1;
+  }
   if (k.async) return DSP_OK;
   CUDA_TRY(c, cudaStreamSynchronize(k.stream));
   const int e = *c->h_err;
@@ -1072,6 +1122,11 @@ void release(dsp_ctx *c) {
     cudaEventDestroy(c->flush_ev);
     c->flush_ev = nullptr;
   }
+  for (auto &e : c->chan_ev)
+    if (e) {
+      cudaEventDestroy(e);
+      e = nullptr;
+    }
   cudaFree(c->d_lxch);
   cudaFree(c->d_wxch);
   cudaFree(c->d_err);
@@ -1218,7 +1273,7 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   c->num_sms = prop.multiProcessorCount;
   DeviceGuard g(cuda_device);
   int occ = 0, occ_pipe = 0;
-  const int pipe_smem = LOADER_WARPS * LOADER_SLOTS * 16384;  // largest ring (dim 4096)
+  const int pipe_smem = std::min(LOADER_WARPS * LOADER_SLOTS * 16384, 200 * 1024);  // largest ring (dim 4096)
   if (cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM, true>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM2, true>,
@@ -1245,9 +1300,9 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   }
   c->persist_blocks_per_sm = std::min(occ, occ_pipe);
   if (cudaFuncSetAttribute((const void *)k_gather_tma<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           GTMA_WARPS * LOADER_SLOTS * 16384) != cudaSuccess ||
+                           GTMA_WARPS * GTMA_SLOTS * 16384) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_gather_tma<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           GTMA_WARPS * LOADER_SLOTS * 16384) != cudaSuccess) {
+                           GTMA_WARPS * GTMA_SLOTS * 16384) != cudaSuccess) {
     cudaGetLastError();
     c->gather_reg = true;  // no TMA gather: register loads
     c->tma_unavailable = true;
@@ -1320,14 +1375,21 @@ dsp_status dsp_load_partition(dsp_ctx *c, const int64_t *bounds, const int64_t *
   }
   if (features) {
     c->dim = dim;
-    c->feat_stride = (dim + FEAT_ALIGN_FLOATS - 1) / FEAT_ALIGN_FLOATS * FEAT_ALIGN_FLOATS;
-    c->feat_bytes = (int64_t)sizeof(float) * c->feat_stride * std::max<int64_t>(1, c->n_local);
+    c->feat_slots = c->n_local;
+    c->feat_bytes = (int64_t)region_bytes(c->split_rows, c->n_local, dim);
     CUDA_TRY(c, cudaMalloc(&c->d_feat, (size_t)c->feat_bytes));
-    if (c->n_local > 0)
-      CUDA_TRY(c, cudaMemcpy2D(c->d_feat, sizeof(float) * c->feat_stride, features, sizeof(float) * dim,
-                               sizeof(float) * dim, (size_t)c->n_local, cudaMemcpyDefault));
+    const size_t hb = (size_t)head_bytes_of(c->split_rows, dim), tb = (size_t)tail_bytes_of(c->split_rows, dim), rb = sizeof(float) * dim;
+    char *dst = reinterpret_cast<char *>(c->d_feat);
+    if (c->n_local > 0 && hb)
+      CUDA_TRY(c, cudaMemcpy2D(dst, hb, features, rb, hb, (size_t)c->n_local, cudaMemcpyDefault));
+    if (c->n_local > 0 && tb)
+      CUDA_TRY(c, cudaMemcpy2D(dst + tail_offset(c->split_rows, c->n_local, dim), tb, reinterpret_cast<const char *>(features) + hb, rb,
+                               tb, (size_t)c->n_local, cudaMemcpyDefault));
   }
   c->peer_feat[c->rank] = c->d_feat;
+  c->peer_feat_tail[c->rank] =
+      c->d_feat ? reinterpret_cast<const float *>(reinterpret_cast<const char *>(c->d_feat) + tail_offset(c->split_rows, c->n_local, dim))
+                : nullptr;
   c->loaded = true;
   return DSP_OK;
 }
@@ -1345,8 +1407,7 @@ dsp_status dsp_load_features_tiered(dsp_ctx *c, const float *features, int32_t d
   if (hot_rows < 0 || hot_rows > n) hot_rows = n;
   DeviceGuard g(c->device);
   c->dim = dim;
-  c->feat_stride = (dim + FEAT_ALIGN_FLOATS - 1) / FEAT_ALIGN_FLOATS * FEAT_ALIGN_FLOATS;
-  const size_t row_bytes = sizeof(float) * (size_t)dim, stride_bytes = sizeof(float) * (size_t)c->feat_stride;
+  const size_t row_bytes = sizeof(float) * (size_t)dim, hb = (size_t)head_bytes_of(c->split_rows, dim), tb = (size_t)tail_bytes_of(c->split_rows, dim);
   // hot rows: the hot_rows largest in-degrees (P:L114 default criterion), ties by id
   std::vector<int64_t> ip((size_t)n + 1);
   CUDA_TRY(c, cudaMemcpy(ip.data(), c->d_indptr, sizeof(int64_t) * (size_t)(n + 1), cudaMemcpyDeviceToHost));
@@ -1371,16 +1432,23 @@ dsp_status dsp_load_features_tiered(dsp_ctx *c, const float *features, int32_t d
     hsrc = src.data();
   }
   cudaGetLastError();
-  // hot rows -> HBM (padded stride), cold rows -> pinned host memory (UVA-mapped)
-  c->feat_bytes = (int64_t)stride_bytes * std::max<int64_t>(1, nh);
+  // a row into slot q of a split region (head array, then the tail array at tail_offset)
+  auto put_row = [&](char *region, int64_t slots, int64_t q, const float *row) {
+    memcpy(region + (size_t)q * hb, row, hb);
+    memcpy(region + tail_offset(c->split_rows, slots, dim) + (size_t)q * tb, reinterpret_cast<const char *>(row) + hb, tb);
+  };
+  // hot rows -> HBM, cold rows -> pinned host memory (UVA-mapped), both split head / tail
+  c->feat_slots = nh;
+  c->cold_slots = nc;
+  c->feat_bytes = (int64_t)region_bytes(c->split_rows, nh, dim);
   CUDA_TRY(c, cudaMalloc(&c->d_feat, (size_t)c->feat_bytes));
   {
-    std::vector<float> stage((size_t)std::max<int64_t>(1, nh) * c->feat_stride, 0.0f);
+    std::vector<char> stage((size_t)c->feat_bytes, 0);
     for (int64_t v = 0; v < n; ++v)
-      if (fpos[(size_t)v] >= 0) memcpy(&stage[(size_t)fpos[(size_t)v] * c->feat_stride], hsrc + (size_t)v * dim, row_bytes);
-    CUDA_TRY(c, cudaMemcpy(c->d_feat, stage.data(), stride_bytes * (size_t)nh, cudaMemcpyHostToDevice));
+      if (fpos[(size_t)v] >= 0) put_row(stage.data(), nh, fpos[(size_t)v], hsrc + (size_t)v * dim);
+    CUDA_TRY(c, cudaMemcpy(c->d_feat, stage.data(), (size_t)c->feat_bytes, cudaMemcpyHostToDevice));
   }
-  c->cold_bytes = (int64_t)stride_bytes * std::max<int64_t>(1, nc);
+  c->cold_bytes = (int64_t)region_bytes(c->split_rows, nc, dim);
   if (c->world > 1) {  // cross-process readable: POSIX shm registered with CUDA
     static int counter = 0;
     snprintf(c->cold_shm, sizeof(c->cold_shm), "/dsp_cold_%d_%d_%d", (int)getpid(), c->rank, counter++);
@@ -1404,7 +1472,7 @@ dsp_status dsp_load_features_tiered(dsp_ctx *c, const float *features, int32_t d
   }
   for (int64_t v = 0; v < n; ++v)
     if (fpos[(size_t)v] < 0)
-      memcpy(c->h_cold + (size_t)(-fpos[(size_t)v] - 1) * c->feat_stride, hsrc + (size_t)v * dim, row_bytes);
+      put_row(reinterpret_cast<char *>(c->h_cold), nc, -fpos[(size_t)v] - 1, hsrc + (size_t)v * dim);
   CUDA_TRY(c, cudaMalloc(&c->d_fpos, sizeof(int32_t) * (size_t)std::max<int64_t>(1, n)));
   if (n > 0) CUDA_TRY(c, cudaMemcpy(c->d_fpos, fpos.data(), sizeof(int32_t) * (size_t)n, cudaMemcpyHostToDevice));
   void *dev_cold = nullptr;
@@ -1412,8 +1480,10 @@ dsp_status dsp_load_features_tiered(dsp_ctx *c, const float *features, int32_t d
   c->tiered = true;
   c->cold_regloads = c->gather_reg;
   c->peer_feat[c->rank] = c->d_feat;
+  c->peer_feat_tail[c->rank] = reinterpret_cast<const float *>(reinterpret_cast<const char *>(c->d_feat) + tail_offset(c->split_rows, nh, dim));
   c->peer_fpos[c->rank] = nc > 0 ? c->d_fpos : nullptr;  // all hot: fpos is the identity
   c->peer_cold[c->rank] = static_cast<const float *>(dev_cold);
+  c->peer_cold_tail[c->rank] = reinterpret_cast<const float *>(static_cast<const char *>(dev_cold) + tail_offset(c->split_rows, nc, dim));
   return DSP_OK;
 }
 
@@ -1448,7 +1518,9 @@ dsp_status dsp_load_weights(dsp_ctx *c, const float *edge_weights) {
     if (bad) {
       cudaFree(c->d_weights);
       c->d_weights = nullptr;
-      return fail(c, DSP_ERR_INVALID_ARG, "%d edge weights outside [0, 65536)", bad);
+      return fail(c, DSP_ERR_INVALID_ARG,
+                  "%d edge weights are neither 0 nor in [2^-16, 65536) (negative, NaN, too large, or a positive "
+                  "weight that would quantize to 0 in 16.16 fixed point)", bad);
     }
   }
   return DSP_OK;
@@ -1476,8 +1548,11 @@ dsp_status dsp_reserve(dsp_ctx *c, int32_t max_seeds, const int32_t *fanouts, in
   if (c->world > 1) {
     DeviceGuard g(c->device);
     c->xl = make_xch_layout(std::max<int64_t>(1, p.max_F), c->kmax);
-    CUDA_TRY(c, cudaMalloc(&c->d_xch, c->xl.bytes));
-    CUDA_TRY(c, cudaMemset(c->d_xch, 0, c->xl.bytes));
+    c->chan_stride = align_up(c->xl.bytes, 256);
+    CUDA_TRY(c, cudaMalloc(&c->d_xch, c->chan_stride * (size_t)c->channels));
+    CUDA_TRY(c, cudaMemset(c->d_xch, 0, c->chan_stride * (size_t)c->channels));
+    for (int ch = 0; ch < c->channels && c->channels > 1; ++ch)
+      CUDA_TRY(c, cudaEventCreateWithFlags(&c->chan_ev[ch], cudaEventDisableTiming));
     CUDA_TRY(c, cudaDeviceSynchronize());
   }
   c->peer_xch[c->rank] = c->d_xch;
@@ -1549,9 +1624,12 @@ dsp_status dsp_export_handle(const dsp_ctx *cc, void *out) {
   h.feat_ptr = (uint64_t)(uintptr_t)c->d_feat;
   h.xch_ptr = (uint64_t)(uintptr_t)c->d_xch;
   h.feat_bytes = c->feat_bytes;
-  h.xch_bytes = (int64_t)c->xl.bytes;
+  h.xch_bytes = (int64_t)(c->chan_stride * (size_t)c->channels);
+  h.channels = c->channels;
   h.dim = c->dim;
-  h.feat_stride = c->feat_stride;
+  h.head_bytes = head_bytes_of(c->split_rows, c->dim);
+  h.feat_slots = c->feat_slots;
+  h.cold_slots = c->cold_slots;
   h.max_seeds = c->max_seeds;
   for (int r = 0; r <= c->world; ++r) h.bounds[r] = c->bounds[r];
   DeviceGuard g(c->device);
@@ -1610,8 +1688,10 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
       return fail(c, DSP_ERR_INVALID_ARG, "handle %d is not rank %d of this world", r, r);
     for (int q = 0; q <= c->world; ++q)
       if (h.bounds[q] != c->bounds[q]) return fail(c, DSP_ERR_STATE, "rank %d has different bounds", r);
-    if (h.dim != c->dim || h.feat_stride != c->feat_stride || h.max_seeds != c->max_seeds)
+    if (h.dim != c->dim || h.head_bytes != head_bytes_of(c->split_rows, c->dim) || h.max_seeds != c->max_seeds)
       return fail(c, DSP_ERR_STATE, "rank %d has a different dim / max_seeds", r);
+    if (h.has_xch && h.channels != c->channels)
+      return fail(c, DSP_ERR_STATE, "rank %d reserved %d exchange channels, this rank %d", r, h.channels, c->channels);
     if ((h.tiered != 0) != c->tiered) return fail(c, DSP_ERR_STATE, "all ranks must use the cold tier or none");
     if (h.lw_max_seeds != (c->lw_reserved ? c->lw_max_seeds : -1) || h.lw_L != c->lw_L ||
         memcmp(h.lw_sizes, c->lw_sizes, sizeof(c->lw_sizes)) != 0)
@@ -1714,6 +1794,13 @@ dsp_status dsp_import_handles(dsp_ctx *c, const void *all) {
         c->peer_xch[r] = static_cast<char *>(p);
       }
     }
+    // the tail arrays of rank r's split feature regions (dsp_kernels.cuh GatherArgs)
+    if (c->peer_feat[r])
+      c->peer_feat_tail[r] = reinterpret_cast<const float *>(reinterpret_cast<const char *>(c->peer_feat[r]) +
+                                                             tail_offset(c->split_rows, h.feat_slots, c->dim));
+    if (c->peer_cold[r])
+      c->peer_cold_tail[r] = reinterpret_cast<const float *>(reinterpret_cast<const char *>(c->peer_cold[r]) +
+                                                             tail_offset(c->split_rows, h.cold_slots, c->dim));
   }
   c->imported = true;
   return DSP_OK;
@@ -1811,6 +1898,17 @@ dsp_status dsp_set_option(dsp_ctx *c, int32_t option, int64_t value) {
       if (value != 0 && value != 1) return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_GATHER_REGLOADS must be 0 or 1");
       c->gather_reg = value != 0 || c->tma_unavailable;
       c->cold_regloads = c->gather_reg;
+      return DSP_OK;
+    case DSP_OPT_SPLIT_ROWS:
+      if (value != 0 && value != 1) return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_SPLIT_ROWS must be 0 or 1");
+      if (c->loaded) return fail(c, DSP_ERR_STATE, "DSP_OPT_SPLIT_ROWS must be set before dsp_load_partition");
+      c->split_rows = value != 0;
+      return DSP_OK;
+    case DSP_OPT_EXCHANGE_CHANNELS:
+      if (value < 1 || value > DSP_MAX_CHANNELS)
+        return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_EXCHANGE_CHANNELS %lld not in [1, %d]", (long long)value, DSP_MAX_CHANNELS);
+      if (c->reserved) return fail(c, DSP_ERR_STATE, "DSP_OPT_EXCHANGE_CHANNELS must be set before dsp_reserve");
+      c->channels = (int)value;
       return DSP_OK;
     default:
       return fail(c, DSP_ERR_INVALID_ARG, "unknown option %d", option);

@@ -47,6 +47,9 @@ DSP_OPT_LANE_ROUNDS = 2
 DSP_OPT_LOADER_WARPS = 3
 DSP_OPT_LOADER_ROWS = 4
 DSP_OPT_GATHER_REGLOADS = 5
+DSP_OPT_EXCHANGE_CHANNELS = 6
+DSP_OPT_SPLIT_ROWS = 7
+DSP_MAX_CHANNELS = 8
 #: DSP_OPT_RELABEL_MAP values
 RELABEL_MAPS = {"auto": 0, "direct": 1, "hash": 2, "direct64": 3}
 

@@ -40,7 +40,7 @@ def _check_pipelined(s, ip, ix, cfg, seeds, rng, slot, sizes):
         raise AssertionError(f"pipelined step rng {rng:#x}: features")
 
 
-def _rank(rank, world, port, q, hot=None, scheme="node"):
+def _rank(rank, world, port, q, hot=None, scheme="node", channels=1):
     import sys
     here = os.path.dirname(os.path.abspath(__file__))
     sys.path[:0] = [os.path.dirname(here), here]
@@ -61,9 +61,10 @@ def _rank(rank, world, port, q, hot=None, scheme="node"):
         feats = datagen.features(lo, hi, cfg.dim)
         sizes = (300, 600) if scheme == "layer" else cfg.fanouts
         s = pkg.Sampler(bnds, sip, six, feats, sizes, 32, rank=rank, world_size=world, device=0,
-                        exchange=pkg.torch_exchange(), n_slots=2,
+                        exchange=pkg.torch_exchange(), n_slots=2 if channels == 1 else 8,
                         hot_rows=None if hot is None else (hi - lo) * hot // 4, scheme=scheme,
-                        max_walks=500, max_walk_length=16)
+                        max_walks=500, max_walk_length=16, n_workspaces=channels,
+                        options={pkg.dsp.DSP_OPT_EXCHANGE_CHANNELS: channels})
         train = datagen.train_ids(cfg.num_nodes, cfg.train_count)
         batches = datagen.rank_seed_batches(train, bnds, rank, 32, 0)
         for step in range(3):
@@ -78,6 +79,26 @@ def _rank(rank, world, port, q, hot=None, scheme="node"):
             exp = datagen.features_of(ref[-1]["src_ids"], cfg.dim)
             if not np.array_equal(feat.cpu().numpy().view(np.uint32), exp.view(np.uint32)):
                 ok, detail = False, f"step {step} features"
+        if channels > 1:
+            # several collective calls in flight per rank: step j on stream j % C with
+            # workspace j % C (exchange channel j % C), each launch on 1/C of the SMs;
+            # pipelined, so step j's features are written by step j + C (or the flush)
+            C = channels
+            pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(0).multi_processor_count // C)
+            streams = [torch.cuda.Stream() for _ in range(C)]
+            n = 8
+            sz = torch.zeros((n, 3 * len(cfg.fanouts)), dtype=torch.int64).pin_memory()
+            dev_seeds = [torch.from_numpy(batches[step]).cuda() for step in range(n)]
+            for st in streams:   # the seeds' copies were issued on the current stream
+                st.wait_stream(torch.cuda.current_stream())
+            for step in range(n):
+                s.sample_gather(dev_seeds[step], 0xD00 + step, slot=step, sizes_out=sz[step],
+                                pipelined=True, ws=step % C, stream=streams[step % C])
+            s.flush()
+            torch.cuda.synchronize()
+            for step in range(n):
+                _check_pipelined(s, ip, ix, cfg, batches[step], 0xD00 + step, step, sz[step])
+            pkg.dsp_set_persistent_blocks(s.ctx, 0)
         if scheme == "node":
             # pipelined steps: the launch of step t samples batch t while its
             # loader warps gather batch t-1 from both processes' shards; flush() the last
@@ -107,17 +128,21 @@ def _rank(rank, world, port, q, hot=None, scheme="node"):
         dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("hot,scheme", [(None, "node"), (1, "node"), (None, "layer")])
-def test_two_processes_one_gpu(hot, scheme):
+@pytest.mark.parametrize("hot,scheme,channels", [(None, "node", 1), (1, "node", 1), (None, "layer", 1),
+                                                 (None, "node", 2)])
+def test_two_processes_one_gpu(hot, scheme, channels):
     """hot = 1: the cold-feature tier with 3/4 of each shard in host memory
-    (POSIX shm mapped into the peer process), read over UVA by both GPUs' gathers."""
+    (POSIX shm mapped into the peer process), read over UVA by both GPUs' gathers.
+    channels = 2: two collective calls in flight per rank on two streams
+    (DSP_OPT_EXCHANGE_CHANNELS), then the synchronous and pipelined steps on a
+    single stream keep rotating through the channels."""
     if not torch.cuda.is_available():
         pytest.fail("needs a GPU")
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_rank, args=(r, 2, port, q, hot, scheme)) for r in range(2)]
+    procs = [ctx.Process(target=_rank, args=(r, 2, port, q, hot, scheme, channels)) for r in range(2)]
     for p in procs:
         p.start()
     res = sorted(q.get(timeout=600) for _ in procs)

@@ -225,6 +225,36 @@ def test_tiny_virtual_ranks(pkg, tiny, P, mode):
     grp.close()
 
 
+@pytest.mark.parametrize("P", [2, 4])
+def test_virtual_ranks_exchange_channels(pkg, tiny, P):
+    """DSP_OPT_EXCHANGE_CHANNELS = 3: consecutive collective calls rotate over
+    three exchange regions with their own sequence numbers (a duplicate-seed
+    error in between must not desynchronise the rotation); every call equals
+    the oracle."""
+    cfg, ip, ix, feats = tiny
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi]))
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P,
+                         options={pkg.dsp.DSP_OPT_EXCHANGE_CHANNELS: 3})
+    per_rank = [seeds_of(cfg, P, r, batch=32) for r in range(P)]
+    for step in range(8):
+        seeds = [per_rank[r][step] for r in range(P)]
+        if step == 4:
+            bad = [np.ascontiguousarray(x) for x in seeds]
+            bad[0] = np.concatenate([bad[0][:3], bad[0][:1]])
+            with pytest.raises(pkg.DSPError) as e:
+                grp.sample([torch.from_numpy(x).cuda() for x in bad], 9)
+            assert e.value.status == pkg.dsp.DSP_ERR_DUPLICATE_SEED
+        res = grp.sample([torch.from_numpy(np.ascontiguousarray(x)).cuda() for x in seeds], 0x600 + step)
+        for r in range(P):
+            assert_blocks_equal(res[r], oracle.sample(ip, ix, seeds[r], cfg.fanouts, 0x600 + step), f"P={P} r{r} {step}")
+    grp.close()
+
+
 @pytest.mark.parametrize("mode", ["direct", "hash"])
 def test_virtual_ranks_errors(pkg, tiny, mode):
     """Device-detected errors at world > 1 (duplicate seed, out-of-range seed)
@@ -577,11 +607,17 @@ def test_biased_errors(pkg, tiny):
         s.sample(torch.arange(4, dtype=torch.int32, device="cuda"), 1, biased=True)
     assert e.value.status == pkg.dsp.DSP_ERR_STATE
     s.close()
-    bad = np.ones(len(ix), np.float32)
-    bad[7] = -1.0
-    with pytest.raises(pkg.DSPError) as e:
-        pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8, edge_weights=bad)
-    assert e.value.status == pkg.dsp.DSP_ERR_INVALID_ARG
+    # negative, >= 2^16, NaN, and positive weights below 2^-16 (they would quantize
+    # to 0 in 16.16 fixed point and never be sampled, R24) are rejected
+    for x in (-1.0, 65536.0, float("nan"), 2.0 ** -17, 1e-30):
+        bad = np.ones(len(ix), np.float32)
+        bad[7] = x
+        with pytest.raises(pkg.DSPError) as e:
+            pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8, edge_weights=bad)
+        assert e.value.status == pkg.dsp.DSP_ERR_INVALID_ARG, x
+    ok = np.ones(len(ix), np.float32)
+    ok[7], ok[8] = 0.0, 2.0 ** -16          # zero and the smallest positive fixed-point weight are accepted
+    pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8, edge_weights=ok).close()
 
 
 # ------------------------------------------------------ random walks

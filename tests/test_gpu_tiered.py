@@ -114,3 +114,53 @@ def test_tiered_errors(pkg, tiny):
         pkg.dsp_load_features_tiered(s.ctx, feats, cfg.dim, 10)
     assert e.value.status == pkg.dsp.DSP_ERR_STATE
     s.close()
+
+
+@pytest.mark.parametrize("dim", [100, 36, 128, 8])
+@pytest.mark.parametrize("P,hot", [(1, None), (1, 3), (2, None), (2, 2)])
+def test_split_rows_layout(pkg, tiny, dim, P, hot):
+    """DSP_OPT_SPLIT_ROWS = 1: rows stored as a 128-byte-line head plus a tail
+    (dim 100: 384 + 16 B, 36: 128 + 16, 128: head only, 8: tail only), in the
+    HBM shard, in the cold region and across virtual ranks; every gather path
+    (standalone, fused, pipelined loader warps) returns the rows bit-exactly."""
+    cfg, ip, ix, _ = tiny
+    feats = datagen.features(0, cfg.num_nodes, dim)
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    opts = {pkg.dsp.DSP_OPT_SPLIT_ROWS: 1}
+    ids = np.random.default_rng(dim + P).permutation(cfg.num_nodes).astype(np.int32)
+    if P == 1:
+        s = pkg.Sampler(bnds, ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2, options=opts,
+                        hot_rows=None if hot is None else cfg.num_nodes * hot // 4)
+        out = s.gather(torch.from_numpy(ids).cuda())
+        s.sync()
+        assert np.array_equal(_bits(out.cpu().numpy()), _bits(oracle.gather(feats, ids)))
+        batches = _seeds(cfg, 1, 0, cfg.batch)
+        blocks, feat = s.sample_gather(torch.from_numpy(batches[0]).cuda(), 21, slot=0)
+        ref = oracle.sample(ip, ix, batches[0], cfg.fanouts, 21)
+        assert np.array_equal(_bits(feat.cpu().numpy()), _bits(oracle.gather(feats, ref[-1]["src_ids"])))
+        L = len(cfg.fanouts)
+        sizes = torch.zeros((3, 3 * L), dtype=torch.int64).pin_memory()
+        for j in range(3):
+            s.sample_gather(torch.from_numpy(batches[1 + j]).cuda(), 30 + j, slot=j % 2, sizes_out=sizes[j],
+                            pipelined=True)
+            if j >= 1:
+                torch.cuda.synchronize()
+                ref = oracle.sample(ip, ix, batches[j], cfg.fanouts, 30 + j - 1)
+                got = s.feat_buffer((j - 1) % 2)[: int(sizes[j - 1][3 * (L - 1) + 1])]
+                assert np.array_equal(_bits(got.cpu().numpy()), _bits(oracle.gather(feats, ref[-1]["src_ids"])))
+        s.flush()
+        s.sync()
+        s.close()
+        return
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi]))
+    hr = None if hot is None else [(int(bnds[r + 1]) - int(bnds[r])) * hot // 4 for r in range(P)]
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P, hot_rows=hr, options=opts)
+    for r in range(P):
+        out = grp.samplers[r].gather(torch.from_numpy(ids).cuda())
+        grp.samplers[r].sync()
+        assert np.array_equal(_bits(out.cpu().numpy()), _bits(oracle.gather(feats, ids)))
+    grp.close()
