@@ -233,7 +233,12 @@ dsp_status dsp_sample(dsp_ctx *ctx, const int32_t *seeds, int32_t num_seeds, con
    (the exchanges through peer memory inside it); ranks sharing a device each
    get 1/n of its SMs on the ctx's own stream, forked from and joined to the
    given stream after all ranks were launched (layer-wise calls likewise).
-   Virtual ranks sharing a device must pass the same stream. */
+   Virtual ranks sharing a device must pass the same stream.  flags: 0,
+   DSP_BIASED or DSP_LAYERWISE, plus DSP_ASYNC: return once every rank's call
+   is enqueued (blocks[.][l].num_* not filled, device errors latch until
+   dsp_sync); with DSP_OPT_EXCHANGE_CHANNELS = C and 1/(ranks per GPU * C)
+   of the SMs per launch (dsp_set_persistent_blocks), C asynchronous group
+   calls on C streams run concurrently. */
 dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *seeds,
                             const int32_t *num_seeds, const int32_t *fanouts, int32_t num_layers,
                             uint64_t rng_seed, dsp_block *const *blocks, void *const *workspaces,

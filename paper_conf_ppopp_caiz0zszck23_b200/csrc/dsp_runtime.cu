@@ -209,8 +209,10 @@ struct dsp_ctx {
   bool tma_unavailable = false;  // the TMA gather's shared memory could not be configured
   WsHeader *d_walk_hdr = nullptr;  // grid-barrier counter of k_walk_multi
   int walk_blocks_per_sm = 2;
-  cudaStream_t aux = nullptr;  // virtual ranks sharing a GPU: each rank's persistent launch on its own stream
-  cudaEvent_t aux_ev[2] = {nullptr, nullptr};
+  // virtual ranks sharing a GPU: each rank's persistent launch on its own
+  // stream, one per exchange channel (concurrent group calls)
+  cudaStream_t aux[DSP_MAX_CHANNELS] = {nullptr};
+  cudaEvent_t aux_ev[DSP_MAX_CHANNELS][2] = {{nullptr}};
   cudaEvent_t flush_ev = nullptr;  // dsp_pipeline_flush: orders a pending gather after its call's stream
   int gather_blocks_per_sm = 1;
   // pipelined steps: per workspace, the gather owed by its previous
@@ -740,6 +742,26 @@ dsp_status stage_persistent(Call &k) {
 
 XchPeers peers_of(const dsp_ctx *c, int channel);
 
+// Virtual ranks sharing a GPU: fork the caller's stream onto the ctx's own
+// stream of channel ch (created on first use), so that every rank of a group
+// call is launched before any is joined (all of them resident at once).
+dsp_status fork_aux(dsp_ctx *c, int ch, cudaStream_t from, cudaStream_t *out) {
+  if (!c->aux[ch]) {
+    CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux[ch], cudaStreamNonBlocking));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[ch][0], cudaEventDisableTiming));
+    CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[ch][1], cudaEventDisableTiming));
+  }
+  CUDA_TRY(c, cudaEventRecord(c->aux_ev[ch][0], from));
+  CUDA_TRY(c, cudaStreamWaitEvent(c->aux[ch], c->aux_ev[ch][0], 0));
+  *out = c->aux[ch];
+  return DSP_OK;
+}
+dsp_status join_aux(dsp_ctx *c, int ch, cudaStream_t to) {
+  CUDA_TRY(c, cudaEventRecord(c->aux_ev[ch][1], c->aux[ch]));
+  CUDA_TRY(c, cudaStreamWaitEvent(to, c->aux_ev[ch][1], 0));
+  return DSP_OK;
+}
+
 // world > 1, node-wise: the whole call in one cooperative kernel per rank
 // (dsp_multi.cuh).  `share` = ranks of this call group on the same GPU
 // (virtual ranks): each launch gets 1/share of the SMs, on the ctx's own
@@ -787,14 +809,8 @@ dsp_status stage_persistent_multi(Call &k, int share) {
   const dim3 grid(blocks), block(PNT);
   cudaStream_t st = k.stream;
   if (share > 1) {  // fork onto the ctx's own stream
-    if (!c->aux) {
-      CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking));
-      CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[0], cudaEventDisableTiming));
-      CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[1], cudaEventDisableTiming));
-    }
-    CUDA_TRY(c, cudaEventRecord(c->aux_ev[0], k.stream));
-    CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->aux_ev[0], 0));
-    st = c->aux;
+    dsp_status fs = fork_aux(c, k.channel, k.stream, &st);
+    if (fs != DSP_OK) return fs;
   }
   void *args[] = {&m};
   cudaEvent_t &cev = c->chan_ev[k.channel];
@@ -833,9 +849,7 @@ dsp_status join_persistent_multi(Call &k, int share) {
   dsp_ctx *c = k.c;
   if (share <= 1) return DSP_OK;
   DeviceGuard g(c->device);
-  CUDA_TRY(c, cudaEventRecord(c->aux_ev[1], c->aux));
-  CUDA_TRY(c, cudaStreamWaitEvent(k.stream, c->aux_ev[1], 0));
-  return DSP_OK;
+  return join_aux(c, k.layerwise ? 0 : k.channel, k.stream);
 }
 
 // A standalone gather: TMA loader warps (k_gather_tma) by default, 16-byte
@@ -977,14 +991,8 @@ dsp_status stage_lw_persistent(Call &k, int share = 1) {
   const dim3 grid(blocks), block(LWT);
   cudaStream_t st = k.stream;
   if (share > 1) {  // fork onto the ctx's own stream (joined by join_persistent_multi)
-    if (!c->aux) {
-      CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking));
-      CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[0], cudaEventDisableTiming));
-      CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[1], cudaEventDisableTiming));
-    }
-    CUDA_TRY(c, cudaEventRecord(c->aux_ev[0], k.stream));
-    CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->aux_ev[0], 0));
-    st = c->aux;
+    dsp_status fs = fork_aux(c, 0, k.stream, &st);
+    if (fs != DSP_OK) return fs;
   }
   void *args[] = {&p};
   CUDA_TRY(c, cudaLaunchCooperativeKernel(c->world > 1 ? (const void *)k_lw_multi : (const void *)k_lw_persistent,
@@ -1111,13 +1119,14 @@ void release(dsp_ctx *c) {
   cudaFree(c->d_feat);
   cudaFree(c->d_xch);
   cudaFree(c->d_walk_hdr);
-  if (c->aux) {
-    cudaStreamSynchronize(c->aux);
-    cudaStreamDestroy(c->aux);
-    cudaEventDestroy(c->aux_ev[0]);
-    cudaEventDestroy(c->aux_ev[1]);
-    c->aux = nullptr;
-  }
+  for (int ch = 0; ch < DSP_MAX_CHANNELS; ++ch)
+    if (c->aux[ch]) {
+      cudaStreamSynchronize(c->aux[ch]);
+      cudaStreamDestroy(c->aux[ch]);
+      cudaEventDestroy(c->aux_ev[ch][0]);
+      cudaEventDestroy(c->aux_ev[ch][1]);
+      c->aux[ch] = nullptr;
+    }
   if (c->flush_ev) {
     cudaEventDestroy(c->flush_ev);
     c->flush_ev = nullptr;
@@ -1188,14 +1197,8 @@ dsp_status run_walks(std::vector<dsp_ctx *> &cs, std::vector<WalkArgs> &as, std:
     CUDA_TRY(c, cudaMemsetAsync(c->d_walk_hdr, 0, sizeof(WsHeader), ss[i]));
     cudaStream_t st_i = ss[i];
     if (share[i] > 1) {  // virtual ranks: each on its own stream with 1/share of the SMs
-      if (!c->aux) {
-        CUDA_TRY(c, cudaStreamCreateWithFlags(&c->aux, cudaStreamNonBlocking));
-        CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[0], cudaEventDisableTiming));
-        CUDA_TRY(c, cudaEventCreateWithFlags(&c->aux_ev[1], cudaEventDisableTiming));
-      }
-      CUDA_TRY(c, cudaEventRecord(c->aux_ev[0], ss[i]));
-      CUDA_TRY(c, cudaStreamWaitEvent(c->aux, c->aux_ev[0], 0));
-      st_i = c->aux;
+      dsp_status fs = fork_aux(c, 0, ss[i], &st_i);
+      if (fs != DSP_OK) return fs;
     }
     WalkPersistArgs p{};
     p.a = as[i];
@@ -1209,8 +1212,8 @@ dsp_status run_walks(std::vector<dsp_ctx *> &cs, std::vector<WalkArgs> &as, std:
     if (share[i] > 1) {
       dsp_ctx *c = cs[i];
       DeviceGuard g(c->device);
-      CUDA_TRY(c, cudaEventRecord(c->aux_ev[1], c->aux));
-      CUDA_TRY(c, cudaStreamWaitEvent(ss[i], c->aux_ev[1], 0));
+      dsp_status js = join_aux(c, 0, ss[i]);
+      if (js != DSP_OK) return js;
     }
   for (auto *c : cs) c->wseq = seq0 + 1 + (unsigned long long)length;
   return DSP_OK;
@@ -1945,11 +1948,12 @@ dsp_status dsp_sample_group(dsp_ctx *const *ctxs, int32_t n, const int32_t *cons
   }
   std::vector<Call> calls(n);
   for (int i = 0; i < n; ++i) {
-    if ((flags & (DSP_ASYNC | DSP_PIPELINED)) != 0)
-      return fail(ctxs[0], DSP_ERR_INVALID_ARG, "dsp_sample_group takes DSP_BIASED only");
+    if ((flags & DSP_PIPELINED) != 0)
+      return fail(ctxs[0], DSP_ERR_INVALID_ARG, "dsp_sample_group takes DSP_BIASED, DSP_LAYERWISE, DSP_ASYNC");
     dsp_status st = prepare_call(calls[i], ctxs[i], seeds[i], num_seeds[i], fanouts, L, rng_seed,
-                                 blocks[i], workspaces[i], workspace_bytes, flags, streams[i]);
+                                 blocks[i], workspaces[i], workspace_bytes, flags & ~DSP_ASYNC, streams[i]);
     if (st != DSP_OK) return st;
+    calls[i].async = (flags & DSP_ASYNC) != 0;
   }
   return run_calls(calls);
 }

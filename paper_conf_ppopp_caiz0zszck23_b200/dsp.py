@@ -493,7 +493,7 @@ class LocalGroup:
 
     def __init__(self, bounds, shards, fanouts, max_seeds: int, devices: Sequence[int], hot_rows=None,
                  scheme: str = "node", max_walks: int | None = None, max_walk_length: int = 1024,
-                 options: dict | None = None):
+                 options: dict | None = None, n_workspaces: int = 1, n_slots: int = 1):
         """shards[r] = (indptr, indices, features[, edge_weights]) of rank r;
         hot_rows[r] (optional) enables the cold-feature tier; options as Sampler."""
         P = len(shards)
@@ -501,7 +501,8 @@ class LocalGroup:
         self.samplers = [Sampler(bounds, s[0], s[1], s[2], fanouts, max_seeds, rank=r, world_size=P,
                                  device=devices[r], connect=False, edge_weights=s[3] if len(s) > 3 else None,
                                  hot_rows=None if hot_rows is None else hot_rows[r], scheme=scheme,
-                                 max_walks=max_walks, max_walk_length=max_walk_length, options=options)
+                                 max_walks=max_walks, max_walk_length=max_walk_length, options=options,
+                                 n_workspaces=n_workspaces, n_slots=n_slots)
                          for r, s in enumerate(shards)]
         handles = [dsp_export_handle(s.ctx) for s in self.samplers]
         for s in self.samplers:
@@ -510,13 +511,18 @@ class LocalGroup:
             s.connected = True
         self.fanouts = list(fanouts)
 
-    def sample(self, seeds_per_rank, rng_seed: int, biased: bool = False) -> list[list[Block]]:
+    def sample(self, seeds_per_rank, rng_seed: int, biased: bool = False, async_: bool = False, ws: int = 0,
+               slot: int = 0, stream=None) -> list[list[Block]] | None:
+        """One group call (every rank).  async_: enqueue only (DSP_ASYNC) on
+        `stream`, with workspace `ws` and output set `slot` of every rank;
+        returns None (sizes via a later synchronous call or the blocks' data)."""
         S = self.samplers
+        st = [s.stream() for s in S] if stream is None else [stream.cuda_stream] * len(S)
         dsp_sample_group([s.ctx for s in S], seeds_per_rank, [x.numel() for x in seeds_per_rank],
-                         self.fanouts, rng_seed, [s._cblocks for s in S], [s.workspace for s in S],
-                         S[0].workspace_bytes, (DSP_BIASED if biased else 0) | S[0]._sflag,
-                         [s.stream() for s in S])
-        return [s.blocks() for s in S]
+                         self.fanouts, rng_seed, [s._sets[slot][1] for s in S], [s.workspaces[ws] for s in S],
+                         S[0].workspace_bytes, (DSP_BIASED if biased else 0) | S[0]._sflag
+                         | (DSP_ASYNC if async_ else 0), st)
+        return None if async_ else [s.blocks(slot) for s in S]
 
     def random_walk(self, starts_per_rank, length: int, rng_seed: int):
         """Walk traces of every rank, CSP push without reshuffle."""
