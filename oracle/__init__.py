@@ -104,6 +104,8 @@ def lib():
         L.oracle_sample_layerwise.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int32, P, ctypes.c_int32,
                                               ctypes.c_uint64, ctypes.POINTER(_Block)]
         L.oracle_random_walk.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64, ctypes.c_int32, ctypes.c_uint64, P]
+        L.oracle_random_walk_independent.argtypes = [ctypes.c_int64, P, P, P, ctypes.c_int64, ctypes.c_int32,
+                                                     ctypes.c_uint64, P]
         _lib = L
     return _lib
 
@@ -272,13 +274,15 @@ def sample_layerwise(indptr, indices, seeds, sizes, rng_seed: int) -> list[dict]
     return out
 
 
-def random_walk(indptr, indices, starts, length: int, rng_seed: int) -> np.ndarray:
-    """Walk traces int32[n][length + 1] (-1 after a dead end)."""
+def random_walk(indptr, indices, starts, length: int, rng_seed: int, independent: bool = False) -> np.ndarray:
+    """Walk traces int32[n][length + 1] (-1 after a dead end).
+    independent: each walk draws with its own index (R35)."""
     ip = _c(indptr, np.int64)
     ix = _c(indices, np.int32)
     st = _c(starts, np.int32)
     out = np.zeros((len(st), length + 1), np.int32)
-    rc = lib().oracle_random_walk(len(ip) - 1, _ptr(ip), _ptr(ix), _ptr(st), len(st), length, rng_seed, _ptr(out))
+    fn = lib().oracle_random_walk_independent if independent else lib().oracle_random_walk
+    rc = fn(len(ip) - 1, _ptr(ip), _ptr(ix), _ptr(st), len(st), length, rng_seed, _ptr(out))
     if rc != OK:
         raise OracleError(rc, "oracle_random_walk")
     return out
