@@ -369,7 +369,11 @@ dsp_status dsp_gather_features(dsp_ctx *ctx, const int32_t *ids, int64_t n, floa
    walk and the remaining entries are -1.  NOTE: the draw is keyed by (node,
    step), not by the walk, so walks with the same start node in one call are
    IDENTICAL; for several independent walks per start node (DeepWalk-style)
-   pass them in calls with different rng_seed values.
+   pass flags = DSP_WALK_INDEPENDENT: then step l of walk i draws from
+   Philox counter {i, v, l, "DSPW"} (i = the walk's index in `starts`;
+   DESIGN.md R35), so walks with the same start are independent.  flags: 0
+   or DSP_WALK_INDEPENDENT (else DSP_ERR_INVALID_ARG); at world_size > 1
+   all ranks pass the same flags (checked in the exchange header).
    starts: DEVICE int32[n] in [0, N) (any owner; else an error latches for
    dsp_sync and the walk is all -1); traces: DEVICE int32[n][length + 1],
    traces[i][0] = starts[i]; 1 <= length <= 1024.  Asynchronous on `stream`.
@@ -380,8 +384,9 @@ dsp_status dsp_gather_features(dsp_ctx *ctx, const int32_t *ids, int64_t n, floa
    round: counts + header + flag), the owner takes the step and
    stores the new node straight into the trace row at the walk's origin rank
    over NVLink.  Traces are bit-identical for any world_size / bounds. */
+#define DSP_WALK_INDEPENDENT 16u
 dsp_status dsp_random_walk(dsp_ctx *ctx, const int32_t *starts, int64_t n, int32_t length, uint64_t rng_seed,
-                           int32_t *traces, void *stream);
+                           int32_t *traces, uint32_t flags, void *stream);
 
 /* Sizes the peer-visible walk region for up to max_walks walks per rank
    (<= 2^27) of up to max_length steps (<= 1024): inboxes of
@@ -396,7 +401,7 @@ dsp_status dsp_reserve_walks(dsp_ctx *ctx, int64_t max_walks, int32_t max_length
    rank by rank.  Arrays are indexed by position in ctxs. */
 dsp_status dsp_random_walk_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *starts,
                                  const int64_t *n, int32_t length, uint64_t rng_seed, int32_t *const *traces,
-                                 void *const *streams);
+                                 uint32_t flags, void *const *streams);
 
 /* Synchronises `stream` and reports a latched device error (then clears it). */
 dsp_status dsp_sync(dsp_ctx *ctx, void *stream);

@@ -44,6 +44,13 @@ __device__ __forceinline__ uint32_t draw_range(uint2 key, uint32_t slot, int32_t
   return (uint32_t)__umul64hi(w, (unsigned long long)m);
 }
 
+// independent random walks (R35): walk i's draw at step l from v
+__device__ __forceinline__ uint32_t walk_draw(uint2 key, uint32_t walk, int32_t v, int32_t l, uint32_t m) {
+  const uint4 x = philox4x32_10(make_uint4(walk, (uint32_t)v, (uint32_t)l, 0x44535057u), key);
+  const unsigned long long w = ((unsigned long long)x.y << 32) | x.x;
+  return (uint32_t)__umul64hi(w, (unsigned long long)m);
+}
+
 // ------------------------------------------------------------ hash table
 // Open addressing, linear probing, one 64-bit word per slot:
 //   word = key << 32 | val,  EMPTY = all ones (keys are < 2^31).

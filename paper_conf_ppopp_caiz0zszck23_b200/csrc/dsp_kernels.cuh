@@ -1371,10 +1371,12 @@ __global__ void k_weights_fixed(const float *w, int64_t n, uint32_t *out, int *b
 // sample of v at layer l (no draw when deg <= 1); a node without neighbours
 // ends the walk (-1 for the remaining steps).  One thread per walk; each step
 // is two dependent random loads (indptr pair, adjacency entry).
+// independent = 1 (DSP_WALK_INDEPENDENT, R35): the draw of walk i is keyed by
+// i instead of slot 0, so walks from the same start are independent.
 __global__ void __launch_bounds__(NT) k_random_walk(const int32_t *starts, int64_t n, int32_t length, uint2 key,
                                                     const int64_t *__restrict__ indptr,
                                                     const int32_t *__restrict__ indices, int64_t N,
-                                                    int32_t *traces, int *err) {
+                                                    int32_t *traces, int *err, int independent) {
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     int32_t v = __ldg(starts + i);
     int32_t *tr = traces + i * (int64_t)(length + 1);
@@ -1390,7 +1392,9 @@ __global__ void __launch_bounds__(NT) k_random_walk(const int32_t *starts, int64
         if (d == 0) {
           v = -1;
         } else {
-          const uint32_t pos = d == 1 ? 0u : draw_range(key, 0u, v, l, (uint32_t)d);
+          const uint32_t pos = d == 1        ? 0u
+                               : independent ? walk_draw(key, (uint32_t)i, v, l, (uint32_t)d)
+                                             : draw_range(key, 0u, v, l, (uint32_t)d);
           v = __ldg(indices + s + pos);
         }
       }

@@ -1147,7 +1147,7 @@ void release(dsp_ctx *c) {
 // Random walks over a partitioned graph: one stage of one rank.
 // stage 0 = init, 1 = shuffle of step l, 2 = step l at the owner, 3 = done, 4 = finish.
 WalkArgs walk_args(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length, uint64_t rng_seed,
-                   int32_t *traces) {
+                   int32_t *traces, uint32_t flags) {
   WalkArgs a{};
   a.starts = starts;
   a.n = n;
@@ -1163,6 +1163,7 @@ WalkArgs walk_args(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length,
   for (int r = 0; r < DSP_MAX_WORLD; ++r) a.peers.base[r] = r < c->world ? c->peer_wxch[r] : nullptr;
   a.traces = traces;
   a.err = c->d_err;
+  a.independent = (flags & DSP_WALK_INDEPENDENT) ? 1 : 0;
   return a;
 }
 
@@ -1974,15 +1975,16 @@ dsp_status dsp_gather_features(dsp_ctx *c, const int32_t *ids, int64_t n, float 
 }
 
 dsp_status dsp_random_walk(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t length, uint64_t rng_seed,
-                           int32_t *traces, void *stream) {
+                           int32_t *traces, uint32_t flags, void *stream) {
   if (!c) return DSP_ERR_INVALID_ARG;
   c->err.clear();
+  if ((flags & ~DSP_WALK_INDEPENDENT) != 0) return fail(c, DSP_ERR_INVALID_ARG, "unknown walk flags 0x%x", flags);
   if (!c->loaded) return fail(c, DSP_ERR_STATE, "dsp_load_partition first");
   dsp_status st = check_walk_call(c, starts, n, length, traces);
   if (st != DSP_OK) return st;
   if (c->world > 1) {  // COLLECTIVE: CSP push without reshuffle
     std::vector<dsp_ctx *> cs{c};
-    std::vector<WalkArgs> as{walk_args(c, starts, n, length, rng_seed, traces)};
+    std::vector<WalkArgs> as{walk_args(c, starts, n, length, rng_seed, traces, flags)};
     std::vector<cudaStream_t> ss{static_cast<cudaStream_t>(stream)};
     return run_walks(cs, as, ss, length);
   }
@@ -1990,15 +1992,17 @@ dsp_status dsp_random_walk(dsp_ctx *c, const int32_t *starts, int64_t n, int32_t
   DeviceGuard g(c->device);
   const int64_t want = (n + NT - 1) / NT;
   k_random_walk<<<(int)std::min<int64_t>(want, grid_for(c, 8)), NT, 0, static_cast<cudaStream_t>(stream)>>>(
-      starts, n, length, key_of(rng_seed), c->d_indptr, c->d_indices, c->N, traces, c->d_err);
+      starts, n, length, key_of(rng_seed), c->d_indptr, c->d_indices, c->N, traces, c->d_err,
+      (flags & DSP_WALK_INDEPENDENT) ? 1 : 0);
   CUDA_TRY(c, cudaGetLastError());
   return DSP_OK;
 }
 
 dsp_status dsp_random_walk_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int32_t *const *starts,
                                  const int64_t *n, int32_t length, uint64_t rng_seed, int32_t *const *traces,
-                                 void *const *streams) {
+                                 uint32_t flags, void *const *streams) {
   if (!ctxs || n_ctx < 1 || !starts || !n || !traces || !streams) return DSP_ERR_INVALID_ARG;
+  if ((flags & ~DSP_WALK_INDEPENDENT) != 0) return fail(ctxs[0], DSP_ERR_INVALID_ARG, "unknown walk flags 0x%x", flags);
   const int world = ctxs[0] ? ctxs[0]->world : 0;
   if (n_ctx != world) return fail(ctxs[0], DSP_ERR_INVALID_ARG, "dsp_random_walk_group needs all %d ranks", world);
   std::vector<int> seen(world, 0);
@@ -2016,10 +2020,10 @@ dsp_status dsp_random_walk_group(dsp_ctx *const *ctxs, int32_t n_ctx, const int3
     dsp_status st = check_walk_call(ctxs[i], starts[i], n[i], length, traces[i]);
     if (st != DSP_OK) return st;
     cs[i] = ctxs[i];
-    as[i] = walk_args(ctxs[i], starts[i], n[i], length, rng_seed, traces[i]);
+    as[i] = walk_args(ctxs[i], starts[i], n[i], length, rng_seed, traces[i], flags);
     ss[i] = static_cast<cudaStream_t>(streams[i]);
   }
-  if (world == 1) return dsp_random_walk(ctxs[0], starts[0], n[0], length, rng_seed, traces[0], streams[0]);
+  if (world == 1) return dsp_random_walk(ctxs[0], starts[0], n[0], length, rng_seed, traces[0], flags, streams[0]);
   return run_walks(cs, as, ss, length);
 }
 

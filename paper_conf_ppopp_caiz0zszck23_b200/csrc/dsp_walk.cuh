@@ -78,6 +78,7 @@ struct WalkArgs {
   WalkPeers peers;
   int32_t *traces;          // caller's output (finish)
   int *err;
+  int32_t independent;      // DSP_WALK_INDEPENDENT: draws keyed by the walk index (R35)
 };
 
 // Origin: trace rows := -1, column 0 := start, walkers of step 0 := the
@@ -146,7 +147,8 @@ __device__ __forceinline__ void walk_scatter_body(const WalkArgs &a, const WalkR
       const uint32_t c = *(volatile uint32_t *)&ctr[2 + o];
       ctr[2 + o] = 0u;
       *walk_hdr(a.peers.base[o], a.L, rd.parity, a.rank) =
-          make_uint4(c, (uint32_t)a.length | ((uint32_t)rd.step << 16), a.key.x, a.key.y);
+          make_uint4(c, (uint32_t)a.length | ((uint32_t)rd.step << 16) | ((uint32_t)a.independent << 30), a.key.x,
+                     a.key.y);
     }
     __threadfence_system();
     for (int o = 0; o < a.bd.world; ++o) st_release_sys(walk_flag(a.peers.base[o], a.L, rd.parity, a.rank), rd.seq);
@@ -166,7 +168,8 @@ __device__ __forceinline__ void walk_step_body(const WalkArgs &a, const WalkRoun
       uint32_t acc = 0;
       for (int s = 0; s < world; ++s) {
         const uint4 h = __ldcv(walk_hdr(self, a.L, rd.parity, s));
-        if (h.y != ((uint32_t)a.length | ((uint32_t)rd.step << 16)) || h.z != a.key.x || h.w != a.key.y)
+        if (h.y != ((uint32_t)a.length | ((uint32_t)rd.step << 16) | ((uint32_t)a.independent << 30)) ||
+            h.z != a.key.x || h.w != a.key.y)
           latch(a.err, E_STATE);
         s_off[s] = acc;
         acc += h.x <= (uint32_t)a.L.cap ? h.x : 0u;
@@ -193,7 +196,12 @@ __device__ __forceinline__ void walk_step_body(const WalkArgs &a, const WalkRoun
         } else {
           int64_t rs, d;
           row_extent(a.indptr, lv, &rs, &d);
-          if (d > 0) u = __ldg(a.indices + rs + (d == 1 ? 0u : draw_range(a.key, 0u, w.y, rd.step, (uint32_t)d)));
+          const uint32_t wi = (uint32_t)w.x & (uint32_t)(WALK_MAX - 1);  // index in the origin's starts
+          if (d > 0)
+            u = __ldg(a.indices + rs +
+                      (d == 1          ? 0u
+                       : a.independent ? walk_draw(a.key, wi, w.y, rd.step, (uint32_t)d)
+                                       : draw_range(a.key, 0u, w.y, rd.step, (uint32_t)d)));
         }
         const int origin = (int)((uint32_t)w.x >> WALK_RANK_SHIFT);
         const int64_t i = (int64_t)((uint32_t)w.x & (uint32_t)(WALK_MAX - 1));

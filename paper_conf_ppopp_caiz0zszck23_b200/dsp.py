@@ -42,6 +42,7 @@ DSP_ASYNC = 1
 DSP_PIPELINED = 2
 DSP_BIASED = 4
 DSP_LAYERWISE = 8
+DSP_WALK_INDEPENDENT = 16
 DSP_OPT_RELABEL_MAP = 1
 DSP_OPT_LANE_ROUNDS = 2
 DSP_OPT_LOADER_WARPS = 3
@@ -106,9 +107,9 @@ def lib(path: str | None = None):
         L.dsp_gather_features.argtypes = [P, P, i64, P, P]
         L.dsp_pipeline_flush.argtypes = [P, P]
         L.dsp_set_persistent_blocks.argtypes = [P, i32]
-        L.dsp_random_walk.argtypes = [P, P, i64, i32, ctypes.c_uint64, P, P]
+        L.dsp_random_walk.argtypes = [P, P, i64, i32, ctypes.c_uint64, P, ctypes.c_uint32, P]
         L.dsp_reserve_walks.argtypes = [P, i64, i32]
-        L.dsp_random_walk_group.argtypes = [P, i32, P, P, i32, ctypes.c_uint64, P, P]
+        L.dsp_random_walk_group.argtypes = [P, i32, P, P, i32, ctypes.c_uint64, P, ctypes.c_uint32, P]
         L.dsp_sync.argtypes = [P, P]
         L.dsp_set_option.argtypes = [P, i32, i64]
         for name in ("dsp_create", "dsp_load_partition", "dsp_load_features_tiered", "dsp_load_weights", "dsp_reserve",
@@ -272,8 +273,8 @@ def dsp_set_persistent_blocks(ctx, blocks: int) -> None:
     _check(lib().dsp_set_persistent_blocks(ctx, blocks), ctx)
 
 
-def dsp_random_walk(ctx, starts, n: int, length: int, rng_seed: int, traces, stream: int) -> None:
-    _check(lib().dsp_random_walk(ctx, _p(starts), n, length, ctypes.c_uint64(rng_seed), _p(traces),
+def dsp_random_walk(ctx, starts, n: int, length: int, rng_seed: int, traces, stream: int, flags: int = 0) -> None:
+    _check(lib().dsp_random_walk(ctx, _p(starts), n, length, ctypes.c_uint64(rng_seed), _p(traces), flags,
                                  ctypes.c_void_p(stream)), ctx)
 
 
@@ -281,15 +282,15 @@ def dsp_reserve_walks(ctx, max_walks: int, max_length: int) -> None:
     _check(lib().dsp_reserve_walks(ctx, max_walks, max_length), ctx)
 
 
-def dsp_random_walk_group(ctxs, starts, n, length: int, rng_seed: int, traces, streams) -> None:
+def dsp_random_walk_group(ctxs, starts, n, length: int, rng_seed: int, traces, streams, flags: int = 0) -> None:
     k = len(ctxs)
     c_ctxs = (ctypes.c_void_p * k)(*[c.value if isinstance(c, ctypes.c_void_p) else c for c in ctxs])
     c_starts = (ctypes.c_void_p * k)(*[x.data_ptr() for x in starts])
     c_n = (ctypes.c_int64 * k)(*[int(x) for x in n])
     c_tr = (ctypes.c_void_p * k)(*[x.data_ptr() for x in traces])
     c_st = (ctypes.c_void_p * k)(*streams)
-    _check(lib().dsp_random_walk_group(c_ctxs, k, c_starts, c_n, length, ctypes.c_uint64(rng_seed), c_tr, c_st),
-           ctxs[0])
+    _check(lib().dsp_random_walk_group(c_ctxs, k, c_starts, c_n, length, ctypes.c_uint64(rng_seed), c_tr, flags,
+                                       c_st), ctxs[0])
 
 
 def dsp_sync(ctx, stream: int) -> None:
@@ -445,15 +446,17 @@ class Sampler:
         dsp_gather_features(self.ctx, ids, n, out, self.stream())
         return out
 
-    def random_walk(self, starts, length: int, rng_seed: int, out=None):
+    def random_walk(self, starts, length: int, rng_seed: int, out=None, independent: bool = False):
         """Walk traces int32[n][length + 1], asynchronous on the stream
-        (into `out` when given: a caller-owned int32[n][length + 1] buffer)."""
+        (into `out` when given: a caller-owned int32[n][length + 1] buffer).
+        independent: DSP_WALK_INDEPENDENT (walks from one start differ, R35)."""
         torch = self.torch
         assert starts.dtype == torch.int32 and starts.is_cuda and starts.is_contiguous()
         if out is None:
             out = torch.empty((starts.numel(), length + 1), dtype=torch.int32, device=starts.device)
         assert out.dtype == torch.int32 and out.is_cuda and out.is_contiguous() and out.shape == (starts.numel(), length + 1)
-        dsp_random_walk(self.ctx, starts, starts.numel(), length, rng_seed, out, self.stream())
+        dsp_random_walk(self.ctx, starts, starts.numel(), length, rng_seed, out, self.stream(),
+                        DSP_WALK_INDEPENDENT if independent else 0)
         return out
 
     def sync(self) -> None:
@@ -524,13 +527,13 @@ class LocalGroup:
                          | (DSP_ASYNC if async_ else 0), st)
         return None if async_ else [s.blocks(slot) for s in S]
 
-    def random_walk(self, starts_per_rank, length: int, rng_seed: int):
+    def random_walk(self, starts_per_rank, length: int, rng_seed: int, independent: bool = False):
         """Walk traces of every rank, CSP push without reshuffle."""
         torch = self.samplers[0].torch
         S = self.samplers
         outs = [torch.empty((x.numel(), length + 1), dtype=torch.int32, device=x.device) for x in starts_per_rank]
         dsp_random_walk_group([s.ctx for s in S], starts_per_rank, [x.numel() for x in starts_per_rank], length,
-                              rng_seed, outs, [s.stream() for s in S])
+                              rng_seed, outs, [s.stream() for s in S], DSP_WALK_INDEPENDENT if independent else 0)
         return outs
 
     def close(self):

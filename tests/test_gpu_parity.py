@@ -255,6 +255,42 @@ def test_virtual_ranks_exchange_channels(pkg, tiny, P):
     grp.close()
 
 
+@pytest.mark.parametrize("P,K", [(2, 2), (4, 3)])
+def test_virtual_ranks_concurrent_group_calls(pkg, tiny, P, K):
+    """K asynchronous group calls in flight on K streams (DSP_ASYNC group calls,
+    DSP_OPT_EXCHANGE_CHANNELS = K, each rank's launch on 1/(P*K) of the SMs),
+    each into its own workspace and output set; every rank's blocks equal the
+    oracle (sizes from the oracle, array contents compared)."""
+    cfg, ip, ix, feats = tiny
+    bnds = datagen.bounds(cfg.num_nodes, P)
+    shards = []
+    for r in range(P):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi]))
+    n = 2 * K
+    grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 32, devices=[0] * P, n_workspaces=K, n_slots=n,
+                         options={pkg.dsp.DSP_OPT_EXCHANGE_CHANNELS: K})
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    for s in grp.samplers:
+        pkg.dsp_set_persistent_blocks(s.ctx, max(1, sms // (P * K)))
+    per_rank = [seeds_of(cfg, P, r, batch=32) for r in range(P)]
+    dev = [[torch.from_numpy(np.ascontiguousarray(per_rank[r][i])).cuda() for r in range(P)] for i in range(n)]
+    streams = [torch.cuda.Stream() for _ in range(K)]
+    torch.cuda.synchronize()
+    for i in range(n):   # call i: stream / workspace i % K, output set i (calls i and i + K share a workspace)
+        grp.sample(dev[i], 0x900 + i, async_=True, ws=i % K, slot=i, stream=streams[i % K])
+    torch.cuda.synchronize()
+    for s in grp.samplers:
+        s.sync()
+    for i in range(n):
+        for r in range(P):
+            ref = oracle.sample(ip, ix, per_rank[r][i], cfg.fanouts, 0x900 + i)
+            sizes = [x for b in ref for x in (b["num_dst"], b["num_src"], b["num_edges"])]
+            assert_blocks_equal(grp.samplers[r].blocks(i, sizes), ref, f"P={P} K={K} call {i} rank {r}")
+    grp.close()
+
+
 @pytest.mark.parametrize("mode", ["direct", "hash"])
 def test_virtual_ranks_errors(pkg, tiny, mode):
     """Device-detected errors at world > 1 (duplicate seed, out-of-range seed)
@@ -668,6 +704,38 @@ def test_random_walks_virtual_ranks(pkg, tiny, P):
         grp.random_walk([torch.zeros(1, dtype=torch.int32, device="cuda") for _ in range(P)], 65, 1)
     assert e.value.status == pkg.dsp.DSP_ERR_CAPACITY
     grp.close()
+
+
+@pytest.mark.parametrize("P", [1, 2, 4])
+def test_random_walks_independent(pkg, tiny, P):
+    """DSP_WALK_INDEPENDENT (R35): walk i draws with its own index, so the
+    repeated starts of one call give different walks; traces equal the
+    oracle's independent mode at P = 1 (thread per walk) and across virtual
+    ranks (CSP push: the walk index travels with the walker)."""
+    cfg, ip, ix, feats = tiny
+    rng = np.random.default_rng(40 + P)
+    hub = int(np.argmax(np.diff(ip)))
+    starts = [np.concatenate([np.full(200, hub, np.int32),
+                              rng.integers(0, cfg.num_nodes, size=300).astype(np.int32)]) for _ in range(P)]
+    L = 20
+    if P == 1:
+        s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8)
+        trs = [s.random_walk(torch.from_numpy(starts[0]).cuda(), L, 0xFEED, independent=True)]
+        s.sync()
+        s.close()
+    else:
+        bnds = datagen.bounds(cfg.num_nodes, P)
+        shards = [datagen.shard(ip, ix, int(bnds[r]), int(bnds[r + 1])) + (feats[int(bnds[r]):int(bnds[r + 1])],)
+                  for r in range(P)]
+        grp = pkg.LocalGroup(bnds, shards, cfg.fanouts, 8, devices=[0] * P, max_walks=1000, max_walk_length=32)
+        trs = grp.random_walk([torch.from_numpy(x).cuda() for x in starts], L, 0xFEED, independent=True)
+        for smp in grp.samplers:
+            smp.sync()
+        grp.close()
+    for r in range(P):
+        got = trs[r].cpu().numpy()
+        assert np.array_equal(got, oracle.random_walk(ip, ix, starts[r], L, 0xFEED, independent=True)), (P, r)
+        assert len({tuple(row) for row in got[:200]}) > 150      # the 200 walks from the hub differ
 
 
 def test_random_walks_need_reservation(pkg, tiny):
