@@ -10,7 +10,7 @@ from __future__ import annotations
 
 import ctypes
 import os
-from typing import Callable, NamedTuple, Sequence
+from typing import Callable, Sequence
 
 import numpy as np
 
@@ -299,14 +299,30 @@ def dsp_sync(ctx, stream: int) -> None:
 
 # ------------------------------------------------------------ conveniences
 
-class Block(NamedTuple):
-    """One sampled layer; tensors are views of the Sampler's device buffers."""
-    num_dst: int
-    num_src: int
-    num_edges: int
-    indptr: "object"   # torch.int32 [num_dst + 1]
-    indices: "object"  # torch.int32 [num_edges] local src ids
-    src_ids: "object"  # torch.int32 [num_src] global ids
+class Block:
+    """One sampled layer: its sizes, and views of the Sampler's device buffers
+    (torch.int32 `indptr` [num_dst + 1], `indices` [num_edges] local src ids,
+    `src_ids` [num_src] global ids) made on first access, so a caller that only
+    needs the sizes pays no tensor slicing per step."""
+    __slots__ = ("num_dst", "num_src", "num_edges", "_bufs", "_views")
+
+    def __init__(self, num_dst: int, num_src: int, num_edges: int, bufs):
+        self.num_dst, self.num_src, self.num_edges = num_dst, num_src, num_edges
+        self._bufs = bufs
+        self._views = None
+
+    def _view(self, j):
+        if self._views is None:
+            ip, ix, sr = self._bufs
+            self._views = (ip[: self.num_dst + 1], ix[: self.num_edges], sr[: self.num_src])
+        return self._views[j]
+
+    indptr = property(lambda self: self._view(0))
+    indices = property(lambda self: self._view(1))
+    src_ids = property(lambda self: self._view(2))
+
+    def __repr__(self):
+        return f"Block(num_dst={self.num_dst}, num_src={self.num_src}, num_edges={self.num_edges})"
 
 
 class Sampler:
@@ -435,7 +451,7 @@ class Sampler:
                 nd, ns, ne = b.num_dst, b.num_src, b.num_edges
             else:
                 nd, ns, ne = (int(x) for x in sizes[3 * l: 3 * l + 3])
-            out.append(Block(nd, ns, ne, ip[: nd + 1], ix[: ne], sr[: ns]))
+            out.append(Block(nd, ns, ne, (ip, ix, sr)))
         return out
 
     def gather(self, ids, out=None):
