@@ -859,8 +859,9 @@ __device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int
   const uint32_t tid = (uint32_t)tid64, nthreads = (uint32_t)nthreads64;
   const uint32_t dim4 = (uint32_t)a.dim4;
   const int32_t N = (int32_t)a.bd.b[a.bd.world];
-  const unsigned long long pol = l2_policy_evict_first(), pol_t = l2_policy_tail();
   const uint32_t head4 = (uint32_t)a.head4;
+  // packed rows (head4 == 0) stream with evict_first; split rows keep their small tail array resident
+  const unsigned long long pol = l2_policy_evict_first(), pol_t = head4 ? l2_policy_tail() : pol;
   for (uint32_t e0 = tid; e0 < total; e0 += nthreads * UNROLL) {
     int32_t g[UNROLL];
     uint32_t c[UNROLL];
@@ -997,7 +998,7 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
   const uint32_t tail_bytes = row_bytes - head_bytes;
   const int64_t nchunks = (n + R - 1) / R;
   char *out = reinterpret_cast<char *>(g.out);
-  const unsigned long long pol = l2_policy_evict_first(), pol_t = l2_policy_tail();
+  const unsigned long long pol = l2_policy_evict_first(), pol_t = head_bytes ? l2_policy_tail() : pol;
   int issued = 0, done = 0;
   int chunk[SLOTS];  // chunk held by each ring slot
   bool exhausted = false;
@@ -1080,7 +1081,7 @@ __device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
   const int R = a.rows_per_chunk;
   const int64_t nchunks = (n + R - 1) / R;
   const uint32_t dim4 = (uint32_t)g.dim4, head4 = (uint32_t)g.head4;
-  const unsigned long long pol = l2_policy_evict_first(), pol_t = l2_policy_tail();
+  const unsigned long long pol = l2_policy_evict_first(), pol_t = head4 ? l2_policy_tail() : pol;
   while (true) {
     int c = 0;
     if (lane == 0) c = (int)atomicAdd(&a.hdr->gcursor, 1u);

@@ -1271,6 +1271,9 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   if (!prop.cooperativeLaunch)
     return fail(nullptr, DSP_ERR_CUDA, "device %d lacks cooperative launch", cuda_device);
   dsp_ctx *c = new dsp_ctx();
+#ifdef DSP_SPLIT_DEFAULT  // experiment build (_build.build_variant): split feature rows by default
+  c->split_rows = true;
+#endif
   c->rank = rank;
   c->world = world_size;
   c->device = cuda_device;
