@@ -555,8 +555,6 @@ def run_dsp(args):
     # the layer-wise scheme keeps one stream there: its exchange region is per ctx)
     K = max(1, args.instances) if world == 1 or not layer else 1
     opts = {pkg.dsp.DSP_OPT_EXCHANGE_CHANNELS: K} if world > 1 and not layer else {}
-    if args.loader_warps:
-        opts[pkg.dsp.DSP_OPT_LOADER_WARPS] = args.loader_warps
     if args.loader_rows:
         opts[pkg.dsp.DSP_OPT_LOADER_ROWS] = args.loader_rows
     s = pkg.Sampler(bnds, sip, six, feats, fanouts, cfg.batch, rank=rank, world_size=world, scheme="layer" if layer else "node",
@@ -963,7 +961,6 @@ def main(argv=None):
     ap.add_argument("--no-breakdown", action="store_true")
     ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
     ap.add_argument("--instances", type=int, default=4, help="concurrent step streams (each on 1/K of the SMs; world > 1: one exchange channel each)")
-    ap.add_argument("--loader-warps", type=int, default=0, help="DSP_OPT_LOADER_WARPS (0: library default)")
     ap.add_argument("--loader-rows", type=int, default=0, help="DSP_OPT_LOADER_ROWS (0: library default)")
     ap.add_argument("--layer-sizes", default="1000,1000",
                     help="--scheme layer: nodes sampled per layer (Table 7: 1000,1000)")

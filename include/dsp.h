@@ -301,8 +301,6 @@ dsp_status dsp_set_persistent_blocks(dsp_ctx *ctx, int32_t blocks);
    DSP_OPT_LANE_ROUNDS     node-wise sampling with lane groups (G lanes per
                            node) while frontier * G <= value * sampling threads,
                            else a thread per node; 1..1024, default 8.
-   DSP_OPT_LOADER_WARPS    TMA loader warps per SM of a DSP_PIPELINED launch:
-                           2, 4 (default) or 8.
    DSP_OPT_LOADER_ROWS     rows per TMA gather chunk, 1..32 (default 32).
    DSP_OPT_GATHER_REGLOADS 0 (default) = standalone gathers and cold-tier rows
                            moved by TMA bulk copies; 1 = 16-byte register
@@ -335,7 +333,6 @@ dsp_status dsp_set_persistent_blocks(dsp_ctx *ctx, int32_t blocks);
                            with dsp_set_persistent_blocks. */
 #define DSP_OPT_RELABEL_MAP 1
 #define DSP_OPT_LANE_ROUNDS 2
-#define DSP_OPT_LOADER_WARPS 3
 #define DSP_OPT_LOADER_ROWS 4
 #define DSP_OPT_GATHER_REGLOADS 5
 #define DSP_OPT_EXCHANGE_CHANNELS 6

@@ -906,15 +906,12 @@ __global__ void __launch_bounds__(NT) k_gather(const __grid_constant__ GatherArg
 
 // ============================================ world == 1: persistent kernel
 constexpr int LOADER_WARPS = 4;                      // TMA gather warps of a pipelined launch (default)
-constexpr int LOADER_WARPS_MAX = 8;                  // ... or 8 (dsp_ctx::loader_warps)
 #ifndef DSP_LOADER_SLOTS
 #define DSP_LOADER_SLOTS 2
 #endif
 constexpr int LOADER_SLOTS = DSP_LOADER_SLOTS;       // ring slots per loader warp of a pipelined launch
 constexpr int GTMA_SLOTS = 2;                        // ring slots per warp of the standalone gather
 constexpr int PIPE_TEAM = PNT - 32 * LOADER_WARPS;   // sampling threads of a pipelined launch
-constexpr int PIPE_TEAM8 = PNT - 32 * LOADER_WARPS_MAX;
-constexpr int PIPE_TEAM2 = PNT - 32 * 2;
 
 struct PersistArgs {
   const int32_t *seeds;
@@ -944,12 +941,14 @@ struct PersistArgs {
   int32_t lane_rounds;      // lane groups per node while F * G <= lane_rounds * team threads
 };
 
-template <int TEAM>
+// BIASED is a template parameter (not a runtime branch) so the uniform
+// kernel carries no biased-sampling code (fewer instruction-cache misses).
+template <int TEAM, bool BIASED>
 __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32_t *frontier, int F, int l,
                                                uint32_t epoch) {
   const int k = a.k[l];
   const LayerBufs &B = a.buf[l & 1];
-  if (a.biased) {
+  if (BIASED) {
     phase_sample_biased<TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.weights, a.lo, a.n_local, B, epoch,
                               a.out.src_ids[l], a.err);
   } else if (k <= 16 && (int64_t)F * (k <= 4 ? 4 : k <= 8 ? 8 : 16) <= (int64_t)a.lane_rounds * gridDim.x * TEAM) {
@@ -1153,10 +1152,10 @@ __global__ void __launch_bounds__(32 * GTMA_WARPS) k_gather_tma(const __grid_con
 // previous call's gather by the loader warps running alongside the sampling
 // (the paper's loader(t-1) || sampler(t)).  No host round trip,
 // no map clearing (epochs).
-template <int TEAM, bool PIPE>
+template <int TEAM, bool PIPE, bool BIASED>
 __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(const __grid_constant__ PersistArgs a) {
   __shared__ Scan2Smem<TEAM> sm;
-  __shared__ __align__(8) uint64_t bars[LOADER_WARPS_MAX][LOADER_SLOTS];
+  __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];
   extern __shared__ __align__(128) char ring_smem[];
   const int blk = blockIdx.x, nblk = gridDim.x;
 
@@ -1199,7 +1198,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(const __grid_constant
     const uint32_t epoch = e0 + 1 + l;
     const int32_t *frontier = l == 0 ? a.seeds : a.out.src_ids[l - 1];
     const int k = a.k[l];
-    persist_sample<TEAM>(a, frontier, F, l, epoch);
+    persist_sample<TEAM, BIASED>(a, frontier, F, l, epoch);
     if (l > 0)
       phase_indices_dups(Fprev, a.k[l - 1], a.buf[(l - 1) & 1], a.out.indptr[l - 1], a.out.indices[l - 1],
                          block_span<TEAM>((int64_t)Fprev * a.k[l - 1]));

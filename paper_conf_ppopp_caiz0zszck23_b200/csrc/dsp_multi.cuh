@@ -353,7 +353,7 @@ __device__ __forceinline__ void multi_unpermute(const MultiArgs &m, const int32_
   }
 }
 
-template <int TEAM, bool PIPE>
+template <int TEAM, bool PIPE, bool BIASED>
 __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ MultiArgs m) {
   __shared__ Scan2Smem<TEAM> sm;
   __shared__ uint32_t s_cnt[8], s_base[8], s_off[9];
@@ -436,7 +436,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ Mu
     team_sync<TEAM>();
     const int T = (int)s_off[world];
     const int G = k <= 4 ? 4 : k <= 8 ? 8 : 16;
-    if (a.biased)
+    if (BIASED)  // a template parameter: the uniform kernel carries no biased code
       multi_sample_biased<TEAM>(m, T, s_off, l, k, par);
     else if (k > 16)
       multi_sample_lanes<32, TEAM>(m, T, s_off, l, k, par);

@@ -202,7 +202,6 @@ struct dsp_ctx {
   // dsp_set_option (performance only; results are identical for every value)
   int lane_rounds = 8;  // DSP_OPT_LANE_ROUNDS (8 measured best with 4 streams)
   int relabel_mode = 0; // DSP_OPT_RELABEL_MAP: 0 by N, 1 compact direct, 2 hash, 3 8-byte direct
-  int loader_warps = 4; // DSP_OPT_LOADER_WARPS: 2, 4 or 8
   int loader_rows = 32;  // DSP_OPT_LOADER_ROWS: rows per TMA chunk, <= 32
   int persist_blocks = 0;  // blocks of the persistent kernel (0 = one per SM x occupancy)
   bool gather_reg = false;    // DSP_OPT_GATHER_REGLOADS: standalone gathers with register loads
@@ -675,7 +674,6 @@ const int32_t *frontier_of(const Call &k, int l) { return l == 0 ? k.seeds : k.b
 uint2 key_of(uint64_t rng_seed) { return make_uint2((uint32_t)rng_seed, (uint32_t)(rng_seed >> 32)); }
 
 // world == 1: the whole call (+ optional gather) in one cooperative kernel
-constexpr int PIPE_SMEM8_MAX = 200 * 1024;  // ring of 8 loader warps (rows up to 12.8 KB)
 
 dsp_status stage_persistent(Call &k) {
   dsp_ctx *c = k.c;
@@ -709,8 +707,9 @@ dsp_status stage_persistent(Call &k) {
   const dim3 grid(c->persist_blocks > 0 ? c->persist_blocks : c->num_sms * c->persist_blocks_per_sm), block(PNT);
   void *args[] = {&a};
   if (!k.pipelined) {
-    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_persistent<PNT, false>, grid, block, args, 0,
-                                            k.stream));
+    CUDA_TRY(c, cudaLaunchCooperativeKernel(k.biased ? (const void *)k_csp_persistent<PNT, false, true>
+                                                     : (const void *)k_csp_persistent<PNT, false, false>,
+                                            grid, block, args, 0, k.stream));
     return DSP_OK;
   }
   dsp_ctx::Pending *pd = c->pending_of(k.ws);
@@ -724,13 +723,9 @@ dsp_status stage_persistent(Call &k) {
   // shared memory is taken from the L1 the sampling phases use
   a.rows_per_chunk = std::max(1, std::min(c->loader_rows, 12800 / std::max(1, row_bytes)));
   a.slot_bytes = (int)align_up((size_t)a.rows_per_chunk * row_bytes, 128);
-  const bool lw8 = c->loader_warps == LOADER_WARPS_MAX &&
-                   (size_t)LOADER_WARPS_MAX * LOADER_SLOTS * a.slot_bytes <= (size_t)PIPE_SMEM8_MAX;
-  const bool lw2 = c->loader_warps == 2;
-  const size_t smem = (size_t)(lw8 ? LOADER_WARPS_MAX : lw2 ? 2 : LOADER_WARPS) * LOADER_SLOTS * a.slot_bytes;
-  CUDA_TRY(c, cudaLaunchCooperativeKernel(lw8   ? (const void *)k_csp_persistent<PIPE_TEAM8, true>
-                                          : lw2 ? (const void *)k_csp_persistent<PIPE_TEAM2, true>
-                                                : (const void *)k_csp_persistent<PIPE_TEAM, true>,
+  const size_t smem = (size_t)LOADER_WARPS * LOADER_SLOTS * a.slot_bytes;
+  CUDA_TRY(c, cudaLaunchCooperativeKernel(k.biased ? (const void *)k_csp_persistent<PIPE_TEAM, true, true>
+                                                   : (const void *)k_csp_persistent<PIPE_TEAM, true, false>,
                                           grid, block, args, smem, k.stream));
   pd->ids = k.blocks[k.L - 1].src_ids;
   pd->out = k.feat_out;
@@ -817,7 +812,9 @@ dsp_status stage_persistent_multi(Call &k, int share) {
   if (c->channels > 1 && c->chan_used[k.channel])  // the channel's previous call (possibly on another stream)
     CUDA_TRY(c, cudaStreamWaitEvent(st, cev, 0));
   if (!k.pipelined) {
-    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_multi<PNT, false>, grid, block, args, 0, st));
+    CUDA_TRY(c, cudaLaunchCooperativeKernel(k.biased ? (const void *)k_csp_multi<PNT, false, true>
+                                                     : (const void *)k_csp_multi<PNT, false, false>,
+                                            grid, block, args, 0, st));
   } else {
     dsp_ctx::Pending *pd = c->pending_of(k.ws);
     if (!pd) return fail(c, DSP_ERR_STATE, "more than 8 workspaces with pending pipelined gathers");
@@ -829,7 +826,9 @@ dsp_status stage_persistent_multi(Call &k, int share) {
     a.slot_bytes = (int)align_up((size_t)std::max(12800, row_bytes), 128);
     a.rows_per_chunk = std::max(1, std::min(c->loader_rows, a.slot_bytes / std::max(1, row_bytes)));
     const size_t smem = (size_t)LOADER_WARPS * LOADER_SLOTS * a.slot_bytes;
-    CUDA_TRY(c, cudaLaunchCooperativeKernel((const void *)k_csp_multi<PIPE_TEAM, true>, grid, block, args, smem, st));
+    CUDA_TRY(c, cudaLaunchCooperativeKernel(k.biased ? (const void *)k_csp_multi<PIPE_TEAM, true, true>
+                                                     : (const void *)k_csp_multi<PIPE_TEAM, true, false>,
+                                            grid, block, args, smem, st));
     pd->ids = k.blocks[k.L - 1].src_ids;
     pd->out = k.feat_out;
     pd->stream = k.stream;
@@ -1281,16 +1280,16 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   DeviceGuard g(cuda_device);
   int occ = 0, occ_pipe = 0;
   const int pipe_smem = std::min(LOADER_WARPS * LOADER_SLOTS * 16384, 200 * 1024);  // largest ring (dim 4096)
-  if (cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM, true>,
+  if (cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM, true, false>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM2, true>,
+      cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM, true, true>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM8, true>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, PIPE_SMEM8_MAX) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_csp_multi<PIPE_TEAM, true>,
+      cudaFuncSetAttribute((const void *)k_csp_multi<PIPE_TEAM, true, false>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_csp_persistent<PNT, false>, PNT, 0) != cudaSuccess ||
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_pipe, k_csp_persistent<PIPE_TEAM, true>, PNT, pipe_smem) !=
+      cudaFuncSetAttribute((const void *)k_csp_multi<PIPE_TEAM, true, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_csp_persistent<PNT, false, false>, PNT, 0) != cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_pipe, k_csp_persistent<PIPE_TEAM, true, false>, PNT, pipe_smem) !=
           cudaSuccess ||
       occ < 1 || occ_pipe < 1) {
     cudaGetLastError();
@@ -1891,11 +1890,6 @@ dsp_status dsp_set_option(dsp_ctx *c, int32_t option, int64_t value) {
     case DSP_OPT_LANE_ROUNDS:
       if (value < 1 || value > 1024) return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_LANE_ROUNDS %lld not in [1, 1024]", (long long)value);
       c->lane_rounds = (int)value;
-      return DSP_OK;
-    case DSP_OPT_LOADER_WARPS:
-      if (value != 2 && value != LOADER_WARPS && value != LOADER_WARPS_MAX)
-        return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_LOADER_WARPS must be 2, 4 or 8");
-      c->loader_warps = (int)value;
       return DSP_OK;
     case DSP_OPT_LOADER_ROWS:
       if (value < 1 || value > 32) return fail(c, DSP_ERR_INVALID_ARG, "DSP_OPT_LOADER_ROWS %lld not in [1, 32]", (long long)value);

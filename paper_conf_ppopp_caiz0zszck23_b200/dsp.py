@@ -45,7 +45,6 @@ DSP_LAYERWISE = 8
 DSP_WALK_INDEPENDENT = 16
 DSP_OPT_RELABEL_MAP = 1
 DSP_OPT_LANE_ROUNDS = 2
-DSP_OPT_LOADER_WARPS = 3
 DSP_OPT_LOADER_ROWS = 4
 DSP_OPT_GATHER_REGLOADS = 5
 DSP_OPT_EXCHANGE_CHANNELS = 6
