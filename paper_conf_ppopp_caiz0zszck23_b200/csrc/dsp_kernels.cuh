@@ -32,6 +32,15 @@
 
 namespace dsp {
 
+// Inlining of the phase bodies into the persistent kernels.  DSP_PHASE_NOINLINE
+// (experiment build) compiles each phase as its own function, so the code a
+// phase runs stays contiguous (instruction-cache footprint of the huge kernels).
+#ifdef DSP_PHASE_NOINLINE
+#define DSP_PHASE __noinline__
+#else
+#define DSP_PHASE __forceinline__
+#endif
+
 constexpr int NT = 256;    // threads per block of the per-phase kernels
 constexpr int PNT = 1024;  // threads per block of the persistent kernel (1 block per SM)
 constexpr int MAX_PERSIST_BLOCKS = 1024;
@@ -207,8 +216,10 @@ __device__ __forceinline__ uint32_t mword_x(const LayerBufs &B, unsigned long lo
          : B.mask  ? 0x1ffffffu - (uint32_t)(w & 0x1ffffffull)
                    : mark_x(w);
 }
-// claims (or finds) the slot of key u; returns its word pointer and the word seen there
-__device__ __forceinline__ unsigned long long *hash_claim(const LayerBufs &B, int32_t u, uint32_t epoch, uint32_t x,
+// claims (or finds) the slot of key u; returns its word pointer and the word seen there.
+// Out of line (like map_find): the probing loops stay out of the hot inlined code of
+// the direct-map layouts (instruction-cache footprint of the persistent kernels).
+__device__ __noinline__ unsigned long long *hash_claim(const LayerBufs &B, int32_t u, uint32_t epoch, uint32_t x,
                                                         unsigned long long *seen) {
   const unsigned long long want = hword(epoch, u, x), hi = want >> 25;
   const unsigned long long tag = (unsigned long long)htag(epoch);
@@ -233,12 +244,15 @@ __device__ __forceinline__ unsigned long long *hash_claim(const LayerBufs &B, in
   }
 }
 // slot of key u (inserted earlier in this epoch); 64-bit layouts only
-__device__ __forceinline__ unsigned long long *map_find(const LayerBufs &B, int32_t u, uint32_t epoch) {
-  if (!B.mask) return B.first + u;
+__device__ __noinline__ unsigned long long *map_find_hashed(const LayerBufs &B, int32_t u, uint32_t epoch) {
   const unsigned long long hi = ((unsigned long long)htag(epoch) << 31) | (uint32_t)u;
   uint32_t h = hash32((uint32_t)u) & B.mask;
   while ((map_ld(B.first + h) >> 25) != hi) h = (h + 1u) & B.mask;
   return B.first + h;
+}
+__device__ __forceinline__ unsigned long long *map_find(const LayerBufs &B, int32_t u, uint32_t epoch) {
+  if (!B.mask) return B.first + u;
+  return map_find_hashed(B, u, epoch);
 }
 // the word of key u (marked earlier in this epoch), compared with mword()
 __device__ __forceinline__ unsigned long long map_get(const LayerBufs &B, int32_t u, uint32_t epoch) {
@@ -412,7 +426,7 @@ __device__ __forceinline__ void mark_dst(const LayerBufs &B, int32_t v, int i, i
 // on separate lanes, Floyd's resolution and the ranking via shuffles
 // (sample_node).  Used for k > 16.
 template <int G, int TEAM = PNT>
-__device__ __forceinline__ void phase_sample_lanes(const int32_t *frontier, int F, int layer, int k, uint2 key,
+__device__ DSP_PHASE void phase_sample_lanes(const int32_t *frontier, int F, int layer, int k, uint2 key,
                                                    const int64_t *__restrict__ indptr,
                                                    const int32_t *__restrict__ indices, int64_t lo,
                                                    int64_t n_local, const LayerBufs &B, uint32_t epoch,
@@ -466,7 +480,7 @@ __device__ __forceinline__ void phase_sample_lanes(const int32_t *frontier, int 
 // marks are issued back to back (memory-level parallelism k per thread, every
 // frontier node in flight at once).
 template <int KB, int TEAM = PNT>
-__device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F, int layer, int k, uint2 key,
+__device__ DSP_PHASE void phase_sample_tpn(const int32_t *frontier, int F, int layer, int k, uint2 key,
                                                  const int64_t *__restrict__ indptr,
                                                  const int32_t *__restrict__ indices, int64_t lo,
                                                  int64_t n_local, const LayerBufs &B, uint32_t epoch,
@@ -539,7 +553,7 @@ __device__ __forceinline__ void phase_sample_tpn(const int32_t *frontier, int F,
 // Biased sampling: one warp per node, sample_node_biased; the
 // sampled neighbours come out in ascending row order (slot = lane).
 template <int TEAM = PNT>
-__device__ __forceinline__ void phase_sample_biased(const int32_t *frontier, int F, int layer, int k, uint2 key,
+__device__ DSP_PHASE void phase_sample_biased(const int32_t *frontier, int F, int layer, int k, uint2 key,
                                                     const int64_t *__restrict__ indptr,
                                                     const int32_t *__restrict__ indices,
                                                     const uint32_t *__restrict__ weights, int64_t lo,
@@ -763,7 +777,7 @@ __device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, in
 // Duplicates of layer l (after pass 2 and a grid barrier): a valid slot q
 // holding -1 - x with x >= F takes the nid stored at its first occurrence's
 // slot x - F.
-__device__ __forceinline__ void phase_indices_dups(int F, int k, const LayerBufs &B, const int32_t *indptr,
+__device__ DSP_PHASE void phase_indices_dups(int F, int k, const LayerBufs &B, const int32_t *indptr,
                                                    int32_t *indices_out, const Span &sp) {
   constexpr int U = 4;  // items per thread in flight
   const FastDiv fd = make_fastdiv((uint32_t)k);
@@ -854,7 +868,7 @@ __device__ __forceinline__ float4 ld_stream_f4(const float4 *p) {
 // flight per thread before any store (Little's law over HBM / NVLink).
 // 32-bit index math (the host guarantees n * dim4 < 2^31).
 template <int UNROLL>
-__device__ __forceinline__ void phase_gather(const GatherArgs &a, int64_t n, int64_t tid64, int64_t nthreads64) {
+__device__ DSP_PHASE void phase_gather(const GatherArgs &a, int64_t n, int64_t tid64, int64_t nthreads64) {
   const uint32_t total = (uint32_t)(n * a.dim4);
   const uint32_t tid = (uint32_t)tid64, nthreads = (uint32_t)nthreads64;
   const uint32_t dim4 = (uint32_t)a.dim4;
@@ -988,7 +1002,7 @@ __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32
 // STATIC: chunks gw, gw + nw, ... instead of the grid-wide cursor (the
 // standalone k_gather_tma, whose warps all gather).
 template <bool MULTI = false, bool STATIC = false, int SLOTS = LOADER_SLOTS>
-__device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, uint64_t *bars, int64_t n,
+__device__ DSP_PHASE void loader_warp(const PersistArgs &a, char *ring, uint64_t *bars, int64_t n,
                                             int64_t gw = 0, int64_t nw = 1) {
   const int lane = threadIdx.x & 31;
   const GatherArgs &g = a.gp;
@@ -1074,7 +1088,7 @@ __device__ __forceinline__ void loader_warp(const PersistArgs &a, char *ring, ui
 // previous call's gather with 16-byte register loads.  MULTI (world > 1):
 // rows of every rank, read from the owner's shard (local or peer-mapped).
 template <bool MULTI = false>
-__device__ __forceinline__ void helper_warp(const PersistArgs &a, int64_t n) {
+__device__ DSP_PHASE void helper_warp(const PersistArgs &a, int64_t n) {
   const int lane = threadIdx.x & 31;
   const GatherArgs &g = a.gp;
   const int R = a.rows_per_chunk;
