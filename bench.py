@@ -513,7 +513,13 @@ def run_walk(args):
                          "traffic": None, "peak_kind": peak_kind,
                          "algorithmic_bytes_per_launch": 24.0 * steps_taken / KS,
                          "achieved_def": "24 B per walk step (indptr pair, adjacency id, trace entry) / elapsed time; "
-                                         "the walk is bound by dependent random DRAM requests, not bytes"},
+                                         "the walk is bound by dependent random DRAM requests, not bytes",
+                         "request_rate": {"achieved": steps_taken / (t_ms * 1e-3), "peak": 47e9, "unit": "requests/s",
+                                          "frac": steps_taken / (t_ms * 1e-3) / 47e9,
+                                          "def": "one random adjacency read (a 32-B DRAM sector) per walk step (the "
+                                                 "indptr pairs hit L2) / elapsed time, against the random-read "
+                                                 "request ceiling measured by tools/micro/random_read_bench.cu "
+                                                 "(~47 G requests/s on B200, 4-64 B per request)"}},
             "e2e": {"value": reduce_sum_over_ranks(e_steps * e2e_frac) / (e2e_ms * 1e-3), "unit": "edges/s",
                     "h2d_bytes_per_step": nw * 4, "d2h_bytes_per_step": nw * (length + 1) * 4, "steps": n_e2e,
                     "api": "starts H2D from pinned host memory, dsp_random_walk, traces D2H into pinned host memory"},

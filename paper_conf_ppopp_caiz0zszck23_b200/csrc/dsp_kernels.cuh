@@ -1088,7 +1088,11 @@ __device__ DSP_PHASE void loader_warp(const PersistArgs &a, char *ring, uint64_t
 // previous call's gather with 16-byte register loads.  MULTI (world > 1):
 // rows of every rank, read from the owner's shard (local or peer-mapped).
 template <bool MULTI = false>
+#ifndef DSP_HELPER_UNROLL
+#define DSP_HELPER_UNROLL 4
+#endif
 __device__ DSP_PHASE void helper_warp(const PersistArgs &a, int64_t n) {
+  constexpr int HU = DSP_HELPER_UNROLL;  // 16-byte loads in flight per lane
   const int lane = threadIdx.x & 31;
   const GatherArgs &g = a.gp;
   const int R = a.rows_per_chunk;
@@ -1103,12 +1107,12 @@ __device__ DSP_PHASE void helper_warp(const PersistArgs &a, int64_t n) {
     if (lane == 0) atomicAdd(&a.hdr->chunks_helper, 1u);
     const int64_t r0 = (int64_t)c * R;
     const uint32_t total = (uint32_t)(min((int64_t)R, n - r0) * dim4);
-    for (uint32_t e0 = lane; e0 < total; e0 += 32 * 4) {
-      float4 v[4];
-      int32_t id[4];
-      uint32_t col[4];
+    for (uint32_t e0 = lane; e0 < total; e0 += 32 * HU) {
+      float4 v[HU];
+      int32_t id[HU];
+      uint32_t col[HU];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < HU; ++u) {
         const uint32_t e = e0 + 32u * u;
         id[u] = -1;
         col[u] = 0;
@@ -1120,12 +1124,12 @@ __device__ DSP_PHASE void helper_warp(const PersistArgs &a, int64_t n) {
       }
       const int32_t N = (int32_t)g.bd.b[MULTI ? g.bd.world : 1];
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
+      for (int u = 0; u < HU; ++u)
         if (id[u] >= 0 && id[u] < N)
           v[u] = ld_f4_hint(row_col(feature_row(g, MULTI ? owner_of(g.bd, id[u]) : 0, id[u]), col[u], head4),
                             col[u] < head4 ? pol : pol_t);
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
+      for (int u = 0; u < HU; ++u) {
         const uint32_t e = e0 + 32u * u;
         if (e < total) {
           if (id[u] >= 0 && id[u] < N)
