@@ -423,15 +423,16 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
       const uint32_t cross = __ballot_sync(FULL_MASK, incl > r);
       const int L = __ffs(cross) - 1;
       uint32_t found = 0, wrem = 0;
-      if (lane == L) {  // the crossing lane alone: branch out at the pick (lane L's segment holds it)
+      if (lane == L) {
         unsigned long long acc = incl - tot;
+        bool done = false;
 #pragma unroll
         for (int j = 0; j < BSEG; ++j) {
-          if (acc + reg[j] > r) {
+          if (!done && acc + reg[j] > r) {
             found = (uint32_t)(lane * S + j);
             wrem = reg[j];
             reg[j] = 0u;  // remove the pick
-            break;
+            done = true;
           }
           acc += reg[j];
         }
