@@ -541,7 +541,10 @@ def run_walk(args):
                                     "sample": f"{n_cpu} x 4096 walks of length {length}, single host thread "
                                               f"(oracle.random_walk), {t_cpu:.1f} s"}
         print(json.dumps(line), flush=True)
+    barrier()
     s.close()
+    if world > 1:
+        dist.destroy_process_group()
     return 0
 
 
@@ -947,6 +950,7 @@ def run_dsp(args):
             "clocks": clk.summary(),
         }
         print(json.dumps(line), flush=True)
+    barrier()   # no rank frees its peer-mapped shard while another may still read it
     s.close()
     if world > 1:
         dist.destroy_process_group()
