@@ -760,3 +760,34 @@ def test_random_walks_products(pkg, products):
     sel = np.arange(0, len(starts), 101)
     assert np.array_equal(tr.cpu().numpy()[sel], oracle.random_walk(ip, ix, starts[sel], 40, 77))
     s.close()
+
+
+def test_set_option_validation(pkg, tiny):
+    """dsp_set_option: unknown options and out-of-range values are
+    DSP_ERR_INVALID_ARG; layout options after the layout exists are
+    DSP_ERR_STATE (the relabel map and the exchange channels after
+    dsp_reserve, the row layout after dsp_load_partition)."""
+    cfg, ip, ix, feats = tiny
+    d = pkg.dsp
+    c = pkg.dsp_create(0, 1, 0)
+    try:
+        for opt, val in ((99, 1), (d.DSP_OPT_RELABEL_MAP, 4), (d.DSP_OPT_LANE_ROUNDS, 0), (d.DSP_OPT_LOADER_ROWS, 33),
+                         (d.DSP_OPT_GATHER_REGLOADS, 2), (d.DSP_OPT_EXCHANGE_CHANNELS, 9), (d.DSP_OPT_SPLIT_ROWS, 2)):
+            with pytest.raises(pkg.DSPError) as e:
+                pkg.dsp_set_option(c, opt, val)
+            assert e.value.status == d.DSP_ERR_INVALID_ARG, (opt, val)
+        pkg.dsp_set_option(c, d.DSP_OPT_SPLIT_ROWS, 1)
+        pkg.dsp_load_partition(c, datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.dim)
+        with pytest.raises(pkg.DSPError) as e:
+            pkg.dsp_set_option(c, d.DSP_OPT_SPLIT_ROWS, 0)
+        assert e.value.status == d.DSP_ERR_STATE
+        pkg.dsp_set_option(c, d.DSP_OPT_RELABEL_MAP, 2)
+        pkg.dsp_reserve(c, 16, cfg.fanouts)
+        for opt in (d.DSP_OPT_RELABEL_MAP, d.DSP_OPT_EXCHANGE_CHANNELS):
+            with pytest.raises(pkg.DSPError) as e:
+                pkg.dsp_set_option(c, opt, 1)
+            assert e.value.status == d.DSP_ERR_STATE
+        pkg.dsp_set_option(c, d.DSP_OPT_LANE_ROUNDS, 4)      # tuning knobs stay settable
+        pkg.dsp_set_option(c, d.DSP_OPT_LOADER_ROWS, 16)
+    finally:
+        pkg.dsp_destroy(c)
