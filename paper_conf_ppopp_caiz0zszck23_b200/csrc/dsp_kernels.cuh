@@ -615,89 +615,111 @@ __device__ DSP_PHASE void phase_sample_biased(const int32_t *frontier, int F, in
 // tile + j*TEAM + t) so every load is a coalesced warp access; the in-block
 // prefix comes from warp ballots plus a table kept in shared memory across
 // the barrier, the flags in registers.
-constexpr int SCAN2_IPT = 8;
+constexpr int SCAN2_IPT = 8;     // stripes per group (registers of one pass over them)
+constexpr int SCAN2_GROUPS = 4;  // groups per block and round of k_csp_multi: up to 32 stripes of TEAM slots
 
 
 __device__ __forceinline__ unsigned long long pack2(uint32_t valid, uint32_t first) {
   return ((unsigned long long)first << 31) | valid;
 }
 
-template <int TEAM>
+template <int TEAM, int GROUPS = 1>
 struct Scan2Smem {
-  unsigned long long tab[SCAN2_IPT * (TEAM / 32)];  // exclusive prefix of (stripe j, warp w)
+  unsigned long long tab[GROUPS * SCAN2_IPT * (TEAM / 32)];  // exclusive prefix of (stripe, warp)
   unsigned long long red[2 * (TEAM / 32) + 2];
 };
 
 struct Scan2Regs {
-  uint32_t vbits, fbits;
+  uint32_t vbits, fbits;  // bit s: slot q0 + s * TEAM holds an edge / is a first occurrence
 };
 
-template <int TEAM>
+// A block's chunk [tile0, tile_end) of one round is processed as up to
+// GROUPS groups of SCAN2_IPT stripes (stripe s = slots tile0 + s * TEAM +
+// [0, TEAM)), so a layer of up to GROUPS * 8 * TEAM slots per block needs one
+// round (two grid barriers) instead of one round per 8 stripes.  The world-1
+// kernel keeps GROUPS = 1 (the bench step is bound by the gather there, and
+// its sampling warps finishing earlier only add DRAM contention: 0.1356 vs
+// 0.1345 ms/step over 5 alternating runs); k_csp_multi, whose ranks run on
+// fractions of the SMs, uses 4 (virtual P = 2 / 4 with 4 channels: 73.3 /
+// 76.4 vs 77.5 / 80.0 us per rank-batch).
+template <int TEAM, int GROUPS = 1>
 __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, uint32_t epoch, int64_t tile0,
                                             int64_t tile_end, Scan2Regs &R, unsigned long long *agg_slot,
-                                            Scan2Smem<TEAM> &sm) {
+                                            Scan2Smem<TEAM, GROUPS> &sm) {
+  constexpr int W = TEAM / 32;
   const uint32_t total = (uint32_t)tile_end;  // < 2^31 by the host's plan check
   const FastDiv fd = make_fastdiv((uint32_t)k);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  const uint32_t q0 = (uint32_t)tile0 + threadIdx.x;
-  // all loads first: counts + sampled ids, then the map words of the valid slots
-  int32_t c[SCAN2_IPT], u[SCAN2_IPT];
-#pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) {
-    const uint32_t q = q0 + j * TEAM;
-    c[j] = -1;
-    u[j] = 0;
-    if (q < total) {
-      const uint32_t i = fdiv(q, fd);
-      c[j] = ldw_i32(B.cnt + i) - (int32_t)(q - i * (uint32_t)k);  // > 0 iff slot q holds an edge
-      u[j] = ldw_i32(B.rows + q);  // garbage unless valid; dereferenced only then
-    }
-  }
-  unsigned long long w[SCAN2_IPT];
-#pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? map_get(B, u[j], epoch) : 0ull;
+  const int groups = (int)min((int64_t)GROUPS,
+                              max((int64_t)1, (tile_end - tile0 + (int64_t)TEAM * SCAN2_IPT - 1) / ((int64_t)TEAM * SCAN2_IPT)));
   R.vbits = R.fbits = 0;
+#pragma unroll 1
+  for (int g = 0; g < groups; ++g) {
+    const uint32_t q0 = (uint32_t)tile0 + (uint32_t)(g * SCAN2_IPT * TEAM) + threadIdx.x;
+    // all loads first: counts + sampled ids, then the map words of the valid slots
+    int32_t c[SCAN2_IPT], u[SCAN2_IPT];
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) {
-    const bool valid = c[j] > 0;
-    const bool first = valid && w[j] == mword(B, epoch, u[j], (uint32_t)F + q0 + j * TEAM);
-    // a valid slot that is not u's first occurrence keeps x (u's smallest order
-    // key: its dst index, or F + the slot of its first occurrence) as -1 - x
-    if (valid && !first) B.rows[q0 + j * TEAM] = -1 - (int32_t)mword_x(B, w[j]);
-    R.vbits |= (valid ? 1u : 0u) << j;
-    R.fbits |= (first ? 1u : 0u) << j;
-    const uint32_t bv = __ballot_sync(FULL_MASK, valid), bf = __ballot_sync(FULL_MASK, first);
-    if (lane == 0) sm.tab[j * (TEAM / 32) + wid] = pack2(__popc(bv), __popc(bf));
+    for (int j = 0; j < SCAN2_IPT; ++j) {
+      const uint32_t q = q0 + j * TEAM;
+      c[j] = -1;
+      u[j] = 0;
+      if (q < total) {
+        const uint32_t i = fdiv(q, fd);
+        c[j] = ldw_i32(B.cnt + i) - (int32_t)(q - i * (uint32_t)k);  // > 0 iff slot q holds an edge
+        u[j] = ldw_i32(B.rows + q);  // garbage unless valid; dereferenced only then
+      }
+    }
+    unsigned long long w[SCAN2_IPT];
+#pragma unroll
+    for (int j = 0; j < SCAN2_IPT; ++j) w[j] = c[j] > 0 ? map_get(B, u[j], epoch) : 0ull;
+#pragma unroll
+    for (int j = 0; j < SCAN2_IPT; ++j) {
+      const bool valid = c[j] > 0;
+      const bool first = valid && w[j] == mword(B, epoch, u[j], (uint32_t)F + q0 + j * TEAM);
+      // a valid slot that is not u's first occurrence keeps x (u's smallest order
+      // key: its dst index, or F + the slot of its first occurrence) as -1 - x
+      if (valid && !first) B.rows[q0 + j * TEAM] = -1 - (int32_t)mword_x(B, w[j]);
+      R.vbits |= (valid ? 1u : 0u) << (g * SCAN2_IPT + j);
+      R.fbits |= (first ? 1u : 0u) << (g * SCAN2_IPT + j);
+      const uint32_t bv = __ballot_sync(FULL_MASK, valid), bf = __ballot_sync(FULL_MASK, first);
+      if (lane == 0) sm.tab[(g * SCAN2_IPT + j) * W + wid] = pack2(__popc(bv), __popc(bf));
+    }
   }
   team_sync<TEAM>();
-  if (wid == 0) {  // exclusive scan of the (stripe, warp) counts, stripe-major
-    constexpr int PER = SCAN2_IPT * (TEAM / 32) / 32;
-    unsigned long long v[PER], run = 0;
+  if (wid == 0) {  // exclusive scan of the (stripe, warp) counts, stripe-major, group by group
+    constexpr int PER = SCAN2_IPT * W / 32;
+    unsigned long long carry = 0;
+#pragma unroll 1
+    for (int g = 0; g < groups; ++g) {
+      unsigned long long *tab = sm.tab + g * SCAN2_IPT * W;
+      unsigned long long v[PER], run = 0;
 #pragma unroll
-    for (int e = 0; e < PER; ++e) {
-      v[e] = sm.tab[lane * PER + e];
-      run += v[e];
-    }
-    unsigned long long incl = run;
+      for (int e = 0; e < PER; ++e) {
+        v[e] = tab[lane * PER + e];
+        run += v[e];
+      }
+      unsigned long long incl = run;
 #pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-      const unsigned long long y = __shfl_up_sync(FULL_MASK, incl, off);
-      if (lane >= off) incl += y;
-    }
-    unsigned long long p = incl - run;
+      for (int off = 1; off < 32; off <<= 1) {
+        const unsigned long long y = __shfl_up_sync(FULL_MASK, incl, off);
+        if (lane >= off) incl += y;
+      }
+      unsigned long long p = carry + incl - run;
 #pragma unroll
-    for (int e = 0; e < PER; ++e) {
-      sm.tab[lane * PER + e] = p;
-      p += v[e];
+      for (int e = 0; e < PER; ++e) {
+        tab[lane * PER + e] = p;
+        p += v[e];
+      }
+      carry += __shfl_sync(FULL_MASK, incl, 31);
     }
-    if (lane == 31) __stcg(agg_slot, incl);
+    if (lane == 0) __stcg(agg_slot, carry);
   }
   team_sync<TEAM>();
 }
 
 // prefix of block `blk` and the round total from the published aggregates
-template <int TEAM>
-__device__ __forceinline__ void scan2_prefix(const unsigned long long *agg, int nblk, int blk, Scan2Smem<TEAM> &sm,
+template <int TEAM, int GROUPS = 1>
+__device__ __forceinline__ void scan2_prefix(const unsigned long long *agg, int nblk, int blk, Scan2Smem<TEAM, GROUPS> &sm,
                                              unsigned long long *prefix, unsigned long long *round_total) {
   unsigned long long p = 0, t = 0;
   for (int b = threadIdx.x; b < nblk; b += TEAM) {
@@ -739,36 +761,44 @@ __device__ __forceinline__ void scan2_prefix(const unsigned long long *agg, int 
 // touched: a duplicate finds its nid through rows[x - F], a coalesced-slot
 // array, instead of a second random map access per edge.  The dst copy of
 // src_out is written by the sample phase.
-template <int TEAM>
+template <int TEAM, int GROUPS = 1>
 __device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, int64_t tile0, int64_t tile_end,
-                                            const Scan2Regs &R, unsigned long long base, const Scan2Smem<TEAM> &sm,
-                                            int32_t *indptr_out, int32_t *indices_out, int32_t *src_out) {
+                                            const Scan2Regs &R, unsigned long long base,
+                                            const Scan2Smem<TEAM, GROUPS> &sm, int32_t *indptr_out,
+                                            int32_t *indices_out, int32_t *src_out) {
+  constexpr int W = TEAM / 32;
   const uint32_t total = (uint32_t)tile_end;
   const FastDiv fd = make_fastdiv((uint32_t)k);
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint32_t lt = (1u << lane) - 1u;
-  const uint32_t q0 = (uint32_t)tile0 + threadIdx.x;
-  int32_t r[SCAN2_IPT];
+  const int groups = (int)min((int64_t)GROUPS,
+                              max((int64_t)1, (tile_end - tile0 + (int64_t)TEAM * SCAN2_IPT - 1) / ((int64_t)TEAM * SCAN2_IPT)));
+#pragma unroll 1
+  for (int g = 0; g < groups; ++g) {
+    const uint32_t q0 = (uint32_t)tile0 + (uint32_t)(g * SCAN2_IPT * TEAM) + threadIdx.x;
+    const uint32_t vb = R.vbits >> (g * SCAN2_IPT), fb = R.fbits >> (g * SCAN2_IPT);
+    int32_t r[SCAN2_IPT];
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) r[j] = ((R.vbits >> j) & 1u) ? ldw_i32(B.rows + q0 + j * TEAM) : 0;
+    for (int j = 0; j < SCAN2_IPT; ++j) r[j] = ((vb >> j) & 1u) ? ldw_i32(B.rows + q0 + j * TEAM) : 0;
 #pragma unroll
-  for (int j = 0; j < SCAN2_IPT; ++j) {
-    const uint32_t bv = __ballot_sync(FULL_MASK, (R.vbits >> j) & 1u);
-    const uint32_t bf = __ballot_sync(FULL_MASK, (R.fbits >> j) & 1u);
-    const uint32_t q = q0 + j * TEAM;
-    if (q < total) {
-      const unsigned long long b = base + sm.tab[j * (TEAM / 32) + wid];
-      const uint32_t e = (uint32_t)(b & 0x7fffffffull) + __popc(bv & lt);  // edge index of slot q (if valid)
-      const uint32_t i = fdiv(q, fd);
-      if (q == i * (uint32_t)k) indptr_out[i] = (int32_t)e;
-      if ((R.fbits >> j) & 1u) {
-        const uint32_t nid = (uint32_t)F + (uint32_t)((b >> 31) & 0x7fffffffull) + __popc(bf & lt);
-        src_out[nid] = r[j];
-        B.rows[q] = (int32_t)nid;
-        indices_out[e] = (int32_t)nid;
-      } else if ((R.vbits >> j) & 1u) {
-        const uint32_t x = (uint32_t)(-1 - r[j]);
-        if (x < (uint32_t)F) indices_out[e] = (int32_t)x;  // dst hit
+    for (int j = 0; j < SCAN2_IPT; ++j) {
+      const uint32_t bv = __ballot_sync(FULL_MASK, (vb >> j) & 1u);
+      const uint32_t bf = __ballot_sync(FULL_MASK, (fb >> j) & 1u);
+      const uint32_t q = q0 + j * TEAM;
+      if (q < total) {
+        const unsigned long long b = base + sm.tab[(g * SCAN2_IPT + j) * W + wid];
+        const uint32_t e = (uint32_t)(b & 0x7fffffffull) + __popc(bv & lt);  // edge index of slot q (if valid)
+        const uint32_t i = fdiv(q, fd);
+        if (q == i * (uint32_t)k) indptr_out[i] = (int32_t)e;
+        if ((fb >> j) & 1u) {
+          const uint32_t nid = (uint32_t)F + (uint32_t)((b >> 31) & 0x7fffffffull) + __popc(bf & lt);
+          src_out[nid] = r[j];
+          B.rows[q] = (int32_t)nid;
+          indices_out[e] = (int32_t)nid;
+        } else if ((vb >> j) & 1u) {
+          const uint32_t x = (uint32_t)(-1 - r[j]);
+          if (x < (uint32_t)F) indices_out[e] = (int32_t)x;  // dst hit
+        }
       }
     }
   }

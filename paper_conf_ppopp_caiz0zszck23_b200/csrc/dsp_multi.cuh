@@ -355,7 +355,7 @@ __device__ __forceinline__ void multi_unpermute(const MultiArgs &m, const int32_
 
 template <int TEAM, bool PIPE, bool BIASED>
 __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ MultiArgs m) {
-  __shared__ Scan2Smem<TEAM> sm;
+  __shared__ Scan2Smem<TEAM, SCAN2_GROUPS> sm;
   __shared__ uint32_t s_cnt[8], s_base[8], s_off[9];
   __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];
   extern __shared__ __align__(128) char ring_smem[];
@@ -460,7 +460,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ Mu
     grid_barrier<TEAM>(a.hdr, bar);
 
     // ---- D: relabel scan (as k_csp_persistent)
-    constexpr int64_t TILE = (int64_t)TEAM * SCAN2_IPT;
+    constexpr int64_t TILE = (int64_t)TEAM * SCAN2_IPT * SCAN2_GROUPS;
     const int64_t total = (int64_t)Fs * k;
     const int64_t rounds = total > 0 ? (total + (int64_t)nblk * TILE - 1) / ((int64_t)nblk * TILE) : 1;
     const int64_t per_round = (total + rounds - 1) / rounds;
@@ -471,11 +471,11 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_multi(const __grid_constant__ Mu
       const int64_t r0 = r * per_round, r1 = min(total, r0 + per_round);
       const int64_t tile0 = min(r1, r0 + (int64_t)blk * chunk), tile_end = min(r1, tile0 + chunk);
       unsigned long long *agg = a.agg + (r & 1) * MAX_PERSIST_BLOCKS;
-      scan2_pass1<TEAM>(Fs, k, a.buf[l & 1], epoch, tile0, tile_end, R, agg + blk, sm);
+      scan2_pass1<TEAM, SCAN2_GROUPS>(Fs, k, a.buf[l & 1], epoch, tile0, tile_end, R, agg + blk, sm);
       grid_barrier<TEAM>(a.hdr, bar);
       unsigned long long prefix, round_total;
-      scan2_prefix<TEAM>(agg, nblk, blk, sm, &prefix, &round_total);
-      scan2_pass2<TEAM>(Fs, k, a.buf[l & 1], tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
+      scan2_prefix<TEAM, SCAN2_GROUPS>(agg, nblk, blk, sm, &prefix, &round_total);
+      scan2_pass2<TEAM, SCAN2_GROUPS>(Fs, k, a.buf[l & 1], tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
                         a.out.indices[l], a.out.src_ids[l]);
       carry += round_total;
       if (r + 1 < rounds) grid_barrier<TEAM>(a.hdr, bar);
