@@ -584,10 +584,13 @@ def test_biased_virtual_ranks(pkg, tiny, tiny_weights, P):
     grp.close()
 
 
-def _long_row_graph():
+def _long_row_graph(heavy=False):
     """30k nodes, rows of degree <= 40 plus hubs of degree 300 / 1000 / 5000
     (chunk-sum path, 256 < d <= 8192), 9000 / 20000 (very long rows), and a hub
-    whose 5000 weights are all zero but 3 (every positive one taken, no draw)."""
+    whose 5000 weights are all zero but 3 (every positive one taken, no draw).
+    Weights below 714 keep every running weight of a row of <= 256 positions
+    under 2^32 (the 32-bit rounds of the register path); heavy weights (up to
+    65535) push rows of more than 32 positions past it (the 64-bit rounds)."""
     rng = np.random.default_rng(31)
     N = 30000
     degs = rng.integers(0, 41, size=N)
@@ -603,17 +606,25 @@ def _long_row_graph():
     ip[1:] = np.cumsum([len(r) for r in rows])
     ix = np.concatenate(rows).astype(np.int32)
     w = (rng.integers(0, 5000, size=len(ix)) / 7.0).astype(np.float32)
+    if heavy:
+        w = (w * 91.75).astype(np.float32)
     w[rng.random(len(ix)) < 0.1] = 0.0
     w[ip[5]:ip[6]] = 0.0
     w[ip[5] + np.array([7, 2000, 4999])] = 3.5
     return N, ip, ix, w
 
 
-def test_biased_long_rows(pkg):
-    """Biased sampling on every row-length path of the warp sampler (registers,
-    chunk sums, very long rows, <= k positive weights) at P = 1 and at virtual
-    P = 2 (the owner-side sampler of the multi-rank kernel)."""
-    N, ip, ix, w = _long_row_graph()
+@pytest.mark.parametrize("heavy", [False, True])
+def test_biased_long_rows(pkg, heavy):
+    """Biased sampling on every row-length path of the warp sampler (one
+    position per lane, registers with 32- or 64-bit running weights, chunk
+    sums, very long rows, <= k positive weights) at P = 1 and at virtual P = 2
+    (the owner-side sampler of the multi-rank kernel)."""
+    N, ip, ix, w = _long_row_graph(heavy)
+    if heavy:
+        wf = np.floor(w.astype(np.float64) * 65536)
+        big = [v for v in range(6, N) if 32 < ip[v + 1] - ip[v] and wf[ip[v]:ip[v + 1]].sum() >= 2 ** 32]
+        assert len(big) > 1000
     feats = datagen.features(0, N, 4)
     fan = (15, 10)
     seeds = np.array([0, 1, 2, 3, 4, 5, 11, 29999, 15000], np.int32)
