@@ -328,16 +328,30 @@ __device__ __forceinline__ unsigned long long warp_incl_scan_u64(unsigned long l
 // without replacement: k times, r = mulhi(Philox{t, v, l, "DSPB"}, W) with W
 // the total weight of the positions not yet picked, and the pick is the first
 // position (row order) whose running weight exceeds r.  When at most k
-// positions have a positive weight they are all taken, no draw.  Lane t < cnt
-// returns the t-th position in ascending row order in *pos.  Warp-uniform.
+// positions have a positive weight they are all taken, no draw.  Lanes t <
+// cnt return a position in *pos and its output slot in *slot (the rank of the
+// position among the cnt returned, so slot order is row order).  Warp-uniform.
 //
-// Rows of up to 32 positions hold one weight per lane and a round's crossing
-// lane is the pick.  Rows of up to 32*BSEG positions keep their weights in registers, lane l
-// holding the contiguous segment [l*S, (l+1)*S): a round is one warp sum, one
-// warp scan of the lane totals and a scan inside the crossing lane's segment,
-// and the pick is removed by zeroing one register.  Longer rows re-read the
-// weights and test membership against the picks so far.
-constexpr int BSEG = 8;
+// Draw words: lane (wbase + t) of `wordg` holds the word of draw t of this
+// node (callers compute the words of several nodes in one Philox pass:
+// biased_group_word).
+//
+// Rows of up to 256 positions whose weights are all <= 2^24 (the common
+// case; every running weight then fits 32 bits) are sampled by lane groups,
+// 32 / G nodes per warp at once (biased_group_pass).  This warp-wide sampler
+// takes the rest: the row is read in 128-byte-aligned chunks of 32 weights
+// (chunk c, lane l: weight index A + 32c + l, A = the row start rounded down
+// to 32; slots outside the row hold 0), one line per coalesced load.  Rows of
+// up to 32 * HSEG chunks keep the chunk sums in registers (lane l: chunks
+// 32j + l) with their running weights (row order) of the positions not yet
+// picked, 64-bit: a round counts the chunks whose running weight is <= r (one
+// REDUX over the lanes' counts: running weights are non-decreasing and a
+// picked position's interval is empty), which is the crossing chunk; it is
+// re-read (earlier picks in it masked out) and scanned; removing the pick
+// subtracts its weight from the running weights behind it.  The pick's rank
+// among the earlier picks is kept on the fly (no sort).  Longer rows re-read
+// the row every round.
+constexpr int HSEG = 4;   // chunk sums per lane of the chunk-sum path
 
 // Lanes t < k hold distinct picks; lane r returns the pick of rank r (ascending):
 // each lane ranks its own pick with k shuffles, then one ballot + shuffle per
@@ -360,217 +374,159 @@ __device__ __forceinline__ unsigned long long biased_word(uint2 key, int t, int3
   return ((unsigned long long)x.y << 32) | x.x;
 }
 
-// The k rounds of the register path (below): lane t's draw word is myword of
-// lane t, incl the inclusive scan of the lane totals tot, W their sum; the pick
-// of round t is left in lane t.  (The same rounds in 32-bit arithmetic when
-// W < 2^32, as a second copy of this loop, measured 8 % slower: 0.331 vs 0.308
-// ms/step, the larger kernel.)
-__device__ __forceinline__ uint32_t biased_reg_rounds(uint32_t (&reg)[BSEG], unsigned long long myword,
-                                                      unsigned long long incl, unsigned long long tot,
-                                                      unsigned long long W, int k, int S) {
+// Draw words of up to G = 32 / k nodes in one Philox pass: lane t (< G * k)
+// computes draw t % k of the node held (as vl) by lane j0 + t / k of the
+// warp.  tq = lane / k and tr = lane % k are precomputed by the caller.
+__device__ __forceinline__ unsigned long long biased_group_word(uint2 key, int layer, int32_t vl, int j0, int G,
+                                                                int tq, int tr) {
+  const int src = min(j0 + tq, 31);
+  const int32_t v = __shfl_sync(FULL_MASK, vl, src);
+  return tq < G ? biased_word(key, tr, v, layer) : 0ull;
+}
+
+// Round t picked position p (warp-uniform): lane t keeps it, and every pick
+// so far keeps its rank among the picks.
+__device__ __forceinline__ void biased_track(int t, uint32_t p, uint32_t &pick, int &rank) {
+  const int lane = threadIdx.x & 31;
+  const uint32_t below = __ballot_sync(FULL_MASK, lane < t && pick < p);
+  if (lane < t && pick > p) ++rank;
+  if (lane == t) {
+    pick = p;
+    rank = __popc(below);
+  }
+}
+
+// Every positive-weight position of the row (at most k of them), in row
+// order: lane t gets the t-th one.  m(j) is the ballot of chunk j.
+template <typename Mask>
+__device__ __forceinline__ uint32_t biased_all_positive(int nch, int off, Mask m) {
+  const int lane = threadIdx.x & 31;
+  int base = 0;
+  uint32_t mine = 0xffffffffu;
+  for (int j = 0; j < nch; ++j) {
+    const uint32_t b = m(j);
+    const int want = lane - base;
+    if (want >= 0 && want < __popc(b)) mine = (uint32_t)(32 * j - off) + __fns(b, 0, want + 1);
+    base += __popc(b);
+  }
+  return mine;
+}
+
+// Sum over the warp of 32-bit values as a 64-bit total (two 32-bit REDUX).
+__device__ __forceinline__ unsigned long long warp_sum_w(uint32_t x) {
+  return (unsigned long long)__reduce_add_sync(FULL_MASK, x & 0xffffu) +
+         ((unsigned long long)__reduce_add_sync(FULL_MASK, x >> 16) << 16);
+}
+
+// Rows of up to 32 * HSEG aligned chunks: lane l holds the sum of chunk
+// 32j + l in cs[j] and the chunk's running weight (inclusive, row order) in
+// CP[j], 64-bit.  A round finds the crossing chunk by counting as above,
+// re-reads it (earlier picks in it masked out) and scans it.
+__device__ __forceinline__ int biased_chunks(const uint32_t *__restrict__ al, int off, int d, int nch, int k,
+                                             unsigned long long wordg, int wbase, uint32_t *pos, int *slot) {
   using U = unsigned long long;
   const int lane = threadIdx.x & 31;
-  uint32_t pick = 0xffffffffu;
-  for (int t = 0; t < k; ++t) {
-    const U r = __umul64hi(__shfl_sync(FULL_MASK, myword, t), W);
-    const uint32_t cross = __ballot_sync(FULL_MASK, incl > r);
-    const int L = __ffs(cross) - 1;
-    uint32_t found = 0, wrem = 0;
-    if (lane == L) {
-      U acc = incl - tot;
-      bool done = false;
+  U cs[HSEG], CP[HSEG];
+  int npos = 0;
 #pragma unroll
-      for (int j = 0; j < BSEG; ++j) {
-        if (!done && acc + reg[j] > r) {
-          found = (uint32_t)(lane * S + j);
-          wrem = reg[j];
-          reg[j] = 0u;  // remove the pick
-          done = true;
-        }
-        acc += reg[j];
+  for (int j = 0; j < HSEG; ++j) {
+    cs[j] = 0;
+    if (32 * j < nch) {
+      const int n = min(32, nch - 32 * j);
+#pragma unroll 4
+      for (int c = 0; c < n; ++c) {
+        const int q = 32 * (32 * j + c) + lane;
+        const uint32_t x = (q >= off && q < off + d) ? __ldg(al + q) : 0u;
+        npos += __popc(__ballot_sync(FULL_MASK, x > 0u));
+        const U s = warp_sum_w(x);
+        if (lane == c) cs[j] = s;
       }
-      tot -= wrem;
     }
-    found = __shfl_sync(FULL_MASK, found, L);
-    wrem = __shfl_sync(FULL_MASK, wrem, L);
-    if (lane >= L) incl -= wrem;
-    W -= wrem;
-    if (lane == t) pick = found;
   }
-  return pick;
+  if (npos <= k) {
+    *pos = biased_all_positive(nch, off, [&](int j) {
+      const int q = 32 * j + lane;
+      return __ballot_sync(FULL_MASK, q >= off && q < off + d && __ldg(al + q) > 0u);
+    });
+    return npos;
+  }
+  U base = 0;
+#pragma unroll
+  for (int j = 0; j < HSEG; ++j) {
+    U s = cs[j];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const U y = __shfl_up_sync(FULL_MASK, s, o);
+      if (lane >= o) s += y;
+    }
+    CP[j] = base + s;
+    base = __shfl_sync(FULL_MASK, CP[j], 31);
+  }
+  U W = base;
+  uint32_t pick = 0xffffffffu;
+  int rank = 0;
+  for (int t = 0; t < k; ++t) {
+    const U r = __umul64hi(__shfl_sync(FULL_MASK, wordg, wbase + t), W);
+    uint32_t c = 0;
+#pragma unroll
+    for (int j = 0; j < HSEG; ++j) c += CP[j] <= r ? 1u : 0u;
+    const int cst = (int)__reduce_add_sync(FULL_MASK, c);  // the crossing chunk
+    const int js = cst >> 5, Lc = cst & 31;
+    U csel = cs[0], psel = CP[0];
+#pragma unroll
+    for (int j = 1; j < HSEG; ++j)
+      if (j == js) {
+        csel = cs[j];
+        psel = CP[j];
+      }
+    const U before = __shfl_sync(FULL_MASK, psel, Lc) - __shfl_sync(FULL_MASK, csel, Lc);
+    const int q = 32 * cst + lane;
+    uint32_t x = (q >= off && q < off + d) ? __ldg(al + q) : 0u;
+    // earlier picks inside this chunk (usually none)
+    uint32_t M = __ballot_sync(FULL_MASK, lane < t && ((pick + (uint32_t)off) >> 5) == (uint32_t)cst);
+    uint32_t taken = 0;
+    while (M) {
+      const int s = __ffs(M) - 1;
+      M &= M - 1;
+      taken |= 1u << ((__shfl_sync(FULL_MASK, pick, s) + (uint32_t)off) & 31u);
+    }
+    if ((taken >> lane) & 1u) x = 0u;
+    U incl = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const U y = __shfl_up_sync(FULL_MASK, incl, o);
+      if (lane >= o) incl += y;
+    }
+    const int Lp = __ffs(__ballot_sync(FULL_MASK, before + incl > r)) - 1;
+    const uint32_t ap = __shfl_sync(FULL_MASK, x, Lp);
+    if (lane == Lc) {
+#pragma unroll
+      for (int j = 0; j < HSEG; ++j)
+        if (j == js) cs[j] -= ap;
+    }
+    const int jt = js + (lane < Lc ? 1 : 0);
+#pragma unroll
+    for (int j = 0; j < HSEG; ++j) CP[j] -= j >= jt ? (U)ap : 0ull;
+    W -= ap;
+    biased_track(t, (uint32_t)(32 * cst + Lp - off), pick, rank);
+  }
+  *pos = pick;
+  *slot = rank;
+  return k;
 }
 
 __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t row_start, int64_t deg, int k,
                                                   int layer, uint2 key, const uint32_t *__restrict__ w,
-                                                  uint32_t *pos) {
+                                                  unsigned long long wordg, int wbase, uint32_t *pos, int *slot) {
   const int lane = threadIdx.x & 31;
+  *slot = lane;
   if (!ok) return 0;
-  const uint32_t *a = w + row_start;
   const int d = (int)deg;
-  if (d <= 32) {
-    // ------------------------------------------ one weight per lane (lane = position)
-    // the crossing lane of a round is the pick itself (no in-lane scan), and the
-    // picks as a lane mask are already in row order
-    const uint32_t x = lane < d ? __ldg(a + lane) : 0u;
-    const uint32_t posm = __ballot_sync(FULL_MASK, x > 0u);
-    const int npos = __popc(posm);
-    if (npos <= k) {
-      *pos = lane < npos ? (uint32_t)__fns(posm, 0, lane + 1) : 0xffffffffu;
-      return npos;
-    }
-    const unsigned long long myword = lane < k ? biased_word(key, lane, v, layer) : 0ull;  // all draws at once
-    unsigned long long incl = warp_incl_scan_u64(x);
-    unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
-    uint32_t pm = 0;
-    for (int t = 0; t < k; ++t) {
-      const unsigned long long r = __umul64hi(__shfl_sync(FULL_MASK, myword, t), W);
-      const int L = __ffs(__ballot_sync(FULL_MASK, incl > r)) - 1;
-      const uint32_t wrem = __shfl_sync(FULL_MASK, x, L);
-      if (lane >= L) incl -= wrem;  // L's interval becomes empty
-      W -= wrem;
-      pm |= 1u << L;
-    }
-    *pos = lane < k ? (uint32_t)__fns(pm, 0, lane + 1) : 0xffffffffu;
-    return k;
-  }
-  if (d <= 32 * BSEG) {
-    // ------------------------------------------------ weights in registers
-    const int S = (d + 31) >> 5;
-    uint32_t reg[BSEG];
-    int mypos = 0;
-#pragma unroll
-    for (int j = 0; j < BSEG; ++j) {
-      const int p = lane * S + j;
-      reg[j] = (j < S && p < d) ? __ldg(a + p) : 0u;
-      mypos += reg[j] > 0u ? 1 : 0;
-    }
-    int npos = mypos;
-#pragma unroll
-    for (int off = 16; off > 0; off >>= 1) npos += __shfl_xor_sync(FULL_MASK, npos, off);
-    if (npos <= k) {  // every positive-weight position, in row order
-      int excl = mypos;
-#pragma unroll
-      for (int off = 1; off < 32; off <<= 1) {
-        const int y = __shfl_up_sync(FULL_MASK, excl, off);
-        if (lane >= off) excl += y;
-      }
-      excl -= mypos;
-      uint32_t mine = 0xffffffffu;
-      // lane t needs the position of rank t: owner lanes hand it over one rank at a time
-      for (int t = 0; t < npos; ++t) {
-        const bool own = t >= excl && t < excl + mypos;
-        uint32_t cand = 0;
-        if (own) {
-          int r = excl;
-#pragma unroll
-          for (int j = 0; j < BSEG; ++j)
-            if (reg[j] > 0u) {
-              if (r == t) cand = (uint32_t)(lane * S + j);
-              ++r;
-            }
-        }
-        const uint32_t b = __ballot_sync(FULL_MASK, own);
-        const uint32_t got = __shfl_sync(FULL_MASK, cand, __ffs(b) - 1);
-        if (lane == t) mine = got;
-      }
-      *pos = mine;
-      return npos;
-    }
-    uint32_t pick = 0xffffffffu;
-    const unsigned long long myword = lane < k ? biased_word(key, lane, v, layer) : 0ull;  // all draws at once
-    // lane totals, their inclusive scan and the remaining weight W, scanned once and
-    // then updated in place: removing weight w at lane L lowers incl of lanes >= L by w
-    unsigned long long tot = 0;
-#pragma unroll
-    for (int j = 0; j < BSEG; ++j) tot += reg[j];
-    const unsigned long long incl = warp_incl_scan_u64(tot);
-    const unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
-    pick = biased_reg_rounds(reg, myword, incl, tot, W, k, S);
-    *pos = biased_sort_picks(pick, k);
-    return k;
-  }
-  // ------------------------------------------- long rows: chunk sums in registers
-  // chunk c = positions [32c, 32c+32); lane l holds the sums of chunks
-  // [l*T, (l+1)*T).  A round finds the crossing chunk from the chunk sums, then
-  // the crossing position inside it (picks already in that chunk masked out).
-  if (d <= 32 * 32 * BSEG) {
-    const int nch = (d + 31) >> 5, T = (nch + 31) >> 5;
-    unsigned long long cs[BSEG];
-    int npos = 0;
-#pragma unroll
-    for (int j = 0; j < BSEG; ++j) cs[j] = 0;
-    for (int c = 0; c < nch; ++c) {
-      const int p = c * 32 + lane;
-      const uint32_t x = p < d ? __ldg(a + p) : 0u;
-      npos += __popc(__ballot_sync(FULL_MASK, x > 0u));
-      const unsigned long long sum = warp_sum_u64(x);
-      if (lane == c / T) {
-#pragma unroll
-        for (int j = 0; j < BSEG; ++j)
-          if (j == c - lane * T) cs[j] = sum;
-      }
-    }
-    if (npos <= k) {
-      int base = 0;
-      uint32_t mine = 0xffffffffu;
-      for (int c0 = 0; c0 < d; c0 += 32) {
-        const bool f = c0 + lane < d && a[c0 + lane] > 0u;
-        const uint32_t b = __ballot_sync(FULL_MASK, f);
-        const int want = lane - base;
-        if (want >= 0 && want < __popc(b)) mine = c0 + (__fns(b, 0, want + 1));
-        base += __popc(b);
-      }
-      *pos = mine;
-      return npos;
-    }
-    uint32_t pick = 0xffffffffu;
-    const unsigned long long myword = lane < k ? biased_word(key, lane, v, layer) : 0ull;  // all draws at once
-    unsigned long long tot = 0;  // scanned once, then updated in place (as above)
-#pragma unroll
-    for (int j = 0; j < BSEG; ++j) tot += cs[j];
-    unsigned long long incl = warp_incl_scan_u64(tot);
-    unsigned long long W = __shfl_sync(FULL_MASK, incl, 31);
-    for (int t = 0; t < k; ++t) {
-      const unsigned long long r = __umul64hi(__shfl_sync(FULL_MASK, myword, t), W);
-      const int L = __ffs(__ballot_sync(FULL_MASK, incl > r)) - 1;
-      int cstar = 0;
-      unsigned long long before = 0;  // weight of the chunks before the crossing one
-      if (lane == L) {
-        unsigned long long acc = incl - tot;
-        bool done = false;
-#pragma unroll
-        for (int j = 0; j < BSEG; ++j) {
-          if (!done && acc + cs[j] > r) {
-            cstar = lane * T + j;
-            before = acc;
-            done = true;
-          }
-          acc += cs[j];
-        }
-      }
-      cstar = __shfl_sync(FULL_MASK, cstar, L);
-      before = __shfl_sync(FULL_MASK, before, L);
-      const int p = cstar * 32 + lane;
-      bool taken = p >= d;
-      for (int j = 0; j < t; ++j) taken |= __shfl_sync(FULL_MASK, pick, j) == (uint32_t)p;
-      const unsigned long long val = taken ? 0ull : (unsigned long long)__ldg(a + min(p, d - 1));
-      const unsigned long long pin = warp_incl_scan_u64(val);
-      const int P2 = __ffs(__ballot_sync(FULL_MASK, before + pin > r)) - 1;
-      const uint32_t found = (uint32_t)(cstar * 32 + P2);
-      const unsigned long long wfound = __shfl_sync(FULL_MASK, val, P2);
-      if (lane == L) {
-#pragma unroll
-        for (int j = 0; j < BSEG; ++j)
-          if (j == cstar - lane * T) cs[j] -= wfound;  // remove the pick
-        tot -= wfound;
-      }
-      if (lane >= L) incl -= wfound;
-      W -= wfound;
-      if (lane == t) pick = found;
-    }
-    *pos = biased_sort_picks(pick, k);
-    return k;
-  }
+  const int off = (int)(row_start & 31);
+  const uint32_t *al = w + (row_start - off);  // 128-byte aligned
+  const int nch = (off + d + 31) >> 5;
+  if (nch <= 32 * HSEG) return biased_chunks(al, off, d, nch, k, wordg, wbase, pos, slot);
+  const uint32_t *a = w + row_start;
   // ---------------------------------------------------------- very long rows
   int npos = 0;
   for (int c0 = 0; c0 < d; c0 += 32) npos += __popc(__ballot_sync(FULL_MASK, c0 + lane < d && a[c0 + lane] > 0u));
@@ -597,7 +553,7 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
       if (!taken) part += a[p];
     }
     const unsigned long long W = warp_sum_u64(part);
-    const unsigned long long r = __umul64hi(biased_word(key, t, v, layer), W);
+    const unsigned long long r = __umul64hi(__shfl_sync(FULL_MASK, wordg, wbase + t), W);
     unsigned long long acc = 0;
     uint32_t found = 0xffffffffu;
     for (int c0 = 0; c0 < d && found == 0xffffffffu; c0 += 32) {
@@ -614,6 +570,169 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
   }
   *pos = biased_sort_picks(pick, k);
   return k;
+}
+
+// ------------------------------------------------ biased sampling by lane groups
+// A group of G lanes samples one node whose row has d <= 8G positions and
+// whose weights are all <= 2^24 (so the row's total, <= 256 * 2^24, fits 32
+// bits unless it is exactly 2^32, which is detected), with k <= G: lane g
+// holds positions [8g, 8g + 8) in registers and their running weights (row
+// order, of the positions not yet picked) P[i].  The successive-sampling
+// round of sample_node_biased then costs one group reduction: the pick p is
+// the number of positions whose running weight is <= r, its weight comes
+// from the lane holding it, and the running weights behind it drop by that
+// weight.  32 / G nodes per warp at once, every collective over the whole
+// warp with width G, the k rounds uniform over the warp (k is the layer's).
+// Lane t < k of a group draws word t.  Out receives the results:
+//   Out::Ctx ctx(int jn)                      (all lanes; jn = claim-local node)
+//   void node(const Ctx &, int32_t v, bool ok, int cnt)   (one lane per node)
+//   void edge(const Ctx &, int slot, int32_t u)           (one lane per edge)
+// Returns the claim-local nodes of cmask that need the warp-wide sampler
+// (a weight above 2^24): their results are not written.
+constexpr uint32_t BGROUP_WMAX = 1u << 24;
+
+template <int G>
+__device__ __forceinline__ uint32_t group_sum(uint32_t x) {
+#pragma unroll
+  for (int o = G / 2; o > 0; o >>= 1) x += __shfl_xor_sync(FULL_MASK, x, o, G);
+  return x;
+}
+
+template <int G, class Out>
+__device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl, bool okl, int64_t sl, int dl, int k,
+                                                      int layer, uint2 key, const uint32_t *__restrict__ w,
+                                                      const int32_t *__restrict__ indices, const Out &out) {
+  constexpr int NPW = 32 / G;
+  const int lane = threadIdx.x & 31, grp = lane / G, g = lane & (G - 1);
+  uint32_t redo = 0;
+  while (cmask) {
+    int jn = -1;
+#pragma unroll
+    for (int q = 0; q < NPW; ++q) {
+      if (cmask) {
+        if (q == grp) jn = __ffs(cmask) - 1;
+        cmask &= cmask - 1;
+      }
+    }
+    const bool act = jn >= 0;
+    const int src = act ? jn : 0;
+    const int32_t v = __shfl_sync(FULL_MASK, vl, src);
+    const bool ok = __shfl_sync(FULL_MASK, okl, src) && act;
+    const int64_t s = __shfl_sync(FULL_MASK, sl, src);
+    const int dsh = __shfl_sync(FULL_MASK, dl, src);
+    const int d = act && ok ? dsh : 0;
+    const typename Out::Ctx c = out.ctx(src);
+    const unsigned long long word = (g < k && d > 0) ? biased_word(key, g, v, layer) : 0ull;
+    uint32_t x[8], P[8];
+    bool heavy = false;
+    uint32_t np = 0, T = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int p = 8 * g + i;
+      x[i] = p < d ? __ldg(w + s + p) : 0u;
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      heavy |= x[i] > BGROUP_WMAX;
+      np += x[i] > 0u ? 1u : 0u;
+      T += x[i];
+      P[i] = T;
+    }
+    // group scans: exclusive prefix of the lane totals and of the positive counts
+    uint32_t incl = T, ipos = np;
+#pragma unroll
+    for (int o = 1; o < G; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL_MASK, incl, o, G), z = __shfl_up_sync(FULL_MASK, ipos, o, G);
+      if (g >= o) {
+        incl += y;
+        ipos += z;
+      }
+    }
+    uint32_t W = __shfl_sync(FULL_MASK, incl, G - 1, G);
+    const uint32_t npos = __shfl_sync(FULL_MASK, ipos, G - 1, G);
+    const uint32_t hb = __ballot_sync(FULL_MASK, heavy);
+    heavy = ((G == 32 ? hb : (hb >> (grp * G)) & ((1u << G) - 1u)) != 0u) || (W == 0u && npos > 0u);
+#pragma unroll
+    for (int i = 0; i < 8; ++i) P[i] += incl - T;
+    const bool allpos = npos <= (uint32_t)k;
+    uint32_t pick = 0xffffffffu;
+    int rank = 0;
+    for (int t = 0; t < k; ++t) {
+      const unsigned long long wt = __shfl_sync(FULL_MASK, word, t, G);
+      // mulhi(word, W) for W < 2^32 (as sample_node_biased's rounds)
+      const uint32_t r = (uint32_t)(((unsigned long long)(uint32_t)(wt >> 32) * W + __umulhi((uint32_t)wt, W)) >> 32);
+      uint32_t cnt = 0;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) cnt += P[i] <= r ? 1u : 0u;
+      const uint32_t p = group_sum<G>(cnt);
+      const int io = (int)(p & 7u);
+      uint32_t xs = x[0];
+#pragma unroll
+      for (int i = 1; i < 8; ++i) xs = io == i ? x[i] : xs;
+      const uint32_t ap = __shfl_sync(FULL_MASK, xs, (int)(p >> 3), G);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) P[i] -= (uint32_t)(8 * g + i) >= p ? ap : 0u;
+      W -= ap;
+      const uint32_t below = __ballot_sync(FULL_MASK, g < t && pick < p);
+      if (g < t && pick > p) ++rank;
+      if (g == t) {
+        pick = p;
+        rank = __popc(G == 32 ? below : (below >> (grp * G)) & ((1u << G) - 1u));
+      }
+    }
+    if (act && !heavy) {
+      const int cnt = allpos ? (int)npos : k;
+      if (g == 0) out.node(c, v, ok, cnt);
+      if (allpos) {  // every positive-weight position, in row order
+        uint32_t sl2 = ipos - np;
+#pragma unroll
+        for (int i = 0; i < 8; ++i)
+          if (x[i] > 0u) out.edge(c, (int)sl2++, __ldg(indices + s + 8 * g + i));
+      } else if (g < k) {
+        out.edge(c, rank, __ldg(indices + s + pick));
+      }
+    }
+    redo |= __reduce_or_sync(FULL_MASK, (act && heavy && g == 0) ? 1u << jn : 0u);
+  }
+  return redo;
+}
+
+// The G of a node's lane group (8, 16 or 32: d <= 8G and k <= G), or 0 for
+// the warp-wide sampler (d > 256).
+__device__ __forceinline__ int biased_group_of(int64_t d, int k) {
+  const int gd = d <= 64 ? 8 : d <= 128 ? 16 : d <= 256 ? 32 : 0;
+  const int gk = k <= 8 ? 8 : k <= 16 ? 16 : 32;
+  return gd == 0 ? 0 : max(gd, gk);
+}
+
+// One claim of nn <= 32 nodes (lane j < nn holds node j's id vl, okl, row
+// start sl and degree dl): the grouped passes, then the warp-wide sampler for
+// long or heavy rows, node by node.
+template <class Out>
+__device__ __forceinline__ void biased_claim(int nn, int32_t vl, bool okl, int64_t sl, int64_t dl, int k, int layer,
+                                             uint2 key, const uint32_t *__restrict__ w,
+                                             const int32_t *__restrict__ indices, const Out &out) {
+  const int lane = threadIdx.x & 31;
+  const int gl = lane < nn ? (okl ? biased_group_of(dl, k) : 8) : -1;
+  const int dg = (int)min(dl, (int64_t)256);
+  uint32_t redo = biased_group_pass<8>(__ballot_sync(FULL_MASK, gl == 8), vl, okl, sl, dg, k, layer, key, w, indices, out);
+  redo |= biased_group_pass<16>(__ballot_sync(FULL_MASK, gl == 16), vl, okl, sl, dg, k, layer, key, w, indices, out);
+  redo |= biased_group_pass<32>(__ballot_sync(FULL_MASK, gl == 32), vl, okl, sl, dg, k, layer, key, w, indices, out);
+  uint32_t rest = redo | __ballot_sync(FULL_MASK, gl == 0);
+  while (rest) {
+    const int j = __ffs(rest) - 1;
+    rest &= rest - 1;
+    const int32_t v = __shfl_sync(FULL_MASK, vl, j);
+    const bool ok = __shfl_sync(FULL_MASK, okl, j);
+    const int64_t s = __shfl_sync(FULL_MASK, sl, j), d = __shfl_sync(FULL_MASK, dl, j);
+    const typename Out::Ctx c = out.ctx(j);
+    const unsigned long long word = lane < k ? biased_word(key, lane, v, layer) : 0ull;
+    uint32_t pos;
+    int slot;
+    const int cnt = sample_node_biased(ok, v, s, d, k, layer, key, w, word, 0, &pos, &slot);
+    if (lane == 0) out.node(c, v, ok, cnt);
+    if (lane < cnt) out.edge(c, slot, __ldg(indices + s + pos));
+  }
 }
 
 }  // namespace dsp

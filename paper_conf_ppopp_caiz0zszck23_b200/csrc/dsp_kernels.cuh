@@ -109,6 +109,7 @@ struct WsHeader {
   unsigned long long t[24];   // %globaltimer at kernel start and when block 0 leaves each grid barrier
   unsigned long long ta[24];  // %globaltimer when block 0 arrives at each grid barrier
   unsigned long long dbg[32]; // debug stamps (DSP_DEBUG_STAMPS builds only)
+  uint32_t scursor[8];        // biased sampling: next frontier node to claim, per layer
 };
 
 // One parity (layer % 2) of the workspace.
@@ -550,59 +551,61 @@ __device__ DSP_PHASE void phase_sample_tpn(const int32_t *frontier, int F, int l
   }
 }
 
-// Biased sampling: one warp per node, sample_node_biased; the
-// sampled neighbours come out in ascending row order (slot = lane).
+// Biased sampling, world 1: warps claim runs of consecutive frontier
+// nodes from a per-layer cursor (row lengths of the frontier span three
+// orders of magnitude, so a static share leaves warps idle at the grid
+// barrier); a claim is about a quarter of a warp's even share, at most 32
+// nodes.  The ids and row extents of a claim are loaded at once (one per
+// lane), then biased_claim samples them: lane groups for rows of <= 256
+// positions, the warp-wide sampler for longer ones.
+struct BiasedOutW1 {
+  const LayerBufs &B;
+  int g0, k, F, layer;
+  uint32_t epoch;
+  int32_t *src_out;
+  int *err;
+  struct Ctx {
+    int i;
+  };
+  __device__ __forceinline__ Ctx ctx(int jn) const { return Ctx{g0 + jn}; }
+  __device__ __forceinline__ void node(const Ctx &c, int32_t v, bool ok, int cnt) const {
+    B.cnt[c.i] = cnt;
+    if (src_out) src_out[c.i] = v;
+    if (ok)
+      mark_dst(B, v, c.i, F, layer, epoch, err);
+    else
+      latch(err, E_RANGE);
+  }
+  __device__ __forceinline__ void edge(const Ctx &c, int slot, int32_t u) const {
+    const uint32_t q = (uint32_t)c.i * (uint32_t)k + (uint32_t)slot;
+    B.rows[q] = u;
+    mark(B, u, epoch, (uint32_t)F + q);
+  }
+};
+
 template <int TEAM = PNT>
 __device__ DSP_PHASE void phase_sample_biased(const int32_t *frontier, int F, int layer, int k, uint2 key,
                                                     const int64_t *__restrict__ indptr,
                                                     const int32_t *__restrict__ indices,
                                                     const uint32_t *__restrict__ weights, int64_t lo,
                                                     int64_t n_local, const LayerBufs &B, uint32_t epoch,
-                                                    int32_t *src_out, int *err) {
+                                                    int32_t *src_out, int *err, uint32_t *cursor) {
   const int lane = threadIdx.x & 31;
-  const Span sp = block_span<TEAM>(F);
-  const int64_t b0 = sp.first - threadIdx.x;
-  const int wib = threadIdx.x >> 5, wpb = TEAM >> 5;
-  // The warp's next 32 nodes (its strided share) have their ids and row extents
-  // loaded at once, one per lane, then are sampled one after the other: one
-  // dependent DRAM round trip per 32 nodes instead of one per node.
-  for (int64_t g0 = b0 + wib; g0 < sp.end; g0 += (int64_t)wpb * 32) {
-    const int64_t il = g0 + (int64_t)lane * wpb;
-    const int32_t vl = il < sp.end ? ldw_i32(frontier + il) : -1;
+  const int nwarps = (int)gridDim.x * (TEAM >> 5);
+  const int csz = max(1, min(32, F / (4 * nwarps)));
+  while (true) {
+    int g0 = 0;
+    if (lane == 0) g0 = (int)atomicAdd(cursor, (uint32_t)csz);
+    g0 = __shfl_sync(FULL_MASK, g0, 0);
+    if (g0 >= F) break;
+    const int nn = min(csz, F - g0);
+    const int32_t vl = lane < nn ? ldw_i32(frontier + g0 + lane) : -1;
     const int64_t lvl = (int64_t)vl - lo;
-    const bool okl = il < sp.end && vl >= 0 && lvl >= 0 && lvl < n_local;
+    const bool okl = lane < nn && vl >= 0 && lvl >= 0 && lvl < n_local;
     int64_t sl = 0, dl = 0;
     if (okl) row_extent(indptr, lvl, &sl, &dl);
-    const int nn = (int)min((int64_t)32, (sp.end - g0 + wpb - 1) / wpb);
-    for (int j = 0; j < nn; ++j) {
-      const int i = (int)(g0 + (int64_t)j * wpb);
-      const int32_t v = __shfl_sync(FULL_MASK, vl, j);
-      const bool ok = __shfl_sync(FULL_MASK, okl, j);
-      const int64_t s = __shfl_sync(FULL_MASK, sl, j);
-      const int64_t d = __shfl_sync(FULL_MASK, dl, j);
-      {  // the next node's weights (rows of up to 32 x 128 B) into L2 while this one is sampled
-        const int jn = min(j + 1, 31);
-        const int64_t sn = __shfl_sync(FULL_MASK, sl, jn), dn = __shfl_sync(FULL_MASK, dl, jn);
-        if (j + 1 < nn && (int64_t)lane * 32 < dn)
-          asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(weights + sn + (int64_t)lane * 32));
-      }
-      uint32_t pos;
-      const int cnt = sample_node_biased(ok, v, s, d, k, layer, key, weights, &pos);
-      if (lane == 0) {
-        B.cnt[i] = cnt;
-        if (src_out) src_out[i] = v;
-        if (ok)
-          mark_dst(B, v, i, F, layer, epoch, err);
-        else
-          latch(err, E_RANGE);
-      }
-      if (lane < cnt) {
-        const int32_t u = __ldg(indices + s + pos);
-        const uint32_t q = (uint32_t)i * (uint32_t)k + (uint32_t)lane;
-        B.rows[q] = u;
-        mark(B, u, epoch, (uint32_t)F + q);
-      }
-    }
+    const BiasedOutW1 out{B, g0, k, F, layer, epoch, src_out, err};
+    biased_claim(nn, vl, okl, sl, dl, k, layer, key, weights, indices, out);
   }
 }
 
@@ -994,7 +997,7 @@ __device__ __forceinline__ void persist_sample(const PersistArgs &a, const int32
   const LayerBufs &B = a.buf[l & 1];
   if (BIASED) {
     phase_sample_biased<TEAM>(frontier, F, l, k, a.key, a.indptr, a.indices, a.weights, a.lo, a.n_local, B, epoch,
-                              a.out.src_ids[l], a.err);
+                              a.out.src_ids[l], a.err, &a.hdr->scursor[l]);
   } else if (k <= 16 && (int64_t)F * (k <= 4 ? 4 : k <= 8 ? 8 : 16) <= (int64_t)a.lane_rounds * gridDim.x * TEAM) {
     // small frontier (the first layers): a lane group per node, so the k
     // Philox draws run in parallel instead of back to back in one thread,

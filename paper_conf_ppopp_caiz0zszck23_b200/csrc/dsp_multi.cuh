@@ -245,8 +245,8 @@ __device__ __forceinline__ void multi_sample_lanes(const MultiArgs &m, int T, co
     int32_t u;
     if (G == 32 && a.biased) {
       uint32_t pos;
-      cnt = sample_node_biased(ok, v, rs, d, k, layer, a.key, a.weights, &pos);
-      slot = lane;
+      const unsigned long long word = lane < k ? biased_word(a.key, lane, v, layer) : 0ull;
+      cnt = sample_node_biased(ok, v, rs, d, k, layer, a.key, a.weights, word, 0, &pos, &slot);
       valid = lane < cnt;
       u = valid ? __ldg(a.indices + rs + pos) : -1;
     } else {
@@ -258,9 +258,25 @@ __device__ __forceinline__ void multi_sample_lanes(const MultiArgs &m, int T, co
   }
 }
 
-// B for biased sampling: warp per task, as phase_sample_biased --
-// the ids and row extents of the warp's next 32 tasks loaded at once, the next
-// task's weight row prefetched into L2 while the current one is sampled.
+// B for biased sampling: as phase_sample_biased (biased_claim on
+// runs of 32 tasks of the block's share, lane groups for rows of <= 256
+// positions), the rows written into the requesters' return slots.
+struct BiasedOutMulti {
+  const MultiArgs &m;
+  int par, k, sl, jl;  // this lane's task of the claim: requester rank, index in its list
+  struct Ctx {
+    int32_t *rows;
+    int32_t *cnt;
+  };
+  __device__ __forceinline__ Ctx ctx(int jn) const {
+    const int s = __shfl_sync(FULL_MASK, sl, jn), j = __shfl_sync(FULL_MASK, jl, jn);
+    char *req = m.peers.base[s];
+    return Ctx{xch_ret_rows(req, m.X, par, m.rank) + (int64_t)j * k, xch_ret_cnt(req, m.X, par, m.rank) + j};
+  }
+  __device__ __forceinline__ void node(const Ctx &c, int32_t, bool, int cnt) const { *c.cnt = cnt; }
+  __device__ __forceinline__ void edge(const Ctx &c, int slot, int32_t u) const { c.rows[slot] = u; }
+};
+
 template <int TEAM>
 __device__ __forceinline__ void multi_sample_biased(const MultiArgs &m, int T, const uint32_t *s_off, int layer,
                                                     int k, int par) {
@@ -287,23 +303,8 @@ __device__ __forceinline__ void multi_sample_biased(const MultiArgs &m, int T, c
       else row_extent(a.indptr, lv, &rsl, &dl);
     }
     const int nn = (int)min((int64_t)32, (sp.end - g0 + wpb - 1) / wpb);
-    for (int t = 0; t < nn; ++t) {
-      const int s = __shfl_sync(FULL_MASK, sl, t), j = __shfl_sync(FULL_MASK, jl, t);
-      const int32_t v = __shfl_sync(FULL_MASK, vl, t);
-      const bool ok = __shfl_sync(FULL_MASK, okl, t);
-      const int64_t rs = __shfl_sync(FULL_MASK, rsl, t), d = __shfl_sync(FULL_MASK, dl, t);
-      {
-        const int tn = min(t + 1, 31);
-        const int64_t sn = __shfl_sync(FULL_MASK, rsl, tn), dn = __shfl_sync(FULL_MASK, dl, tn);
-        if (t + 1 < nn && (int64_t)lane * 32 < dn)
-          asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(a.weights + sn + (int64_t)lane * 32));
-      }
-      uint32_t pos;
-      const int cnt = sample_node_biased(ok, v, rs, d, k, layer, a.key, a.weights, &pos);
-      char *req = m.peers.base[s];
-      if (lane == 0) xch_ret_cnt(req, m.X, par, m.rank)[j] = cnt;
-      if (lane < cnt) xch_ret_rows(req, m.X, par, m.rank)[(int64_t)j * k + lane] = __ldg(a.indices + rs + pos);
-    }
+    const BiasedOutMulti out{m, par, k, sl, jl};
+    biased_claim(nn, vl, okl, rsl, dl, k, layer, a.key, a.weights, a.indices, out);
   }
 }
 
