@@ -427,22 +427,35 @@ __device__ __forceinline__ int biased_chunks(const uint32_t *__restrict__ al, in
   using U = unsigned long long;
   const int lane = threadIdx.x & 31;
   U cs[HSEG], CP[HSEG];
-  int npos = 0;
+  // lane l sums chunk 32j + l: one aligned 128-byte line, 8 vector loads, all
+  // lanes' lines in flight at once (slots outside the row masked to 0)
+  uint32_t np = 0;
 #pragma unroll
   for (int j = 0; j < HSEG; ++j) {
     cs[j] = 0;
-    if (32 * j < nch) {
-      const int n = min(32, nch - 32 * j);
-#pragma unroll 4
-      for (int c = 0; c < n; ++c) {
-        const int q = 32 * (32 * j + c) + lane;
-        const uint32_t x = (q >= off && q < off + d) ? __ldg(al + q) : 0u;
-        npos += __popc(__ballot_sync(FULL_MASK, x > 0u));
-        const U s = warp_sum_w(x);
-        if (lane == c) cs[j] = s;
+    const int c = 32 * j + lane;
+    if (32 * j < nch && c < nch) {
+      const uint4 *line = reinterpret_cast<const uint4 *>(al + 32 * c);
+      uint4 q4[8];
+#pragma unroll
+      for (int e = 0; e < 8; ++e) q4[e] = __ldg(line + e);
+      const int lo = max(0, off - 32 * c), hi = min(32, off + d - 32 * c);  // valid slots [lo, hi)
+      U s = 0;
+#pragma unroll
+      for (int e = 0; e < 8; ++e) {
+        const uint32_t v4[4] = {q4[e].x, q4[e].y, q4[e].z, q4[e].w};
+#pragma unroll
+        for (int f = 0; f < 4; ++f) {
+          const int i = 4 * e + f;
+          const uint32_t x = (i >= lo && i < hi) ? v4[f] : 0u;
+          s += x;
+          np += x > 0u ? 1u : 0u;
+        }
       }
+      cs[j] = s;
     }
   }
+  const int npos = (int)__reduce_add_sync(FULL_MASK, np);
   if (npos <= k) {
     *pos = biased_all_positive(nch, off, [&](int j) {
       const int q = 32 * j + lane;
@@ -591,6 +604,12 @@ __device__ __forceinline__ int sample_node_biased(bool ok, int32_t v, int64_t ro
 // (a weight above 2^24): their results are not written.
 constexpr uint32_t BGROUP_WMAX = 1u << 24;
 
+// the bits of lane group grp (G lanes) of a warp ballot
+template <int G>
+__device__ __forceinline__ uint32_t bslice(uint32_t b, int grp) {
+  return G == 32 ? b : (b >> (grp * G)) & ((1u << G) - 1u);
+}
+
 template <int G>
 __device__ __forceinline__ uint32_t group_sum(uint32_t x) {
 #pragma unroll
@@ -598,10 +617,18 @@ __device__ __forceinline__ uint32_t group_sum(uint32_t x) {
   return x;
 }
 
+#ifdef DSP_BPROF
+#define BPROF_T(var) const long long var = clock64()
+#define BPROF_ADD(idx, val) do { if (bprof && (threadIdx.x & 31) == 0) atomicAdd(bprof + (idx), (unsigned long long)(val)); } while (0)
+#else
+#define BPROF_T(var)
+#define BPROF_ADD(idx, val) do { } while (0)
+#endif
 template <int G, class Out>
 __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl, bool okl, int64_t sl, int dl, int k,
                                                       int layer, uint2 key, const uint32_t *__restrict__ w,
-                                                      const int32_t *__restrict__ indices, const Out &out) {
+                                                      const int32_t *__restrict__ indices, const Out &out,
+                                                      unsigned long long *bprof = nullptr) {
   constexpr int NPW = 32 / G;
   const int lane = threadIdx.x & 31, grp = lane / G, g = lane & (G - 1);
   uint32_t redo = 0;
@@ -614,6 +641,7 @@ __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl
         cmask &= cmask - 1;
       }
     }
+    BPROF_T(s0);
     const bool act = jn >= 0;
     const int src = act ? jn : 0;
     const int32_t v = __shfl_sync(FULL_MASK, vl, src);
@@ -623,6 +651,7 @@ __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl
     const int d = act && ok ? dsh : 0;
     const typename Out::Ctx c = out.ctx(src);
     const unsigned long long word = (g < k && d > 0) ? biased_word(key, g, v, layer) : 0ull;
+    BPROF_T(s1);
     uint32_t x[8], P[8];
     bool heavy = false;
     uint32_t np = 0, T = 0;
@@ -651,19 +680,24 @@ __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl
     uint32_t W = __shfl_sync(FULL_MASK, incl, G - 1, G);
     const uint32_t npos = __shfl_sync(FULL_MASK, ipos, G - 1, G);
     const uint32_t hb = __ballot_sync(FULL_MASK, heavy);
-    heavy = ((G == 32 ? hb : (hb >> (grp * G)) & ((1u << G) - 1u)) != 0u) || (W == 0u && npos > 0u);
+    heavy = bslice<G>(hb, grp) != 0u || (W == 0u && npos > 0u);
 #pragma unroll
     for (int i = 0; i < 8; ++i) P[i] += incl - T;
     const bool allpos = npos <= (uint32_t)k;
+    BPROF_T(s2);
     uint32_t pick = 0xffffffffu;
     int rank = 0;
+    unsigned long long wt = __shfl_sync(FULL_MASK, word, 0, G);
     for (int t = 0; t < k; ++t) {
-      const unsigned long long wt = __shfl_sync(FULL_MASK, word, t, G);
       // mulhi(word, W) for W < 2^32 (as sample_node_biased's rounds)
       const uint32_t r = (uint32_t)(((unsigned long long)(uint32_t)(wt >> 32) * W + __umulhi((uint32_t)wt, W)) >> 32);
+      wt = __shfl_sync(FULL_MASK, word, min(t + 1, G - 1), G);  // the next round's word, off the chain
       uint32_t cnt = 0;
 #pragma unroll
       for (int i = 0; i < 8; ++i) cnt += P[i] <= r ? 1u : 0u;
+      // running weights are non-decreasing along the group's positions, so the
+      // lanes before the pick's lane count 8, the pick's lane counts its index
+      // (0..7) and the lanes behind it 0: p = 8 * #(lanes counting 8) + that index
       const uint32_t p = group_sum<G>(cnt);
       const int io = (int)(p & 7u);
       uint32_t xs = x[0];
@@ -673,13 +707,14 @@ __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl
 #pragma unroll
       for (int i = 0; i < 8; ++i) P[i] -= (uint32_t)(8 * g + i) >= p ? ap : 0u;
       W -= ap;
-      const uint32_t below = __ballot_sync(FULL_MASK, g < t && pick < p);
+      const uint32_t below = bslice<G>(__ballot_sync(FULL_MASK, g < t && pick < p), grp);
       if (g < t && pick > p) ++rank;
       if (g == t) {
         pick = p;
-        rank = __popc(G == 32 ? below : (below >> (grp * G)) & ((1u << G) - 1u));
+        rank = __popc(below);
       }
     }
+    BPROF_T(s3);
     if (act && !heavy) {
       const int cnt = allpos ? (int)npos : k;
       if (g == 0) out.node(c, v, ok, cnt);
@@ -693,6 +728,11 @@ __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl
       }
     }
     redo |= __reduce_or_sync(FULL_MASK, (act && heavy && g == 0) ? 1u << jn : 0u);
+    BPROF_T(s4);
+    if (G == 8) {
+      BPROF_ADD(11, s1 - s0); BPROF_ADD(12, s2 - s1); BPROF_ADD(13, s3 - s2); BPROF_ADD(14, s4 - s3);
+      BPROF_ADD(15, 1);
+    }
   }
   return redo;
 }
@@ -711,14 +751,36 @@ __device__ __forceinline__ int biased_group_of(int64_t d, int k) {
 template <class Out>
 __device__ __forceinline__ void biased_claim(int nn, int32_t vl, bool okl, int64_t sl, int64_t dl, int k, int layer,
                                              uint2 key, const uint32_t *__restrict__ w,
-                                             const int32_t *__restrict__ indices, const Out &out) {
+                                             const int32_t *__restrict__ indices, const Out &out,
+                                             unsigned long long *bprof = nullptr) {
   const int lane = threadIdx.x & 31;
+  // every node's weight and adjacency rows (their first 8 lines) into L2 at
+  // once, so the passes below find them there instead of each waiting on DRAM
+  if (lane < nn && okl) {
+    const char *pw = reinterpret_cast<const char *>(w + sl), *pi = reinterpret_cast<const char *>(indices + sl);
+    const int lines = (int)min((int64_t)8, ((sl & 31) + dl + 31) >> 5);
+    for (int i = 0; i < lines; ++i) {
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(pw + 128 * i));
+      asm volatile("prefetch.global.L2 [%0];" ::"l"(pi + 128 * i));
+    }
+  }
   const int gl = lane < nn ? (okl ? biased_group_of(dl, k) : 8) : -1;
   const int dg = (int)min(dl, (int64_t)256);
-  uint32_t redo = biased_group_pass<8>(__ballot_sync(FULL_MASK, gl == 8), vl, okl, sl, dg, k, layer, key, w, indices, out);
+  BPROF_T(c0);
+  uint32_t redo = biased_group_pass<8>(__ballot_sync(FULL_MASK, gl == 8), vl, okl, sl, dg, k, layer, key, w, indices, out, bprof);
+  BPROF_T(c1);
   redo |= biased_group_pass<16>(__ballot_sync(FULL_MASK, gl == 16), vl, okl, sl, dg, k, layer, key, w, indices, out);
+  BPROF_T(c2);
   redo |= biased_group_pass<32>(__ballot_sync(FULL_MASK, gl == 32), vl, okl, sl, dg, k, layer, key, w, indices, out);
+  BPROF_T(c3);
+  BPROF_ADD(1, c1 - c0); BPROF_ADD(2, c2 - c1); BPROF_ADD(3, c3 - c2);
+#ifdef DSP_BPROF
+  const int n8 = __popc(__ballot_sync(FULL_MASK, gl == 8)), n16 = __popc(__ballot_sync(FULL_MASK, gl == 16)),
+            n32 = __popc(__ballot_sync(FULL_MASK, gl == 32));
+  BPROF_ADD(5, n8); BPROF_ADD(6, n16); BPROF_ADD(7, n32);
+#endif
   uint32_t rest = redo | __ballot_sync(FULL_MASK, gl == 0);
+  BPROF_ADD(8, __popc(rest));
   while (rest) {
     const int j = __ffs(rest) - 1;
     rest &= rest - 1;
@@ -733,6 +795,8 @@ __device__ __forceinline__ void biased_claim(int nn, int32_t vl, bool okl, int64
     if (lane == 0) out.node(c, v, ok, cnt);
     if (lane < cnt) out.edge(c, slot, __ldg(indices + s + pos));
   }
+  BPROF_T(c4);
+  BPROF_ADD(4, c4 - c3);
 }
 
 }  // namespace dsp

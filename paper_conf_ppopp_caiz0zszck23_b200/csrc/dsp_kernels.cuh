@@ -593,20 +593,33 @@ __device__ DSP_PHASE void phase_sample_biased(const int32_t *frontier, int F, in
   const int lane = threadIdx.x & 31;
   const int nwarps = (int)gridDim.x * (TEAM >> 5);
   const int csz = max(1, min(32, F / (4 * nwarps)));
+#ifdef DSP_BPROF
+  unsigned long long *bprof = layer == DSP_BPROF ? reinterpret_cast<unsigned long long *>(cursor - layer) - 32 : nullptr;
+  const long long p0 = clock64();
+#else
+  unsigned long long *bprof = nullptr;
+#endif
   while (true) {
+    BPROF_T(q0);
     int g0 = 0;
     if (lane == 0) g0 = (int)atomicAdd(cursor, (uint32_t)csz);
     g0 = __shfl_sync(FULL_MASK, g0, 0);
     if (g0 >= F) break;
+    const int32_t vl = lane < min(csz, F - g0) ? ldw_i32(frontier + g0 + lane) : -1;
     const int nn = min(csz, F - g0);
-    const int32_t vl = lane < nn ? ldw_i32(frontier + g0 + lane) : -1;
     const int64_t lvl = (int64_t)vl - lo;
     const bool okl = lane < nn && vl >= 0 && lvl >= 0 && lvl < n_local;
     int64_t sl = 0, dl = 0;
     if (okl) row_extent(indptr, lvl, &sl, &dl);
     const BiasedOutW1 out{B, g0, k, F, layer, epoch, src_out, err};
-    biased_claim(nn, vl, okl, sl, dl, k, layer, key, weights, indices, out);
+    BPROF_T(q1);
+    BPROF_ADD(0, q1 - q0);
+    BPROF_ADD(9, 1);
+    biased_claim(nn, vl, okl, sl, dl, k, layer, key, weights, indices, out, bprof);
   }
+#ifdef DSP_BPROF
+  BPROF_ADD(10, clock64() - p0);
+#endif
 }
 
 // ------------------------------------------- scan, two-phase (persistent)

@@ -1501,7 +1501,10 @@ dsp_status dsp_load_weights(dsp_ctx *c, const float *edge_weights) {
   if (!edge_weights && c->nnz > 0) return fail(c, DSP_ERR_INVALID_ARG, "edge_weights is NULL");
   DeviceGuard g(c->device);
   const size_t n = (size_t)std::max<int64_t>(1, c->nnz);
-  CUDA_TRY(c, cudaMalloc(&c->d_weights, sizeof(uint32_t) * n));
+  // 32 zero words of padding: the biased sampler reads rows as whole aligned
+  // 128-byte lines, the last one possibly past the last weight
+  CUDA_TRY(c, cudaMalloc(&c->d_weights, sizeof(uint32_t) * (n + 32)));
+  CUDA_TRY(c, cudaMemset(c->d_weights, 0, sizeof(uint32_t) * (n + 32)));
   if (c->nnz > 0) {
     float *tmp = nullptr;
     CUDA_TRY(c, cudaMalloc(&tmp, sizeof(float) * n));
