@@ -754,16 +754,6 @@ __device__ __forceinline__ void biased_claim(int nn, int32_t vl, bool okl, int64
                                              const int32_t *__restrict__ indices, const Out &out,
                                              unsigned long long *bprof = nullptr) {
   const int lane = threadIdx.x & 31;
-  // every node's weight and adjacency rows (their first 8 lines) into L2 at
-  // once, so the passes below find them there instead of each waiting on DRAM
-  if (lane < nn && okl) {
-    const char *pw = reinterpret_cast<const char *>(w + sl), *pi = reinterpret_cast<const char *>(indices + sl);
-    const int lines = (int)min((int64_t)8, ((sl & 31) + dl + 31) >> 5);
-    for (int i = 0; i < lines; ++i) {
-      asm volatile("prefetch.global.L2 [%0];" ::"l"(pw + 128 * i));
-      asm volatile("prefetch.global.L2 [%0];" ::"l"(pi + 128 * i));
-    }
-  }
   const int gl = lane < nn ? (okl ? biased_group_of(dl, k) : 8) : -1;
   const int dg = (int)min(dl, (int64_t)256);
   BPROF_T(c0);

@@ -554,7 +554,7 @@ __device__ DSP_PHASE void phase_sample_tpn(const int32_t *frontier, int F, int l
 // Biased sampling, world 1: warps claim runs of consecutive frontier
 // nodes from a per-layer cursor (row lengths of the frontier span three
 // orders of magnitude, so a static share leaves warps idle at the grid
-// barrier); a claim is about a quarter of a warp's even share, at most 32
+// barrier); a claim is about half a warp's even share, at most 32
 // nodes.  The ids and row extents of a claim are loaded at once (one per
 // lane), then biased_claim samples them: lane groups for rows of <= 256
 // positions, the warp-wide sampler for longer ones.
@@ -592,7 +592,7 @@ __device__ DSP_PHASE void phase_sample_biased(const int32_t *frontier, int F, in
                                                     int32_t *src_out, int *err, uint32_t *cursor) {
   const int lane = threadIdx.x & 31;
   const int nwarps = (int)gridDim.x * (TEAM >> 5);
-  const int csz = max(1, min(32, F / (4 * nwarps)));
+  const int csz = max(1, min(32, F / (2 * nwarps)));
 #ifdef DSP_BPROF
   unsigned long long *bprof = layer == DSP_BPROF ? reinterpret_cast<unsigned long long *>(cursor - layer) - 32 : nullptr;
   const long long p0 = clock64();
