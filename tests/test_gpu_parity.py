@@ -647,6 +647,73 @@ def test_biased_long_rows(pkg, heavy):
     grp.close()
 
 
+def _group_boundary_graph():
+    """Rows on both sides of every boundary of the biased sampler (lane groups
+    of 8 / 16 / 32 lanes x 8 positions: degrees 64 / 128 / 256; aligned
+    chunk sums up to 4 x 32 lines, then re-reads), at every alignment of the
+    row start inside a 128-byte line, with weights in (0, 256] (the lane-group
+    limit is 2^24 = 256.0 in 16.16), some heavier than 256 (the warp-wide
+    sampler takes those rows), zero weights, a row of 256 weights of exactly
+    256.0 (its total is 2^32: the 32-bit running weights would wrap, so the
+    warp-wide sampler takes it) and rows whose positive weights are <= k."""
+    rng = np.random.default_rng(77)
+    special = [0, 1, 2, 5, 7, 8, 9, 16, 17, 31, 32, 33, 63, 64, 65, 100, 127, 128, 129, 200, 255, 256, 257,
+               300, 1000, 4000, 4033, 4064, 4065, 4100, 6000]
+    N = 20000
+    degs = rng.integers(0, 60, size=N)
+    hubs = []
+    for r, d in enumerate(special * 3):
+        hubs.append(r)
+        degs[r] = d
+    rows = []
+    for v in range(N):
+        nb = rng.choice(N - 1, size=int(degs[v]), replace=False)
+        nb[nb >= v] += 1
+        rows.append(np.sort(nb))
+    ip = np.zeros(N + 1, np.int64)
+    ip[1:] = np.cumsum([len(r) for r in rows])
+    ix = np.concatenate(rows).astype(np.int32)
+    w = (rng.integers(1, 4097, size=len(ix)) / 16.0).astype(np.float32)   # (0, 256], exact in 16.16
+    w[rng.random(len(ix)) < 0.05] = 0.0
+    n = len(special)
+    heavy_rows = list(range(n, 2 * n))          # second copy: a few weights above 256
+    for v in heavy_rows:
+        a, b = ip[v], ip[v + 1]
+        if b > a:
+            w[a + rng.integers(0, b - a, size=max(1, (b - a) // 16))] = 300.5
+    full = special.index(256) + 2 * n            # third copy of degree 256: every weight 256.0
+    w[ip[full]:ip[full + 1]] = 256.0
+    few = special.index(100) + 2 * n             # third copy of degree 100: 3 positive weights
+    w[ip[few]:ip[few + 1]] = 0.0
+    w[ip[few] + np.array([3, 50, 99])] = 1.5
+    return N, ip, ix, w, hubs
+
+
+@pytest.mark.parametrize("fan", [(5, 3), (8, 1), (9, 16), (17, 2), (32, 5)])
+def test_biased_group_boundaries(pkg, fan):
+    N, ip, ix, w, hubs = _group_boundary_graph()
+    feats = datagen.features(0, N, 4)
+    seeds = np.array(hubs, np.int32)
+    s = pkg.Sampler(datagen.bounds(N, 1), ip, ix, feats, fan, len(seeds), edge_weights=w)
+    for rng_seed in (3, 4):
+        blocks = s.sample(torch.from_numpy(seeds).cuda(), rng_seed, biased=True)
+        assert_blocks_equal(blocks, oracle.sample(ip, ix, seeds, fan, rng_seed, weights=w), f"fan {fan} rng {rng_seed}")
+    s.close()
+    # the owner-side sampler of the multi-rank kernel (virtual P = 2)
+    bnds = datagen.bounds(N, 2)
+    shards = []
+    for r in range(2):
+        lo, hi = int(bnds[r]), int(bnds[r + 1])
+        sip, six = datagen.shard(ip, ix, lo, hi)
+        shards.append((sip, six, feats[lo:hi], w[ip[lo]:ip[hi]]))
+    grp = pkg.LocalGroup(bnds, shards, fan, len(seeds), devices=[0, 0])
+    rs = [seeds[seeds < bnds[1]], seeds[seeds >= bnds[1]]]
+    res = grp.sample([torch.from_numpy(np.ascontiguousarray(x)).cuda() for x in rs], 11, biased=True)
+    for r in range(2):
+        assert_blocks_equal(res[r], oracle.sample(ip, ix, rs[r], fan, 11, weights=w), f"fan {fan} P=2 rank {r}")
+    grp.close()
+
+
 def test_biased_errors(pkg, tiny):
     cfg, ip, ix, feats = tiny
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, 8)
