@@ -647,6 +647,7 @@ struct Scan2Smem {
 
 struct Scan2Regs {
   uint32_t vbits, fbits;  // bit s: slot q0 + s * TEAM holds an edge / is a first occurrence
+  int32_t r[SCAN2_IPT];   // GROUPS == 1: the slot's rows[] value after pass 1 (pass 2 reads no memory for it)
 };
 
 // A block's chunk [tile0, tile_end) of one round is processed as up to
@@ -694,7 +695,9 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
       const bool first = valid && w[j] == mword(B, epoch, u[j], (uint32_t)F + q0 + j * TEAM);
       // a valid slot that is not u's first occurrence keeps x (u's smallest order
       // key: its dst index, or F + the slot of its first occurrence) as -1 - x
-      if (valid && !first) B.rows[q0 + j * TEAM] = -1 - (int32_t)mword_x(B, w[j]);
+      const int32_t rv = valid && !first ? -1 - (int32_t)mword_x(B, w[j]) : u[j];
+      if (valid && !first) B.rows[q0 + j * TEAM] = rv;
+      if (GROUPS == 1) R.r[j] = rv;
       R.vbits |= (valid ? 1u : 0u) << (g * SCAN2_IPT + j);
       R.fbits |= (first ? 1u : 0u) << (g * SCAN2_IPT + j);
       const uint32_t bv = __ballot_sync(FULL_MASK, valid), bf = __ballot_sync(FULL_MASK, first);
@@ -703,7 +706,7 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
   }
   team_sync<TEAM>();
   if (wid == 0) {  // exclusive scan of the (stripe, warp) counts, stripe-major, group by group
-    constexpr int PER = SCAN2_IPT * W / 32;
+    constexpr int PER = (SCAN2_IPT * W + 31) / 32;  // entries per lane (the last lanes' tail may be empty)
     unsigned long long carry = 0;
 #pragma unroll 1
     for (int g = 0; g < groups; ++g) {
@@ -711,7 +714,7 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
       unsigned long long v[PER], run = 0;
 #pragma unroll
       for (int e = 0; e < PER; ++e) {
-        v[e] = tab[lane * PER + e];
+        v[e] = lane * PER + e < SCAN2_IPT * W ? tab[lane * PER + e] : 0ull;
         run += v[e];
       }
       unsigned long long incl = run;
@@ -723,7 +726,7 @@ __device__ __forceinline__ void scan2_pass1(int F, int k, const LayerBufs &B, ui
       unsigned long long p = carry + incl - run;
 #pragma unroll
       for (int e = 0; e < PER; ++e) {
-        tab[lane * PER + e] = p;
+        if (lane * PER + e < SCAN2_IPT * W) tab[lane * PER + e] = p;
         p += v[e];
       }
       carry += __shfl_sync(FULL_MASK, incl, 31);
@@ -795,7 +798,8 @@ __device__ __forceinline__ void scan2_pass2(int F, int k, const LayerBufs &B, in
     const uint32_t vb = R.vbits >> (g * SCAN2_IPT), fb = R.fbits >> (g * SCAN2_IPT);
     int32_t r[SCAN2_IPT];
 #pragma unroll
-    for (int j = 0; j < SCAN2_IPT; ++j) r[j] = ((vb >> j) & 1u) ? ldw_i32(B.rows + q0 + j * TEAM) : 0;
+    for (int j = 0; j < SCAN2_IPT; ++j)
+      r[j] = GROUPS == 1 ? R.r[j] : ((vb >> j) & 1u) ? ldw_i32(B.rows + q0 + j * TEAM) : 0;
 #pragma unroll
     for (int j = 0; j < SCAN2_IPT; ++j) {
       const uint32_t bv = __ballot_sync(FULL_MASK, (vb >> j) & 1u);
@@ -972,6 +976,13 @@ constexpr int LOADER_WARPS = 4;                      // TMA gather warps of a pi
 constexpr int LOADER_SLOTS = DSP_LOADER_SLOTS;       // ring slots per loader warp of a pipelined launch
 constexpr int GTMA_SLOTS = 2;                        // ring slots per warp of the standalone gather
 constexpr int PIPE_TEAM = PNT - 32 * LOADER_WARPS;   // sampling threads of a pipelined launch
+#ifndef DSP_BIASED_LOADERS
+#define DSP_BIASED_LOADERS 3
+#endif
+// biased sampling is bound by the sampling, not the gather: 3 loader warps
+// (29 sampling warps) measured 0.2136-0.2148 vs 0.2166 ms/step with 4, 0.219 with 2
+constexpr int BIASED_LOADER_WARPS = DSP_BIASED_LOADERS;
+constexpr int BIASED_PIPE_TEAM = PNT - 32 * BIASED_LOADER_WARPS;
 
 struct PersistArgs {
   const int32_t *seeds;

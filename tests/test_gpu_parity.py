@@ -451,14 +451,38 @@ def test_products_fused_step(pkg, products):
     s.close()
 
 
-def _check_step(s, slot, sizes, seeds, rng, ip, ix, feats_of):
-    ref = oracle.sample(ip, ix, seeds, s.fanouts, rng)
+def _check_step(s, slot, sizes, seeds, rng, ip, ix, feats_of, weights=None):
+    ref = oracle.sample(ip, ix, seeds, s.fanouts, rng, weights=weights)
     exp = [v for r in ref for v in (r["num_dst"], r["num_src"], r["num_edges"])]
     assert [int(x) for x in sizes] == exp
     blocks = s.blocks(slot, sizes=[int(x) for x in sizes])
     assert_blocks_equal(blocks, ref, f"pipelined rng {rng}")
     feat = s.feat_buffer(slot)[: blocks[-1].num_src]
     assert np.array_equal(feat.cpu().numpy().view(np.uint32), feats_of(ref[-1]["src_ids"]).view(np.uint32))
+
+
+def test_pipelined_steps_biased(pkg, tiny, tiny_weights):
+    """DSP_PIPELINED with DSP_BIASED (its own launch shape: fewer loader warps)."""
+    cfg, ip, ix, feats = tiny
+    s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2,
+                    edge_weights=tiny_weights)
+    batches = seeds_of(cfg, 1, 0)
+    L = len(cfg.fanouts)
+    sizes = torch.zeros((6, 3 * L), dtype=torch.int64).pin_memory()
+    for j in range(6):
+        s.sample_gather(torch.from_numpy(batches[j]).cuda(), 500 + j, slot=j % 2, sizes_out=sizes[j],
+                        pipelined=True, biased=True)
+        if j >= 1:
+            s.sync()
+            ref = oracle.sample(ip, ix, batches[j - 1], cfg.fanouts, 500 + j - 1, weights=tiny_weights)
+            assert [int(x) for x in sizes[j - 1]] == [v for r in ref for v in (r["num_dst"], r["num_src"], r["num_edges"])]
+            blocks = s.blocks((j - 1) % 2, sizes=[int(x) for x in sizes[j - 1]])
+            assert_blocks_equal(blocks, ref, f"biased pipelined step {j - 1}")
+            feat = s.feat_buffer((j - 1) % 2)[: blocks[-1].num_src]
+            assert np.array_equal(feat.cpu().numpy(), oracle.gather(feats, ref[-1]["src_ids"]))
+    s.flush()
+    s.sync()
+    s.close()
 
 
 def test_pipelined_steps(pkg, tiny):
@@ -505,7 +529,8 @@ def test_products_pipelined(pkg, products):
 
 
 @pytest.mark.slow
-def test_products_bench_launch_configuration(pkg, products):
+@pytest.mark.parametrize("biased", [False, True])
+def test_products_bench_launch_configuration(pkg, products, biased):
     """configs[1] at full size in exactly the launch configuration bench.py
     times: 4 concurrent step streams, each pipelined persistent launch on 37
     SMs with its own workspace, 8 output sets, sizes returned asynchronously;
@@ -513,9 +538,10 @@ def test_products_bench_launch_configuration(pkg, products):
     (blocks bit-exact, every gathered row against the closed-form features)."""
     cfg, ip, ix = products
     feats = datagen.features(0, cfg.num_nodes, cfg.dim)
+    ew = datagen.edge_weights(ix, datagen.node_weights(cfg.num_nodes)) if biased else None
     K = 4
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2 * K,
-                    n_workspaces=K)
+                    n_workspaces=K, edge_weights=ew)
     pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(0).multi_processor_count // K)
     batches = seeds_of(cfg, 1, 0)
     L = len(cfg.fanouts)
@@ -528,7 +554,7 @@ def test_products_bench_launch_configuration(pkg, products):
         st.wait_stream(main)
     for i in range(n):
         s.sample_gather(dev[i], 0x5EED + i, slot=i % (2 * K), sizes_out=sizes[i],
-                        async_=True, pipelined=True, ws=i % K, stream=streams[i % K])
+                        async_=True, pipelined=True, biased=biased, ws=i % K, stream=streams[i % K])
     for st in streams:
         with torch.cuda.stream(st):
             s.flush()
@@ -538,7 +564,7 @@ def test_products_bench_launch_configuration(pkg, products):
     torch.cuda.synchronize()
     feats_of = lambda ids: datagen.features_of(ids, cfg.dim)
     for i in range(n - 2 * K, n):
-        _check_step(s, i % (2 * K), sizes[i], batches[i], 0x5EED + i, ip, ix, feats_of)
+        _check_step(s, i % (2 * K), sizes[i], batches[i], 0x5EED + i, ip, ix, feats_of, weights=ew)
     s.close()
 
 
