@@ -970,7 +970,12 @@ __global__ void __launch_bounds__(NT) k_gather(const __grid_constant__ GatherArg
 }
 
 // ============================================ world == 1: persistent kernel
-constexpr int LOADER_WARPS = 4;                      // TMA gather warps of a pipelined launch (default)
+#ifndef DSP_LOADER_WARPS
+#define DSP_LOADER_WARPS 5
+#endif
+// TMA gather warps of a pipelined launch: 5 (27 sampling warps) measured 0.1314 vs
+// 0.1322 ms/step with 4 and 0.1335 with 3; 6 rings exceed the shared memory
+constexpr int LOADER_WARPS = DSP_LOADER_WARPS;
 #ifndef DSP_LOADER_SLOTS
 #define DSP_LOADER_SLOTS 2
 #endif
@@ -1127,7 +1132,7 @@ __device__ __forceinline__ void gather_rows_regs(const PersistArgs &a, int64_t r
 // into a shared-memory ring slot, completion counted on the slot's mbarrier,
 // then one bulk store of the R contiguous output rows).  Chunks come from a
 // grid-wide cursor, so the sampling warps can join when they are done.
-// 4 warps per SM sustain ~5 TB/s on random 400-byte rows
+// LOADER_WARPS warps per SM sustain ~5 TB/s on random 400-byte rows
 // (tools/micro/tma_gather_bench.cu), leaving 28 warps for the sampling.
 // MULTI (world > 1): rows of every rank, the bulk copy reading the owner's
 // shard (local, or a peer's over NVLink through its mapping).
