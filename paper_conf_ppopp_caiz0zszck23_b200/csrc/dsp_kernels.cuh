@@ -1133,7 +1133,7 @@ __device__ __forceinline__ void gather_rows_regs(const PersistArgs &a, int64_t r
 // then one bulk store of the R contiguous output rows).  Chunks come from a
 // grid-wide cursor, so the sampling warps can join when they are done.
 // LOADER_WARPS warps per SM sustain ~5 TB/s on random 400-byte rows
-// (tools/micro/tma_gather_bench.cu), leaving 28 warps for the sampling.
+// (tools/micro/tma_gather_bench.cu), leaving the other warps for the sampling.
 // MULTI (world > 1): rows of every rank, the bulk copy reading the owner's
 // shard (local, or a peer's over NVLink through its mapping).
 // STATIC: chunks gw, gw + nw, ... instead of the grid-wide cursor (the
@@ -1146,7 +1146,6 @@ __device__ DSP_PHASE void loader_warp(const PersistArgs &a, char *ring, uint64_t
   const int R = a.rows_per_chunk;
   const uint32_t row_bytes = (uint32_t)g.dim4 * 16u, head_bytes = (uint32_t)g.head4 * 16u;
   const uint32_t tail_bytes = row_bytes - head_bytes;
-  const int64_t nchunks = (n + R - 1) / R;
   char *out = reinterpret_cast<char *>(g.out);
   const unsigned long long pol = l2_policy_evict_first(), pol_t = head_bytes ? l2_policy_tail() : pol;
   int issued = 0, done = 0;
