@@ -1270,7 +1270,8 @@ __global__ void __launch_bounds__(32 * GTMA_WARPS) k_gather_tma(const __grid_con
 // no map clearing (epochs).
 template <int TEAM, bool PIPE, bool BIASED>
 __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(const __grid_constant__ PersistArgs a) {
-  __shared__ Scan2Smem<TEAM> sm;
+  constexpr int SG = 1;  // scan groups per round (2 / 4 measured equal at 4 streams; 1 keeps pass 1's rows in registers)
+  __shared__ Scan2Smem<TEAM, SG> sm;
   __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];
   extern __shared__ __align__(128) char ring_smem[];
   const int blk = blockIdx.x, nblk = gridDim.x;
@@ -1320,7 +1321,7 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(const __grid_constant
                          block_span<TEAM>((int64_t)Fprev * a.k[l - 1]));
     grid_barrier<TEAM>(a.hdr, bar);
     // scan over the F*k edge slots: each block one contiguous chunk of <= TEAM*IPT slots per round
-    constexpr int64_t TILE = (int64_t)TEAM * SCAN2_IPT;
+    constexpr int64_t TILE = (int64_t)TEAM * SCAN2_IPT * SG;
     const int64_t total = (int64_t)F * k;
     const int64_t rounds = total > 0 ? (total + (int64_t)nblk * TILE - 1) / ((int64_t)nblk * TILE) : 1;
     const int64_t per_round = (total + rounds - 1) / rounds;
@@ -1331,11 +1332,11 @@ __global__ void __launch_bounds__(PNT, 1) k_csp_persistent(const __grid_constant
       const int64_t r0 = r * per_round, r1 = min(total, r0 + per_round);
       const int64_t tile0 = min(r1, r0 + (int64_t)blk * chunk), tile_end = min(r1, tile0 + chunk);
       unsigned long long *agg = a.agg + (r & 1) * MAX_PERSIST_BLOCKS;
-      scan2_pass1<TEAM>(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, agg + blk, sm);
+      scan2_pass1<TEAM, SG>(F, k, a.buf[l & 1], epoch, tile0, tile_end, R, agg + blk, sm);
       grid_barrier<TEAM>(a.hdr, bar);
       unsigned long long prefix, round_total;
-      scan2_prefix<TEAM>(agg, nblk, blk, sm, &prefix, &round_total);
-      scan2_pass2<TEAM>(F, k, a.buf[l & 1], tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
+      scan2_prefix<TEAM, SG>(agg, nblk, blk, sm, &prefix, &round_total);
+      scan2_pass2<TEAM, SG>(F, k, a.buf[l & 1], tile0, tile_end, R, carry + prefix, sm, a.out.indptr[l],
                         a.out.indices[l], a.out.src_ids[l]);
       carry += round_total;
       if (r + 1 < rounds) grid_barrier<TEAM>(a.hdr, bar);
