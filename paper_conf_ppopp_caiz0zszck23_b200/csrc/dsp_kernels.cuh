@@ -988,7 +988,13 @@ constexpr int PIPE_TEAM = PNT - 32 * LOADER_WARPS;   // sampling threads of a pi
 // biased sampling is bound by the sampling, not the gather: 3 loader warps
 // (29 sampling warps) measured 0.2136-0.2148 vs 0.2166 ms/step with 4, 0.219 with 2
 constexpr int BIASED_LOADER_WARPS = DSP_BIASED_LOADERS;
-constexpr int BIASED_PIPE_TEAM = PNT - 32 * BIASED_LOADER_WARPS;
+#ifndef DSP_BIASED_BLOCK
+#define DSP_BIASED_BLOCK 1024
+#endif
+// threads per block of the biased persistent kernels: 1024 (64 registers) measured 0.2126-0.2173
+// ms/step vs 0.2196-0.2209 with 896 (72 registers) and 0.228 with 768 (80 registers): warps beat registers
+constexpr int BIASED_BLK = DSP_BIASED_BLOCK;
+constexpr int BIASED_PIPE_TEAM = BIASED_BLK - 32 * BIASED_LOADER_WARPS;
 
 struct PersistArgs {
   const int32_t *seeds;
@@ -1268,8 +1274,8 @@ __global__ void __launch_bounds__(32 * GTMA_WARPS) k_gather_tma(const __grid_con
 // previous call's gather by the loader warps running alongside the sampling
 // (the paper's loader(t-1) || sampler(t)).  No host round trip,
 // no map clearing (epochs).
-template <int TEAM, bool PIPE, bool BIASED>
-__global__ void __launch_bounds__(PNT, 1) k_csp_persistent(const __grid_constant__ PersistArgs a) {
+template <int TEAM, bool PIPE, bool BIASED, int BLK = PNT>
+__global__ void __launch_bounds__(BLK, 1) k_csp_persistent(const __grid_constant__ PersistArgs a) {
   constexpr int SG = 1;  // scan groups per round (2 / 4 measured equal at 4 streams; 1 keeps pass 1's rows in registers)
   __shared__ Scan2Smem<TEAM, SG> sm;
   __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];

@@ -707,9 +707,9 @@ dsp_status stage_persistent(Call &k) {
   const dim3 grid(c->persist_blocks > 0 ? c->persist_blocks : c->num_sms * c->persist_blocks_per_sm), block(PNT);
   void *args[] = {&a};
   if (!k.pipelined) {
-    CUDA_TRY(c, cudaLaunchCooperativeKernel(k.biased ? (const void *)k_csp_persistent<PNT, false, true>
+    CUDA_TRY(c, cudaLaunchCooperativeKernel(k.biased ? (const void *)k_csp_persistent<BIASED_BLK, false, true, BIASED_BLK>
                                                      : (const void *)k_csp_persistent<PNT, false, false>,
-                                            grid, block, args, 0, k.stream));
+                                            grid, k.biased ? dim3(BIASED_BLK) : block, args, 0, k.stream));
     return DSP_OK;
   }
   dsp_ctx::Pending *pd = c->pending_of(k.ws);
@@ -724,9 +724,9 @@ dsp_status stage_persistent(Call &k) {
   a.rows_per_chunk = std::max(1, std::min(c->loader_rows, 12800 / std::max(1, row_bytes)));
   a.slot_bytes = (int)align_up((size_t)a.rows_per_chunk * row_bytes, 128);
   const size_t smem = (size_t)(k.biased ? BIASED_LOADER_WARPS : LOADER_WARPS) * LOADER_SLOTS * a.slot_bytes;
-  CUDA_TRY(c, cudaLaunchCooperativeKernel(k.biased ? (const void *)k_csp_persistent<BIASED_PIPE_TEAM, true, true>
+  CUDA_TRY(c, cudaLaunchCooperativeKernel(k.biased ? (const void *)k_csp_persistent<BIASED_PIPE_TEAM, true, true, BIASED_BLK>
                                                    : (const void *)k_csp_persistent<PIPE_TEAM, true, false>,
-                                          grid, block, args, smem, k.stream));
+                                          grid, k.biased ? dim3(BIASED_BLK) : block, args, smem, k.stream));
   pd->ids = k.blocks[k.L - 1].src_ids;
   pd->out = k.feat_out;
   pd->stream = k.stream;
@@ -1282,7 +1282,7 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   const int pipe_smem = std::min(LOADER_WARPS * LOADER_SLOTS * 16384, 200 * 1024);  // largest ring (dim 4096)
   if (cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM, true, false>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_csp_persistent<BIASED_PIPE_TEAM, true, true>,
+      cudaFuncSetAttribute((const void *)k_csp_persistent<BIASED_PIPE_TEAM, true, true, BIASED_BLK>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
       cudaFuncSetAttribute((const void *)k_csp_multi<PIPE_TEAM, true, false>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
