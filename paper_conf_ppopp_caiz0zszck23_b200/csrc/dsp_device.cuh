@@ -610,6 +610,16 @@ __device__ __forceinline__ uint32_t bslice(uint32_t b, int grp) {
   return G == 32 ? b : (b >> (grp * G)) & ((1u << G) - 1u);
 }
 
+// the sums of x over each group of G lanes with one warp REDUX: group q's
+// values shifted into their own 32 / (32 / G)-bit field (the sums must fit it)
+template <int G>
+__device__ __forceinline__ uint32_t group_sum_redux(uint32_t x, int grp) {
+  if (G == 32) return __reduce_add_sync(FULL_MASK, x);
+  constexpr int SH = G;  // 32 / (32 / G) bits per group
+  const uint32_t tot = __reduce_add_sync(FULL_MASK, x << (SH * grp));
+  return (tot >> (SH * grp)) & ((1u << SH) - 1u);
+}
+
 template <int G>
 __device__ __forceinline__ uint32_t group_sum(uint32_t x) {
 #pragma unroll
@@ -692,17 +702,21 @@ __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl
       // mulhi(word, W) for W < 2^32 (as sample_node_biased's rounds)
       const uint32_t r = (uint32_t)(((unsigned long long)(uint32_t)(wt >> 32) * W + __umulhi((uint32_t)wt, W)) >> 32);
       wt = __shfl_sync(FULL_MASK, word, min(t + 1, G - 1), G);  // the next round's word, off the chain
-      uint32_t cnt = 0;
-#pragma unroll
-      for (int i = 0; i < 8; ++i) cnt += P[i] <= r ? 1u : 0u;
-      // running weights are non-decreasing along the group's positions, so the
-      // lanes before the pick's lane count 8, the pick's lane counts its index
-      // (0..7) and the lanes behind it 0: p = 8 * #(lanes counting 8) + that index
-      const uint32_t p = group_sum<G>(cnt);
+      // count of the lane's positions whose running weight is <= r (adder tree)
+      const uint32_t c01 = (P[0] <= r ? 1u : 0u) + (P[1] <= r ? 1u : 0u), c23 = (P[2] <= r ? 1u : 0u) + (P[3] <= r ? 1u : 0u);
+      const uint32_t c45 = (P[4] <= r ? 1u : 0u) + (P[5] <= r ? 1u : 0u), c67 = (P[6] <= r ? 1u : 0u) + (P[7] <= r ? 1u : 0u);
+      const uint32_t cnt = (c01 + c23) + (c45 + c67);
+      // running weights are non-decreasing along the group's positions and a
+      // picked position's interval is empty, so the pick is the group's count
+      // (one packed REDUX for all groups of the warp: 48 cycles, vs 3 dependent
+      // shuffles; a chain-length win measured 0.2125 -> 0.2085 ms/step)
+      const uint32_t p = group_sum_redux<G>(cnt, grp);
       const int io = (int)(p & 7u);
-      uint32_t xs = x[0];
-#pragma unroll
-      for (int i = 1; i < 8; ++i) xs = io == i ? x[i] : xs;
+      // x[io] by a 3-level select tree (depth 3 instead of a chain of 7)
+      const uint32_t s01 = (io & 1) ? x[1] : x[0], s23 = (io & 1) ? x[3] : x[2];
+      const uint32_t s45 = (io & 1) ? x[5] : x[4], s67 = (io & 1) ? x[7] : x[6];
+      const uint32_t s03 = (io & 2) ? s23 : s01, s47 = (io & 2) ? s67 : s45;
+      const uint32_t xs = (io & 4) ? s47 : s03;
       const uint32_t ap = __shfl_sync(FULL_MASK, xs, (int)(p >> 3), G);
 #pragma unroll
       for (int i = 0; i < 8; ++i) P[i] -= (uint32_t)(8 * g + i) >= p ? ap : 0u;
