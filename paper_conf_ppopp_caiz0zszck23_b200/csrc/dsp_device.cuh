@@ -614,17 +614,13 @@ __device__ __forceinline__ uint32_t bslice(uint32_t b, int grp) {
 // values shifted into their own 32 / (32 / G)-bit field (the sums must fit it)
 template <int G>
 __device__ __forceinline__ uint32_t group_sum_redux(uint32_t x, int grp) {
-  if (G == 32) return __reduce_add_sync(FULL_MASK, x);
-  constexpr int SH = G;  // 32 / (32 / G) bits per group
-  const uint32_t tot = __reduce_add_sync(FULL_MASK, x << (SH * grp));
-  return (tot >> (SH * grp)) & ((1u << SH) - 1u);
-}
-
-template <int G>
-__device__ __forceinline__ uint32_t group_sum(uint32_t x) {
-#pragma unroll
-  for (int o = G / 2; o > 0; o >>= 1) x += __shfl_xor_sync(FULL_MASK, x, o, G);
-  return x;
+  if constexpr (G == 32) {
+    return __reduce_add_sync(FULL_MASK, x);
+  } else {
+    constexpr int SH = G;  // 32 / (32 / G) bits per group
+    const uint32_t tot = __reduce_add_sync(FULL_MASK, x << (SH * grp));
+    return (tot >> (SH * grp)) & ((1u << SH) - 1u);
+  }
 }
 
 #ifdef DSP_BPROF
