@@ -673,18 +673,15 @@ __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl
       T += x[i];
       P[i] = T;
     }
-    // group scans: exclusive prefix of the lane totals and of the positive counts
-    uint32_t incl = T, ipos = np;
+    // group scan of the lane totals; the group's positive count by a packed REDUX
+    uint32_t incl = T;
 #pragma unroll
     for (int o = 1; o < G; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL_MASK, incl, o, G), z = __shfl_up_sync(FULL_MASK, ipos, o, G);
-      if (g >= o) {
-        incl += y;
-        ipos += z;
-      }
+      const uint32_t y = __shfl_up_sync(FULL_MASK, incl, o, G);
+      if (g >= o) incl += y;
     }
     uint32_t W = __shfl_sync(FULL_MASK, incl, G - 1, G);
-    const uint32_t npos = __shfl_sync(FULL_MASK, ipos, G - 1, G);
+    const uint32_t npos = group_sum_redux<G>(np, grp);
     const uint32_t hb = __ballot_sync(FULL_MASK, heavy);
     heavy = bslice<G>(hb, grp) != 0u || (W == 0u && npos > 0u);
 #pragma unroll
@@ -729,6 +726,14 @@ __device__ __forceinline__ uint32_t biased_group_pass(uint32_t cmask, int32_t vl
       const int cnt = allpos ? (int)npos : k;
       if (g == 0) out.node(c, v, ok, cnt);
       if (allpos) {  // every positive-weight position, in row order
+        // the group's lanes are all here (act, heavy and allpos are per group)
+        const unsigned gm = G == 32 ? FULL_MASK : ((1u << G) - 1u) << (grp * G);
+        uint32_t ipos = np;
+#pragma unroll
+        for (int o = 1; o < G; o <<= 1) {
+          const uint32_t z = __shfl_up_sync(gm, ipos, o, G);
+          if (g >= o) ipos += z;
+        }
         uint32_t sl2 = ipos - np;
 #pragma unroll
         for (int i = 0; i < 8; ++i)
