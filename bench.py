@@ -4,8 +4,8 @@ One step = one pass of the whole hot path over one mini-batch per GPU: one
 dsp_sample_gather call -- CSP over all layers (shuffle / sample / reshuffle /
 relabel) and the feature gather of the sampled nodes
 (a8) -- pipelined as in the paper: the launch of step t samples
-batch t while its loader warps gather batch t-1; at N=1 four step streams run
-concurrently on 37 SMs each.  Workload at N=1: BASELINE.json configs[1]
+batch t while its loader warps gather batch t-1; at N=1 two step streams run
+concurrently on 74 SMs each (biased / layer-wise: four on 37).  Workload at N=1: BASELINE.json configs[1]
 (ogbn-products-shaped synthetic R-MAT, fan-out [15,10,5], 1024 seeds/GPU,
 dim 100); N>1: configs[2] (the same graph partitioned over N GPUs, weak
 scaling).  --config papers | friendster, --scheme biased | layer | walk and
@@ -970,7 +970,9 @@ def main(argv=None):
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-breakdown", action="store_true")
     ap.add_argument("--no-pipeline", action="store_true", help="time non-pipelined fused steps")
-    ap.add_argument("--instances", type=int, default=4, help="concurrent step streams (each on 1/K of the SMs; world > 1: one exchange channel each)")
+    ap.add_argument("--instances", type=int, default=None,
+                    help="concurrent step streams (each on 1/K of the SMs; world > 1: one exchange channel each); "
+                         "default: 2 for uniform node-wise steps at world 1, else 4")
     ap.add_argument("--loader-rows", type=int, default=0, help="DSP_OPT_LOADER_ROWS (0: library default)")
     ap.add_argument("--layer-sizes", default="1000,1000",
                     help="--scheme layer: nodes sampled per layer (Table 7: 1000,1000)")
@@ -987,6 +989,13 @@ def main(argv=None):
         raise SystemExit("--warmup must be >= 3")
     if args.config is None:
         args.config = "products"
+    if args.instances is None:
+        # measured per workload: uniform node-wise steps with 5 loader
+        # warps per SM run best as 2 streams x 74 SMs (products 0.1264-0.1269 vs 0.1287-0.1300
+        # ms/step with 4, papers 0.631 vs 0.604, Friendster 0.830 vs 0.797 of HBM); biased
+        # and layer-wise steps (sampling-bound) as 4 x 37; world > 1 keeps 4 exchange channels
+        ws = int(os.environ.get("WORLD_SIZE", "1"))
+        args.instances = 2 if (args.scheme == "uniform" and ws == 1) else 4
     if args.impl == "reference":
         return run_reference(args)
     if args.scheme == "walk":

@@ -532,14 +532,15 @@ def test_products_pipelined(pkg, products):
 @pytest.mark.parametrize("biased", [False, True])
 def test_products_bench_launch_configuration(pkg, products, biased):
     """configs[1] at full size in exactly the launch configuration bench.py
-    times: 4 concurrent step streams, each pipelined persistent launch on 37
-    SMs with its own workspace, 8 output sets, sizes returned asynchronously;
+    times: K concurrent step streams (2 for uniform steps, 4 for biased ones),
+    each pipelined persistent launch on 148 / K SMs with its own workspace,
+    2K output sets, sizes returned asynchronously;
     every step whose output set survives is checked against the oracle
     (blocks bit-exact, every gathered row against the closed-form features)."""
     cfg, ip, ix = products
     feats = datagen.features(0, cfg.num_nodes, cfg.dim)
     ew = datagen.edge_weights(ix, datagen.node_weights(cfg.num_nodes)) if biased else None
-    K = 4
+    K = 4 if biased else 2
     s = pkg.Sampler(datagen.bounds(cfg.num_nodes, 1), ip, ix, feats, cfg.fanouts, cfg.batch, n_slots=2 * K,
                     n_workspaces=K, edge_weights=ew)
     pkg.dsp_set_persistent_blocks(s.ctx, torch.cuda.get_device_properties(0).multi_processor_count // K)
