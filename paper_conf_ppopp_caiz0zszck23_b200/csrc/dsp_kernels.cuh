@@ -1276,7 +1276,10 @@ __global__ void __launch_bounds__(32 * GTMA_WARPS) k_gather_tma(const __grid_con
 // no map clearing (epochs).
 template <int TEAM, bool PIPE, bool BIASED, int BLK = PNT>
 __global__ void __launch_bounds__(BLK, 1) k_csp_persistent(const __grid_constant__ PersistArgs a) {
-  constexpr int SG = 1;  // scan groups per round (2 / 4 measured equal at 4 streams; 1 keeps pass 1's rows in registers)
+#ifndef DSP_W1_GROUPS
+#define DSP_W1_GROUPS 1
+#endif
+  constexpr int SG = DSP_W1_GROUPS;  // scan groups per round: 1 keeps pass 1's rows in registers (2 / 4: 0.130 vs 0.127 ms/step)
   __shared__ Scan2Smem<TEAM, SG> sm;
   __shared__ __align__(8) uint64_t bars[LOADER_WARPS][LOADER_SLOTS];
   extern __shared__ __align__(128) char ring_smem[];
