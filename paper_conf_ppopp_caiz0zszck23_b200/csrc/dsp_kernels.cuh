@@ -974,7 +974,8 @@ __global__ void __launch_bounds__(NT) k_gather(const __grid_constant__ GatherArg
 #define DSP_LOADER_WARPS 5
 #endif
 // TMA gather warps of a pipelined launch: 5 (27 sampling warps) measured 0.1314 vs
-// 0.1322 ms/step with 4 and 0.1335 with 3; 6 rings exceed the shared memory
+// 0.1322 ms/step with 4 and 0.1335 with 3 (4 streams); at 2 streams 0.1266 vs 0.1334 with 4
+// and 0.1323 with 6
 constexpr int LOADER_WARPS = DSP_LOADER_WARPS;
 #ifndef DSP_LOADER_SLOTS
 #define DSP_LOADER_SLOTS 2

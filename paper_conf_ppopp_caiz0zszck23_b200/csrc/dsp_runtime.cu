@@ -1280,17 +1280,24 @@ dsp_status dsp_create(int32_t rank, int32_t world_size, int32_t cuda_device, dsp
   DeviceGuard g(cuda_device);
   int occ = 0, occ_pipe = 0;
   const int pipe_smem = std::min(LOADER_WARPS * LOADER_SLOTS * 16384, 200 * 1024);  // largest ring (dim 4096)
-  if (cudaFuncSetAttribute((const void *)k_csp_persistent<PIPE_TEAM, true, false>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_csp_persistent<BIASED_PIPE_TEAM, true, true, BIASED_BLK>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_csp_multi<PIPE_TEAM, true, false>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
-      cudaFuncSetAttribute((const void *)k_csp_multi<PIPE_TEAM, true, true>,
-                           cudaFuncAttributeMaxDynamicSharedMemorySize, pipe_smem) != cudaSuccess ||
+  // each pipelined kernel may use up to the largest ring that fits beside its static shared memory
+  auto ring_cap = [&](const void *f) {
+    cudaFuncAttributes fa{};
+    if (cudaFuncGetAttributes(&fa, f) != cudaSuccess) return -1;
+    return std::min(pipe_smem, (int)prop.sharedMemPerBlockOptin - (int)fa.sharedSizeBytes);
+  };
+  const void *pk[4] = {(const void *)k_csp_persistent<PIPE_TEAM, true, false>,
+                       (const void *)k_csp_persistent<BIASED_PIPE_TEAM, true, true, BIASED_BLK>,
+                       (const void *)k_csp_multi<PIPE_TEAM, true, false>, (const void *)k_csp_multi<PIPE_TEAM, true, true>};
+  bool attr_ok = true;
+  for (const void *f : pk) {
+    const int cap = ring_cap(f);
+    attr_ok = attr_ok && cap > 0 && cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, cap) == cudaSuccess;
+  }
+  if (!attr_ok ||
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_csp_persistent<PNT, false, false>, PNT, 0) != cudaSuccess ||
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_pipe, k_csp_persistent<PIPE_TEAM, true, false>, PNT, pipe_smem) !=
-          cudaSuccess ||
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_pipe, k_csp_persistent<PIPE_TEAM, true, false>, PNT,
+                                                    ring_cap(pk[0])) != cudaSuccess ||
       occ < 1 || occ_pipe < 1) {
     cudaGetLastError();
     delete c;
