@@ -957,6 +957,15 @@ def run_dsp(args):
     return 0
 
 
+def default_instances(scheme: str, world: int) -> int:
+    """Concurrent step streams when --instances is not given, measured per workload
+    (DESIGN.md "Measurement"): uniform node-wise steps with 5 loader warps per SM run best
+    as 2 streams x 74 SMs (products 0.1264-0.1269 vs 0.1287-0.1300 ms/step with 4, papers
+    0.631 vs 0.604, Friendster 0.830 vs 0.797 of HBM); biased and layer-wise steps
+    (sampling-bound) and random walks as 4; world > 1 keeps 4 exchange channels."""
+    return 2 if (scheme == "uniform" and world == 1) else 4
+
+
 def main(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -990,12 +999,7 @@ def main(argv=None):
     if args.config is None:
         args.config = "products"
     if args.instances is None:
-        # measured per workload: uniform node-wise steps with 5 loader
-        # warps per SM run best as 2 streams x 74 SMs (products 0.1264-0.1269 vs 0.1287-0.1300
-        # ms/step with 4, papers 0.631 vs 0.604, Friendster 0.830 vs 0.797 of HBM); biased
-        # and layer-wise steps (sampling-bound) as 4 x 37; world > 1 keeps 4 exchange channels
-        ws = int(os.environ.get("WORLD_SIZE", "1"))
-        args.instances = 2 if (args.scheme == "uniform" and ws == 1) else 4
+        args.instances = default_instances(args.scheme, int(os.environ.get("WORLD_SIZE", "1")))
     if args.impl == "reference":
         return run_reference(args)
     if args.scheme == "walk":

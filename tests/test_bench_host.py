@@ -54,3 +54,23 @@ def test_host_cpu_reports_model_and_cores():
     h = bench.host_cpu()
     assert h["logical_cores"] >= 1 and 1 <= h["cores_available"] <= h["logical_cores"]
     assert h["model"] is None or isinstance(h["model"], str)
+
+
+def test_default_instances():
+    """--instances defaults: 2 streams for uniform node-wise steps at world 1, else 4."""
+    assert bench.default_instances("uniform", 1) == 2
+    for scheme in ("biased", "layer", "walk"):
+        assert bench.default_instances(scheme, 1) == 4
+    assert bench.default_instances("uniform", 2) == 4 and bench.default_instances("uniform", 8) == 4
+
+
+def test_ncu_traffic_keys():
+    """The bench-configuration capture keeps the plain kernel name bench.py reads;
+    other workloads' captures of the same kernel do not overwrite it."""
+    sys.path.insert(0, os.path.join(ROOT, "tools"))
+    import ncu_summary
+    k = "k_csp_persistent<864, 1, 0, 1024>"
+    assert ncu_summary.traffic_key(k, "r02g") == "k_csp_persistent"
+    assert ncu_summary.traffic_key(k, "biased_r02g") == "k_csp_persistent@biased"
+    assert ncu_summary.traffic_key(k, "single_r02g") == "k_csp_persistent@single"
+    assert ncu_summary.traffic_key("k_gather_tma<0>", "gather_r02") == "k_gather_tma@gather"

@@ -14,6 +14,15 @@ import sys
 from collections import defaultdict
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def traffic_key(kernel: str, tag: str) -> str:
+    """Key of a capture in profiles/ncu_traffic.json: bench.py reads the plain kernel
+    name for the default (uniform, bench-configuration) capture; captures of other
+    workloads keep their own key (kernel@kind)."""
+    kind = next((w for w in ("biased", "single", "walk", "layer", "gather", "papers", "friendster")
+                 if tag.startswith(w) or f"_{w}" in tag), None)
+    return kernel.split("<")[0] + (f"@{kind}" if kind else "")
 METRICS = {
     "gpu__time_duration.sum": "duration",
     "dram__bytes_read.sum": "dram_read",
@@ -88,11 +97,7 @@ def main(rep, launches, tag):
                      f"{avg('occupancy_pct'):.1f} | {int(avg('regs'))} | {int(avg('grid'))} x {int(avg('block'))} | "
                      + ", ".join(f"{k} {100 * v:.0f}%" for k, v in st.items()) + " |")
         big = max(recs, key=lambda r: r.get("dram_read", 0) + r.get("dram_write", 0))  # the fused launch
-        # bench.py reads the plain kernel name for the default (uniform, bench-config) capture;
-        # captures of other workloads keep their own key
-        kind = next((w for w in ("biased", "single", "walk", "layer", "gather", "papers", "friendster")
-                     if tag.startswith(w) or f"_{w}" in tag), None)
-        traffic[name.split("<")[0] + (f"@{kind}" if kind else "")] = {"dram_bytes_per_launch": big.get("dram_read", 0) + big.get("dram_write", 0),
+        traffic[traffic_key(name, tag)] = {"dram_bytes_per_launch": big.get("dram_read", 0) + big.get("dram_write", 0),
                          "dram_read_bytes": big.get("dram_read", 0), "dram_write_bytes": big.get("dram_write", 0),
                          "duration_s_ncu": big.get("duration", 0), "source": f"profiles/ncu_{tag}.md",
                          "note": "largest-traffic capture of this kernel (the fused sample+gather launch bench.py times)"}
